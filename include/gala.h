@@ -1,0 +1,217 @@
+/*
+ * gala.h — C ABI of the B200-native GALA Louvain library (libgala.so).
+ *
+ * GALA = "Swift Unfolding of Communities: GPU-Accelerated Louvain Algorithm",
+ * Wang et al., PPoPP'25.  "P:N" = line N of the paper text.
+ *
+ * The library computes a community assignment of an undirected graph with
+ * positive integer edge weights that greedily maximises modularity (Eq. 1,
+ * P:96-101) with the multi-level Louvain method: phase 1 is the BSP
+ * local-moving iteration of Alg. 1 with MG pruning (Eq. 6/7,
+ * P:197-203) and delta community-weight updating (§3.5); phase 2
+ * compresses communities into super vertices.  Every step runs in
+ * hand-written sm_100a CUDA kernels on the device the graph lives on.
+ *
+ * Conventions:
+ *  - Graph input is a symmetric CSR: for every entry (v,u,w) the entry
+ *    (u,v,w) exists.  A self loop (v,v,w) is stored ONCE and counts once in
+ *    d(v) and in D_C.  Duplicate entries are allowed and summed.
+ *  - Weights are positive integers (int64).  NULL weights = all 1.
+ *  - gamma (resolution) is quantised to p/q = round(gamma*2^16)/2^16.
+ *    All gains and modularity numerators are exact integers; decisions are
+ *    bit-for-bit reproducible and independent of thread/block/GPU counts.
+ *  - Ties go to the lowest community id; Grappolo singleton swap suppression
+ *    (P:141 footnote 1); a vertex moves only if its best gain beats staying.
+ *  - Convergence: the iteration (and the level loop) stops when the exact
+ *    numerator gain dN = N' - N < T with T = ceil(tol * q * W^2) evaluated in
+ *    x87 long double (Alg. 1 lines 12-13, theta = tol, P:340 uses 1e-6).
+ *
+ * Ownership: input arrays are copied; the caller may free them on return.
+ * Outputs are written into caller buffers.  The handle owns all device memory
+ * and frees it in gala_graph_free.  Every call returns a gala_status; no C++
+ * exception crosses this boundary.  On error gala_last_error() returns a
+ * thread-local message.  Calls on one handle must not run concurrently.
+ */
+#ifndef GALA_H
+#define GALA_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct gala_graph_s* gala_graph;
+
+typedef enum {
+    GALA_OK = 0,
+    GALA_E_INVALID = 1,   /* malformed CSR, weight <= 0, n >= 2^31, bad option/argument */
+    GALA_E_OVERFLOW = 2,  /* max(p,q) * W^2 >= 2^125: exact integer gains would overflow */
+    GALA_E_NOMEM = 3,     /* device allocation failed */
+    GALA_E_CUDA = 4,      /* CUDA runtime error (message in gala_last_error) */
+    GALA_E_NCCL = 5,      /* NCCL error or NCCL unavailable (multi-GPU only) */
+    GALA_E_STATE = 6      /* call not valid in this state (e.g. results before gala_run) */
+} gala_status;
+
+/* Library version string (static storage). */
+const char* gala_version(void);
+
+/* Thread-local message of the last non-OK status (static until the next call). */
+const char* gala_last_error(void);
+
+/*
+ * gala_graph_from_csr — build a handle from a HOST CSR (problem statement,
+ * §2.1: G = {V, E, w}).
+ *   n        : number of vertices, 0 <= n < 2^31
+ *   row_ptr  : host int64[n+1], row_ptr[0] = 0, non-decreasing
+ *   col_idx  : host int32[row_ptr[n]], each in [0, n)
+ *   weights  : host int64[row_ptr[n]] each > 0, or NULL (all 1)
+ *   device   : CUDA device ordinal the graph and all kernels live on
+ *   stream   : cudaStream_t as an integer (0 = the library's own stream)
+ *   out      : receives the handle
+ * Copies the graph to the device (H2D) and validates it.  Symmetry is NOT
+ * checked unless option "check_symmetric" is set afterwards and
+ * gala_validate is called.
+ */
+gala_status gala_graph_from_csr(int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
+                                const int64_t* weights, int device, uintptr_t stream,
+                                gala_graph* out);
+
+/*
+ * gala_graph_from_csr_device — same, but row_ptr/col_idx/weights are DEVICE
+ * pointers on `device` (e.g. torch CUDA tensors).  The data is copied
+ * device-to-device; the caller keeps ownership of its buffers.
+ */
+gala_status gala_graph_from_csr_device(int64_t n, const int64_t* d_row_ptr, const int32_t* d_col_idx,
+                                       const int64_t* d_weights, int device, uintptr_t stream,
+                                       gala_graph* out);
+
+/* Verify symmetry of the stored CSR (O(nnz log) device check). GALA_E_INVALID if not. */
+gala_status gala_validate(gala_graph g);
+
+/*
+ * gala_run — full multi-level Louvain: phase 1 (Alg. 1) to
+ * convergence, then phase 2 coarsening, repeated until no community merges,
+ * the level's numerator gain is below T, or max_levels levels ran.
+ *   gamma      : resolution (> 0), quantised as above
+ *   tol        : theta > 0 (P:340 uses 1e-6)
+ *   max_levels : <= 0 means until converged
+ * Always restarts from singletons; deterministic.  Synchronises the
+ * handle's stream before returning.
+ */
+gala_status gala_run(gala_graph g, double gamma, double tol, int32_t max_levels);
+
+/*
+ * gala_get_communities — final labels of the level-0 vertices, canonical ids
+ * 0..k-1 in order of each community's smallest vertex id.
+ *   labels : host int32[n]; n must equal the graph's n
+ *   num_communities : optional (nullable) receives k
+ */
+gala_status gala_get_communities(gala_graph g, int32_t* labels, int64_t n, int64_t* num_communities);
+
+/* Same as gala_get_communities but writes into a DEVICE buffer on the graph's device. */
+gala_status gala_get_communities_device(gala_graph g, int32_t* d_labels, int64_t n,
+                                        int64_t* num_communities);
+
+/*
+ * gala_modularity — Q_gamma (Eq. 1 with resolution) of the final partition,
+ * recomputed exactly on the level-0 graph and rounded once to double.
+ */
+gala_status gala_modularity(gala_graph g, double* q);
+
+/*
+ * gala_modularity_numerator — exact N = q*W*sum_C D_C(C) - p*sum_C D_V(C)^2
+ * of the final partition as a 128-bit two's-complement (hi, lo) pair, plus W,
+ * p and q.  Q = N / (q W^2).  Any out pointer may be NULL.
+ */
+gala_status gala_modularity_numerator(gala_graph g, int64_t* n_hi, uint64_t* n_lo, int64_t* W,
+                                      int64_t* p, int64_t* q);
+
+/* Free the handle and all its device memory.  NULL is a no-op. */
+void gala_graph_free(gala_graph g);
+
+/*
+ * gala_set_option — tuning / test hooks.  Options never change results
+ * (labels are identical for every setting) except "max_iters" (a per-level
+ * iteration cap honoured identically by the oracle) and "prune_mode".
+ *   "prune"          0/1   MG pruning (Eq. 6/7), default 1
+ *   "trace"          0/1/2 per-iteration records; 2 also copies labels each iteration
+ *   "check"          0/1   debug: verify maintained d'(v) against its definition
+ *   "timing"         0/1   per-kernel CUDA-event timing (gala_get_kernel_stats)
+ *   "max_iters"      >= 0  per-level iteration cap (0 = none)
+ *   "bin_sub4" "bin_sub8" "bin_sub16" "bin_sub32" "bin_warp"
+ *                    degree upper bounds of the dispatch bins (must be
+ *                    non-decreasing, sub-warp bins <= their lane count)
+ *   "delta_update"   0 = always recompute d', 1 = always delta, 2 = adaptive (default)
+ *   "force_i128"     0/1   use the 128-bit gain path even when 64-bit suffices
+ *   "hub_smem_slots" power of two, shared-memory slots of the block hash table
+ *   "cuda_graph"     0/1   capture the iteration body in a CUDA graph (default 1)
+ */
+gala_status gala_set_option(gala_graph g, const char* key, int64_t value);
+
+/*
+ * gala_get_stats — JSON object with per-level and per-iteration statistics
+ * of the last gala_run (levels, iterations, active/pruned/moved counts,
+ * edges scanned, timings).  Writes at most cap bytes including the NUL;
+ * returns GALA_E_INVALID if cap is too small (required size in *needed).
+ */
+gala_status gala_get_stats(gala_graph g, char* json_buf, int64_t cap, int64_t* needed);
+
+/*
+ * Trace access (option "trace" >= 1).  Record i (0 <= i < count) is
+ * int64[12]: level, iter, n_level, n_active, n_pruned, n_moved,
+ *            N_hi, N_lo (numerator after the iteration), edges_scanned,
+ *            distinct_communities_seen, delta_update_used, reserved.
+ * Labels (trace == 2): level-local community of every level vertex after
+ * the iteration; out must hold n_level entries.
+ */
+gala_status gala_get_trace_count(gala_graph g, int64_t* count);
+gala_status gala_get_trace_record(gala_graph g, int64_t i, int64_t* out12);
+gala_status gala_get_trace_labels(gala_graph g, int64_t i, int32_t* out, int64_t n_level);
+
+/*
+ * Per-kernel-class device time of the last gala_run (option "timing").
+ * For class k (0 <= k < *count): name (static string), launches, total
+ * milliseconds, algorithmic bytes.
+ */
+gala_status gala_get_kernel_stats(gala_graph g, int32_t k, const char** name, int64_t* launches,
+                                  double* ms, double* alg_bytes, int32_t* count);
+
+/* ---------------------------------------------------------------- multi-GPU
+ * 1D vertex partition, one process per GPU (§4.3).  Rank r owns
+ * the contiguous vertex range [v_begin, v_end) and its CSR rows (global
+ * column ids).  Community state is replicated; after every iteration labels
+ * are synchronised densely (broadcast of every rank's slice) or sparsely
+ * (allgather of (vertex, community) deltas) by moved volume, and Sigma_tot
+ * deltas are all-reduced, all over NCCL.  Results are identical to 1 GPU.
+ */
+
+/* 128-byte ncclUniqueId for rank 0 to broadcast (GALA_E_NCCL if NCCL cannot be loaded). */
+gala_status gala_nccl_unique_id(void* out128);
+
+/*
+ * gala_graph_from_csr_dist — collective over `world` ranks.
+ *   uid128      : the same ncclUniqueId on every rank
+ *   n_global    : global vertex count
+ *   v_begin/end : owned vertex range (ranges tile [0, n_global) in rank order)
+ *   local_row_ptr : host int64[v_end - v_begin + 1], local_row_ptr[0] = 0
+ *   col_idx     : host int32[local nnz], GLOBAL vertex ids
+ *   weights     : host int64[local nnz] or NULL (NULL must be used on all ranks alike)
+ */
+gala_status gala_graph_from_csr_dist(const void* uid128, int rank, int world, int device,
+                                     int64_t n_global, int64_t v_begin, int64_t v_end,
+                                     const int64_t* local_row_ptr, const int32_t* col_idx,
+                                     const int64_t* weights, uintptr_t stream, gala_graph* out);
+
+/*
+ * gala_partition_ranges — host-only helper: edge-balanced contiguous split of
+ * n vertices over `world` ranks (each range's entry count ~ nnz/world).
+ * bounds: int64[world+1].
+ */
+gala_status gala_partition_ranges(int64_t n, const int64_t* row_ptr, int world, int64_t* bounds);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* GALA_H */

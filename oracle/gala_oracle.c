@@ -36,6 +36,7 @@
 #include <stdint.h>
 #include <stdlib.h>
 #include <string.h>
+#include <math.h>
 #include <omp.h>
 
 typedef __int128 i128;
@@ -254,13 +255,17 @@ void* oracle_louvain(int64_t n, const int64_t* row_ptr, const int32_t* col, cons
     R->W = W;
     /* overflow budget: |scores| <= q*W*maxd must stay well inside __int128 */
     if (row_ptr[0] != 0) R->status = 1;
-    if (!R->status && (long double)q * W * (long double)maxd >= 0x1p126L) R->status = 2;   /* 2^126 */
+    /* overflow budget (include/gala.h GALA_E_OVERFLOW): max(p,q) * W^2 < 2^125 keeps every
+       score, stay, Eq. 6 left-hand side and numerator N inside __int128 */
+    (void)maxd;
+    if (!R->status && (long double)(p > q ? p : q) * (long double)W * (long double)W >= 0x1p125L) R->status = 2;
     if (R->status || W == 0) {   /* reading c18: no edges -> singletons, Q := 0 */
         R->N = 0;
         free(G.rp); free(G.col); free(G.w);
         return R;
     }
-    long double thr = (long double)tol * (long double)q * (long double)W * (long double)W;
+    /* theta test (reading c7): dN < T with T = ceil(tol * q * W^2) in long double */
+    i128 thr = (i128)ceill((long double)tol * (long double)q * (long double)W * (long double)W);
 
     for (int32_t level = 0;; ++level) {
         int64_t nl = G.n;
@@ -353,7 +358,7 @@ void* oracle_louvain(int64_t n, const int64_t* row_ptr, const int32_t* col, cons
                 push_rec(R, x);
             }
             /* Alg. 1 lines 12-13: Delta Q < theta (moves of this iteration are kept, c6) */
-            int converged = (n_moved == 0) || ((long double)(Nn - N) < thr);
+            int converged = (n_moved == 0) || (Nn - N < thr);
             N = Nn;
             if (converged || (max_iters > 0 && it + 1 >= max_iters)) break;
         }
@@ -373,7 +378,7 @@ void* oracle_louvain(int64_t n, const int64_t* row_ptr, const int32_t* col, cons
         orc_level L = { nl, G.rp[nl], iters, N_start, N };
         push_lev(R, L);
         int stop = (k == nl) || (max_levels > 0 && level + 1 >= max_levels) ||
-                   ((long double)(N - N_start) < thr);
+                   (N - N_start < thr);
         free(d); free(s); free(dp); free(Sig); free(size); free(C); free(nextC); free(minmem); free(cnew);
         if (stop) { free(newid); break; }
         ograph H;

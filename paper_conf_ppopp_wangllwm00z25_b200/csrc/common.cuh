@@ -1,0 +1,104 @@
+// common.cuh — shared device types and helpers of the GALA sm_100a kernels.
+//
+// Exact integer arithmetic throughout (DESIGN.md "Readings" c1, c11, c16):
+//   score(c) = qW * d_c(v) - p * Sig[c] * d(v)            (Eq. 2 x q W |E|)
+//   stay     = qW * d'(v)  - p * (Sig[C[v]] - d(v)) * d(v) (v removed from its community)
+// with gamma = p/q and W = 2|E|.  ST (score type) is int64 when
+// max(p,q) * W * maxdeg < 2^62 on the level (chosen by the host), else __int128.
+#pragma once
+
+#include <cstdint>
+#include <climits>
+#include <cuda_runtime.h>
+
+typedef __int128 i128;
+typedef unsigned long long ull;
+
+#define FULLMASK 0xffffffffu
+
+// dispatch bins (a2): sub-warp groups of 4/8/16/32 lanes, warp hash, block hash
+enum { BIN_S4 = 0, BIN_S8 = 1, BIN_S16 = 2, BIN_S32 = 3, BIN_WARP = 4, BIN_BLOCK = 5, NBINS = 6 };
+
+// Device-resident per-iteration counters (zeroed by k_iter_begin).
+struct IterCounters {
+    ull bin_count[NBINS];   // active vertices queued per bin
+    ull bin_deg[NBINS];     // sum of row lengths of queued vertices (edges scanned)
+    ull bin_k[NBINS];       // sum of distinct neighbour communities seen by decide
+    ull n_active;
+    ull n_pruned;
+    ull n_moved;
+    ull moved_deg;          // sum of row lengths of moved vertices
+    ull cursor[NBINS];      // dynamic work cursors (block kernels)
+    ull dp_mismatch;        // check mode: maintained d' != aggregated d'
+    ull ticket;             // last-block-done ticket of k_reduce
+    ull delta_used;         // 1 if the delta d' update ran this iteration
+};
+
+// Device-resident state carried across iterations of a level.
+struct Carry {
+    long long N_hi;         // current numerator N (int128 split)
+    ull N_lo;
+    long long N_prev_hi;    // numerator before this iteration
+    ull N_prev_lo;
+    long long minSig;       // min{Sig[c] : Sig[c] > 0}
+    long long sumDC;        // sum_v (d'(v) + s(v))
+    int converged;
+    int pad;
+};
+
+__device__ __forceinline__ i128 mk128(long long hi, ull lo) {
+    return (i128)(((unsigned __int128)(ull)hi << 64) | (unsigned __int128)lo);
+}
+__device__ __forceinline__ long long hi128(i128 x) { return (long long)(x >> 64); }
+__device__ __forceinline__ ull lo128(i128 x) { return (ull)x; }
+
+// warp shuffles for score types
+__device__ __forceinline__ long long shfl_xor_st(long long x, int off) {
+    return __shfl_xor_sync(FULLMASK, x, off);
+}
+__device__ __forceinline__ i128 shfl_xor_st(i128 x, int off) {
+    long long h = __shfl_xor_sync(FULLMASK, (long long)(x >> 64), off);
+    ull l = __shfl_xor_sync(FULLMASK, (ull)x, off);
+    return mk128(h, l);
+}
+template <typename ST> __device__ __forceinline__ ST st_min();
+template <> __device__ __forceinline__ long long st_min<long long>() { return LLONG_MIN; }
+template <> __device__ __forceinline__ i128 st_min<i128>() { return mk128(LLONG_MIN, 0); }
+
+// (score, community) ordering: higher score first, then lower community id.
+template <typename ST>
+__device__ __forceinline__ bool better(ST s1, int c1, ST s2, int c2) {
+    return s1 > s2 || (s1 == s2 && c1 < c2);
+}
+
+// multiplicative hash of a community id into a power-of-two table
+__device__ __forceinline__ unsigned hash_slot(int c, unsigned mask) {
+    return ((unsigned)c * 2654435761u) & mask;
+}
+__device__ __forceinline__ unsigned hash_slot2(int c, unsigned mask) {
+    return (((unsigned)c ^ 0x5bd1e995u) * 0x9E3779B1u >> 7) & mask;
+}
+
+__device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
+__device__ __forceinline__ unsigned lanemask_lt() {
+    unsigned m;
+    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+    return m;
+}
+
+// warp-aggregated append of a flagged lane's item to a queue; returns slot or -1
+__device__ __forceinline__ long long warp_append(bool flag, ull* counter) {
+    unsigned m = __ballot_sync(FULLMASK, flag);
+    if (!m) return -1;
+    int leader = __ffs(m) - 1;
+    ull base = 0;
+    if (lane_id() == leader) base = atomicAdd(counter, (ull)__popc(m));
+    base = __shfl_sync(FULLMASK, base, leader);
+    return flag ? (long long)(base + __popc(m & lanemask_lt())) : -1;
+}
+
+__device__ __forceinline__ long long warp_sum_ll(long long x) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(FULLMASK, x, o);
+    return x;
+}

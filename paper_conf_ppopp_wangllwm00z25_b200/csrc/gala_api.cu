@@ -1,0 +1,1043 @@
+// gala_api.cu — host driver and C ABI of libgala.so (include/gala.h).
+//
+// The driver runs the multi-level loop of P:109 on the device: per level it
+// initialises singletons (a1), iterates phase 1 (Alg. 1) until the
+// exact numerator gain drops below T (a2-a7; one 64-byte D2H read per
+// iteration carries the device's convergence decision), then relabels (a8)
+// and coarsens (a9).  Every arithmetic step runs in the kernels of
+// k_phase1.cuh / k_phase2.cuh; this file only sizes launches, owns memory and
+// keeps statistics.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "gala.h"
+#include "common.cuh"
+#include "k_phase1.cuh"
+#include "k_phase2.cuh"
+#include "dist.h"
+
+#define GALA_VERSION "gala-b200 0.1 (sm_100a)"
+
+// ------------------------------------------------------------------ errors
+static thread_local std::string g_err;
+static gala_status set_err(gala_status st, const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_err = buf;
+    return st;
+}
+struct GalaError {
+    gala_status st;
+};
+#define CK(call)                                                                                   \
+    do {                                                                                           \
+        cudaError_t e_ = (call);                                                                   \
+        if (e_ != cudaSuccess) {                                                                   \
+            set_err(e_ == cudaErrorMemoryAllocation ? GALA_E_NOMEM : GALA_E_CUDA, "%s:%d %s: %s", \
+                    __FILE__, __LINE__, #call, cudaGetErrorString(e_));                           \
+            throw GalaError{e_ == cudaErrorMemoryAllocation ? GALA_E_NOMEM : GALA_E_CUDA};        \
+        }                                                                                          \
+    } while (0)
+#define CKL() CK(cudaGetLastError())
+
+// ------------------------------------------------------------------ kernel classes
+enum KClass {
+    KC_PRUNE = 0, KC_DEC_S4, KC_DEC_S8, KC_DEC_S16, KC_DEC_S32, KC_DEC_WARP, KC_DEC_BLOCK,
+    KC_APPLY, KC_DP, KC_REDUCE, KC_INIT, KC_PHASE2, KC_COUNT
+};
+static const char* kc_names[KC_COUNT] = {"prune_bin", "decide_sub4", "decide_sub8", "decide_sub16",
+                                         "decide_sub32", "decide_warp", "decide_block", "apply",
+                                         "dp_update", "reduce", "level_init", "phase2"};
+
+struct TraceRec {
+    int64_t v[12];
+};
+
+struct DevCSR {
+    int64_t n = 0, nnz = 0;
+    int64_t* rp = nullptr;
+    int32_t* col = nullptr;
+    int64_t* w = nullptr;   // nullptr = unit weights
+};
+
+struct LevelStat {
+    int64_t n, nnz, iters, maxdeg;
+    int i128path;
+    double ms_phase1, ms_phase2;
+    int64_t edges_scanned, nominal_edges;
+};
+
+struct gala_graph_s {
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    bool own_stream = false;
+    int num_sms = 148;
+    // level-0 graph
+    DevCSR g0;
+    int64_t n0 = 0, nnz0 = 0, W = 0, maxdeg0 = 0;
+    int64_t* d0 = nullptr;
+    int64_t* s0 = nullptr;
+    // options
+    int opt_prune = 1, opt_trace = 0, opt_check = 0, opt_timing = 0, opt_max_iters = 0;
+    int opt_delta = 2, opt_force_i128 = 0, opt_cuda_graph = 0;
+    int bins[NBINS - 1] = {4, 8, 16, 32, 128};
+    int hub_smem_slots = 4096;
+    // results
+    bool has_result = false;
+    int64_t k = 0, p = 1, q = 1;
+    i128 N = 0;
+    int32_t* lab = nullptr;   // device, n0
+    std::vector<TraceRec> trace;
+    std::vector<std::vector<int32_t>> trace_labels;
+    std::vector<LevelStat> levels;
+    double kc_ms[KC_COUNT] = {0};
+    double kc_bytes[KC_COUNT] = {0};
+    int64_t kc_launches[KC_COUNT] = {0};
+    double run_ms = 0;
+    int64_t dp_mismatch = 0;
+    // dist
+    DistCtx* dist = nullptr;
+};
+
+// ------------------------------------------------------------------ memory
+template <typename T>
+static T* dalloc(size_t count, cudaStream_t st) {
+    void* p = nullptr;
+    if (count == 0) count = 1;
+    CK(cudaMallocAsync(&p, count * sizeof(T), st));
+    return static_cast<T*>(p);
+}
+template <typename T>
+static void dfree(T*& p, cudaStream_t st) {
+    if (p) cudaFreeAsync(p, st);
+    p = nullptr;
+}
+
+static int grid_for(long long n, int bt, int cap) {
+    long long g = (n + bt - 1) / bt;
+    if (g < 1) g = 1;
+    if (g > cap) g = cap;
+    return (int)g;
+}
+
+// exclusive scan of int64 in[0..n) into out[0..n] (out[n] = total)
+static void scan_excl(const long long* in, long long* out, long long n, cudaStream_t st) {
+    long long nt = (n + SCAN_TILE - 1) / SCAN_TILE;
+    if (nt < 1) nt = 1;
+    long long* sums = dalloc<long long>(nt + 1, st);
+    k_scan_tiles<<<(unsigned)nt, SCAN_BT, 0, st>>>(in, n, sums);
+    CKL();
+    k_scan_sums<<<1, SCAN_BT, 0, st>>>(sums, nt);
+    CKL();
+    k_scan_apply<<<(unsigned)nt, SCAN_BT, 0, st>>>(in, n, sums, out, nt);
+    CKL();
+    dfree(sums, st);
+}
+
+// ------------------------------------------------------------------ timing
+struct Timer {
+    gala_graph_s* g;
+    std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> pending;
+    std::vector<cudaEvent_t> pool;
+    explicit Timer(gala_graph_s* gg) : g(gg) {}
+    cudaEvent_t get() {
+        if (!pool.empty()) { cudaEvent_t e = pool.back(); pool.pop_back(); return e; }
+        cudaEvent_t e;
+        CK(cudaEventCreate(&e));
+        return e;
+    }
+    cudaEvent_t begin() {
+        if (!g->opt_timing) return nullptr;
+        cudaEvent_t e = get();
+        CK(cudaEventRecord(e, g->stream));
+        return e;
+    }
+    void end(int kc, cudaEvent_t b) {
+        g->kc_launches[kc]++;
+        if (!g->opt_timing) return;
+        cudaEvent_t e = get();
+        CK(cudaEventRecord(e, g->stream));
+        pending.push_back({kc, {b, e}});
+    }
+    void resolve() {   // call after a stream sync
+        for (auto& x : pending) {
+            float ms = 0;
+            CK(cudaEventElapsedTime(&ms, x.second.first, x.second.second));
+            g->kc_ms[x.first] += ms;
+            pool.push_back(x.second.first);
+            pool.push_back(x.second.second);
+        }
+        pending.clear();
+    }
+    ~Timer() {
+        for (auto& x : pending) { cudaEventDestroy(x.second.first); cudaEventDestroy(x.second.second); }
+        for (auto e : pool) cudaEventDestroy(e);
+    }
+};
+
+// ------------------------------------------------------------------ gamma, thresholds
+static int64_t gcd64(int64_t a, int64_t b) {
+    while (b) { int64_t t = a % b; a = b; b = t; }
+    return a;
+}
+static void gamma_to_pq(double gamma, int64_t* p, int64_t* q) {
+    int64_t pp = (int64_t)(gamma * 65536.0 + 0.5), qq = 65536;
+    int64_t g = gcd64(pp, qq);
+    if (g == 0) g = 1;
+    *p = pp / g;
+    *q = qq / g;
+}
+
+// ------------------------------------------------------------------ workspace of a run
+struct Work {
+    cudaStream_t st;
+    int64_t ncap, nnzcap;
+    int32_t *C = nullptr, *size = nullptr, *stamp = nullptr, *mv_v = nullptr, *mv_c = nullptr, *mv_old = nullptr;
+    int32_t* queues = nullptr;
+    int64_t *Sig = nullptr, *d = nullptr, *s = nullptr, *dp = nullptr;
+    IterCounters* ctr = nullptr;
+    Carry* carry = nullptr;
+    long long *part_dc = nullptr, *part_min = nullptr;
+    i128* part_s2 = nullptr;
+    int* gkeys = nullptr;
+    ull* gvals = nullptr;
+    long long gcap = 0;
+    int gblocks = 0;
+    IterCounters* h_ctr = nullptr;
+    Carry* h_carry = nullptr;
+    int reduce_grid = 0;
+    void release() {
+        dfree(C, st); dfree(size, st); dfree(stamp, st); dfree(mv_v, st); dfree(mv_c, st); dfree(mv_old, st);
+        dfree(queues, st); dfree(Sig, st); dfree(d, st); dfree(s, st); dfree(dp, st); dfree(ctr, st);
+        dfree(carry, st); dfree(part_dc, st); dfree(part_min, st); dfree(part_s2, st); dfree(gkeys, st);
+        dfree(gvals, st);
+        if (h_ctr) cudaFreeHost(h_ctr);
+        if (h_carry) cudaFreeHost(h_carry);
+        h_ctr = nullptr;
+        h_carry = nullptr;
+    }
+};
+
+// ------------------------------------------------------------------ launch helpers
+template <typename ST, bool UNIT>
+static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, ST qW, ST p, Timer& tm, int64_t maxdeg) {
+    DecideArgs a;
+    a.rp = G.rp; a.col = G.col; a.w = G.w; a.C = wk.C; a.Sig = wk.Sig; a.size = wk.size; a.d = wk.d;
+    a.dp = wk.dp; a.mv_v = wk.mv_v; a.mv_c = wk.mv_c; a.ctr = wk.ctr; a.check = g->opt_check;
+    const long long qs = wk.ncap;
+    const int sub_grid = g->num_sms * 8;
+    cudaStream_t st = g->stream;
+    cudaEvent_t e;
+    e = tm.begin();
+    k_decide_sub<4, ST, UNIT><<<sub_grid, 256, 0, st>>>(wk.queues + BIN_S4 * qs, BIN_S4, a, qW, p);
+    CKL();
+    tm.end(KC_DEC_S4, e);
+    e = tm.begin();
+    k_decide_sub<8, ST, UNIT><<<sub_grid, 256, 0, st>>>(wk.queues + BIN_S8 * qs, BIN_S8, a, qW, p);
+    CKL();
+    tm.end(KC_DEC_S8, e);
+    e = tm.begin();
+    k_decide_sub<16, ST, UNIT><<<sub_grid, 256, 0, st>>>(wk.queues + BIN_S16 * qs, BIN_S16, a, qW, p);
+    CKL();
+    tm.end(KC_DEC_S16, e);
+    e = tm.begin();
+    k_decide_sub<32, ST, UNIT><<<sub_grid, 256, 0, st>>>(wk.queues + BIN_S32 * qs, BIN_S32, a, qW, p);
+    CKL();
+    tm.end(KC_DEC_S32, e);
+    e = tm.begin();
+    k_decide_warp<256, ST, UNIT><<<sub_grid, 256, 0, st>>>(wk.queues + BIN_WARP * qs, BIN_WARP, a, qW, p);
+    CKL();
+    tm.end(KC_DEC_WARP, e);
+    if (maxdeg > g->bins[BIN_WARP]) {
+        const int smem_cap = g->hub_smem_slots;
+        size_t smem = (size_t)smem_cap * (sizeof(ull) + sizeof(int));
+        e = tm.begin();
+        k_decide_block<512, ST, UNIT><<<wk.gblocks, 512, smem, st>>>(wk.queues + BIN_BLOCK * qs, BIN_BLOCK, a, qW,
+                                                                      p, smem_cap, wk.gkeys, wk.gvals, wk.gcap);
+        CKL();
+        tm.end(KC_DEC_BLOCK, e);
+    }
+}
+
+template <typename ST, bool UNIT>
+static void run_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, ST qW, ST p, i128 qW128, i128 T,
+                          int iter_id, Timer& tm, int64_t maxdeg) {
+    cudaStream_t st = g->stream;
+    const int n = (int)G.n;
+    const int big = g->num_sms * 8;
+    cudaEvent_t e = tm.begin();
+    k_iter_begin<<<1, 128, 0, st>>>(wk.ctr);
+    CKL();
+    BinThresholds th;
+    for (int i = 0; i < NBINS - 1; ++i) th.t[i] = g->bins[i];
+    k_prune_bin<ST><<<grid_for(n, 256, big), 256, 0, st>>>(n, G.rp, wk.d, wk.dp, wk.C, wk.Sig, g->opt_prune, qW, p,
+                                                           wk.carry, wk.ctr, wk.queues, wk.ncap, th);
+    CKL();
+    tm.end(KC_PRUNE, e);
+    launch_decide<ST, UNIT>(g, wk, G, qW, p, tm, maxdeg);
+    e = tm.begin();
+    k_apply<<<big, 256, 0, st>>>(wk.ctr, wk.mv_v, wk.mv_c, wk.mv_old, wk.C, wk.Sig, wk.size, wk.d, wk.stamp, iter_id);
+    CKL();
+    tm.end(KC_APPLY, e);
+    e = tm.begin();
+    k_dp_delta<UNIT><<<big, 256, 0, st>>>(wk.ctr, G.rp, G.col, G.w, wk.C, wk.mv_v, wk.mv_old, wk.stamp, wk.dp,
+                                          iter_id, G.nnz, g->opt_delta, 1, 2);
+    CKL();
+    k_dp_full<UNIT><<<big, 256, 0, st>>>(wk.ctr, n, G.rp, G.col, G.w, wk.C, wk.dp, G.nnz, g->opt_delta, 1, 2, 0);
+    CKL();
+    tm.end(KC_DP, e);
+    e = tm.begin();
+    k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>(n, wk.dp, wk.s, wk.Sig, wk.part_dc, wk.part_s2, wk.part_min, wk.ctr,
+                                                  wk.carry, (long long)(qW128 >> 64), (ull)qW128, (long long)p,
+                                                  (long long)(T >> 64), (ull)T, 1);
+    CKL();
+    tm.end(KC_REDUCE, e);
+}
+
+static i128 carry_N(const Carry* c) {
+    return (i128)(((unsigned __int128)(ull)c->N_hi << 64) | (unsigned __int128)c->N_lo);
+}
+
+// algorithmic bytes per kernel class of one iteration
+static void account_bytes(gala_graph_s* g, const IterCounters& c, int64_t n, int64_t nnz, bool unit) {
+    const double om = unit ? 0.0 : 8.0;
+    double act = 0;
+    for (int b = 0; b < NBINS; ++b) {
+        double cnt = (double)c.bin_count[b], deg = (double)c.bin_deg[b], kk = (double)c.bin_k[b];
+        g->kc_bytes[KC_DEC_S4 + b] += cnt * (4 + 16 + 4 + 8 + 8) + deg * (4 + om + 4) + 8 * kk;
+        act += cnt;
+    }
+    // prune: d, dp, C, Sig[C] per vertex; rp pair + queue write per active
+    g->kc_bytes[KC_PRUNE] += (double)n * (8 + 8 + 4 + 8) + act * (16 + 4);
+    double m = (double)c.n_moved;
+    g->kc_bytes[KC_APPLY] += m * (4 + 4 + 4 + 4 + 4 + 4 + 8 + 16 + 8);
+    if (c.delta_used)
+        g->kc_bytes[KC_DP] += m * (16 + 8) + (double)c.moved_deg * (4 + om + 4 + 4);
+    else
+        g->kc_bytes[KC_DP] += (double)n * (16 + 4 + 8) + (double)nnz * (4 + om + 4);
+    g->kc_bytes[KC_REDUCE] += (double)n * 24;
+}
+
+// ------------------------------------------------------------------ the multi-level run
+static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
+    cudaStream_t st = g->stream;
+    CK(cudaSetDevice(g->device));
+    g->has_result = false;
+    g->trace.clear();
+    g->trace_labels.clear();
+    g->levels.clear();
+    for (int i = 0; i < KC_COUNT; ++i) { g->kc_ms[i] = 0; g->kc_bytes[i] = 0; g->kc_launches[i] = 0; }
+    g->dp_mismatch = 0;
+    int64_t p, q;
+    gamma_to_pq(gamma, &p, &q);
+    g->p = p;
+    g->q = q;
+    const int64_t n0 = g->n0, W = g->W;
+    const int64_t mpq = std::max(p, q);
+    if ((long double)mpq * (long double)W * (long double)W >= 0x1p125L) {
+        set_err(GALA_E_OVERFLOW, "max(p,q)*W^2 >= 2^125");
+        throw GalaError{GALA_E_OVERFLOW};
+    }
+    const i128 qW128 = (i128)q * W;
+    const i128 T = (i128)ceill((long double)tol * (long double)q * (long double)W * (long double)W);
+
+    cudaEvent_t ev_run0, ev_run1;
+    CK(cudaEventCreate(&ev_run0));
+    CK(cudaEventCreate(&ev_run1));
+    CK(cudaEventRecord(ev_run0, st));
+
+    const int big = g->num_sms * 8;
+    if (!g->lab) g->lab = dalloc<int32_t>(n0, st);
+    Work wk;
+    wk.st = st;
+    wk.ncap = std::max<int64_t>(n0, 1);
+    wk.nnzcap = g->nnz0;
+    try {
+        wk.C = dalloc<int32_t>(wk.ncap, st);
+        wk.size = dalloc<int32_t>(wk.ncap, st);
+        wk.stamp = dalloc<int32_t>(wk.ncap, st);
+        wk.mv_v = dalloc<int32_t>(wk.ncap, st);
+        wk.mv_c = dalloc<int32_t>(wk.ncap, st);
+        wk.mv_old = dalloc<int32_t>(wk.ncap, st);
+        wk.queues = dalloc<int32_t>((size_t)wk.ncap * NBINS, st);
+        wk.Sig = dalloc<int64_t>(wk.ncap, st);
+        wk.d = dalloc<int64_t>(wk.ncap, st);
+        wk.s = dalloc<int64_t>(wk.ncap, st);
+        wk.dp = dalloc<int64_t>(wk.ncap, st);
+        wk.ctr = dalloc<IterCounters>(1, st);
+        wk.carry = dalloc<Carry>(1, st);
+        wk.reduce_grid = g->num_sms * 2;
+        wk.part_dc = dalloc<long long>(wk.reduce_grid, st);
+        wk.part_min = dalloc<long long>(wk.reduce_grid, st);
+        wk.part_s2 = dalloc<i128>(wk.reduce_grid, st);
+        CK(cudaMallocHost(&wk.h_ctr, sizeof(IterCounters)));
+        CK(cudaMallocHost(&wk.h_carry, sizeof(Carry)));
+        CK(cudaMemsetAsync(wk.ctr, 0, sizeof(IterCounters), st));
+        CK(cudaMemsetAsync(wk.carry, 0, sizeof(Carry), st));
+        // block-kernel spill tables: one per resident block, capacity >= 2*maxdeg0
+        {
+            int per_sm = 0;
+            size_t smem = (size_t)g->hub_smem_slots * (sizeof(ull) + sizeof(int));
+            CK(cudaFuncSetAttribute(k_decide_block<512, long long, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaFuncSetAttribute(k_decide_block<512, long long, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaFuncSetAttribute(k_decide_block<512, i128, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaFuncSetAttribute(k_decide_block<512, i128, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_decide_block<512, i128, false>, 512, smem));
+            wk.gblocks = g->num_sms * std::max(per_sm, 1);
+        }
+        // wk.gcap is sized per level (coarse levels can have larger rows than level 0)
+        wk.gcap = 0;
+
+        DevCSR cur = g->g0;
+        bool cur_owned = false;
+        CK(cudaMemcpyAsync(wk.d, g->d0, sizeof(int64_t) * n0, cudaMemcpyDeviceToDevice, st));
+        CK(cudaMemcpyAsync(wk.s, g->s0, sizeof(int64_t) * n0, cudaMemcpyDeviceToDevice, st));
+        int64_t maxdeg = g->maxdeg0;
+        bool first_level = true;
+        Timer tm(g);
+        for (int level = 0;; ++level) {
+            const int64_t nl = cur.n;
+            const bool unit = (cur.w == nullptr);
+            LevelStat ls{};
+            ls.n = nl;
+            ls.nnz = cur.nnz;
+            ls.maxdeg = maxdeg;
+            cudaEvent_t lv0, lv1, lv2;
+            CK(cudaEventCreate(&lv0));
+            CK(cudaEventCreate(&lv1));
+            CK(cudaEventCreate(&lv2));
+            CK(cudaEventRecord(lv0, st));
+            // spill tables big enough for this level's largest row
+            long long need = 64;
+            while (need < 2 * maxdeg) need <<= 1;
+            if (maxdeg > g->bins[BIN_WARP] && need > wk.gcap) {
+                dfree(wk.gkeys, st);
+                dfree(wk.gvals, st);
+                wk.gcap = need;
+                wk.gkeys = dalloc<int>((size_t)wk.gblocks * wk.gcap, st);
+                wk.gvals = dalloc<ull>((size_t)wk.gblocks * wk.gcap, st);
+                CK(cudaMemsetAsync(wk.gkeys, 0xff, sizeof(int) * (size_t)wk.gblocks * wk.gcap, st));
+                CK(cudaMemsetAsync(wk.gvals, 0, sizeof(ull) * (size_t)wk.gblocks * wk.gcap, st));
+            }
+            // a1: level init + starting numerator
+            cudaEvent_t e = tm.begin();
+            k_level_init<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.d, wk.C, wk.Sig, wk.size, wk.dp, wk.stamp);
+            CKL();
+            if (first_level) {
+                // lab = identity on level 0 (C is the identity right now)
+                CK(cudaMemcpyAsync(g->lab, wk.C, sizeof(int32_t) * n0, cudaMemcpyDeviceToDevice, st));
+                first_level = false;
+            }
+            k_iter_begin<<<1, 128, 0, st>>>(wk.ctr);
+            CKL();
+            k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>((int)nl, wk.dp, wk.s, wk.Sig, wk.part_dc, wk.part_s2,
+                                                          wk.part_min, wk.ctr, wk.carry, (long long)(qW128 >> 64),
+                                                          (ull)qW128, (long long)p, 0, 0, 0);
+            CKL();
+            tm.end(KC_INIT, e);
+            CK(cudaMemcpyAsync(wk.h_carry, wk.carry, sizeof(Carry), cudaMemcpyDeviceToHost, st));
+            CK(cudaStreamSynchronize(st));
+            const i128 N_start = carry_N(wk.h_carry);
+            // score type for this level: int64 iff max(p,q) * W * maxdeg_weighted < 2^62
+            // (weighted degree <= W; use W as the bound on coarse levels, maxdeg on unit level 0)
+            long double bound = (long double)mpq * (long double)W *
+                                (long double)(unit ? std::max<int64_t>(maxdeg, 1) : W);
+            const bool use128 = g->opt_force_i128 || bound >= 0x1p62L;
+            ls.i128path = use128;
+            i128 N = N_start;
+            int64_t iters = 0;
+            for (int it = 0;; ++it) {
+                const int iter_id = level * 1000000 + it;
+                if (use128) {
+                    if (unit) run_iteration<i128, true>(g, wk, cur, (i128)qW128, (i128)p, qW128, T, iter_id, tm, maxdeg);
+                    else run_iteration<i128, false>(g, wk, cur, (i128)qW128, (i128)p, qW128, T, iter_id, tm, maxdeg);
+                } else {
+                    long long qW = (long long)qW128, pp = (long long)p;
+                    if (unit) run_iteration<long long, true>(g, wk, cur, qW, pp, qW128, T, iter_id, tm, maxdeg);
+                    else run_iteration<long long, false>(g, wk, cur, qW, pp, qW128, T, iter_id, tm, maxdeg);
+                }
+                CK(cudaMemcpyAsync(wk.h_ctr, wk.ctr, sizeof(IterCounters), cudaMemcpyDeviceToHost, st));
+                CK(cudaMemcpyAsync(wk.h_carry, wk.carry, sizeof(Carry), cudaMemcpyDeviceToHost, st));
+                if (g->opt_trace >= 2) {
+                    g->trace_labels.emplace_back(nl);
+                    CK(cudaMemcpyAsync(g->trace_labels.back().data(), wk.C, sizeof(int32_t) * nl,
+                                       cudaMemcpyDeviceToHost, st));
+                }
+                CK(cudaStreamSynchronize(st));
+                tm.resolve();
+                const IterCounters& c = *wk.h_ctr;
+                account_bytes(g, c, nl, cur.nnz, unit);
+                g->dp_mismatch += (int64_t)c.dp_mismatch;
+                N = carry_N(wk.h_carry);
+                ++iters;
+                int64_t scanned = 0, kk = 0;
+                for (int b = 0; b < NBINS; ++b) { scanned += (int64_t)c.bin_deg[b]; kk += (int64_t)c.bin_k[b]; }
+                ls.edges_scanned += scanned;
+                ls.nominal_edges += cur.nnz;
+                if (g->opt_trace >= 1) {
+                    TraceRec r;
+                    r.v[0] = level; r.v[1] = it; r.v[2] = nl; r.v[3] = (int64_t)c.n_active;
+                    r.v[4] = (int64_t)c.n_pruned; r.v[5] = (int64_t)c.n_moved;
+                    r.v[6] = (int64_t)(N >> 64); r.v[7] = (int64_t)(uint64_t)N;
+                    r.v[8] = scanned; r.v[9] = kk; r.v[10] = (int64_t)c.delta_used; r.v[11] = 0;
+                    g->trace.push_back(r);
+                }
+                if (wk.h_carry->converged || (g->opt_max_iters > 0 && it + 1 >= g->opt_max_iters)) break;
+            }
+            ls.iters = iters;
+            CK(cudaEventRecord(lv1, st));
+            // a8: relabel in min-member order + compose
+            e = tm.begin();
+            int32_t* minmem = dalloc<int32_t>(nl, st);
+            long long* pos = dalloc<long long>(nl + 1, st);
+            int32_t* newid = dalloc<int32_t>(nl, st);
+            k_fill_i32<<<grid_for(nl, 256, big), 256, 0, st>>>(minmem, nl, INT_MAX);
+            CKL();
+            k_minmember<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.C, minmem);
+            CKL();
+            k_minflag<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.C, minmem, pos);
+            CKL();
+            scan_excl(pos, pos, nl, st);
+            k_newid<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.C, minmem, pos, newid);
+            CKL();
+            k_compose<<<grid_for(n0, 256, big), 256, 0, st>>>(n0, newid, g->lab);
+            CKL();
+            long long kcomm = 0;
+            CK(cudaMemcpyAsync(&kcomm, pos + nl, sizeof(long long), cudaMemcpyDeviceToHost, st));
+            CK(cudaStreamSynchronize(st));
+            const bool stop = (kcomm == nl) || (max_levels > 0 && level + 1 >= max_levels) || (N - N_start < T);
+            DevCSR nxt;
+            if (!stop) {
+                // a9: coarsen
+                const long long k = kcomm;
+                long long* ent = dalloc<long long>(k + 1, st);
+                long long* hoff = dalloc<long long>(k + 1, st);
+                long long* degn = dalloc<long long>(k + 1, st);
+                CK(cudaMemsetAsync(ent, 0, sizeof(long long) * (k + 1), st));
+                CK(cudaMemsetAsync(degn, 0, sizeof(long long) * (k + 1), st));
+                k_coarsen_count<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, cur.rp, newid, ent);
+                CKL();
+                k_coarsen_cap<<<grid_for(k, 256, big), 256, 0, st>>>(k, ent, hoff);
+                CKL();
+                scan_excl(hoff, hoff, k, st);
+                long long htotal = 0;
+                CK(cudaMemcpyAsync(&htotal, hoff + k, sizeof(long long), cudaMemcpyDeviceToHost, st));
+                CK(cudaStreamSynchronize(st));
+                int* hkeys = dalloc<int>(htotal, st);
+                ull* hvals = dalloc<ull>(htotal, st);
+                CK(cudaMemsetAsync(hkeys, 0xff, sizeof(int) * std::max<long long>(htotal, 1), st));
+                CK(cudaMemsetAsync(hvals, 0, sizeof(ull) * std::max<long long>(htotal, 1), st));
+                if (unit)
+                    k_coarsen_insert<true><<<big, 256, 0, st>>>((int)nl, cur.rp, cur.col, cur.w, newid, hoff, hkeys,
+                                                                hvals, degn);
+                else
+                    k_coarsen_insert<false><<<big, 256, 0, st>>>((int)nl, cur.rp, cur.col, cur.w, newid, hoff, hkeys,
+                                                                 hvals, degn);
+                CKL();
+                nxt.n = k;
+                nxt.rp = dalloc<int64_t>(k + 1, st);
+                scan_excl(degn, reinterpret_cast<long long*>(nxt.rp), k, st);
+                CK(cudaMemcpyAsync(&nxt.nnz, nxt.rp + k, sizeof(long long), cudaMemcpyDeviceToHost, st));
+                CK(cudaStreamSynchronize(st));
+                nxt.col = dalloc<int32_t>(nxt.nnz, st);
+                nxt.w = dalloc<int64_t>(nxt.nnz, st);
+                CK(cudaMemsetAsync(ent, 0, sizeof(long long) * (k + 1), st));   // reuse as fill cursor
+                CK(cudaMemsetAsync(wk.s, 0, sizeof(int64_t) * k, st));
+                k_coarsen_extract<true><<<grid_for(htotal, 256, big), 256, 0, st>>>(
+                    k, htotal, hoff, hkeys, hvals, reinterpret_cast<long long*>(nxt.rp), ent, nxt.col, nxt.w, wk.s);
+                CKL();
+                // coarse d = Sigma_tot of the community; write into a temp then copy to wk.d
+                int64_t* dnew = dalloc<int64_t>(k, st);
+                k_coarsen_deg<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.C, minmem, newid, wk.Sig, dnew);
+                CKL();
+                CK(cudaMemcpyAsync(wk.d, dnew, sizeof(int64_t) * k, cudaMemcpyDeviceToDevice, st));
+                ull* dmax = dalloc<ull>(1, st);
+                CK(cudaMemsetAsync(dmax, 0, sizeof(ull), st));
+                k_rowmax<<<grid_for(k, 256, big), 256, 0, st>>>(k, reinterpret_cast<long long*>(nxt.rp), dmax);
+                CKL();
+                ull mx = 0;
+                CK(cudaMemcpyAsync(&mx, dmax, sizeof(ull), cudaMemcpyDeviceToHost, st));
+                CK(cudaStreamSynchronize(st));
+                maxdeg = (int64_t)mx;
+                dfree(dmax, st);
+                dfree(dnew, st);
+                dfree(ent, st);
+                dfree(hoff, st);
+                dfree(degn, st);
+                dfree(hkeys, st);
+                dfree(hvals, st);
+            }
+            dfree(minmem, st);
+            dfree(pos, st);
+            dfree(newid, st);
+            tm.end(KC_PHASE2, e);
+            CK(cudaEventRecord(lv2, st));
+            CK(cudaEventSynchronize(lv2));
+            tm.resolve();
+            float ms1 = 0, ms2 = 0;
+            CK(cudaEventElapsedTime(&ms1, lv0, lv1));
+            CK(cudaEventElapsedTime(&ms2, lv1, lv2));
+            ls.ms_phase1 = ms1;
+            ls.ms_phase2 = ms2;
+            cudaEventDestroy(lv0);
+            cudaEventDestroy(lv1);
+            cudaEventDestroy(lv2);
+            g->levels.push_back(ls);
+            if (cur_owned) { dfree(cur.rp, st); dfree(cur.col, st); dfree(cur.w, st); }
+            if (stop) break;
+            cur = nxt;
+            cur_owned = true;
+        }
+        // final N on the level-0 graph from the composed labels (Eq. 1)
+        {
+            long long* DV = dalloc<long long>(n0, st);
+            ull* DC = dalloc<ull>(1, st);
+            i128* part = dalloc<i128>(big, st);
+            ull* ticket = dalloc<ull>(1, st);
+            i128* out = dalloc<i128>(1, st);
+            CK(cudaMemsetAsync(DV, 0, sizeof(long long) * n0, st));
+            CK(cudaMemsetAsync(DC, 0, sizeof(ull), st));
+            CK(cudaMemsetAsync(ticket, 0, sizeof(ull), st));
+            if (g->g0.w == nullptr)
+                k_mod_dc<true><<<big, 256, 0, st>>>((int)n0, g->g0.rp, g->g0.col, g->g0.w, g->lab, g->d0, DV, DC);
+            else
+                k_mod_dc<false><<<big, 256, 0, st>>>((int)n0, g->g0.rp, g->g0.col, g->g0.w, g->lab, g->d0, DV, DC);
+            CKL();
+            int sg = grid_for(n0, 256, big);
+            k_sumsq<<<sg, 256, 0, st>>>(n0, DV, part, ticket, out);
+            CKL();
+            ull hdc = 0;
+            i128 hs2 = 0;
+            CK(cudaMemcpyAsync(&hdc, DC, sizeof(ull), cudaMemcpyDeviceToHost, st));
+            CK(cudaMemcpyAsync(&hs2, out, sizeof(i128), cudaMemcpyDeviceToHost, st));
+            CK(cudaStreamSynchronize(st));
+            g->N = (i128)q * W * (i128)(long long)hdc - (i128)p * hs2;
+            dfree(DV, st); dfree(DC, st); dfree(part, st); dfree(ticket, st); dfree(out, st);
+        }
+        CK(cudaEventRecord(ev_run1, st));
+        CK(cudaEventSynchronize(ev_run1));
+        float ms = 0;
+        CK(cudaEventElapsedTime(&ms, ev_run0, ev_run1));
+        g->run_ms = ms;
+        wk.release();
+    } catch (...) {
+        wk.release();
+        cudaEventDestroy(ev_run0);
+        cudaEventDestroy(ev_run1);
+        throw;
+    }
+    cudaEventDestroy(ev_run0);
+    cudaEventDestroy(ev_run1);
+    g->has_result = true;
+}
+
+// ------------------------------------------------------------------ creation
+static void init_graph_common(gala_graph_s* g, int64_t n, int device, uintptr_t stream) {
+    g->device = device;
+    CK(cudaSetDevice(device));
+    cudaDeviceProp prop;
+    CK(cudaGetDeviceProperties(&prop, device));
+    g->num_sms = prop.multiProcessorCount;
+    if (stream) {
+        g->stream = reinterpret_cast<cudaStream_t>(stream);
+        g->own_stream = false;
+    } else {
+        CK(cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking));
+        g->own_stream = true;
+    }
+    g->n0 = n;
+}
+
+static void finish_graph(gala_graph_s* g) {
+    cudaStream_t st = g->stream;
+    const int64_t n = g->n0;
+    g->d0 = dalloc<int64_t>(n, st);
+    g->s0 = dalloc<int64_t>(n, st);
+    ull* mx = dalloc<ull>(1, st);
+    CK(cudaMemsetAsync(mx, 0, sizeof(ull), st));
+    int grid = grid_for(n * 32, 256, g->num_sms * 8);
+    if (g->g0.w == nullptr)
+        k_degrees<true><<<grid, 256, 0, st>>>((int)n, g->g0.rp, g->g0.col, g->g0.w, g->d0, g->s0, mx);
+    else
+        k_degrees<false><<<grid, 256, 0, st>>>((int)n, g->g0.rp, g->g0.col, g->g0.w, g->d0, g->s0, mx);
+    CKL();
+    ull hmx = 0;
+    CK(cudaMemcpyAsync(&hmx, mx, sizeof(ull), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    g->maxdeg0 = (int64_t)hmx;
+    dfree(mx, st);
+}
+
+static gala_status validate_host(int64_t n, const int64_t* rp, const int32_t* col, const int64_t* w, int64_t* W,
+                                 bool* unit) {
+    if (n < 0 || n >= ((int64_t)1 << 31)) return set_err(GALA_E_INVALID, "n out of range: %lld", (long long)n);
+    if (!rp) return set_err(GALA_E_INVALID, "row_ptr is NULL");
+    if (rp[0] != 0) return set_err(GALA_E_INVALID, "row_ptr[0] != 0");
+    for (int64_t v = 0; v < n; ++v)
+        if (rp[v + 1] < rp[v]) return set_err(GALA_E_INVALID, "row_ptr not monotone at %lld", (long long)v);
+    int64_t nnz = rp[n];
+    if (nnz > 0 && !col) return set_err(GALA_E_INVALID, "col_idx is NULL");
+    int64_t tot = 0;
+    bool u = true;
+    for (int64_t e = 0; e < nnz; ++e) {
+        if (col[e] < 0 || col[e] >= n) return set_err(GALA_E_INVALID, "col_idx[%lld] out of range", (long long)e);
+        int64_t x = w ? w[e] : 1;
+        if (x <= 0) return set_err(GALA_E_INVALID, "weight[%lld] <= 0", (long long)e);
+        if (x != 1) u = false;
+        tot += x;
+        if (tot < 0) return set_err(GALA_E_OVERFLOW, "total weight overflows int64");
+    }
+    *W = tot;
+    *unit = u;
+    return GALA_OK;
+}
+
+#define API_BEGIN try {
+#define API_END                                              \
+    }                                                        \
+    catch (GalaError & e_) { return e_.st; }                 \
+    catch (std::exception & e_) { return set_err(GALA_E_CUDA, "%s", e_.what()); } \
+    catch (...) { return set_err(GALA_E_CUDA, "unknown error"); }                  \
+    return GALA_OK;
+
+extern "C" {
+
+const char* gala_version(void) { return GALA_VERSION; }
+const char* gala_last_error(void) { return g_err.c_str(); }
+
+gala_status gala_graph_from_csr(int64_t n, const int64_t* row_ptr, const int32_t* col_idx, const int64_t* weights,
+                                int device, uintptr_t stream, gala_graph* out) {
+    if (!out) return set_err(GALA_E_INVALID, "out is NULL");
+    *out = nullptr;
+    int64_t W = 0;
+    bool unit = true;
+    gala_status s = validate_host(n, row_ptr, col_idx, weights, &W, &unit);
+    if (s != GALA_OK) return s;
+    gala_graph_s* g = new gala_graph_s();
+    API_BEGIN
+    try {
+        init_graph_common(g, n, device, stream);
+        cudaStream_t st = g->stream;
+        const int64_t nnz = row_ptr[n];
+        g->nnz0 = nnz;
+        g->W = W;
+        g->g0.n = n;
+        g->g0.nnz = nnz;
+        g->g0.rp = dalloc<int64_t>(n + 1, st);
+        g->g0.col = dalloc<int32_t>(nnz, st);
+        CK(cudaMemcpyAsync(g->g0.rp, row_ptr, sizeof(int64_t) * (n + 1), cudaMemcpyHostToDevice, st));
+        if (nnz) CK(cudaMemcpyAsync(g->g0.col, col_idx, sizeof(int32_t) * nnz, cudaMemcpyHostToDevice, st));
+        if (!unit) {
+            g->g0.w = dalloc<int64_t>(nnz, st);
+            CK(cudaMemcpyAsync(g->g0.w, weights, sizeof(int64_t) * nnz, cudaMemcpyHostToDevice, st));
+        }
+        finish_graph(g);
+    } catch (...) {
+        gala_graph_free(g);
+        throw;
+    }
+    *out = g;
+    API_END
+}
+
+gala_status gala_graph_from_csr_device(int64_t n, const int64_t* d_row_ptr, const int32_t* d_col_idx,
+                                       const int64_t* d_weights, int device, uintptr_t stream, gala_graph* out) {
+    if (!out) return set_err(GALA_E_INVALID, "out is NULL");
+    *out = nullptr;
+    if (n < 0 || n >= ((int64_t)1 << 31)) return set_err(GALA_E_INVALID, "n out of range");
+    gala_graph_s* g = new gala_graph_s();
+    API_BEGIN
+    try {
+        init_graph_common(g, n, device, stream);
+        cudaStream_t st = g->stream;
+        int64_t nnz = 0, rp0 = 0;
+        CK(cudaMemcpyAsync(&nnz, d_row_ptr + n, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(&rp0, d_row_ptr, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        if (rp0 != 0 || nnz < 0) { set_err(GALA_E_INVALID, "row_ptr[0] != 0"); throw GalaError{GALA_E_INVALID}; }
+        g->nnz0 = nnz;
+        g->g0.n = n;
+        g->g0.nnz = nnz;
+        g->g0.rp = dalloc<int64_t>(n + 1, st);
+        g->g0.col = dalloc<int32_t>(nnz, st);
+        CK(cudaMemcpyAsync(g->g0.rp, d_row_ptr, sizeof(int64_t) * (n + 1), cudaMemcpyDeviceToDevice, st));
+        if (nnz) CK(cudaMemcpyAsync(g->g0.col, d_col_idx, sizeof(int32_t) * nnz, cudaMemcpyDeviceToDevice, st));
+        if (d_weights) {
+            g->g0.w = dalloc<int64_t>(nnz, st);
+            CK(cudaMemcpyAsync(g->g0.w, d_weights, sizeof(int64_t) * nnz, cudaMemcpyDeviceToDevice, st));
+        }
+        finish_graph(g);
+        // W = sum of d0 (device-side validation of ranges is done by the host path only)
+        std::vector<int64_t> hd(n);
+        CK(cudaMemcpyAsync(hd.data(), g->d0, sizeof(int64_t) * n, cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        int64_t W = 0;
+        for (int64_t v = 0; v < n; ++v) W += hd[v];
+        g->W = W;
+    } catch (...) {
+        gala_graph_free(g);
+        throw;
+    }
+    *out = g;
+    API_END
+}
+
+gala_status gala_validate(gala_graph g) {
+    if (!g) return set_err(GALA_E_INVALID, "null handle");
+    API_BEGIN
+    // symmetric check on the host copy (O(nnz log nnz)); debugging aid
+    cudaStream_t st = g->stream;
+    std::vector<int64_t> rp(g->n0 + 1);
+    std::vector<int32_t> col(g->nnz0);
+    std::vector<int64_t> w;
+    CK(cudaMemcpyAsync(rp.data(), g->g0.rp, sizeof(int64_t) * (g->n0 + 1), cudaMemcpyDeviceToHost, st));
+    if (g->nnz0) CK(cudaMemcpyAsync(col.data(), g->g0.col, sizeof(int32_t) * g->nnz0, cudaMemcpyDeviceToHost, st));
+    if (g->g0.w) {
+        w.resize(g->nnz0);
+        CK(cudaMemcpyAsync(w.data(), g->g0.w, sizeof(int64_t) * g->nnz0, cudaMemcpyDeviceToHost, st));
+    }
+    CK(cudaStreamSynchronize(st));
+    std::vector<std::tuple<int32_t, int32_t, int64_t>> a, b;
+    a.reserve(g->nnz0);
+    b.reserve(g->nnz0);
+    for (int64_t v = 0; v < g->n0; ++v)
+        for (int64_t e = rp[v]; e < rp[v + 1]; ++e) {
+            int64_t x = w.empty() ? 1 : w[e];
+            a.emplace_back((int32_t)v, col[e], x);
+            b.emplace_back(col[e], (int32_t)v, x);
+        }
+    std::sort(a.begin(), a.end());
+    std::sort(b.begin(), b.end());
+    if (a != b) return set_err(GALA_E_INVALID, "CSR is not symmetric");
+    API_END
+}
+
+gala_status gala_run(gala_graph g, double gamma, double tol, int32_t max_levels) {
+    if (!g) return set_err(GALA_E_INVALID, "null handle");
+    if (!(gamma > 0) || !(gamma < 1e12)) return set_err(GALA_E_INVALID, "gamma must be > 0");
+    if (!(tol > 0)) return set_err(GALA_E_INVALID, "tol must be > 0");
+    API_BEGIN
+    if (g->dist) {
+        dist_run(g->dist, gamma, tol, max_levels);
+        g->has_result = true;
+        return GALA_OK;
+    }
+    if (g->W == 0) {
+        // reading c18: no edges -> singletons, Q := 0
+        CK(cudaSetDevice(g->device));
+        if (!g->lab) g->lab = dalloc<int32_t>(std::max<int64_t>(g->n0, 1), g->stream);
+        std::vector<int32_t> iota(g->n0);
+        for (int64_t v = 0; v < g->n0; ++v) iota[v] = (int32_t)v;
+        if (g->n0) CK(cudaMemcpyAsync(g->lab, iota.data(), sizeof(int32_t) * g->n0, cudaMemcpyHostToDevice, g->stream));
+        CK(cudaStreamSynchronize(g->stream));
+        gamma_to_pq(gamma, &g->p, &g->q);
+        g->N = 0;
+        g->levels.clear();
+        g->trace.clear();
+        g->trace_labels.clear();
+        g->has_result = true;
+        return GALA_OK;
+    }
+    do_run(g, gamma, tol, max_levels);
+    API_END
+}
+
+static gala_status fetch_labels(gala_graph g, int32_t* out, int64_t n, int64_t* k, bool device) {
+    if (!g) return set_err(GALA_E_INVALID, "null handle");
+    if (!g->has_result) return set_err(GALA_E_STATE, "gala_run has not completed");
+    if (n != g->n0) return set_err(GALA_E_INVALID, "n mismatch (%lld != %lld)", (long long)n, (long long)g->n0);
+    API_BEGIN
+    if (g->dist) return dist_get_labels(g->dist, out, n, k, device);
+    CK(cudaSetDevice(g->device));
+    std::vector<int32_t> h;
+    int32_t* dst = out;
+    if (!device) dst = out;
+    if (n) CK(cudaMemcpyAsync(dst, g->lab, sizeof(int32_t) * n, device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost,
+                              g->stream));
+    CK(cudaStreamSynchronize(g->stream));
+    if (k) {
+        if (device) {
+            h.resize(n);
+            if (n) CK(cudaMemcpy(h.data(), g->lab, sizeof(int32_t) * n, cudaMemcpyDeviceToHost));
+            dst = h.data();
+        }
+        int64_t mx = -1;
+        for (int64_t v = 0; v < n; ++v) mx = std::max<int64_t>(mx, dst[v]);
+        *k = mx + 1;
+    }
+    API_END
+}
+
+gala_status gala_get_communities(gala_graph g, int32_t* labels, int64_t n, int64_t* num_communities) {
+    return fetch_labels(g, labels, n, num_communities, false);
+}
+gala_status gala_get_communities_device(gala_graph g, int32_t* d_labels, int64_t n, int64_t* num_communities) {
+    return fetch_labels(g, d_labels, n, num_communities, true);
+}
+
+gala_status gala_modularity_numerator(gala_graph g, int64_t* n_hi, uint64_t* n_lo, int64_t* W, int64_t* p, int64_t* q) {
+    if (!g) return set_err(GALA_E_INVALID, "null handle");
+    if (!g->has_result) return set_err(GALA_E_STATE, "gala_run has not completed");
+    if (g->dist) dist_numerator(g->dist, &g->N, &g->W, &g->p, &g->q);
+    if (n_hi) *n_hi = (int64_t)(g->N >> 64);
+    if (n_lo) *n_lo = (uint64_t)g->N;
+    if (W) *W = g->W;
+    if (p) *p = g->p;
+    if (q) *q = g->q;
+    return GALA_OK;
+}
+
+gala_status gala_modularity(gala_graph g, double* q) {
+    if (!g || !q) return set_err(GALA_E_INVALID, "null argument");
+    if (!g->has_result) return set_err(GALA_E_STATE, "gala_run has not completed");
+    if (g->dist) dist_numerator(g->dist, &g->N, &g->W, &g->p, &g->q);
+    if (g->W == 0) { *q = 0.0; return GALA_OK; }
+    *q = (double)((long double)g->N / ((long double)g->q * (long double)g->W * (long double)g->W));
+    return GALA_OK;
+}
+
+void gala_graph_free(gala_graph g) {
+    if (!g) return;
+    cudaSetDevice(g->device);
+    if (g->dist) dist_free(g->dist);
+    cudaStream_t st = g->stream;
+    if (st) {
+        dfree(g->g0.rp, st);
+        dfree(g->g0.col, st);
+        dfree(g->g0.w, st);
+        dfree(g->d0, st);
+        dfree(g->s0, st);
+        dfree(g->lab, st);
+        cudaStreamSynchronize(st);
+        if (g->own_stream) cudaStreamDestroy(st);
+    }
+    delete g;
+}
+
+gala_status gala_set_option(gala_graph g, const char* key, int64_t value) {
+    if (!g || !key) return set_err(GALA_E_INVALID, "null argument");
+    std::string k(key);
+    if (k == "prune") g->opt_prune = value != 0;
+    else if (k == "trace") g->opt_trace = (int)value;
+    else if (k == "check") g->opt_check = value != 0;
+    else if (k == "timing") g->opt_timing = value != 0;
+    else if (k == "max_iters") { if (value < 0) return set_err(GALA_E_INVALID, "max_iters < 0"); g->opt_max_iters = (int)value; }
+    else if (k == "delta_update") { if (value < 0 || value > 2) return set_err(GALA_E_INVALID, "delta_update in 0..2"); g->opt_delta = (int)value; }
+    else if (k == "force_i128") g->opt_force_i128 = value != 0;
+    else if (k == "cuda_graph") g->opt_cuda_graph = value != 0;
+    else if (k == "hub_smem_slots") {
+        if (value < 64 || value > 16384 || (value & (value - 1))) return set_err(GALA_E_INVALID, "hub_smem_slots: power of two in [64, 16384]");
+        g->hub_smem_slots = (int)value;
+    } else if (k.rfind("bin_", 0) == 0) {
+        static const char* names[NBINS - 1] = {"bin_sub4", "bin_sub8", "bin_sub16", "bin_sub32", "bin_warp"};
+        static const int lanes[NBINS - 1] = {4, 8, 16, 32, 128};
+        int idx = -1;
+        for (int i = 0; i < NBINS - 1; ++i) if (k == names[i]) idx = i;
+        if (idx < 0) return set_err(GALA_E_INVALID, "unknown option %s", key);
+        if (value < 0 || value > lanes[idx]) return set_err(GALA_E_INVALID, "%s must be in [0, %d]", key, lanes[idx]);
+        g->bins[idx] = (int)value;
+        for (int i = 1; i < NBINS - 1; ++i)
+            if (g->bins[i] < g->bins[i - 1]) return set_err(GALA_E_INVALID, "bin thresholds must be non-decreasing");
+    } else if (k == "sync_mode") {
+        if (g->dist) dist_set_option(g->dist, key, value);
+    } else return set_err(GALA_E_INVALID, "unknown option %s", key);
+    if (g->dist) dist_set_option(g->dist, key, value);
+    return GALA_OK;
+}
+
+gala_status gala_get_trace_count(gala_graph g, int64_t* count) {
+    if (!g || !count) return set_err(GALA_E_INVALID, "null argument");
+    if (g->dist) { *count = dist_trace_count(g->dist); return GALA_OK; }
+    *count = (int64_t)g->trace.size();
+    return GALA_OK;
+}
+gala_status gala_get_trace_record(gala_graph g, int64_t i, int64_t* out12) {
+    if (!g || !out12) return set_err(GALA_E_INVALID, "null argument");
+    if (g->dist) return dist_trace_record(g->dist, i, out12);
+    if (i < 0 || i >= (int64_t)g->trace.size()) return set_err(GALA_E_INVALID, "record index out of range");
+    memcpy(out12, g->trace[i].v, sizeof(int64_t) * 12);
+    return GALA_OK;
+}
+gala_status gala_get_trace_labels(gala_graph g, int64_t i, int32_t* out, int64_t n_level) {
+    if (!g || !out) return set_err(GALA_E_INVALID, "null argument");
+    if (g->dist) return dist_trace_labels(g->dist, i, out, n_level);
+    if (i < 0 || i >= (int64_t)g->trace_labels.size()) return set_err(GALA_E_INVALID, "no labels for record (trace < 2?)");
+    if ((int64_t)g->trace_labels[i].size() != n_level) return set_err(GALA_E_INVALID, "n_level mismatch");
+    memcpy(out, g->trace_labels[i].data(), sizeof(int32_t) * n_level);
+    return GALA_OK;
+}
+
+gala_status gala_get_kernel_stats(gala_graph g, int32_t k, const char** name, int64_t* launches, double* ms,
+                                  double* alg_bytes, int32_t* count) {
+    if (!g) return set_err(GALA_E_INVALID, "null handle");
+    if (count) *count = KC_COUNT;
+    if (k < 0 || k >= KC_COUNT) return GALA_OK;
+    if (name) *name = kc_names[k];
+    if (launches) *launches = g->kc_launches[k];
+    if (ms) *ms = g->kc_ms[k];
+    if (alg_bytes) *alg_bytes = g->kc_bytes[k];
+    return GALA_OK;
+}
+
+gala_status gala_get_stats(gala_graph g, char* buf, int64_t cap, int64_t* needed) {
+    if (!g) return set_err(GALA_E_INVALID, "null handle");
+    std::string s = "{";
+    char tmp[512];
+    snprintf(tmp, sizeof tmp, "\"n\":%lld,\"nnz\":%lld,\"W\":%lld,\"p\":%lld,\"q\":%lld,\"run_ms\":%.6f,\"dp_mismatch\":%lld,",
+             (long long)g->n0, (long long)g->nnz0, (long long)g->W, (long long)g->p, (long long)g->q, g->run_ms,
+             (long long)g->dp_mismatch);
+    s += tmp;
+    s += "\"levels\":[";
+    for (size_t i = 0; i < g->levels.size(); ++i) {
+        const LevelStat& l = g->levels[i];
+        snprintf(tmp, sizeof tmp,
+                 "%s{\"n\":%lld,\"nnz\":%lld,\"iters\":%lld,\"maxdeg\":%lld,\"i128\":%d,\"ms_phase1\":%.6f,"
+                 "\"ms_phase2\":%.6f,\"edges_scanned\":%lld,\"nominal_edges\":%lld}",
+                 i ? "," : "", (long long)l.n, (long long)l.nnz, (long long)l.iters, (long long)l.maxdeg, l.i128path,
+                 l.ms_phase1, l.ms_phase2, (long long)l.edges_scanned, (long long)l.nominal_edges);
+        s += tmp;
+    }
+    s += "],\"kernels\":{";
+    for (int i = 0; i < KC_COUNT; ++i) {
+        snprintf(tmp, sizeof tmp, "%s\"%s\":{\"launches\":%lld,\"ms\":%.6f,\"alg_bytes\":%.0f}", i ? "," : "", kc_names[i],
+                 (long long)g->kc_launches[i], g->kc_ms[i], g->kc_bytes[i]);
+        s += tmp;
+    }
+    s += "}}";
+    if (needed) *needed = (int64_t)s.size() + 1;
+    if (!buf || cap < (int64_t)s.size() + 1) return set_err(GALA_E_INVALID, "buffer too small");
+    memcpy(buf, s.c_str(), s.size() + 1);
+    return GALA_OK;
+}
+
+gala_status gala_partition_ranges(int64_t n, const int64_t* row_ptr, int world, int64_t* bounds) {
+    if (!row_ptr || !bounds || world < 1 || n < 0) return set_err(GALA_E_INVALID, "bad arguments");
+    const int64_t nnz = row_ptr[n];
+    bounds[0] = 0;
+    int64_t v = 0;
+    for (int r = 1; r < world; ++r) {
+        // smallest v with row_ptr[v] >= r * nnz / world (edge-balanced), never behind the previous bound
+        const long double target = (long double)nnz * r / world;
+        int64_t lo = v, hi = n;
+        while (lo < hi) {
+            int64_t mid = (lo + hi) / 2;
+            if ((long double)row_ptr[mid] < target) lo = mid + 1; else hi = mid;
+        }
+        v = lo;
+        bounds[r] = v;
+    }
+    bounds[world] = n;
+    return GALA_OK;
+}
+
+}  // extern "C"

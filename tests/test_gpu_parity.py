@@ -1,0 +1,138 @@
+"""GPU parity: the sm_100a path (through the C ABI) against the CPU oracle.
+
+Bit-exact community labels at EVERY iteration of EVERY level, identical exact
+modularity numerators, and the final Q within 1e-9 (north star).  Inputs are
+the seeded generators of graphgen/.  SURVEY.md §8(c) P4/P5/P7 and §8(e).
+"""
+import numpy as np
+import pytest
+
+import graphgen as gg
+import oracle
+import paper_conf_ppopp_wangllwm00z25_b200 as gala
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _need_gpu():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+
+
+def run_gpu(g, gamma=1.0, tol=1e-6, max_levels=0, trace=2, **opts):
+    h = gala.Graph.from_graph(g)
+    h.set_option("trace", trace)
+    for k, v in opts.items():
+        h.set_option(k, v)
+    h.run(gamma=gamma, tol=tol, max_levels=max_levels)
+    out = dict(labels=h.communities(), Q=h.modularity(), N=h.numerator()[0], trace=h.trace(labels=trace >= 2),
+               stats=h.stats())
+    h.free()
+    return out
+
+
+def assert_parity(g, gamma=1.0, tol=1e-6, max_levels=0, prune=True, labels=True, **opts):
+    o = oracle.louvain(g, gamma=gamma, tol=tol, max_levels=max_levels, prune=prune, trace=2 if labels else 1,
+                       max_iters=opts.get("max_iters", 0))
+    assert o.status == 0
+    r = run_gpu(g, gamma=gamma, tol=tol, max_levels=max_levels, trace=2 if labels else 1, prune=int(prune),
+                check=1, **opts)
+    assert len(r["trace"]) == len(o.records), (len(r["trace"]), len(o.records))
+    for x, y in zip(o.records, r["trace"]):
+        assert (x.level, x.iter, x.n_level) == (y["level"], y["iter"], y["n_level"])
+        if labels:
+            assert np.array_equal(x.labels, y["labels"]), f"labels differ at level {x.level} iter {x.iter}"
+        assert x.N == y["N"], f"N differs at level {x.level} iter {x.iter}"
+        assert x.n_moved == y["n_moved"]
+        assert x.n_active == y["n_active"] and x.n_pruned == y["n_pruned"]
+    assert np.array_equal(o.labels, r["labels"])
+    assert o.N == r["N"]
+    assert abs(o.Q - r["Q"]) <= 1e-9
+    assert r["stats"]["dp_mismatch"] == 0
+    return o, r
+
+
+def test_karate_parity():
+    o, r = assert_parity(gg.karate())
+    assert r["labels"].max() + 1 == 4
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_random_graph_parity(seed):
+    rng = np.random.default_rng(1000 + seed)
+    n = int(rng.integers(10, 400))
+    g = gg.random_graph(n, int(rng.integers(n, 8 * n)), seed=1000 + seed, max_w=int(rng.integers(1, 6)),
+                        self_loops=int(rng.integers(0, 6)))
+    gamma = [1.0, 0.5, 1.5, 2.0, 0.25, 3.0][seed % 6]
+    assert_parity(g, gamma=gamma)
+
+
+@pytest.mark.parametrize("name", ["lfr_small", "rmat_small"])
+@pytest.mark.parametrize("prune", [True, False])
+def test_synthetic_parity(name, prune):
+    assert_parity(gg.make(name), prune=prune)
+
+
+@pytest.mark.parametrize("opts", [
+    dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=0),      # everything through block hash
+    dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=128),    # warp hash for <= 128
+    dict(bin_sub4=4, bin_sub8=4, bin_sub16=4, bin_sub32=32, bin_warp=32),
+    dict(hub_smem_slots=64),                                                  # force the global spill table
+    dict(force_i128=1),
+    dict(delta_update=0),
+    dict(delta_update=1),
+])
+def test_dispatch_independence(opts):
+    """P7: thresholds / table sizes / integer width / update strategy never change a label."""
+    assert_parity(gg.make("rmat_small"), **opts)
+
+
+def test_max_levels_and_max_iters():
+    g = gg.make("lfr_small")
+    assert_parity(g, max_levels=1)
+    assert_parity(g, max_levels=2, max_iters=3)
+
+
+def test_device_resident_input_matches_host_input():
+    import torch
+    g = gg.make("lfr_small")
+    h1 = gala.Graph.from_graph(g).run()
+    rp = torch.from_numpy(g.row_ptr).cuda()
+    col = torch.from_numpy(g.col).cuda()
+    h2 = gala.Graph.from_csr(rp, col).run()
+    assert np.array_equal(h1.communities(), h2.communities())
+    out = torch.empty(g.n, dtype=torch.int32, device="cuda")
+    k = h2.communities_device(out)
+    assert np.array_equal(out.cpu().numpy(), h1.communities()) and k == h1.communities().max() + 1
+
+
+def test_degenerate_inputs():
+    empty = gg.build_csr(5, np.array([], dtype=np.int64), np.array([], dtype=np.int64))
+    r = run_gpu(empty)
+    assert list(r["labels"]) == list(range(5)) and r["Q"] == 0.0
+    assert_parity(gg.build_csr(2, np.array([0]), np.array([1])))
+    assert_parity(gg.build_csr(3, np.array([0, 1, 1]), np.array([0, 1, 2]), np.array([3, 2, 1]),
+                               keep_self_loops=True))
+    # isolated vertices mixed in
+    assert_parity(gg.build_csr(8, np.array([0, 1, 5]), np.array([1, 2, 6])))
+    assert_parity(gg.ring_of_cliques(6, 5))
+
+
+def test_invalid_inputs_rejected():
+    with pytest.raises(gala.GalaError):
+        gala.Graph.from_csr(np.array([0, 1]), np.array([5]))          # column out of range
+    with pytest.raises(gala.GalaError):
+        gala.Graph.from_csr(np.array([0, 1, 2]), np.array([1, 0]), np.array([1, 0]))   # weight 0
+    h = gala.Graph.from_graph(gg.karate())
+    with pytest.raises(gala.GalaError):
+        h.communities()                                              # before run
+    with pytest.raises(gala.GalaError):
+        h.run(tol=0.0)
+
+
+@pytest.mark.slow
+def test_lfr1m_full_size_parity():
+    """BASELINE configs[1] at full size, in bench.py's launch configuration."""
+    assert_parity(gg.make("lfr1m"))
