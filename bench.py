@@ -1,0 +1,332 @@
+#!/usr/bin/env python
+"""bench.py — GALA Louvain on B200: local-move GTEPS + end-to-end Louvain seconds + modularity.
+
+Contract (driver): `python bench.py --gpus N --steps K --warmup W [--impl reference]` prints ONE
+JSON line on rank 0.  A *step* is one full multi-level Louvain run (gala_run: every SURVEY.md §8(a)
+row: init, MG prune/bin, DecideAndMove, apply, d' update, reductions, relabel, coarsen) over the
+synthetic graph of the workload (default: BASELINE.json configs[1], LFR 1M / mu=0.3), restarting
+from singletons each step.
+
+value  = local-move GTEPS = sum over levels and iterations of the level's CSR entries (the edges the
+         unpruned method traverses; identical for every correct implementation because labels and
+         iteration counts are bit-identical) / step seconds, whole job.  Inputs resident in HBM.
+e2e    = the same metric through the C ABI with HOST inputs: gala_graph_from_csr (H2D) + gala_run +
+         gala_get_communities (D2H) inside the timed region.
+roofline: dominant kernel class (by device time, CUDA events inside the library on its stream)
+         algorithmic bytes / time vs MEASURED_PEAKS.json hbm_gbs.
+cpu_baseline: the CPU oracle (oracle/, plain C + OpenMP) on the same graph, all host cores.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+WORKLOADS = {
+    "lfr1m": "LFR planted partition 1M vertices / ~20M edges, mu=0.3 (BASELINE.json configs[1])",
+    "karate": "Zachary karate club (BASELINE.json configs[0])",
+    "rmat_lj": "R-MAT LiveJournal-shaped 4.8M / 69M (BASELINE.json configs[2])",
+    "orkut": "Orkut-shaped LFR 3.1M / 117M (BASELINE.json configs[3])",
+    "lfr_small": "LFR 20k (test size)",
+}
+METRIC = "local-move GTEPS and end-to-end Louvain seconds at 1/2/4/8 B200; modularity Q"
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)", d
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)", {}
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device: int):
+        self.device = device
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.device}", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *exc):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [x.strip() for x in ln.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                sm.append(float(parts[1]))
+                mx = float(parts[2])
+            except ValueError:
+                continue
+            for nm, val in zip(names, parts[5:9]):
+                if val.lower() == "active":
+                    reasons.add(nm)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": 0}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def nominal_edges(stats: dict) -> int:
+    return sum(lv["nominal_edges"] for lv in stats["levels"])
+
+
+def oracle_baseline(g, steps=1):
+    """The CPU oracle (test infrastructure) on the same graph, all host cores."""
+    import oracle
+    cores = len(os.sched_getaffinity(0))
+    times = []
+    res = None
+    for _ in range(steps):
+        t0 = time.perf_counter()
+        res = oracle.louvain(g, prune=True, trace=1)
+        times.append(time.perf_counter() - t0)
+    edges = 0
+    for lv in res.levels:
+        edges += lv.iters * lv.nnz
+    return dict(seconds=statistics.median(times), edges=edges, cores=cores, Q=res.Q, N=res.N, labels=res.labels,
+                iters=sum(lv.iters for lv in res.levels))
+
+
+def cpu_model():
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                return ln.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return "unknown"
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the CPU oracle as the reference arm (rank 0 only)."""
+    if rank != 0:
+        return
+    import graphgen as gg
+    g = gg.make(args.config)
+    for _ in range(args.warmup):
+        oracle_baseline(g, 1)
+    secs, edges, cores, Q = [], 0, 0, 0.0
+    for _ in range(args.steps):
+        r = oracle_baseline(g, 1)
+        secs.append(r["seconds"])
+        edges, cores, Q = r["edges"], r["cores"], r["Q"]
+    total = sum(secs)
+    value = edges * args.steps / total / 1e9
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "GTEPS", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * total / args.steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+        "config": {"workload": args.config, "desc": WORKLOADS.get(args.config, ""), "n": g.n, "nnz": g.nnz},
+        "louvain_seconds": total / args.steps, "modularity": Q,
+        "cpu_baseline": {"value": value, "unit": "GTEPS", "cores": cores, "kind": "oracle",
+                         "sample": f"full multi-level oracle run on {args.config} per step ({cpu_model()})"},
+        "e2e": {"value": value, "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="gala", choices=["gala", "reference"])
+    ap.add_argument("--config", default="lfr1m", choices=sorted(WORKLOADS))
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-timing", action="store_true", help="disable per-kernel events (roofline)")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3) if args.impl != "reference" else args.warmup
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", str(args.gpus)))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+
+    if args.impl == "reference":
+        return run_reference(args, rank, world)
+
+    import torch
+    import graphgen as gg
+    import paper_conf_ppopp_wangllwm00z25_b200 as gala
+
+    if world > 1:
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl")
+        return run_dist(args, rank, world, local_rank)
+
+    dev = 0
+    torch.cuda.set_device(dev)
+    stream = torch.cuda.Stream(device=dev)
+    g = gg.make(args.config)
+    peak, peak_src, peaks = load_peaks()
+
+    # ------------------------------------------------------------ device-resident timing (value)
+    h = gala.Graph.from_graph(g, device=dev, stream=stream.cuda_stream)
+    h.set_option("timing", 0 if args.no_timing else 1)
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device=dev)   # > 126 MB L2
+    for _ in range(args.warmup):
+        h.run()
+    torch.cuda.synchronize()
+    step_ms, edges, scanned, launches = [], 0, 0, 0
+    kstats = {}
+    with ClockSampler(dev) as clk:
+        for _ in range(args.steps):
+            with torch.cuda.stream(stream):
+                flush.add_(1)                                    # L2 flush between timed steps
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            torch.cuda.synchronize()
+            e0.record(stream)
+            h.run()
+            e1.record(stream)
+            torch.cuda.synchronize()
+            step_ms.append(e0.elapsed_time(e1))
+            st = h.stats()
+            edges += nominal_edges(st)
+            scanned += sum(lv["edges_scanned"] for lv in st["levels"])
+            launches += st["kernel_launches"]
+            for k, v in h.kernel_stats().items():
+                acc = kstats.setdefault(k, dict(launches=0, ms=0.0, alg_bytes=0.0))
+                for f in acc:
+                    acc[f] += v[f]
+    labels = h.communities()
+    Q = h.modularity()
+    last_stats = h.stats()
+    h.free()
+    total_s = sum(step_ms) / 1e3
+    value = edges / total_s / 1e9
+
+    # dominant kernel (by device time) roofline
+    dom = max(kstats.items(), key=lambda kv: kv[1]["ms"]) if kstats else None
+    roofline = None
+    if dom and dom[1]["ms"] > 0:
+        name, ks = dom
+        achieved = ks["alg_bytes"] / (ks["ms"] / 1e3) / 1e9
+        traffic = None
+        tpath = os.path.join(ROOT, "profiles", "traffic.json")
+        if os.path.exists(tpath):
+            t = json.load(open(tpath))
+            traffic = t.get(name, {}).get("dram_bytes_per_launch")
+        roofline = {"bound": "hbm", "kernel": name, "achieved": achieved, "peak": peak, "unit": "GB/s",
+                    "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
+                    "alg_bytes_per_launch": ks["alg_bytes"] / max(ks["launches"], 1),
+                    "avg_launch_us": 1e3 * ks["ms"] / max(ks["launches"], 1)}
+    decide = {k: v for k, v in kstats.items() if k.startswith("decide")}
+    dec_ms = sum(v["ms"] for v in decide.values())
+    dec_by = sum(v["alg_bytes"] for v in decide.values())
+
+    # ------------------------------------------------------------ e2e through the C ABI with host buffers
+    rp = torch.from_numpy(g.row_ptr).pin_memory()
+    col = torch.from_numpy(g.col).pin_memory()
+    lab_host = torch.empty(g.n, dtype=torch.int32).pin_memory()
+    e2e_ms, e2e_edges, iters_total = [], 0, 0
+    import ctypes
+    L = gala.lib()
+    for i in range(args.warmup + args.steps):
+        with torch.cuda.stream(stream):
+            flush.add_(1)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        hh = ctypes.c_void_p()
+        gala._check(L.gala_graph_from_csr(g.n, rp.data_ptr(), col.data_ptr(), None, dev, stream.cuda_stream,
+                                          ctypes.byref(hh)))
+        gala._check(L.gala_run(hh, 1.0, 1e-6, 0))
+        k = ctypes.c_int64()
+        gala._check(L.gala_get_communities(hh, lab_host.data_ptr(), g.n, ctypes.byref(k)))
+        e1.record(stream)
+        torch.cuda.synchronize()
+        gh = gala.Graph(hh, g.n)
+        st = gh.stats()
+        gh.free()
+        if i >= args.warmup:
+            e2e_ms.append(e0.elapsed_time(e1))
+            e2e_edges += nominal_edges(st)
+            iters_total = sum(lv["iters"] for lv in st["levels"])
+    e2e_value = e2e_edges / (sum(e2e_ms) / 1e3) / 1e9
+    h2d = g.row_ptr.nbytes + g.col.nbytes
+    d2h = g.n * 4 + iters_total * 2 * 128
+
+    # ------------------------------------------------------------ CPU oracle baseline
+    cpu = None
+    parity = None
+    if not args.no_cpu_baseline:
+        ob = oracle_baseline(g, 1)
+        cpu = {"value": ob["edges"] / ob["seconds"] / 1e9, "unit": "GTEPS", "cores": ob["cores"], "kind": "oracle",
+               "sample": f"one full multi-level oracle run (prune on) on {args.config}, {ob['seconds']:.2f} s "
+                         f"({cpu_model()})"}
+        parity = bool(np.array_equal(ob["labels"], labels)) and ob["edges"] == edges // args.steps
+
+    lv0 = last_stats["levels"][0]
+    line = {
+        "metric": METRIC, "value": value, "unit": "GTEPS", "n_gpus": 1, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": 1e3 * total_s / args.steps, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": "int64", "data": "synthetic",
+        "config": {"workload": args.config, "desc": WORKLOADS.get(args.config, ""), "n": g.n, "nnz": g.nnz,
+                   "gamma": 1.0, "tol": 1e-6, "prune": 1, "parallelism": "1 GPU",
+                   "l2": "flushed between timed steps (256 MB write)"},
+        "louvain_seconds": total_s / args.steps,
+        "modularity": Q,
+        "levels": len(last_stats["levels"]),
+        "iterations": sum(lv["iters"] for lv in last_stats["levels"]),
+        "gteps_scanned": scanned / total_s / 1e9,
+        "level0_phase1_gteps": lv0["nominal_edges"] / (lv0["ms_phase1"] / 1e3) / 1e9,
+        "decide_roofline": {"achieved": dec_by / (dec_ms / 1e3) / 1e9 if dec_ms else None, "peak": peak,
+                            "frac": (dec_by / (dec_ms / 1e3) / 1e9) / peak if dec_ms else None,
+                            "ms_per_step": dec_ms / args.steps},
+        "kernels_ms_per_step": {k: round(v["ms"] / args.steps, 4) for k, v in sorted(kstats.items())},
+        "roofline": roofline,
+        "cpu_baseline": cpu,
+        "oracle_parity": parity,
+        "e2e": {"value": e2e_value, "unit": "GTEPS", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+                "louvain_seconds": sum(e2e_ms) / 1e3 / len(e2e_ms)},
+        "gpu_launches": launches,
+        "clocks": clk.summary(),
+    }
+    print(json.dumps(line), flush=True)
+
+
+def run_dist(args, rank, world, local_rank):
+    raise SystemExit("multi-GPU bench path not built yet")
+
+
+if __name__ == "__main__":
+    main()

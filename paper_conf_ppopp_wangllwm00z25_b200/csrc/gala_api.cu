@@ -48,7 +48,13 @@ struct GalaError {
             throw GalaError{e_ == cudaErrorMemoryAllocation ? GALA_E_NOMEM : GALA_E_CUDA};        \
         }                                                                                          \
     } while (0)
-#define CKL() CK(cudaGetLastError())
+// every kernel launch site is followed by CKL(), which also counts the launch
+static thread_local long long g_launches = 0;
+#define CKL()                       \
+    do {                            \
+        ++g_launches;               \
+        CK(cudaGetLastError());     \
+    } while (0)
 
 // ------------------------------------------------------------------ kernel classes
 enum KClass {
@@ -105,6 +111,7 @@ struct gala_graph_s {
     int64_t kc_launches[KC_COUNT] = {0};
     double run_ms = 0;
     int64_t dp_mismatch = 0;
+    long long launches = 0;   // kernels launched by the last gala_run
     // dist
     DistCtx* dist = nullptr;
 };
@@ -338,6 +345,7 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
     g->levels.clear();
     for (int i = 0; i < KC_COUNT; ++i) { g->kc_ms[i] = 0; g->kc_bytes[i] = 0; g->kc_launches[i] = 0; }
     g->dp_mismatch = 0;
+    const long long launches0 = g_launches;
     int64_t p, q;
     gamma_to_pq(gamma, &p, &q);
     g->p = p;
@@ -629,6 +637,7 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
         float ms = 0;
         CK(cudaEventElapsedTime(&ms, ev_run0, ev_run1));
         g->run_ms = ms;
+        g->launches = g_launches - launches0;
         wk.release();
     } catch (...) {
         wk.release();
@@ -993,9 +1002,10 @@ gala_status gala_get_stats(gala_graph g, char* buf, int64_t cap, int64_t* needed
     if (!g) return set_err(GALA_E_INVALID, "null handle");
     std::string s = "{";
     char tmp[512];
-    snprintf(tmp, sizeof tmp, "\"n\":%lld,\"nnz\":%lld,\"W\":%lld,\"p\":%lld,\"q\":%lld,\"run_ms\":%.6f,\"dp_mismatch\":%lld,",
+    snprintf(tmp, sizeof tmp, "\"n\":%lld,\"nnz\":%lld,\"W\":%lld,\"p\":%lld,\"q\":%lld,\"run_ms\":%.6f,\"dp_mismatch\":%lld,"
+             "\"kernel_launches\":%lld,",
              (long long)g->n0, (long long)g->nnz0, (long long)g->W, (long long)g->p, (long long)g->q, g->run_ms,
-             (long long)g->dp_mismatch);
+             (long long)g->dp_mismatch, g->launches);
     s += tmp;
     s += "\"levels\":[";
     for (size_t i = 0; i < g->levels.size(); ++i) {
