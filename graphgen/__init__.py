@@ -73,7 +73,8 @@ class CSR:
 
 def build_csr(n: int, src, dst, w=None, keep_self_loops: bool = False, merge_dups: bool = True,
               name: str = "") -> CSR:
-    """Undirected edge list -> symmetric CSR (rows sorted, duplicates merged).
+    """Undirected edge list -> symmetric CSR (rows sorted, duplicates merged: weights summed when
+    `w` is given, dropped (unit weight) when it is not).
 
     A pair (u, v), u != v, yields entries (u, v) and (v, u); a self loop (v, v, w)
     yields one entry (v, v, w) when kept (the library's convention: stored once,
@@ -91,9 +92,11 @@ def build_csr(n: int, src, dst, w=None, keep_self_loops: bool = False, merge_dup
     if nnz < 0:
         raise ValueError("edge endpoint out of range")
     col = col[:nnz].copy()
+    if w is None:
+        # unweighted input: duplicates are dropped (simple graph, unit weights)
+        return CSR(n=n, row_ptr=row_ptr, col=col, w=None, name=name)
     wout = wout[:nnz].copy()
-    unit = bool(nnz == 0 or (w is None and np.all(wout == 1)))
-    return CSR(n=n, row_ptr=row_ptr, col=col, w=None if unit else wout, name=name)
+    return CSR(n=n, row_ptr=row_ptr, col=col, w=wout, name=name)
 
 
 def random_permutation(n: int, seed: int, stream: int = 0) -> np.ndarray:

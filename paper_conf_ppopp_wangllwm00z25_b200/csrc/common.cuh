@@ -43,6 +43,17 @@ struct Carry {
     long long minSig;       // min{Sig[c] : Sig[c] > 0}
     long long sumDC;        // sum_v (d'(v) + s(v))
     int converged;
+    int iter;               // iteration index within the level (also the d' stamp id)
+    int more;               // loop condition written by k_record
+    int log_base;           // log slot of iteration `log_base` is 0
+};
+
+// One record per phase-1 iteration, written on the device by k_record.
+struct IterLog {
+    IterCounters ctr;
+    long long N_hi;
+    ull N_lo;
+    int converged;
     int pad;
 };
 

@@ -86,6 +86,7 @@ struct LevelStat {
 struct gala_graph_s {
     int device = 0;
     cudaStream_t stream = nullptr;
+    cudaMemPool_t pool = nullptr;
     bool own_stream = false;
     int num_sms = 148;
     // level-0 graph
@@ -95,7 +96,7 @@ struct gala_graph_s {
     int64_t* s0 = nullptr;
     // options
     int opt_prune = 1, opt_trace = 0, opt_check = 0, opt_timing = 0, opt_max_iters = 0;
-    int opt_delta = 2, opt_force_i128 = 0, opt_cuda_graph = 0;
+    int opt_delta = 2, opt_force_i128 = 0, opt_cuda_graph = 1, opt_log_cap = 4096;
     int bins[NBINS - 1] = {4, 8, 16, 32, 128};
     int hub_smem_slots = 4096;
     // results
@@ -112,16 +113,27 @@ struct gala_graph_s {
     double run_ms = 0;
     int64_t dp_mismatch = 0;
     long long launches = 0;   // kernels launched by the last gala_run
+    int check_mismatch = 0;   // check mode: final N on G0 differs from the last level's N
     // dist
     DistCtx* dist = nullptr;
 };
 
 // ------------------------------------------------------------------ memory
+// All device memory of a handle comes from its own stream-ordered pool whose
+// release threshold is "keep everything": repeated runs reuse the pages
+// instead of re-mapping them (set per API call by PoolScope).
+static thread_local cudaMemPool_t g_pool = nullptr;
+struct PoolScope {
+    cudaMemPool_t prev;
+    explicit PoolScope(cudaMemPool_t p) : prev(g_pool) { g_pool = p; }
+    ~PoolScope() { g_pool = prev; }
+};
 template <typename T>
 static T* dalloc(size_t count, cudaStream_t st) {
     void* p = nullptr;
     if (count == 0) count = 1;
-    CK(cudaMallocAsync(&p, count * sizeof(T), st));
+    if (g_pool) CK(cudaMallocFromPoolAsync(&p, count * sizeof(T), g_pool, st));
+    else CK(cudaMallocAsync(&p, count * sizeof(T), st));
     return static_cast<T*>(p);
 }
 template <typename T>
@@ -209,76 +221,82 @@ static void gamma_to_pq(double gamma, int64_t* p, int64_t* q) {
 struct Work {
     cudaStream_t st;
     int64_t ncap, nnzcap;
-    int32_t *C = nullptr, *size = nullptr, *stamp = nullptr, *mv_v = nullptr, *mv_c = nullptr, *mv_old = nullptr;
+    int32_t *C = nullptr, *size = nullptr, *stamp = nullptr, *mv_v = nullptr, *mv_old = nullptr, *nextC = nullptr;
     int32_t* queues = nullptr;
     int64_t *Sig = nullptr, *d = nullptr, *s = nullptr, *dp = nullptr;
     IterCounters* ctr = nullptr;
     Carry* carry = nullptr;
+    IterLog* log = nullptr;
+    int log_cap = 4096;
     long long *part_dc = nullptr, *part_min = nullptr;
     i128* part_s2 = nullptr;
     int* gkeys = nullptr;
     ull* gvals = nullptr;
     long long gcap = 0;
     int gblocks = 0;
-    IterCounters* h_ctr = nullptr;
+    IterLog* h_log = nullptr;
     Carry* h_carry = nullptr;
     int reduce_grid = 0;
     void release() {
-        dfree(C, st); dfree(size, st); dfree(stamp, st); dfree(mv_v, st); dfree(mv_c, st); dfree(mv_old, st);
+        dfree(C, st); dfree(size, st); dfree(stamp, st); dfree(mv_v, st); dfree(mv_old, st); dfree(nextC, st);
         dfree(queues, st); dfree(Sig, st); dfree(d, st); dfree(s, st); dfree(dp, st); dfree(ctr, st);
-        dfree(carry, st); dfree(part_dc, st); dfree(part_min, st); dfree(part_s2, st); dfree(gkeys, st);
-        dfree(gvals, st);
-        if (h_ctr) cudaFreeHost(h_ctr);
+        dfree(carry, st); dfree(log, st); dfree(part_dc, st); dfree(part_min, st); dfree(part_s2, st);
+        dfree(gkeys, st); dfree(gvals, st);
+        if (h_log) cudaFreeHost(h_log);
         if (h_carry) cudaFreeHost(h_carry);
-        h_ctr = nullptr;
+        h_log = nullptr;
         h_carry = nullptr;
     }
 };
+
+#define BLOCK_BT 256
+#define BLOCK_E 4
 
 // ------------------------------------------------------------------ launch helpers
 template <typename ST, bool UNIT>
 static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, ST qW, ST p, Timer& tm, int64_t maxdeg) {
     DecideArgs a;
     a.rp = G.rp; a.col = G.col; a.w = G.w; a.C = wk.C; a.Sig = wk.Sig; a.size = wk.size; a.d = wk.d;
-    a.dp = wk.dp; a.mv_v = wk.mv_v; a.mv_c = wk.mv_c; a.ctr = wk.ctr; a.check = g->opt_check;
+    a.dp = wk.dp; a.nextC = wk.nextC; a.ctr = wk.ctr; a.check = g->opt_check;
     const long long qs = wk.ncap;
-    const int sub_grid = g->num_sms * 8;
+    const int grid = g->num_sms * 8;
     cudaStream_t st = g->stream;
     cudaEvent_t e;
     e = tm.begin();
-    k_decide_sub<4, ST, UNIT><<<sub_grid, 256, 0, st>>>(wk.queues + BIN_S4 * qs, BIN_S4, a, qW, p);
+    k_decide_sub<4, 4, ST, UNIT><<<grid, 256, 0, st>>>(wk.queues + BIN_S4 * qs, BIN_S4, a, qW, p);
     CKL();
     tm.end(KC_DEC_S4, e);
     e = tm.begin();
-    k_decide_sub<8, ST, UNIT><<<sub_grid, 256, 0, st>>>(wk.queues + BIN_S8 * qs, BIN_S8, a, qW, p);
+    k_decide_sub<8, 4, ST, UNIT><<<grid, 256, 0, st>>>(wk.queues + BIN_S8 * qs, BIN_S8, a, qW, p);
     CKL();
     tm.end(KC_DEC_S8, e);
     e = tm.begin();
-    k_decide_sub<16, ST, UNIT><<<sub_grid, 256, 0, st>>>(wk.queues + BIN_S16 * qs, BIN_S16, a, qW, p);
+    k_decide_sub<16, 2, ST, UNIT><<<grid, 256, 0, st>>>(wk.queues + BIN_S16 * qs, BIN_S16, a, qW, p);
     CKL();
     tm.end(KC_DEC_S16, e);
     e = tm.begin();
-    k_decide_sub<32, ST, UNIT><<<sub_grid, 256, 0, st>>>(wk.queues + BIN_S32 * qs, BIN_S32, a, qW, p);
+    k_decide_sub<32, 2, ST, UNIT><<<grid, 256, 0, st>>>(wk.queues + BIN_S32 * qs, BIN_S32, a, qW, p);
     CKL();
     tm.end(KC_DEC_S32, e);
     e = tm.begin();
-    k_decide_warp<256, ST, UNIT><<<sub_grid, 256, 0, st>>>(wk.queues + BIN_WARP * qs, BIN_WARP, a, qW, p);
+    k_decide_warp<4, ST, UNIT><<<grid, 256, 0, st>>>(wk.queues + BIN_WARP * qs, BIN_WARP, a, qW, p);
     CKL();
     tm.end(KC_DEC_WARP, e);
     if (maxdeg > g->bins[BIN_WARP]) {
         const int smem_cap = g->hub_smem_slots;
         size_t smem = (size_t)smem_cap * (sizeof(ull) + sizeof(int));
         e = tm.begin();
-        k_decide_block<512, ST, UNIT><<<wk.gblocks, 512, smem, st>>>(wk.queues + BIN_BLOCK * qs, BIN_BLOCK, a, qW,
-                                                                      p, smem_cap, wk.gkeys, wk.gvals, wk.gcap);
+        k_decide_block<BLOCK_BT, BLOCK_E, ST, UNIT><<<wk.gblocks, BLOCK_BT, smem, st>>>(
+            wk.queues + BIN_BLOCK * qs, BIN_BLOCK, a, qW, p, smem_cap, wk.gkeys, wk.gvals, wk.gcap);
         CKL();
         tm.end(KC_DEC_BLOCK, e);
     }
 }
 
+// one phase-1 iteration (Alg. 1 lines 3-13) + its device log record
 template <typename ST, bool UNIT>
-static void run_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, ST qW, ST p, i128 qW128, i128 T,
-                          int iter_id, Timer& tm, int64_t maxdeg) {
+static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, ST qW, ST p, i128 qW128, i128 T,
+                            Timer& tm, int64_t maxdeg, unsigned long long cond) {
     cudaStream_t st = g->stream;
     const int n = (int)G.n;
     const int big = g->num_sms * 8;
@@ -287,18 +305,19 @@ static void run_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, ST qW, ST 
     CKL();
     BinThresholds th;
     for (int i = 0; i < NBINS - 1; ++i) th.t[i] = g->bins[i];
-    k_prune_bin<ST><<<grid_for(n, 256, big), 256, 0, st>>>(n, G.rp, wk.d, wk.dp, wk.C, wk.Sig, g->opt_prune, qW, p,
-                                                           wk.carry, wk.ctr, wk.queues, wk.ncap, th);
+    k_prune_bin<ST><<<grid_for((n + PB_IPT - 1) / PB_IPT, PB_BT, big), PB_BT, 0, st>>>(
+        n, G.rp, wk.d, wk.dp, wk.C, wk.Sig, g->opt_prune, qW, p, wk.carry, wk.ctr, wk.queues, wk.ncap, th);
     CKL();
     tm.end(KC_PRUNE, e);
     launch_decide<ST, UNIT>(g, wk, G, qW, p, tm, maxdeg);
     e = tm.begin();
-    k_apply<<<big, 256, 0, st>>>(wk.ctr, wk.mv_v, wk.mv_c, wk.mv_old, wk.C, wk.Sig, wk.size, wk.d, wk.stamp, iter_id);
+    k_apply<<<grid_for(n, AP_BT, big), AP_BT, 0, st>>>(wk.ctr, wk.queues, wk.ncap, wk.nextC, wk.C, wk.Sig, wk.size,
+                                                       wk.d, G.rp, wk.stamp, wk.carry, wk.mv_v, wk.mv_old);
     CKL();
     tm.end(KC_APPLY, e);
     e = tm.begin();
     k_dp_delta<UNIT><<<big, 256, 0, st>>>(wk.ctr, G.rp, G.col, G.w, wk.C, wk.mv_v, wk.mv_old, wk.stamp, wk.dp,
-                                          iter_id, G.nnz, g->opt_delta, 1, 2);
+                                          wk.carry, G.nnz, g->opt_delta, 1, 2);
     CKL();
     k_dp_full<UNIT><<<big, 256, 0, st>>>(wk.ctr, n, G.rp, G.col, G.w, wk.C, wk.dp, G.nnz, g->opt_delta, 1, 2, 0);
     CKL();
@@ -308,11 +327,98 @@ static void run_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, ST qW, ST 
                                                   wk.carry, (long long)(qW128 >> 64), (ull)qW128, (long long)p,
                                                   (long long)(T >> 64), (ull)T, 1);
     CKL();
+    k_record<<<1, 32, 0, st>>>(wk.ctr, wk.carry, wk.log, wk.log_cap, g->opt_max_iters, cond);
+    CKL();
     tm.end(KC_REDUCE, e);
+}
+
+// Phase 1 of one level to convergence.  Graph mode: the iteration body is
+// captured once into the body of a conditional WHILE node whose condition
+// k_record sets on the device (no host round trip per iteration).  Stepwise
+// mode (trace labels, per-kernel timing, or cuda_graph=0): one host loop trip
+// per iteration.  Both issue the identical kernels.
+template <typename ST, bool UNIT>
+static void phase1_level(gala_graph_s* g, Work& wk, const DevCSR& G, ST qW, ST p, i128 qW128, i128 T, Timer& tm,
+                         int64_t maxdeg, std::vector<IterLog>& out, int level) {
+    cudaStream_t st = g->stream;
+    const bool stepwise = !g->opt_cuda_graph || g->opt_trace >= 2 || g->opt_timing;
+    out.clear();
+    if (stepwise) {
+        for (;;) {
+            issue_iteration<ST, UNIT>(g, wk, G, qW, p, qW128, T, tm, maxdeg, 0ull);
+            CK(cudaMemcpyAsync(wk.h_carry, wk.carry, sizeof(Carry), cudaMemcpyDeviceToHost, st));
+            const int slot = (int)out.size() % wk.log_cap;   // log_base is advanced below
+            CK(cudaMemcpyAsync(wk.h_log, wk.log + slot, sizeof(IterLog), cudaMemcpyDeviceToHost, st));
+            if (g->opt_trace >= 2) {
+                g->trace_labels.emplace_back(G.n);
+                CK(cudaMemcpyAsync(g->trace_labels.back().data(), wk.C, sizeof(int32_t) * G.n, cudaMemcpyDeviceToHost, st));
+            }
+            CK(cudaStreamSynchronize(st));
+            tm.resolve();
+            out.push_back(*wk.h_log);
+            const Carry& c = *wk.h_carry;
+            const bool cap_hit = g->opt_max_iters > 0 && c.iter >= g->opt_max_iters;
+            if (c.converged || cap_hit) break;
+            if (!c.more) {   // log full: restart slots at the current iteration
+                int base = c.iter;
+                CK(cudaMemcpyAsync(&wk.carry->log_base, &base, sizeof(int), cudaMemcpyHostToDevice, st));
+            }
+        }
+        return;
+    }
+    cudaGraph_t graph = nullptr;
+    cudaGraphExec_t exec = nullptr;
+    CK(cudaGraphCreate(&graph, 0));
+    try {
+        cudaGraphConditionalHandle handle;
+        CK(cudaGraphConditionalHandleCreate(&handle, graph, 1, cudaGraphCondAssignDefault));
+        cudaGraphNodeParams cp = {};
+        cp.type = cudaGraphNodeTypeConditional;
+        cp.conditional.handle = handle;
+        cp.conditional.type = cudaGraphCondTypeWhile;
+        cp.conditional.size = 1;
+        cudaGraphNode_t node;
+        CK(cudaGraphAddNode(&node, graph, nullptr, 0, &cp));
+        cudaGraph_t body = cp.conditional.phGraph_out[0];
+        CK(cudaStreamBeginCaptureToGraph(st, body, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed));
+        try {
+            issue_iteration<ST, UNIT>(g, wk, G, qW, p, qW128, T, tm, maxdeg, (unsigned long long)handle);
+        } catch (...) {
+            cudaGraph_t dummy;
+            cudaStreamEndCapture(st, &dummy);
+            throw;
+        }
+        CK(cudaStreamEndCapture(st, &body));
+        CK(cudaGraphInstantiate(&exec, graph, 0));
+        for (;;) {
+            CK(cudaGraphLaunch(exec, st));
+            CK(cudaMemcpyAsync(wk.h_carry, wk.carry, sizeof(Carry), cudaMemcpyDeviceToHost, st));
+            CK(cudaStreamSynchronize(st));
+            const Carry c = *wk.h_carry;
+            const int nrec = c.iter - c.log_base;
+            CK(cudaMemcpyAsync(wk.h_log, wk.log, sizeof(IterLog) * nrec, cudaMemcpyDeviceToHost, st));
+            CK(cudaStreamSynchronize(st));
+            for (int i = 0; i < nrec; ++i) out.push_back(wk.h_log[i]);
+            const bool cap_hit = g->opt_max_iters > 0 && c.iter >= g->opt_max_iters;
+            if (c.converged || cap_hit) break;
+            int base = c.iter;   // log full: continue with fresh slots
+            CK(cudaMemcpyAsync(&wk.carry->log_base, &base, sizeof(int), cudaMemcpyHostToDevice, st));
+        }
+    } catch (...) {
+        if (exec) cudaGraphExecDestroy(exec);
+        cudaGraphDestroy(graph);
+        throw;
+    }
+    cudaGraphExecDestroy(exec);
+    cudaGraphDestroy(graph);
+    (void)level;
 }
 
 static i128 carry_N(const Carry* c) {
     return (i128)(((unsigned __int128)(ull)c->N_hi << 64) | (unsigned __int128)c->N_lo);
+}
+static i128 log_N(const IterLog& l) {
+    return (i128)(((unsigned __int128)(ull)l.N_hi << 64) | (unsigned __int128)l.N_lo);
 }
 
 // algorithmic bytes per kernel class of one iteration
@@ -321,22 +427,129 @@ static void account_bytes(gala_graph_s* g, const IterCounters& c, int64_t n, int
     double act = 0;
     for (int b = 0; b < NBINS; ++b) {
         double cnt = (double)c.bin_count[b], deg = (double)c.bin_deg[b], kk = (double)c.bin_k[b];
-        g->kc_bytes[KC_DEC_S4 + b] += cnt * (4 + 16 + 4 + 8 + 8) + deg * (4 + om + 4) + 8 * kk;
+        // per vertex: queue 4, row_ptr pair 16, C[v] 4, d 8, Sig[C[v]] 8, nextC 4; per entry: col 4 (+w), C[u] 4;
+        // per distinct neighbour community: Sig 8
+        g->kc_bytes[KC_DEC_S4 + b] += cnt * (4 + 16 + 4 + 8 + 8 + 4) + deg * (4 + om + 4) + 8 * kk;
         act += cnt;
     }
-    // prune: d, dp, C, Sig[C] per vertex; rp pair + queue write per active
+    // prune: d, dp, C, Sig[C] per vertex; row_ptr pair + queue write per active
     g->kc_bytes[KC_PRUNE] += (double)n * (8 + 8 + 4 + 8) + act * (16 + 4);
     double m = (double)c.n_moved;
-    g->kc_bytes[KC_APPLY] += m * (4 + 4 + 4 + 4 + 4 + 4 + 8 + 16 + 8);
+    // apply: queue + nextC + C per active; per mover C, stamp, d, 2 Sig, 2 size, row_ptr pair, list 8
+    g->kc_bytes[KC_APPLY] += act * (4 + 4 + 4) + m * (4 + 4 + 8 + 16 + 8 + 16 + 8);
     if (c.delta_used)
-        g->kc_bytes[KC_DP] += m * (16 + 8) + (double)c.moved_deg * (4 + om + 4 + 4);
+        g->kc_bytes[KC_DP] += m * (8 + 16 + 4 + 8) + (double)c.moved_deg * (4 + om + 4 + 4);
     else
         g->kc_bytes[KC_DP] += (double)n * (16 + 4 + 8) + (double)nnz * (4 + om + 4);
     g->kc_bytes[KC_REDUCE] += (double)n * 24;
 }
 
+// ------------------------------------------------------------------ phase 2 (a9)
+// Coarsen level graph `cur` with community ids newid[v] in [0, k) into `nxt`
+// (reading c10: the diagonal carries D_C(c) once).  Per-community hash
+// tables (capacity nextpow2(2 min(entries, k))) are filled by k_coarsen_insert
+// and compacted into CSR rows; coarse d(c) = Sigma_tot(c), s(c) = diagonal.
+static void coarsen(gala_graph_s* g, Work& wk, const DevCSR& cur, int64_t nl, long long k, const int32_t* newid,
+                    const int32_t* minmem, bool unit, DevCSR& nxt, int64_t& maxdeg) {
+    cudaStream_t st = g->stream;
+    const int big = g->num_sms * 8;
+    long long* ent = dalloc<long long>(k + 1, st);
+    long long* hoff = dalloc<long long>(k + 1, st);
+    long long* degn = dalloc<long long>(k + 1, st);
+    CK(cudaMemsetAsync(ent, 0, sizeof(long long) * (k + 1), st));
+    CK(cudaMemsetAsync(degn, 0, sizeof(long long) * (k + 1), st));
+    k_coarsen_count<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, cur.rp, newid, ent);
+    CKL();
+    k_coarsen_cap<<<grid_for(k, 256, big), 256, 0, st>>>(k, ent, hoff);
+    CKL();
+    scan_excl(hoff, hoff, k, st);
+    long long htotal = 0;
+    CK(cudaMemcpyAsync(&htotal, hoff + k, sizeof(long long), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    int* hkeys = dalloc<int>(htotal, st);
+    ull* hvals = dalloc<ull>(htotal, st);
+    CK(cudaMemsetAsync(hkeys, 0xff, sizeof(int) * std::max<long long>(htotal, 1), st));
+    CK(cudaMemsetAsync(hvals, 0, sizeof(ull) * std::max<long long>(htotal, 1), st));
+    if (unit)
+        k_coarsen_insert<true><<<big, 256, 0, st>>>((int)nl, cur.rp, cur.col, cur.w, newid, hoff, hkeys, hvals, degn);
+    else
+        k_coarsen_insert<false><<<big, 256, 0, st>>>((int)nl, cur.rp, cur.col, cur.w, newid, hoff, hkeys, hvals, degn);
+    CKL();
+    nxt.n = k;
+    nxt.rp = dalloc<int64_t>(k + 1, st);
+    scan_excl(degn, reinterpret_cast<long long*>(nxt.rp), k, st);
+    ull* dmax = dalloc<ull>(1, st);
+    CK(cudaMemsetAsync(dmax, 0, sizeof(ull), st));
+    k_rowmax<<<grid_for(k, 256, big), 256, 0, st>>>(k, reinterpret_cast<long long*>(nxt.rp), dmax);
+    CKL();
+    ull mx = 0;
+    CK(cudaMemcpyAsync(&nxt.nnz, nxt.rp + k, sizeof(long long), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(&mx, dmax, sizeof(ull), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    maxdeg = (int64_t)mx;
+    nxt.col = dalloc<int32_t>(nxt.nnz, st);
+    nxt.w = dalloc<int64_t>(nxt.nnz, st);
+    CK(cudaMemsetAsync(ent, 0, sizeof(long long) * (k + 1), st));   // reuse as fill cursor
+    int64_t* snew = dalloc<int64_t>(k, st);
+    int64_t* dnew = dalloc<int64_t>(k, st);
+    CK(cudaMemsetAsync(snew, 0, sizeof(int64_t) * k, st));
+    k_coarsen_extract<<<grid_for(htotal, 256, big * 2), 256, 0, st>>>(k, htotal, hoff, hkeys, hvals,
+                                                                      reinterpret_cast<long long*>(nxt.rp), ent,
+                                                                      nxt.col, nxt.w, snew);
+    CKL();
+    // coarse d = Sigma_tot of the community (exactly maintained by phase 1)
+    k_coarsen_deg<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.C, minmem, newid, wk.Sig, dnew);
+    CKL();
+    CK(cudaMemcpyAsync(wk.d, dnew, sizeof(int64_t) * k, cudaMemcpyDeviceToDevice, st));
+    CK(cudaMemcpyAsync(wk.s, snew, sizeof(int64_t) * k, cudaMemcpyDeviceToDevice, st));
+    dfree(snew, st);
+    dfree(dnew, st);
+    dfree(dmax, st);
+    dfree(ent, st);
+    dfree(hoff, st);
+    dfree(degn, st);
+    dfree(hkeys, st);
+    dfree(hvals, st);
+}
+
+// Final numerator.  The last level's N equals N of the composed labels on the
+// level-0 graph (coarsening preserves Q exactly, invariant P4); with option
+// "check" it is recomputed on G0 from the labels (Eq. 1) and compared.
+static void final_numerator(gala_graph_s* g, int64_t p, int64_t q, int64_t W, i128 N_last) {
+    g->N = N_last;
+    g->check_mismatch = 0;
+    if (!g->opt_check) return;
+    cudaStream_t st = g->stream;
+    const int64_t n0 = g->n0;
+    const int big = g->num_sms * 8;
+    long long* DV = dalloc<long long>(n0, st);
+    ull* DC = dalloc<ull>(1, st);
+    i128* part = dalloc<i128>(big, st);
+    ull* ticket = dalloc<ull>(1, st);
+    i128* out = dalloc<i128>(1, st);
+    CK(cudaMemsetAsync(DV, 0, sizeof(long long) * n0, st));
+    CK(cudaMemsetAsync(DC, 0, sizeof(ull), st));
+    CK(cudaMemsetAsync(ticket, 0, sizeof(ull), st));
+    if (g->g0.w == nullptr)
+        k_mod_dc<true><<<big, 256, 0, st>>>((int)n0, g->g0.rp, g->g0.col, g->g0.w, g->lab, g->d0, DV, DC);
+    else
+        k_mod_dc<false><<<big, 256, 0, st>>>((int)n0, g->g0.rp, g->g0.col, g->g0.w, g->lab, g->d0, DV, DC);
+    CKL();
+    k_sumsq<<<grid_for(n0, 256, big), 256, 0, st>>>(n0, DV, part, ticket, out);
+    CKL();
+    ull hdc = 0;
+    i128 hs2 = 0;
+    CK(cudaMemcpyAsync(&hdc, DC, sizeof(ull), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(&hs2, out, sizeof(i128), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    const i128 N0 = (i128)q * W * (i128)(long long)hdc - (i128)p * hs2;
+    if (N0 != N_last) g->check_mismatch = 1;
+    dfree(DV, st); dfree(DC, st); dfree(part, st); dfree(ticket, st); dfree(out, st);
+}
+
 // ------------------------------------------------------------------ the multi-level run
 static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
+    PoolScope pool_scope(g->pool);
     cudaStream_t st = g->stream;
     CK(cudaSetDevice(g->device));
     g->has_result = false;
@@ -370,13 +583,14 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
     wk.st = st;
     wk.ncap = std::max<int64_t>(n0, 1);
     wk.nnzcap = g->nnz0;
+    wk.log_cap = g->opt_log_cap;
     try {
         wk.C = dalloc<int32_t>(wk.ncap, st);
         wk.size = dalloc<int32_t>(wk.ncap, st);
         wk.stamp = dalloc<int32_t>(wk.ncap, st);
         wk.mv_v = dalloc<int32_t>(wk.ncap, st);
-        wk.mv_c = dalloc<int32_t>(wk.ncap, st);
         wk.mv_old = dalloc<int32_t>(wk.ncap, st);
+        wk.nextC = dalloc<int32_t>(wk.ncap, st);
         wk.queues = dalloc<int32_t>((size_t)wk.ncap * NBINS, st);
         wk.Sig = dalloc<int64_t>(wk.ncap, st);
         wk.d = dalloc<int64_t>(wk.ncap, st);
@@ -384,27 +598,27 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
         wk.dp = dalloc<int64_t>(wk.ncap, st);
         wk.ctr = dalloc<IterCounters>(1, st);
         wk.carry = dalloc<Carry>(1, st);
-        wk.reduce_grid = g->num_sms * 2;
+        wk.log = dalloc<IterLog>(wk.log_cap, st);
+        wk.reduce_grid = g->num_sms * 4;
         wk.part_dc = dalloc<long long>(wk.reduce_grid, st);
         wk.part_min = dalloc<long long>(wk.reduce_grid, st);
         wk.part_s2 = dalloc<i128>(wk.reduce_grid, st);
-        CK(cudaMallocHost(&wk.h_ctr, sizeof(IterCounters)));
+        CK(cudaMallocHost(&wk.h_log, sizeof(IterLog) * wk.log_cap));
         CK(cudaMallocHost(&wk.h_carry, sizeof(Carry)));
         CK(cudaMemsetAsync(wk.ctr, 0, sizeof(IterCounters), st));
         CK(cudaMemsetAsync(wk.carry, 0, sizeof(Carry), st));
-        // block-kernel spill tables: one per resident block, capacity >= 2*maxdeg0
+        // block-kernel spill tables: one per resident block
         {
             int per_sm = 0;
             size_t smem = (size_t)g->hub_smem_slots * (sizeof(ull) + sizeof(int));
-            CK(cudaFuncSetAttribute(k_decide_block<512, long long, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-            CK(cudaFuncSetAttribute(k_decide_block<512, long long, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-            CK(cudaFuncSetAttribute(k_decide_block<512, i128, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-            CK(cudaFuncSetAttribute(k_decide_block<512, i128, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-            CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_decide_block<512, i128, false>, 512, smem));
+            CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, long long, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, long long, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, i128, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, i128, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_decide_block<BLOCK_BT, BLOCK_E, i128, false>, BLOCK_BT, smem));
             wk.gblocks = g->num_sms * std::max(per_sm, 1);
         }
-        // wk.gcap is sized per level (coarse levels can have larger rows than level 0)
-        wk.gcap = 0;
+        wk.gcap = 0;   // sized per level (coarse levels can have larger rows than level 0)
 
         DevCSR cur = g->g0;
         bool cur_owned = false;
@@ -413,6 +627,7 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
         int64_t maxdeg = g->maxdeg0;
         bool first_level = true;
         Timer tm(g);
+        std::vector<IterLog> logs;
         for (int level = 0;; ++level) {
             const int64_t nl = cur.n;
             const bool unit = (cur.w == nullptr);
@@ -439,7 +654,8 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
             }
             // a1: level init + starting numerator
             cudaEvent_t e = tm.begin();
-            k_level_init<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.d, wk.C, wk.Sig, wk.size, wk.dp, wk.stamp);
+            k_level_init<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.d, wk.C, wk.Sig, wk.size, wk.dp, wk.stamp,
+                                                                 wk.carry);
             CKL();
             if (first_level) {
                 // lab = identity on level 0 (C is the identity right now)
@@ -456,53 +672,40 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
             CK(cudaMemcpyAsync(wk.h_carry, wk.carry, sizeof(Carry), cudaMemcpyDeviceToHost, st));
             CK(cudaStreamSynchronize(st));
             const i128 N_start = carry_N(wk.h_carry);
-            // score type for this level: int64 iff max(p,q) * W * maxdeg_weighted < 2^62
-            // (weighted degree <= W; use W as the bound on coarse levels, maxdeg on unit level 0)
+            // score type for this level: int64 iff max(p,q) * W * max weighted degree < 2^62
+            // (level 0 unit weights: weighted degree = row length; coarse levels: bounded by W)
             long double bound = (long double)mpq * (long double)W *
                                 (long double)(unit ? std::max<int64_t>(maxdeg, 1) : W);
             const bool use128 = g->opt_force_i128 || bound >= 0x1p62L;
             ls.i128path = use128;
+            if (use128) {
+                if (unit) phase1_level<i128, true>(g, wk, cur, (i128)qW128, (i128)p, qW128, T, tm, maxdeg, logs, level);
+                else phase1_level<i128, false>(g, wk, cur, (i128)qW128, (i128)p, qW128, T, tm, maxdeg, logs, level);
+            } else {
+                long long qW = (long long)qW128, pp = (long long)p;
+                if (unit) phase1_level<long long, true>(g, wk, cur, qW, pp, qW128, T, tm, maxdeg, logs, level);
+                else phase1_level<long long, false>(g, wk, cur, qW, pp, qW128, T, tm, maxdeg, logs, level);
+            }
             i128 N = N_start;
-            int64_t iters = 0;
-            for (int it = 0;; ++it) {
-                const int iter_id = level * 1000000 + it;
-                if (use128) {
-                    if (unit) run_iteration<i128, true>(g, wk, cur, (i128)qW128, (i128)p, qW128, T, iter_id, tm, maxdeg);
-                    else run_iteration<i128, false>(g, wk, cur, (i128)qW128, (i128)p, qW128, T, iter_id, tm, maxdeg);
-                } else {
-                    long long qW = (long long)qW128, pp = (long long)p;
-                    if (unit) run_iteration<long long, true>(g, wk, cur, qW, pp, qW128, T, iter_id, tm, maxdeg);
-                    else run_iteration<long long, false>(g, wk, cur, qW, pp, qW128, T, iter_id, tm, maxdeg);
-                }
-                CK(cudaMemcpyAsync(wk.h_ctr, wk.ctr, sizeof(IterCounters), cudaMemcpyDeviceToHost, st));
-                CK(cudaMemcpyAsync(wk.h_carry, wk.carry, sizeof(Carry), cudaMemcpyDeviceToHost, st));
-                if (g->opt_trace >= 2) {
-                    g->trace_labels.emplace_back(nl);
-                    CK(cudaMemcpyAsync(g->trace_labels.back().data(), wk.C, sizeof(int32_t) * nl,
-                                       cudaMemcpyDeviceToHost, st));
-                }
-                CK(cudaStreamSynchronize(st));
-                tm.resolve();
-                const IterCounters& c = *wk.h_ctr;
+            for (size_t it = 0; it < logs.size(); ++it) {
+                const IterCounters& c = logs[it].ctr;
                 account_bytes(g, c, nl, cur.nnz, unit);
                 g->dp_mismatch += (int64_t)c.dp_mismatch;
-                N = carry_N(wk.h_carry);
-                ++iters;
+                N = log_N(logs[it]);
                 int64_t scanned = 0, kk = 0;
                 for (int b = 0; b < NBINS; ++b) { scanned += (int64_t)c.bin_deg[b]; kk += (int64_t)c.bin_k[b]; }
                 ls.edges_scanned += scanned;
                 ls.nominal_edges += cur.nnz;
                 if (g->opt_trace >= 1) {
                     TraceRec r;
-                    r.v[0] = level; r.v[1] = it; r.v[2] = nl; r.v[3] = (int64_t)c.n_active;
+                    r.v[0] = level; r.v[1] = (int64_t)it; r.v[2] = nl; r.v[3] = (int64_t)c.n_active;
                     r.v[4] = (int64_t)c.n_pruned; r.v[5] = (int64_t)c.n_moved;
                     r.v[6] = (int64_t)(N >> 64); r.v[7] = (int64_t)(uint64_t)N;
                     r.v[8] = scanned; r.v[9] = kk; r.v[10] = (int64_t)c.delta_used; r.v[11] = 0;
                     g->trace.push_back(r);
                 }
-                if (wk.h_carry->converged || (g->opt_max_iters > 0 && it + 1 >= g->opt_max_iters)) break;
             }
-            ls.iters = iters;
+            ls.iters = (int64_t)logs.size();
             CK(cudaEventRecord(lv1, st));
             // a8: relabel in min-member order + compose
             e = tm.begin();
@@ -525,66 +728,7 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
             CK(cudaStreamSynchronize(st));
             const bool stop = (kcomm == nl) || (max_levels > 0 && level + 1 >= max_levels) || (N - N_start < T);
             DevCSR nxt;
-            if (!stop) {
-                // a9: coarsen
-                const long long k = kcomm;
-                long long* ent = dalloc<long long>(k + 1, st);
-                long long* hoff = dalloc<long long>(k + 1, st);
-                long long* degn = dalloc<long long>(k + 1, st);
-                CK(cudaMemsetAsync(ent, 0, sizeof(long long) * (k + 1), st));
-                CK(cudaMemsetAsync(degn, 0, sizeof(long long) * (k + 1), st));
-                k_coarsen_count<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, cur.rp, newid, ent);
-                CKL();
-                k_coarsen_cap<<<grid_for(k, 256, big), 256, 0, st>>>(k, ent, hoff);
-                CKL();
-                scan_excl(hoff, hoff, k, st);
-                long long htotal = 0;
-                CK(cudaMemcpyAsync(&htotal, hoff + k, sizeof(long long), cudaMemcpyDeviceToHost, st));
-                CK(cudaStreamSynchronize(st));
-                int* hkeys = dalloc<int>(htotal, st);
-                ull* hvals = dalloc<ull>(htotal, st);
-                CK(cudaMemsetAsync(hkeys, 0xff, sizeof(int) * std::max<long long>(htotal, 1), st));
-                CK(cudaMemsetAsync(hvals, 0, sizeof(ull) * std::max<long long>(htotal, 1), st));
-                if (unit)
-                    k_coarsen_insert<true><<<big, 256, 0, st>>>((int)nl, cur.rp, cur.col, cur.w, newid, hoff, hkeys,
-                                                                hvals, degn);
-                else
-                    k_coarsen_insert<false><<<big, 256, 0, st>>>((int)nl, cur.rp, cur.col, cur.w, newid, hoff, hkeys,
-                                                                 hvals, degn);
-                CKL();
-                nxt.n = k;
-                nxt.rp = dalloc<int64_t>(k + 1, st);
-                scan_excl(degn, reinterpret_cast<long long*>(nxt.rp), k, st);
-                CK(cudaMemcpyAsync(&nxt.nnz, nxt.rp + k, sizeof(long long), cudaMemcpyDeviceToHost, st));
-                CK(cudaStreamSynchronize(st));
-                nxt.col = dalloc<int32_t>(nxt.nnz, st);
-                nxt.w = dalloc<int64_t>(nxt.nnz, st);
-                CK(cudaMemsetAsync(ent, 0, sizeof(long long) * (k + 1), st));   // reuse as fill cursor
-                CK(cudaMemsetAsync(wk.s, 0, sizeof(int64_t) * k, st));
-                k_coarsen_extract<true><<<grid_for(htotal, 256, big), 256, 0, st>>>(
-                    k, htotal, hoff, hkeys, hvals, reinterpret_cast<long long*>(nxt.rp), ent, nxt.col, nxt.w, wk.s);
-                CKL();
-                // coarse d = Sigma_tot of the community; write into a temp then copy to wk.d
-                int64_t* dnew = dalloc<int64_t>(k, st);
-                k_coarsen_deg<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.C, minmem, newid, wk.Sig, dnew);
-                CKL();
-                CK(cudaMemcpyAsync(wk.d, dnew, sizeof(int64_t) * k, cudaMemcpyDeviceToDevice, st));
-                ull* dmax = dalloc<ull>(1, st);
-                CK(cudaMemsetAsync(dmax, 0, sizeof(ull), st));
-                k_rowmax<<<grid_for(k, 256, big), 256, 0, st>>>(k, reinterpret_cast<long long*>(nxt.rp), dmax);
-                CKL();
-                ull mx = 0;
-                CK(cudaMemcpyAsync(&mx, dmax, sizeof(ull), cudaMemcpyDeviceToHost, st));
-                CK(cudaStreamSynchronize(st));
-                maxdeg = (int64_t)mx;
-                dfree(dmax, st);
-                dfree(dnew, st);
-                dfree(ent, st);
-                dfree(hoff, st);
-                dfree(degn, st);
-                dfree(hkeys, st);
-                dfree(hvals, st);
-            }
+            if (!stop) coarsen(g, wk, cur, nl, kcomm, newid, minmem, unit, nxt, maxdeg);
             dfree(minmem, st);
             dfree(pos, st);
             dfree(newid, st);
@@ -606,31 +750,12 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
             cur = nxt;
             cur_owned = true;
         }
-        // final N on the level-0 graph from the composed labels (Eq. 1)
         {
-            long long* DV = dalloc<long long>(n0, st);
-            ull* DC = dalloc<ull>(1, st);
-            i128* part = dalloc<i128>(big, st);
-            ull* ticket = dalloc<ull>(1, st);
-            i128* out = dalloc<i128>(1, st);
-            CK(cudaMemsetAsync(DV, 0, sizeof(long long) * n0, st));
-            CK(cudaMemsetAsync(DC, 0, sizeof(ull), st));
-            CK(cudaMemsetAsync(ticket, 0, sizeof(ull), st));
-            if (g->g0.w == nullptr)
-                k_mod_dc<true><<<big, 256, 0, st>>>((int)n0, g->g0.rp, g->g0.col, g->g0.w, g->lab, g->d0, DV, DC);
-            else
-                k_mod_dc<false><<<big, 256, 0, st>>>((int)n0, g->g0.rp, g->g0.col, g->g0.w, g->lab, g->d0, DV, DC);
-            CKL();
-            int sg = grid_for(n0, 256, big);
-            k_sumsq<<<sg, 256, 0, st>>>(n0, DV, part, ticket, out);
-            CKL();
-            ull hdc = 0;
-            i128 hs2 = 0;
-            CK(cudaMemcpyAsync(&hdc, DC, sizeof(ull), cudaMemcpyDeviceToHost, st));
-            CK(cudaMemcpyAsync(&hs2, out, sizeof(i128), cudaMemcpyDeviceToHost, st));
+            i128 N_last = 0;
+            CK(cudaMemcpyAsync(wk.h_carry, wk.carry, sizeof(Carry), cudaMemcpyDeviceToHost, st));
             CK(cudaStreamSynchronize(st));
-            g->N = (i128)q * W * (i128)(long long)hdc - (i128)p * hs2;
-            dfree(DV, st); dfree(DC, st); dfree(part, st); dfree(ticket, st); dfree(out, st);
+            N_last = carry_N(wk.h_carry);
+            final_numerator(g, p, q, W, N_last);
         }
         CK(cudaEventRecord(ev_run1, st));
         CK(cudaEventSynchronize(ev_run1));
@@ -661,10 +786,18 @@ static void init_graph_common(gala_graph_s* g, int64_t n, int device, uintptr_t 
         g->stream = reinterpret_cast<cudaStream_t>(stream);
         g->own_stream = false;
     } else {
-        CK(cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking));
+        CK(cudaStreamCreate(&g->stream));   // blocking: ordered after legacy-default-stream work
         g->own_stream = true;
     }
     g->n0 = n;
+    cudaMemPoolProps props = {};
+    props.allocType = cudaMemAllocationTypePinned;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = device;
+    CK(cudaMemPoolCreate(&g->pool, &props));
+    uint64_t keep = UINT64_MAX;
+    CK(cudaMemPoolSetAttribute(g->pool, cudaMemPoolAttrReleaseThreshold, &keep));
+    g_pool = g->pool;
 }
 
 static void finish_graph(gala_graph_s* g) {
@@ -733,6 +866,7 @@ gala_status gala_graph_from_csr(int64_t n, const int64_t* row_ptr, const int32_t
     gala_status s = validate_host(n, row_ptr, col_idx, weights, &W, &unit);
     if (s != GALA_OK) return s;
     gala_graph_s* g = new gala_graph_s();
+    PoolScope pool_scope(nullptr);
     API_BEGIN
     try {
         init_graph_common(g, n, device, stream);
@@ -765,6 +899,7 @@ gala_status gala_graph_from_csr_device(int64_t n, const int64_t* d_row_ptr, cons
     *out = nullptr;
     if (n < 0 || n >= ((int64_t)1 << 31)) return set_err(GALA_E_INVALID, "n out of range");
     gala_graph_s* g = new gala_graph_s();
+    PoolScope pool_scope(nullptr);
     API_BEGIN
     try {
         init_graph_common(g, n, device, stream);
@@ -930,6 +1065,8 @@ void gala_graph_free(gala_graph g) {
         cudaStreamSynchronize(st);
         if (g->own_stream) cudaStreamDestroy(st);
     }
+    if (g->pool) cudaMemPoolDestroy(g->pool);
+    if (g_pool == g->pool) g_pool = nullptr;
     delete g;
 }
 
@@ -944,6 +1081,7 @@ gala_status gala_set_option(gala_graph g, const char* key, int64_t value) {
     else if (k == "delta_update") { if (value < 0 || value > 2) return set_err(GALA_E_INVALID, "delta_update in 0..2"); g->opt_delta = (int)value; }
     else if (k == "force_i128") g->opt_force_i128 = value != 0;
     else if (k == "cuda_graph") g->opt_cuda_graph = value != 0;
+    else if (k == "log_cap") { if (value < 2 || value > (1 << 20)) return set_err(GALA_E_INVALID, "log_cap in [2, 2^20]"); g->opt_log_cap = (int)value; }
     else if (k == "hub_smem_slots") {
         if (value < 64 || value > 16384 || (value & (value - 1))) return set_err(GALA_E_INVALID, "hub_smem_slots: power of two in [64, 16384]");
         g->hub_smem_slots = (int)value;
@@ -1003,9 +1141,9 @@ gala_status gala_get_stats(gala_graph g, char* buf, int64_t cap, int64_t* needed
     std::string s = "{";
     char tmp[512];
     snprintf(tmp, sizeof tmp, "\"n\":%lld,\"nnz\":%lld,\"W\":%lld,\"p\":%lld,\"q\":%lld,\"run_ms\":%.6f,\"dp_mismatch\":%lld,"
-             "\"kernel_launches\":%lld,",
+             "\"kernel_launches\":%lld,\"check_mismatch\":%d,",
              (long long)g->n0, (long long)g->nnz0, (long long)g->W, (long long)g->p, (long long)g->q, g->run_ms,
-             (long long)g->dp_mismatch, g->launches);
+             (long long)g->dp_mismatch, g->launches, g->check_mismatch);
     s += tmp;
     s += "\"levels\":[";
     for (size_t i = 0; i < g->levels.size(); ++i) {

@@ -1,9 +1,32 @@
 // k_phase1.cuh — phase-1 kernels (Alg. 1): level init, MG pruning
 // frontier + degree binning, DecideAndMove (sub-warp shuffle, warp hash,
-// block hierarchical hash), apply moves, d' update, Q/convergence reduction.
-// SURVEY.md §8(a) rows a1-a7; DESIGN.md "Kernels".
+// block hierarchical hash), apply moves, d' update, Q/convergence reduction,
+// per-iteration device log.  SURVEY.md §8(a) rows a1-a7; DESIGN.md "Kernels".
+//
+// Throughput notes: the decide kernels are bound by
+// dependent random gathers (queue -> row_ptr -> col -> C[u] -> Sigma_tot[c]).
+// Each warp therefore works on several independent vertices at once (U-way
+// interleave in the sub-warp kernel, E-way batched row loads elsewhere), and
+// every queue append / counter update is aggregated per block so that no
+// global address sees more than one atomic per block and tile.
 #pragma once
 #include "common.cuh"
+
+// ---------------------------------------------------------------------------
+// block-level helpers
+// ---------------------------------------------------------------------------
+template <int BT>
+__device__ __forceinline__ ull block_sum_ull(ull x) {   // result valid in thread 0
+    __shared__ ull sh[BT / 32];
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(FULLMASK, x, o);
+    __syncthreads();
+    if (lane_id() == 0) sh[threadIdx.x >> 5] = x;
+    __syncthreads();
+    if (threadIdx.x == 0)
+        for (int i = 1; i < BT / 32; ++i) x += sh[i];
+    return x;
+}
 
 // ---------------------------------------------------------------------------
 // a1: weighted degree d(v) and self-loop weight s(v) of every vertex (warp per row)
@@ -38,7 +61,7 @@ __global__ void k_degrees(int n, const int64_t* __restrict__ rp, const int32_t* 
 // a1: every vertex its own community
 __global__ void k_level_init(int n, const int64_t* __restrict__ d, int32_t* __restrict__ C,
                              int64_t* __restrict__ Sig, int32_t* __restrict__ size, int64_t* __restrict__ dp,
-                             int32_t* __restrict__ stamp) {
+                             int32_t* __restrict__ stamp, Carry* __restrict__ carry) {
     for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n;
          v += (long long)gridDim.x * blockDim.x) {
         C[v] = (int32_t)v;
@@ -47,6 +70,7 @@ __global__ void k_level_init(int n, const int64_t* __restrict__ d, int32_t* __re
         dp[v] = 0;
         stamp[v] = -1;
     }
+    if (blockIdx.x == 0 && threadIdx.x == 0) { carry->iter = 0; carry->converged = 0; carry->log_base = 0; }
 }
 
 __global__ void k_iter_begin(IterCounters* ctr) {
@@ -57,77 +81,105 @@ __global__ void k_iter_begin(IterCounters* ctr) {
 // ---------------------------------------------------------------------------
 // a2: MG pruning frontier (Eq. 6/7) fused with degree binning.
 //   inactive iff  qW (2 d'(v) - d(v)) + p (minSig - Sig[C[v]]) d(v) >= 0
-// Active vertices are appended to the queue of their degree bin with
-// warp-aggregated atomics.  Bin choice never changes results (P7).
+// Tiles of PB_BT*PB_IPT vertices; per-bin offsets are aggregated in shared
+// memory, one global atomic per bin per tile.  Bin choice never changes
+// results (P7).
 // ---------------------------------------------------------------------------
 struct BinThresholds {
     int t[NBINS - 1];   // upper row-length bound of bins 0..4; bin 5 = rest
 };
+#define PB_BT 256
+#define PB_IPT 4
 
 template <typename ST>
-__global__ void __launch_bounds__(256) k_prune_bin(int n, const int64_t* __restrict__ rp,
-                                                   const int64_t* __restrict__ d, const int64_t* __restrict__ dp,
-                                                   const int32_t* __restrict__ C, const int64_t* __restrict__ Sig,
-                                                   int prune, ST qW, ST p, const Carry* __restrict__ carry,
-                                                   IterCounters* __restrict__ ctr, int32_t* __restrict__ queues,
-                                                   long long qstride, BinThresholds th) {
+__global__ void __launch_bounds__(PB_BT) k_prune_bin(int n, const int64_t* __restrict__ rp,
+                                                     const int64_t* __restrict__ d, const int64_t* __restrict__ dp,
+                                                     const int32_t* __restrict__ C, const int64_t* __restrict__ Sig,
+                                                     int prune, ST qW, ST p, const Carry* __restrict__ carry,
+                                                     IterCounters* __restrict__ ctr, int32_t* __restrict__ queues,
+                                                     long long qstride, BinThresholds th) {
+    __shared__ unsigned s_cnt[NBINS];
+    __shared__ ull s_base[NBINS];
     const long long minSig = carry->minSig;
     ull my_active = 0, my_pruned = 0;
-    ull my_deg[NBINS] = {0, 0, 0, 0, 0, 0};
-    const long long stride = (long long)gridDim.x * blockDim.x;
-    for (long long base = (long long)blockIdx.x * blockDim.x; base < n; base += stride) {
-        long long v = base + threadIdx.x;
-        int bin = -1;
-        int deg = 0;
-        if (v < n) {
-            long long dv = d[v];
-            if (dv > 0) {
+    ull my_deg[NBINS];
+#pragma unroll
+    for (int b = 0; b < NBINS; ++b) my_deg[b] = 0;
+    const long long tile = (long long)PB_BT * PB_IPT;
+    for (long long t0 = (long long)blockIdx.x * tile; t0 < n; t0 += (long long)gridDim.x * tile) {
+        if (threadIdx.x < NBINS) s_cnt[threadIdx.x] = 0;
+        int bin[PB_IPT];
+        long long dv[PB_IPT], dpv[PB_IPT];
+        int cv[PB_IPT];
+#pragma unroll
+        for (int j = 0; j < PB_IPT; ++j) {
+            long long v = t0 + (long long)j * PB_BT + threadIdx.x;
+            bool ok = v < n;
+            dv[j] = ok ? d[v] : 0;
+            dpv[j] = ok ? dp[v] : 0;
+            cv[j] = ok ? C[v] : 0;
+        }
+        long long sg[PB_IPT];
+#pragma unroll
+        for (int j = 0; j < PB_IPT; ++j) sg[j] = (prune && dv[j] > 0) ? Sig[cv[j]] : 0;
+        int deg[PB_IPT];
+#pragma unroll
+        for (int j = 0; j < PB_IPT; ++j) {
+            long long v = t0 + (long long)j * PB_BT + threadIdx.x;
+            bin[j] = -1;
+            deg[j] = 0;
+            if (dv[j] > 0) {
                 bool active = true;
                 if (prune) {
-                    long long dpv = dp[v];
-                    long long sg = Sig[C[v]];
-                    ST lhs = qW * (ST)(2 * dpv - dv) + p * (ST)(minSig - sg) * (ST)dv;
+                    ST lhs = qW * (ST)(2 * dpv[j] - dv[j]) + p * (ST)(minSig - sg[j]) * (ST)dv[j];
                     active = lhs < (ST)0;
                 }
                 if (active) {
                     long long dg = rp[v + 1] - rp[v];
-                    deg = (int)(dg > INT_MAX ? INT_MAX : dg);
-                    bin = NBINS - 1;
+                    deg[j] = (int)(dg > INT_MAX ? INT_MAX : dg);
+                    int b = NBINS - 1;
 #pragma unroll
-                    for (int b = NBINS - 2; b >= 0; --b)
-                        if (deg <= th.t[b]) bin = b;
+                    for (int k = NBINS - 2; k >= 0; --k)
+                        if (deg[j] <= th.t[k]) b = k;
+                    bin[j] = b;
                     my_active++;
+                    my_deg[b] += (ull)deg[j];
                 } else {
                     my_pruned++;
                 }
             }
         }
-        // warp-aggregated append per bin
-        unsigned peers = __match_any_sync(FULLMASK, bin);
-        int leader = __ffs(peers) - 1;
-        ull basepos = 0;
-        if (bin >= 0 && lane_id() == leader) basepos = atomicAdd(&ctr->bin_count[bin], (ull)__popc(peers));
-        basepos = __shfl_sync(FULLMASK, basepos, leader);
-        if (bin >= 0) {
-            long long pos = (long long)basepos + __popc(peers & lanemask_lt());
-            queues[(long long)bin * qstride + pos] = (int32_t)v;
+        __syncthreads();   // s_cnt reset visible
+        unsigned off[PB_IPT];
 #pragma unroll
-            for (int b = 0; b < NBINS; ++b)
-                if (b == bin) my_deg[b] += (ull)deg;
+        for (int j = 0; j < PB_IPT; ++j) {
+            unsigned peers = __match_any_sync(FULLMASK, bin[j]);
+            int leader = __ffs(peers) - 1;
+            unsigned base = 0;
+            if (bin[j] >= 0 && lane_id() == leader) base = atomicAdd(&s_cnt[bin[j]], (unsigned)__popc(peers));
+            base = __shfl_sync(FULLMASK, base, leader);
+            off[j] = base + __popc(peers & lanemask_lt());
+        }
+        __syncthreads();
+        if (threadIdx.x < NBINS)
+            s_base[threadIdx.x] = s_cnt[threadIdx.x] ? atomicAdd(&ctr->bin_count[threadIdx.x], (ull)s_cnt[threadIdx.x]) : 0;
+        __syncthreads();
+#pragma unroll
+        for (int j = 0; j < PB_IPT; ++j) {
+            if (bin[j] >= 0) {
+                long long v = t0 + (long long)j * PB_BT + threadIdx.x;
+                queues[(long long)bin[j] * qstride + (long long)s_base[bin[j]] + off[j]] = (int32_t)v;
+            }
         }
     }
-    // counters (one atomic per warp)
-    ull a = __reduce_add_sync(FULLMASK, (unsigned)my_active);
-    ull pr = __reduce_add_sync(FULLMASK, (unsigned)my_pruned);
-    if (lane_id() == 0) {
-        if (a) atomicAdd(&ctr->n_active, a);
-        if (pr) atomicAdd(&ctr->n_pruned, pr);
-    }
+    ull a = block_sum_ull<PB_BT>(my_active);
+    if (threadIdx.x == 0 && a) atomicAdd(&ctr->n_active, a);
+    ull pr = block_sum_ull<PB_BT>(my_pruned);
+    if (threadIdx.x == 0 && pr) atomicAdd(&ctr->n_pruned, pr);
 #pragma unroll
     for (int b = 0; b < NBINS; ++b) {
-        ull x = my_deg[b];
-        for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(FULLMASK, x, o);
-        if (lane_id() == 0 && x) atomicAdd(&ctr->bin_deg[b], x);
+        ull x = block_sum_ull<PB_BT>(my_deg[b]);
+        if (threadIdx.x == 0 && x) atomicAdd(&ctr->bin_deg[b], x);
     }
 }
 
@@ -135,10 +187,9 @@ __global__ void __launch_bounds__(256) k_prune_bin(int n, const int64_t* __restr
 // decision shared by all DecideAndMove kernels
 // ---------------------------------------------------------------------------
 template <typename ST>
-__device__ __forceinline__ int decide_final(int cv, long long dv, long long own, ST best_s, int best_c,
-                                            const int64_t* __restrict__ Sig, const int32_t* __restrict__ size,
-                                            ST qW, ST p) {
-    ST stay = qW * (ST)own - p * (ST)(Sig[cv] - dv) * (ST)dv;
+__device__ __forceinline__ int decide_final(int cv, long long dv, long long own, long long sig_cv, ST best_s,
+                                            int best_c, const int32_t* __restrict__ size, ST qW, ST p) {
+    ST stay = qW * (ST)own - p * (ST)(sig_cv - dv) * (ST)dv;
     int tgt = cv;
     if (best_c != INT_MAX && best_s > stay) {          // strictly better than staying (c4)
         tgt = best_c;
@@ -156,8 +207,7 @@ struct DecideArgs {
     const int32_t* size;
     const int64_t* d;
     const int64_t* dp;
-    int32_t* mv_v;      // moved list: vertex
-    int32_t* mv_c;      // moved list: target community
+    int32_t* nextC;     // decision of every processed vertex (C[v] to stay)
     IterCounters* ctr;
     int check;
 };
@@ -167,9 +217,10 @@ struct DecideArgs {
 // lane, community aggregation with __match_any_sync (Alg. 2).
 // Weighted levels sum the peers' weights with shared-memory atomics onto the
 // group leader; unit-weight levels use popc(peers).  Argmax over the group
-// with an xor-shuffle butterfly on (score, -community).
+// with an xor-shuffle butterfly on (score, -community).  Each group handles U
+// independent vertices per iteration, all their loads issued before use.
 // ---------------------------------------------------------------------------
-template <int G, typename ST, bool UNIT>
+template <int G, int U, typename ST, bool UNIT>
 __global__ void __launch_bounds__(256) k_decide_sub(const int32_t* __restrict__ queue, int bin, DecideArgs a,
                                                     ST qW, ST p) {
     __shared__ ull s_acc[8][32];
@@ -178,70 +229,90 @@ __global__ void __launch_bounds__(256) k_decide_sub(const int32_t* __restrict__ 
     const unsigned gmask = (G == 32) ? FULLMASK : (((1u << G) - 1u) << (gid * G));
     const long long count = (long long)a.ctr->bin_count[bin];
     const long long nwarps = (long long)gridDim.x * (blockDim.x >> 5);
-    const long long per = 32 / G;
-    ull my_k = 0, my_moved_deg = 0;
+    const long long per = (32 / G) * U;
+    ull my_k = 0;
     for (long long base = ((long long)blockIdx.x * (blockDim.x >> 5) + wib) * per; base < count;
          base += nwarps * per) {
-        long long i = base + gid;
-        bool valid = i < count;
-        int v = valid ? queue[i] : 0;
-        int64_t beg = valid ? a.rp[v] : 0;
-        int deg = valid ? (int)(a.rp[v + 1] - beg) : 0;
-        bool has = valid && gl < deg;
-        int u = has ? a.col[beg + gl] : -1;
-        if (u == v) has = false;                          // self loop is not a neighbour
-        long long wt = has ? (UNIT ? 1 : a.w[beg + gl]) : 0;
-        int cu = has ? a.C[u] : (-1 - lane);              // unique sentinel per empty lane
-        unsigned peers = __match_any_sync(FULLMASK, cu) & gmask;
-        int leader = __ffs(peers) - 1;
-        bool isL = has && lane == leader;
-        long long wc;
-        if (UNIT) {
-            wc = __popc(peers);
-        } else {
-            s_acc[wib][lane] = 0;
-            __syncwarp();
-            if (has) atomicAdd(&s_acc[wib][leader], (ull)wt);
-            __syncwarp();
-            wc = (long long)s_acc[wib][lane];
-            __syncwarp();
-        }
-        int cv = valid ? a.C[v] : -2;
-        long long dv = valid ? a.d[v] : 0;
-        ST bs = st_min<ST>();
-        int bc = INT_MAX;
-        long long own = 0;
-        if (isL) {
-            my_k++;
-            if (cu == cv) own = wc;
-            else { bs = qW * (ST)wc - p * (ST)a.Sig[cu] * (ST)dv; bc = cu; }
+        int v[U], deg[U], cv[U], u[U], cu[U];
+        int64_t beg[U];
+        long long dv[U], wt[U];
+        bool valid[U], has[U];
+#pragma unroll
+        for (int k = 0; k < U; ++k) {
+            long long i = base + (long long)k * (32 / G) + gid;
+            valid[k] = i < count;
+            v[k] = valid[k] ? queue[i] : 0;
         }
 #pragma unroll
-        for (int off = G / 2; off > 0; off >>= 1) {
-            ST os = shfl_xor_st(bs, off);
-            int oc = __shfl_xor_sync(FULLMASK, bc, off);
-            own += __shfl_xor_sync(FULLMASK, own, off);
-            if (better(os, oc, bs, bc)) { bs = os; bc = oc; }
+        for (int k = 0; k < U; ++k) {
+            beg[k] = valid[k] ? a.rp[v[k]] : 0;
+            int64_t e = valid[k] ? a.rp[v[k] + 1] : 0;
+            deg[k] = (int)(e - beg[k]);
+            cv[k] = valid[k] ? a.C[v[k]] : -2;
+            dv[k] = valid[k] ? a.d[v[k]] : 0;
         }
-        int tgt = cv;
-        if (valid && gl == 0) {
-            if (a.check && own != a.dp[v]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
-            if (dv > 0) tgt = decide_final<ST>(cv, dv, own, bs, bc, a.Sig, a.size, qW, p);
+#pragma unroll
+        for (int k = 0; k < U; ++k) {
+            has[k] = valid[k] && gl < deg[k];
+            u[k] = has[k] ? a.col[beg[k] + gl] : -1;
+            wt[k] = (has[k] && !UNIT) ? a.w[beg[k] + gl] : 1;
         }
-        bool mover = valid && gl == 0 && tgt != cv;
-        long long pos = warp_append(mover, &a.ctr->n_moved);
-        if (mover) {
-            a.mv_v[pos] = v;
-            a.mv_c[pos] = tgt;
-            my_moved_deg += (ull)deg;
+#pragma unroll
+        for (int k = 0; k < U; ++k) {
+            if (u[k] == v[k]) has[k] = false;                 // self loop is not a neighbour
+            cu[k] = has[k] ? a.C[u[k]] : (-1 - lane);         // unique sentinel per empty lane
         }
+        unsigned peers[U];
+        bool isL[U];
+        long long sig[U], sigv[U];
+#pragma unroll
+        for (int k = 0; k < U; ++k) {
+            peers[k] = __match_any_sync(FULLMASK, cu[k]) & gmask;
+            isL[k] = has[k] && lane == __ffs(peers[k]) - 1;
+            sig[k] = (isL[k] && cu[k] != cv[k]) ? a.Sig[cu[k]] : 0;
+            sigv[k] = (valid[k] && gl == 0) ? a.Sig[cv[k]] : 0;
+        }
+        int tgt[U];
+#pragma unroll
+        for (int k = 0; k < U; ++k) {
+            long long wc;
+            if (UNIT) {
+                wc = __popc(peers[k]);
+            } else {
+                s_acc[wib][lane] = 0;
+                __syncwarp();
+                if (has[k]) atomicAdd(&s_acc[wib][__ffs(peers[k]) - 1], (ull)wt[k]);
+                __syncwarp();
+                wc = (long long)s_acc[wib][lane];
+                __syncwarp();
+            }
+            ST bs = st_min<ST>();
+            int bc = INT_MAX;
+            long long own = 0;
+            if (isL[k]) {
+                my_k++;
+                if (cu[k] == cv[k]) own = wc;
+                else { bs = qW * (ST)wc - p * (ST)sig[k] * (ST)dv[k]; bc = cu[k]; }
+            }
+#pragma unroll
+            for (int off = G / 2; off > 0; off >>= 1) {
+                ST os = shfl_xor_st(bs, off);
+                int oc = __shfl_xor_sync(FULLMASK, bc, off);
+                own += __shfl_xor_sync(FULLMASK, own, off);
+                if (better(os, oc, bs, bc)) { bs = os; bc = oc; }
+            }
+            tgt[k] = cv[k];
+            if (valid[k] && gl == 0) {
+                if (a.check && own != a.dp[v[k]]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
+                tgt[k] = decide_final<ST>(cv[k], dv[k], own, sigv[k], bs, bc, a.size, qW, p);
+            }
+        }
+#pragma unroll
+        for (int k = 0; k < U; ++k)
+            if (valid[k] && gl == 0) a.nextC[v[k]] = tgt[k];
     }
-    ull k = __reduce_add_sync(FULLMASK, (unsigned)my_k);
-    ull md = __reduce_add_sync(FULLMASK, (unsigned)my_moved_deg);
-    if (lane == 0) {
-        if (k) atomicAdd(&a.ctr->bin_k[bin], k);
-        if (md) atomicAdd(&a.ctr->moved_deg, md);
-    }
+    ull k = block_sum_ull<256>(my_k);
+    if (threadIdx.x == 0 && k) atomicAdd(&a.ctr->bin_k[bin], k);
 }
 
 // ---------------------------------------------------------------------------
@@ -267,11 +338,13 @@ __device__ __forceinline__ bool ht_insert(int c, ull wt, int* keys, ull* vals, u
 
 // ---------------------------------------------------------------------------
 // a4 (mid degree): one warp per vertex, per-warp shared-memory hash table with
-// capacity nextpow2(2 deg) <= WCAP (load factor <= 1/2, never spills).
+// capacity nextpow2(2 deg) <= 64*E (load factor <= 1/2, never spills).  Each
+// lane loads its (up to E) neighbours' columns and communities in one batch.
 // ---------------------------------------------------------------------------
-template <int WCAP, typename ST, bool UNIT>
+template <int E, typename ST, bool UNIT>
 __global__ void __launch_bounds__(256) k_decide_warp(const int32_t* __restrict__ queue, int bin, DecideArgs a,
                                                      ST qW, ST p) {
+    constexpr int WCAP = 64 * E;
     __shared__ int s_key[8][WCAP];
     __shared__ ull s_val[8][WCAP];
     const int lane = lane_id(), wib = threadIdx.x >> 5;
@@ -280,25 +353,37 @@ __global__ void __launch_bounds__(256) k_decide_warp(const int32_t* __restrict__
     const long long count = (long long)a.ctr->bin_count[bin];
     const long long nwarps = (long long)gridDim.x * (blockDim.x >> 5);
     ull my_k = 0;
-    for (long long i = (long long)blockIdx.x * (blockDim.x >> 5) + wib; i < count; i += nwarps) {
-        int v = queue[i];
+    long long i = (long long)blockIdx.x * (blockDim.x >> 5) + wib;
+    int v = i < count ? queue[i] : 0;
+    for (; i < count; i += nwarps) {
         int64_t beg = a.rp[v];
         int deg = (int)(a.rp[v + 1] - beg);
+        int cv = a.C[v];
+        long long dv = a.d[v];
+        // prefetch the next queue entry (independent of this vertex)
+        long long inext = i + nwarps;
+        int vnext = inext < count ? queue[inext] : 0;
         int cap = 64;
         while (cap < 2 * deg && cap < WCAP) cap <<= 1;
         unsigned mask = (unsigned)cap - 1;
         for (int j = lane; j < cap; j += 32) { keys[j] = -1; vals[j] = 0; }
-        __syncwarp();
-        for (int j = lane; j < deg; j += 32) {
-            int u = a.col[beg + j];
-            if (u == v) continue;
-            ull wt = UNIT ? 1ull : (ull)a.w[beg + j];
-            int c = a.C[u];
-            ht_insert(c, wt, keys, vals, mask, hash_slot(c, mask), cap);
+        int uu[E];
+        long long ww[E];
+#pragma unroll
+        for (int k = 0; k < E; ++k) {
+            int j = lane + 32 * k;
+            uu[k] = j < deg ? a.col[beg + j] : -1;
+            ww[k] = (j < deg && !UNIT) ? a.w[beg + j] : 1;
         }
+        int cc[E];
+#pragma unroll
+        for (int k = 0; k < E; ++k) cc[k] = (uu[k] >= 0 && uu[k] != v) ? a.C[uu[k]] : -1;
         __syncwarp();
-        int cv = a.C[v];
-        long long dv = a.d[v];
+#pragma unroll
+        for (int k = 0; k < E; ++k)
+            if (cc[k] >= 0) ht_insert(cc[k], (ull)ww[k], keys, vals, mask, hash_slot(cc[k], mask), cap);
+        __syncwarp();
+        long long sig_cv = a.Sig[cv];
         ST bs = st_min<ST>();
         int bc = INT_MAX;
         long long own = 0;
@@ -320,18 +405,13 @@ __global__ void __launch_bounds__(256) k_decide_warp(const int32_t* __restrict__
         }
         if (lane == 0) {
             if (a.check && own != a.dp[v]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
-            int tgt = decide_final<ST>(cv, dv, own, bs, bc, a.Sig, a.size, qW, p);
-            if (tgt != cv) {
-                ull pos = atomicAdd(&a.ctr->n_moved, 1ull);
-                a.mv_v[pos] = v;
-                a.mv_c[pos] = tgt;
-                atomicAdd(&a.ctr->moved_deg, (ull)deg);
-            }
+            a.nextC[v] = decide_final<ST>(cv, dv, own, sig_cv, bs, bc, a.size, qW, p);
         }
         __syncwarp();
+        v = vnext;
     }
-    ull k = __reduce_add_sync(FULLMASK, (unsigned)my_k);
-    if (lane == 0 && k) atomicAdd(&a.ctr->bin_k[bin], k);
+    ull k = block_sum_ull<256>(my_k);
+    if (threadIdx.x == 0 && k) atomicAdd(&a.ctr->bin_k[bin], k);
 }
 
 // ---------------------------------------------------------------------------
@@ -339,10 +419,11 @@ __global__ void __launch_bounds__(256) k_decide_warp(const int32_t* __restrict__
 // (§4.2 "Hierarchical"): shared-memory table H0 probed first
 // (window of HWIN slots), overflow to a per-block global table H1 with linear
 // probing.  H1 is left clean (all empty) after every vertex: the scan phase
-// resets the slots it reads.  Vertices are fetched dynamically.
+// resets the slots it reads.  Vertices are fetched dynamically; each thread
+// batches E row entries per round.
 // ---------------------------------------------------------------------------
 #define HWIN 16
-template <int BT, typename ST, bool UNIT>
+template <int BT, int E, typename ST, bool UNIT>
 __global__ void __launch_bounds__(BT) k_decide_block(const int32_t* __restrict__ queue, int bin, DecideArgs a,
                                                      ST qW, ST p, int smem_cap, int* __restrict__ gkeys_all,
                                                      ull* __restrict__ gvals_all, long long gcap) {
@@ -379,14 +460,25 @@ __global__ void __launch_bounds__(BT) k_decide_block(const int32_t* __restrict__
         unsigned gmask = (unsigned)gc - 1;
         for (int j = threadIdx.x; j < cap; j += BT) { keys[j] = -1; vals[j] = 0; }
         __syncthreads();
-        for (int j = threadIdx.x; j < deg; j += BT) {
-            int u = a.col[beg + j];
-            if (u == v) continue;
-            ull wt = UNIT ? 1ull : (ull)a.w[beg + j];
-            int c = a.C[u];
-            if (!ht_insert(c, wt, keys, vals, mask, hash_slot(c, mask), win)) {
-                if (!s_spill) s_spill = 1;
-                ht_insert(c, wt, gkeys, gvals, gmask, hash_slot2(c, gmask), (int)gc);
+        for (int j0 = threadIdx.x; j0 < deg; j0 += BT * E) {
+            int uu[E];
+            long long ww[E];
+#pragma unroll
+            for (int k = 0; k < E; ++k) {
+                int j = j0 + k * BT;
+                uu[k] = j < deg ? a.col[beg + j] : -1;
+                ww[k] = (j < deg && !UNIT) ? a.w[beg + j] : 1;
+            }
+            int cc[E];
+#pragma unroll
+            for (int k = 0; k < E; ++k) cc[k] = (uu[k] >= 0 && uu[k] != v) ? a.C[uu[k]] : -1;
+#pragma unroll
+            for (int k = 0; k < E; ++k) {
+                if (cc[k] < 0) continue;
+                if (!ht_insert(cc[k], (ull)ww[k], keys, vals, mask, hash_slot(cc[k], mask), win)) {
+                    if (!s_spill) s_spill = 1;
+                    ht_insert(cc[k], (ull)ww[k], gkeys, gvals, gmask, hash_slot2(cc[k], gmask), (int)gc);
+                }
             }
         }
         __syncthreads();
@@ -439,43 +531,78 @@ __global__ void __launch_bounds__(BT) k_decide_block(const int32_t* __restrict__
             }
             if (lane == 0) {
                 if (a.check && own != a.dp[v]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
-                int tgt = decide_final<ST>(cv, dv, own, bs, bc, a.Sig, a.size, qW, p);
-                if (tgt != cv) {
-                    ull pos = atomicAdd(&a.ctr->n_moved, 1ull);
-                    a.mv_v[pos] = v;
-                    a.mv_c[pos] = tgt;
-                    atomicAdd(&a.ctr->moved_deg, (ull)deg);
-                }
+                a.nextC[v] = decide_final<ST>(cv, dv, own, a.Sig[cv], bs, bc, a.size, qW, p);
             }
         }
         __syncthreads();   // table reuse / s_item
     }
-    ull k = __reduce_add_sync(FULLMASK, (unsigned)my_k);
-    if (lane == 0 && k) atomicAdd(&a.ctr->bin_k[bin], k);
+    ull k = block_sum_ull<BT>(my_k);
+    if (threadIdx.x == 0 && k) atomicAdd(&a.ctr->bin_k[bin], k);
 }
 
 // ---------------------------------------------------------------------------
-// a5: apply moves (Alg. 1 line 5): Sigma_tot and sizes by int atomics
-// (order-independent), C[v] <- new, remember the old community for a6.
+// a5: apply moves (Alg. 1 line 5) for every queued (active) vertex whose
+// decision differs: Sigma_tot and sizes by int atomics (order-independent),
+// C[v] <- nextC[v], stamp[v] <- iteration, and the moved list (v, old) with
+// one global atomic per block and tile.
 // ---------------------------------------------------------------------------
-__global__ void k_apply(IterCounters* __restrict__ ctr, const int32_t* __restrict__ mv_v,
-                        const int32_t* __restrict__ mv_c, int32_t* __restrict__ mv_old, int32_t* __restrict__ C,
-                        int64_t* __restrict__ Sig, int32_t* __restrict__ size, const int64_t* __restrict__ d,
-                        int32_t* __restrict__ stamp, int iter_id) {
-    const long long m = (long long)ctr->n_moved;
-    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < m;
-         i += (long long)gridDim.x * blockDim.x) {
-        int v = mv_v[i], nc = mv_c[i];
-        int oc = C[v];
-        long long dv = d[v];
-        mv_old[i] = oc;
-        C[v] = nc;
-        stamp[v] = iter_id;
-        atomicAdd(reinterpret_cast<ull*>(&Sig[oc]), (ull)(-dv));
-        atomicAdd(reinterpret_cast<ull*>(&Sig[nc]), (ull)dv);
-        atomicSub(&size[oc], 1);
-        atomicAdd(&size[nc], 1);
+#define AP_BT 256
+__global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr, const int32_t* __restrict__ queues,
+                                                 long long qstride, const int32_t* __restrict__ nextC,
+                                                 int32_t* __restrict__ C, int64_t* __restrict__ Sig,
+                                                 int32_t* __restrict__ size, const int64_t* __restrict__ d,
+                                                 const int64_t* __restrict__ rp, int32_t* __restrict__ stamp,
+                                                 const Carry* __restrict__ carry, int32_t* __restrict__ mv_v,
+                                                 int32_t* __restrict__ mv_old) {
+    __shared__ unsigned s_cnt;
+    __shared__ ull s_base;
+    long long cnt[NBINS];
+    long long total = 0;
+#pragma unroll
+    for (int b = 0; b < NBINS; ++b) { cnt[b] = (long long)ctr->bin_count[b]; total += cnt[b]; }
+    const int iter_id = carry->iter;
+    ull my_deg = 0;
+    for (long long t0 = (long long)blockIdx.x * AP_BT; t0 < total; t0 += (long long)gridDim.x * AP_BT) {
+        long long i = t0 + threadIdx.x;
+        bool mover = false;
+        int v = 0, oc = 0;
+        if (i < total) {
+            int b = 0;
+            long long r = i;
+#pragma unroll
+            for (int k = 0; k < NBINS - 1; ++k)
+                if (b == k && r >= cnt[k]) { r -= cnt[k]; b = k + 1; }
+            v = queues[(long long)b * qstride + r];
+            int nc = nextC[v];
+            oc = C[v];
+            if (nc != oc) {
+                mover = true;
+                long long dv = d[v];
+                C[v] = nc;
+                stamp[v] = iter_id;
+                atomicAdd(reinterpret_cast<ull*>(&Sig[oc]), (ull)(-dv));
+                atomicAdd(reinterpret_cast<ull*>(&Sig[nc]), (ull)dv);
+                atomicSub(&size[oc], 1);
+                atomicAdd(&size[nc], 1);
+                my_deg += (ull)(rp[v + 1] - rp[v]);
+            }
+        }
+        if (threadIdx.x == 0) s_cnt = 0;
+        __syncthreads();
+        unsigned m = __ballot_sync(FULLMASK, mover);
+        unsigned off = 0;
+        if (m && lane_id() == __ffs(m) - 1) off = atomicAdd(&s_cnt, (unsigned)__popc(m));
+        off = __shfl_sync(FULLMASK, off, m ? __ffs(m) - 1 : 0) + __popc(m & lanemask_lt());
+        __syncthreads();
+        if (threadIdx.x == 0) s_base = s_cnt ? atomicAdd(&ctr->n_moved, (ull)s_cnt) : 0;
+        __syncthreads();
+        if (mover) {
+            mv_v[s_base + off] = v;
+            mv_old[s_base + off] = oc;
+        }
     }
+    ull md = block_sum_ull<AP_BT>(my_deg);
+    if (threadIdx.x == 0 && md) atomicAdd(&ctr->moved_deg, md);
 }
 
 // ---------------------------------------------------------------------------
@@ -498,10 +625,11 @@ __global__ void __launch_bounds__(256) k_dp_delta(IterCounters* __restrict__ ctr
                                                   const int32_t* __restrict__ C, const int32_t* __restrict__ mv_v,
                                                   const int32_t* __restrict__ mv_old,
                                                   const int32_t* __restrict__ stamp, int64_t* __restrict__ dp,
-                                                  int iter_id, long long nnz, int mode, long long fnum,
-                                                  long long fden) {
+                                                  const Carry* __restrict__ carry, long long nnz, int mode,
+                                                  long long fnum, long long fden) {
     if (!use_delta(ctr, nnz, mode, fnum, fden)) return;
     if (blockIdx.x == 0 && threadIdx.x == 0) ctr->delta_used = 1;
+    const int iter_id = carry->iter;
     const int lane = lane_id();
     const long long m = (long long)ctr->n_moved;
     long long wid = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -544,7 +672,15 @@ __global__ void __launch_bounds__(256) k_dp_full(IterCounters* __restrict__ ctr,
         if (v < n) {
             int cv = C[v];
             int64_t b = rp[v], e = rp[v + 1];
-            for (int64_t j = b + gl; j < e; j += 8) {
+            int64_t j = b + gl;
+            for (; j + 8 < e; j += 16) {    // two entries per lane in flight
+                int x0 = col[j], x1 = col[j + 8];
+                long long w0 = UNIT ? 1 : w[j], w1 = UNIT ? 1 : w[j + 8];
+                int c0 = C[x0], c1 = C[x1];
+                if (x0 != v && c0 == cv) acc += w0;
+                if (x1 != v && c1 == cv) acc += w1;
+            }
+            if (j < e) {
                 int x = col[j];
                 if (x != v && C[x] == cv) acc += UNIT ? 1 : w[j];
             }
@@ -576,7 +712,20 @@ __global__ void __launch_bounds__(BT) k_reduce(int n, const int64_t* __restrict_
     __shared__ bool amLast;
     long long dc = 0, mn = LLONG_MAX;
     i128 s2 = 0;
-    for (long long v = (long long)blockIdx.x * BT + threadIdx.x; v < n; v += (long long)gridDim.x * BT) {
+    const long long stride = (long long)gridDim.x * BT;
+    long long v = (long long)blockIdx.x * BT + threadIdx.x;
+    for (; v + 3 * stride < n; v += 4 * stride) {
+        long long a0 = dp[v], a1 = dp[v + stride], a2 = dp[v + 2 * stride], a3 = dp[v + 3 * stride];
+        long long b0 = s[v], b1 = s[v + stride], b2 = s[v + 2 * stride], b3 = s[v + 3 * stride];
+        long long g0 = Sig[v], g1 = Sig[v + stride], g2 = Sig[v + 2 * stride], g3 = Sig[v + 3 * stride];
+        dc += a0 + a1 + a2 + a3 + b0 + b1 + b2 + b3;
+        s2 += (i128)g0 * g0 + (i128)g1 * g1 + (i128)g2 * g2 + (i128)g3 * g3;
+        if (g0 > 0 && g0 < mn) mn = g0;
+        if (g1 > 0 && g1 < mn) mn = g1;
+        if (g2 > 0 && g2 < mn) mn = g2;
+        if (g3 > 0 && g3 < mn) mn = g3;
+    }
+    for (; v < n; v += stride) {
         dc += dp[v] + s[v];
         long long sg = Sig[v];
         s2 += (i128)sg * sg;
@@ -633,4 +782,28 @@ __global__ void __launch_bounds__(BT) k_reduce(int n, const int64_t* __restrict_
         carry->converged = conv;
         ctr->ticket = 0;
     }
+}
+
+// ---------------------------------------------------------------------------
+// end of iteration: append the counters to the device log, advance the
+// iteration index and (graph mode) set the loop condition of the enclosing
+// conditional while-node: continue iff not converged, under the iteration
+// cap and with room in the log.
+// ---------------------------------------------------------------------------
+__global__ void k_record(const IterCounters* __restrict__ ctr, Carry* __restrict__ carry, IterLog* __restrict__ log,
+                         int log_cap, int max_iters, unsigned long long cond_handle) {
+    if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    const int it = carry->iter;
+    const int slot = it - carry->log_base;
+    if (slot >= 0 && slot < log_cap) {
+        IterLog& L = log[slot];
+        L.ctr = *ctr;
+        L.N_hi = carry->N_hi;
+        L.N_lo = carry->N_lo;
+        L.converged = carry->converged;
+    }
+    carry->iter = it + 1;
+    const int more = !carry->converged && (max_iters <= 0 || it + 1 < max_iters) && (slot + 1 < log_cap);
+    carry->more = more;
+    if (cond_handle) cudaGraphSetConditional((cudaGraphConditionalHandle)cond_handle, more ? 1u : 0u);
 }

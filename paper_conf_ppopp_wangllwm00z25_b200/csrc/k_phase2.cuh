@@ -148,8 +148,10 @@ __global__ void k_coarsen_cap(long long k, const long long* __restrict__ ent, lo
     }
 }
 
-// warp per vertex: insert (newid[u], w) into the table of newid[v]; warp-level
-// pre-aggregation of equal keys with __match_any_sync; first inserter of a
+// warp per vertex: insert (newid[u], w) into the table of newid[v].  Equal
+// keys of a 32-entry chunk are combined first (__match_any_sync; popc on unit
+// weights, shared-memory atomics onto the group leader otherwise) so the
+// table sees one atomic per distinct key per chunk; the first inserter of a
 // key bumps deg_new[c'].
 template <bool UNIT>
 __global__ void __launch_bounds__(256) k_coarsen_insert(int n, const int64_t* __restrict__ rp,
@@ -158,7 +160,8 @@ __global__ void __launch_bounds__(256) k_coarsen_insert(int n, const int64_t* __
                                                         const int32_t* __restrict__ newid,
                                                         const long long* __restrict__ hoff, int* __restrict__ hkeys,
                                                         ull* __restrict__ hvals, long long* __restrict__ deg_new) {
-    const int lane = lane_id();
+    __shared__ ull s_acc[8][32];
+    const int lane = lane_id(), wib = threadIdx.x >> 5;
     long long wid = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
     for (long long v = wid; v < n; v += nw) {
@@ -174,16 +177,19 @@ __global__ void __launch_bounds__(256) k_coarsen_insert(int n, const int64_t* __
             int key = has ? newid[col[j]] : (-1 - lane);
             ull wt = has ? (UNIT ? 1ull : (ull)w[j]) : 0ull;
             unsigned peers = __match_any_sync(FULLMASK, key);
-            // sum weights of equal keys onto the leader
-            ull sum = 0;
-            unsigned m = peers;
-            while (m) {
-                int src = __ffs(m) - 1;
-                m &= m - 1;
-                ull x = __shfl_sync(peers, wt, src);
-                sum += x;
+            int leader = __ffs(peers) - 1;
+            ull sum;
+            if (UNIT) {
+                sum = (ull)__popc(peers);
+            } else {
+                s_acc[wib][lane] = 0;
+                __syncwarp();
+                if (has) atomicAdd(&s_acc[wib][leader], wt);
+                __syncwarp();
+                sum = s_acc[wib][lane];
+                __syncwarp();
             }
-            if (has && lane == __ffs(peers) - 1) {
+            if (has && lane == leader) {
                 unsigned h = hash_slot(key, mask);
                 for (;;) {
                     int k0 = *(volatile int*)&keys[h];
@@ -204,29 +210,44 @@ __global__ void __launch_bounds__(256) k_coarsen_insert(int n, const int64_t* __
     }
 }
 
-// thread per table slot: write occupied slots into the coarse CSR rows
-template <bool DUMMY>
-__global__ void k_coarsen_extract(long long k, long long total, const long long* __restrict__ hoff,
-                                  const int* __restrict__ hkeys, const ull* __restrict__ hvals,
-                                  const long long* __restrict__ rp_new, long long* __restrict__ fill,
-                                  int32_t* __restrict__ col_new, int64_t* __restrict__ w_new,
-                                  int64_t* __restrict__ s_new) {
-    for (long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x; t < total;
-         t += (long long)gridDim.x * blockDim.x) {
-        int key = hkeys[t];
-        if (key < 0) continue;
-        // segment: largest c with hoff[c] <= t
-        long long lo = 0, hi = k - 1;
-        while (lo < hi) {
-            long long mid = (lo + hi + 1) >> 1;
-            if (hoff[mid] <= t) lo = mid; else hi = mid - 1;
+// largest c in [lo, hi] with hoff[c] <= t
+__device__ __forceinline__ long long seg_search(const long long* __restrict__ hoff, long long lo, long long hi,
+                                                long long t) {
+    while (lo < hi) {
+        long long mid = (lo + hi + 1) >> 1;
+        if (hoff[mid] <= t) lo = mid; else hi = mid - 1;
+    }
+    return lo;
+}
+
+// 256 consecutive table slots per block: the block's first/last slot find
+// their community by binary search; every other slot searches only between
+// the two (usually zero steps).  Occupied slots go to the coarse CSR rows.
+__global__ void __launch_bounds__(256) k_coarsen_extract(long long k, long long total,
+                                                         const long long* __restrict__ hoff,
+                                                         const int* __restrict__ hkeys, const ull* __restrict__ hvals,
+                                                         const long long* __restrict__ rp_new,
+                                                         long long* __restrict__ fill, int32_t* __restrict__ col_new,
+                                                         int64_t* __restrict__ w_new, int64_t* __restrict__ s_new) {
+    __shared__ long long s_lo, s_hi;
+    for (long long t0 = (long long)blockIdx.x * 256; t0 < total; t0 += (long long)gridDim.x * 256) {
+        long long last = t0 + 255 < total ? t0 + 255 : total - 1;
+        if (threadIdx.x == 0) s_lo = seg_search(hoff, 0, k - 1, t0);
+        if (threadIdx.x == 32) s_hi = seg_search(hoff, 0, k - 1, last);
+        __syncthreads();
+        long long t = t0 + threadIdx.x;
+        if (t < total) {
+            int key = hkeys[t];
+            if (key >= 0) {
+                long long c = seg_search(hoff, s_lo, s_hi, t);
+                ull pos = atomicAdd(reinterpret_cast<ull*>(&fill[c]), 1ull);
+                long long o = rp_new[c] + (long long)pos;
+                col_new[o] = key;
+                w_new[o] = (int64_t)hvals[t];
+                if (key == c) s_new[c] = (int64_t)hvals[t];
+            }
         }
-        long long c = lo;
-        ull pos = atomicAdd(reinterpret_cast<ull*>(&fill[c]), 1ull);
-        long long o = rp_new[c] + (long long)pos;
-        col_new[o] = key;
-        w_new[o] = (int64_t)hvals[t];
-        if (key == c) s_new[c] = (int64_t)hvals[t];
+        __syncthreads();
     }
 }
 

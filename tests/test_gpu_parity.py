@@ -89,10 +89,24 @@ def test_dispatch_independence(opts):
     assert_parity(gg.make("rmat_small"), **opts)
 
 
+@pytest.mark.parametrize("name", ["karate", "lfr_small", "rmat_small"])
+def test_graph_mode_parity(name):
+    """Default launch mode (conditional-while CUDA graph per level, no per-iteration host sync):
+    per-iteration N / moved / active counts and final labels equal the oracle's."""
+    assert_parity(gg.make(name), labels=False)
+
+
+def test_graph_mode_log_relaunch():
+    """A tiny device log forces the host to relaunch the level graph mid-level."""
+    assert_parity(gg.make("lfr_small"), labels=False, log_cap=3)
+    assert_parity(gg.make("lfr_small"), labels=True, log_cap=2, cuda_graph=0)
+
+
 def test_max_levels_and_max_iters():
     g = gg.make("lfr_small")
     assert_parity(g, max_levels=1)
     assert_parity(g, max_levels=2, max_iters=3)
+    assert_parity(g, max_levels=2, max_iters=3, labels=False)
 
 
 def test_device_resident_input_matches_host_input():

@@ -14,9 +14,11 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="lfr1m")
 ap.add_argument("--warm", type=int, default=1)
 ap.add_argument("--max-levels", type=int, default=0)
+ap.add_argument("--cuda-graph", type=int, default=0, help="ncu cannot see kernels inside conditional graphs")
 args = ap.parse_args()
 g = gg.make(args.config)
 h = gala.Graph.from_graph(g)
+h.set_option("cuda_graph", args.cuda_graph)
 for _ in range(args.warm):
     h.run(max_levels=args.max_levels)
 torch.cuda.synchronize()
