@@ -16,8 +16,8 @@ typedef unsigned long long ull;
 
 #define FULLMASK 0xffffffffu
 
-// dispatch bins (a2): sub-warp groups of 4/8/16/32 lanes, warp hash, block hash
-enum { BIN_S4 = 0, BIN_S8 = 1, BIN_S16 = 2, BIN_S32 = 3, BIN_WARP = 4, BIN_BLOCK = 5, NBINS = 6 };
+// dispatch bins (a2): sub-warp groups of 4/8/16/32 lanes, warp hash (<=128, <=512), block hash
+enum { BIN_S4 = 0, BIN_S8 = 1, BIN_S16 = 2, BIN_S32 = 3, BIN_WARP = 4, BIN_WARP2 = 5, BIN_BLOCK = 6, NBINS = 7 };
 
 // Device-resident per-iteration counters (zeroed by k_iter_begin).
 struct IterCounters {
@@ -106,6 +106,25 @@ __device__ __forceinline__ long long warp_append(bool flag, ull* counter) {
     if (lane_id() == leader) base = atomicAdd(counter, (ull)__popc(m));
     base = __shfl_sync(FULLMASK, base, leader);
     return flag ? (long long)(base + __popc(m & lanemask_lt())) : -1;
+}
+
+// Sum of `x` over the lanes of this lane's __match_any_sync group `peers`.
+// 32-bit values use redux.sync with the group mask (every lane of a group
+// passes the same mask, as the warp-primitive contract requires; the
+// match_any + reduce pattern of Alg. 2); 64-bit values go through
+// a per-warp shared-memory scratch (`scratch` = 32 slots of this warp).
+__device__ __forceinline__ unsigned group_sum(unsigned peers, unsigned x, unsigned*) {
+    return __reduce_add_sync(peers, x);
+}
+__device__ __forceinline__ ull group_sum(unsigned peers, ull x, ull* scratch) {
+    const int lane = threadIdx.x & 31;
+    scratch[lane] = 0;
+    __syncwarp();
+    atomicAdd(&scratch[__ffs(peers) - 1], x);
+    __syncwarp();
+    ull r = scratch[__ffs(peers) - 1];
+    __syncwarp();
+    return r;
 }
 
 __device__ __forceinline__ long long warp_sum_ll(long long x) {

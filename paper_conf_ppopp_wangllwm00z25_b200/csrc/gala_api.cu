@@ -20,6 +20,7 @@
 #include "gala.h"
 #include "common.cuh"
 #include "k_phase1.cuh"
+#include "k_decide.cuh"
 #include "k_phase2.cuh"
 #include "dist.h"
 
@@ -58,11 +59,11 @@ static thread_local long long g_launches = 0;
 
 // ------------------------------------------------------------------ kernel classes
 enum KClass {
-    KC_PRUNE = 0, KC_DEC_S4, KC_DEC_S8, KC_DEC_S16, KC_DEC_S32, KC_DEC_WARP, KC_DEC_BLOCK,
+    KC_PRUNE = 0, KC_DEC_S4, KC_DEC_S8, KC_DEC_S16, KC_DEC_S32, KC_DEC_WARP, KC_DEC_WARP2, KC_DEC_BLOCK,
     KC_APPLY, KC_DP, KC_REDUCE, KC_INIT, KC_PHASE2, KC_COUNT
 };
 static const char* kc_names[KC_COUNT] = {"prune_bin", "decide_sub4", "decide_sub8", "decide_sub16",
-                                         "decide_sub32", "decide_warp", "decide_block", "apply",
+                                         "decide_sub32", "decide_warp", "decide_warp512", "decide_block", "apply",
                                          "dp_update", "reduce", "level_init", "phase2"};
 
 struct TraceRec {
@@ -91,13 +92,14 @@ struct gala_graph_s {
     int num_sms = 148;
     // level-0 graph
     DevCSR g0;
-    int64_t n0 = 0, nnz0 = 0, W = 0, maxdeg0 = 0;
+    int64_t n0 = 0, nnz0 = 0, W = 0, maxdeg0 = 0, maxw0 = 0;
     int64_t* d0 = nullptr;
     int64_t* s0 = nullptr;
     // options
     int opt_prune = 1, opt_trace = 0, opt_check = 0, opt_timing = 0, opt_max_iters = 0;
-    int opt_delta = 2, opt_force_i128 = 0, opt_cuda_graph = 1, opt_log_cap = 4096;
-    int bins[NBINS - 1] = {4, 8, 16, 32, 128};
+    int opt_delta = 2, opt_force_i128 = 0, opt_force_wide = 0, opt_cuda_graph = 1, opt_log_cap = 4096, opt_singleton = 1;
+    bool rows_distinct0 = false;   // level-0 rows strictly increasing (no duplicate entries)
+    int bins[NBINS - 1] = {4, 8, 16, 32, 128, 512};
     int hub_smem_slots = 4096;
     // results
     bool has_result = false;
@@ -116,6 +118,7 @@ struct gala_graph_s {
     int check_mismatch = 0;   // check mode: final N on G0 differs from the last level's N
     // dist
     DistCtx* dist = nullptr;
+    struct Work* wk = nullptr;   // persistent run workspace (sized for level 0, reused by every run)
 };
 
 // ------------------------------------------------------------------ memory
@@ -232,16 +235,20 @@ struct Work {
     i128* part_s2 = nullptr;
     int* gkeys = nullptr;
     ull* gvals = nullptr;
+    int* glist = nullptr;
     long long gcap = 0;
     int gblocks = 0;
     IterLog* h_log = nullptr;
     Carry* h_carry = nullptr;
     int reduce_grid = 0;
+    int smem_cap = 0;
+    cudaEvent_t ev[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};
     void release() {
+        for (auto& e : ev) if (e) { cudaEventDestroy(e); e = nullptr; }
         dfree(C, st); dfree(size, st); dfree(stamp, st); dfree(mv_v, st); dfree(mv_old, st); dfree(nextC, st);
         dfree(queues, st); dfree(Sig, st); dfree(d, st); dfree(s, st); dfree(dp, st); dfree(ctr, st);
         dfree(carry, st); dfree(log, st); dfree(part_dc, st); dfree(part_min, st); dfree(part_s2, st);
-        dfree(gkeys, st); dfree(gvals, st);
+        dfree(gkeys, st); dfree(gvals, st); dfree(glist, st);
         if (h_log) cudaFreeHost(h_log);
         if (h_carry) cudaFreeHost(h_carry);
         h_log = nullptr;
@@ -253,50 +260,94 @@ struct Work {
 #define BLOCK_E 4
 
 // ------------------------------------------------------------------ launch helpers
-template <typename ST, bool UNIT>
-static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, ST qW, ST p, Timer& tm, int64_t maxdeg) {
+template <int MAXDEG, int M>
+static void set_warp_smem() {
+    CK(cudaFuncSetAttribute(k_decide_warp<MAXDEG, M, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)WarpSmem<MAXDEG, M>::bytes));
+    CK(cudaFuncSetAttribute(k_decide_warp<MAXDEG, M, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)WarpSmem<MAXDEG, M>::bytes));
+}
+template <int M>
+static size_t block_smem_bytes(int cap) { return (size_t)cap * (sizeof(typename ModeT<M>::VT) + 2 * sizeof(int)); }
+
+template <int M, bool UNIT>
+static void launch_single(gala_graph_s* g, Work& wk, const DecideArgs& a, typename ModeT<M>::ST qW,
+                          typename ModeT<M>::ST p, Timer& tm, int64_t maxdeg) {
+    const long long qs = wk.ncap;
+    const int grid = g->num_sms * 8;
+    cudaStream_t st = g->stream;
+    static const int kcs[NBINS] = {KC_DEC_S4, KC_DEC_S8, KC_DEC_S16, KC_DEC_S32, KC_DEC_WARP, KC_DEC_WARP2, KC_DEC_BLOCK};
+    for (int b = 0; b < NBINS; ++b) {
+        if (b > BIN_S32 && maxdeg <= g->bins[b - 1]) break;
+        cudaEvent_t e = tm.begin();
+        const int32_t* q = wk.queues + b * qs;
+        switch (b) {
+            case BIN_S4: k_decide_single<4, M, UNIT><<<grid, 256, 0, st>>>(q, b, a, qW, p); break;
+            case BIN_S8: k_decide_single<8, M, UNIT><<<grid, 256, 0, st>>>(q, b, a, qW, p); break;
+            case BIN_S16: k_decide_single<16, M, UNIT><<<grid, 256, 0, st>>>(q, b, a, qW, p); break;
+            default: k_decide_single<32, M, UNIT><<<grid, 256, 0, st>>>(q, b, a, qW, p); break;
+        }
+        CKL();
+        tm.end(kcs[b], e);
+    }
+}
+
+template <int M, bool UNIT>
+static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, typename ModeT<M>::ST qW,
+                          typename ModeT<M>::ST p, Timer& tm, int64_t maxdeg, int idbits, bool single) {
     DecideArgs a;
     a.rp = G.rp; a.col = G.col; a.w = G.w; a.C = wk.C; a.Sig = wk.Sig; a.size = wk.size; a.d = wk.d;
     a.dp = wk.dp; a.nextC = wk.nextC; a.ctr = wk.ctr; a.check = g->opt_check;
+    a.idbits = idbits;
+    a.idmask = (1LL << idbits) - 1;
+    if (single) return launch_single<M, UNIT>(g, wk, a, qW, p, tm, maxdeg);
     const long long qs = wk.ncap;
     const int grid = g->num_sms * 8;
     cudaStream_t st = g->stream;
     cudaEvent_t e;
     e = tm.begin();
-    k_decide_sub<4, 4, ST, UNIT><<<grid, 256, 0, st>>>(wk.queues + BIN_S4 * qs, BIN_S4, a, qW, p);
+    k_decide_sub<4, 4, M, UNIT><<<grid, 256, 0, st>>>(wk.queues + BIN_S4 * qs, BIN_S4, a, qW, p);
     CKL();
     tm.end(KC_DEC_S4, e);
     e = tm.begin();
-    k_decide_sub<8, 4, ST, UNIT><<<grid, 256, 0, st>>>(wk.queues + BIN_S8 * qs, BIN_S8, a, qW, p);
+    k_decide_sub<8, 4, M, UNIT><<<grid, 256, 0, st>>>(wk.queues + BIN_S8 * qs, BIN_S8, a, qW, p);
     CKL();
     tm.end(KC_DEC_S8, e);
     e = tm.begin();
-    k_decide_sub<16, 2, ST, UNIT><<<grid, 256, 0, st>>>(wk.queues + BIN_S16 * qs, BIN_S16, a, qW, p);
+    k_decide_sub<16, 2, M, UNIT><<<grid, 256, 0, st>>>(wk.queues + BIN_S16 * qs, BIN_S16, a, qW, p);
     CKL();
     tm.end(KC_DEC_S16, e);
     e = tm.begin();
-    k_decide_sub<32, 2, ST, UNIT><<<grid, 256, 0, st>>>(wk.queues + BIN_S32 * qs, BIN_S32, a, qW, p);
+    k_decide_sub<32, 2, M, UNIT><<<grid, 256, 0, st>>>(wk.queues + BIN_S32 * qs, BIN_S32, a, qW, p);
     CKL();
     tm.end(KC_DEC_S32, e);
     e = tm.begin();
-    k_decide_warp<4, ST, UNIT><<<grid, 256, 0, st>>>(wk.queues + BIN_WARP * qs, BIN_WARP, a, qW, p);
+    k_decide_warp<128, M, UNIT><<<grid, 32 * WarpSmem<128, M>::WPB, WarpSmem<128, M>::bytes, st>>>(
+        wk.queues + BIN_WARP * qs, BIN_WARP, a, qW, p);
     CKL();
     tm.end(KC_DEC_WARP, e);
     if (maxdeg > g->bins[BIN_WARP]) {
-        const int smem_cap = g->hub_smem_slots;
-        size_t smem = (size_t)smem_cap * (sizeof(ull) + sizeof(int));
         e = tm.begin();
-        k_decide_block<BLOCK_BT, BLOCK_E, ST, UNIT><<<wk.gblocks, BLOCK_BT, smem, st>>>(
-            wk.queues + BIN_BLOCK * qs, BIN_BLOCK, a, qW, p, smem_cap, wk.gkeys, wk.gvals, wk.gcap);
+        k_decide_warp<512, M, UNIT><<<grid, 32 * WarpSmem<512, M>::WPB, WarpSmem<512, M>::bytes, st>>>(
+            wk.queues + BIN_WARP2 * qs, BIN_WARP2, a, qW, p);
+        CKL();
+        tm.end(KC_DEC_WARP2, e);
+    }
+    if (maxdeg > g->bins[BIN_WARP2]) {
+        const int smem_cap = g->hub_smem_slots;
+        e = tm.begin();
+        k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT><<<wk.gblocks, BLOCK_BT, block_smem_bytes<M>(smem_cap), st>>>(
+            wk.queues + BIN_BLOCK * qs, BIN_BLOCK, a, qW, p, smem_cap, wk.gkeys, wk.gvals, wk.glist, wk.gcap);
         CKL();
         tm.end(KC_DEC_BLOCK, e);
     }
 }
 
 // one phase-1 iteration (Alg. 1 lines 3-13) + its device log record
-template <typename ST, bool UNIT>
-static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, ST qW, ST p, i128 qW128, i128 T,
-                            Timer& tm, int64_t maxdeg, unsigned long long cond) {
+template <int M, bool UNIT>
+static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, typename ModeT<M>::ST qW,
+                            typename ModeT<M>::ST p, i128 qW128, i128 T, Timer& tm, int64_t maxdeg, int idbits,
+                            unsigned long long cond, bool single) {
     cudaStream_t st = g->stream;
     const int n = (int)G.n;
     const int big = g->num_sms * 8;
@@ -305,11 +356,11 @@ static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, ST qW, S
     CKL();
     BinThresholds th;
     for (int i = 0; i < NBINS - 1; ++i) th.t[i] = g->bins[i];
-    k_prune_bin<ST><<<grid_for((n + PB_IPT - 1) / PB_IPT, PB_BT, big), PB_BT, 0, st>>>(
+    k_prune_bin<typename ModeT<M>::ST><<<grid_for((n + PB_IPT - 1) / PB_IPT, PB_BT, big), PB_BT, 0, st>>>(
         n, G.rp, wk.d, wk.dp, wk.C, wk.Sig, g->opt_prune, qW, p, wk.carry, wk.ctr, wk.queues, wk.ncap, th);
     CKL();
     tm.end(KC_PRUNE, e);
-    launch_decide<ST, UNIT>(g, wk, G, qW, p, tm, maxdeg);
+    launch_decide<M, UNIT>(g, wk, G, qW, p, tm, maxdeg, idbits, single);
     e = tm.begin();
     k_apply<<<grid_for(n, AP_BT, big), AP_BT, 0, st>>>(wk.ctr, wk.queues, wk.ncap, wk.nextC, wk.C, wk.Sig, wk.size,
                                                        wk.d, G.rp, wk.stamp, wk.carry, wk.mv_v, wk.mv_old);
@@ -337,17 +388,20 @@ static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, ST qW, S
 // k_record sets on the device (no host round trip per iteration).  Stepwise
 // mode (trace labels, per-kernel timing, or cuda_graph=0): one host loop trip
 // per iteration.  Both issue the identical kernels.
-template <typename ST, bool UNIT>
-static void phase1_level(gala_graph_s* g, Work& wk, const DevCSR& G, ST qW, ST p, i128 qW128, i128 T, Timer& tm,
-                         int64_t maxdeg, std::vector<IterLog>& out, int level) {
+template <int M, bool UNIT>
+static void phase1_level(gala_graph_s* g, Work& wk, const DevCSR& G, typename ModeT<M>::ST qW,
+                         typename ModeT<M>::ST p, i128 qW128, i128 T, Timer& tm, int64_t maxdeg, int idbits,
+                         std::vector<IterLog>& out, int level, bool single_ok) {
     cudaStream_t st = g->stream;
     const bool stepwise = !g->opt_cuda_graph || g->opt_trace >= 2 || g->opt_timing;
     out.clear();
-    if (stepwise) {
+    // first iteration of a level: singleton fast path when rows hold distinct columns
+    bool first_single = single_ok && g->opt_singleton;
+    int log_base_host = 0;   // mirror of carry->log_base
+    if (stepwise || first_single) {
         for (;;) {
-            issue_iteration<ST, UNIT>(g, wk, G, qW, p, qW128, T, tm, maxdeg, 0ull);
-            CK(cudaMemcpyAsync(wk.h_carry, wk.carry, sizeof(Carry), cudaMemcpyDeviceToHost, st));
-            const int slot = (int)out.size() % wk.log_cap;   // log_base is advanced below
+            issue_iteration<M, UNIT>(g, wk, G, qW, p, qW128, T, tm, maxdeg, idbits, 0ull, first_single);            CK(cudaMemcpyAsync(wk.h_carry, wk.carry, sizeof(Carry), cudaMemcpyDeviceToHost, st));
+            const int slot = (int)out.size() - log_base_host;
             CK(cudaMemcpyAsync(wk.h_log, wk.log + slot, sizeof(IterLog), cudaMemcpyDeviceToHost, st));
             if (g->opt_trace >= 2) {
                 g->trace_labels.emplace_back(G.n);
@@ -358,13 +412,15 @@ static void phase1_level(gala_graph_s* g, Work& wk, const DevCSR& G, ST qW, ST p
             out.push_back(*wk.h_log);
             const Carry& c = *wk.h_carry;
             const bool cap_hit = g->opt_max_iters > 0 && c.iter >= g->opt_max_iters;
-            if (c.converged || cap_hit) break;
+            if (c.converged || cap_hit) return;
             if (!c.more) {   // log full: restart slots at the current iteration
-                int base = c.iter;
-                CK(cudaMemcpyAsync(&wk.carry->log_base, &base, sizeof(int), cudaMemcpyHostToDevice, st));
+                log_base_host = c.iter;
+                CK(cudaMemcpyAsync(&wk.carry->log_base, &log_base_host, sizeof(int), cudaMemcpyHostToDevice, st));
+                CK(cudaStreamSynchronize(st));
             }
+            first_single = false;
+            if (!stepwise) break;   // continue in graph mode
         }
-        return;
     }
     cudaGraph_t graph = nullptr;
     cudaGraphExec_t exec = nullptr;
@@ -382,7 +438,7 @@ static void phase1_level(gala_graph_s* g, Work& wk, const DevCSR& G, ST qW, ST p
         cudaGraph_t body = cp.conditional.phGraph_out[0];
         CK(cudaStreamBeginCaptureToGraph(st, body, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed));
         try {
-            issue_iteration<ST, UNIT>(g, wk, G, qW, p, qW128, T, tm, maxdeg, (unsigned long long)handle);
+            issue_iteration<M, UNIT>(g, wk, G, qW, p, qW128, T, tm, maxdeg, idbits, (unsigned long long)handle, false);
         } catch (...) {
             cudaGraph_t dummy;
             cudaStreamEndCapture(st, &dummy);
@@ -395,14 +451,15 @@ static void phase1_level(gala_graph_s* g, Work& wk, const DevCSR& G, ST qW, ST p
             CK(cudaMemcpyAsync(wk.h_carry, wk.carry, sizeof(Carry), cudaMemcpyDeviceToHost, st));
             CK(cudaStreamSynchronize(st));
             const Carry c = *wk.h_carry;
-            const int nrec = c.iter - c.log_base;
-            CK(cudaMemcpyAsync(wk.h_log, wk.log, sizeof(IterLog) * nrec, cudaMemcpyDeviceToHost, st));
+            const int first = (int)out.size() - log_base_host, last = c.iter - log_base_host;
+            if (last > first)
+                CK(cudaMemcpyAsync(wk.h_log, wk.log + first, sizeof(IterLog) * (last - first), cudaMemcpyDeviceToHost, st));
             CK(cudaStreamSynchronize(st));
-            for (int i = 0; i < nrec; ++i) out.push_back(wk.h_log[i]);
+            for (int i = 0; i < last - first; ++i) out.push_back(wk.h_log[i]);
             const bool cap_hit = g->opt_max_iters > 0 && c.iter >= g->opt_max_iters;
             if (c.converged || cap_hit) break;
-            int base = c.iter;   // log full: continue with fresh slots
-            CK(cudaMemcpyAsync(&wk.carry->log_base, &base, sizeof(int), cudaMemcpyHostToDevice, st));
+            log_base_host = c.iter;   // log full: continue with fresh slots
+            CK(cudaMemcpyAsync(&wk.carry->log_base, &log_base_host, sizeof(int), cudaMemcpyHostToDevice, st));
         }
     } catch (...) {
         if (exec) cudaGraphExecDestroy(exec);
@@ -446,70 +503,114 @@ static void account_bytes(gala_graph_s* g, const IterCounters& c, int64_t n, int
 
 // ------------------------------------------------------------------ phase 2 (a9)
 // Coarsen level graph `cur` with community ids newid[v] in [0, k) into `nxt`
-// (reading c10: the diagonal carries D_C(c) once).  Per-community hash
-// tables (capacity nextpow2(2 min(entries, k))) are filled by k_coarsen_insert
-// and compacted into CSR rows; coarse d(c) = Sigma_tot(c), s(c) = diagonal.
+// (reading c10: the diagonal carries D_C(c) once).  See k_phase2.cuh for
+// the per-community aggregation paths.  Coarse d(c) = Sigma_tot(c), s(c) = diagonal.
+#define AGG_BLOCK_BT 512
+static size_t agg_block_smem(int scap) { return (size_t)scap * (sizeof(ull) + sizeof(int)) + (size_t)(scap / 2) * sizeof(int); }
+
 static void coarsen(gala_graph_s* g, Work& wk, const DevCSR& cur, int64_t nl, long long k, const int32_t* newid,
-                    const int32_t* minmem, bool unit, DevCSR& nxt, int64_t& maxdeg) {
+                    const int32_t* minmem, bool unit, DevCSR& nxt, int64_t& maxdeg, int64_t& dmax) {
     cudaStream_t st = g->stream;
     const int big = g->num_sms * 8;
+    long long* cnt = dalloc<long long>(k + 1, st);
     long long* ent = dalloc<long long>(k + 1, st);
-    long long* hoff = dalloc<long long>(k + 1, st);
-    long long* degn = dalloc<long long>(k + 1, st);
-    CK(cudaMemsetAsync(ent, 0, sizeof(long long) * (k + 1), st));
-    CK(cudaMemsetAsync(degn, 0, sizeof(long long) * (k + 1), st));
-    k_coarsen_count<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, cur.rp, newid, ent);
-    CKL();
-    k_coarsen_cap<<<grid_for(k, 256, big), 256, 0, st>>>(k, ent, hoff);
-    CKL();
-    scan_excl(hoff, hoff, k, st);
-    long long htotal = 0;
-    CK(cudaMemcpyAsync(&htotal, hoff + k, sizeof(long long), cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
-    int* hkeys = dalloc<int>(htotal, st);
-    ull* hvals = dalloc<ull>(htotal, st);
-    CK(cudaMemsetAsync(hkeys, 0xff, sizeof(int) * std::max<long long>(htotal, 1), st));
-    CK(cudaMemsetAsync(hvals, 0, sizeof(ull) * std::max<long long>(htotal, 1), st));
-    if (unit)
-        k_coarsen_insert<true><<<big, 256, 0, st>>>((int)nl, cur.rp, cur.col, cur.w, newid, hoff, hkeys, hvals, degn);
-    else
-        k_coarsen_insert<false><<<big, 256, 0, st>>>((int)nl, cur.rp, cur.col, cur.w, newid, hoff, hkeys, hvals, degn);
-    CKL();
-    nxt.n = k;
-    nxt.rp = dalloc<int64_t>(k + 1, st);
-    scan_excl(degn, reinterpret_cast<long long*>(nxt.rp), k, st);
-    ull* dmax = dalloc<ull>(1, st);
-    CK(cudaMemsetAsync(dmax, 0, sizeof(ull), st));
-    k_rowmax<<<grid_for(k, 256, big), 256, 0, st>>>(k, reinterpret_cast<long long*>(nxt.rp), dmax);
-    CKL();
-    ull mx = 0;
-    CK(cudaMemcpyAsync(&nxt.nnz, nxt.rp + k, sizeof(long long), cudaMemcpyDeviceToHost, st));
-    CK(cudaMemcpyAsync(&mx, dmax, sizeof(ull), cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
-    maxdeg = (int64_t)mx;
-    nxt.col = dalloc<int32_t>(nxt.nnz, st);
-    nxt.w = dalloc<int64_t>(nxt.nnz, st);
-    CK(cudaMemsetAsync(ent, 0, sizeof(long long) * (k + 1), st));   // reuse as fill cursor
+    long long* moff = dalloc<long long>(k + 1, st);
+    long long* eoff = dalloc<long long>(k + 1, st);
+    long long* dn = dalloc<long long>(k + 1, st);
+    int32_t* mem = dalloc<int32_t>(nl, st);
+    int* tkey = dalloc<int>(cur.nnz, st);
+    int64_t* tval = dalloc<int64_t>(cur.nnz, st);
     int64_t* snew = dalloc<int64_t>(k, st);
     int64_t* dnew = dalloc<int64_t>(k, st);
+    ull* dev_max = dalloc<ull>(2, st);
+    int32_t* bigc = dalloc<int32_t>(k, st);
+    long long* bigcap = dalloc<long long>(k + 1, st);
+    int* nbig_dev = dalloc<int>(1, st);
+    CK(cudaMemsetAsync(cnt, 0, sizeof(long long) * (k + 1), st));
+    CK(cudaMemsetAsync(ent, 0, sizeof(long long) * (k + 1), st));
+    CK(cudaMemsetAsync(dn, 0, sizeof(long long) * (k + 1), st));
     CK(cudaMemsetAsync(snew, 0, sizeof(int64_t) * k, st));
-    k_coarsen_extract<<<grid_for(htotal, 256, big * 2), 256, 0, st>>>(k, htotal, hoff, hkeys, hvals,
-                                                                      reinterpret_cast<long long*>(nxt.rp), ent,
-                                                                      nxt.col, nxt.w, snew);
+    CK(cudaMemsetAsync(dev_max, 0, sizeof(ull) * 2, st));
+    CK(cudaMemsetAsync(nbig_dev, 0, sizeof(int), st));
+    k_comm_stats<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, cur.rp, newid, cnt, ent);
+    CKL();
+    scan_excl(cnt, moff, k, st);
+    scan_excl(ent, eoff, k, st);
+    CK(cudaMemsetAsync(cnt, 0, sizeof(long long) * (k + 1), st));   // reuse as member cursor
+    k_members<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, newid, moff, cnt, mem);
+    CKL();
+    // shared-memory capacity of the block path: up to 8192 slots (14 B each)
+    int scap = 512;
+    while (scap < 8192 && scap < 2 * k) scap <<= 1;
+    k_agg_bigflag<<<grid_for(k, 256, big), 256, 0, st>>>(k, ent, scap, bigc, bigcap, nbig_dev);
+    CKL();
+    AggArgs a;
+    a.k = k; a.ent = ent; a.eoff = eoff; a.moff = moff; a.mem = mem; a.rp = cur.rp; a.col = cur.col; a.w = cur.w;
+    a.newid = newid; a.tkey = tkey; a.tval = tval; a.dn = dn; a.snew = snew;
+    if (unit) k_agg_warp<true><<<big, 256, 0, st>>>(a);
+    else k_agg_warp<false><<<big, 256, 0, st>>>(a);
+    CKL();
+    if (scap > AGG_WSLOTS) {
+        const size_t sm = agg_block_smem(scap);
+        CK(cudaFuncSetAttribute(k_agg_block<AGG_BLOCK_BT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+        CK(cudaFuncSetAttribute(k_agg_block<AGG_BLOCK_BT, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+        const int gb = (int)std::min<long long>(k, (long long)g->num_sms * 2);
+        if (unit) k_agg_block<AGG_BLOCK_BT, true><<<gb, AGG_BLOCK_BT, sm, st>>>(a, scap);
+        else k_agg_block<AGG_BLOCK_BT, false><<<gb, AGG_BLOCK_BT, sm, st>>>(a, scap);
+        CKL();
+    }
+    int nbig = 0;
+    CK(cudaMemcpyAsync(&nbig, nbig_dev, sizeof(int), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (nbig > 0) {
+        long long* goff = dalloc<long long>(nbig + 1, st);
+        scan_excl(bigcap, goff, nbig, st);
+        long long gtot = 0;
+        CK(cudaMemcpyAsync(&gtot, goff + nbig, sizeof(long long), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        int* gkeys = dalloc<int>(gtot, st);
+        ull* gvals = dalloc<ull>(gtot, st);
+        int* glist = dalloc<int>(gtot / 2 + 1, st);
+        int* gcnt = dalloc<int>(nbig, st);
+        CK(cudaMemsetAsync(gkeys, 0xff, sizeof(int) * gtot, st));
+        CK(cudaMemsetAsync(gvals, 0, sizeof(ull) * gtot, st));
+        CK(cudaMemsetAsync(gcnt, 0, sizeof(int) * nbig, st));
+        const int bpc = 32;
+        if (unit) k_agg_big_insert<true><<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
+        else k_agg_big_insert<false><<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
+        CKL();
+        k_agg_big_emit<<<std::min(nbig, big), 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt);
+        CKL();
+        dfree(goff, st); dfree(gkeys, st); dfree(gvals, st); dfree(glist, st); dfree(gcnt, st);
+    }
+    nxt.n = k;
+    nxt.rp = dalloc<int64_t>(k + 1, st);
+    scan_excl(dn, reinterpret_cast<long long*>(nxt.rp), k, st);
+    k_rowmax<<<grid_for(k, 256, big), 256, 0, st>>>(k, reinterpret_cast<long long*>(nxt.rp), dev_max);
     CKL();
     // coarse d = Sigma_tot of the community (exactly maintained by phase 1)
     k_coarsen_deg<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.C, minmem, newid, wk.Sig, dnew);
     CKL();
+    k_max_i64<<<grid_for(k, 256, big), 256, 0, st>>>(k, dnew, dev_max + 1);
+    CKL();
+    ull hm[2] = {0, 0};
+    CK(cudaMemcpyAsync(&nxt.nnz, nxt.rp + k, sizeof(long long), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(hm, dev_max, sizeof(ull) * 2, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    maxdeg = (int64_t)hm[0];
+    dmax = (int64_t)hm[1];
+    nxt.col = dalloc<int32_t>(nxt.nnz, st);
+    nxt.w = dalloc<int64_t>(nxt.nnz, st);
+    k_compact<<<grid_for(k * 32, 256, big), 256, 0, st>>>(k, eoff, reinterpret_cast<long long*>(nxt.rp), tkey, tval,
+                                                          nxt.col, nxt.w);
+    CKL();
     CK(cudaMemcpyAsync(wk.d, dnew, sizeof(int64_t) * k, cudaMemcpyDeviceToDevice, st));
     CK(cudaMemcpyAsync(wk.s, snew, sizeof(int64_t) * k, cudaMemcpyDeviceToDevice, st));
-    dfree(snew, st);
-    dfree(dnew, st);
-    dfree(dmax, st);
-    dfree(ent, st);
-    dfree(hoff, st);
-    dfree(degn, st);
-    dfree(hkeys, st);
-    dfree(hvals, st);
+    g->kc_bytes[KC_PHASE2] += (double)nl * (4 + 4 + 8 + 16 + 4 + 4) + (double)cur.nnz * (4 + 4 + (unit ? 0 : 8) + 12) +
+                              (double)nxt.nnz * 24;
+    dfree(cnt, st); dfree(ent, st); dfree(moff, st); dfree(eoff, st); dfree(dn, st); dfree(mem, st);
+    dfree(tkey, st); dfree(tval, st); dfree(snew, st); dfree(dnew, st); dfree(dev_max, st); dfree(bigc, st);
+    dfree(bigcap, st); dfree(nbig_dev, st);
 }
 
 // Final numerator.  The last level's N equals N of the composed labels on the
@@ -572,59 +673,71 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
     const i128 qW128 = (i128)q * W;
     const i128 T = (i128)ceill((long double)tol * (long double)q * (long double)W * (long double)W);
 
-    cudaEvent_t ev_run0, ev_run1;
-    CK(cudaEventCreate(&ev_run0));
-    CK(cudaEventCreate(&ev_run1));
-    CK(cudaEventRecord(ev_run0, st));
-
     const int big = g->num_sms * 8;
     if (!g->lab) g->lab = dalloc<int32_t>(n0, st);
-    Work wk;
-    wk.st = st;
-    wk.ncap = std::max<int64_t>(n0, 1);
-    wk.nnzcap = g->nnz0;
-    wk.log_cap = g->opt_log_cap;
+    if (g->wk && g->wk->log_cap != g->opt_log_cap) { g->wk->release(); delete g->wk; g->wk = nullptr; }
+    if (!g->wk) {
+        g->wk = new Work();
+        Work& wk = *g->wk;
+        wk.st = st;
+        wk.ncap = std::max<int64_t>(n0, 1);
+        wk.nnzcap = g->nnz0;
+        wk.log_cap = g->opt_log_cap;
+        try {
+            wk.C = dalloc<int32_t>(wk.ncap, st);
+            wk.size = dalloc<int32_t>(wk.ncap, st);
+            wk.stamp = dalloc<int32_t>(wk.ncap, st);
+            wk.mv_v = dalloc<int32_t>(wk.ncap, st);
+            wk.mv_old = dalloc<int32_t>(wk.ncap, st);
+            wk.nextC = dalloc<int32_t>(wk.ncap, st);
+            wk.queues = dalloc<int32_t>((size_t)wk.ncap * NBINS, st);
+            wk.Sig = dalloc<int64_t>(wk.ncap, st);
+            wk.d = dalloc<int64_t>(wk.ncap, st);
+            wk.s = dalloc<int64_t>(wk.ncap, st);
+            wk.dp = dalloc<int64_t>(wk.ncap, st);
+            wk.ctr = dalloc<IterCounters>(1, st);
+            wk.carry = dalloc<Carry>(1, st);
+            wk.log = dalloc<IterLog>(wk.log_cap, st);
+            wk.reduce_grid = g->num_sms * 4;
+            wk.part_dc = dalloc<long long>(wk.reduce_grid, st);
+            wk.part_min = dalloc<long long>(wk.reduce_grid, st);
+            wk.part_s2 = dalloc<i128>(wk.reduce_grid, st);
+            CK(cudaMallocHost(&wk.h_log, sizeof(IterLog) * wk.log_cap));
+            CK(cudaMallocHost(&wk.h_carry, sizeof(Carry)));
+            for (int i = 0; i < 5; ++i) CK(cudaEventCreate(&wk.ev[i]));
+            // dynamic shared memory opt-ins, once per workspace
+            int per_sm = 0;
+            const int cap = g->hub_smem_slots;
+            CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, DM_FAST, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)block_smem_bytes<DM_FAST>(cap)));
+            CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, DM_FAST, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)block_smem_bytes<DM_FAST>(cap)));
+            CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, DM_W64, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)block_smem_bytes<DM_W64>(cap)));
+            CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, DM_W64, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)block_smem_bytes<DM_W64>(cap)));
+            CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, DM_W128, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)block_smem_bytes<DM_W128>(cap)));
+            CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, DM_W128, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)block_smem_bytes<DM_W128>(cap)));
+            CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_decide_block<BLOCK_BT, BLOCK_E, DM_W128, false>, BLOCK_BT, block_smem_bytes<DM_W128>(cap)));
+            set_warp_smem<128, DM_FAST>(); set_warp_smem<128, DM_W64>(); set_warp_smem<128, DM_W128>();
+            set_warp_smem<512, DM_FAST>(); set_warp_smem<512, DM_W64>(); set_warp_smem<512, DM_W128>();
+            wk.gblocks = g->num_sms * std::max(per_sm, 1);
+            wk.gcap = 0;   // spill tables sized on demand (coarse levels can have larger rows than level 0)
+            wk.smem_cap = cap;
+        } catch (...) {
+            wk.release();
+            delete g->wk;
+            g->wk = nullptr;
+            throw;
+        }
+    }
+    Work& wk = *g->wk;
+    cudaEvent_t ev_run0 = wk.ev[0], ev_run1 = wk.ev[1];
+    CK(cudaEventRecord(ev_run0, st));
     try {
-        wk.C = dalloc<int32_t>(wk.ncap, st);
-        wk.size = dalloc<int32_t>(wk.ncap, st);
-        wk.stamp = dalloc<int32_t>(wk.ncap, st);
-        wk.mv_v = dalloc<int32_t>(wk.ncap, st);
-        wk.mv_old = dalloc<int32_t>(wk.ncap, st);
-        wk.nextC = dalloc<int32_t>(wk.ncap, st);
-        wk.queues = dalloc<int32_t>((size_t)wk.ncap * NBINS, st);
-        wk.Sig = dalloc<int64_t>(wk.ncap, st);
-        wk.d = dalloc<int64_t>(wk.ncap, st);
-        wk.s = dalloc<int64_t>(wk.ncap, st);
-        wk.dp = dalloc<int64_t>(wk.ncap, st);
-        wk.ctr = dalloc<IterCounters>(1, st);
-        wk.carry = dalloc<Carry>(1, st);
-        wk.log = dalloc<IterLog>(wk.log_cap, st);
-        wk.reduce_grid = g->num_sms * 4;
-        wk.part_dc = dalloc<long long>(wk.reduce_grid, st);
-        wk.part_min = dalloc<long long>(wk.reduce_grid, st);
-        wk.part_s2 = dalloc<i128>(wk.reduce_grid, st);
-        CK(cudaMallocHost(&wk.h_log, sizeof(IterLog) * wk.log_cap));
-        CK(cudaMallocHost(&wk.h_carry, sizeof(Carry)));
         CK(cudaMemsetAsync(wk.ctr, 0, sizeof(IterCounters), st));
         CK(cudaMemsetAsync(wk.carry, 0, sizeof(Carry), st));
-        // block-kernel spill tables: one per resident block
-        {
-            int per_sm = 0;
-            size_t smem = (size_t)g->hub_smem_slots * (sizeof(ull) + sizeof(int));
-            CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, long long, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-            CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, long long, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-            CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, i128, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-            CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, i128, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-            CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_decide_block<BLOCK_BT, BLOCK_E, i128, false>, BLOCK_BT, smem));
-            wk.gblocks = g->num_sms * std::max(per_sm, 1);
-        }
-        wk.gcap = 0;   // sized per level (coarse levels can have larger rows than level 0)
-
         DevCSR cur = g->g0;
         bool cur_owned = false;
         CK(cudaMemcpyAsync(wk.d, g->d0, sizeof(int64_t) * n0, cudaMemcpyDeviceToDevice, st));
         CK(cudaMemcpyAsync(wk.s, g->s0, sizeof(int64_t) * n0, cudaMemcpyDeviceToDevice, st));
-        int64_t maxdeg = g->maxdeg0;
+        int64_t maxdeg = g->maxdeg0, dmax = g->maxw0;
         bool first_level = true;
         Timer tm(g);
         std::vector<IterLog> logs;
@@ -635,20 +748,19 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
             ls.n = nl;
             ls.nnz = cur.nnz;
             ls.maxdeg = maxdeg;
-            cudaEvent_t lv0, lv1, lv2;
-            CK(cudaEventCreate(&lv0));
-            CK(cudaEventCreate(&lv1));
-            CK(cudaEventCreate(&lv2));
+            cudaEvent_t lv0 = wk.ev[2], lv1 = wk.ev[3], lv2 = wk.ev[4];
             CK(cudaEventRecord(lv0, st));
             // spill tables big enough for this level's largest row
             long long need = 64;
             while (need < 2 * maxdeg) need <<= 1;
-            if (maxdeg > g->bins[BIN_WARP] && need > wk.gcap) {
+            if (maxdeg > g->bins[BIN_WARP2] && need > wk.gcap) {
                 dfree(wk.gkeys, st);
                 dfree(wk.gvals, st);
+                dfree(wk.glist, st);
                 wk.gcap = need;
                 wk.gkeys = dalloc<int>((size_t)wk.gblocks * wk.gcap, st);
                 wk.gvals = dalloc<ull>((size_t)wk.gblocks * wk.gcap, st);
+                wk.glist = dalloc<int>((size_t)wk.gblocks * wk.gcap, st);
                 CK(cudaMemsetAsync(wk.gkeys, 0xff, sizeof(int) * (size_t)wk.gblocks * wk.gcap, st));
                 CK(cudaMemsetAsync(wk.gvals, 0, sizeof(ull) * (size_t)wk.gblocks * wk.gcap, st));
             }
@@ -672,19 +784,28 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
             CK(cudaMemcpyAsync(wk.h_carry, wk.carry, sizeof(Carry), cudaMemcpyDeviceToHost, st));
             CK(cudaStreamSynchronize(st));
             const i128 N_start = carry_N(wk.h_carry);
-            // score type for this level: int64 iff max(p,q) * W * max weighted degree < 2^62
-            // (level 0 unit weights: weighted degree = row length; coarse levels: bounded by W)
-            long double bound = (long double)mpq * (long double)W *
-                                (long double)(unit ? std::max<int64_t>(maxdeg, 1) : W);
-            const bool use128 = g->opt_force_i128 || bound >= 0x1p62L;
-            ls.i128path = use128;
-            if (use128) {
-                if (unit) phase1_level<i128, true>(g, wk, cur, (i128)qW128, (i128)p, qW128, T, tm, maxdeg, logs, level);
-                else phase1_level<i128, false>(g, wk, cur, (i128)qW128, (i128)p, qW128, T, tm, maxdeg, logs, level);
+            // gain arithmetic for this level (reading c16):
+            //   |score| <= max(p,q) * W * dmax  (dmax = max weighted degree of the level)
+            //   int64 iff that bound < 2^62; packed (score,-c) keys iff < 2^(62 - idbits); 32-bit
+            //   aggregates iff W < 2^31.
+            int idbits = 1;
+            while (idbits < 31 && ((int64_t)1 << idbits) < nl) ++idbits;
+            const long double bound = (long double)mpq * (long double)W * (long double)std::max<int64_t>(dmax, 1);
+            int mode = DM_FAST;
+            if (g->opt_force_i128 || bound >= 0x1p62L) mode = DM_W128;
+            else if (W >= ((int64_t)1 << 31) || bound * (long double)((int64_t)1 << idbits) >= 0x1p62L || g->opt_force_wide)
+                mode = DM_W64;
+            ls.i128path = mode;
+            const long long qW64 = (long long)qW128, p64 = (long long)p;
+            if (mode == DM_W128) {
+                if (unit) phase1_level<DM_W128, true>(g, wk, cur, (i128)qW128, (i128)p, qW128, T, tm, maxdeg, idbits, logs, level, level > 0 || g->rows_distinct0);
+                else phase1_level<DM_W128, false>(g, wk, cur, (i128)qW128, (i128)p, qW128, T, tm, maxdeg, idbits, logs, level, level > 0 || g->rows_distinct0);
+            } else if (mode == DM_W64) {
+                if (unit) phase1_level<DM_W64, true>(g, wk, cur, qW64, p64, qW128, T, tm, maxdeg, idbits, logs, level, level > 0 || g->rows_distinct0);
+                else phase1_level<DM_W64, false>(g, wk, cur, qW64, p64, qW128, T, tm, maxdeg, idbits, logs, level, level > 0 || g->rows_distinct0);
             } else {
-                long long qW = (long long)qW128, pp = (long long)p;
-                if (unit) phase1_level<long long, true>(g, wk, cur, qW, pp, qW128, T, tm, maxdeg, logs, level);
-                else phase1_level<long long, false>(g, wk, cur, qW, pp, qW128, T, tm, maxdeg, logs, level);
+                if (unit) phase1_level<DM_FAST, true>(g, wk, cur, qW64, p64, qW128, T, tm, maxdeg, idbits, logs, level, level > 0 || g->rows_distinct0);
+                else phase1_level<DM_FAST, false>(g, wk, cur, qW64, p64, qW128, T, tm, maxdeg, idbits, logs, level, level > 0 || g->rows_distinct0);
             }
             i128 N = N_start;
             for (size_t it = 0; it < logs.size(); ++it) {
@@ -728,7 +849,7 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
             CK(cudaStreamSynchronize(st));
             const bool stop = (kcomm == nl) || (max_levels > 0 && level + 1 >= max_levels) || (N - N_start < T);
             DevCSR nxt;
-            if (!stop) coarsen(g, wk, cur, nl, kcomm, newid, minmem, unit, nxt, maxdeg);
+            if (!stop) coarsen(g, wk, cur, nl, kcomm, newid, minmem, unit, nxt, maxdeg, dmax);
             dfree(minmem, st);
             dfree(pos, st);
             dfree(newid, st);
@@ -741,9 +862,6 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
             CK(cudaEventElapsedTime(&ms2, lv1, lv2));
             ls.ms_phase1 = ms1;
             ls.ms_phase2 = ms2;
-            cudaEventDestroy(lv0);
-            cudaEventDestroy(lv1);
-            cudaEventDestroy(lv2);
             g->levels.push_back(ls);
             if (cur_owned) { dfree(cur.rp, st); dfree(cur.col, st); dfree(cur.w, st); }
             if (stop) break;
@@ -763,15 +881,12 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
         CK(cudaEventElapsedTime(&ms, ev_run0, ev_run1));
         g->run_ms = ms;
         g->launches = g_launches - launches0;
-        wk.release();
     } catch (...) {
         wk.release();
-        cudaEventDestroy(ev_run0);
-        cudaEventDestroy(ev_run1);
+        delete g->wk;
+        g->wk = nullptr;
         throw;
     }
-    cudaEventDestroy(ev_run0);
-    cudaEventDestroy(ev_run1);
     g->has_result = true;
 }
 
@@ -817,6 +932,18 @@ static void finish_graph(gala_graph_s* g) {
     CK(cudaMemcpyAsync(&hmx, mx, sizeof(ull), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
     g->maxdeg0 = (int64_t)hmx;
+    CK(cudaMemsetAsync(mx, 0, sizeof(ull), st));
+    k_max_i64<<<grid_for(n, 256, g->num_sms * 8), 256, 0, st>>>(n, g->d0, mx);
+    CKL();
+    CK(cudaMemcpyAsync(&hmx, mx, sizeof(ull), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    g->maxw0 = (int64_t)hmx;
+    CK(cudaMemsetAsync(mx, 0, sizeof(ull), st));
+    k_rows_not_increasing<<<grid_for(n * 32, 256, g->num_sms * 8), 256, 0, st>>>((int)n, g->g0.rp, g->g0.col, mx);
+    CKL();
+    CK(cudaMemcpyAsync(&hmx, mx, sizeof(ull), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    g->rows_distinct0 = (hmx == 0);
     dfree(mx, st);
 }
 
@@ -1055,6 +1182,7 @@ void gala_graph_free(gala_graph g) {
     cudaSetDevice(g->device);
     if (g->dist) dist_free(g->dist);
     cudaStream_t st = g->stream;
+    if (g->wk) { g->wk->release(); delete g->wk; g->wk = nullptr; }
     if (st) {
         dfree(g->g0.rp, st);
         dfree(g->g0.col, st);
@@ -1080,14 +1208,17 @@ gala_status gala_set_option(gala_graph g, const char* key, int64_t value) {
     else if (k == "max_iters") { if (value < 0) return set_err(GALA_E_INVALID, "max_iters < 0"); g->opt_max_iters = (int)value; }
     else if (k == "delta_update") { if (value < 0 || value > 2) return set_err(GALA_E_INVALID, "delta_update in 0..2"); g->opt_delta = (int)value; }
     else if (k == "force_i128") g->opt_force_i128 = value != 0;
+    else if (k == "force_wide") g->opt_force_wide = value != 0;
+    else if (k == "singleton") g->opt_singleton = value != 0;
     else if (k == "cuda_graph") g->opt_cuda_graph = value != 0;
     else if (k == "log_cap") { if (value < 2 || value > (1 << 20)) return set_err(GALA_E_INVALID, "log_cap in [2, 2^20]"); g->opt_log_cap = (int)value; }
     else if (k == "hub_smem_slots") {
         if (value < 64 || value > 16384 || (value & (value - 1))) return set_err(GALA_E_INVALID, "hub_smem_slots: power of two in [64, 16384]");
         g->hub_smem_slots = (int)value;
+        if (g->wk) { g->wk->release(); delete g->wk; g->wk = nullptr; }
     } else if (k.rfind("bin_", 0) == 0) {
-        static const char* names[NBINS - 1] = {"bin_sub4", "bin_sub8", "bin_sub16", "bin_sub32", "bin_warp"};
-        static const int lanes[NBINS - 1] = {4, 8, 16, 32, 128};
+        static const char* names[NBINS - 1] = {"bin_sub4", "bin_sub8", "bin_sub16", "bin_sub32", "bin_warp", "bin_warp512"};
+        static const int lanes[NBINS - 1] = {4, 8, 16, 32, 128, 512};
         int idx = -1;
         for (int i = 0; i < NBINS - 1; ++i) if (k == names[i]) idx = i;
         if (idx < 0) return set_err(GALA_E_INVALID, "unknown option %s", key);
@@ -1149,7 +1280,7 @@ gala_status gala_get_stats(gala_graph g, char* buf, int64_t cap, int64_t* needed
     for (size_t i = 0; i < g->levels.size(); ++i) {
         const LevelStat& l = g->levels[i];
         snprintf(tmp, sizeof tmp,
-                 "%s{\"n\":%lld,\"nnz\":%lld,\"iters\":%lld,\"maxdeg\":%lld,\"i128\":%d,\"ms_phase1\":%.6f,"
+                 "%s{\"n\":%lld,\"nnz\":%lld,\"iters\":%lld,\"maxdeg\":%lld,\"mode\":%d,\"ms_phase1\":%.6f,"
                  "\"ms_phase2\":%.6f,\"edges_scanned\":%lld,\"nominal_edges\":%lld}",
                  i ? "," : "", (long long)l.n, (long long)l.nnz, (long long)l.iters, (long long)l.maxdeg, l.i128path,
                  l.ms_phase1, l.ms_phase2, (long long)l.edges_scanned, (long long)l.nominal_edges);

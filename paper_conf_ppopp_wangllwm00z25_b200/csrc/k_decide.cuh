@@ -1,0 +1,548 @@
+// k_decide.cuh — DecideAndMove kernels (Alg. 1 lines 14-16), §8(a) a3/a4.
+//
+// Every kernel computes, for each queued (active) vertex v, the exact integer
+// decision of reading c1/c4/c5:
+//   score(c) = qW d_c(v) - p Sig[c] d(v)          for neighbouring c != C[v]
+//   stay     = qW d'(v) - p (Sig[C[v]] - d(v)) d(v)
+//   move to argmax (score, lowest c) iff score > stay, unless singleton swap.
+// and writes nextC[v] (C[v] to stay).  The kernels differ only in how the
+// per-community weights d_c(v) are aggregated:
+//   k_decide_sub   (a3) deg <= G lanes: __match_any_sync over the group (Alg. 2)
+//   k_decide_warp  (a4) deg <= 32*E: per-warp shared-memory hash table
+//   k_decide_block (a4) larger: per-block shared-memory table H0 spilling to a
+//                  per-block global table H1 (hierarchical hash, §4.2)
+// Hash kernels follow Alg. 3's ownership rule (footnote 2): the thread
+// that inserts a community into the table owns it and evaluates its gain once
+// all inserts are done, so only occupied slots are ever visited.
+//
+// Modes (chosen per level by the host, never changing a result):
+//   DM_FAST : int64 gains, 32-bit aggregates (W < 2^31), (score, -c) packed in
+//             one int64 key so the argmax is a single 64-bit max reduction
+//             (needs max(p,q) W maxdeg < 2^(62 - idbits))
+//   DM_W64  : int64 gains, 64-bit aggregates, (score, c) pairs
+//   DM_W128 : __int128 gains (reading c16), 64-bit aggregates
+#pragma once
+#include "common.cuh"
+
+enum { DM_FAST = 0, DM_W64 = 1, DM_W128 = 2 };
+template <int M> struct ModeT;
+template <> struct ModeT<DM_FAST> { typedef long long ST; typedef unsigned VT; static constexpr bool PK = true; };
+template <> struct ModeT<DM_W64> { typedef long long ST; typedef ull VT; static constexpr bool PK = false; };
+template <> struct ModeT<DM_W128> { typedef i128 ST; typedef ull VT; static constexpr bool PK = false; };
+
+// running argmax over (score, -community)
+template <typename ST, bool PK> struct Arg {
+    ST s;
+    int c;
+    __device__ __forceinline__ void init(int, long long) { s = st_min<ST>(); c = INT_MAX; }
+    __device__ __forceinline__ void offer(ST sc, int cc) { if (better(sc, cc, s, c)) { s = sc; c = cc; } }
+    __device__ __forceinline__ void xor_merge(int off) {
+        ST os = shfl_xor_st(s, off);
+        int oc = __shfl_xor_sync(FULLMASK, c, off);
+        if (better(os, oc, s, c)) { s = os; c = oc; }
+    }
+    __device__ __forceinline__ bool valid() const { return c != INT_MAX; }
+    __device__ __forceinline__ ST score() const { return s; }
+    __device__ __forceinline__ int comm() const { return c; }
+};
+template <> struct Arg<long long, true> {
+    long long k;
+    int bits;
+    long long mask;
+    __device__ __forceinline__ void init(int idbits, long long idmask) { k = LLONG_MIN; bits = idbits; mask = idmask; }
+    __device__ __forceinline__ void offer(long long sc, int cc) {
+        long long kk = (long long)((ull)sc << bits) | (mask - cc);
+        k = kk > k ? kk : k;
+    }
+    __device__ __forceinline__ void xor_merge(int off) {
+        long long o = __shfl_xor_sync(FULLMASK, k, off);
+        k = o > k ? o : k;
+    }
+    __device__ __forceinline__ bool valid() const { return k != LLONG_MIN; }
+    __device__ __forceinline__ long long score() const { return k >> bits; }
+    __device__ __forceinline__ int comm() const { return (int)(mask - (k & mask)); }
+};
+
+template <typename ST>
+__device__ __forceinline__ ST gain(ST qW, ST p, long long wc, long long sig, long long dv) {
+    return qW * (ST)wc - p * (ST)sig * (ST)dv;
+}
+
+template <typename ST, typename A>
+__device__ __forceinline__ int decide_final(int cv, long long dv, long long own, long long sig_cv, const A& best,
+                                            const int32_t* __restrict__ size, ST qW, ST p) {
+    ST stay = qW * (ST)own - p * (ST)(sig_cv - dv) * (ST)dv;
+    int tgt = cv;
+    if (best.valid() && best.score() > stay) {          // strictly better than staying (c4)
+        tgt = best.comm();
+        if (size[tgt] == 1 && size[cv] == 1 && tgt > cv) tgt = cv;   // swap suppression (c5)
+    }
+    return tgt;
+}
+
+struct DecideArgs {
+    const int64_t* rp;
+    const int32_t* col;
+    const int64_t* w;
+    const int32_t* C;
+    const int64_t* Sig;
+    const int32_t* size;
+    const int64_t* d;
+    const int64_t* dp;
+    int32_t* nextC;     // decision of every processed vertex (C[v] to stay)
+    IterCounters* ctr;
+    int check;
+    int idbits;         // packed-key layout (DM_FAST)
+    long long idmask;
+};
+
+// ---------------------------------------------------------------------------
+// a3: sub-warp groups of G lanes, one neighbour per lane (Alg. 2).
+// Equal communities are found with __match_any_sync; d_c(v) is popc(peers) on
+// unit-weight levels, else the peers' weights summed onto the group leader
+// with shared-memory atomics.  Each group handles U independent vertices per
+// iteration with all their loads issued before use.
+// ---------------------------------------------------------------------------
+template <int G, int U, int M, bool UNIT>
+__global__ void __launch_bounds__(256) k_decide_sub(const int32_t* __restrict__ queue, int bin, DecideArgs a,
+                                                    typename ModeT<M>::ST qW, typename ModeT<M>::ST p) {
+    typedef typename ModeT<M>::ST ST;
+    typedef typename ModeT<M>::VT VT;
+    __shared__ VT s_acc[8][32];
+    const int lane = lane_id(), wib = threadIdx.x >> 5;
+    const int gid = lane / G, gl = lane % G;
+    const unsigned gmask = (G == 32) ? FULLMASK : (((1u << G) - 1u) << (gid * G));
+    const int glead = gid * G;
+    const long long count = (long long)a.ctr->bin_count[bin];
+    const long long nwarps = (long long)gridDim.x * (blockDim.x >> 5);
+    const long long per = (32 / G) * U;
+    unsigned my_k = 0;
+    for (long long base = ((long long)blockIdx.x * (blockDim.x >> 5) + wib) * per; base < count;
+         base += nwarps * per) {
+        int v[U], deg[U], cv[U], u[U], cu[U];
+        int64_t beg[U];
+        long long dv[U], wt[U];
+        bool valid[U], has[U];
+#pragma unroll
+        for (int k = 0; k < U; ++k) {
+            long long i = base + (long long)k * (32 / G) + gid;
+            valid[k] = i < count;
+            v[k] = valid[k] ? queue[i] : 0;
+        }
+#pragma unroll
+        for (int k = 0; k < U; ++k) {
+            beg[k] = valid[k] ? a.rp[v[k]] : 0;
+            int64_t e = valid[k] ? a.rp[v[k] + 1] : 0;
+            deg[k] = (int)(e - beg[k]);
+            cv[k] = valid[k] ? a.C[v[k]] : -2;
+            dv[k] = valid[k] ? a.d[v[k]] : 0;
+        }
+#pragma unroll
+        for (int k = 0; k < U; ++k) {
+            has[k] = valid[k] && gl < deg[k];
+            u[k] = has[k] ? a.col[beg[k] + gl] : -1;
+            wt[k] = (has[k] && !UNIT) ? a.w[beg[k] + gl] : 1;
+        }
+        long long sigv[U];
+#pragma unroll
+        for (int k = 0; k < U; ++k) {
+            if (u[k] == v[k]) has[k] = false;                 // self loop is not a neighbour
+            cu[k] = has[k] ? a.C[u[k]] : (-1 - lane);         // unique sentinel per empty lane
+            sigv[k] = (valid[k] && gl == 0) ? a.Sig[cv[k]] : 0;
+        }
+        unsigned peers[U];
+        bool isL[U];
+        long long sig[U];
+#pragma unroll
+        for (int k = 0; k < U; ++k) {
+            peers[k] = __match_any_sync(FULLMASK, cu[k]) & gmask;
+            isL[k] = has[k] && lane == __ffs(peers[k]) - 1;
+            sig[k] = (isL[k] && cu[k] != cv[k]) ? a.Sig[cu[k]] : 0;
+        }
+        int tgt[U];
+#pragma unroll
+        for (int k = 0; k < U; ++k) {
+            long long wc, own;
+            if (UNIT) {
+                wc = __popc(peers[k]);
+                own = __popc(__ballot_sync(FULLMASK, has[k] && cu[k] == cv[k]) & gmask);
+            } else {
+                wc = (long long)group_sum(peers[k], has[k] ? (VT)wt[k] : (VT)0, s_acc[wib]);
+                unsigned om = __ballot_sync(FULLMASK, isL[k] && cu[k] == cv[k]) & gmask;
+                long long wl = __shfl_sync(FULLMASK, wc, om ? __ffs(om) - 1 : 0);
+                own = om ? wl : 0;
+            }
+            my_k += isL[k];
+            Arg<ST, ModeT<M>::PK> best;
+            best.init(a.idbits, a.idmask);
+            if (isL[k] && cu[k] != cv[k]) best.offer(gain<ST>(qW, p, wc, sig[k], dv[k]), cu[k]);
+#pragma unroll
+            for (int off = G / 2; off > 0; off >>= 1) best.xor_merge(off);
+            tgt[k] = cv[k];
+            if (valid[k] && lane == glead) {
+                if (a.check && own != a.dp[v[k]]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
+                tgt[k] = decide_final<ST>(cv[k], dv[k], own, sigv[k], best, a.size, qW, p);
+            }
+        }
+#pragma unroll
+        for (int k = 0; k < U; ++k)
+            if (valid[k] && gl == 0) a.nextC[v[k]] = tgt[k];
+    }
+    ull k = block_sum_ull<256>((ull)my_k);
+    if (threadIdx.x == 0 && k) atomicAdd(&a.ctr->bin_k[bin], k);
+}
+
+// ---------------------------------------------------------------------------
+// open-addressing insert of (c, +w): CAS on the key, atomicAdd on the value
+// (Alg. 3 lines 6-10).  Linear probing over at most `win` slots.
+// Returns the slot and sets *fresh when this thread created the key; returns
+// -1 when the window holds only other keys.
+// ---------------------------------------------------------------------------
+template <typename VT>
+__device__ __forceinline__ int ht_insert(int c, VT wt, int* keys, VT* vals, unsigned mask, unsigned h, int win,
+                                         bool* fresh) {
+    *fresh = false;
+    for (int t = 0; t < win; ++t) {
+        int k = *(volatile int*)&keys[h];
+        if (k == -1) {
+            int old = atomicCAS(&keys[h], -1, c);
+            if (old == -1) { *fresh = true; atomicAdd(&vals[h], wt); return (int)h; }
+            if (old == c) { atomicAdd(&vals[h], wt); return (int)h; }
+        } else if (k == c) {
+            atomicAdd(&vals[h], wt);
+            return (int)h;
+        }
+        h = (h + 1) & mask;
+    }
+    return -1;
+}
+
+// ---------------------------------------------------------------------------
+// a4 (mid degree): one warp per vertex (deg <= MAXDEG), per-warp shared-memory
+// table of 2*MAXDEG slots (load <= 1/2, never spills) and a distinct-key list.
+// Rows are loaded 4 entries per lane at a time (4 independent gathers in
+// flight per lane).  The table is cleared once per kernel; every vertex clears
+// exactly the slots it used.  Dynamic shared memory: WPB warps per block.
+// ---------------------------------------------------------------------------
+template <int MAXDEG, int M>
+struct WarpSmem {
+    static constexpr int WCAP = 2 * MAXDEG;
+    static constexpr int WPB = MAXDEG <= 128 ? 8 : 4;
+    static constexpr size_t per_warp = 32 * sizeof(ull) + (size_t)WCAP * (sizeof(int) + sizeof(typename ModeT<M>::VT)) +
+                                       (size_t)MAXDEG * sizeof(short) + 16;
+    static constexpr size_t bytes = per_warp * WPB;
+};
+
+template <int MAXDEG, int M, bool UNIT>
+__global__ void __launch_bounds__(32 * WarpSmem<MAXDEG, M>::WPB) k_decide_warp(const int32_t* __restrict__ queue,
+                                                                              int bin, DecideArgs a,
+                                                                              typename ModeT<M>::ST qW,
+                                                                              typename ModeT<M>::ST p) {
+    typedef typename ModeT<M>::ST ST;
+    typedef typename ModeT<M>::VT VT;
+    typedef WarpSmem<MAXDEG, M> SM;
+    constexpr int WCAP = SM::WCAP;
+    constexpr unsigned WMASK = WCAP - 1;
+    constexpr int CH = 4;   // entries per lane per round
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const int lane = lane_id(), wib = threadIdx.x >> 5;
+    unsigned char* base = smem_raw + SM::per_warp * wib;
+    VT* scratch = reinterpret_cast<VT*>(base);
+    base += 32 * sizeof(ull);
+    VT* vals = reinterpret_cast<VT*>(base);
+    int* keys = reinterpret_cast<int*>(base + (size_t)WCAP * sizeof(VT));
+    short* list = reinterpret_cast<short*>(base + (size_t)WCAP * (sizeof(VT) + sizeof(int)));
+    int* cnt = reinterpret_cast<int*>(base + (size_t)WCAP * (sizeof(VT) + sizeof(int)) + (size_t)MAXDEG * sizeof(short));
+    for (int j = lane; j < WCAP; j += 32) { keys[j] = -1; vals[j] = 0; }
+    if (lane == 0) *cnt = 0;
+    __syncwarp();
+    const long long count = (long long)a.ctr->bin_count[bin];
+    const long long nwarps = (long long)gridDim.x * SM::WPB;
+    unsigned my_k = 0;
+    long long i = (long long)blockIdx.x * SM::WPB + wib;
+    int v = i < count ? queue[i] : 0;
+    for (; i < count; i += nwarps) {
+        int64_t beg = a.rp[v];
+        int deg = (int)(a.rp[v + 1] - beg);
+        int cv = a.C[v];
+        long long dv = a.d[v];
+        long long inext = i + nwarps;
+        int vnext = inext < count ? queue[inext] : 0;          // prefetch the next queue entry
+        long long sig_cv = lane == 0 ? a.Sig[cv] : 0;
+        for (int r0 = 0; r0 < deg; r0 += 32 * CH) {          // warp-uniform rounds
+            int uu[CH];
+            VT ww[CH];
+#pragma unroll
+            for (int k = 0; k < CH; ++k) {
+                int j = r0 + lane + 32 * k;
+                uu[k] = j < deg ? a.col[beg + j] : -1;
+                ww[k] = (j < deg && !UNIT) ? (VT)a.w[beg + j] : (VT)1;
+            }
+            int cc[CH];
+#pragma unroll
+            for (int k = 0; k < CH; ++k) cc[k] = (uu[k] >= 0 && uu[k] != v) ? a.C[uu[k]] : -1;
+#pragma unroll
+            for (int k = 0; k < CH; ++k) {
+                if (r0 + 32 * k >= deg) break;                // warp-uniform
+                // combine equal communities of this 32-entry chunk first (one insert per community)
+                const unsigned peers = __match_any_sync(FULLMASK, cc[k] >= 0 ? cc[k] : -1 - lane);
+                const VT sum = UNIT ? (VT)__popc(peers) : group_sum(peers, cc[k] >= 0 ? ww[k] : (VT)0, scratch);
+                if (cc[k] >= 0 && lane == __ffs(peers) - 1) {
+                    bool fresh;
+                    int slot = ht_insert<VT>(cc[k], sum, keys, vals, WMASK, hash_slot(cc[k], WMASK), WCAP, &fresh);
+                    if (fresh) list[atomicAdd(cnt, 1)] = (short)slot;
+                }
+            }
+        }
+        __syncwarp();
+        const int m = *cnt;
+        my_k += (lane == 0) ? m : 0;
+        Arg<ST, ModeT<M>::PK> best;
+        best.init(a.idbits, a.idmask);
+        long long own = 0;
+        for (int t0 = lane; t0 < m; t0 += 32 * CH) {
+            int cs[CH];
+            long long ws[CH];
+#pragma unroll
+            for (int k = 0; k < CH; ++k) {
+                int t = t0 + 32 * k;
+                cs[k] = -1;
+                ws[k] = 0;
+                if (t < m) {
+                    int slot = list[t];
+                    cs[k] = keys[slot];
+                    ws[k] = (long long)vals[slot];
+                    keys[slot] = -1;
+                    vals[slot] = 0;
+                }
+            }
+            long long sg[CH];
+#pragma unroll
+            for (int k = 0; k < CH; ++k) sg[k] = (cs[k] >= 0 && cs[k] != cv) ? a.Sig[cs[k]] : 0;
+#pragma unroll
+            for (int k = 0; k < CH; ++k) {
+                if (cs[k] < 0) continue;
+                if (cs[k] == cv) own = ws[k];
+                else best.offer(gain<ST>(qW, p, ws[k], sg[k], dv), cs[k]);
+            }
+        }
+        __syncwarp();
+        if (lane == 0) *cnt = 0;
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) best.xor_merge(off);
+        own = warp_sum_ll(own);
+        if (lane == 0) {
+            if (a.check && own != a.dp[v]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
+            a.nextC[v] = decide_final<ST>(cv, dv, own, sig_cv, best, a.size, qW, p);
+        }
+        __syncwarp();
+        v = vnext;
+    }
+    ull k = block_sum_ull<32 * SM::WPB>((ull)my_k);
+    if (threadIdx.x == 0 && k) atomicAdd(&a.ctr->bin_k[bin], k);
+}
+
+// ---------------------------------------------------------------------------
+// a4 (high degree / hubs): one block per vertex, hierarchical table (§4.2
+// "Hierarchical"): shared-memory H0 (smem_cap slots, probed over a
+// window of HWIN slots when the row cannot fit at load 1/2), overflow to the
+// block's global H1 with linear probing.  New keys are appended to a distinct
+// list (shared memory for H0, global for H1); after the inserts each list
+// entry is evaluated and its slot cleared, so both tables stay empty between
+// vertices.  Vertices are fetched dynamically; each thread batches E entries.
+// ---------------------------------------------------------------------------
+#define HWIN 16
+template <int BT, int E, int M, bool UNIT>
+__global__ void __launch_bounds__(BT) k_decide_block(const int32_t* __restrict__ queue, int bin, DecideArgs a,
+                                                     typename ModeT<M>::ST qW, typename ModeT<M>::ST p, int smem_cap,
+                                                     int* __restrict__ gkeys_all, ull* __restrict__ gvals_all,
+                                                     int* __restrict__ glist_all, long long gcap) {
+    typedef typename ModeT<M>::ST ST;
+    typedef typename ModeT<M>::VT VT;
+    typedef Arg<ST, ModeT<M>::PK> A;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    VT* vals = reinterpret_cast<VT*>(smem_raw);
+    int* keys = reinterpret_cast<int*>(smem_raw + (size_t)smem_cap * sizeof(VT));
+    int* list = keys + smem_cap;
+    __shared__ long long s_item;
+    __shared__ int s_cnt, s_gcnt;
+    __shared__ A r_a[BT / 32];
+    __shared__ long long r_own[BT / 32];
+    __shared__ VT s_scr[BT / 32][32];
+    const int lane = lane_id(), wib = threadIdx.x >> 5;
+    int* gkeys = gkeys_all + (long long)blockIdx.x * gcap;
+    ull* gvals = gvals_all + (long long)blockIdx.x * gcap;
+    int* glist = glist_all + (long long)blockIdx.x * gcap;
+    const unsigned smask = (unsigned)smem_cap - 1;
+    for (int j = threadIdx.x; j < smem_cap; j += BT) { keys[j] = -1; vals[j] = 0; }
+    if (threadIdx.x == 0) { s_cnt = 0; s_gcnt = 0; }
+    const long long count = (long long)a.ctr->bin_count[bin];
+    unsigned my_k = 0;
+    for (;;) {
+        if (threadIdx.x == 0) s_item = (long long)atomicAdd(&a.ctr->cursor[bin], 1ull);
+        __syncthreads();
+        long long i = s_item;
+        if (i >= count) break;
+        int v = queue[i];
+        int64_t beg = a.rp[v];
+        int deg = (int)(a.rp[v + 1] - beg);
+        int win = (smem_cap >= 2 * deg) ? smem_cap : HWIN;    // fits at load <= 1/2: never spills
+        long long gc = 64;
+        while (gc < 2LL * deg && gc < gcap) gc <<= 1;
+        unsigned gmask = (unsigned)gc - 1;
+        for (int r0 = 0; r0 < deg; r0 += BT * E) {          // block-uniform rounds
+            int uu[E];
+            VT ww[E];
+#pragma unroll
+            for (int k = 0; k < E; ++k) {
+                int j = r0 + threadIdx.x + k * BT;
+                uu[k] = j < deg ? a.col[beg + j] : -1;
+                ww[k] = (j < deg && !UNIT) ? (VT)a.w[beg + j] : (VT)1;
+            }
+            int cc[E];
+#pragma unroll
+            for (int k = 0; k < E; ++k) cc[k] = (uu[k] >= 0 && uu[k] != v) ? a.C[uu[k]] : -1;
+#pragma unroll
+            for (int k = 0; k < E; ++k) {
+                const unsigned peers = __match_any_sync(FULLMASK, cc[k] >= 0 ? cc[k] : -1 - lane);
+                const VT sum = UNIT ? (VT)__popc(peers) : group_sum(peers, cc[k] >= 0 ? ww[k] : (VT)0, s_scr[wib]);
+                if (cc[k] < 0 || lane != __ffs(peers) - 1) continue;
+                bool fresh;
+                int slot = ht_insert<VT>(cc[k], sum, keys, vals, smask, hash_slot(cc[k], smask), win, &fresh);
+                if (slot >= 0) {
+                    if (fresh) list[atomicAdd(&s_cnt, 1)] = slot;
+                } else {
+                    slot = ht_insert<ull>(cc[k], (ull)sum, gkeys, gvals, gmask, hash_slot2(cc[k], gmask), (int)gc,
+                                          &fresh);
+                    if (fresh) glist[atomicAdd(&s_gcnt, 1)] = slot;
+                }
+            }
+        }
+        __syncthreads();
+        const int m = s_cnt, gm = s_gcnt;
+        const int cv = a.C[v];
+        const long long dv = a.d[v];
+        A best;
+        best.init(a.idbits, a.idmask);
+        long long own = 0;
+        my_k += (threadIdx.x == 0) ? (unsigned)(m + gm) : 0u;
+        for (int t0 = threadIdx.x; t0 < m; t0 += BT * E) {
+            int cs[E];
+            long long ws[E];
+#pragma unroll
+            for (int k = 0; k < E; ++k) {
+                int t = t0 + k * BT;
+                cs[k] = -1;
+                if (t < m) {
+                    int slot = list[t];
+                    cs[k] = keys[slot];
+                    ws[k] = (long long)vals[slot];
+                    keys[slot] = -1;
+                    vals[slot] = 0;
+                }
+            }
+            long long sg[E];
+#pragma unroll
+            for (int k = 0; k < E; ++k) sg[k] = (cs[k] >= 0 && cs[k] != cv) ? a.Sig[cs[k]] : 0;
+#pragma unroll
+            for (int k = 0; k < E; ++k) {
+                if (cs[k] < 0) continue;
+                if (cs[k] == cv) own = ws[k];
+                else best.offer(gain<ST>(qW, p, ws[k], sg[k], dv), cs[k]);
+            }
+        }
+        for (int t = threadIdx.x; t < gm; t += BT) {
+            int slot = glist[t];
+            int c = gkeys[slot];
+            long long wc = (long long)gvals[slot];
+            gkeys[slot] = -1;
+            gvals[slot] = 0;
+            if (c == cv) own = wc;
+            else best.offer(gain<ST>(qW, p, wc, a.Sig[c], dv), c);
+        }
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) best.xor_merge(off);
+        own = warp_sum_ll(own);
+        if (lane == 0) { r_a[wib] = best; r_own[wib] = own; }
+        __syncthreads();
+        if (wib == 0) {
+            if (lane < BT / 32) { best = r_a[lane]; own = r_own[lane]; }
+            else { best.init(a.idbits, a.idmask); own = 0; }
+#pragma unroll
+            for (int off = 16; off > 0; off >>= 1) best.xor_merge(off);
+            own = warp_sum_ll(own);
+            if (lane == 0) {
+                if (a.check && own != a.dp[v]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
+                a.nextC[v] = decide_final<ST>(cv, dv, own, a.Sig[cv], best, a.size, qW, p);
+                s_cnt = 0;
+                s_gcnt = 0;
+            }
+        }
+        __syncthreads();   // table / list / s_item reuse
+    }
+    ull k = block_sum_ull<BT>((ull)my_k);
+    if (threadIdx.x == 0 && k) atomicAdd(&a.ctr->bin_k[bin], k);
+}
+
+// ---------------------------------------------------------------------------
+// a3/a4, first iteration of a level: every vertex is a singleton (C[u] = u,
+// Sig[u] = d(u), size 1, d'(v) = 0) and rows hold distinct columns, so
+// d_c(v) = w(v,u) for c = u and no aggregation is needed:
+//   score(u) = qW w(v,u) - p d(u) d(v),  stay = 0,
+//   move to the best u iff score > 0 and u < v (swap suppression, both
+//   singletons) — the iteration-1 closed form.  G lanes per
+//   vertex stream the row, 4 entries per lane in flight.
+// ---------------------------------------------------------------------------
+template <int G, int M, bool UNIT>
+__global__ void __launch_bounds__(256) k_decide_single(const int32_t* __restrict__ queue, int bin, DecideArgs a,
+                                                       typename ModeT<M>::ST qW, typename ModeT<M>::ST p) {
+    typedef typename ModeT<M>::ST ST;
+    const int lane = lane_id(), wib = threadIdx.x >> 5;
+    const int gid = lane / G, gl = lane % G;
+    const long long count = (long long)a.ctr->bin_count[bin];
+    const long long nwarps = (long long)gridDim.x * (blockDim.x >> 5);
+    const long long per = 32 / G;
+    unsigned my_k = 0;
+    for (long long base = ((long long)blockIdx.x * (blockDim.x >> 5) + wib) * per; base < count; base += nwarps * per) {
+        const long long i = base + gid;
+        const bool valid = i < count;
+        const int v = valid ? queue[i] : 0;
+        const int64_t beg = valid ? a.rp[v] : 0;
+        const int deg = valid ? (int)(a.rp[v + 1] - beg) : 0;
+        const long long dv = valid ? a.d[v] : 0;
+        Arg<ST, ModeT<M>::PK> best;
+        best.init(a.idbits, a.idmask);
+        int dmax = deg;   // warp-uniform round count: max row length of the warp's groups
+#pragma unroll
+        for (int o = 16; o >= G; o >>= 1) dmax = max(dmax, __shfl_xor_sync(FULLMASK, dmax, o));
+        for (int r0 = 0; r0 < dmax; r0 += 4 * G) {
+            int uu[4];
+            long long ww[4];
+#pragma unroll
+            for (int t = 0; t < 4; ++t) {
+                int j = r0 + gl + t * G;
+                uu[t] = j < deg ? a.col[beg + j] : -1;
+                ww[t] = (j < deg && !UNIT) ? a.w[beg + j] : 1;
+            }
+            long long du[4];
+#pragma unroll
+            for (int t = 0; t < 4; ++t) du[t] = (uu[t] >= 0 && uu[t] != v) ? a.Sig[uu[t]] : 0;
+#pragma unroll
+            for (int t = 0; t < 4; ++t) {
+                if (uu[t] < 0 || uu[t] == v) continue;
+                my_k++;
+                best.offer(gain<ST>(qW, p, ww[t], du[t], dv), uu[t]);
+            }
+        }
+#pragma unroll
+        for (int off = G / 2; off > 0; off >>= 1) best.xor_merge(off);
+        if (valid && gl == 0) {
+            int tgt = v;
+            if (best.valid() && best.score() > (ST)0 && best.comm() < v) tgt = best.comm();
+            if (a.check && a.dp[v] != 0) atomicAdd(&a.ctr->dp_mismatch, 1ull);
+            a.nextC[v] = tgt;
+        }
+    }
+    ull k = block_sum_ull<256>((ull)my_k);
+    if (threadIdx.x == 0 && k) atomicAdd(&a.ctr->bin_k[bin], k);
+}

@@ -184,363 +184,6 @@ __global__ void __launch_bounds__(PB_BT) k_prune_bin(int n, const int64_t* __res
 }
 
 // ---------------------------------------------------------------------------
-// decision shared by all DecideAndMove kernels
-// ---------------------------------------------------------------------------
-template <typename ST>
-__device__ __forceinline__ int decide_final(int cv, long long dv, long long own, long long sig_cv, ST best_s,
-                                            int best_c, const int32_t* __restrict__ size, ST qW, ST p) {
-    ST stay = qW * (ST)own - p * (ST)(sig_cv - dv) * (ST)dv;
-    int tgt = cv;
-    if (best_c != INT_MAX && best_s > stay) {          // strictly better than staying (c4)
-        tgt = best_c;
-        if (size[tgt] == 1 && size[cv] == 1 && tgt > cv) tgt = cv;   // swap suppression (c5)
-    }
-    return tgt;
-}
-
-struct DecideArgs {
-    const int64_t* rp;
-    const int32_t* col;
-    const int64_t* w;
-    const int32_t* C;
-    const int64_t* Sig;
-    const int32_t* size;
-    const int64_t* d;
-    const int64_t* dp;
-    int32_t* nextC;     // decision of every processed vertex (C[v] to stay)
-    IterCounters* ctr;
-    int check;
-};
-
-// ---------------------------------------------------------------------------
-// a3: low-degree DecideAndMove — sub-warp groups of G lanes, one neighbour per
-// lane, community aggregation with __match_any_sync (Alg. 2).
-// Weighted levels sum the peers' weights with shared-memory atomics onto the
-// group leader; unit-weight levels use popc(peers).  Argmax over the group
-// with an xor-shuffle butterfly on (score, -community).  Each group handles U
-// independent vertices per iteration, all their loads issued before use.
-// ---------------------------------------------------------------------------
-template <int G, int U, typename ST, bool UNIT>
-__global__ void __launch_bounds__(256) k_decide_sub(const int32_t* __restrict__ queue, int bin, DecideArgs a,
-                                                    ST qW, ST p) {
-    __shared__ ull s_acc[8][32];
-    const int lane = lane_id(), wib = threadIdx.x >> 5;
-    const int gid = lane / G, gl = lane % G;
-    const unsigned gmask = (G == 32) ? FULLMASK : (((1u << G) - 1u) << (gid * G));
-    const long long count = (long long)a.ctr->bin_count[bin];
-    const long long nwarps = (long long)gridDim.x * (blockDim.x >> 5);
-    const long long per = (32 / G) * U;
-    ull my_k = 0;
-    for (long long base = ((long long)blockIdx.x * (blockDim.x >> 5) + wib) * per; base < count;
-         base += nwarps * per) {
-        int v[U], deg[U], cv[U], u[U], cu[U];
-        int64_t beg[U];
-        long long dv[U], wt[U];
-        bool valid[U], has[U];
-#pragma unroll
-        for (int k = 0; k < U; ++k) {
-            long long i = base + (long long)k * (32 / G) + gid;
-            valid[k] = i < count;
-            v[k] = valid[k] ? queue[i] : 0;
-        }
-#pragma unroll
-        for (int k = 0; k < U; ++k) {
-            beg[k] = valid[k] ? a.rp[v[k]] : 0;
-            int64_t e = valid[k] ? a.rp[v[k] + 1] : 0;
-            deg[k] = (int)(e - beg[k]);
-            cv[k] = valid[k] ? a.C[v[k]] : -2;
-            dv[k] = valid[k] ? a.d[v[k]] : 0;
-        }
-#pragma unroll
-        for (int k = 0; k < U; ++k) {
-            has[k] = valid[k] && gl < deg[k];
-            u[k] = has[k] ? a.col[beg[k] + gl] : -1;
-            wt[k] = (has[k] && !UNIT) ? a.w[beg[k] + gl] : 1;
-        }
-#pragma unroll
-        for (int k = 0; k < U; ++k) {
-            if (u[k] == v[k]) has[k] = false;                 // self loop is not a neighbour
-            cu[k] = has[k] ? a.C[u[k]] : (-1 - lane);         // unique sentinel per empty lane
-        }
-        unsigned peers[U];
-        bool isL[U];
-        long long sig[U], sigv[U];
-#pragma unroll
-        for (int k = 0; k < U; ++k) {
-            peers[k] = __match_any_sync(FULLMASK, cu[k]) & gmask;
-            isL[k] = has[k] && lane == __ffs(peers[k]) - 1;
-            sig[k] = (isL[k] && cu[k] != cv[k]) ? a.Sig[cu[k]] : 0;
-            sigv[k] = (valid[k] && gl == 0) ? a.Sig[cv[k]] : 0;
-        }
-        int tgt[U];
-#pragma unroll
-        for (int k = 0; k < U; ++k) {
-            long long wc;
-            if (UNIT) {
-                wc = __popc(peers[k]);
-            } else {
-                s_acc[wib][lane] = 0;
-                __syncwarp();
-                if (has[k]) atomicAdd(&s_acc[wib][__ffs(peers[k]) - 1], (ull)wt[k]);
-                __syncwarp();
-                wc = (long long)s_acc[wib][lane];
-                __syncwarp();
-            }
-            ST bs = st_min<ST>();
-            int bc = INT_MAX;
-            long long own = 0;
-            if (isL[k]) {
-                my_k++;
-                if (cu[k] == cv[k]) own = wc;
-                else { bs = qW * (ST)wc - p * (ST)sig[k] * (ST)dv[k]; bc = cu[k]; }
-            }
-#pragma unroll
-            for (int off = G / 2; off > 0; off >>= 1) {
-                ST os = shfl_xor_st(bs, off);
-                int oc = __shfl_xor_sync(FULLMASK, bc, off);
-                own += __shfl_xor_sync(FULLMASK, own, off);
-                if (better(os, oc, bs, bc)) { bs = os; bc = oc; }
-            }
-            tgt[k] = cv[k];
-            if (valid[k] && gl == 0) {
-                if (a.check && own != a.dp[v[k]]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
-                tgt[k] = decide_final<ST>(cv[k], dv[k], own, sigv[k], bs, bc, a.size, qW, p);
-            }
-        }
-#pragma unroll
-        for (int k = 0; k < U; ++k)
-            if (valid[k] && gl == 0) a.nextC[v[k]] = tgt[k];
-    }
-    ull k = block_sum_ull<256>(my_k);
-    if (threadIdx.x == 0 && k) atomicAdd(&a.ctr->bin_k[bin], k);
-}
-
-// ---------------------------------------------------------------------------
-// open-addressing insert: (key, +w) with CAS on the key, atomicAdd on the value
-// (Alg. 3 lines 6-10).  Linear probing up to `win` slots; returns false
-// if the window is full of other keys.
-// ---------------------------------------------------------------------------
-__device__ __forceinline__ bool ht_insert(int c, ull wt, int* keys, ull* vals, unsigned mask, unsigned h,
-                                          int win) {
-    for (int t = 0; t < win; ++t) {
-        int k = *(volatile int*)&keys[h];
-        if (k == -1) {
-            int old = atomicCAS(&keys[h], -1, c);
-            if (old == -1 || old == c) { atomicAdd(&vals[h], wt); return true; }
-        } else if (k == c) {
-            atomicAdd(&vals[h], wt);
-            return true;
-        }
-        h = (h + 1) & mask;
-    }
-    return false;
-}
-
-// ---------------------------------------------------------------------------
-// a4 (mid degree): one warp per vertex, per-warp shared-memory hash table with
-// capacity nextpow2(2 deg) <= 64*E (load factor <= 1/2, never spills).  Each
-// lane loads its (up to E) neighbours' columns and communities in one batch.
-// ---------------------------------------------------------------------------
-template <int E, typename ST, bool UNIT>
-__global__ void __launch_bounds__(256) k_decide_warp(const int32_t* __restrict__ queue, int bin, DecideArgs a,
-                                                     ST qW, ST p) {
-    constexpr int WCAP = 64 * E;
-    __shared__ int s_key[8][WCAP];
-    __shared__ ull s_val[8][WCAP];
-    const int lane = lane_id(), wib = threadIdx.x >> 5;
-    int* keys = s_key[wib];
-    ull* vals = s_val[wib];
-    const long long count = (long long)a.ctr->bin_count[bin];
-    const long long nwarps = (long long)gridDim.x * (blockDim.x >> 5);
-    ull my_k = 0;
-    long long i = (long long)blockIdx.x * (blockDim.x >> 5) + wib;
-    int v = i < count ? queue[i] : 0;
-    for (; i < count; i += nwarps) {
-        int64_t beg = a.rp[v];
-        int deg = (int)(a.rp[v + 1] - beg);
-        int cv = a.C[v];
-        long long dv = a.d[v];
-        // prefetch the next queue entry (independent of this vertex)
-        long long inext = i + nwarps;
-        int vnext = inext < count ? queue[inext] : 0;
-        int cap = 64;
-        while (cap < 2 * deg && cap < WCAP) cap <<= 1;
-        unsigned mask = (unsigned)cap - 1;
-        for (int j = lane; j < cap; j += 32) { keys[j] = -1; vals[j] = 0; }
-        int uu[E];
-        long long ww[E];
-#pragma unroll
-        for (int k = 0; k < E; ++k) {
-            int j = lane + 32 * k;
-            uu[k] = j < deg ? a.col[beg + j] : -1;
-            ww[k] = (j < deg && !UNIT) ? a.w[beg + j] : 1;
-        }
-        int cc[E];
-#pragma unroll
-        for (int k = 0; k < E; ++k) cc[k] = (uu[k] >= 0 && uu[k] != v) ? a.C[uu[k]] : -1;
-        __syncwarp();
-#pragma unroll
-        for (int k = 0; k < E; ++k)
-            if (cc[k] >= 0) ht_insert(cc[k], (ull)ww[k], keys, vals, mask, hash_slot(cc[k], mask), cap);
-        __syncwarp();
-        long long sig_cv = a.Sig[cv];
-        ST bs = st_min<ST>();
-        int bc = INT_MAX;
-        long long own = 0;
-        for (int j = lane; j < cap; j += 32) {
-            int c = keys[j];
-            if (c < 0) continue;
-            my_k++;
-            long long wc = (long long)vals[j];
-            if (c == cv) { own = wc; continue; }
-            ST sc = qW * (ST)wc - p * (ST)a.Sig[c] * (ST)dv;
-            if (better(sc, c, bs, bc)) { bs = sc; bc = c; }
-        }
-#pragma unroll
-        for (int off = 16; off > 0; off >>= 1) {
-            ST os = shfl_xor_st(bs, off);
-            int oc = __shfl_xor_sync(FULLMASK, bc, off);
-            own += __shfl_xor_sync(FULLMASK, own, off);
-            if (better(os, oc, bs, bc)) { bs = os; bc = oc; }
-        }
-        if (lane == 0) {
-            if (a.check && own != a.dp[v]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
-            a.nextC[v] = decide_final<ST>(cv, dv, own, sig_cv, bs, bc, a.size, qW, p);
-        }
-        __syncwarp();
-        v = vnext;
-    }
-    ull k = block_sum_ull<256>(my_k);
-    if (threadIdx.x == 0 && k) atomicAdd(&a.ctr->bin_k[bin], k);
-}
-
-// ---------------------------------------------------------------------------
-// a4 (high degree / hubs): one block per vertex, hierarchical hash table
-// (§4.2 "Hierarchical"): shared-memory table H0 probed first
-// (window of HWIN slots), overflow to a per-block global table H1 with linear
-// probing.  H1 is left clean (all empty) after every vertex: the scan phase
-// resets the slots it reads.  Vertices are fetched dynamically; each thread
-// batches E row entries per round.
-// ---------------------------------------------------------------------------
-#define HWIN 16
-template <int BT, int E, typename ST, bool UNIT>
-__global__ void __launch_bounds__(BT) k_decide_block(const int32_t* __restrict__ queue, int bin, DecideArgs a,
-                                                     ST qW, ST p, int smem_cap, int* __restrict__ gkeys_all,
-                                                     ull* __restrict__ gvals_all, long long gcap) {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    ull* vals = reinterpret_cast<ull*>(smem_raw);
-    int* keys = reinterpret_cast<int*>(smem_raw + (size_t)smem_cap * sizeof(ull));
-    __shared__ long long s_item;
-    __shared__ int s_spill;
-    __shared__ ST r_s[BT / 32];
-    __shared__ int r_c[BT / 32];
-    __shared__ long long r_own[BT / 32];
-    const int lane = lane_id(), wib = threadIdx.x >> 5;
-    int* gkeys = gkeys_all + (long long)blockIdx.x * gcap;
-    ull* gvals = gvals_all + (long long)blockIdx.x * gcap;
-    const long long count = (long long)a.ctr->bin_count[bin];
-    ull my_k = 0;
-    for (;;) {
-        if (threadIdx.x == 0) {
-            s_item = (long long)atomicAdd(&a.ctr->cursor[bin], 1ull);
-            s_spill = 0;
-        }
-        __syncthreads();
-        long long i = s_item;
-        if (i >= count) break;
-        int v = queue[i];
-        int64_t beg = a.rp[v];
-        int deg = (int)(a.rp[v + 1] - beg);
-        int cap = 64;
-        while (cap < 2 * deg && cap < smem_cap) cap <<= 1;
-        unsigned mask = (unsigned)cap - 1;
-        int win = (cap >= 2 * deg) ? cap : HWIN;      // fits: plain linear probing, never spills
-        long long gc = 64;
-        while (gc < 2LL * deg && gc < gcap) gc <<= 1;
-        unsigned gmask = (unsigned)gc - 1;
-        for (int j = threadIdx.x; j < cap; j += BT) { keys[j] = -1; vals[j] = 0; }
-        __syncthreads();
-        for (int j0 = threadIdx.x; j0 < deg; j0 += BT * E) {
-            int uu[E];
-            long long ww[E];
-#pragma unroll
-            for (int k = 0; k < E; ++k) {
-                int j = j0 + k * BT;
-                uu[k] = j < deg ? a.col[beg + j] : -1;
-                ww[k] = (j < deg && !UNIT) ? a.w[beg + j] : 1;
-            }
-            int cc[E];
-#pragma unroll
-            for (int k = 0; k < E; ++k) cc[k] = (uu[k] >= 0 && uu[k] != v) ? a.C[uu[k]] : -1;
-#pragma unroll
-            for (int k = 0; k < E; ++k) {
-                if (cc[k] < 0) continue;
-                if (!ht_insert(cc[k], (ull)ww[k], keys, vals, mask, hash_slot(cc[k], mask), win)) {
-                    if (!s_spill) s_spill = 1;
-                    ht_insert(cc[k], (ull)ww[k], gkeys, gvals, gmask, hash_slot2(cc[k], gmask), (int)gc);
-                }
-            }
-        }
-        __syncthreads();
-        int cv = a.C[v];
-        long long dv = a.d[v];
-        ST bs = st_min<ST>();
-        int bc = INT_MAX;
-        long long own = 0;
-        for (int j = threadIdx.x; j < cap; j += BT) {
-            int c = keys[j];
-            if (c < 0) continue;
-            my_k++;
-            long long wc = (long long)vals[j];
-            if (c == cv) { own = wc; continue; }
-            ST sc = qW * (ST)wc - p * (ST)a.Sig[c] * (ST)dv;
-            if (better(sc, c, bs, bc)) { bs = sc; bc = c; }
-        }
-        if (s_spill) {
-            for (long long j = threadIdx.x; j < gc; j += BT) {
-                int c = gkeys[j];
-                if (c < 0) continue;
-                my_k++;
-                long long wc = (long long)gvals[j];
-                gkeys[j] = -1;
-                gvals[j] = 0;
-                if (c == cv) { own = wc; continue; }
-                ST sc = qW * (ST)wc - p * (ST)a.Sig[c] * (ST)dv;
-                if (better(sc, c, bs, bc)) { bs = sc; bc = c; }
-            }
-        }
-#pragma unroll
-        for (int off = 16; off > 0; off >>= 1) {
-            ST os = shfl_xor_st(bs, off);
-            int oc = __shfl_xor_sync(FULLMASK, bc, off);
-            own += __shfl_xor_sync(FULLMASK, own, off);
-            if (better(os, oc, bs, bc)) { bs = os; bc = oc; }
-        }
-        if (lane == 0) { r_s[wib] = bs; r_c[wib] = bc; r_own[wib] = own; }
-        __syncthreads();
-        if (wib == 0) {
-            bs = lane < BT / 32 ? r_s[lane] : st_min<ST>();
-            bc = lane < BT / 32 ? r_c[lane] : INT_MAX;
-            own = lane < BT / 32 ? r_own[lane] : 0;
-#pragma unroll
-            for (int off = 16; off > 0; off >>= 1) {
-                ST os = shfl_xor_st(bs, off);
-                int oc = __shfl_xor_sync(FULLMASK, bc, off);
-                own += __shfl_xor_sync(FULLMASK, own, off);
-                if (better(os, oc, bs, bc)) { bs = os; bc = oc; }
-            }
-            if (lane == 0) {
-                if (a.check && own != a.dp[v]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
-                a.nextC[v] = decide_final<ST>(cv, dv, own, a.Sig[cv], bs, bc, a.size, qW, p);
-            }
-        }
-        __syncthreads();   // table reuse / s_item
-    }
-    ull k = block_sum_ull<BT>(my_k);
-    if (threadIdx.x == 0 && k) atomicAdd(&a.ctr->bin_k[bin], k);
-}
-
-// ---------------------------------------------------------------------------
 // a5: apply moves (Alg. 1 line 5) for every queued (active) vertex whose
 // decision differs: Sigma_tot and sizes by int atomics (order-independent),
 // C[v] <- nextC[v], stamp[v] <- iteration, and the moved list (v, old) with
@@ -755,15 +398,32 @@ __global__ void __launch_bounds__(BT) k_reduce(int n, const int64_t* __restrict_
         amLast = (t == gridDim.x - 1);
     }
     __syncthreads();
-    if (amLast && threadIdx.x == 0) {
-        __threadfence();
-        long long tdc = 0, tmn = LLONG_MAX;
-        i128 ts2 = 0;
-        for (int b = 0; b < (int)gridDim.x; ++b) {
-            tdc += *(volatile long long*)&part_dc[b];
-            ts2 += part_s2[b];
-            long long m2 = *(volatile long long*)&part_min[b];
-            tmn = m2 < tmn ? m2 : tmn;
+    if (!amLast) return;
+    // last block: combine the per-block partials in parallel
+    __threadfence();
+    long long tdc = 0, tmn = LLONG_MAX;
+    i128 ts2 = 0;
+    for (int b = threadIdx.x; b < (int)gridDim.x; b += BT) {
+        tdc += *(volatile long long*)&part_dc[b];
+        ts2 += mk128(*(volatile long long*)((volatile char*)&part_s2[b] + 8), *(volatile ull*)&part_s2[b]);
+        long long m2 = *(volatile long long*)&part_min[b];
+        tmn = m2 < tmn ? m2 : tmn;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        tdc += __shfl_xor_sync(FULLMASK, tdc, o);
+        ts2 += shfl_xor_st(ts2, o);
+        long long om = __shfl_xor_sync(FULLMASK, tmn, o);
+        tmn = om < tmn ? om : tmn;
+    }
+    __syncthreads();
+    if (lane == 0) { sh_dc[wib] = tdc; sh_s2[wib] = ts2; sh_min[wib] = tmn; }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int i = 1; i < BT / 32; ++i) {
+            tdc += sh_dc[i];
+            ts2 += sh_s2[i];
+            tmn = sh_min[i] < tmn ? sh_min[i] : tmn;
         }
         i128 qW = mk128(qW_hi, qW_lo);
         i128 Nn = qW * (i128)tdc - (i128)p * ts2;

@@ -129,125 +129,246 @@ __global__ void k_compose(long long n0, const int32_t* __restrict__ newid, int32
 // weight = sum of w(v,u) over entries with newid[v] = c', newid[u] = x'.
 // The diagonal (internal weight D_C, reading c10) is one entry.
 // ---------------------------------------------------------------------------
-// ent[c'] += deg(v)
-__global__ void k_coarsen_count(int n, const int64_t* __restrict__ rp, const int32_t* __restrict__ newid,
-                                long long* __restrict__ ent) {
+// Coarsening runs per community c' = newid of a community:
+//   1. k_comm_stats   : members and row entries per community
+//   2. k_members      : member lists (counting sort by community)
+//   3. aggregation of (newid[u], w) over the rows of c's members into a hash
+//      table keyed by coarse neighbour, by the cheapest path that fits:
+//        k_agg_warp  (table <= 256 slots, one warp per community),
+//        k_agg_block (table <= smem capacity, one block per community),
+//        k_agg_big_* (larger: global table shared by BPC blocks);
+//      distinct entries go to a temporary segment at eoff[c'] (its row-entry
+//      offset, an upper bound), their count to dn[c'], the diagonal to snew.
+//   4. k_compact      : segments -> coarse CSR rows (rp_new = scan of dn).
+// Per-community tables are in shared memory on the common paths: the
+// inserts are shared-memory atomics (P:304-316's point about keeping hot
+// state on chip applies to phase 2 as well).
+__global__ void k_comm_stats(int n, const int64_t* __restrict__ rp, const int32_t* __restrict__ newid,
+                             long long* __restrict__ cnt, long long* __restrict__ ent) {
     for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x) {
+        int c = newid[v];
+        atomicAdd(reinterpret_cast<ull*>(&cnt[c]), 1ull);
         long long dg = rp[v + 1] - rp[v];
-        if (dg) atomicAdd(reinterpret_cast<ull*>(&ent[newid[v]]), (ull)dg);
+        if (dg) atomicAdd(reinterpret_cast<ull*>(&ent[c]), (ull)dg);
     }
 }
 
-// per-community hash capacity: nextpow2(2 * min(ent, k)), at least 2
-__global__ void k_coarsen_cap(long long k, const long long* __restrict__ ent, long long* __restrict__ cap) {
-    for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c < k; c += (long long)gridDim.x * blockDim.x) {
-        long long m = ent[c] < k ? ent[c] : k;
-        long long x = 2;
-        while (x < 2 * m) x <<= 1;
-        cap[c] = ent[c] ? x : 0;
+__global__ void k_members(int n, const int32_t* __restrict__ newid, const long long* __restrict__ moff,
+                          long long* __restrict__ cur, int32_t* __restrict__ mem) {
+    for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x) {
+        int c = newid[v];
+        ull pos = atomicAdd(reinterpret_cast<ull*>(&cur[c]), 1ull);
+        mem[moff[c] + (long long)pos] = (int32_t)v;
     }
 }
 
-// warp per vertex: insert (newid[u], w) into the table of newid[v].  Equal
-// keys of a 32-entry chunk are combined first (__match_any_sync; popc on unit
-// weights, shared-memory atomics onto the group leader otherwise) so the
-// table sees one atomic per distinct key per chunk; the first inserter of a
-// key bumps deg_new[c'].
+// table capacity a community needs: nextpow2(2 * min(entries, k)) (0 if no entries)
+__device__ __forceinline__ long long agg_cap(long long ent, long long k) {
+    if (ent == 0) return 0;
+    long long m = ent < k ? ent : k;
+    long long x = 2;
+    while (x < 2 * m) x <<= 1;
+    return x;
+}
+
+struct AggArgs {
+    long long k;
+    const long long* ent;
+    const long long* eoff;     // row-entry offsets (exclusive scan of ent)
+    const long long* moff;     // member offsets
+    const int32_t* mem;
+    const int64_t* rp;
+    const int32_t* col;
+    const int64_t* w;
+    const int32_t* newid;
+    int* tkey;                 // temporary aggregated segments
+    int64_t* tval;
+    long long* dn;             // distinct entries per community
+    int64_t* snew;             // diagonal weight per community
+};
+
+template <typename VT>
+__device__ __forceinline__ int agg_insert(int key, VT wt, int* keys, VT* vals, unsigned mask, int* list, int* cnt) {
+    unsigned h = hash_slot(key, mask);
+    for (;;) {
+        int k0 = *(volatile int*)&keys[h];
+        if (k0 == key) { atomicAdd(&vals[h], wt); return 0; }
+        if (k0 == -1) {
+            int old = atomicCAS(&keys[h], -1, key);
+            if (old == -1) {
+                atomicAdd(&vals[h], wt);
+                list[atomicAdd(cnt, 1)] = (int)h;
+                return 1;
+            }
+            if (old == key) { atomicAdd(&vals[h], wt); return 0; }
+        }
+        h = (h + 1) & mask;
+    }
+}
+
+// the warp streams the rows of its community's members (4 entries per lane in
+// flight); equal keys of each 32-entry chunk are combined before inserting.
+template <bool UNIT, typename VT>
+__device__ __forceinline__ void agg_rows_warp(const AggArgs& a, long long m0, long long m1, int lane, int* keys,
+                                              VT* vals, unsigned mask, int* list, int* cnt, int mstride,
+                                              int mfirst, ull* scratch) {
+    for (long long mi = m0 + mfirst; mi < m1; mi += mstride) {
+        int v = a.mem[mi];
+        int64_t b = a.rp[v], e = a.rp[v + 1];
+        for (int64_t r0 = b; r0 < e; r0 += 128) {          // warp-uniform rounds
+            int uu[4];
+            VT ww[4];
+#pragma unroll
+            for (int t = 0; t < 4; ++t) {
+                int64_t j = r0 + lane + 32 * t;
+                uu[t] = j < e ? a.col[j] : -1;
+                ww[t] = (j < e && !UNIT) ? (VT)a.w[j] : (VT)1;
+            }
+            int kk[4];
+#pragma unroll
+            for (int t = 0; t < 4; ++t) kk[t] = uu[t] >= 0 ? a.newid[uu[t]] : -1;
+#pragma unroll
+            for (int t = 0; t < 4; ++t) {
+                if (r0 + 32 * t >= e) break;
+                const unsigned peers = __match_any_sync(FULLMASK, kk[t] >= 0 ? kk[t] : -1 - lane);
+                const ull sum = UNIT ? (ull)__popc(peers) : group_sum(peers, kk[t] >= 0 ? (ull)ww[t] : 0ull, scratch);
+                if (kk[t] >= 0 && lane == __ffs(peers) - 1) agg_insert<VT>(kk[t], (VT)sum, keys, vals, mask, list, cnt);
+            }
+        }
+    }
+}
+
+// write the distinct entries of community c to its temporary segment
+template <typename VT>
+__device__ __forceinline__ void agg_emit(const AggArgs& a, long long c, int m, const int* list, int* keys, VT* vals,
+                                         int tid, int nt) {
+    const long long o = a.eoff[c];
+    for (int t = tid; t < m; t += nt) {
+        int slot = list[t];
+        int key = keys[slot];
+        int64_t val = (int64_t)vals[slot];
+        keys[slot] = -1;
+        vals[slot] = 0;
+        a.tkey[o + t] = key;
+        a.tval[o + t] = val;
+        if (key == (int)c) a.snew[c] = val;
+    }
+}
+
+#define AGG_WSLOTS 256
 template <bool UNIT>
-__global__ void __launch_bounds__(256) k_coarsen_insert(int n, const int64_t* __restrict__ rp,
-                                                        const int32_t* __restrict__ col,
-                                                        const int64_t* __restrict__ w,
-                                                        const int32_t* __restrict__ newid,
-                                                        const long long* __restrict__ hoff, int* __restrict__ hkeys,
-                                                        ull* __restrict__ hvals, long long* __restrict__ deg_new) {
-    __shared__ ull s_acc[8][32];
+__global__ void __launch_bounds__(256) k_agg_warp(AggArgs a) {
+    __shared__ int s_key[8][AGG_WSLOTS];
+    __shared__ ull s_val[8][AGG_WSLOTS];
+    __shared__ int s_list[8][AGG_WSLOTS / 2];
+    __shared__ int s_cnt[8];
+    __shared__ ull s_scr[8][32];
     const int lane = lane_id(), wib = threadIdx.x >> 5;
-    long long wid = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
-    for (long long v = wid; v < n; v += nw) {
-        int cs = newid[v];
-        int64_t b = rp[v], e = rp[v + 1];
-        long long off = hoff[cs];
-        unsigned mask = (unsigned)(hoff[cs + 1] - off) - 1u;
-        int* keys = hkeys + off;
-        ull* vals = hvals + off;
-        for (int64_t j0 = b; j0 < e; j0 += 32) {
-            int64_t j = j0 + lane;
-            bool has = j < e;
-            int key = has ? newid[col[j]] : (-1 - lane);
-            ull wt = has ? (UNIT ? 1ull : (ull)w[j]) : 0ull;
-            unsigned peers = __match_any_sync(FULLMASK, key);
-            int leader = __ffs(peers) - 1;
-            ull sum;
-            if (UNIT) {
-                sum = (ull)__popc(peers);
-            } else {
-                s_acc[wib][lane] = 0;
-                __syncwarp();
-                if (has) atomicAdd(&s_acc[wib][leader], wt);
-                __syncwarp();
-                sum = s_acc[wib][lane];
-                __syncwarp();
-            }
-            if (has && lane == leader) {
-                unsigned h = hash_slot(key, mask);
-                for (;;) {
-                    int k0 = *(volatile int*)&keys[h];
-                    if (k0 == key) { atomicAdd(&vals[h], sum); break; }
-                    if (k0 == -1) {
-                        int old = atomicCAS(&keys[h], -1, key);
-                        if (old == -1) {
-                            atomicAdd(&vals[h], sum);
-                            atomicAdd(reinterpret_cast<ull*>(&deg_new[cs]), 1ull);
-                            break;
-                        }
-                        if (old == key) { atomicAdd(&vals[h], sum); break; }
-                    }
-                    h = (h + 1) & mask;
-                }
-            }
+    int* keys = s_key[wib];
+    ull* vals = s_val[wib];
+    int* list = s_list[wib];
+    for (int j = lane; j < AGG_WSLOTS; j += 32) { keys[j] = -1; vals[j] = 0; }
+    if (lane == 0) s_cnt[wib] = 0;
+    __syncwarp();
+    const long long nw = (long long)gridDim.x * 8;
+    for (long long c = (long long)blockIdx.x * 8 + wib; c < a.k; c += nw) {
+        long long cap = agg_cap(a.ent[c], a.k);
+        if (cap == 0) { if (lane == 0) a.dn[c] = 0; continue; }
+        if (cap > AGG_WSLOTS) continue;
+        agg_rows_warp<UNIT, ull>(a, a.moff[c], a.moff[c + 1], lane, keys, vals, (unsigned)cap - 1, list, &s_cnt[wib],
+                                 1, 0, s_scr[wib]);
+        __syncwarp();
+        int m = s_cnt[wib];
+        agg_emit<ull>(a, c, m, list, keys, vals, lane, 32);
+        __syncwarp();
+        if (lane == 0) { a.dn[c] = m; s_cnt[wib] = 0; }
+        __syncwarp();
+    }
+}
+
+template <int BT, bool UNIT>
+__global__ void __launch_bounds__(BT) k_agg_block(AggArgs a, int scap) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    ull* vals = reinterpret_cast<ull*>(smem_raw);
+    int* keys = reinterpret_cast<int*>(smem_raw + (size_t)scap * sizeof(ull));
+    int* list = keys + scap;
+    __shared__ int s_cnt;
+    __shared__ ull s_scr[BT / 32][32];
+    const int lane = lane_id(), wib = threadIdx.x >> 5;
+    for (int j = threadIdx.x; j < scap; j += BT) { keys[j] = -1; vals[j] = 0; }
+    if (threadIdx.x == 0) s_cnt = 0;
+    __syncthreads();
+    for (long long c = blockIdx.x; c < a.k; c += gridDim.x) {
+        long long cap = agg_cap(a.ent[c], a.k);
+        if (cap <= AGG_WSLOTS || cap > scap) continue;   // block-uniform
+        agg_rows_warp<UNIT, ull>(a, a.moff[c], a.moff[c + 1], lane, keys, vals, (unsigned)cap - 1, list, &s_cnt,
+                                 BT / 32, wib, s_scr[wib]);
+        __syncthreads();
+        int m = s_cnt;
+        agg_emit<ull>(a, c, m, list, keys, vals, threadIdx.x, BT);
+        __syncthreads();
+        if (threadIdx.x == 0) { a.dn[c] = m; s_cnt = 0; }
+        __syncthreads();
+    }
+}
+
+// big communities: BPC blocks per community insert into its global table
+template <bool UNIT>
+__global__ void __launch_bounds__(256) k_agg_big_insert(AggArgs a, const int32_t* __restrict__ bigc, int nbig,
+                                                        const long long* __restrict__ goff, int* __restrict__ gkeys,
+                                                        ull* __restrict__ gvals, int* __restrict__ glist,
+                                                        int* __restrict__ gcnt, int bpc) {
+    __shared__ ull s_scr[8][32];
+    const int lane = lane_id(), wib = threadIdx.x >> 5;
+    for (long long b = blockIdx.x; b < (long long)nbig * bpc; b += gridDim.x) {
+        int bi = (int)(b / bpc), part = (int)(b % bpc);
+        long long c = bigc[bi];
+        long long off = goff[bi];
+        unsigned mask = (unsigned)(goff[bi + 1] - off) - 1u;
+        agg_rows_warp<UNIT, ull>(a, a.moff[c], a.moff[c + 1], lane, gkeys + off, gvals + off, mask, glist + off / 2,
+                                 &gcnt[bi], bpc * 8, part * 8 + wib, s_scr[wib]);
+    }
+}
+
+__global__ void __launch_bounds__(256) k_agg_big_emit(AggArgs a, const int32_t* __restrict__ bigc, int nbig,
+                                                      const long long* __restrict__ goff, int* __restrict__ gkeys,
+                                                      ull* __restrict__ gvals, const int* __restrict__ glist,
+                                                      const int* __restrict__ gcnt) {
+    for (int bi = blockIdx.x; bi < nbig; bi += gridDim.x) {
+        long long c = bigc[bi];
+        long long off = goff[bi];
+        int m = gcnt[bi];
+        agg_emit<ull>(a, c, m, glist + off / 2, gkeys + off, gvals + off, threadIdx.x, 256);
+        if (threadIdx.x == 0) a.dn[c] = m;
+    }
+}
+
+// flag + list of communities whose table exceeds the shared-memory capacity
+__global__ void k_agg_bigflag(long long k, const long long* __restrict__ ent, int scap, int32_t* __restrict__ bigc,
+                              long long* __restrict__ bigcap, int* __restrict__ nbig) {
+    for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c < k; c += (long long)gridDim.x * blockDim.x) {
+        long long cap = agg_cap(ent[c], k);
+        if (cap > scap) {
+            int i = atomicAdd(nbig, 1);
+            bigc[i] = (int32_t)c;
+            bigcap[i] = cap;
         }
     }
 }
 
-// largest c in [lo, hi] with hoff[c] <= t
-__device__ __forceinline__ long long seg_search(const long long* __restrict__ hoff, long long lo, long long hi,
-                                                long long t) {
-    while (lo < hi) {
-        long long mid = (lo + hi + 1) >> 1;
-        if (hoff[mid] <= t) lo = mid; else hi = mid - 1;
-    }
-    return lo;
-}
-
-// 256 consecutive table slots per block: the block's first/last slot find
-// their community by binary search; every other slot searches only between
-// the two (usually zero steps).  Occupied slots go to the coarse CSR rows.
-__global__ void __launch_bounds__(256) k_coarsen_extract(long long k, long long total,
-                                                         const long long* __restrict__ hoff,
-                                                         const int* __restrict__ hkeys, const ull* __restrict__ hvals,
-                                                         const long long* __restrict__ rp_new,
-                                                         long long* __restrict__ fill, int32_t* __restrict__ col_new,
-                                                         int64_t* __restrict__ w_new, int64_t* __restrict__ s_new) {
-    __shared__ long long s_lo, s_hi;
-    for (long long t0 = (long long)blockIdx.x * 256; t0 < total; t0 += (long long)gridDim.x * 256) {
-        long long last = t0 + 255 < total ? t0 + 255 : total - 1;
-        if (threadIdx.x == 0) s_lo = seg_search(hoff, 0, k - 1, t0);
-        if (threadIdx.x == 32) s_hi = seg_search(hoff, 0, k - 1, last);
-        __syncthreads();
-        long long t = t0 + threadIdx.x;
-        if (t < total) {
-            int key = hkeys[t];
-            if (key >= 0) {
-                long long c = seg_search(hoff, s_lo, s_hi, t);
-                ull pos = atomicAdd(reinterpret_cast<ull*>(&fill[c]), 1ull);
-                long long o = rp_new[c] + (long long)pos;
-                col_new[o] = key;
-                w_new[o] = (int64_t)hvals[t];
-                if (key == c) s_new[c] = (int64_t)hvals[t];
-            }
+// warp per community: copy its aggregated segment into the coarse CSR row
+__global__ void __launch_bounds__(256) k_compact(long long k, const long long* __restrict__ eoff,
+                                                 const long long* __restrict__ rp_new, const int* __restrict__ tkey,
+                                                 const int64_t* __restrict__ tval, int32_t* __restrict__ col_new,
+                                                 int64_t* __restrict__ w_new) {
+    const int lane = lane_id();
+    const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+    for (long long c = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < k; c += nw) {
+        long long o = eoff[c], r = rp_new[c], m = rp_new[c + 1] - r;
+        for (long long t = lane; t < m; t += 32) {
+            col_new[r + t] = tkey[o + t];
+            w_new[r + t] = tval[o + t];
         }
-        __syncthreads();
     }
 }
 
@@ -257,6 +378,28 @@ __global__ void k_coarsen_deg(int n, const int32_t* __restrict__ C, const int32_
                               int64_t* __restrict__ d_new) {
     for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x)
         if (minmem[C[v]] == v) d_new[newid[v]] = Sig[C[v]];
+}
+
+// *bad != 0 iff some row is not strictly increasing (so may hold duplicate columns)
+__global__ void k_rows_not_increasing(int n, const int64_t* __restrict__ rp, const int32_t* __restrict__ col,
+                                      ull* __restrict__ bad) {
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) {
+        for (int64_t j = rp[v] + 1; j < rp[v + 1]; ++j)
+            if (col[j] <= col[j - 1]) { atomicAdd(bad, 1ull); break; }
+    }
+}
+
+// max of a non-negative int64 array
+__global__ void k_max_i64(long long n, const int64_t* __restrict__ x, ull* __restrict__ out) {
+    ull m = 0;
+    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
+        m = (ull)x[i] > m ? (ull)x[i] : m;
+    for (int o = 16; o > 0; o >>= 1) {
+        ull y = __shfl_xor_sync(FULLMASK, m, o);
+        m = y > m ? y : m;
+    }
+    if (lane_id() == 0 && m) atomicMax(out, m);
 }
 
 // max row length of the coarse graph

