@@ -243,7 +243,10 @@ def main():
     value = edges / total_s / 1e9
 
     # dominant kernel (by device time) roofline
-    dom = max(kstats.items(), key=lambda kv: kv[1]["ms"]) if kstats else None
+    # dominant single-kernel class of the phase-1 hot path (phase2 / level_init are multi-kernel
+    # regions with host syncs, reported in kernels_ms_per_step only)
+    cand = {k: v for k, v in kstats.items() if k not in ("phase2", "level_init") and v["alg_bytes"] > 0}
+    dom = max(cand.items(), key=lambda kv: kv[1]["ms"]) if cand else None
     roofline = None
     if dom and dom[1]["ms"] > 0:
         name, ks = dom
