@@ -34,6 +34,20 @@ struct IterCounters {
     ull delta_used;         // 1 if the delta d' update ran this iteration
 };
 
+// Queue record of an active vertex, written by k_prune_bin (which already
+// reads these fields) so the decide kernels start from one coalesced 48-byte
+// load instead of a chain of dependent gathers.
+struct __align__(16) QRec {
+    int v;          // vertex
+    int deg;        // row length
+    long long beg;  // row_ptr[v]
+    int cv;         // C[v]
+    int szv;        // size[C[v]]
+    long long dv;   // d(v)
+    long long sigv; // Sigma_tot[C[v]]
+    long long pad;
+};
+
 // Device-resident state carried across iterations of a level.
 struct Carry {
     long long N_hi;         // current numerator N (int128 split)

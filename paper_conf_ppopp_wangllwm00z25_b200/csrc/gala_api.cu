@@ -225,7 +225,7 @@ struct Work {
     cudaStream_t st;
     int64_t ncap, nnzcap;
     int32_t *C = nullptr, *size = nullptr, *stamp = nullptr, *mv_v = nullptr, *mv_old = nullptr, *nextC = nullptr;
-    int32_t* queues = nullptr;
+    QRec* queues = nullptr;
     int64_t *Sig = nullptr, *d = nullptr, *s = nullptr, *dp = nullptr;
     IterCounters* ctr = nullptr;
     Carry* carry = nullptr;
@@ -280,11 +280,13 @@ static void launch_single(gala_graph_s* g, Work& wk, const DecideArgs& a, typena
     for (int b = 0; b < NBINS; ++b) {
         if (b > BIN_S32 && maxdeg <= g->bins[b - 1]) break;
         cudaEvent_t e = tm.begin();
-        const int32_t* q = wk.queues + b * qs;
+        const QRec* q = wk.queues + b * qs;
+        // G lanes per vertex with 4 row entries per lane in flight: G ~ deg / 4
         switch (b) {
-            case BIN_S4: k_decide_single<4, M, UNIT><<<grid, 256, 0, st>>>(q, b, a, qW, p); break;
-            case BIN_S8: k_decide_single<8, M, UNIT><<<grid, 256, 0, st>>>(q, b, a, qW, p); break;
-            case BIN_S16: k_decide_single<16, M, UNIT><<<grid, 256, 0, st>>>(q, b, a, qW, p); break;
+            case BIN_S4: k_decide_single<1, M, UNIT><<<grid, 256, 0, st>>>(q, b, a, qW, p); break;
+            case BIN_S8: k_decide_single<2, M, UNIT><<<grid, 256, 0, st>>>(q, b, a, qW, p); break;
+            case BIN_S16: k_decide_single<4, M, UNIT><<<grid, 256, 0, st>>>(q, b, a, qW, p); break;
+            case BIN_S32: k_decide_single<8, M, UNIT><<<grid, 256, 0, st>>>(q, b, a, qW, p); break;
             default: k_decide_single<32, M, UNIT><<<grid, 256, 0, st>>>(q, b, a, qW, p); break;
         }
         CKL();
@@ -357,7 +359,7 @@ static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, typename
     BinThresholds th;
     for (int i = 0; i < NBINS - 1; ++i) th.t[i] = g->bins[i];
     k_prune_bin<typename ModeT<M>::ST><<<grid_for((n + PB_IPT - 1) / PB_IPT, PB_BT, big), PB_BT, 0, st>>>(
-        n, G.rp, wk.d, wk.dp, wk.C, wk.Sig, g->opt_prune, qW, p, wk.carry, wk.ctr, wk.queues, wk.ncap, th);
+        n, G.rp, wk.d, wk.dp, wk.C, wk.Sig, wk.size, g->opt_prune, qW, p, wk.carry, wk.ctr, wk.queues, wk.ncap, th);
     CKL();
     tm.end(KC_PRUNE, e);
     launch_decide<M, UNIT>(g, wk, G, qW, p, tm, maxdeg, idbits, single);
@@ -690,7 +692,7 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
             wk.mv_v = dalloc<int32_t>(wk.ncap, st);
             wk.mv_old = dalloc<int32_t>(wk.ncap, st);
             wk.nextC = dalloc<int32_t>(wk.ncap, st);
-            wk.queues = dalloc<int32_t>((size_t)wk.ncap * NBINS, st);
+            wk.queues = dalloc<QRec>((size_t)wk.ncap * NBINS, st);
             wk.Sig = dalloc<int64_t>(wk.ncap, st);
             wk.d = dalloc<int64_t>(wk.ncap, st);
             wk.s = dalloc<int64_t>(wk.ncap, st);

@@ -69,13 +69,13 @@ __device__ __forceinline__ ST gain(ST qW, ST p, long long wc, long long sig, lon
 }
 
 template <typename ST, typename A>
-__device__ __forceinline__ int decide_final(int cv, long long dv, long long own, long long sig_cv, const A& best,
-                                            const int32_t* __restrict__ size, ST qW, ST p) {
+__device__ __forceinline__ int decide_final(int cv, int szv, long long dv, long long own, long long sig_cv,
+                                            const A& best, const int32_t* __restrict__ size, ST qW, ST p) {
     ST stay = qW * (ST)own - p * (ST)(sig_cv - dv) * (ST)dv;
     int tgt = cv;
     if (best.valid() && best.score() > stay) {          // strictly better than staying (c4)
         tgt = best.comm();
-        if (size[tgt] == 1 && size[cv] == 1 && tgt > cv) tgt = cv;   // swap suppression (c5)
+        if (szv == 1 && tgt > cv && size[tgt] == 1) tgt = cv;   // swap suppression (c5)
     }
     return tgt;
 }
@@ -104,7 +104,7 @@ struct DecideArgs {
 // iteration with all their loads issued before use.
 // ---------------------------------------------------------------------------
 template <int G, int U, int M, bool UNIT>
-__global__ void __launch_bounds__(256) k_decide_sub(const int32_t* __restrict__ queue, int bin, DecideArgs a,
+__global__ void __launch_bounds__(256) k_decide_sub(const QRec* __restrict__ queue, int bin, DecideArgs a,
                                                     typename ModeT<M>::ST qW, typename ModeT<M>::ST p) {
     typedef typename ModeT<M>::ST ST;
     typedef typename ModeT<M>::VT VT;
@@ -119,36 +119,27 @@ __global__ void __launch_bounds__(256) k_decide_sub(const int32_t* __restrict__ 
     unsigned my_k = 0;
     for (long long base = ((long long)blockIdx.x * (blockDim.x >> 5) + wib) * per; base < count;
          base += nwarps * per) {
-        int v[U], deg[U], cv[U], u[U], cu[U];
-        int64_t beg[U];
-        long long dv[U], wt[U];
+        QRec q[U];
+        int u[U], cu[U];
+        long long wt[U];
         bool valid[U], has[U];
 #pragma unroll
         for (int k = 0; k < U; ++k) {
             long long i = base + (long long)k * (32 / G) + gid;
             valid[k] = i < count;
-            v[k] = valid[k] ? queue[i] : 0;
+            if (valid[k]) q[k] = queue[i];
+            else { q[k].v = 0; q[k].deg = 0; q[k].beg = 0; q[k].cv = -2; q[k].szv = 0; q[k].dv = 0; q[k].sigv = 0; }
         }
 #pragma unroll
         for (int k = 0; k < U; ++k) {
-            beg[k] = valid[k] ? a.rp[v[k]] : 0;
-            int64_t e = valid[k] ? a.rp[v[k] + 1] : 0;
-            deg[k] = (int)(e - beg[k]);
-            cv[k] = valid[k] ? a.C[v[k]] : -2;
-            dv[k] = valid[k] ? a.d[v[k]] : 0;
+            has[k] = valid[k] && gl < q[k].deg;
+            u[k] = has[k] ? a.col[q[k].beg + gl] : -1;
+            wt[k] = (has[k] && !UNIT) ? a.w[q[k].beg + gl] : 1;
         }
 #pragma unroll
         for (int k = 0; k < U; ++k) {
-            has[k] = valid[k] && gl < deg[k];
-            u[k] = has[k] ? a.col[beg[k] + gl] : -1;
-            wt[k] = (has[k] && !UNIT) ? a.w[beg[k] + gl] : 1;
-        }
-        long long sigv[U];
-#pragma unroll
-        for (int k = 0; k < U; ++k) {
-            if (u[k] == v[k]) has[k] = false;                 // self loop is not a neighbour
+            if (u[k] == q[k].v) has[k] = false;               // self loop is not a neighbour
             cu[k] = has[k] ? a.C[u[k]] : (-1 - lane);         // unique sentinel per empty lane
-            sigv[k] = (valid[k] && gl == 0) ? a.Sig[cv[k]] : 0;
         }
         unsigned peers[U];
         bool isL[U];
@@ -157,7 +148,7 @@ __global__ void __launch_bounds__(256) k_decide_sub(const int32_t* __restrict__ 
         for (int k = 0; k < U; ++k) {
             peers[k] = __match_any_sync(FULLMASK, cu[k]) & gmask;
             isL[k] = has[k] && lane == __ffs(peers[k]) - 1;
-            sig[k] = (isL[k] && cu[k] != cv[k]) ? a.Sig[cu[k]] : 0;
+            sig[k] = (isL[k] && cu[k] != q[k].cv) ? a.Sig[cu[k]] : 0;
         }
         int tgt[U];
 #pragma unroll
@@ -165,28 +156,28 @@ __global__ void __launch_bounds__(256) k_decide_sub(const int32_t* __restrict__ 
             long long wc, own;
             if (UNIT) {
                 wc = __popc(peers[k]);
-                own = __popc(__ballot_sync(FULLMASK, has[k] && cu[k] == cv[k]) & gmask);
+                own = __popc(__ballot_sync(FULLMASK, has[k] && cu[k] == q[k].cv) & gmask);
             } else {
                 wc = (long long)group_sum(peers[k], has[k] ? (VT)wt[k] : (VT)0, s_acc[wib]);
-                unsigned om = __ballot_sync(FULLMASK, isL[k] && cu[k] == cv[k]) & gmask;
+                unsigned om = __ballot_sync(FULLMASK, isL[k] && cu[k] == q[k].cv) & gmask;
                 long long wl = __shfl_sync(FULLMASK, wc, om ? __ffs(om) - 1 : 0);
                 own = om ? wl : 0;
             }
             my_k += isL[k];
             Arg<ST, ModeT<M>::PK> best;
             best.init(a.idbits, a.idmask);
-            if (isL[k] && cu[k] != cv[k]) best.offer(gain<ST>(qW, p, wc, sig[k], dv[k]), cu[k]);
+            if (isL[k] && cu[k] != q[k].cv) best.offer(gain<ST>(qW, p, wc, sig[k], q[k].dv), cu[k]);
 #pragma unroll
             for (int off = G / 2; off > 0; off >>= 1) best.xor_merge(off);
-            tgt[k] = cv[k];
+            tgt[k] = q[k].cv;
             if (valid[k] && lane == glead) {
-                if (a.check && own != a.dp[v[k]]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
-                tgt[k] = decide_final<ST>(cv[k], dv[k], own, sigv[k], best, a.size, qW, p);
+                if (a.check && own != a.dp[q[k].v]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
+                tgt[k] = decide_final<ST>(q[k].cv, q[k].szv, q[k].dv, own, q[k].sigv, best, a.size, qW, p);
             }
         }
 #pragma unroll
         for (int k = 0; k < U; ++k)
-            if (valid[k] && gl == 0) a.nextC[v[k]] = tgt[k];
+            if (valid[k] && gl == 0) a.nextC[q[k].v] = tgt[k];
     }
     ull k = block_sum_ull<256>((ull)my_k);
     if (threadIdx.x == 0 && k) atomicAdd(&a.ctr->bin_k[bin], k);
@@ -234,7 +225,7 @@ struct WarpSmem {
 };
 
 template <int MAXDEG, int M, bool UNIT>
-__global__ void __launch_bounds__(32 * WarpSmem<MAXDEG, M>::WPB) k_decide_warp(const int32_t* __restrict__ queue,
+__global__ void __launch_bounds__(32 * WarpSmem<MAXDEG, M>::WPB) k_decide_warp(const QRec* __restrict__ queue,
                                                                               int bin, DecideArgs a,
                                                                               typename ModeT<M>::ST qW,
                                                                               typename ModeT<M>::ST p) {
@@ -260,15 +251,15 @@ __global__ void __launch_bounds__(32 * WarpSmem<MAXDEG, M>::WPB) k_decide_warp(c
     const long long nwarps = (long long)gridDim.x * SM::WPB;
     unsigned my_k = 0;
     long long i = (long long)blockIdx.x * SM::WPB + wib;
-    int v = i < count ? queue[i] : 0;
+    QRec qn;
+    if (i < count) qn = queue[i];
     for (; i < count; i += nwarps) {
-        int64_t beg = a.rp[v];
-        int deg = (int)(a.rp[v + 1] - beg);
-        int cv = a.C[v];
-        long long dv = a.d[v];
-        long long inext = i + nwarps;
-        int vnext = inext < count ? queue[inext] : 0;          // prefetch the next queue entry
-        long long sig_cv = lane == 0 ? a.Sig[cv] : 0;
+        const QRec q = qn;
+        const int v = q.v, deg = q.deg, cv = q.cv;
+        const int64_t beg = q.beg;
+        const long long dv = q.dv, sig_cv = q.sigv;
+        const long long inext = i + nwarps;
+        if (inext < count) qn = queue[inext];                 // prefetch the next record
         for (int r0 = 0; r0 < deg; r0 += 32 * CH) {          // warp-uniform rounds
             int uu[CH];
             VT ww[CH];
@@ -333,10 +324,9 @@ __global__ void __launch_bounds__(32 * WarpSmem<MAXDEG, M>::WPB) k_decide_warp(c
         own = warp_sum_ll(own);
         if (lane == 0) {
             if (a.check && own != a.dp[v]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
-            a.nextC[v] = decide_final<ST>(cv, dv, own, sig_cv, best, a.size, qW, p);
+            a.nextC[v] = decide_final<ST>(cv, q.szv, dv, own, sig_cv, best, a.size, qW, p);
         }
         __syncwarp();
-        v = vnext;
     }
     ull k = block_sum_ull<32 * SM::WPB>((ull)my_k);
     if (threadIdx.x == 0 && k) atomicAdd(&a.ctr->bin_k[bin], k);
@@ -353,7 +343,7 @@ __global__ void __launch_bounds__(32 * WarpSmem<MAXDEG, M>::WPB) k_decide_warp(c
 // ---------------------------------------------------------------------------
 #define HWIN 16
 template <int BT, int E, int M, bool UNIT>
-__global__ void __launch_bounds__(BT) k_decide_block(const int32_t* __restrict__ queue, int bin, DecideArgs a,
+__global__ void __launch_bounds__(BT) k_decide_block(const QRec* __restrict__ queue, int bin, DecideArgs a,
                                                      typename ModeT<M>::ST qW, typename ModeT<M>::ST p, int smem_cap,
                                                      int* __restrict__ gkeys_all, ull* __restrict__ gvals_all,
                                                      int* __restrict__ glist_all, long long gcap) {
@@ -383,9 +373,9 @@ __global__ void __launch_bounds__(BT) k_decide_block(const int32_t* __restrict__
         __syncthreads();
         long long i = s_item;
         if (i >= count) break;
-        int v = queue[i];
-        int64_t beg = a.rp[v];
-        int deg = (int)(a.rp[v + 1] - beg);
+        const QRec q = queue[i];
+        const int v = q.v, deg = q.deg;
+        const int64_t beg = q.beg;
         int win = (smem_cap >= 2 * deg) ? smem_cap : HWIN;    // fits at load <= 1/2: never spills
         long long gc = 64;
         while (gc < 2LL * deg && gc < gcap) gc <<= 1;
@@ -420,8 +410,8 @@ __global__ void __launch_bounds__(BT) k_decide_block(const int32_t* __restrict__
         }
         __syncthreads();
         const int m = s_cnt, gm = s_gcnt;
-        const int cv = a.C[v];
-        const long long dv = a.d[v];
+        const int cv = q.cv;
+        const long long dv = q.dv;
         A best;
         best.init(a.idbits, a.idmask);
         long long own = 0;
@@ -473,7 +463,7 @@ __global__ void __launch_bounds__(BT) k_decide_block(const int32_t* __restrict__
             own = warp_sum_ll(own);
             if (lane == 0) {
                 if (a.check && own != a.dp[v]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
-                a.nextC[v] = decide_final<ST>(cv, dv, own, a.Sig[cv], best, a.size, qW, p);
+                a.nextC[v] = decide_final<ST>(cv, q.szv, dv, own, q.sigv, best, a.size, qW, p);
                 s_cnt = 0;
                 s_gcnt = 0;
             }
@@ -494,7 +484,7 @@ __global__ void __launch_bounds__(BT) k_decide_block(const int32_t* __restrict__
 //   vertex stream the row, 4 entries per lane in flight.
 // ---------------------------------------------------------------------------
 template <int G, int M, bool UNIT>
-__global__ void __launch_bounds__(256) k_decide_single(const int32_t* __restrict__ queue, int bin, DecideArgs a,
+__global__ void __launch_bounds__(256) k_decide_single(const QRec* __restrict__ queue, int bin, DecideArgs a,
                                                        typename ModeT<M>::ST qW, typename ModeT<M>::ST p) {
     typedef typename ModeT<M>::ST ST;
     const int lane = lane_id(), wib = threadIdx.x >> 5;
@@ -506,10 +496,12 @@ __global__ void __launch_bounds__(256) k_decide_single(const int32_t* __restrict
     for (long long base = ((long long)blockIdx.x * (blockDim.x >> 5) + wib) * per; base < count; base += nwarps * per) {
         const long long i = base + gid;
         const bool valid = i < count;
-        const int v = valid ? queue[i] : 0;
-        const int64_t beg = valid ? a.rp[v] : 0;
-        const int deg = valid ? (int)(a.rp[v + 1] - beg) : 0;
-        const long long dv = valid ? a.d[v] : 0;
+        QRec q;
+        if (valid) q = queue[i];
+        const int v = valid ? q.v : 0;
+        const int64_t beg = valid ? q.beg : 0;
+        const int deg = valid ? q.deg : 0;
+        const long long dv = valid ? q.dv : 0;
         Arg<ST, ModeT<M>::PK> best;
         best.init(a.idbits, a.idmask);
         int dmax = deg;   // warp-uniform round count: max row length of the warp's groups

@@ -95,9 +95,9 @@ template <typename ST>
 __global__ void __launch_bounds__(PB_BT) k_prune_bin(int n, const int64_t* __restrict__ rp,
                                                      const int64_t* __restrict__ d, const int64_t* __restrict__ dp,
                                                      const int32_t* __restrict__ C, const int64_t* __restrict__ Sig,
-                                                     int prune, ST qW, ST p, const Carry* __restrict__ carry,
-                                                     IterCounters* __restrict__ ctr, int32_t* __restrict__ queues,
-                                                     long long qstride, BinThresholds th) {
+                                                     const int32_t* __restrict__ size, int prune, ST qW, ST p,
+                                                     const Carry* __restrict__ carry, IterCounters* __restrict__ ctr,
+                                                     QRec* __restrict__ queues, long long qstride, BinThresholds th) {
     __shared__ unsigned s_cnt[NBINS];
     __shared__ ull s_base[NBINS];
     const long long minSig = carry->minSig;
@@ -121,13 +121,15 @@ __global__ void __launch_bounds__(PB_BT) k_prune_bin(int n, const int64_t* __res
         }
         long long sg[PB_IPT];
 #pragma unroll
-        for (int j = 0; j < PB_IPT; ++j) sg[j] = (prune && dv[j] > 0) ? Sig[cv[j]] : 0;
+        for (int j = 0; j < PB_IPT; ++j) sg[j] = dv[j] > 0 ? Sig[cv[j]] : 0;
         int deg[PB_IPT];
+        long long beg[PB_IPT];
 #pragma unroll
         for (int j = 0; j < PB_IPT; ++j) {
             long long v = t0 + (long long)j * PB_BT + threadIdx.x;
             bin[j] = -1;
             deg[j] = 0;
+            beg[j] = 0;
             if (dv[j] > 0) {
                 bool active = true;
                 if (prune) {
@@ -135,7 +137,8 @@ __global__ void __launch_bounds__(PB_BT) k_prune_bin(int n, const int64_t* __res
                     active = lhs < (ST)0;
                 }
                 if (active) {
-                    long long dg = rp[v + 1] - rp[v];
+                    beg[j] = rp[v];
+                    long long dg = rp[v + 1] - beg[j];
                     deg[j] = (int)(dg > INT_MAX ? INT_MAX : dg);
                     int b = NBINS - 1;
 #pragma unroll
@@ -149,6 +152,9 @@ __global__ void __launch_bounds__(PB_BT) k_prune_bin(int n, const int64_t* __res
                 }
             }
         }
+        int szv[PB_IPT];
+#pragma unroll
+        for (int j = 0; j < PB_IPT; ++j) szv[j] = bin[j] >= 0 ? size[cv[j]] : 0;
         __syncthreads();   // s_cnt reset visible
         unsigned off[PB_IPT];
 #pragma unroll
@@ -167,8 +173,16 @@ __global__ void __launch_bounds__(PB_BT) k_prune_bin(int n, const int64_t* __res
 #pragma unroll
         for (int j = 0; j < PB_IPT; ++j) {
             if (bin[j] >= 0) {
-                long long v = t0 + (long long)j * PB_BT + threadIdx.x;
-                queues[(long long)bin[j] * qstride + (long long)s_base[bin[j]] + off[j]] = (int32_t)v;
+                QRec q;
+                q.v = (int)(t0 + (long long)j * PB_BT + threadIdx.x);
+                q.deg = deg[j];
+                q.beg = beg[j];
+                q.cv = cv[j];
+                q.szv = szv[j];
+                q.dv = dv[j];
+                q.sigv = sg[j];
+                q.pad = 0;
+                queues[(long long)bin[j] * qstride + (long long)s_base[bin[j]] + off[j]] = q;
             }
         }
     }
@@ -190,7 +204,7 @@ __global__ void __launch_bounds__(PB_BT) k_prune_bin(int n, const int64_t* __res
 // one global atomic per block and tile.
 // ---------------------------------------------------------------------------
 #define AP_BT 256
-__global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr, const int32_t* __restrict__ queues,
+__global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr, const QRec* __restrict__ queues,
                                                  long long qstride, const int32_t* __restrict__ nextC,
                                                  int32_t* __restrict__ C, int64_t* __restrict__ Sig,
                                                  int32_t* __restrict__ size, const int64_t* __restrict__ d,
@@ -215,19 +229,20 @@ __global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr,
 #pragma unroll
             for (int k = 0; k < NBINS - 1; ++k)
                 if (b == k && r >= cnt[k]) { r -= cnt[k]; b = k + 1; }
-            v = queues[(long long)b * qstride + r];
+            const QRec q = queues[(long long)b * qstride + r];
+            v = q.v;
             int nc = nextC[v];
-            oc = C[v];
+            oc = q.cv;
             if (nc != oc) {
                 mover = true;
-                long long dv = d[v];
+                long long dv = q.dv;
                 C[v] = nc;
                 stamp[v] = iter_id;
                 atomicAdd(reinterpret_cast<ull*>(&Sig[oc]), (ull)(-dv));
                 atomicAdd(reinterpret_cast<ull*>(&Sig[nc]), (ull)dv);
                 atomicSub(&size[oc], 1);
                 atomicAdd(&size[nc], 1);
-                my_deg += (ull)(rp[v + 1] - rp[v]);
+                my_deg += (ull)q.deg;
             }
         }
         if (threadIdx.x == 0) s_cnt = 0;
