@@ -74,7 +74,8 @@ struct DevCSR {
     int64_t n = 0, nnz = 0;
     int64_t* rp = nullptr;
     int32_t* col = nullptr;
-    int64_t* w = nullptr;   // nullptr = unit weights
+    int64_t* w = nullptr;     // nullptr = unit weights
+    int32_t* row = nullptr;   // row (source vertex) of every entry, for edge-parallel passes
 };
 
 struct LevelStat {
@@ -372,7 +373,10 @@ static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, typename
     k_dp_delta<UNIT><<<big, 256, 0, st>>>(wk.ctr, G.rp, G.col, G.w, wk.C, wk.mv_v, wk.mv_old, wk.stamp, wk.dp,
                                           wk.carry, G.nnz, g->opt_delta, 1, 2);
     CKL();
-    k_dp_full<UNIT><<<big, 256, 0, st>>>(wk.ctr, n, G.rp, G.col, G.w, wk.C, wk.dp, G.nnz, g->opt_delta, 1, 2, 0);
+    k_dp_zero<<<big, 256, 0, st>>>(wk.ctr, n, wk.dp, G.nnz, g->opt_delta, 1, 2);
+    CKL();
+    k_dp_full<UNIT><<<grid_for((G.nnz + 127) / 128 * 32, 256, big), 256, 0, st>>>(wk.ctr, G.nnz, G.row, G.col, G.w,
+                                                                                 wk.C, wk.dp, g->opt_delta, 1, 2);
     CKL();
     tm.end(KC_DP, e);
     e = tm.begin();
@@ -516,10 +520,8 @@ static void coarsen(gala_graph_s* g, Work& wk, const DevCSR& cur, int64_t nl, lo
     const int big = g->num_sms * 8;
     long long* cnt = dalloc<long long>(k + 1, st);
     long long* ent = dalloc<long long>(k + 1, st);
-    long long* moff = dalloc<long long>(k + 1, st);
     long long* eoff = dalloc<long long>(k + 1, st);
     long long* dn = dalloc<long long>(k + 1, st);
-    int32_t* mem = dalloc<int32_t>(nl, st);
     int* tkey = dalloc<int>(cur.nnz, st);
     int64_t* tval = dalloc<int64_t>(cur.nnz, st);
     int64_t* snew = dalloc<int64_t>(k, st);
@@ -534,21 +536,29 @@ static void coarsen(gala_graph_s* g, Work& wk, const DevCSR& cur, int64_t nl, lo
     CK(cudaMemsetAsync(snew, 0, sizeof(int64_t) * k, st));
     CK(cudaMemsetAsync(dev_max, 0, sizeof(ull) * 2, st));
     CK(cudaMemsetAsync(nbig_dev, 0, sizeof(int), st));
-    k_comm_stats<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, cur.rp, newid, cnt, ent);
+    k_comm_stats<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, cur.rp, newid, ent);
     CKL();
-    scan_excl(cnt, moff, k, st);
     scan_excl(ent, eoff, k, st);
-    CK(cudaMemsetAsync(cnt, 0, sizeof(long long) * (k + 1), st));   // reuse as member cursor
-    k_members<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, newid, moff, cnt, mem);
+    // segment position of every row (cnt reused as the per-community cursor), then an
+    // edge-parallel copy of the coarse keys into the segments
+    long long* vpos = dalloc<long long>(nl, st);
+    k_vpos<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, cur.rp, newid, eoff, cnt, vpos);
     CKL();
+    if (unit)
+        k_gather_flat<true><<<grid_for((cur.nnz + 127) / 128 * 32, 256, big), 256, 0, st>>>(
+            cur.nnz, cur.row, cur.rp, cur.col, cur.w, newid, vpos, tkey, tval);
+    else
+        k_gather_flat<false><<<grid_for((cur.nnz + 127) / 128 * 32, 256, big), 256, 0, st>>>(
+            cur.nnz, cur.row, cur.rp, cur.col, cur.w, newid, vpos, tkey, tval);
+    CKL();
+    dfree(vpos, st);
     // shared-memory capacity of the block path: up to 8192 slots (14 B each)
     int scap = 512;
     while (scap < 8192 && scap < 2 * k) scap <<= 1;
     k_agg_bigflag<<<grid_for(k, 256, big), 256, 0, st>>>(k, ent, scap, bigc, bigcap, nbig_dev);
     CKL();
     AggArgs a;
-    a.k = k; a.ent = ent; a.eoff = eoff; a.moff = moff; a.mem = mem; a.rp = cur.rp; a.col = cur.col; a.w = cur.w;
-    a.newid = newid; a.tkey = tkey; a.tval = tval; a.dn = dn; a.snew = snew;
+    a.k = k; a.ent = ent; a.eoff = eoff; a.tkey = tkey; a.tval = tval; a.dn = dn; a.snew = snew;
     if (unit) k_agg_warp<true><<<big, 256, 0, st>>>(a);
     else k_agg_warp<false><<<big, 256, 0, st>>>(a);
     CKL();
@@ -556,7 +566,7 @@ static void coarsen(gala_graph_s* g, Work& wk, const DevCSR& cur, int64_t nl, lo
         const size_t sm = agg_block_smem(scap);
         CK(cudaFuncSetAttribute(k_agg_block<AGG_BLOCK_BT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
         CK(cudaFuncSetAttribute(k_agg_block<AGG_BLOCK_BT, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
-        const int gb = (int)std::min<long long>(k, (long long)g->num_sms * 2);
+        const int gb = (int)std::min<long long>(k, (long long)g->num_sms * 4);
         if (unit) k_agg_block<AGG_BLOCK_BT, true><<<gb, AGG_BLOCK_BT, sm, st>>>(a, scap);
         else k_agg_block<AGG_BLOCK_BT, false><<<gb, AGG_BLOCK_BT, sm, st>>>(a, scap);
         CKL();
@@ -603,14 +613,15 @@ static void coarsen(gala_graph_s* g, Work& wk, const DevCSR& cur, int64_t nl, lo
     dmax = (int64_t)hm[1];
     nxt.col = dalloc<int32_t>(nxt.nnz, st);
     nxt.w = dalloc<int64_t>(nxt.nnz, st);
+    nxt.row = dalloc<int32_t>(nxt.nnz, st);
     k_compact<<<grid_for(k * 32, 256, big), 256, 0, st>>>(k, eoff, reinterpret_cast<long long*>(nxt.rp), tkey, tval,
-                                                          nxt.col, nxt.w);
+                                                          nxt.col, nxt.w, nxt.row);
     CKL();
     CK(cudaMemcpyAsync(wk.d, dnew, sizeof(int64_t) * k, cudaMemcpyDeviceToDevice, st));
     CK(cudaMemcpyAsync(wk.s, snew, sizeof(int64_t) * k, cudaMemcpyDeviceToDevice, st));
     g->kc_bytes[KC_PHASE2] += (double)nl * (4 + 4 + 8 + 16 + 4 + 4) + (double)cur.nnz * (4 + 4 + (unit ? 0 : 8) + 12) +
                               (double)nxt.nnz * 24;
-    dfree(cnt, st); dfree(ent, st); dfree(moff, st); dfree(eoff, st); dfree(dn, st); dfree(mem, st);
+    dfree(cnt, st); dfree(ent, st); dfree(eoff, st); dfree(dn, st);
     dfree(tkey, st); dfree(tval, st); dfree(snew, st); dfree(dnew, st); dfree(dev_max, st); dfree(bigc, st);
     dfree(bigcap, st); dfree(nbig_dev, st);
 }
@@ -865,7 +876,7 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
             ls.ms_phase1 = ms1;
             ls.ms_phase2 = ms2;
             g->levels.push_back(ls);
-            if (cur_owned) { dfree(cur.rp, st); dfree(cur.col, st); dfree(cur.w, st); }
+            if (cur_owned) { dfree(cur.rp, st); dfree(cur.col, st); dfree(cur.w, st); dfree(cur.row, st); }
             if (stop) break;
             cur = nxt;
             cur_owned = true;
@@ -922,6 +933,9 @@ static void finish_graph(gala_graph_s* g) {
     const int64_t n = g->n0;
     g->d0 = dalloc<int64_t>(n, st);
     g->s0 = dalloc<int64_t>(n, st);
+    g->g0.row = dalloc<int32_t>(g->g0.nnz, st);
+    k_fill_rows<<<grid_for(n * 32, 256, g->num_sms * 8), 256, 0, st>>>((int)n, g->g0.rp, g->g0.row);
+    CKL();
     ull* mx = dalloc<ull>(1, st);
     CK(cudaMemsetAsync(mx, 0, sizeof(ull), st));
     int grid = grid_for(n * 32, 256, g->num_sms * 8);
@@ -1189,6 +1203,7 @@ void gala_graph_free(gala_graph g) {
         dfree(g->g0.rp, st);
         dfree(g->g0.col, st);
         dfree(g->g0.w, st);
+        dfree(g->g0.row, st);
         dfree(g->d0, st);
         dfree(g->s0, st);
         dfree(g->lab, st);

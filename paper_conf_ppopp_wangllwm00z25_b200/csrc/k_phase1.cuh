@@ -313,40 +313,52 @@ __global__ void __launch_bounds__(256) k_dp_delta(IterCounters* __restrict__ ctr
     }
 }
 
-// d'(v) = sum of w(v,u), u != v, C[u] == C[v]   (definition; 8 lanes per vertex)
+// d'(v) = sum of w(v,u), u != v, C[u] == C[v]   (definition), edge-parallel:
+// every lane takes entries (row r, col u) 32 apart (4 in flight), equal rows of
+// a 32-entry chunk are summed with __match_any_sync and one atomic per row.
+__global__ void k_dp_zero(IterCounters* __restrict__ ctr, int n, int64_t* __restrict__ dp, long long nnz, int mode,
+                          long long fnum, long long fden) {
+    if (use_delta(ctr, nnz, mode, fnum, fden)) return;
+    for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x)
+        dp[v] = 0;
+}
+
 template <bool UNIT>
-__global__ void __launch_bounds__(256) k_dp_full(IterCounters* __restrict__ ctr, int n,
-                                                 const int64_t* __restrict__ rp, const int32_t* __restrict__ col,
+__global__ void __launch_bounds__(256) k_dp_full(IterCounters* __restrict__ ctr, long long nnz,
+                                                 const int32_t* __restrict__ row, const int32_t* __restrict__ col,
                                                  const int64_t* __restrict__ w, const int32_t* __restrict__ C,
-                                                 int64_t* __restrict__ dp, long long nnz, int mode, long long fnum,
-                                                 long long fden, int force) {
-    if (!force && use_delta(ctr, nnz, mode, fnum, fden)) return;
-    const int lane = lane_id(), gl = lane & 7;
-    const long long ngroups = ((long long)gridDim.x * blockDim.x) >> 3;
-    for (long long base = ((long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31)) >> 3; base < n;
-         base += ngroups) {
-        long long v = base + (lane >> 3);
-        long long acc = 0;
-        if (v < n) {
-            int cv = C[v];
-            int64_t b = rp[v], e = rp[v + 1];
-            int64_t j = b + gl;
-            for (; j + 8 < e; j += 16) {    // two entries per lane in flight
-                int x0 = col[j], x1 = col[j + 8];
-                long long w0 = UNIT ? 1 : w[j], w1 = UNIT ? 1 : w[j + 8];
-                int c0 = C[x0], c1 = C[x1];
-                if (x0 != v && c0 == cv) acc += w0;
-                if (x1 != v && c1 == cv) acc += w1;
-            }
-            if (j < e) {
-                int x = col[j];
-                if (x != v && C[x] == cv) acc += UNIT ? 1 : w[j];
-            }
+                                                 int64_t* __restrict__ dp, int mode, long long fnum, long long fden) {
+    __shared__ ull s_scr[8][32];
+    if (use_delta(ctr, nnz, mode, fnum, fden)) return;
+    const int lane = lane_id(), wib = threadIdx.x >> 5;
+    const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+    for (long long base = (((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * 128; base < nnz;
+         base += nw * 128) {
+        int r[4], u[4];
+        long long wt[4];
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+            long long e = base + lane + 32 * t;
+            r[t] = e < nnz ? row[e] : -1;
+            u[t] = e < nnz ? col[e] : -1;
+            wt[t] = (e < nnz && !UNIT) ? w[e] : 1;
         }
-        acc += __shfl_xor_sync(FULLMASK, acc, 4);
-        acc += __shfl_xor_sync(FULLMASK, acc, 2);
-        acc += __shfl_xor_sync(FULLMASK, acc, 1);
-        if (v < n && gl == 0) dp[v] = acc;
+        int cr[4], cu[4];
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+            cr[t] = r[t] >= 0 ? C[r[t]] : 0;
+            cu[t] = u[t] >= 0 ? C[u[t]] : 1;
+        }
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+            const bool hit = r[t] >= 0 && u[t] != r[t] && cu[t] == cr[t];
+            const unsigned peers = __match_any_sync(FULLMASK, r[t]);
+            const ull x = hit ? (ull)wt[t] : 0ull;
+            ull sum;
+            if (UNIT) sum = (ull)__popc(__ballot_sync(FULLMASK, hit) & peers);
+            else sum = group_sum(peers, x, s_scr[wib]);
+            if (r[t] >= 0 && lane == __ffs(peers) - 1 && sum) atomicAdd(reinterpret_cast<ull*>(&dp[r[t]]), sum);
+        }
     }
 }
 

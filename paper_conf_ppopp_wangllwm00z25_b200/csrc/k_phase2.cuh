@@ -130,36 +130,83 @@ __global__ void k_compose(long long n0, const int32_t* __restrict__ newid, int32
 // The diagonal (internal weight D_C, reading c10) is one entry.
 // ---------------------------------------------------------------------------
 // Coarsening runs per community c' = newid of a community:
-//   1. k_comm_stats   : members and row entries per community
-//   2. k_members      : member lists (counting sort by community)
-//   3. aggregation of (newid[u], w) over the rows of c's members into a hash
-//      table keyed by coarse neighbour, by the cheapest path that fits:
+//   1. k_comm_stats  : row entries per community -> eoff (exclusive scan)
+//   2. k_gather_rows : every row's coarse keys newid[u] (and weights) are copied
+//                      into its community's contiguous segment [eoff[c'], eoff[c'+1])
+//   3. aggregation of each segment into a hash table keyed by coarse neighbour,
+//      by the cheapest path that fits:
 //        k_agg_warp  (table <= 256 slots, one warp per community),
 //        k_agg_block (table <= smem capacity, one block per community),
 //        k_agg_big_* (larger: global table shared by BPC blocks);
-//      distinct entries go to a temporary segment at eoff[c'] (its row-entry
-//      offset, an upper bound), their count to dn[c'], the diagonal to snew.
-//   4. k_compact      : segments -> coarse CSR rows (rp_new = scan of dn).
-// Per-community tables are in shared memory on the common paths: the
-// inserts are shared-memory atomics (P:304-316's point about keeping hot
-// state on chip applies to phase 2 as well).
+//      segments are read coalesced, 4 entries per lane in flight, equal keys of
+//      every 32-entry chunk combined with __match_any_sync before inserting;
+//      distinct entries are written back to the segment start, their count to
+//      dn[c'], the diagonal weight to snew[c'].
+//   4. k_compact     : segments -> coarse CSR rows (rp_new = scan of dn).
+// Tables live in shared memory on the common paths (P:304-316's point about
+// keeping hot state on chip applies to phase 2 as well).
 __global__ void k_comm_stats(int n, const int64_t* __restrict__ rp, const int32_t* __restrict__ newid,
-                             long long* __restrict__ cnt, long long* __restrict__ ent) {
+                             long long* __restrict__ ent) {
     for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x) {
-        int c = newid[v];
-        atomicAdd(reinterpret_cast<ull*>(&cnt[c]), 1ull);
         long long dg = rp[v + 1] - rp[v];
-        if (dg) atomicAdd(reinterpret_cast<ull*>(&ent[c]), (ull)dg);
+        if (dg) atomicAdd(reinterpret_cast<ull*>(&ent[newid[v]]), (ull)dg);
     }
 }
 
-__global__ void k_members(int n, const int32_t* __restrict__ newid, const long long* __restrict__ moff,
-                          long long* __restrict__ cur, int32_t* __restrict__ mem) {
+// segment position of every row: eoff[c'] + its offset among c's rows
+__global__ void k_vpos(int n, const int64_t* __restrict__ rp, const int32_t* __restrict__ newid,
+                       const long long* __restrict__ eoff, long long* __restrict__ ecur, long long* __restrict__ vpos) {
     for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x) {
-        int c = newid[v];
-        ull pos = atomicAdd(reinterpret_cast<ull*>(&cur[c]), 1ull);
-        mem[moff[c] + (long long)pos] = (int32_t)v;
+        const long long dg = rp[v + 1] - rp[v];
+        const int c = newid[v];
+        vpos[v] = dg ? eoff[c] + (long long)atomicAdd(reinterpret_cast<ull*>(&ecur[c]), (ull)dg) : 0;
     }
+}
+
+// edge-parallel: entry e of row r goes to vpos[r] + (e - rp[r]) with key newid[col[e]];
+// 4 entries per lane in flight, coalesced row/col streams
+template <bool UNIT>
+__global__ void __launch_bounds__(256) k_gather_flat(long long nnz, const int32_t* __restrict__ row,
+                                                     const int64_t* __restrict__ rp, const int32_t* __restrict__ col,
+                                                     const int64_t* __restrict__ w, const int32_t* __restrict__ newid,
+                                                     const long long* __restrict__ vpos, int* __restrict__ tkey,
+                                                     int64_t* __restrict__ tval) {
+    const int lane = lane_id();
+    const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+    for (long long base = (((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * 128; base < nnz;
+         base += nw * 128) {
+        int r[4], u[4];
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+            long long e = base + lane + 32 * t;
+            r[t] = e < nnz ? row[e] : 0;
+            u[t] = e < nnz ? col[e] : 0;
+        }
+        int kk[4];
+        long long dst[4];
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+            long long e = base + lane + 32 * t;
+            kk[t] = e < nnz ? newid[u[t]] : 0;
+            dst[t] = e < nnz ? vpos[r[t]] + (e - rp[r[t]]) : 0;
+        }
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+            long long e = base + lane + 32 * t;
+            if (e < nnz) {
+                tkey[dst[t]] = kk[t];
+                if (!UNIT) tval[dst[t]] = w[e];
+            }
+        }
+    }
+}
+
+// row id of every CSR entry (warp per row)
+__global__ void k_fill_rows(int n, const int64_t* __restrict__ rp, int32_t* __restrict__ row) {
+    const int lane = lane_id();
+    const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+    for (long long v = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5; v < n; v += nw)
+        for (int64_t j = rp[v] + lane; j < rp[v + 1]; j += 32) row[j] = (int32_t)v;
 }
 
 // table capacity a community needs: nextpow2(2 * min(entries, k)) (0 if no entries)
@@ -174,15 +221,9 @@ __device__ __forceinline__ long long agg_cap(long long ent, long long k) {
 struct AggArgs {
     long long k;
     const long long* ent;
-    const long long* eoff;     // row-entry offsets (exclusive scan of ent)
-    const long long* moff;     // member offsets
-    const int32_t* mem;
-    const int64_t* rp;
-    const int32_t* col;
-    const int64_t* w;
-    const int32_t* newid;
-    int* tkey;                 // temporary aggregated segments
-    int64_t* tval;
+    const long long* eoff;     // segment offsets (exclusive scan of ent)
+    int* tkey;                 // segments: coarse keys in, distinct keys out
+    int64_t* tval;             // weights in (weighted levels), aggregated weights out
     long long* dn;             // distinct entries per community
     int64_t* snew;             // diagonal weight per community
 };
@@ -206,39 +247,33 @@ __device__ __forceinline__ int agg_insert(int key, VT wt, int* keys, VT* vals, u
     }
 }
 
-// the warp streams the rows of its community's members (4 entries per lane in
-// flight); equal keys of each 32-entry chunk are combined before inserting.
+// `nt` threads (tid = this thread's index among them, whole warps) stream
+// segment entries [s0, s1) with 4 entries per lane in flight; equal keys of
+// every 32-entry chunk are combined before inserting.
 template <bool UNIT, typename VT>
-__device__ __forceinline__ void agg_rows_warp(const AggArgs& a, long long m0, long long m1, int lane, int* keys,
-                                              VT* vals, unsigned mask, int* list, int* cnt, int mstride,
-                                              int mfirst, ull* scratch) {
-    for (long long mi = m0 + mfirst; mi < m1; mi += mstride) {
-        int v = a.mem[mi];
-        int64_t b = a.rp[v], e = a.rp[v + 1];
-        for (int64_t r0 = b; r0 < e; r0 += 128) {          // warp-uniform rounds
-            int uu[4];
-            VT ww[4];
+__device__ __forceinline__ void agg_segment(const AggArgs& a, long long s0, long long s1, int tid, int nt, int* keys,
+                                            VT* vals, unsigned mask, int* list, int* cnt, ull* scratch) {
+    const int lane = tid & 31;
+    for (long long r0 = s0 + (tid & ~31) * 4; r0 < s1; r0 += (long long)nt * 4) {   // warp-uniform
+        int kk[4];
+        ull ww[4];
 #pragma unroll
-            for (int t = 0; t < 4; ++t) {
-                int64_t j = r0 + lane + 32 * t;
-                uu[t] = j < e ? a.col[j] : -1;
-                ww[t] = (j < e && !UNIT) ? (VT)a.w[j] : (VT)1;
-            }
-            int kk[4];
+        for (int t = 0; t < 4; ++t) {
+            long long j = r0 + lane + 32 * t;
+            kk[t] = j < s1 ? a.tkey[j] : -1;
+            ww[t] = (j < s1 && !UNIT) ? (ull)a.tval[j] : 1ull;
+        }
 #pragma unroll
-            for (int t = 0; t < 4; ++t) kk[t] = uu[t] >= 0 ? a.newid[uu[t]] : -1;
-#pragma unroll
-            for (int t = 0; t < 4; ++t) {
-                if (r0 + 32 * t >= e) break;
-                const unsigned peers = __match_any_sync(FULLMASK, kk[t] >= 0 ? kk[t] : -1 - lane);
-                const ull sum = UNIT ? (ull)__popc(peers) : group_sum(peers, kk[t] >= 0 ? (ull)ww[t] : 0ull, scratch);
-                if (kk[t] >= 0 && lane == __ffs(peers) - 1) agg_insert<VT>(kk[t], (VT)sum, keys, vals, mask, list, cnt);
-            }
+        for (int t = 0; t < 4; ++t) {
+            if (r0 + 32 * t >= s1) break;
+            const unsigned peers = __match_any_sync(FULLMASK, kk[t] >= 0 ? kk[t] : -1 - lane);
+            const ull sum = UNIT ? (ull)__popc(peers) : group_sum(peers, kk[t] >= 0 ? ww[t] : 0ull, scratch);
+            if (kk[t] >= 0 && lane == __ffs(peers) - 1) agg_insert<VT>(kk[t], (VT)sum, keys, vals, mask, list, cnt);
         }
     }
 }
 
-// write the distinct entries of community c to its temporary segment
+// write the distinct entries of community c to the start of its segment
 template <typename VT>
 __device__ __forceinline__ void agg_emit(const AggArgs& a, long long c, int m, const int* list, int* keys, VT* vals,
                                          int tid, int nt) {
@@ -275,8 +310,8 @@ __global__ void __launch_bounds__(256) k_agg_warp(AggArgs a) {
         long long cap = agg_cap(a.ent[c], a.k);
         if (cap == 0) { if (lane == 0) a.dn[c] = 0; continue; }
         if (cap > AGG_WSLOTS) continue;
-        agg_rows_warp<UNIT, ull>(a, a.moff[c], a.moff[c + 1], lane, keys, vals, (unsigned)cap - 1, list, &s_cnt[wib],
-                                 1, 0, s_scr[wib]);
+        agg_segment<UNIT, ull>(a, a.eoff[c], a.eoff[c + 1], lane, 32, keys, vals, (unsigned)cap - 1, list, &s_cnt[wib],
+                               s_scr[wib]);
         __syncwarp();
         int m = s_cnt[wib];
         agg_emit<ull>(a, c, m, list, keys, vals, lane, 32);
@@ -294,15 +329,15 @@ __global__ void __launch_bounds__(BT) k_agg_block(AggArgs a, int scap) {
     int* list = keys + scap;
     __shared__ int s_cnt;
     __shared__ ull s_scr[BT / 32][32];
-    const int lane = lane_id(), wib = threadIdx.x >> 5;
+    const int wib = threadIdx.x >> 5;
     for (int j = threadIdx.x; j < scap; j += BT) { keys[j] = -1; vals[j] = 0; }
     if (threadIdx.x == 0) s_cnt = 0;
     __syncthreads();
     for (long long c = blockIdx.x; c < a.k; c += gridDim.x) {
         long long cap = agg_cap(a.ent[c], a.k);
         if (cap <= AGG_WSLOTS || cap > scap) continue;   // block-uniform
-        agg_rows_warp<UNIT, ull>(a, a.moff[c], a.moff[c + 1], lane, keys, vals, (unsigned)cap - 1, list, &s_cnt,
-                                 BT / 32, wib, s_scr[wib]);
+        agg_segment<UNIT, ull>(a, a.eoff[c], a.eoff[c + 1], threadIdx.x, BT, keys, vals, (unsigned)cap - 1, list,
+                               &s_cnt, s_scr[wib]);
         __syncthreads();
         int m = s_cnt;
         agg_emit<ull>(a, c, m, list, keys, vals, threadIdx.x, BT);
@@ -312,21 +347,23 @@ __global__ void __launch_bounds__(BT) k_agg_block(AggArgs a, int scap) {
     }
 }
 
-// big communities: BPC blocks per community insert into its global table
+// big communities: BPC blocks per community stream chunks of its segment into its global table
 template <bool UNIT>
 __global__ void __launch_bounds__(256) k_agg_big_insert(AggArgs a, const int32_t* __restrict__ bigc, int nbig,
                                                         const long long* __restrict__ goff, int* __restrict__ gkeys,
                                                         ull* __restrict__ gvals, int* __restrict__ glist,
                                                         int* __restrict__ gcnt, int bpc) {
     __shared__ ull s_scr[8][32];
-    const int lane = lane_id(), wib = threadIdx.x >> 5;
+    const int wib = threadIdx.x >> 5;
     for (long long b = blockIdx.x; b < (long long)nbig * bpc; b += gridDim.x) {
-        int bi = (int)(b / bpc), part = (int)(b % bpc);
-        long long c = bigc[bi];
-        long long off = goff[bi];
-        unsigned mask = (unsigned)(goff[bi + 1] - off) - 1u;
-        agg_rows_warp<UNIT, ull>(a, a.moff[c], a.moff[c + 1], lane, gkeys + off, gvals + off, mask, glist + off / 2,
-                                 &gcnt[bi], bpc * 8, part * 8 + wib, s_scr[wib]);
+        const int bi = (int)(b / bpc), part = (int)(b % bpc);
+        const long long c = bigc[bi];
+        const long long off = goff[bi];
+        const unsigned mask = (unsigned)(goff[bi + 1] - off) - 1u;
+        const long long s0 = a.eoff[c], len = a.eoff[c + 1] - s0;
+        const long long lo = s0 + len * part / bpc, hi = s0 + len * (part + 1) / bpc;
+        agg_segment<UNIT, ull>(a, lo, hi, threadIdx.x, 256, gkeys + off, gvals + off, mask, glist + off / 2,
+                               &gcnt[bi], s_scr[wib]);
     }
 }
 
@@ -360,7 +397,7 @@ __global__ void k_agg_bigflag(long long k, const long long* __restrict__ ent, in
 __global__ void __launch_bounds__(256) k_compact(long long k, const long long* __restrict__ eoff,
                                                  const long long* __restrict__ rp_new, const int* __restrict__ tkey,
                                                  const int64_t* __restrict__ tval, int32_t* __restrict__ col_new,
-                                                 int64_t* __restrict__ w_new) {
+                                                 int64_t* __restrict__ w_new, int32_t* __restrict__ row_new) {
     const int lane = lane_id();
     const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
     for (long long c = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < k; c += nw) {
@@ -368,6 +405,7 @@ __global__ void __launch_bounds__(256) k_compact(long long k, const long long* _
         for (long long t = lane; t < m; t += 32) {
             col_new[r + t] = tkey[o + t];
             w_new[r + t] = tval[o + t];
+            row_new[r + t] = (int32_t)c;
         }
     }
 }
