@@ -928,63 +928,64 @@ static void init_graph_common(gala_graph_s* g, int64_t n, int device, uintptr_t 
     g_pool = g->pool;
 }
 
+// Device-side validation of the copied CSR (GALA_E_INVALID), unit-weight
+// detection, d(v), s(v), max row length, max weighted degree, W (int128-checked)
+// and the level-0 row-id array.
 static void finish_graph(gala_graph_s* g) {
     cudaStream_t st = g->stream;
     const int64_t n = g->n0;
+    const int big = g->num_sms * 8;
+    unsigned* flags = dalloc<unsigned>(1, st);
+    CK(cudaMemsetAsync(flags, 0, sizeof(unsigned), st));
+    k_validate<<<grid_for(std::max<int64_t>(n, g->g0.nnz), 256, big), 256, 0, st>>>((int)n, g->g0.nnz, g->g0.rp,
+                                                                                   g->g0.col, g->g0.w, flags);
+    CKL();
+    unsigned hf = 0;
+    CK(cudaMemcpyAsync(&hf, flags, sizeof(unsigned), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    dfree(flags, st);
+    if (hf & 1u) { set_err(GALA_E_INVALID, "row_ptr not monotone"); throw GalaError{GALA_E_INVALID}; }
+    if (hf & 2u) { set_err(GALA_E_INVALID, "col_idx out of range"); throw GalaError{GALA_E_INVALID}; }
+    if (hf & 4u) { set_err(GALA_E_INVALID, "weight <= 0"); throw GalaError{GALA_E_INVALID}; }
+    if (g->g0.w && !(hf & 8u)) dfree(g->g0.w, st);   // all weights 1: unit-weight level 0
     g->d0 = dalloc<int64_t>(n, st);
     g->s0 = dalloc<int64_t>(n, st);
     g->g0.row = dalloc<int32_t>(g->g0.nnz, st);
-    k_fill_rows<<<grid_for(n * 32, 256, g->num_sms * 8), 256, 0, st>>>((int)n, g->g0.rp, g->g0.row);
+    k_fill_rows<<<grid_for(n * 32, 256, big), 256, 0, st>>>((int)n, g->g0.rp, g->g0.row);
     CKL();
-    ull* mx = dalloc<ull>(1, st);
-    CK(cudaMemsetAsync(mx, 0, sizeof(ull), st));
-    int grid = grid_for(n * 32, 256, g->num_sms * 8);
+    ull* mx = dalloc<ull>(3, st);
+    CK(cudaMemsetAsync(mx, 0, 3 * sizeof(ull), st));
+    int grid = grid_for(n * 32, 256, big);
     if (g->g0.w == nullptr)
         k_degrees<true><<<grid, 256, 0, st>>>((int)n, g->g0.rp, g->g0.col, g->g0.w, g->d0, g->s0, mx);
     else
         k_degrees<false><<<grid, 256, 0, st>>>((int)n, g->g0.rp, g->g0.col, g->g0.w, g->d0, g->s0, mx);
     CKL();
-    ull hmx = 0;
-    CK(cudaMemcpyAsync(&hmx, mx, sizeof(ull), cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
-    g->maxdeg0 = (int64_t)hmx;
-    CK(cudaMemsetAsync(mx, 0, sizeof(ull), st));
-    k_max_i64<<<grid_for(n, 256, g->num_sms * 8), 256, 0, st>>>(n, g->d0, mx);
+    k_max_i64<<<grid_for(n, 256, big), 256, 0, st>>>(n, g->d0, mx + 1);
     CKL();
-    CK(cudaMemcpyAsync(&hmx, mx, sizeof(ull), cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
-    g->maxw0 = (int64_t)hmx;
-    CK(cudaMemsetAsync(mx, 0, sizeof(ull), st));
-    k_rows_not_increasing<<<grid_for(n * 32, 256, g->num_sms * 8), 256, 0, st>>>((int)n, g->g0.rp, g->g0.col, mx);
+    k_rows_not_increasing<<<grid_for(n, 256, big), 256, 0, st>>>((int)n, g->g0.rp, g->g0.col, mx + 2);
     CKL();
-    CK(cudaMemcpyAsync(&hmx, mx, sizeof(ull), cudaMemcpyDeviceToHost, st));
+    i128* part = dalloc<i128>(big, st);
+    ull* ticket = dalloc<ull>(1, st);
+    i128* wsum = dalloc<i128>(1, st);
+    CK(cudaMemsetAsync(ticket, 0, sizeof(ull), st));
+    k_sum_i128<<<grid_for(n, 256, big), 256, 0, st>>>(n, g->d0, part, ticket, wsum);
+    CKL();
+    ull hm[3];
+    i128 hW = 0;
+    CK(cudaMemcpyAsync(hm, mx, 3 * sizeof(ull), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(&hW, wsum, sizeof(i128), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
-    g->rows_distinct0 = (hmx == 0);
+    g->maxdeg0 = (int64_t)hm[0];
+    g->maxw0 = (int64_t)hm[1];
+    g->rows_distinct0 = (hm[2] == 0);
     dfree(mx, st);
-}
-
-static gala_status validate_host(int64_t n, const int64_t* rp, const int32_t* col, const int64_t* w, int64_t* W,
-                                 bool* unit) {
-    if (n < 0 || n >= ((int64_t)1 << 31)) return set_err(GALA_E_INVALID, "n out of range: %lld", (long long)n);
-    if (!rp) return set_err(GALA_E_INVALID, "row_ptr is NULL");
-    if (rp[0] != 0) return set_err(GALA_E_INVALID, "row_ptr[0] != 0");
-    for (int64_t v = 0; v < n; ++v)
-        if (rp[v + 1] < rp[v]) return set_err(GALA_E_INVALID, "row_ptr not monotone at %lld", (long long)v);
-    int64_t nnz = rp[n];
-    if (nnz > 0 && !col) return set_err(GALA_E_INVALID, "col_idx is NULL");
-    int64_t tot = 0;
-    bool u = true;
-    for (int64_t e = 0; e < nnz; ++e) {
-        if (col[e] < 0 || col[e] >= n) return set_err(GALA_E_INVALID, "col_idx[%lld] out of range", (long long)e);
-        int64_t x = w ? w[e] : 1;
-        if (x <= 0) return set_err(GALA_E_INVALID, "weight[%lld] <= 0", (long long)e);
-        if (x != 1) u = false;
-        tot += x;
-        if (tot < 0) return set_err(GALA_E_OVERFLOW, "total weight overflows int64");
-    }
-    *W = tot;
-    *unit = u;
-    return GALA_OK;
+    dfree(part, st);
+    dfree(ticket, st);
+    dfree(wsum, st);
+    if (n == 0) hW = 0;
+    if (hW >= ((i128)1 << 62)) { set_err(GALA_E_OVERFLOW, "total weight W >= 2^62"); throw GalaError{GALA_E_OVERFLOW}; }
+    g->W = (int64_t)hW;
 }
 
 #define API_BEGIN try {
@@ -1004,10 +1005,10 @@ gala_status gala_graph_from_csr(int64_t n, const int64_t* row_ptr, const int32_t
                                 int device, uintptr_t stream, gala_graph* out) {
     if (!out) return set_err(GALA_E_INVALID, "out is NULL");
     *out = nullptr;
-    int64_t W = 0;
-    bool unit = true;
-    gala_status s = validate_host(n, row_ptr, col_idx, weights, &W, &unit);
-    if (s != GALA_OK) return s;
+    if (n < 0 || n >= ((int64_t)1 << 31)) return set_err(GALA_E_INVALID, "n out of range: %lld", (long long)n);
+    if (!row_ptr) return set_err(GALA_E_INVALID, "row_ptr is NULL");
+    if (row_ptr[0] != 0 || row_ptr[n] < 0) return set_err(GALA_E_INVALID, "row_ptr[0] != 0 or row_ptr[n] < 0");
+    if (row_ptr[n] > 0 && !col_idx) return set_err(GALA_E_INVALID, "col_idx is NULL");
     gala_graph_s* g = new gala_graph_s();
     PoolScope pool_scope(nullptr);
     API_BEGIN
@@ -1016,14 +1017,13 @@ gala_status gala_graph_from_csr(int64_t n, const int64_t* row_ptr, const int32_t
         cudaStream_t st = g->stream;
         const int64_t nnz = row_ptr[n];
         g->nnz0 = nnz;
-        g->W = W;
         g->g0.n = n;
         g->g0.nnz = nnz;
         g->g0.rp = dalloc<int64_t>(n + 1, st);
         g->g0.col = dalloc<int32_t>(nnz, st);
         CK(cudaMemcpyAsync(g->g0.rp, row_ptr, sizeof(int64_t) * (n + 1), cudaMemcpyHostToDevice, st));
         if (nnz) CK(cudaMemcpyAsync(g->g0.col, col_idx, sizeof(int32_t) * nnz, cudaMemcpyHostToDevice, st));
-        if (!unit) {
+        if (weights) {
             g->g0.w = dalloc<int64_t>(nnz, st);
             CK(cudaMemcpyAsync(g->g0.w, weights, sizeof(int64_t) * nnz, cudaMemcpyHostToDevice, st));
         }
@@ -1064,13 +1064,6 @@ gala_status gala_graph_from_csr_device(int64_t n, const int64_t* d_row_ptr, cons
             CK(cudaMemcpyAsync(g->g0.w, d_weights, sizeof(int64_t) * nnz, cudaMemcpyDeviceToDevice, st));
         }
         finish_graph(g);
-        // W = sum of d0 (device-side validation of ranges is done by the host path only)
-        std::vector<int64_t> hd(n);
-        CK(cudaMemcpyAsync(hd.data(), g->d0, sizeof(int64_t) * n, cudaMemcpyDeviceToHost, st));
-        CK(cudaStreamSynchronize(st));
-        int64_t W = 0;
-        for (int64_t v = 0; v < n; ++v) W += hd[v];
-        g->W = W;
     } catch (...) {
         gala_graph_free(g);
         throw;

@@ -418,6 +418,54 @@ __global__ void k_coarsen_deg(int n, const int32_t* __restrict__ C, const int32_
         if (minmem[C[v]] == v) d_new[newid[v]] = Sig[C[v]];
 }
 
+// input validation on the device: flags |= 1 row_ptr decreasing, 2 column out of
+// range, 4 weight <= 0, 8 some weight != 1
+__global__ void k_validate(int n, long long nnz, const int64_t* __restrict__ rp, const int32_t* __restrict__ col,
+                           const int64_t* __restrict__ w, unsigned* __restrict__ flags) {
+    unsigned f = 0;
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride)
+        if (rp[v + 1] < rp[v]) f |= 1u;
+    for (long long e = (long long)blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += stride) {
+        int c = col[e];
+        if (c < 0 || c >= n) f |= 2u;
+        if (w) {
+            long long x = w[e];
+            if (x <= 0) f |= 4u;
+            if (x != 1) f |= 8u;
+        }
+    }
+    f = __reduce_or_sync(FULLMASK, f);
+    if (lane_id() == 0 && f) atomicOr(flags, f);
+}
+
+// sum of a non-negative int64 array as int128 (per-block partials + last block)
+__global__ void __launch_bounds__(256) k_sum_i128(long long n, const int64_t* __restrict__ x, i128* __restrict__ part,
+                                                  ull* __restrict__ ticket, i128* __restrict__ out) {
+    __shared__ i128 sh[8];
+    __shared__ bool amLast;
+    i128 s = 0;
+    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
+        s += (i128)x[i];
+    for (int o = 16; o > 0; o >>= 1) s += shfl_xor_st(s, o);
+    if (lane_id() == 0) sh[threadIdx.x >> 5] = s;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int i = 1; i < (int)(blockDim.x >> 5); ++i) s += sh[i];
+        part[blockIdx.x] = s;
+        __threadfence();
+        amLast = atomicAdd(ticket, 1ull) == gridDim.x - 1;
+    }
+    __syncthreads();
+    if (amLast && threadIdx.x == 0) {
+        __threadfence();
+        i128 t = 0;
+        for (int b = 0; b < (int)gridDim.x; ++b) t += part[b];
+        *out = t;
+        *ticket = 0;
+    }
+}
+
 // *bad != 0 iff some row is not strictly increasing (so may hold duplicate columns)
 __global__ void k_rows_not_increasing(int n, const int64_t* __restrict__ rp, const int32_t* __restrict__ col,
                                       ull* __restrict__ bad) {
