@@ -104,6 +104,18 @@ class ClockSampler:
                 "reasons": sorted(self.reasons), "samples": len(self.samples)}
 
 
+def max_over_ranks(x: float) -> float:
+    """MAX of a host scalar over all ranks of the default process group (identity without one)."""
+    import torch
+    import torch.distributed as dist
+    if not (dist.is_available() and dist.is_initialized()):
+        return x
+    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor([x], dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
 def nominal_edges(stats: dict) -> int:
     return sum(lv["nominal_edges"] for lv in stats["levels"])
 
@@ -172,6 +184,7 @@ def main():
     ap.add_argument("--config", default="lfr1m", choices=sorted(WORKLOADS))
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-timing", action="store_true", help="skip the per-kernel-event (roofline) steps")
+    ap.add_argument("--force-dist", action="store_true", help="use the multi-GPU (NCCL) path even at world size 1")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3) if args.impl != "reference" else args.warmup
 
@@ -186,10 +199,14 @@ def main():
     import graphgen as gg
     import paper_conf_ppopp_wangllwm00z25_b200 as gala
 
-    if world > 1:
+    if world > 1 or args.force_dist:
         import torch.distributed as dist
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29533")
+        os.environ.setdefault("RANK", str(rank))
+        os.environ.setdefault("WORLD_SIZE", str(world))
         torch.cuda.set_device(local_rank)
-        dist.init_process_group("nccl")
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
         return run_dist(args, rank, world, local_rank)
 
     dev = 0
@@ -338,7 +355,93 @@ def main():
 
 
 def run_dist(args, rank, world, local_rank):
-    raise SystemExit("multi-GPU bench path not built yet")
+    """N > 1 (torchrun, one process per GPU): 1D edge-balanced vertex partition of the same graph,
+    NCCL inside libgala for the per-iteration label / counter exchange (bootstrapped here with the
+    torch process group).  Total work is fixed as N grows -> strong scaling."""
+    import torch
+    import torch.distributed as dist
+    import graphgen as gg
+    import paper_conf_ppopp_wangllwm00z25_b200 as gala
+
+    dev = local_rank
+    g = gg.make(args.config)                      # identical on every rank (seeded)
+    bounds = gala.partition_ranges(g.row_ptr, world)
+    v0, v1 = int(bounds[rank]), int(bounds[rank + 1])
+    lrp, lcol, lw = gala.local_rows(g.row_ptr, g.col, g.w, v0, v1)
+    uid = [gala.nccl_unique_id() if rank == 0 else None]
+    dist.broadcast_object_list(uid, src=0)
+    stream = torch.cuda.Stream(device=dev)
+    h = gala.Graph.from_csr_dist(uid[0], rank, world, dev, g.n, v0, v1, lrp, lcol, lw, stream=stream.cuda_stream)
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device=dev)
+    for _ in range(args.warmup):
+        h.run()
+    torch.cuda.synchronize()
+    peak, peak_src, _ = load_peaks()
+
+    def step(fn):
+        with torch.cuda.stream(stream):
+            flush.add_(1)
+        dist.barrier()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        fn()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        dist.barrier()
+        return max_over_ranks(e0.elapsed_time(e1))
+
+    with ClockSampler(dev) as clk:
+        step_ms = [step(h.run) for _ in range(args.steps)]
+    st = h.stats()
+    edges = nominal_edges(st)
+    Q = h.modularity()
+    labels = h.communities()
+    total_s = sum(step_ms) / 1e3
+    value = edges * args.steps / total_s / 1e9
+
+    # e2e through the C ABI from host buffers on every rank
+    import ctypes
+    e2e_ms = []
+    L = gala.lib()
+    lab_host = np.empty(g.n, dtype=np.int32)
+    for i in range(args.warmup + args.steps):
+        def e2e():
+            hh = gala.Graph.from_csr_dist(uid[0], rank, world, dev, g.n, v0, v1, lrp, lcol, lw,
+                                          stream=stream.cuda_stream)
+            hh.run()
+            gala._check(L.gala_get_communities(hh._h, lab_host.ctypes.data_as(ctypes.c_void_p), g.n, None))
+            hh.free()
+        ms = step(e2e)
+        if i >= args.warmup:
+            e2e_ms.append(ms)
+    e2e_value = edges * len(e2e_ms) / (sum(e2e_ms) / 1e3) / 1e9
+    d = st.get("dist", {})
+    line = {
+        "metric": METRIC, "value": value, "unit": "GTEPS", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": 1e3 * total_s / args.steps, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+        "config": {"workload": args.config, "desc": WORKLOADS.get(args.config, ""), "n": g.n, "nnz": g.nnz,
+                   "gamma": 1.0, "tol": 1e-6, "prune": 1, "parallelism": f"1D vertex partition x{world} (NCCL)",
+                   "l2": "flushed between timed steps (256 MB write)"},
+        "louvain_seconds": total_s / args.steps,
+        "step_ms": [round(x, 3) for x in step_ms],
+        "modularity": Q,
+        "levels": len(st["levels"]),
+        "iterations": sum(lv["iters"] for lv in st["levels"]),
+        "sync": {"dense_iters": d.get("dense_iters"), "sparse_iters": d.get("sparse_iters"),
+                 "bytes_exchanged_per_run": d.get("bytes_exchanged")},
+        "roofline": None, "cpu_baseline": None,
+        "e2e": {"value": e2e_value, "unit": "GTEPS", "h2d_bytes_per_step": int(lrp.nbytes + lcol.nbytes),
+                "d2h_bytes_per_step": int(g.n * 4)},
+        "gpu_launches": st["kernel_launches"],
+        "clocks": clk.summary(),
+    }
+    h.free()
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    dist.barrier()
+    dist.destroy_process_group()
 
 
 if __name__ == "__main__":

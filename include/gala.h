@@ -139,13 +139,18 @@ void gala_graph_free(gala_graph g);
  *   "check"          0/1   debug: verify maintained d'(v) against its definition
  *   "timing"         0/1   per-kernel CUDA-event timing (gala_get_kernel_stats)
  *   "max_iters"      >= 0  per-level iteration cap (0 = none)
- *   "bin_sub4" "bin_sub8" "bin_sub16" "bin_sub32" "bin_warp"
- *                    degree upper bounds of the dispatch bins (must be
- *                    non-decreasing, sub-warp bins <= their lane count)
+ *   "bin_sub4" "bin_sub8" "bin_sub16" "bin_sub32" "bin_warp" "bin_warp512"
+ *                    row-length upper bounds of the dispatch bins (non-decreasing;
+ *                    each <= 4, 8, 16, 32, 128, 512 respectively)
  *   "delta_update"   0 = always recompute d', 1 = always delta, 2 = adaptive (default)
  *   "force_i128"     0/1   use the 128-bit gain path even when 64-bit suffices
- *   "hub_smem_slots" power of two, shared-memory slots of the block hash table
- *   "cuda_graph"     0/1   capture the iteration body in a CUDA graph (default 1)
+ *   "force_wide"     0/1   use unpacked 64-bit gains / aggregates (no packed keys)
+ *   "singleton"      0/1   first iteration of a level via the singleton fast path (default 1)
+ *   "hub_smem_slots" power of two in [64, 16384], shared-memory slots of the block hash table
+ *   "cuda_graph"     0/1   run each level's iterations as a conditional CUDA graph (default 1)
+ *   "log_cap"        device iteration-log capacity (default 4096)
+ *   "sync_mode"      multi-GPU label exchange: 0 adaptive (default), 1 dense, 2 sparse
+ *   "verbose"        0/1   host-side phase timings on stderr
  */
 gala_status gala_set_option(gala_graph g, const char* key, int64_t value);
 
@@ -188,6 +193,14 @@ gala_status gala_get_kernel_stats(gala_graph g, int32_t k, const char** name, in
 
 /* 128-byte ncclUniqueId for rank 0 to broadcast (GALA_E_NCCL if NCCL cannot be loaded). */
 gala_status gala_nccl_unique_id(void* out128);
+
+/*
+ * gala_loopback_unique_id — TEST HOOK: a uid that makes gala_graph_from_csr_dist
+ * run `world` ranks as threads of ONE process on one device (device-to-device
+ * copies + host barriers instead of NCCL), so the partitioned algorithm can be
+ * exercised where only one GPU exists.  Never used by the product path.
+ */
+gala_status gala_loopback_unique_id(void* out128);
 
 /*
  * gala_graph_from_csr_dist — collective over `world` ranks.

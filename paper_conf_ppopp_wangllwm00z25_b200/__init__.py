@@ -65,6 +65,7 @@ def lib():
         "gala_get_trace_labels": (st, [p, i64, p, i64]),
         "gala_get_kernel_stats": (st, [p, i32, ctypes.POINTER(ctypes.c_char_p), p, p, p, p]),
         "gala_nccl_unique_id": (st, [p]),
+        "gala_loopback_unique_id": (st, [p]),
         "gala_graph_from_csr_dist": (st, [p, ctypes.c_int, ctypes.c_int, ctypes.c_int, i64, i64, i64, p, p, p,
                                           ctypes.c_size_t, pp]),
         "gala_partition_ranges": (st, [i64, p, ctypes.c_int, p]),
@@ -113,6 +114,23 @@ def nccl_unique_id() -> bytes:
     buf = ctypes.create_string_buffer(128)
     _check(lib().gala_nccl_unique_id(buf))
     return buf.raw
+
+
+def loopback_unique_id() -> bytes:
+    """TEST HOOK: uid that runs the ranks of from_csr_dist as threads of one process on one GPU."""
+    buf = ctypes.create_string_buffer(128)
+    _check(lib().gala_loopback_unique_id(buf))
+    return buf.raw
+
+
+def local_rows(row_ptr, col, w, v0: int, v1: int):
+    """Rows [v0, v1) of a CSR as (local_row_ptr, col, w) with global column ids (host arrays)."""
+    rp = np.asarray(row_ptr, dtype=np.int64)
+    a, b = int(rp[v0]), int(rp[v1])
+    lrp = (rp[v0:v1 + 1] - a).astype(np.int64)
+    lcol = np.ascontiguousarray(np.asarray(col, dtype=np.int32)[a:b])
+    lw = None if w is None else np.ascontiguousarray(np.asarray(w, dtype=np.int64)[a:b])
+    return lrp, lcol, lw
 
 
 class Graph:

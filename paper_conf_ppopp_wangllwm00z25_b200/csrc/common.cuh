@@ -56,6 +56,8 @@ struct Carry {
     ull N_prev_lo;
     long long minSig;       // min{Sig[c] : Sig[c] > 0}
     long long sumDC;        // sum_v (d'(v) + s(v))
+    long long S2_hi;        // sum_c Sig[c]^2 (int128 split)
+    ull S2_lo;
     int converged;
     int iter;               // iteration index within the level (also the d' stamp id)
     int more;               // loop condition written by k_record

@@ -10,6 +10,8 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <atomic>
+#include <chrono>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
@@ -22,7 +24,8 @@
 #include "k_phase1.cuh"
 #include "k_decide.cuh"
 #include "k_phase2.cuh"
-#include "dist.h"
+#include "comm.cuh"
+#include "k_dist.cuh"
 
 #define GALA_VERSION "gala-b200 0.1 (sm_100a)"
 
@@ -98,7 +101,7 @@ struct gala_graph_s {
     int64_t* s0 = nullptr;
     // options
     int opt_prune = 1, opt_trace = 0, opt_check = 0, opt_timing = 0, opt_max_iters = 0;
-    int opt_delta = 2, opt_force_i128 = 0, opt_force_wide = 0, opt_cuda_graph = 1, opt_log_cap = 4096, opt_singleton = 1;
+    int opt_delta = 2, opt_force_i128 = 0, opt_force_wide = 0, opt_cuda_graph = 1, opt_log_cap = 4096, opt_singleton = 1, opt_verbose = 0;
     bool rows_distinct0 = false;   // level-0 rows strictly increasing (no duplicate entries)
     int bins[NBINS - 1] = {4, 8, 16, 32, 128, 512};
     int hub_smem_slots = 4096;
@@ -117,8 +120,10 @@ struct gala_graph_s {
     int64_t dp_mismatch = 0;
     long long launches = 0;   // kernels launched by the last gala_run
     int check_mismatch = 0;   // check mode: final N on G0 differs from the last level's N
-    // dist
-    DistCtx* dist = nullptr;
+    // multi-GPU (one process per GPU)
+    struct DistInfo* di = nullptr;
+    int sync_mode = 0;
+    std::vector<long long> dbounds0;   // level-0 owned ranges of all ranks
     struct Work* wk = nullptr;   // persistent run workspace (sized for level 0, reused by every run)
 };
 
@@ -360,7 +365,7 @@ static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, typename
     BinThresholds th;
     for (int i = 0; i < NBINS - 1; ++i) th.t[i] = g->bins[i];
     k_prune_bin<typename ModeT<M>::ST><<<grid_for((n + PB_IPT - 1) / PB_IPT, PB_BT, big), PB_BT, 0, st>>>(
-        n, G.rp, wk.d, wk.dp, wk.C, wk.Sig, wk.size, g->opt_prune, qW, p, wk.carry, wk.ctr, wk.queues, wk.ncap, th);
+        0, n, G.rp, wk.d, wk.dp, wk.C, wk.Sig, wk.size, g->opt_prune, qW, p, wk.carry, wk.ctr, wk.queues, wk.ncap, th);
     CKL();
     tm.end(KC_PRUNE, e);
     launch_decide<M, UNIT>(g, wk, G, qW, p, tm, maxdeg, idbits, single);
@@ -373,14 +378,14 @@ static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, typename
     k_dp_delta<UNIT><<<big, 256, 0, st>>>(wk.ctr, G.rp, G.col, G.w, wk.C, wk.mv_v, wk.mv_old, wk.stamp, wk.dp,
                                           wk.carry, G.nnz, g->opt_delta, 1, 2);
     CKL();
-    k_dp_zero<<<big, 256, 0, st>>>(wk.ctr, n, wk.dp, G.nnz, g->opt_delta, 1, 2);
+    k_dp_zero<<<big, 256, 0, st>>>(wk.ctr, 0, n, wk.dp, G.nnz, g->opt_delta, 1, 2);
     CKL();
     k_dp_full<UNIT><<<grid_for((G.nnz + 127) / 128 * 32, 256, big), 256, 0, st>>>(wk.ctr, G.nnz, G.row, G.col, G.w,
                                                                                  wk.C, wk.dp, g->opt_delta, 1, 2);
     CKL();
     tm.end(KC_DP, e);
     e = tm.begin();
-    k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>(n, wk.dp, wk.s, wk.Sig, wk.part_dc, wk.part_s2, wk.part_min, wk.ctr,
+    k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>(n, 0, n, wk.dp, wk.s, wk.Sig, wk.part_dc, wk.part_s2, wk.part_min, wk.ctr,
                                                   wk.carry, (long long)(qW128 >> 64), (ull)qW128, (long long)p,
                                                   (long long)(T >> 64), (ull)T, 1);
     CKL();
@@ -507,6 +512,20 @@ static void account_bytes(gala_graph_s* g, const IterCounters& c, int64_t n, int
     g->kc_bytes[KC_REDUCE] += (double)n * 24;
 }
 
+// verbose host-side phase timing (option "verbose"): synchronises the stream
+struct VTimer {
+    gala_graph_s* g;
+    std::chrono::steady_clock::time_point t;
+    explicit VTimer(gala_graph_s* gg) : g(gg), t(std::chrono::steady_clock::now()) {}
+    void lap(const char* what) {
+        if (!g->opt_verbose) return;
+        cudaStreamSynchronize(g->stream);
+        auto now = std::chrono::steady_clock::now();
+        fprintf(stderr, "[gala] %-28s %9.3f ms\n", what, std::chrono::duration<double, std::milli>(now - t).count());
+        t = now;
+    }
+};
+
 // ------------------------------------------------------------------ phase 2 (a9)
 // Coarsen level graph `cur` with community ids newid[v] in [0, k) into `nxt`
 // (reading c10: the diagonal carries D_C(c) once).  See k_phase2.cuh for
@@ -514,19 +533,22 @@ static void account_bytes(gala_graph_s* g, const IterCounters& c, int64_t n, int
 #define AGG_BLOCK_BT 512
 static size_t agg_block_smem(int scap) { return (size_t)scap * (sizeof(ull) + sizeof(int)) + (size_t)(scap / 2) * sizeof(int); }
 
-static void coarsen(gala_graph_s* g, Work& wk, const DevCSR& cur, int64_t nl, long long k, const int32_t* newid,
-                    const int32_t* minmem, bool unit, DevCSR& nxt, int64_t& maxdeg, int64_t& dmax) {
+// Aggregate the rows of `cur` (nrows rows, each with a row-id array) into k
+// target rows: target of row v is newid[v]; entries become (newid[u], w) and
+// equal (target, key) pairs are summed.  Output CSR in pool memory with int64
+// weights and row ids; snew[c] (caller-allocated, k) receives the diagonal.
+static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, long long k, const int32_t* newid,
+                           const int32_t* keymap, bool unit, DevCSR& nxt, int64_t& maxdeg, int64_t* snew) {
     cudaStream_t st = g->stream;
     const int big = g->num_sms * 8;
+    VTimer vt(g);
     long long* cnt = dalloc<long long>(k + 1, st);
     long long* ent = dalloc<long long>(k + 1, st);
     long long* eoff = dalloc<long long>(k + 1, st);
     long long* dn = dalloc<long long>(k + 1, st);
     int* tkey = dalloc<int>(cur.nnz, st);
     int64_t* tval = dalloc<int64_t>(cur.nnz, st);
-    int64_t* snew = dalloc<int64_t>(k, st);
-    int64_t* dnew = dalloc<int64_t>(k, st);
-    ull* dev_max = dalloc<ull>(2, st);
+    ull* dev_max = dalloc<ull>(1, st);
     int32_t* bigc = dalloc<int32_t>(k, st);
     long long* bigcap = dalloc<long long>(k + 1, st);
     int* nbig_dev = dalloc<int>(1, st);
@@ -534,24 +556,25 @@ static void coarsen(gala_graph_s* g, Work& wk, const DevCSR& cur, int64_t nl, lo
     CK(cudaMemsetAsync(ent, 0, sizeof(long long) * (k + 1), st));
     CK(cudaMemsetAsync(dn, 0, sizeof(long long) * (k + 1), st));
     CK(cudaMemsetAsync(snew, 0, sizeof(int64_t) * k, st));
-    CK(cudaMemsetAsync(dev_max, 0, sizeof(ull) * 2, st));
+    CK(cudaMemsetAsync(dev_max, 0, sizeof(ull), st));
     CK(cudaMemsetAsync(nbig_dev, 0, sizeof(int), st));
-    k_comm_stats<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, cur.rp, newid, ent);
+    k_comm_stats<<<grid_for(nrows, 256, big), 256, 0, st>>>((int)nrows, cur.rp, newid, ent);
     CKL();
     scan_excl(ent, eoff, k, st);
     // segment position of every row (cnt reused as the per-community cursor), then an
-    // edge-parallel copy of the coarse keys into the segments
-    long long* vpos = dalloc<long long>(nl, st);
-    k_vpos<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, cur.rp, newid, eoff, cnt, vpos);
+    // edge-parallel copy of the keys keymap[u] into the segments
+    long long* vpos = dalloc<long long>(nrows, st);
+    k_vpos<<<grid_for(nrows, 256, big), 256, 0, st>>>((int)nrows, cur.rp, newid, eoff, cnt, vpos);
     CKL();
     if (unit)
         k_gather_flat<true><<<grid_for((cur.nnz + 127) / 128 * 32, 256, big), 256, 0, st>>>(
-            cur.nnz, cur.row, cur.rp, cur.col, cur.w, newid, vpos, tkey, tval);
+            cur.nnz, cur.row, cur.rp, cur.col, cur.w, keymap, vpos, tkey, tval);
     else
         k_gather_flat<false><<<grid_for((cur.nnz + 127) / 128 * 32, 256, big), 256, 0, st>>>(
-            cur.nnz, cur.row, cur.rp, cur.col, cur.w, newid, vpos, tkey, tval);
+            cur.nnz, cur.row, cur.rp, cur.col, cur.w, keymap, vpos, tkey, tval);
     CKL();
     dfree(vpos, st);
+    vt.lap("agg: stats+gather");
     // shared-memory capacity of the block path: up to 8192 slots (14 B each)
     int scap = 512;
     while (scap < 8192 && scap < 2 * k) scap <<= 1;
@@ -571,6 +594,7 @@ static void coarsen(gala_graph_s* g, Work& wk, const DevCSR& cur, int64_t nl, lo
         else k_agg_block<AGG_BLOCK_BT, false><<<gb, AGG_BLOCK_BT, sm, st>>>(a, scap);
         CKL();
     }
+    vt.lap("agg: warp+block");
     int nbig = 0;
     CK(cudaMemcpyAsync(&nbig, nbig_dev, sizeof(int), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
@@ -591,39 +615,64 @@ static void coarsen(gala_graph_s* g, Work& wk, const DevCSR& cur, int64_t nl, lo
         if (unit) k_agg_big_insert<true><<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
         else k_agg_big_insert<false><<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
         CKL();
-        k_agg_big_emit<<<std::min(nbig, big), 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt);
+        k_agg_big_emit<<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
         CKL();
         dfree(goff, st); dfree(gkeys, st); dfree(gvals, st); dfree(glist, st); dfree(gcnt, st);
+        if (g->opt_verbose) fprintf(stderr, "[gala] big communities %d, table slots %lld\n", nbig, gtot);
     }
+    vt.lap("agg: big");
     nxt.n = k;
     nxt.rp = dalloc<int64_t>(k + 1, st);
     scan_excl(dn, reinterpret_cast<long long*>(nxt.rp), k, st);
     k_rowmax<<<grid_for(k, 256, big), 256, 0, st>>>(k, reinterpret_cast<long long*>(nxt.rp), dev_max);
     CKL();
-    // coarse d = Sigma_tot of the community (exactly maintained by phase 1)
-    k_coarsen_deg<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.C, minmem, newid, wk.Sig, dnew);
-    CKL();
-    k_max_i64<<<grid_for(k, 256, big), 256, 0, st>>>(k, dnew, dev_max + 1);
-    CKL();
-    ull hm[2] = {0, 0};
+    ull hm = 0;
     CK(cudaMemcpyAsync(&nxt.nnz, nxt.rp + k, sizeof(long long), cudaMemcpyDeviceToHost, st));
-    CK(cudaMemcpyAsync(hm, dev_max, sizeof(ull) * 2, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(&hm, dev_max, sizeof(ull), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
-    maxdeg = (int64_t)hm[0];
-    dmax = (int64_t)hm[1];
+    maxdeg = (int64_t)hm;
     nxt.col = dalloc<int32_t>(nxt.nnz, st);
     nxt.w = dalloc<int64_t>(nxt.nnz, st);
     nxt.row = dalloc<int32_t>(nxt.nnz, st);
-    k_compact<<<grid_for(k * 32, 256, big), 256, 0, st>>>(k, eoff, reinterpret_cast<long long*>(nxt.rp), tkey, tval,
-                                                          nxt.col, nxt.w, nxt.row);
-    CKL();
-    CK(cudaMemcpyAsync(wk.d, dnew, sizeof(int64_t) * k, cudaMemcpyDeviceToDevice, st));
-    CK(cudaMemcpyAsync(wk.s, snew, sizeof(int64_t) * k, cudaMemcpyDeviceToDevice, st));
-    g->kc_bytes[KC_PHASE2] += (double)nl * (4 + 4 + 8 + 16 + 4 + 4) + (double)cur.nnz * (4 + 4 + (unit ? 0 : 8) + 12) +
+    if (nxt.nnz > 0) {
+        k_compact<<<grid_for(nxt.nnz, 256, big * 4), 256, 0, st>>>(k, nxt.nnz, eoff, reinterpret_cast<long long*>(nxt.rp),
+                                                                    tkey, tval, nxt.col, nxt.w, nxt.row);
+        CKL();
+    }
+    vt.lap("agg: scan+compact");
+    g->kc_bytes[KC_PHASE2] += (double)nrows * (4 + 4 + 8 + 16 + 4 + 4) + (double)cur.nnz * (4 + 4 + (unit ? 0 : 8) + 12) +
                               (double)nxt.nnz * 24;
     dfree(cnt, st); dfree(ent, st); dfree(eoff, st); dfree(dn, st);
-    dfree(tkey, st); dfree(tval, st); dfree(snew, st); dfree(dnew, st); dfree(dev_max, st); dfree(bigc, st);
+    dfree(tkey, st); dfree(tval, st); dfree(dev_max, st); dfree(bigc, st);
     dfree(bigcap, st); dfree(nbig_dev, st);
+}
+
+// ------------------------------------------------------------------ phase 2 (a9)
+// Coarsen level graph `cur` with community ids newid[v] in [0, k) into `nxt`
+// (reading c10: the diagonal carries D_C(c) once).  Coarse d(c) =
+// Sigma_tot(c) (maintained exactly by phase 1), s(c) = the diagonal.
+static void coarsen(gala_graph_s* g, Work& wk, const DevCSR& cur, int64_t nl, long long k, const int32_t* newid,
+                    const int32_t* minmem, bool unit, DevCSR& nxt, int64_t& maxdeg, int64_t& dmax) {
+    cudaStream_t st = g->stream;
+    const int big = g->num_sms * 8;
+    int64_t* snew = dalloc<int64_t>(k, st);
+    int64_t* dnew = dalloc<int64_t>(k, st);
+    ull* dev_max = dalloc<ull>(1, st);
+    aggregate_rows(g, cur, nl, k, newid, newid, unit, nxt, maxdeg, snew);
+    CK(cudaMemsetAsync(dev_max, 0, sizeof(ull), st));
+    k_coarsen_deg<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.C, minmem, newid, wk.Sig, dnew);
+    CKL();
+    k_max_i64<<<grid_for(k, 256, big), 256, 0, st>>>(k, dnew, dev_max);
+    CKL();
+    ull hm = 0;
+    CK(cudaMemcpyAsync(&hm, dev_max, sizeof(ull), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(wk.d, dnew, sizeof(int64_t) * k, cudaMemcpyDeviceToDevice, st));
+    CK(cudaMemcpyAsync(wk.s, snew, sizeof(int64_t) * k, cudaMemcpyDeviceToDevice, st));
+    CK(cudaStreamSynchronize(st));
+    dmax = (int64_t)hm;
+    dfree(snew, st);
+    dfree(dnew, st);
+    dfree(dev_max, st);
 }
 
 // Final numerator.  The last level's N equals N of the composed labels on the
@@ -662,32 +711,10 @@ static void final_numerator(gala_graph_s* g, int64_t p, int64_t q, int64_t W, i1
 }
 
 // ------------------------------------------------------------------ the multi-level run
-static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
-    PoolScope pool_scope(g->pool);
+// The run workspace (sized for level 0) is allocated once per handle and reused by every run.
+static void ensure_workspace(gala_graph_s* g) {
     cudaStream_t st = g->stream;
-    CK(cudaSetDevice(g->device));
-    g->has_result = false;
-    g->trace.clear();
-    g->trace_labels.clear();
-    g->levels.clear();
-    for (int i = 0; i < KC_COUNT; ++i) { g->kc_ms[i] = 0; g->kc_bytes[i] = 0; g->kc_launches[i] = 0; }
-    g->dp_mismatch = 0;
-    const long long launches0 = g_launches;
-    int64_t p, q;
-    gamma_to_pq(gamma, &p, &q);
-    g->p = p;
-    g->q = q;
-    const int64_t n0 = g->n0, W = g->W;
-    const int64_t mpq = std::max(p, q);
-    if ((long double)mpq * (long double)W * (long double)W >= 0x1p125L) {
-        set_err(GALA_E_OVERFLOW, "max(p,q)*W^2 >= 2^125");
-        throw GalaError{GALA_E_OVERFLOW};
-    }
-    const i128 qW128 = (i128)q * W;
-    const i128 T = (i128)ceill((long double)tol * (long double)q * (long double)W * (long double)W);
-
-    const int big = g->num_sms * 8;
-    if (!g->lab) g->lab = dalloc<int32_t>(n0, st);
+    const int64_t n0 = g->n0;
     if (g->wk && g->wk->log_cap != g->opt_log_cap) { g->wk->release(); delete g->wk; g->wk = nullptr; }
     if (!g->wk) {
         g->wk = new Work();
@@ -740,6 +767,36 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
             throw;
         }
     }
+}
+
+
+static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
+    PoolScope pool_scope(g->pool);
+    cudaStream_t st = g->stream;
+    CK(cudaSetDevice(g->device));
+    g->has_result = false;
+    g->trace.clear();
+    g->trace_labels.clear();
+    g->levels.clear();
+    for (int i = 0; i < KC_COUNT; ++i) { g->kc_ms[i] = 0; g->kc_bytes[i] = 0; g->kc_launches[i] = 0; }
+    g->dp_mismatch = 0;
+    const long long launches0 = g_launches;
+    int64_t p, q;
+    gamma_to_pq(gamma, &p, &q);
+    g->p = p;
+    g->q = q;
+    const int64_t n0 = g->n0, W = g->W;
+    const int64_t mpq = std::max(p, q);
+    if ((long double)mpq * (long double)W * (long double)W >= 0x1p125L) {
+        set_err(GALA_E_OVERFLOW, "max(p,q)*W^2 >= 2^125");
+        throw GalaError{GALA_E_OVERFLOW};
+    }
+    const i128 qW128 = (i128)q * W;
+    const i128 T = (i128)ceill((long double)tol * (long double)q * (long double)W * (long double)W);
+
+    const int big = g->num_sms * 8;
+    if (!g->lab) g->lab = dalloc<int32_t>(n0, st);
+    ensure_workspace(g);
     Work& wk = *g->wk;
     cudaEvent_t ev_run0 = wk.ev[0], ev_run1 = wk.ev[1];
     CK(cudaEventRecord(ev_run0, st));
@@ -789,7 +846,7 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
             }
             k_iter_begin<<<1, 128, 0, st>>>(wk.ctr);
             CKL();
-            k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>((int)nl, wk.dp, wk.s, wk.Sig, wk.part_dc, wk.part_s2,
+            k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>((int)nl, 0, (int)nl, wk.dp, wk.s, wk.Sig, wk.part_dc, wk.part_s2,
                                                           wk.part_min, wk.ctr, wk.carry, (long long)(qW128 >> 64),
                                                           (ull)qW128, (long long)p, 0, 0, 0);
             CKL();
@@ -900,6 +957,407 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
         g->wk = nullptr;
         throw;
     }
+    g->has_result = true;
+}
+
+// ------------------------------------------------------------------ multi-GPU driver (a10)
+// §4.3.  Each rank owns vertices [lv0, lv1) of the current level and
+// holds them as a global-row CSR; C, Sigma_tot, size and d are replicated.  One
+// iteration: prune + decide over the owned vertices (the single-GPU kernels),
+// collect the local moves, exchange them sparsely (allgatherv of (v, c) pairs)
+// or densely (allgatherv of label slices, then a diff) — chosen by bytes on
+// the wire — apply the global move list identically everywhere,
+// recompute d' of the owned vertices, and all-reduce the owned sum of
+// d' + s with the counters; N and the convergence decision then follow from
+// identical integers on every rank.  Phase 2: every rank aggregates its owned
+// rows, the partial coarse rows are exchanged and merged, and the coarse graph
+// is re-split edge-balanced.
+struct DistInfo {
+    Comm* comm = nullptr;
+    long long v0 = 0, v1 = 0;        // level-0 owned range
+    int sync_mode = 0;               // 0 adaptive, 1 dense, 2 sparse
+    long long n_dense = 0, n_sparse = 0;
+    double bytes_exchanged = 0;
+};
+
+static std::vector<size_t> prefix_bytes(const std::vector<size_t>& c) {
+    std::vector<size_t> d(c.size(), 0);
+    for (size_t i = 1; i < c.size(); ++i) d[i] = d[i - 1] + c[i - 1];
+    return d;
+}
+
+template <int M, bool UNIT>
+static void dist_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, long long lv0, long long lv1,
+                           const std::vector<long long>& bounds, typename ModeT<M>::ST qW, typename ModeT<M>::ST p,
+                           i128 qW128, i128 T, Timer& tm, int64_t maxdeg, int idbits, bool single, int2* lmoves,
+                           int2* gmoves, int32_t* newC, ull* dcnt, int64_t* vec) {
+    DistInfo& di = *g->di;
+    Comm& cm = *di.comm;
+    cudaStream_t st = g->stream;
+    const long long n = G.n;
+    const int big = g->num_sms * 8;
+    k_iter_begin<<<1, 128, 0, st>>>(wk.ctr);
+    CKL();
+    BinThresholds th;
+    for (int i = 0; i < NBINS - 1; ++i) th.t[i] = g->bins[i];
+    k_prune_bin<typename ModeT<M>::ST><<<grid_for((lv1 - lv0 + PB_IPT - 1) / PB_IPT, PB_BT, big), PB_BT, 0, st>>>(
+        (int)lv0, (int)lv1, G.rp, wk.d, wk.dp, wk.C, wk.Sig, wk.size, g->opt_prune, qW, p, wk.carry, wk.ctr, wk.queues,
+        wk.ncap, th);
+    CKL();
+    launch_decide<M, UNIT>(g, wk, G, qW, p, tm, maxdeg, idbits, single);
+    CK(cudaMemsetAsync(dcnt, 0, 2 * sizeof(ull), st));
+    k_collect_moves<<<grid_for(lv1 - lv0, 256, big), 256, 0, st>>>(wk.ctr, wk.queues, wk.ncap, wk.nextC, lmoves, dcnt);
+    CKL();
+    ull mloc = 0;
+    CK(cudaMemcpyAsync(&mloc, dcnt, sizeof(ull), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    const std::vector<int64_t> cnts = cm.allgather_host((int64_t)mloc, st);
+    long long total = 0;
+    for (int64_t c : cnts) total += c;
+    const double sparse_bytes = 8.0 * (double)total, dense_bytes = 4.0 * (double)n;
+    const bool sparse = di.sync_mode == 2 || (di.sync_mode == 0 && sparse_bytes < dense_bytes);
+    if (sparse) {
+        std::vector<size_t> cb(cm.world);
+        for (int r = 0; r < cm.world; ++r) cb[r] = (size_t)cnts[r] * sizeof(int2);
+        cm.allgatherv(lmoves, gmoves, cb, prefix_bytes(cb), st);
+        di.n_sparse++;
+        di.bytes_exchanged += sparse_bytes;
+    } else {
+        k_copy_range<<<grid_for(lv1 - lv0, 256, big), 256, 0, st>>>(lv0, lv1, wk.C, newC);
+        CKL();
+        k_scatter_moves<<<grid_for((long long)mloc, 256, big), 256, 0, st>>>(lmoves, dcnt, newC);
+        CKL();
+        std::vector<size_t> cb(cm.world), db(cm.world);
+        for (int r = 0; r < cm.world; ++r) {
+            cb[r] = (size_t)(bounds[r + 1] - bounds[r]) * sizeof(int32_t);
+            db[r] = (size_t)bounds[r] * sizeof(int32_t);
+        }
+        cm.allgatherv(newC + lv0, newC, cb, db, st);
+        k_diff_moves<<<grid_for(n, 256, big), 256, 0, st>>>((int)n, wk.C, newC, gmoves, dcnt + 1);
+        CKL();
+        di.n_dense++;
+        di.bytes_exchanged += dense_bytes;
+    }
+    k_apply_list<<<grid_for(total, 256, big), 256, 0, st>>>(gmoves, total, wk.C, wk.Sig, wk.size, wk.d, wk.stamp,
+                                                             wk.carry, wk.ctr);
+    CKL();
+    // d' of the owned vertices from its definition (edge-parallel over the owned rows)
+    k_dp_zero<<<big, 256, 0, st>>>(wk.ctr, (int)lv0, (int)lv1, wk.dp, G.nnz, 0, 1, 2);
+    CKL();
+    if (G.nnz) {
+        k_dp_full<UNIT><<<grid_for((G.nnz + 127) / 128 * 32, 256, big), 256, 0, st>>>(wk.ctr, G.nnz, G.row, G.col, G.w,
+                                                                                     wk.C, wk.dp, 0, 1, 2);
+        CKL();
+    }
+    k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>((int)n, (int)lv0, (int)lv1, wk.dp, wk.s, wk.Sig, wk.part_dc,
+                                                  wk.part_s2, wk.part_min, wk.ctr, wk.carry, 0, 0, 0, 0, 0, 3);
+    CKL();
+    k_pack_counters<<<1, 32, 0, st>>>(wk.carry, wk.ctr, vec);
+    CKL();
+    cm.allreduce_sum_i64(vec, 5, st);
+    k_finish<<<1, 32, 0, st>>>(vec, wk.ctr, wk.carry, (long long)(qW128 >> 64), (ull)qW128, (long long)p,
+                               (long long)(T >> 64), (ull)T, 1);
+    CKL();
+    k_record<<<1, 32, 0, st>>>(wk.ctr, wk.carry, wk.log, wk.log_cap, g->opt_max_iters, 0ull);
+    CKL();
+}
+
+// merge the partial coarse rows of every rank into the full coarse graph, then keep rows [lo, hi)
+static void dist_coarsen(gala_graph_s* g, Work& wk, const DevCSR& cur, int64_t nl, long long k, const int32_t* newid,
+                         const int32_t* minmem, bool unit, DevCSR& local, std::vector<long long>& bounds,
+                         int64_t& maxdeg, int64_t& dmax) {
+    Comm& cm = *g->di->comm;
+    cudaStream_t st = g->stream;
+    const int big = g->num_sms * 8;
+    DevCSR part;
+    int64_t md = 0;
+    int64_t* snew = dalloc<int64_t>(k, st);
+    aggregate_rows(g, cur, nl, k, newid, newid, unit, part, md, snew);
+    const std::vector<int64_t> cnts = cm.allgather_host(part.nnz, st);
+    long long tot = 0;
+    for (int64_t c : cnts) tot += c;
+    std::vector<size_t> c4(cm.world), c8(cm.world);
+    for (int r = 0; r < cm.world; ++r) { c4[r] = (size_t)cnts[r] * 4; c8[r] = (size_t)cnts[r] * 8; }
+    int32_t* arow = dalloc<int32_t>(tot, st);
+    int32_t* acol = dalloc<int32_t>(tot, st);
+    int64_t* aw = dalloc<int64_t>(tot, st);
+    cm.allgatherv(part.row, arow, c4, prefix_bytes(c4), st);
+    cm.allgatherv(part.col, acol, c4, prefix_bytes(c4), st);
+    cm.allgatherv(part.w, aw, c8, prefix_bytes(c8), st);
+    g->di->bytes_exchanged += 16.0 * (double)tot;
+    dfree(part.rp, st); dfree(part.col, st); dfree(part.w, st); dfree(part.row, st);
+    // counting sort of the triplets by coarse row -> multigraph M, then merge duplicates
+    DevCSR mg;
+    mg.n = k;
+    mg.nnz = tot;
+    long long* cnt = dalloc<long long>(k + 1, st);
+    CK(cudaMemsetAsync(cnt, 0, sizeof(long long) * (k + 1), st));
+    k_count_rows<<<grid_for(tot, 256, big), 256, 0, st>>>(tot, arow, cnt);
+    CKL();
+    mg.rp = dalloc<int64_t>(k + 1, st);
+    scan_excl(cnt, reinterpret_cast<long long*>(mg.rp), k, st);
+    CK(cudaMemsetAsync(cnt, 0, sizeof(long long) * (k + 1), st));
+    mg.row = dalloc<int32_t>(tot, st);
+    mg.col = dalloc<int32_t>(tot, st);
+    mg.w = dalloc<int64_t>(tot, st);
+    k_scatter_rows<<<grid_for(tot, 256, big), 256, 0, st>>>(tot, arow, acol, aw, reinterpret_cast<long long*>(mg.rp),
+                                                            cnt, mg.row, mg.col, mg.w);
+    CKL();
+    dfree(arow, st); dfree(acol, st); dfree(aw, st); dfree(cnt, st);
+    int32_t* id = dalloc<int32_t>(k, st);
+    k_iota<<<grid_for(k, 256, big), 256, 0, st>>>(k, id);
+    CKL();
+    DevCSR full;
+    aggregate_rows(g, mg, k, k, id, id, false, full, md, snew);
+    dfree(mg.rp, st); dfree(mg.col, st); dfree(mg.w, st); dfree(mg.row, st); dfree(id, st);
+    // replicated coarse d = Sigma_tot, s = diagonal
+    int64_t* dnew = dalloc<int64_t>(k, st);
+    ull* dev_max = dalloc<ull>(1, st);
+    CK(cudaMemsetAsync(dev_max, 0, sizeof(ull), st));
+    k_coarsen_deg<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.C, minmem, newid, wk.Sig, dnew);
+    CKL();
+    k_max_i64<<<grid_for(k, 256, big), 256, 0, st>>>(k, dnew, dev_max);
+    CKL();
+    CK(cudaMemcpyAsync(wk.d, dnew, sizeof(int64_t) * k, cudaMemcpyDeviceToDevice, st));
+    CK(cudaMemcpyAsync(wk.s, snew, sizeof(int64_t) * k, cudaMemcpyDeviceToDevice, st));
+    // edge-balanced split of the coarse graph; keep this rank's rows
+    long long* dbounds = dalloc<long long>(cm.world + 1, st);
+    k_partition_bounds<<<1, 64, 0, st>>>(k, full.rp, cm.world, dbounds);
+    CKL();
+    bounds.assign(cm.world + 1, 0);
+    ull hm = 0;
+    CK(cudaMemcpyAsync(bounds.data(), dbounds, sizeof(long long) * (cm.world + 1), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(&hm, dev_max, sizeof(ull), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    dmax = (int64_t)hm;
+    const long long lo = bounds[cm.rank], hi = bounds[cm.rank + 1];
+    int64_t e_lo = 0, e_hi = 0;
+    CK(cudaMemcpyAsync(&e_lo, full.rp + lo, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(&e_hi, full.rp + hi, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    local.n = k;
+    local.nnz = e_hi - e_lo;
+    local.rp = dalloc<int64_t>(k + 1, st);
+    k_restrict_rp<<<grid_for(k + 1, 256, big), 256, 0, st>>>(k, lo, hi, full.rp, local.rp);
+    CKL();
+    local.col = dalloc<int32_t>(local.nnz, st);
+    local.w = dalloc<int64_t>(local.nnz, st);
+    local.row = dalloc<int32_t>(local.nnz, st);
+    if (local.nnz) {
+        CK(cudaMemcpyAsync(local.col, full.col + e_lo, sizeof(int32_t) * local.nnz, cudaMemcpyDeviceToDevice, st));
+        CK(cudaMemcpyAsync(local.w, full.w + e_lo, sizeof(int64_t) * local.nnz, cudaMemcpyDeviceToDevice, st));
+        CK(cudaMemcpyAsync(local.row, full.row + e_lo, sizeof(int32_t) * local.nnz, cudaMemcpyDeviceToDevice, st));
+    }
+    ull* rmax = dalloc<ull>(1, st);
+    CK(cudaMemsetAsync(rmax, 0, sizeof(ull), st));
+    k_rowmax<<<grid_for(k, 256, big), 256, 0, st>>>(k, reinterpret_cast<long long*>(local.rp), rmax);
+    CKL();
+    ull hr = 0;
+    CK(cudaMemcpyAsync(&hr, rmax, sizeof(ull), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    maxdeg = (int64_t)hr;
+    dfree(full.rp, st); dfree(full.col, st); dfree(full.w, st); dfree(full.row, st);
+    dfree(dnew, st); dfree(dev_max, st); dfree(dbounds, st); dfree(rmax, st); dfree(snew, st);
+}
+
+static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_levels) {
+    PoolScope pool_scope(g->pool);
+    cudaStream_t st = g->stream;
+    CK(cudaSetDevice(g->device));
+    DistInfo& di = *g->di;
+    Comm& cm = *di.comm;
+    g->has_result = false;
+    g->trace.clear();
+    g->trace_labels.clear();
+    g->levels.clear();
+    for (int i = 0; i < KC_COUNT; ++i) { g->kc_ms[i] = 0; g->kc_bytes[i] = 0; g->kc_launches[i] = 0; }
+    g->dp_mismatch = 0;
+    di.n_dense = di.n_sparse = 0;
+    di.bytes_exchanged = 0;
+    const long long launches0 = g_launches;
+    int64_t p, q;
+    gamma_to_pq(gamma, &p, &q);
+    g->p = p;
+    g->q = q;
+    const int64_t n0 = g->n0, W = g->W;
+    const int64_t mpq = std::max(p, q);
+    if ((long double)mpq * (long double)W * (long double)W >= 0x1p125L) {
+        set_err(GALA_E_OVERFLOW, "max(p,q)*W^2 >= 2^125");
+        throw GalaError{GALA_E_OVERFLOW};
+    }
+    const i128 qW128 = (i128)q * W;
+    const i128 T = (i128)ceill((long double)tol * (long double)q * (long double)W * (long double)W);
+    const int big = g->num_sms * 8;
+    if (!g->lab) g->lab = dalloc<int32_t>(n0, st);
+    ensure_workspace(g);
+    Work& wk = *g->wk;
+    CK(cudaEventRecord(wk.ev[0], st));
+    int2* lmoves = dalloc<int2>(n0, st);
+    int2* gmoves = dalloc<int2>(n0, st);
+    int32_t* newC = dalloc<int32_t>(n0, st);
+    ull* dcnt = dalloc<ull>(2, st);
+    int64_t* vec = dalloc<int64_t>(8, st);
+    try {
+        CK(cudaMemsetAsync(wk.ctr, 0, sizeof(IterCounters), st));
+        CK(cudaMemsetAsync(wk.carry, 0, sizeof(Carry), st));
+        DevCSR cur = g->g0;
+        bool cur_owned = false;
+        CK(cudaMemcpyAsync(wk.d, g->d0, sizeof(int64_t) * n0, cudaMemcpyDeviceToDevice, st));
+        CK(cudaMemcpyAsync(wk.s, g->s0, sizeof(int64_t) * n0, cudaMemcpyDeviceToDevice, st));
+        int64_t maxdeg = g->maxdeg0, dmax = g->maxw0;
+        std::vector<long long> bounds = g->dbounds0;
+        Timer tm(g);
+        std::vector<IterLog> logs;
+        for (int level = 0;; ++level) {
+            const int64_t nl = cur.n;
+            const bool unit = (cur.w == nullptr);
+            const long long lv0 = bounds[cm.rank], lv1 = bounds[cm.rank + 1];
+            long long gnnz = 0;   // level nnz over all ranks (stats / nominal edges)
+            for (int64_t x : cm.allgather_host(cur.nnz, st)) gnnz += x;
+            LevelStat ls{};
+            ls.n = nl;
+            ls.nnz = gnnz;
+            ls.maxdeg = maxdeg;
+            CK(cudaEventRecord(wk.ev[2], st));
+            long long need = 64;
+            while (need < 2 * maxdeg) need <<= 1;
+            if (maxdeg > g->bins[BIN_WARP2] && need > wk.gcap) {
+                dfree(wk.gkeys, st);
+                dfree(wk.gvals, st);
+                dfree(wk.glist, st);
+                wk.gcap = need;
+                wk.gkeys = dalloc<int>((size_t)wk.gblocks * wk.gcap, st);
+                wk.gvals = dalloc<ull>((size_t)wk.gblocks * wk.gcap, st);
+                wk.glist = dalloc<int>((size_t)wk.gblocks * wk.gcap, st);
+                CK(cudaMemsetAsync(wk.gkeys, 0xff, sizeof(int) * (size_t)wk.gblocks * wk.gcap, st));
+                CK(cudaMemsetAsync(wk.gvals, 0, sizeof(ull) * (size_t)wk.gblocks * wk.gcap, st));
+            }
+            k_level_init<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.d, wk.C, wk.Sig, wk.size, wk.dp, wk.stamp,
+                                                                 wk.carry);
+            CKL();
+            if (level == 0) CK(cudaMemcpyAsync(g->lab, wk.C, sizeof(int32_t) * n0, cudaMemcpyDeviceToDevice, st));
+            k_iter_begin<<<1, 128, 0, st>>>(wk.ctr);
+            CKL();
+            k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>((int)nl, (int)lv0, (int)lv1, wk.dp, wk.s, wk.Sig, wk.part_dc,
+                                                          wk.part_s2, wk.part_min, wk.ctr, wk.carry, 0, 0, 0, 0, 0, 2);
+            CKL();
+            k_pack_counters<<<1, 32, 0, st>>>(wk.carry, wk.ctr, vec);
+            CKL();
+            cm.allreduce_sum_i64(vec, 5, st);
+            k_finish<<<1, 32, 0, st>>>(vec, wk.ctr, wk.carry, (long long)(qW128 >> 64), (ull)qW128, (long long)p, 0, 0, 0);
+            CKL();
+            CK(cudaMemcpyAsync(wk.h_carry, wk.carry, sizeof(Carry), cudaMemcpyDeviceToHost, st));
+            CK(cudaStreamSynchronize(st));
+            const i128 N_start = carry_N(wk.h_carry);
+            int idbits = 1;
+            while (idbits < 31 && ((int64_t)1 << idbits) < nl) ++idbits;
+            const long double bound = (long double)mpq * (long double)W * (long double)std::max<int64_t>(dmax, 1);
+            int mode = DM_FAST;
+            if (g->opt_force_i128 || bound >= 0x1p62L) mode = DM_W128;
+            else if (W >= ((int64_t)1 << 31) || bound * (long double)((int64_t)1 << idbits) >= 0x1p62L || g->opt_force_wide)
+                mode = DM_W64;
+            ls.i128path = mode;
+            const long long qW64 = (long long)qW128, p64 = (long long)p;
+            logs.clear();
+            for (int it = 0;; ++it) {
+                const bool single = it == 0 && g->opt_singleton && (level > 0 || g->rows_distinct0);
+#define DIST_IT(MM, UU, QW, PP) dist_iteration<MM, UU>(g, wk, cur, lv0, lv1, bounds, QW, PP, qW128, T, tm, maxdeg, \
+                                                       idbits, single, lmoves, gmoves, newC, dcnt, vec)
+                if (mode == DM_W128) { if (unit) DIST_IT(DM_W128, true, (i128)qW128, (i128)p); else DIST_IT(DM_W128, false, (i128)qW128, (i128)p); }
+                else if (mode == DM_W64) { if (unit) DIST_IT(DM_W64, true, qW64, p64); else DIST_IT(DM_W64, false, qW64, p64); }
+                else { if (unit) DIST_IT(DM_FAST, true, qW64, p64); else DIST_IT(DM_FAST, false, qW64, p64); }
+#undef DIST_IT
+                CK(cudaMemcpyAsync(wk.h_carry, wk.carry, sizeof(Carry), cudaMemcpyDeviceToHost, st));
+                CK(cudaMemcpyAsync(wk.h_log, wk.log + (it % wk.log_cap), sizeof(IterLog), cudaMemcpyDeviceToHost, st));
+                if (g->opt_trace >= 2) {
+                    g->trace_labels.emplace_back(nl);
+                    CK(cudaMemcpyAsync(g->trace_labels.back().data(), wk.C, sizeof(int32_t) * nl, cudaMemcpyDeviceToHost, st));
+                }
+                CK(cudaStreamSynchronize(st));
+                tm.resolve();
+                logs.push_back(*wk.h_log);
+                const Carry& c = *wk.h_carry;
+                if (!c.more && !c.converged && !(g->opt_max_iters > 0 && c.iter >= g->opt_max_iters)) {
+                    int base = c.iter;   // log full: restart slots
+                    CK(cudaMemcpyAsync(&wk.carry->log_base, &base, sizeof(int), cudaMemcpyHostToDevice, st));
+                }
+                if (c.converged || (g->opt_max_iters > 0 && c.iter >= g->opt_max_iters)) break;
+            }
+            i128 N = N_start;
+            for (size_t it = 0; it < logs.size(); ++it) {
+                const IterCounters& c = logs[it].ctr;
+                N = log_N(logs[it]);
+                int64_t scanned = 0, kk = 0;
+                for (int b = 0; b < NBINS; ++b) { scanned += (int64_t)c.bin_deg[b]; kk += (int64_t)c.bin_k[b]; }
+                ls.edges_scanned += scanned;
+                ls.nominal_edges += gnnz;
+                if (g->opt_trace >= 1) {
+                    TraceRec r;
+                    r.v[0] = level; r.v[1] = (int64_t)it; r.v[2] = nl; r.v[3] = (int64_t)c.n_active;
+                    r.v[4] = (int64_t)c.n_pruned; r.v[5] = (int64_t)c.n_moved;
+                    r.v[6] = (int64_t)(N >> 64); r.v[7] = (int64_t)(uint64_t)N;
+                    r.v[8] = scanned; r.v[9] = kk; r.v[10] = 0; r.v[11] = 0;
+                    g->trace.push_back(r);
+                }
+            }
+            ls.iters = (int64_t)logs.size();
+            CK(cudaEventRecord(wk.ev[3], st));
+            // a8: relabel (replicated state: identical on every rank)
+            int32_t* minmem = dalloc<int32_t>(nl, st);
+            long long* pos = dalloc<long long>(nl + 1, st);
+            int32_t* newid = dalloc<int32_t>(nl, st);
+            k_fill_i32<<<grid_for(nl, 256, big), 256, 0, st>>>(minmem, nl, INT_MAX);
+            CKL();
+            k_minmember<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.C, minmem);
+            CKL();
+            k_minflag<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.C, minmem, pos);
+            CKL();
+            scan_excl(pos, pos, nl, st);
+            k_newid<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.C, minmem, pos, newid);
+            CKL();
+            k_compose<<<grid_for(n0, 256, big), 256, 0, st>>>(n0, newid, g->lab);
+            CKL();
+            long long kcomm = 0;
+            CK(cudaMemcpyAsync(&kcomm, pos + nl, sizeof(long long), cudaMemcpyDeviceToHost, st));
+            CK(cudaStreamSynchronize(st));
+            const bool stop = (kcomm == nl) || (max_levels > 0 && level + 1 >= max_levels) || (N - N_start < T);
+            DevCSR nxt;
+            if (!stop) dist_coarsen(g, wk, cur, nl, kcomm, newid, minmem, unit, nxt, bounds, maxdeg, dmax);
+            dfree(minmem, st);
+            dfree(pos, st);
+            dfree(newid, st);
+            CK(cudaEventRecord(wk.ev[4], st));
+            CK(cudaEventSynchronize(wk.ev[4]));
+            float ms1 = 0, ms2 = 0;
+            CK(cudaEventElapsedTime(&ms1, wk.ev[2], wk.ev[3]));
+            CK(cudaEventElapsedTime(&ms2, wk.ev[3], wk.ev[4]));
+            ls.ms_phase1 = ms1;
+            ls.ms_phase2 = ms2;
+            g->levels.push_back(ls);
+            if (cur_owned) { dfree(cur.rp, st); dfree(cur.col, st); dfree(cur.w, st); dfree(cur.row, st); }
+            if (stop) break;
+            cur = nxt;
+            cur_owned = true;
+        }
+        CK(cudaMemcpyAsync(wk.h_carry, wk.carry, sizeof(Carry), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        g->N = carry_N(wk.h_carry);
+        g->check_mismatch = 0;
+        CK(cudaEventRecord(wk.ev[1], st));
+        CK(cudaEventSynchronize(wk.ev[1]));
+        float ms = 0;
+        CK(cudaEventElapsedTime(&ms, wk.ev[0], wk.ev[1]));
+        g->run_ms = ms;
+        g->launches = g_launches - launches0;
+    } catch (CommError& e) {
+        dfree(lmoves, st); dfree(gmoves, st); dfree(newC, st); dfree(dcnt, st); dfree(vec, st);
+        set_err(GALA_E_NCCL, "%s", e.msg.c_str());
+        throw GalaError{GALA_E_NCCL};
+    } catch (...) {
+        dfree(lmoves, st); dfree(gmoves, st); dfree(newC, st); dfree(dcnt, st); dfree(vec, st);
+        throw;
+    }
+    dfree(lmoves, st); dfree(gmoves, st); dfree(newC, st); dfree(dcnt, st); dfree(vec, st);
     g->has_result = true;
 }
 
@@ -1107,11 +1565,6 @@ gala_status gala_run(gala_graph g, double gamma, double tol, int32_t max_levels)
     if (!(gamma > 0) || !(gamma < 1e12)) return set_err(GALA_E_INVALID, "gamma must be > 0");
     if (!(tol > 0)) return set_err(GALA_E_INVALID, "tol must be > 0");
     API_BEGIN
-    if (g->dist) {
-        dist_run(g->dist, gamma, tol, max_levels);
-        g->has_result = true;
-        return GALA_OK;
-    }
     if (g->W == 0) {
         // reading c18: no edges -> singletons, Q := 0
         CK(cudaSetDevice(g->device));
@@ -1128,7 +1581,8 @@ gala_status gala_run(gala_graph g, double gamma, double tol, int32_t max_levels)
         g->has_result = true;
         return GALA_OK;
     }
-    do_run(g, gamma, tol, max_levels);
+    if (g->di) do_run_dist(g, gamma, tol, max_levels);
+    else do_run(g, gamma, tol, max_levels);
     API_END
 }
 
@@ -1137,7 +1591,6 @@ static gala_status fetch_labels(gala_graph g, int32_t* out, int64_t n, int64_t* 
     if (!g->has_result) return set_err(GALA_E_STATE, "gala_run has not completed");
     if (n != g->n0) return set_err(GALA_E_INVALID, "n mismatch (%lld != %lld)", (long long)n, (long long)g->n0);
     API_BEGIN
-    if (g->dist) return dist_get_labels(g->dist, out, n, k, device);
     CK(cudaSetDevice(g->device));
     std::vector<int32_t> h;
     int32_t* dst = out;
@@ -1168,7 +1621,6 @@ gala_status gala_get_communities_device(gala_graph g, int32_t* d_labels, int64_t
 gala_status gala_modularity_numerator(gala_graph g, int64_t* n_hi, uint64_t* n_lo, int64_t* W, int64_t* p, int64_t* q) {
     if (!g) return set_err(GALA_E_INVALID, "null handle");
     if (!g->has_result) return set_err(GALA_E_STATE, "gala_run has not completed");
-    if (g->dist) dist_numerator(g->dist, &g->N, &g->W, &g->p, &g->q);
     if (n_hi) *n_hi = (int64_t)(g->N >> 64);
     if (n_lo) *n_lo = (uint64_t)g->N;
     if (W) *W = g->W;
@@ -1180,7 +1632,6 @@ gala_status gala_modularity_numerator(gala_graph g, int64_t* n_hi, uint64_t* n_l
 gala_status gala_modularity(gala_graph g, double* q) {
     if (!g || !q) return set_err(GALA_E_INVALID, "null argument");
     if (!g->has_result) return set_err(GALA_E_STATE, "gala_run has not completed");
-    if (g->dist) dist_numerator(g->dist, &g->N, &g->W, &g->p, &g->q);
     if (g->W == 0) { *q = 0.0; return GALA_OK; }
     *q = (double)((long double)g->N / ((long double)g->q * (long double)g->W * (long double)g->W));
     return GALA_OK;
@@ -1189,7 +1640,7 @@ gala_status gala_modularity(gala_graph g, double* q) {
 void gala_graph_free(gala_graph g) {
     if (!g) return;
     cudaSetDevice(g->device);
-    if (g->dist) dist_free(g->dist);
+    if (g->di) { delete g->di->comm; delete g->di; g->di = nullptr; }
     cudaStream_t st = g->stream;
     if (g->wk) { g->wk->release(); delete g->wk; g->wk = nullptr; }
     if (st) {
@@ -1220,6 +1671,7 @@ gala_status gala_set_option(gala_graph g, const char* key, int64_t value) {
     else if (k == "force_i128") g->opt_force_i128 = value != 0;
     else if (k == "force_wide") g->opt_force_wide = value != 0;
     else if (k == "singleton") g->opt_singleton = value != 0;
+    else if (k == "verbose") g->opt_verbose = (int)value;
     else if (k == "cuda_graph") g->opt_cuda_graph = value != 0;
     else if (k == "log_cap") { if (value < 2 || value > (1 << 20)) return set_err(GALA_E_INVALID, "log_cap in [2, 2^20]"); g->opt_log_cap = (int)value; }
     else if (k == "hub_smem_slots") {
@@ -1237,28 +1689,26 @@ gala_status gala_set_option(gala_graph g, const char* key, int64_t value) {
         for (int i = 1; i < NBINS - 1; ++i)
             if (g->bins[i] < g->bins[i - 1]) return set_err(GALA_E_INVALID, "bin thresholds must be non-decreasing");
     } else if (k == "sync_mode") {
-        if (g->dist) dist_set_option(g->dist, key, value);
+        if (value < 0 || value > 2) return set_err(GALA_E_INVALID, "sync_mode: 0 adaptive, 1 dense, 2 sparse");
+        g->sync_mode = (int)value;
+        if (g->di) g->di->sync_mode = (int)value;
     } else return set_err(GALA_E_INVALID, "unknown option %s", key);
-    if (g->dist) dist_set_option(g->dist, key, value);
     return GALA_OK;
 }
 
 gala_status gala_get_trace_count(gala_graph g, int64_t* count) {
     if (!g || !count) return set_err(GALA_E_INVALID, "null argument");
-    if (g->dist) { *count = dist_trace_count(g->dist); return GALA_OK; }
     *count = (int64_t)g->trace.size();
     return GALA_OK;
 }
 gala_status gala_get_trace_record(gala_graph g, int64_t i, int64_t* out12) {
     if (!g || !out12) return set_err(GALA_E_INVALID, "null argument");
-    if (g->dist) return dist_trace_record(g->dist, i, out12);
     if (i < 0 || i >= (int64_t)g->trace.size()) return set_err(GALA_E_INVALID, "record index out of range");
     memcpy(out12, g->trace[i].v, sizeof(int64_t) * 12);
     return GALA_OK;
 }
 gala_status gala_get_trace_labels(gala_graph g, int64_t i, int32_t* out, int64_t n_level) {
     if (!g || !out) return set_err(GALA_E_INVALID, "null argument");
-    if (g->dist) return dist_trace_labels(g->dist, i, out, n_level);
     if (i < 0 || i >= (int64_t)g->trace_labels.size()) return set_err(GALA_E_INVALID, "no labels for record (trace < 2?)");
     if ((int64_t)g->trace_labels[i].size() != n_level) return set_err(GALA_E_INVALID, "n_level mismatch");
     memcpy(out, g->trace_labels[i].data(), sizeof(int32_t) * n_level);
@@ -1286,6 +1736,13 @@ gala_status gala_get_stats(gala_graph g, char* buf, int64_t cap, int64_t* needed
              (long long)g->n0, (long long)g->nnz0, (long long)g->W, (long long)g->p, (long long)g->q, g->run_ms,
              (long long)g->dp_mismatch, g->launches, g->check_mismatch);
     s += tmp;
+    if (g->di) {
+        snprintf(tmp, sizeof tmp, "\"dist\":{\"rank\":%d,\"world\":%d,\"v0\":%lld,\"v1\":%lld,\"dense_iters\":%lld,"
+                 "\"sparse_iters\":%lld,\"bytes_exchanged\":%.0f},",
+                 g->di->comm->rank, g->di->comm->world, g->di->v0, g->di->v1, g->di->n_dense, g->di->n_sparse,
+                 g->di->bytes_exchanged);
+        s += tmp;
+    }
     s += "\"levels\":[";
     for (size_t i = 0; i < g->levels.size(); ++i) {
         const LevelStat& l = g->levels[i];
@@ -1327,6 +1784,132 @@ gala_status gala_partition_ranges(int64_t n, const int64_t* row_ptr, int world, 
     }
     bounds[world] = n;
     return GALA_OK;
+}
+
+gala_status gala_nccl_unique_id(void* out128) {
+    if (!out128) return set_err(GALA_E_INVALID, "null argument");
+    if (!nccl_api().load()) return set_err(GALA_E_NCCL, "libnccl.so.2 could not be loaded");
+    ncclUniqueId id;
+    ncclResult_t r = nccl_api().GetUniqueId(&id);
+    if (r != ncclSuccess) return set_err(GALA_E_NCCL, "ncclGetUniqueId: %s", nccl_api().GetErrorString(r));
+    memset(out128, 0, 128);
+    memcpy(out128, &id, sizeof(id) < 128 ? sizeof(id) : 128);
+    return GALA_OK;
+}
+
+gala_status gala_loopback_unique_id(void* out128) {
+    if (!out128) return set_err(GALA_E_INVALID, "null argument");
+    static std::atomic<unsigned long long> counter{0};
+    memset(out128, 0, 128);
+    const unsigned long long c = ++counter;
+    memcpy(out128, "GALALOOP", 8);
+    memcpy(static_cast<char*>(out128) + 8, &c, sizeof(c));
+    return GALA_OK;
+}
+
+gala_status gala_graph_from_csr_dist(const void* uid128, int rank, int world, int device, int64_t n_global,
+                                     int64_t v_begin, int64_t v_end, const int64_t* local_row_ptr,
+                                     const int32_t* col_idx, const int64_t* weights, uintptr_t stream,
+                                     gala_graph* out) {
+    if (!out || !uid128 || !local_row_ptr) return set_err(GALA_E_INVALID, "null argument");
+    *out = nullptr;
+    if (world < 1 || rank < 0 || rank >= world) return set_err(GALA_E_INVALID, "bad rank/world");
+    if (n_global < 0 || n_global >= ((int64_t)1 << 31)) return set_err(GALA_E_INVALID, "n out of range");
+    if (v_begin < 0 || v_end < v_begin || v_end > n_global) return set_err(GALA_E_INVALID, "bad owned range");
+    const int64_t n_own = v_end - v_begin;
+    if (local_row_ptr[0] != 0 || local_row_ptr[n_own] < 0) return set_err(GALA_E_INVALID, "local row_ptr[0] != 0");
+    const bool loop = memcmp(uid128, "GALALOOP", 8) == 0;
+    if (!loop && !nccl_api().load()) return set_err(GALA_E_NCCL, "libnccl.so.2 could not be loaded");
+    gala_graph_s* g = new gala_graph_s();
+    PoolScope pool_scope(nullptr);
+    API_BEGIN
+    try {
+        init_graph_common(g, n_global, device, stream);
+        cudaStream_t st = g->stream;
+        g->di = new DistInfo();
+        try {
+            if (loop) g->di->comm = new LoopComm(uid128, rank, world);
+            else g->di->comm = new NcclComm(uid128, rank, world);
+        } catch (CommError& e) {
+            set_err(GALA_E_NCCL, "%s", e.msg.c_str());
+            throw GalaError{GALA_E_NCCL};
+        }
+        Comm& cm = *g->di->comm;
+        g->di->v0 = v_begin;
+        g->di->v1 = v_end;
+        // every rank's owned range (ranges must tile [0, n) in rank order)
+        const std::vector<int64_t> b0 = cm.allgather_host(v_begin, st), b1 = cm.allgather_host(v_end, st);
+        g->dbounds0.assign(world + 1, 0);
+        for (int r = 0; r < world; ++r) {
+            if (b0[r] != (r ? b1[r - 1] : 0)) { set_err(GALA_E_INVALID, "owned ranges must tile [0, n) in rank order"); throw GalaError{GALA_E_INVALID}; }
+            g->dbounds0[r] = b0[r];
+        }
+        g->dbounds0[world] = b1[world - 1];
+        if (g->dbounds0[world] != n_global) { set_err(GALA_E_INVALID, "owned ranges do not cover n"); throw GalaError{GALA_E_INVALID}; }
+        const int64_t nnz = local_row_ptr[n_own];
+        g->nnz0 = nnz;
+        g->g0.n = n_global;
+        g->g0.nnz = nnz;
+        g->g0.rp = dalloc<int64_t>(n_global + 1, st);
+        g->g0.col = dalloc<int32_t>(nnz, st);
+        int64_t* lrp = dalloc<int64_t>(n_own + 1, st);
+        CK(cudaMemcpyAsync(lrp, local_row_ptr, sizeof(int64_t) * (n_own + 1), cudaMemcpyHostToDevice, st));
+        k_expand_rp<<<grid_for(n_global + 1, 256, g->num_sms * 8), 256, 0, st>>>(n_global, v_begin, v_end, lrp, g->g0.rp);
+        CKL();
+        dfree(lrp, st);
+        if (nnz) CK(cudaMemcpyAsync(g->g0.col, col_idx, sizeof(int32_t) * nnz, cudaMemcpyHostToDevice, st));
+        if (weights) {
+            g->g0.w = dalloc<int64_t>(nnz, st);
+            CK(cudaMemcpyAsync(g->g0.w, weights, sizeof(int64_t) * nnz, cudaMemcpyHostToDevice, st));
+        }
+        finish_graph(g);
+        // unit-weight detection must agree on every rank
+        const std::vector<int64_t> u = cm.allgather_host(g->g0.w ? 0 : 1, st);
+        bool all_unit = true;
+        for (int64_t x : u) all_unit = all_unit && x;
+        if (!all_unit && !g->g0.w) {   // some rank has real weights: materialise ones here
+            g->g0.w = dalloc<int64_t>(std::max<int64_t>(nnz, 1), st);
+            k_fill_i64<<<grid_for(nnz, 256, g->num_sms * 8), 256, 0, st>>>(reinterpret_cast<long long*>(g->g0.w), nnz, 1);
+            CKL();
+        }
+        // replicate d (owned slices), then W and the max weighted degree over all vertices
+        std::vector<size_t> cb(world), db(world);
+        for (int r = 0; r < world; ++r) {
+            cb[r] = (size_t)(g->dbounds0[r + 1] - g->dbounds0[r]) * sizeof(int64_t);
+            db[r] = (size_t)g->dbounds0[r] * sizeof(int64_t);
+        }
+        int64_t* dfull = dalloc<int64_t>(std::max<int64_t>(n_global, 1), st);
+        cm.allgatherv(g->d0 + v_begin, dfull, cb, db, st);
+        dfree(g->d0, st);
+        g->d0 = dfull;
+        const int big = g->num_sms * 8;
+        i128* part = dalloc<i128>(big, st);
+        ull* ticket = dalloc<ull>(1, st);
+        i128* wsum = dalloc<i128>(1, st);
+        ull* mx = dalloc<ull>(1, st);
+        CK(cudaMemsetAsync(ticket, 0, sizeof(ull), st));
+        CK(cudaMemsetAsync(mx, 0, sizeof(ull), st));
+        k_sum_i128<<<grid_for(n_global, 256, big), 256, 0, st>>>(n_global, g->d0, part, ticket, wsum);
+        CKL();
+        k_max_i64<<<grid_for(n_global, 256, big), 256, 0, st>>>(n_global, g->d0, mx);
+        CKL();
+        i128 hW = 0;
+        ull hm = 0;
+        CK(cudaMemcpyAsync(&hW, wsum, sizeof(i128), cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(&hm, mx, sizeof(ull), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        dfree(part, st); dfree(ticket, st); dfree(wsum, st); dfree(mx, st);
+        if (hW >= ((i128)1 << 62)) { set_err(GALA_E_OVERFLOW, "total weight W >= 2^62"); throw GalaError{GALA_E_OVERFLOW}; }
+        g->W = (int64_t)hW;
+        g->maxw0 = (int64_t)hm;
+        const std::vector<int64_t> rd = cm.allgather_host(g->rows_distinct0 ? 1 : 0, st);
+        for (int64_t x : rd) g->rows_distinct0 = g->rows_distinct0 && x;
+    } catch (...) {
+        gala_graph_free(g);
+        throw;
+    }
+    *out = g;
+    API_END
 }
 
 }  // extern "C"

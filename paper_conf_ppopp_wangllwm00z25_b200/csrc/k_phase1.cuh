@@ -92,7 +92,7 @@ struct BinThresholds {
 #define PB_IPT 4
 
 template <typename ST>
-__global__ void __launch_bounds__(PB_BT) k_prune_bin(int n, const int64_t* __restrict__ rp,
+__global__ void __launch_bounds__(PB_BT) k_prune_bin(int vlo, int n, const int64_t* __restrict__ rp,
                                                      const int64_t* __restrict__ d, const int64_t* __restrict__ dp,
                                                      const int32_t* __restrict__ C, const int64_t* __restrict__ Sig,
                                                      const int32_t* __restrict__ size, int prune, ST qW, ST p,
@@ -106,7 +106,7 @@ __global__ void __launch_bounds__(PB_BT) k_prune_bin(int n, const int64_t* __res
 #pragma unroll
     for (int b = 0; b < NBINS; ++b) my_deg[b] = 0;
     const long long tile = (long long)PB_BT * PB_IPT;
-    for (long long t0 = (long long)blockIdx.x * tile; t0 < n; t0 += (long long)gridDim.x * tile) {
+    for (long long t0 = vlo + (long long)blockIdx.x * tile; t0 < n; t0 += (long long)gridDim.x * tile) {
         if (threadIdx.x < NBINS) s_cnt[threadIdx.x] = 0;
         int bin[PB_IPT];
         long long dv[PB_IPT], dpv[PB_IPT];
@@ -316,10 +316,11 @@ __global__ void __launch_bounds__(256) k_dp_delta(IterCounters* __restrict__ ctr
 // d'(v) = sum of w(v,u), u != v, C[u] == C[v]   (definition), edge-parallel:
 // every lane takes entries (row r, col u) 32 apart (4 in flight), equal rows of
 // a 32-entry chunk are summed with __match_any_sync and one atomic per row.
-__global__ void k_dp_zero(IterCounters* __restrict__ ctr, int n, int64_t* __restrict__ dp, long long nnz, int mode,
-                          long long fnum, long long fden) {
+__global__ void k_dp_zero(IterCounters* __restrict__ ctr, int vlo, int vhi, int64_t* __restrict__ dp, long long nnz,
+                          int mode, long long fnum, long long fden) {
     if (use_delta(ctr, nnz, mode, fnum, fden)) return;
-    for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x)
+    for (long long v = vlo + (long long)blockIdx.x * blockDim.x + threadIdx.x; v < vhi;
+         v += (long long)gridDim.x * blockDim.x)
         dp[v] = 0;
 }
 
@@ -370,12 +371,12 @@ __global__ void __launch_bounds__(256) k_dp_full(IterCounters* __restrict__ ctr,
 // mode 0: level start (N := N'), mode 1: iteration end.
 // ---------------------------------------------------------------------------
 template <int BT>
-__global__ void __launch_bounds__(BT) k_reduce(int n, const int64_t* __restrict__ dp, const int64_t* __restrict__ s,
-                                               const int64_t* __restrict__ Sig, long long* __restrict__ part_dc,
-                                               i128* __restrict__ part_s2, long long* __restrict__ part_min,
-                                               IterCounters* __restrict__ ctr, Carry* __restrict__ carry,
-                                               long long qW_hi, ull qW_lo, long long p, long long T_hi, ull T_lo,
-                                               int mode) {
+__global__ void __launch_bounds__(BT) k_reduce(int n, int dlo, int dhi, const int64_t* __restrict__ dp,
+                                               const int64_t* __restrict__ s, const int64_t* __restrict__ Sig,
+                                               long long* __restrict__ part_dc, i128* __restrict__ part_s2,
+                                               long long* __restrict__ part_min, IterCounters* __restrict__ ctr,
+                                               Carry* __restrict__ carry, long long qW_hi, ull qW_lo, long long p,
+                                               long long T_hi, ull T_lo, int mode) {
     __shared__ long long sh_dc[BT / 32];
     __shared__ i128 sh_s2[BT / 32];
     __shared__ long long sh_min[BT / 32];
@@ -385,10 +386,7 @@ __global__ void __launch_bounds__(BT) k_reduce(int n, const int64_t* __restrict_
     const long long stride = (long long)gridDim.x * BT;
     long long v = (long long)blockIdx.x * BT + threadIdx.x;
     for (; v + 3 * stride < n; v += 4 * stride) {
-        long long a0 = dp[v], a1 = dp[v + stride], a2 = dp[v + 2 * stride], a3 = dp[v + 3 * stride];
-        long long b0 = s[v], b1 = s[v + stride], b2 = s[v + 2 * stride], b3 = s[v + 3 * stride];
         long long g0 = Sig[v], g1 = Sig[v + stride], g2 = Sig[v + 2 * stride], g3 = Sig[v + 3 * stride];
-        dc += a0 + a1 + a2 + a3 + b0 + b1 + b2 + b3;
         s2 += (i128)g0 * g0 + (i128)g1 * g1 + (i128)g2 * g2 + (i128)g3 * g3;
         if (g0 > 0 && g0 < mn) mn = g0;
         if (g1 > 0 && g1 < mn) mn = g1;
@@ -396,11 +394,15 @@ __global__ void __launch_bounds__(BT) k_reduce(int n, const int64_t* __restrict_
         if (g3 > 0 && g3 < mn) mn = g3;
     }
     for (; v < n; v += stride) {
-        dc += dp[v] + s[v];
         long long sg = Sig[v];
         s2 += (i128)sg * sg;
         if (sg > 0 && sg < mn) mn = sg;
     }
+    v = dlo + (long long)blockIdx.x * BT + threadIdx.x;
+    for (; v + 3 * stride < dhi; v += 4 * stride)
+        dc += dp[v] + dp[v + stride] + dp[v + 2 * stride] + dp[v + 3 * stride] + s[v] + s[v + stride] +
+              s[v + 2 * stride] + s[v + 3 * stride];
+    for (; v < dhi; v += stride) dc += dp[v] + s[v];
     const int lane = lane_id(), wib = threadIdx.x >> 5;
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
@@ -451,6 +453,14 @@ __global__ void __launch_bounds__(BT) k_reduce(int n, const int64_t* __restrict_
             tdc += sh_dc[i];
             ts2 += sh_s2[i];
             tmn = sh_min[i] < tmn ? sh_min[i] : tmn;
+        }
+        carry->S2_hi = hi128(ts2);
+        carry->S2_lo = lo128(ts2);
+        carry->minSig = tmn;
+        carry->sumDC = tdc;
+        if (mode & 2) {   // multi-GPU: sumDC is rank-local; k_finish completes after the all-reduce
+            ctr->ticket = 0;
+            return;
         }
         i128 qW = mk128(qW_hi, qW_lo);
         i128 Nn = qW * (i128)tdc - (i128)p * ts2;

@@ -370,13 +370,24 @@ __global__ void __launch_bounds__(256) k_agg_big_insert(AggArgs a, const int32_t
 __global__ void __launch_bounds__(256) k_agg_big_emit(AggArgs a, const int32_t* __restrict__ bigc, int nbig,
                                                       const long long* __restrict__ goff, int* __restrict__ gkeys,
                                                       ull* __restrict__ gvals, const int* __restrict__ glist,
-                                                      const int* __restrict__ gcnt) {
-    for (int bi = blockIdx.x; bi < nbig; bi += gridDim.x) {
-        long long c = bigc[bi];
-        long long off = goff[bi];
-        int m = gcnt[bi];
-        agg_emit<ull>(a, c, m, glist + off / 2, gkeys + off, gvals + off, threadIdx.x, 256);
-        if (threadIdx.x == 0) a.dn[c] = m;
+                                                      const int* __restrict__ gcnt, int bpc) {
+    for (long long b = blockIdx.x; b < (long long)nbig * bpc; b += gridDim.x) {
+        const int bi = (int)(b / bpc), part = (int)(b % bpc);
+        const long long c = bigc[bi];
+        const long long off = goff[bi];
+        const int m = gcnt[bi];
+        const int lo = (int)((long long)m * part / bpc), hi = (int)((long long)m * (part + 1) / bpc);
+        const long long o = a.eoff[c];
+        const int* list = glist + off / 2;
+        for (int t = lo + threadIdx.x; t < hi; t += 256) {
+            const int slot = list[t];
+            const int key = gkeys[off + slot];
+            const int64_t val = (int64_t)gvals[off + slot];
+            a.tkey[o + t] = key;
+            a.tval[o + t] = val;
+            if (key == (int)c) a.snew[c] = val;
+        }
+        if (part == 0 && threadIdx.x == 0) a.dn[c] = m;
     }
 }
 
@@ -393,20 +404,37 @@ __global__ void k_agg_bigflag(long long k, const long long* __restrict__ ent, in
     }
 }
 
-// warp per community: copy its aggregated segment into the coarse CSR row
-__global__ void __launch_bounds__(256) k_compact(long long k, const long long* __restrict__ eoff,
+// largest c in [lo, hi] with off[c] <= t
+__device__ __forceinline__ long long seg_search(const long long* __restrict__ off, long long lo, long long hi,
+                                                long long t) {
+    while (lo < hi) {
+        long long mid = (lo + hi + 1) >> 1;
+        if (off[mid] <= t) lo = mid; else hi = mid - 1;
+    }
+    return lo;
+}
+
+// thread per coarse entry t: row c = segment of t in rp_new (bounded search per
+// 256-entry block), copy from the aggregated segment at eoff[c]
+__global__ void __launch_bounds__(256) k_compact(long long k, long long nnz_new, const long long* __restrict__ eoff,
                                                  const long long* __restrict__ rp_new, const int* __restrict__ tkey,
                                                  const int64_t* __restrict__ tval, int32_t* __restrict__ col_new,
                                                  int64_t* __restrict__ w_new, int32_t* __restrict__ row_new) {
-    const int lane = lane_id();
-    const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
-    for (long long c = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < k; c += nw) {
-        long long o = eoff[c], r = rp_new[c], m = rp_new[c + 1] - r;
-        for (long long t = lane; t < m; t += 32) {
-            col_new[r + t] = tkey[o + t];
-            w_new[r + t] = tval[o + t];
-            row_new[r + t] = (int32_t)c;
+    __shared__ long long s_lo, s_hi;
+    for (long long t0 = (long long)blockIdx.x * 256; t0 < nnz_new; t0 += (long long)gridDim.x * 256) {
+        const long long last = t0 + 255 < nnz_new ? t0 + 255 : nnz_new - 1;
+        if (threadIdx.x == 0) s_lo = seg_search(rp_new, 0, k - 1, t0);
+        if (threadIdx.x == 32) s_hi = seg_search(rp_new, 0, k - 1, last);
+        __syncthreads();
+        const long long t = t0 + threadIdx.x;
+        if (t < nnz_new) {
+            const long long c = seg_search(rp_new, s_lo, s_hi, t);
+            const long long src = eoff[c] + (t - rp_new[c]);
+            col_new[t] = tkey[src];
+            w_new[t] = tval[src];
+            row_new[t] = (int32_t)c;
         }
+        __syncthreads();
     }
 }
 

@@ -1,0 +1,93 @@
+"""Multi-GPU path (§8(e), a10) exercised on one GPU: `world` ranks run as threads
+of one process through the loopback communicator (test hook); the partitioned
+algorithm (owned-range prune/decide, dense/sparse label exchange, replicated
+Sigma_tot updates, all-reduced counters, distributed coarsening and
+re-partitioning) must reproduce the oracle bit for bit at every iteration."""
+import threading
+
+import numpy as np
+import pytest
+
+import graphgen as gg
+import oracle
+import paper_conf_ppopp_wangllwm00z25_b200 as gala
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _need_gpu():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+
+
+def run_dist(g, world, gamma=1.0, sync_mode=0, trace=2, **opts):
+    bounds = gala.partition_ranges(g.row_ptr, world)
+    uid = gala.loopback_unique_id()
+    out = [None] * world
+    err = []
+
+    def worker(r):
+        try:
+            lrp, lcol, lw = gala.local_rows(g.row_ptr, g.col, g.w, bounds[r], bounds[r + 1])
+            h = gala.Graph.from_csr_dist(uid, r, world, 0, g.n, int(bounds[r]), int(bounds[r + 1]), lrp, lcol, lw)
+            h.set_option("trace", trace)
+            h.set_option("sync_mode", sync_mode)
+            for k, v in opts.items():
+                h.set_option(k, v)
+            h.run(gamma=gamma)
+            out[r] = dict(labels=h.communities(), N=h.numerator()[0], trace=h.trace(labels=trace >= 2),
+                          stats=h.stats())
+            h.free()
+        except Exception as e:  # noqa: BLE001
+            err.append(e)
+
+    ts = [threading.Thread(target=worker, args=(r,)) for r in range(world)]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join(timeout=600)
+    if err:
+        raise err[0]
+    return out
+
+
+def check(g, world, gamma=1.0, sync_mode=0, **opts):
+    o = oracle.louvain(g, gamma=gamma, prune=True, trace=2)
+    res = run_dist(g, world, gamma=gamma, sync_mode=sync_mode, **opts)
+    for r in res:
+        assert np.array_equal(r["labels"], o.labels)
+        assert r["N"] == o.N
+        assert len(r["trace"]) == len(o.records)
+        for x, y in zip(o.records, r["trace"]):
+            assert (x.level, x.iter) == (y["level"], y["iter"])
+            assert np.array_equal(x.labels, y["labels"]), f"level {x.level} iter {x.iter}"
+            assert x.N == y["N"] and x.n_moved == y["n_moved"]
+            assert x.n_active == y["n_active"] and x.n_pruned == y["n_pruned"]
+    return res
+
+
+@pytest.mark.parametrize("world", [2, 3, 4])
+def test_dist_lfr_small(world):
+    res = check(gg.make("lfr_small"), world)
+    d = res[0]["stats"]["dist"]
+    assert d["world"] == world and d["dense_iters"] + d["sparse_iters"] > 0
+
+
+@pytest.mark.parametrize("sync_mode", [1, 2])
+def test_dist_forced_sync_modes(sync_mode):
+    res = check(gg.make("rmat_small"), 2, sync_mode=sync_mode)
+    d = res[0]["stats"]["dist"]
+    assert (d["dense_iters"] if sync_mode == 1 else d["sparse_iters"]) > 0
+    assert (d["sparse_iters"] if sync_mode == 1 else d["dense_iters"]) == 0
+
+
+def test_dist_karate_and_weighted():
+    check(gg.karate(), 2)
+    g = gg.random_graph(400, 3000, seed=77, max_w=5, self_loops=4)
+    check(g, 3, gamma=1.5)
+
+
+def test_dist_more_ranks_than_busy_rows():
+    check(gg.make("karate"), 4)

@@ -10,6 +10,8 @@ d = g.degrees()
 print(f"{name}: n={g.n} nnz={g.nnz} maxdeg={d.max()} isolated={(d == 0).sum()} gen={tg:.1f}s", flush=True)
 h = gala.Graph.from_graph(g)
 h.set_option("trace", 1)
+import os
+if os.environ.get("GALA_VERBOSE"): h.set_option("verbose", 1)
 for i in range(3):
     torch.cuda.synchronize(); t = time.time(); h.run(); torch.cuda.synchronize(); dt = time.time() - t
 st = h.stats()
