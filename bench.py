@@ -406,7 +406,7 @@ def run_dist(args, rank, world, local_rank):
     L = gala.lib()
     lab_host = np.empty(g.n, dtype=np.int32)
     for i in range(args.warmup + args.steps):
-        def e2e():
+        def e2e():   # same uid: the library reuses its cached NCCL communicator
             hh = gala.Graph.from_csr_dist(uid[0], rank, world, dev, g.n, v0, v1, lrp, lcol, lw,
                                           stream=stream.cuda_stream)
             hh.run()

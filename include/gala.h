@@ -209,7 +209,10 @@ gala_status gala_loopback_unique_id(void* out128);
  *   v_begin/end : owned vertex range (ranges tile [0, n_global) in rank order)
  *   local_row_ptr : host int64[v_end - v_begin + 1], local_row_ptr[0] = 0
  *   col_idx     : host int32[local nnz], GLOBAL vertex ids
- *   weights     : host int64[local nnz] or NULL (NULL must be used on all ranks alike)
+ *   weights     : host int64[local nnz] or NULL
+ * The NCCL communicator is created on the first call with a given uid and
+ * cached for the life of the process; later handles built with the same uid
+ * (on the same ranks) reuse it.
  */
 gala_status gala_graph_from_csr_dist(const void* uid128, int rank, int world, int device,
                                      int64_t n_global, int64_t v_begin, int64_t v_end,

@@ -99,16 +99,19 @@ struct NcclComm : Comm {
     void allreduce_sum_i64(int64_t* buf, size_t count, cudaStream_t st) override {
         ck(api.AllReduce(buf, buf, count, ncclInt64, ncclSum, comm, st));
     }
+    int64_t* scratch = nullptr;   // world + 1 int64, allocated once
+    int64_t* hscratch = nullptr;  // pinned mirror
     std::vector<int64_t> allgather_host(int64_t x, cudaStream_t st) override {
-        int64_t* d = nullptr;
-        cudaMallocAsync(&d, sizeof(int64_t) * (world + 1), st);
-        cudaMemcpyAsync(d + world, &x, sizeof(int64_t), cudaMemcpyHostToDevice, st);
-        ck(api.AllGather(d + world, d, 1, ncclInt64, comm, st));
-        std::vector<int64_t> out(world);
-        cudaMemcpyAsync(out.data(), d, sizeof(int64_t) * world, cudaMemcpyDeviceToHost, st);
-        cudaFreeAsync(d, st);
+        if (!scratch) {
+            cudaMalloc(&scratch, sizeof(int64_t) * (world + 1));
+            cudaMallocHost(&hscratch, sizeof(int64_t) * (world + 1));
+        }
+        hscratch[world] = x;
+        cudaMemcpyAsync(scratch + world, hscratch + world, sizeof(int64_t), cudaMemcpyHostToDevice, st);
+        ck(api.AllGather(scratch + world, scratch, 1, ncclInt64, comm, st));
+        cudaMemcpyAsync(hscratch, scratch, sizeof(int64_t) * world, cudaMemcpyDeviceToHost, st);
         cudaStreamSynchronize(st);
-        return out;
+        return std::vector<int64_t>(hscratch, hscratch + world);
     }
 };
 
@@ -188,15 +191,20 @@ struct LoopComm : Comm {
                 cudaMemcpyAsync(static_cast<char*>(recv) + displs[r], sh->ptr[r], counts[r], cudaMemcpyDeviceToDevice, st);
         finish(st);
     }
+    int64_t* tmp = nullptr;
+    size_t tmp_cap = 0;
     void allreduce_sum_i64(int64_t* buf, size_t count, cudaStream_t st) override {
-        int64_t* tmp = nullptr;
-        cudaMallocAsync(&tmp, sizeof(int64_t) * count * world + 8, st);
+        if (tmp_cap < count * world) {
+            cudaStreamSynchronize(st);
+            if (tmp) cudaFree(tmp);
+            tmp_cap = count * world + 64;
+            cudaMalloc(&tmp, sizeof(int64_t) * tmp_cap);
+        }
         publish(buf, st);
         for (int r = 0; r < world; ++r)
             cudaMemcpyAsync(tmp + (size_t)r * count, sh->ptr[r], sizeof(int64_t) * count, cudaMemcpyDeviceToDevice, st);
         finish(st);   // everyone has copied every buffer before anyone overwrites its own
         k_sum_rows_i64<<<(unsigned)std::min<size_t>((count + 255) / 256 + 1, 1024), 256, 0, st>>>(buf, tmp, count, world);
-        cudaFreeAsync(tmp, st);
     }
     std::vector<int64_t> allgather_host(int64_t x, cudaStream_t st) override {
         cudaStreamSynchronize(st);

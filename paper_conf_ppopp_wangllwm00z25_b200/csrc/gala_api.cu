@@ -980,6 +980,22 @@ struct DistInfo {
     double bytes_exchanged = 0;
 };
 
+// Communicators are created once per (uid, rank) and cached for the process
+// lifetime: handles built with the same uid share one NCCL communicator, so
+// rebuilding a graph (e.g. end-to-end timing) does not re-run ncclCommInitRank.
+static Comm* comm_for(const void* uid, int rank, int world, bool loop) {
+    static std::mutex mu;
+    static std::map<std::string, Comm*> cache;
+    std::string key(static_cast<const char*>(uid), 128);
+    key += std::to_string(rank) + "/" + std::to_string(world);
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = cache.find(key);
+    if (it != cache.end()) return it->second;
+    Comm* c = loop ? static_cast<Comm*>(new LoopComm(uid, rank, world)) : static_cast<Comm*>(new NcclComm(uid, rank, world));
+    cache[key] = c;
+    return c;
+}
+
 static std::vector<size_t> prefix_bytes(const std::vector<size_t>& c) {
     std::vector<size_t> d(c.size(), 0);
     for (size_t i = 1; i < c.size(); ++i) d[i] = d[i - 1] + c[i - 1];
@@ -996,6 +1012,7 @@ static void dist_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, long long
     cudaStream_t st = g->stream;
     const long long n = G.n;
     const int big = g->num_sms * 8;
+    VTimer vt(g);
     k_iter_begin<<<1, 128, 0, st>>>(wk.ctr);
     CKL();
     BinThresholds th;
@@ -1005,6 +1022,7 @@ static void dist_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, long long
         wk.ncap, th);
     CKL();
     launch_decide<M, UNIT>(g, wk, G, qW, p, tm, maxdeg, idbits, single);
+    vt.lap("dist: prune+decide");
     CK(cudaMemsetAsync(dcnt, 0, 2 * sizeof(ull), st));
     k_collect_moves<<<grid_for(lv1 - lv0, 256, big), 256, 0, st>>>(wk.ctr, wk.queues, wk.ncap, wk.nextC, lmoves, dcnt);
     CKL();
@@ -1012,6 +1030,7 @@ static void dist_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, long long
     CK(cudaMemcpyAsync(&mloc, dcnt, sizeof(ull), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
     const std::vector<int64_t> cnts = cm.allgather_host((int64_t)mloc, st);
+    vt.lap("dist: collect+count");
     long long total = 0;
     for (int64_t c : cnts) total += c;
     const double sparse_bytes = 8.0 * (double)total, dense_bytes = 4.0 * (double)n;
@@ -1038,6 +1057,7 @@ static void dist_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, long long
         di.n_dense++;
         di.bytes_exchanged += dense_bytes;
     }
+    vt.lap(sparse ? "dist: exchange sparse" : "dist: exchange dense");
     k_apply_list<<<grid_for(total, 256, big), 256, 0, st>>>(gmoves, total, wk.C, wk.Sig, wk.size, wk.d, wk.stamp,
                                                              wk.carry, wk.ctr);
     CKL();
@@ -1049,6 +1069,7 @@ static void dist_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, long long
                                                                                      wk.C, wk.dp, 0, 1, 2);
         CKL();
     }
+    vt.lap("dist: apply+dp");
     k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>((int)n, (int)lv0, (int)lv1, wk.dp, wk.s, wk.Sig, wk.part_dc,
                                                   wk.part_s2, wk.part_min, wk.ctr, wk.carry, 0, 0, 0, 0, 0, 3);
     CKL();
@@ -1060,6 +1081,7 @@ static void dist_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, long long
     CKL();
     k_record<<<1, 32, 0, st>>>(wk.ctr, wk.carry, wk.log, wk.log_cap, g->opt_max_iters, 0ull);
     CKL();
+    vt.lap("dist: reduce+allreduce");
 }
 
 // merge the partial coarse rows of every rank into the full coarse graph, then keep rows [lo, hi)
@@ -1640,7 +1662,7 @@ gala_status gala_modularity(gala_graph g, double* q) {
 void gala_graph_free(gala_graph g) {
     if (!g) return;
     cudaSetDevice(g->device);
-    if (g->di) { delete g->di->comm; delete g->di; g->di = nullptr; }
+    if (g->di) { delete g->di; g->di = nullptr; }   // communicators are cached (comm_for)
     cudaStream_t st = g->stream;
     if (g->wk) { g->wk->release(); delete g->wk; g->wk = nullptr; }
     if (st) {
@@ -1828,8 +1850,7 @@ gala_status gala_graph_from_csr_dist(const void* uid128, int rank, int world, in
         cudaStream_t st = g->stream;
         g->di = new DistInfo();
         try {
-            if (loop) g->di->comm = new LoopComm(uid128, rank, world);
-            else g->di->comm = new NcclComm(uid128, rank, world);
+            g->di->comm = comm_for(uid128, rank, world, loop);
         } catch (CommError& e) {
             set_err(GALA_E_NCCL, "%s", e.msg.c_str());
             throw GalaError{GALA_E_NCCL};
