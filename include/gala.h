@@ -133,7 +133,8 @@ void gala_graph_free(gala_graph g);
 /*
  * gala_set_option — tuning / test hooks.  Options never change results
  * (labels are identical for every setting) except "max_iters" (a per-level
- * iteration cap honoured identically by the oracle) and "prune_mode".
+ * iteration cap honoured identically by the oracle) and "prune" (pruning
+ * changes which vertices are evaluated; the oracle takes the same flag).
  *   "prune"          0/1   MG pruning (Eq. 6/7), default 1
  *   "trace"          0/1/2 per-iteration records; 2 also copies labels each iteration
  *   "check"          0/1   debug: verify maintained d'(v) against its definition
@@ -146,6 +147,8 @@ void gala_graph_free(gala_graph g);
  *   "force_i128"     0/1   use the 128-bit gain path even when 64-bit suffices
  *   "force_wide"     0/1   use unpacked 64-bit gains / aggregates (no packed keys)
  *   "singleton"      0/1   first iteration of a level via the singleton fast path (default 1)
+ *   "ckey"           0/1   keep a per-entry copy of C[col] on level 0, maintained by the delta
+ *                          update (default 0; trades nnz*4 bytes for one gather per entry)
  *   "hub_smem_slots" power of two in [64, 16384], shared-memory slots of the block hash table
  *   "cuda_graph"     0/1   run each level's iterations as a conditional CUDA graph (default 1)
  *   "log_cap"        device iteration-log capacity (default 4096)

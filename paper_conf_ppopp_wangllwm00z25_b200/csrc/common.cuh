@@ -62,6 +62,8 @@ struct Carry {
     int iter;               // iteration index within the level (also the d' stamp id)
     int more;               // loop condition written by k_record
     int log_base;           // log slot of iteration `log_base` is 0
+    int ckey_valid;         // the per-entry community array matches C (set by full d' passes)
+    int pad2;
 };
 
 // One record per phase-1 iteration, written on the device by k_record.

@@ -62,11 +62,11 @@ static thread_local long long g_launches = 0;
 
 // ------------------------------------------------------------------ kernel classes
 enum KClass {
-    KC_PRUNE = 0, KC_DEC_S4, KC_DEC_S8, KC_DEC_S16, KC_DEC_S32, KC_DEC_WARP, KC_DEC_WARP2, KC_DEC_BLOCK,
+    KC_PRUNE = 0, KC_DEC_SMALL, KC_DEC_WARP, KC_DEC_WARP2, KC_DEC_BLOCK,
     KC_APPLY, KC_DP, KC_REDUCE, KC_INIT, KC_PHASE2, KC_COUNT
 };
-static const char* kc_names[KC_COUNT] = {"prune_bin", "decide_sub4", "decide_sub8", "decide_sub16",
-                                         "decide_sub32", "decide_warp", "decide_warp512", "decide_block", "apply",
+static const char* kc_names[KC_COUNT] = {"prune_bin", "decide_small", "decide_warp", "decide_warp512",
+                                         "decide_block", "apply",
                                          "dp_update", "reduce", "level_init", "phase2"};
 
 struct TraceRec {
@@ -103,6 +103,8 @@ struct gala_graph_s {
     int opt_prune = 1, opt_trace = 0, opt_check = 0, opt_timing = 0, opt_max_iters = 0;
     int opt_delta = 2, opt_force_i128 = 0, opt_force_wide = 0, opt_cuda_graph = 1, opt_log_cap = 4096, opt_singleton = 1, opt_verbose = 0;
     bool rows_distinct0 = false;   // level-0 rows strictly increasing (no duplicate entries)
+    int32_t* rev0 = nullptr;       // level-0 reverse-entry index (enables the per-entry community array)
+    int opt_ckey = 0;
     int bins[NBINS - 1] = {4, 8, 16, 32, 128, 512};
     int hub_smem_slots = 4096;
     // results
@@ -232,6 +234,7 @@ struct Work {
     int64_t ncap, nnzcap;
     int32_t *C = nullptr, *size = nullptr, *stamp = nullptr, *mv_v = nullptr, *mv_old = nullptr, *nextC = nullptr;
     QRec* queues = nullptr;
+    int32_t* ckey = nullptr;   // level-0 per-entry neighbour community
     int64_t *Sig = nullptr, *d = nullptr, *s = nullptr, *dp = nullptr;
     IterCounters* ctr = nullptr;
     Carry* carry = nullptr;
@@ -252,7 +255,7 @@ struct Work {
     void release() {
         for (auto& e : ev) if (e) { cudaEventDestroy(e); e = nullptr; }
         dfree(C, st); dfree(size, st); dfree(stamp, st); dfree(mv_v, st); dfree(mv_old, st); dfree(nextC, st);
-        dfree(queues, st); dfree(Sig, st); dfree(d, st); dfree(s, st); dfree(dp, st); dfree(ctr, st);
+        dfree(queues, st); dfree(ckey, st); dfree(Sig, st); dfree(d, st); dfree(s, st); dfree(dp, st); dfree(ctr, st);
         dfree(carry, st); dfree(log, st); dfree(part_dc, st); dfree(part_min, st); dfree(part_s2, st);
         dfree(gkeys, st); dfree(gvals, st); dfree(glist, st);
         if (h_log) cudaFreeHost(h_log);
@@ -266,12 +269,17 @@ struct Work {
 #define BLOCK_E 4
 
 // ------------------------------------------------------------------ launch helpers
-template <int MAXDEG, int M>
+// the per-entry neighbour-community array is used on level 0 of single-GPU runs
+static bool use_ckey(const gala_graph_s* g, const Work& wk, const DevCSR& G) {
+    return g->opt_ckey && g->rev0 && wk.ckey && !g->di && G.col == g->g0.col;
+}
+
+template <int GW, int MAXDEG, int M>
 static void set_warp_smem() {
-    CK(cudaFuncSetAttribute(k_decide_warp<MAXDEG, M, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                            (int)WarpSmem<MAXDEG, M>::bytes));
-    CK(cudaFuncSetAttribute(k_decide_warp<MAXDEG, M, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                            (int)WarpSmem<MAXDEG, M>::bytes));
+    CK(cudaFuncSetAttribute(k_decide_warp<GW, MAXDEG, M, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)WarpSmem<GW, MAXDEG, M>::bytes));
+    CK(cudaFuncSetAttribute(k_decide_warp<GW, MAXDEG, M, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)WarpSmem<GW, MAXDEG, M>::bytes));
 }
 template <int M>
 static size_t block_smem_bytes(int cap) { return (size_t)cap * (sizeof(typename ModeT<M>::VT) + 2 * sizeof(int)); }
@@ -282,21 +290,17 @@ static void launch_single(gala_graph_s* g, Work& wk, const DecideArgs& a, typena
     const long long qs = wk.ncap;
     const int grid = g->num_sms * 8;
     cudaStream_t st = g->stream;
-    static const int kcs[NBINS] = {KC_DEC_S4, KC_DEC_S8, KC_DEC_S16, KC_DEC_S32, KC_DEC_WARP, KC_DEC_WARP2, KC_DEC_BLOCK};
-    for (int b = 0; b < NBINS; ++b) {
-        if (b > BIN_S32 && maxdeg <= g->bins[b - 1]) break;
-        cudaEvent_t e = tm.begin();
-        const QRec* q = wk.queues + b * qs;
-        // G lanes per vertex with 4 row entries per lane in flight: G ~ deg / 4
-        switch (b) {
-            case BIN_S4: k_decide_single<1, M, UNIT><<<grid, 256, 0, st>>>(q, b, a, qW, p); break;
-            case BIN_S8: k_decide_single<2, M, UNIT><<<grid, 256, 0, st>>>(q, b, a, qW, p); break;
-            case BIN_S16: k_decide_single<4, M, UNIT><<<grid, 256, 0, st>>>(q, b, a, qW, p); break;
-            case BIN_S32: k_decide_single<8, M, UNIT><<<grid, 256, 0, st>>>(q, b, a, qW, p); break;
-            default: k_decide_single<32, M, UNIT><<<grid, 256, 0, st>>>(q, b, a, qW, p); break;
-        }
+    cudaEvent_t e = tm.begin();
+    k_decide_single_small<M, UNIT><<<grid, 256, 0, st>>>(wk.queues, qs, a, qW, p);
+    CKL();
+    tm.end(KC_DEC_SMALL, e);
+    static const int kcs[3] = {KC_DEC_WARP, KC_DEC_WARP2, KC_DEC_BLOCK};
+    for (int b = BIN_WARP; b < NBINS; ++b) {
+        if (maxdeg <= g->bins[b - 1]) break;
+        e = tm.begin();
+        k_decide_single<M, UNIT><<<grid, 256, 0, st>>>(wk.queues + b * qs, b, a, qW, p);
         CKL();
-        tm.end(kcs[b], e);
+        tm.end(kcs[b - BIN_WARP], e);
     }
 }
 
@@ -306,6 +310,8 @@ static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, typename M
     DecideArgs a;
     a.rp = G.rp; a.col = G.col; a.w = G.w; a.C = wk.C; a.Sig = wk.Sig; a.size = wk.size; a.d = wk.d;
     a.dp = wk.dp; a.nextC = wk.nextC; a.ctr = wk.ctr; a.check = g->opt_check;
+    a.ckey = use_ckey(g, wk, G) ? wk.ckey : nullptr;
+    a.ckey_valid = &wk.carry->ckey_valid;
     a.idbits = idbits;
     a.idmask = (1LL << idbits) - 1;
     if (single) return launch_single<M, UNIT>(g, wk, a, qW, p, tm, maxdeg);
@@ -314,29 +320,17 @@ static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, typename M
     cudaStream_t st = g->stream;
     cudaEvent_t e;
     e = tm.begin();
-    k_decide_sub<4, 4, M, UNIT><<<grid, 256, 0, st>>>(wk.queues + BIN_S4 * qs, BIN_S4, a, qW, p);
+    k_decide_small<M, UNIT><<<grid, 256, 0, st>>>(wk.queues, qs, a, qW, p);
     CKL();
-    tm.end(KC_DEC_S4, e);
+    tm.end(KC_DEC_SMALL, e);
     e = tm.begin();
-    k_decide_sub<8, 4, M, UNIT><<<grid, 256, 0, st>>>(wk.queues + BIN_S8 * qs, BIN_S8, a, qW, p);
-    CKL();
-    tm.end(KC_DEC_S8, e);
-    e = tm.begin();
-    k_decide_sub<16, 2, M, UNIT><<<grid, 256, 0, st>>>(wk.queues + BIN_S16 * qs, BIN_S16, a, qW, p);
-    CKL();
-    tm.end(KC_DEC_S16, e);
-    e = tm.begin();
-    k_decide_sub<32, 2, M, UNIT><<<grid, 256, 0, st>>>(wk.queues + BIN_S32 * qs, BIN_S32, a, qW, p);
-    CKL();
-    tm.end(KC_DEC_S32, e);
-    e = tm.begin();
-    k_decide_warp<128, M, UNIT><<<grid, 32 * WarpSmem<128, M>::WPB, WarpSmem<128, M>::bytes, st>>>(
+    k_decide_warp<32, 128, M, UNIT><<<grid, 32 * WarpSmem<32, 128, M>::WPB, WarpSmem<32, 128, M>::bytes, st>>>(
         wk.queues + BIN_WARP * qs, BIN_WARP, a, qW, p);
     CKL();
     tm.end(KC_DEC_WARP, e);
     if (maxdeg > g->bins[BIN_WARP]) {
         e = tm.begin();
-        k_decide_warp<512, M, UNIT><<<grid, 32 * WarpSmem<512, M>::WPB, WarpSmem<512, M>::bytes, st>>>(
+        k_decide_warp<32, 512, M, UNIT><<<grid, 32 * WarpSmem<32, 512, M>::WPB, WarpSmem<32, 512, M>::bytes, st>>>(
             wk.queues + BIN_WARP2 * qs, BIN_WARP2, a, qW, p);
         CKL();
         tm.end(KC_DEC_WARP2, e);
@@ -375,13 +369,16 @@ static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, typename
     CKL();
     tm.end(KC_APPLY, e);
     e = tm.begin();
+    const bool ck = use_ckey(g, wk, G);
     k_dp_delta<UNIT><<<big, 256, 0, st>>>(wk.ctr, G.rp, G.col, G.w, wk.C, wk.mv_v, wk.mv_old, wk.stamp, wk.dp,
-                                          wk.carry, G.nnz, g->opt_delta, 1, 2);
+                                          wk.carry, G.nnz, g->opt_delta, 1, 2, ck ? wk.ckey : nullptr,
+                                          ck ? g->rev0 : nullptr);
     CKL();
     k_dp_zero<<<big, 256, 0, st>>>(wk.ctr, 0, n, wk.dp, G.nnz, g->opt_delta, 1, 2);
     CKL();
     k_dp_full<UNIT><<<grid_for((G.nnz + 127) / 128 * 32, 256, big), 256, 0, st>>>(wk.ctr, G.nnz, G.row, G.col, G.w,
-                                                                                 wk.C, wk.dp, g->opt_delta, 1, 2);
+                                                                                 wk.C, wk.dp, g->opt_delta, 1, 2,
+                                                                                 ck ? wk.ckey : nullptr, &wk.carry->ckey_valid);
     CKL();
     tm.end(KC_DP, e);
     e = tm.begin();
@@ -497,7 +494,8 @@ static void account_bytes(gala_graph_s* g, const IterCounters& c, int64_t n, int
         double cnt = (double)c.bin_count[b], deg = (double)c.bin_deg[b], kk = (double)c.bin_k[b];
         // per vertex: queue 4, row_ptr pair 16, C[v] 4, d 8, Sig[C[v]] 8, nextC 4; per entry: col 4 (+w), C[u] 4;
         // per distinct neighbour community: Sig 8
-        g->kc_bytes[KC_DEC_S4 + b] += cnt * (4 + 16 + 4 + 8 + 8 + 4) + deg * (4 + om + 4) + 8 * kk;
+        const int kc = b <= BIN_S32 ? KC_DEC_SMALL : KC_DEC_WARP + (b - BIN_WARP);
+        g->kc_bytes[kc] += cnt * (4 + 16 + 4 + 8 + 8 + 4) + deg * (4 + om + 4) + 8 * kk;
         act += cnt;
     }
     // prune: d, dp, C, Sig[C] per vertex; row_ptr pair + queue write per active
@@ -731,6 +729,7 @@ static void ensure_workspace(gala_graph_s* g) {
             wk.mv_old = dalloc<int32_t>(wk.ncap, st);
             wk.nextC = dalloc<int32_t>(wk.ncap, st);
             wk.queues = dalloc<QRec>((size_t)wk.ncap * NBINS, st);
+            if (g->rev0) wk.ckey = dalloc<int32_t>(g->nnz0, st);
             wk.Sig = dalloc<int64_t>(wk.ncap, st);
             wk.d = dalloc<int64_t>(wk.ncap, st);
             wk.s = dalloc<int64_t>(wk.ncap, st);
@@ -755,8 +754,8 @@ static void ensure_workspace(gala_graph_s* g) {
             CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, DM_W128, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)block_smem_bytes<DM_W128>(cap)));
             CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, DM_W128, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)block_smem_bytes<DM_W128>(cap)));
             CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_decide_block<BLOCK_BT, BLOCK_E, DM_W128, false>, BLOCK_BT, block_smem_bytes<DM_W128>(cap)));
-            set_warp_smem<128, DM_FAST>(); set_warp_smem<128, DM_W64>(); set_warp_smem<128, DM_W128>();
-            set_warp_smem<512, DM_FAST>(); set_warp_smem<512, DM_W64>(); set_warp_smem<512, DM_W128>();
+            set_warp_smem<32, 128, DM_FAST>(); set_warp_smem<32, 128, DM_W64>(); set_warp_smem<32, 128, DM_W128>();
+            set_warp_smem<32, 512, DM_FAST>(); set_warp_smem<32, 512, DM_W64>(); set_warp_smem<32, 512, DM_W128>();
             wk.gblocks = g->num_sms * std::max(per_sm, 1);
             wk.gcap = 0;   // spill tables sized on demand (coarse levels can have larger rows than level 0)
             wk.smem_cap = cap;
@@ -842,6 +841,11 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
             if (first_level) {
                 // lab = identity on level 0 (C is the identity right now)
                 CK(cudaMemcpyAsync(g->lab, wk.C, sizeof(int32_t) * n0, cudaMemcpyDeviceToDevice, st));
+                if (use_ckey(g, wk, cur) && cur.nnz) {
+                    k_ckey_init<<<grid_for(cur.nnz, 256, big), 256, 0, st>>>(cur.nnz, cur.row, cur.col, wk.ckey,
+                                                                             wk.carry);
+                    CKL();
+                }
                 first_level = false;
             }
             k_iter_begin<<<1, 128, 0, st>>>(wk.ctr);
@@ -1066,7 +1070,7 @@ static void dist_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, long long
     CKL();
     if (G.nnz) {
         k_dp_full<UNIT><<<grid_for((G.nnz + 127) / 128 * 32, 256, big), 256, 0, st>>>(wk.ctr, G.nnz, G.row, G.col, G.w,
-                                                                                     wk.C, wk.dp, 0, 1, 2);
+                                                                                     wk.C, wk.dp, 0, 1, 2, nullptr, nullptr);
         CKL();
     }
     vt.lap("dist: apply+dp");
@@ -1466,6 +1470,20 @@ static void finish_graph(gala_graph_s* g) {
     if (n == 0) hW = 0;
     if (hW >= ((i128)1 << 62)) { set_err(GALA_E_OVERFLOW, "total weight W >= 2^62"); throw GalaError{GALA_E_OVERFLOW}; }
     g->W = (int64_t)hW;
+    // reverse-entry index for the per-entry neighbour-community array (single GPU, sorted rows)
+    if (!g->di && g->rows_distinct0 && g->g0.nnz > 0 && g->g0.nnz < ((int64_t)1 << 31)) {
+        g->rev0 = dalloc<int32_t>(g->g0.nnz, st);
+        ull* bad = dalloc<ull>(1, st);
+        CK(cudaMemsetAsync(bad, 0, sizeof(ull), st));
+        k_reverse_entries<<<grid_for(g->g0.nnz, 256, big), 256, 0, st>>>(g->g0.nnz, g->g0.rp, g->g0.row, g->g0.col,
+                                                                         g->rev0, bad);
+        CKL();
+        ull hb = 0;
+        CK(cudaMemcpyAsync(&hb, bad, sizeof(ull), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        dfree(bad, st);
+        if (hb) dfree(g->rev0, st);   // not symmetric: keep gathering C[col] in the decide kernels
+    }
 }
 
 #define API_BEGIN try {
@@ -1586,6 +1604,8 @@ gala_status gala_run(gala_graph g, double gamma, double tol, int32_t max_levels)
     if (!g) return set_err(GALA_E_INVALID, "null handle");
     if (!(gamma > 0) || !(gamma < 1e12)) return set_err(GALA_E_INVALID, "gamma must be > 0");
     if (!(tol > 0)) return set_err(GALA_E_INVALID, "tol must be > 0");
+    for (int i = 1; i < NBINS - 1; ++i)
+        if (g->bins[i] < g->bins[i - 1]) return set_err(GALA_E_INVALID, "bin thresholds must be non-decreasing");
     API_BEGIN
     if (g->W == 0) {
         // reading c18: no edges -> singletons, Q := 0
@@ -1670,6 +1690,7 @@ void gala_graph_free(gala_graph g) {
         dfree(g->g0.col, st);
         dfree(g->g0.w, st);
         dfree(g->g0.row, st);
+        dfree(g->rev0, st);
         dfree(g->d0, st);
         dfree(g->s0, st);
         dfree(g->lab, st);
@@ -1693,6 +1714,7 @@ gala_status gala_set_option(gala_graph g, const char* key, int64_t value) {
     else if (k == "force_i128") g->opt_force_i128 = value != 0;
     else if (k == "force_wide") g->opt_force_wide = value != 0;
     else if (k == "singleton") g->opt_singleton = value != 0;
+    else if (k == "ckey") g->opt_ckey = value != 0;
     else if (k == "verbose") g->opt_verbose = (int)value;
     else if (k == "cuda_graph") g->opt_cuda_graph = value != 0;
     else if (k == "log_cap") { if (value < 2 || value > (1 << 20)) return set_err(GALA_E_INVALID, "log_cap in [2, 2^20]"); g->opt_log_cap = (int)value; }
@@ -1701,15 +1723,14 @@ gala_status gala_set_option(gala_graph g, const char* key, int64_t value) {
         g->hub_smem_slots = (int)value;
         if (g->wk) { g->wk->release(); delete g->wk; g->wk = nullptr; }
     } else if (k.rfind("bin_", 0) == 0) {
-        static const char* names[NBINS - 1] = {"bin_sub4", "bin_sub8", "bin_sub16", "bin_sub32", "bin_warp", "bin_warp512"};
+        static const char* names[NBINS - 1] = {"bin_sub4", "bin_sub8", "bin_sub16", "bin_sub32", "bin_warp",
+                                               "bin_warp512"};
         static const int lanes[NBINS - 1] = {4, 8, 16, 32, 128, 512};
         int idx = -1;
         for (int i = 0; i < NBINS - 1; ++i) if (k == names[i]) idx = i;
         if (idx < 0) return set_err(GALA_E_INVALID, "unknown option %s", key);
         if (value < 0 || value > lanes[idx]) return set_err(GALA_E_INVALID, "%s must be in [0, %d]", key, lanes[idx]);
-        g->bins[idx] = (int)value;
-        for (int i = 1; i < NBINS - 1; ++i)
-            if (g->bins[i] < g->bins[i - 1]) return set_err(GALA_E_INVALID, "bin thresholds must be non-decreasing");
+        g->bins[idx] = (int)value;   // monotonicity is checked by gala_run
     } else if (k == "sync_mode") {
         if (value < 0 || value > 2) return set_err(GALA_E_INVALID, "sync_mode: 0 adaptive, 1 dense, 2 sparse");
         g->sync_mode = (int)value;

@@ -90,6 +90,9 @@ struct DecideArgs {
     const int64_t* d;
     const int64_t* dp;
     int32_t* nextC;     // decision of every processed vertex (C[v] to stay)
+    const int32_t* ckey;   // level 0: C[col[e]] per CSR entry (-1 = self loop), rewritten by every full
+                           // d' pass; used while *ckey_valid, else C[col[e]] is gathered here
+    const int* ckey_valid;
     IterCounters* ctr;
     int check;
     int idbits;         // packed-key layout (DM_FAST)
@@ -104,11 +107,11 @@ struct DecideArgs {
 // iteration with all their loads issued before use.
 // ---------------------------------------------------------------------------
 template <int G, int U, int M, bool UNIT>
-__global__ void __launch_bounds__(256) k_decide_sub(const QRec* __restrict__ queue, int bin, DecideArgs a,
-                                                    typename ModeT<M>::ST qW, typename ModeT<M>::ST p) {
+__device__ __forceinline__ unsigned decide_sub_bin(const QRec* __restrict__ queue, int bin, const DecideArgs& a,
+                                                   typename ModeT<M>::ST qW, typename ModeT<M>::ST p,
+                                                   typename ModeT<M>::VT (*s_acc)[32]) {
     typedef typename ModeT<M>::ST ST;
     typedef typename ModeT<M>::VT VT;
-    __shared__ VT s_acc[8][32];
     const int lane = lane_id(), wib = threadIdx.x >> 5;
     const int gid = lane / G, gl = lane % G;
     const unsigned gmask = (G == 32) ? FULLMASK : (((1u << G) - 1u) << (gid * G));
@@ -130,16 +133,30 @@ __global__ void __launch_bounds__(256) k_decide_sub(const QRec* __restrict__ que
             if (valid[k]) q[k] = queue[i];
             else { q[k].v = 0; q[k].deg = 0; q[k].beg = 0; q[k].cv = -2; q[k].szv = 0; q[k].dv = 0; q[k].sigv = 0; }
         }
+        if (a.ckey) {   // neighbour communities read straight from the per-entry array
 #pragma unroll
-        for (int k = 0; k < U; ++k) {
-            has[k] = valid[k] && gl < q[k].deg;
-            u[k] = has[k] ? a.col[q[k].beg + gl] : -1;
-            wt[k] = (has[k] && !UNIT) ? a.w[q[k].beg + gl] : 1;
-        }
+            for (int k = 0; k < U; ++k) {
+                has[k] = valid[k] && gl < q[k].deg;
+                u[k] = has[k] ? a.ckey[q[k].beg + gl] : -1;
+                wt[k] = (has[k] && !UNIT) ? a.w[q[k].beg + gl] : 1;
+            }
 #pragma unroll
-        for (int k = 0; k < U; ++k) {
-            if (u[k] == q[k].v) has[k] = false;               // self loop is not a neighbour
-            cu[k] = has[k] ? a.C[u[k]] : (-1 - lane);         // unique sentinel per empty lane
+            for (int k = 0; k < U; ++k) {
+                if (u[k] < 0) has[k] = false;                 // self loop is not a neighbour
+                cu[k] = has[k] ? u[k] : (-1 - lane);
+            }
+        } else {
+#pragma unroll
+            for (int k = 0; k < U; ++k) {
+                has[k] = valid[k] && gl < q[k].deg;
+                u[k] = has[k] ? a.col[q[k].beg + gl] : -1;
+                wt[k] = (has[k] && !UNIT) ? a.w[q[k].beg + gl] : 1;
+            }
+#pragma unroll
+            for (int k = 0; k < U; ++k) {
+                if (u[k] == q[k].v) has[k] = false;           // self loop is not a neighbour
+                cu[k] = has[k] ? a.C[u[k]] : (-1 - lane);     // unique sentinel per empty lane
+            }
         }
         unsigned peers[U];
         bool isL[U];
@@ -179,8 +196,27 @@ __global__ void __launch_bounds__(256) k_decide_sub(const QRec* __restrict__ que
         for (int k = 0; k < U; ++k)
             if (valid[k] && gl == 0) a.nextC[q[k].v] = tgt[k];
     }
-    ull k = block_sum_ull<256>((ull)my_k);
-    if (threadIdx.x == 0 && k) atomicAdd(&a.ctr->bin_k[bin], k);
+    return my_k;
+}
+
+// bins 0-3 (rows <= 4, 8, 16, 32) in one launch: the block's warps sweep each
+// bin with its own group size, so empty bins cost nothing
+template <int M, bool UNIT>
+__global__ void __launch_bounds__(256) k_decide_small(const QRec* __restrict__ queues, long long qstride,
+                                                      DecideArgs a, typename ModeT<M>::ST qW,
+                                                      typename ModeT<M>::ST p) {
+    __shared__ typename ModeT<M>::VT s_acc[8][32];
+    if (a.ckey && !*a.ckey_valid) a.ckey = nullptr;
+    unsigned k0 = decide_sub_bin<4, 4, M, UNIT>(queues + BIN_S4 * qstride, BIN_S4, a, qW, p, s_acc);
+    unsigned k1 = decide_sub_bin<8, 4, M, UNIT>(queues + BIN_S8 * qstride, BIN_S8, a, qW, p, s_acc);
+    unsigned k2 = decide_sub_bin<16, 2, M, UNIT>(queues + BIN_S16 * qstride, BIN_S16, a, qW, p, s_acc);
+    unsigned k3 = decide_sub_bin<32, 2, M, UNIT>(queues + BIN_S32 * qstride, BIN_S32, a, qW, p, s_acc);
+    const unsigned kk[4] = {k0, k1, k2, k3};
+#pragma unroll
+    for (int b = 0; b < 4; ++b) {
+        ull t = block_sum_ull<256>((ull)kk[b]);
+        if (threadIdx.x == 0 && t) atomicAdd(&a.ctr->bin_k[b], t);
+    }
 }
 
 // ---------------------------------------------------------------------------
@@ -215,68 +251,83 @@ __device__ __forceinline__ int ht_insert(int c, VT wt, int* keys, VT* vals, unsi
 // flight per lane).  The table is cleared once per kernel; every vertex clears
 // exactly the slots it used.  Dynamic shared memory: WPB warps per block.
 // ---------------------------------------------------------------------------
-template <int MAXDEG, int M>
+template <int GW, int MAXDEG, int M>
 struct WarpSmem {
-    static constexpr int WCAP = 2 * MAXDEG;
-    static constexpr int WPB = MAXDEG <= 128 ? 8 : 4;
-    static constexpr size_t per_warp = 32 * sizeof(ull) + (size_t)WCAP * (sizeof(int) + sizeof(typename ModeT<M>::VT)) +
-                                       (size_t)MAXDEG * sizeof(short) + 16;
+    static constexpr int WCAP = 2 * MAXDEG;                 // table slots per group (load <= 1/2)
+    static constexpr int WPB = MAXDEG <= 128 ? 8 : 4;       // warps per block
+    static constexpr size_t per_group =
+        (size_t)WCAP * (sizeof(int) + sizeof(typename ModeT<M>::VT)) + (size_t)MAXDEG * sizeof(short) + 16;
+    static constexpr size_t per_warp = 32 * sizeof(ull) + per_group * (32 / GW);
     static constexpr size_t bytes = per_warp * WPB;
 };
 
-template <int MAXDEG, int M, bool UNIT>
-__global__ void __launch_bounds__(32 * WarpSmem<MAXDEG, M>::WPB) k_decide_warp(const QRec* __restrict__ queue,
-                                                                              int bin, DecideArgs a,
-                                                                              typename ModeT<M>::ST qW,
-                                                                              typename ModeT<M>::ST p) {
+// GW lanes (16 or 32) per vertex, deg <= MAXDEG = 4 * GW; 32/GW vertices per warp
+template <int GW, int MAXDEG, int M, bool UNIT>
+__global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB) k_decide_warp(const QRec* __restrict__ queue,
+                                                                                  int bin, DecideArgs a,
+                                                                                  typename ModeT<M>::ST qW,
+                                                                                  typename ModeT<M>::ST p) {
+    if (a.ckey && !*a.ckey_valid) a.ckey = nullptr;
     typedef typename ModeT<M>::ST ST;
     typedef typename ModeT<M>::VT VT;
-    typedef WarpSmem<MAXDEG, M> SM;
+    typedef WarpSmem<GW, MAXDEG, M> SM;
     constexpr int WCAP = SM::WCAP;
     constexpr unsigned WMASK = WCAP - 1;
-    constexpr int CH = 4;   // entries per lane per round
+    constexpr int CH = MAXDEG / GW;   // entries per lane per round
+    constexpr int NG = 32 / GW;       // vertices per warp
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int lane = lane_id(), wib = threadIdx.x >> 5;
-    unsigned char* base = smem_raw + SM::per_warp * wib;
-    VT* scratch = reinterpret_cast<VT*>(base);
-    base += 32 * sizeof(ull);
+    const int gid = lane / GW, gl = lane % GW;
+    const unsigned gmask = GW == 32 ? FULLMASK : (((1u << GW) - 1u) << (gid * GW));
+    unsigned char* wbase = smem_raw + SM::per_warp * wib;
+    VT* scratch = reinterpret_cast<VT*>(wbase);
+    unsigned char* base = wbase + 32 * sizeof(ull) + SM::per_group * gid;
     VT* vals = reinterpret_cast<VT*>(base);
     int* keys = reinterpret_cast<int*>(base + (size_t)WCAP * sizeof(VT));
     short* list = reinterpret_cast<short*>(base + (size_t)WCAP * (sizeof(VT) + sizeof(int)));
     int* cnt = reinterpret_cast<int*>(base + (size_t)WCAP * (sizeof(VT) + sizeof(int)) + (size_t)MAXDEG * sizeof(short));
-    for (int j = lane; j < WCAP; j += 32) { keys[j] = -1; vals[j] = 0; }
-    if (lane == 0) *cnt = 0;
+    for (int j = gl; j < WCAP; j += GW) { keys[j] = -1; vals[j] = 0; }
+    if (gl == 0) *cnt = 0;
     __syncwarp();
     const long long count = (long long)a.ctr->bin_count[bin];
     const long long nwarps = (long long)gridDim.x * SM::WPB;
     unsigned my_k = 0;
-    long long i = (long long)blockIdx.x * SM::WPB + wib;
+    long long base_i = ((long long)blockIdx.x * SM::WPB + wib) * NG;
     QRec qn;
-    if (i < count) qn = queue[i];
-    for (; i < count; i += nwarps) {
+    if (base_i + gid < count) qn = queue[base_i + gid];
+    for (; base_i < count; base_i += nwarps * NG) {            // warp-uniform
+        const bool valid = base_i + gid < count;
         const QRec q = qn;
-        const int v = q.v, deg = q.deg, cv = q.cv;
-        const int64_t beg = q.beg;
-        const long long dv = q.dv, sig_cv = q.sigv;
-        const long long inext = i + nwarps;
-        if (inext < count) qn = queue[inext];                 // prefetch the next record
-        for (int r0 = 0; r0 < deg; r0 += 32 * CH) {          // warp-uniform rounds
+        const int v = valid ? q.v : 0, deg = valid ? q.deg : 0, cv = valid ? q.cv : -2;
+        const int64_t beg = valid ? q.beg : 0;
+        const long long dv = valid ? q.dv : 0, sig_cv = valid ? q.sigv : 0;
+        const long long inext = base_i + nwarps * NG + gid;
+        if (inext < count) qn = queue[inext];                  // prefetch the next record
+        int dmax = deg;
+#pragma unroll
+        for (int o = 16; o >= GW; o >>= 1) dmax = max(dmax, __shfl_xor_sync(FULLMASK, dmax, o));
+        for (int r0 = 0; r0 < dmax; r0 += GW * CH) {           // warp-uniform rounds
             int uu[CH];
             VT ww[CH];
-#pragma unroll
-            for (int k = 0; k < CH; ++k) {
-                int j = r0 + lane + 32 * k;
-                uu[k] = j < deg ? a.col[beg + j] : -1;
-                ww[k] = (j < deg && !UNIT) ? (VT)a.w[beg + j] : (VT)1;
-            }
             int cc[CH];
 #pragma unroll
-            for (int k = 0; k < CH; ++k) cc[k] = (uu[k] >= 0 && uu[k] != v) ? a.C[uu[k]] : -1;
+            for (int k = 0; k < CH; ++k) {
+                int j = r0 + gl + GW * k;
+                uu[k] = j < deg ? (a.ckey ? a.ckey[beg + j] : a.col[beg + j]) : -1;
+                ww[k] = (j < deg && !UNIT) ? (VT)a.w[beg + j] : (VT)1;
+            }
+            if (a.ckey) {
+#pragma unroll
+                for (int k = 0; k < CH; ++k) cc[k] = uu[k];
+            } else {
+#pragma unroll
+                for (int k = 0; k < CH; ++k) cc[k] = (uu[k] >= 0 && uu[k] != v) ? a.C[uu[k]] : -1;
+            }
 #pragma unroll
             for (int k = 0; k < CH; ++k) {
-                if (r0 + 32 * k >= deg) break;                // warp-uniform
-                // combine equal communities of this 32-entry chunk first (one insert per community)
-                const unsigned peers = __match_any_sync(FULLMASK, cc[k] >= 0 ? cc[k] : -1 - lane);
+                if (r0 + GW * k >= dmax) break;                // warp-uniform
+                // combine equal communities of this chunk first (one insert per community)
+                const unsigned peers = __match_any_sync(FULLMASK, cc[k] >= 0 ? cc[k] : -1 - lane) & gmask;
                 const VT sum = UNIT ? (VT)__popc(peers) : group_sum(peers, cc[k] >= 0 ? ww[k] : (VT)0, scratch);
                 if (cc[k] >= 0 && lane == __ffs(peers) - 1) {
                     bool fresh;
@@ -287,16 +338,16 @@ __global__ void __launch_bounds__(32 * WarpSmem<MAXDEG, M>::WPB) k_decide_warp(c
         }
         __syncwarp();
         const int m = *cnt;
-        my_k += (lane == 0) ? m : 0;
+        my_k += (gl == 0) ? m : 0;
         Arg<ST, ModeT<M>::PK> best;
         best.init(a.idbits, a.idmask);
         long long own = 0;
-        for (int t0 = lane; t0 < m; t0 += 32 * CH) {
+        for (int t0 = gl; t0 < m; t0 += GW * CH) {
             int cs[CH];
             long long ws[CH];
 #pragma unroll
             for (int k = 0; k < CH; ++k) {
-                int t = t0 + 32 * k;
+                int t = t0 + GW * k;
                 cs[k] = -1;
                 ws[k] = 0;
                 if (t < m) {
@@ -318,11 +369,13 @@ __global__ void __launch_bounds__(32 * WarpSmem<MAXDEG, M>::WPB) k_decide_warp(c
             }
         }
         __syncwarp();
-        if (lane == 0) *cnt = 0;
+        if (gl == 0) *cnt = 0;
 #pragma unroll
-        for (int off = 16; off > 0; off >>= 1) best.xor_merge(off);
-        own = warp_sum_ll(own);
-        if (lane == 0) {
+        for (int off = GW / 2; off > 0; off >>= 1) {
+            best.xor_merge(off);
+            own += __shfl_xor_sync(FULLMASK, own, off);
+        }
+        if (valid && gl == 0) {
             if (a.check && own != a.dp[v]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
             a.nextC[v] = decide_final<ST>(cv, q.szv, dv, own, sig_cv, best, a.size, qW, p);
         }
@@ -347,6 +400,7 @@ __global__ void __launch_bounds__(BT) k_decide_block(const QRec* __restrict__ qu
                                                      typename ModeT<M>::ST qW, typename ModeT<M>::ST p, int smem_cap,
                                                      int* __restrict__ gkeys_all, ull* __restrict__ gvals_all,
                                                      int* __restrict__ glist_all, long long gcap) {
+    if (a.ckey && !*a.ckey_valid) a.ckey = nullptr;
     typedef typename ModeT<M>::ST ST;
     typedef typename ModeT<M>::VT VT;
     typedef Arg<ST, ModeT<M>::PK> A;
@@ -383,15 +437,20 @@ __global__ void __launch_bounds__(BT) k_decide_block(const QRec* __restrict__ qu
         for (int r0 = 0; r0 < deg; r0 += BT * E) {          // block-uniform rounds
             int uu[E];
             VT ww[E];
+            int cc[E];
 #pragma unroll
             for (int k = 0; k < E; ++k) {
                 int j = r0 + threadIdx.x + k * BT;
-                uu[k] = j < deg ? a.col[beg + j] : -1;
+                uu[k] = j < deg ? (a.ckey ? a.ckey[beg + j] : a.col[beg + j]) : -1;
                 ww[k] = (j < deg && !UNIT) ? (VT)a.w[beg + j] : (VT)1;
             }
-            int cc[E];
+            if (a.ckey) {
 #pragma unroll
-            for (int k = 0; k < E; ++k) cc[k] = (uu[k] >= 0 && uu[k] != v) ? a.C[uu[k]] : -1;
+                for (int k = 0; k < E; ++k) cc[k] = uu[k];
+            } else {
+#pragma unroll
+                for (int k = 0; k < E; ++k) cc[k] = (uu[k] >= 0 && uu[k] != v) ? a.C[uu[k]] : -1;
+            }
 #pragma unroll
             for (int k = 0; k < E; ++k) {
                 const unsigned peers = __match_any_sync(FULLMASK, cc[k] >= 0 ? cc[k] : -1 - lane);
@@ -484,8 +543,8 @@ __global__ void __launch_bounds__(BT) k_decide_block(const QRec* __restrict__ qu
 //   vertex stream the row, 4 entries per lane in flight.
 // ---------------------------------------------------------------------------
 template <int G, int M, bool UNIT>
-__global__ void __launch_bounds__(256) k_decide_single(const QRec* __restrict__ queue, int bin, DecideArgs a,
-                                                       typename ModeT<M>::ST qW, typename ModeT<M>::ST p) {
+__device__ __forceinline__ unsigned decide_single_bin(const QRec* __restrict__ queue, int bin, const DecideArgs& a,
+                                                      typename ModeT<M>::ST qW, typename ModeT<M>::ST p) {
     typedef typename ModeT<M>::ST ST;
     const int lane = lane_id(), wib = threadIdx.x >> 5;
     const int gid = lane / G, gl = lane % G;
@@ -535,6 +594,27 @@ __global__ void __launch_bounds__(256) k_decide_single(const QRec* __restrict__ 
             a.nextC[v] = tgt;
         }
     }
-    ull k = block_sum_ull<256>((ull)my_k);
-    if (threadIdx.x == 0 && k) atomicAdd(&a.ctr->bin_k[bin], k);
+    return my_k;
+}
+
+// first iteration: bins 0-3 in one launch (G ~ row length / 4), the other bins one launch each
+template <int M, bool UNIT>
+__global__ void __launch_bounds__(256) k_decide_single_small(const QRec* __restrict__ queues, long long qstride,
+                                                             DecideArgs a, typename ModeT<M>::ST qW,
+                                                             typename ModeT<M>::ST p) {
+    const unsigned kk[4] = {decide_single_bin<1, M, UNIT>(queues + BIN_S4 * qstride, BIN_S4, a, qW, p),
+                            decide_single_bin<2, M, UNIT>(queues + BIN_S8 * qstride, BIN_S8, a, qW, p),
+                            decide_single_bin<4, M, UNIT>(queues + BIN_S16 * qstride, BIN_S16, a, qW, p),
+                            decide_single_bin<8, M, UNIT>(queues + BIN_S32 * qstride, BIN_S32, a, qW, p)};
+#pragma unroll
+    for (int b = 0; b < 4; ++b) {
+        ull t = block_sum_ull<256>((ull)kk[b]);
+        if (threadIdx.x == 0 && t) atomicAdd(&a.ctr->bin_k[b], t);
+    }
+}
+template <int M, bool UNIT>
+__global__ void __launch_bounds__(256) k_decide_single(const QRec* __restrict__ queue, int bin, DecideArgs a,
+                                                       typename ModeT<M>::ST qW, typename ModeT<M>::ST p) {
+    ull t = block_sum_ull<256>((ull)decide_single_bin<32, M, UNIT>(queue, bin, a, qW, p));
+    if (threadIdx.x == 0 && t) atomicAdd(&a.ctr->bin_k[bin], t);
 }

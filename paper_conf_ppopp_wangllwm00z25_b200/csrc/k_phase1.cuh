@@ -284,9 +284,13 @@ __global__ void __launch_bounds__(256) k_dp_delta(IterCounters* __restrict__ ctr
                                                   const int32_t* __restrict__ mv_old,
                                                   const int32_t* __restrict__ stamp, int64_t* __restrict__ dp,
                                                   const Carry* __restrict__ carry, long long nnz, int mode,
-                                                  long long fnum, long long fden) {
+                                                  long long fnum, long long fden, int32_t* __restrict__ ckey,
+                                                  const int32_t* __restrict__ rev) {
     if (!use_delta(ctr, nnz, mode, fnum, fden)) return;
-    if (blockIdx.x == 0 && threadIdx.x == 0) ctr->delta_used = 1;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        ctr->delta_used = 1;
+        if (ckey) const_cast<Carry*>(carry)->ckey_valid = 0;   // per-entry communities now stale
+    }
     const int iter_id = carry->iter;
     const int lane = lane_id();
     const long long m = (long long)ctr->n_moved;
@@ -328,9 +332,11 @@ template <bool UNIT>
 __global__ void __launch_bounds__(256) k_dp_full(IterCounters* __restrict__ ctr, long long nnz,
                                                  const int32_t* __restrict__ row, const int32_t* __restrict__ col,
                                                  const int64_t* __restrict__ w, const int32_t* __restrict__ C,
-                                                 int64_t* __restrict__ dp, int mode, long long fnum, long long fden) {
+                                                 int64_t* __restrict__ dp, int mode, long long fnum, long long fden,
+                                                 int32_t* __restrict__ ckey, int* __restrict__ carry_valid) {
     __shared__ ull s_scr[8][32];
     if (use_delta(ctr, nnz, mode, fnum, fden)) return;
+    if (ckey && blockIdx.x == 0 && threadIdx.x == 0) carry_valid[0] = 1;   // rewritten below for every entry
     const int lane = lane_id(), wib = threadIdx.x >> 5;
     const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
     for (long long base = (((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * 128; base < nnz;
@@ -349,6 +355,11 @@ __global__ void __launch_bounds__(256) k_dp_full(IterCounters* __restrict__ ctr,
         for (int t = 0; t < 4; ++t) {
             cr[t] = r[t] >= 0 ? C[r[t]] : 0;
             cu[t] = u[t] >= 0 ? C[u[t]] : 1;
+        }
+        if (ckey) {   // refresh the per-entry neighbour communities for the next decide
+#pragma unroll
+            for (int t = 0; t < 4; ++t)
+                if (r[t] >= 0) ckey[base + lane + 32 * t] = u[t] == r[t] ? -1 : cu[t];
         }
 #pragma unroll
         for (int t = 0; t < 4; ++t) {
@@ -503,4 +514,28 @@ __global__ void k_record(const IterCounters* __restrict__ ctr, Carry* __restrict
     const int more = !carry->converged && (max_iters <= 0 || it + 1 < max_iters) && (slot + 1 < log_cap);
     carry->more = more;
     if (cond_handle) cudaGraphSetConditional((cudaGraphConditionalHandle)cond_handle, more ? 1u : 0u);
+}
+
+// level-0 init of the per-entry neighbour communities: C = identity
+__global__ void k_ckey_init(long long nnz, const int32_t* __restrict__ row, const int32_t* __restrict__ col,
+                            int32_t* __restrict__ ckey, Carry* __restrict__ carry) {
+    if (blockIdx.x == 0 && threadIdx.x == 0) carry->ckey_valid = 1;
+    for (long long e = (long long)blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += (long long)gridDim.x * blockDim.x)
+        ckey[e] = col[e] == row[e] ? -1 : col[e];
+}
+
+// reverse entry of every CSR entry (rows sorted, distinct): rev[e] = position of
+// (col[e], row[e]) in row col[e]; *bad != 0 if some reverse entry is missing
+__global__ void k_reverse_entries(long long nnz, const int64_t* __restrict__ rp, const int32_t* __restrict__ row,
+                                  const int32_t* __restrict__ col, int32_t* __restrict__ rev, ull* __restrict__ bad) {
+    for (long long e = (long long)blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += (long long)gridDim.x * blockDim.x) {
+        const int v = row[e], u = col[e];
+        long long lo = rp[u], hi = rp[u + 1];
+        while (lo < hi) {
+            long long mid = (lo + hi) >> 1;
+            if (col[mid] < v) lo = mid + 1; else hi = mid;
+        }
+        if (lo < rp[u + 1] && col[lo] == v) rev[e] = (int32_t)lo;
+        else { rev[e] = 0; atomicAdd(bad, 1ull); }
+    }
 }

@@ -76,9 +76,9 @@ def test_synthetic_parity(name, prune):
 
 
 @pytest.mark.parametrize("opts", [
-    dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=0, bin_warp512=0),   # all through block hash
-    dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=128),    # warp hash for <= 128
-    dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=0),      # warp512 hash for <= 512
+    dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=0, bin_warp512=0),   # block hash
+    dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=128),                # warp hash <= 128
+    dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=0),                  # warp512 hash <= 512
     dict(bin_sub4=4, bin_sub8=4, bin_sub16=4, bin_sub32=32, bin_warp=32),
     dict(hub_smem_slots=64),                                                  # force the global spill table
     dict(force_i128=1),
@@ -86,6 +86,8 @@ def test_synthetic_parity(name, prune):
     dict(delta_update=0),
     dict(delta_update=1),
     dict(singleton=0),
+    dict(ckey=1),
+    dict(delta_update=1, ckey=1),
 ])
 def test_dispatch_independence(opts):
     """P7: thresholds / table sizes / integer width / update strategy never change a label."""
