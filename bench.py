@@ -218,9 +218,6 @@ def main():
     # ------------------------------------------------------------ device-resident timing (value)
     h = gala.Graph.from_graph(g, device=dev, stream=stream.cuda_stream)
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device=dev)   # > 126 MB L2
-    for _ in range(args.warmup):
-        h.run()
-    torch.cuda.synchronize()
 
     def timed_steps(nsteps, timing):
         h.set_option("timing", int(timing))
@@ -248,6 +245,7 @@ def main():
         return ms, edges, scanned, launches, kst
 
     with ClockSampler(dev) as clk:
+        timed_steps(args.warmup, False)          # warm-up: identical steps (flush included), untimed
         step_ms, edges, scanned, launches, _ = timed_steps(args.steps, False)
     run_ms = h.stats()["run_ms"]
     # per-kernel CUDA-event timing (stepwise launch mode) for the roofline, same workload
@@ -373,9 +371,6 @@ def run_dist(args, rank, world, local_rank):
     stream = torch.cuda.Stream(device=dev)
     h = gala.Graph.from_csr_dist(uid[0], rank, world, dev, g.n, v0, v1, lrp, lcol, lw, stream=stream.cuda_stream)
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device=dev)
-    for _ in range(args.warmup):
-        h.run()
-    torch.cuda.synchronize()
     peak, peak_src, _ = load_peaks()
 
     def step(fn):
@@ -392,6 +387,8 @@ def run_dist(args, rank, world, local_rank):
         return max_over_ranks(e0.elapsed_time(e1))
 
     with ClockSampler(dev) as clk:
+        for _ in range(args.warmup):
+            step(h.run)
         step_ms = [step(h.run) for _ in range(args.steps)]
     st = h.stats()
     edges = nominal_edges(st)
