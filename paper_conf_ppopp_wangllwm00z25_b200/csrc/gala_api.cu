@@ -17,6 +17,8 @@
 #include <cstdio>
 #include <cstring>
 #include <string>
+#include <map>
+#include <unordered_map>
 #include <vector>
 
 #include "gala.h"
@@ -91,7 +93,7 @@ struct LevelStat {
 struct gala_graph_s {
     int device = 0;
     cudaStream_t stream = nullptr;
-    cudaMemPool_t pool = nullptr;
+    struct DevCache* cache = nullptr;
     bool own_stream = false;
     int num_sms = 148;
     // level-0 graph
@@ -130,26 +132,72 @@ struct gala_graph_s {
 };
 
 // ------------------------------------------------------------------ memory
-// All device memory of a handle comes from its own stream-ordered pool whose
-// release threshold is "keep everything": repeated runs reuse the pages
-// instead of re-mapping them (set per API call by PoolScope).
-static thread_local cudaMemPool_t g_pool = nullptr;
+// All device memory of a handle comes from its own stream-ordered pool (release
+// threshold "keep everything") through a size-class cache: freed blocks are
+// kept per handle and handed back to the next request of (nearly) the same
+// size.  A run on the same graph repeats its allocation sequence, so from the
+// second run on no allocation reaches the pool -- pool reuse alone would still
+// remap physical pages to new virtual ranges (tens of ms per GB on big levels).
+// Every user of a handle's memory is ordered on the handle's stream, which makes
+// reuse without events safe.  The active cache is set per API call (PoolScope).
+struct DevCache {
+    cudaMemPool_t pool = nullptr;
+    std::multimap<size_t, void*> freeb;        // cached free blocks by size
+    std::unordered_map<void*, size_t> sz;      // every block this cache handed out
+    static size_t round(size_t b) {
+        if (b <= 4096) return (b + 255) & ~(size_t)255;
+        if (b < ((size_t)2 << 20)) { size_t r = 8192; while (r < b) r <<= 1; return r; }
+        return (b + ((size_t)2 << 20) - 1) & ~(((size_t)2 << 20) - 1);
+    }
+    void* get(size_t bytes, cudaStream_t st) {
+        const size_t r = round(bytes);
+        auto it = freeb.lower_bound(r);
+        if (it != freeb.end() && it->first <= r + r / 4) {
+            void* p = it->second;
+            freeb.erase(it);
+            return p;
+        }
+        void* p = nullptr;
+        cudaError_t e = cudaMallocFromPoolAsync(&p, r, pool, st);
+        if (e == cudaErrorMemoryAllocation) {   // give cached blocks back and retry once
+            cudaGetLastError();
+            trim(st);
+            cudaStreamSynchronize(st);
+            cudaMemPoolTrimTo(pool, 0);
+            e = cudaMallocFromPoolAsync(&p, r, pool, st);
+        }
+        CK(e);
+        sz[p] = r;
+        return p;
+    }
+    bool put(void* p) {
+        auto it = sz.find(p);
+        if (it == sz.end()) return false;
+        freeb.emplace(it->second, p);
+        return true;
+    }
+    void trim(cudaStream_t st) {
+        for (auto& kv : freeb) { cudaFreeAsync(kv.second, st); sz.erase(kv.second); }
+        freeb.clear();
+    }
+};
+static thread_local DevCache* g_cache = nullptr;
 struct PoolScope {
-    cudaMemPool_t prev;
-    explicit PoolScope(cudaMemPool_t p) : prev(g_pool) { g_pool = p; }
-    ~PoolScope() { g_pool = prev; }
+    DevCache* prev;
+    explicit PoolScope(DevCache* c) : prev(g_cache) { g_cache = c; }
+    ~PoolScope() { g_cache = prev; }
 };
 template <typename T>
 static T* dalloc(size_t count, cudaStream_t st) {
-    void* p = nullptr;
     if (count == 0) count = 1;
-    if (g_pool) CK(cudaMallocFromPoolAsync(&p, count * sizeof(T), g_pool, st));
-    else CK(cudaMallocAsync(&p, count * sizeof(T), st));
+    if (g_cache) return static_cast<T*>(g_cache->get(count * sizeof(T), st));
+    void* p = nullptr;
+    CK(cudaMallocAsync(&p, count * sizeof(T), st));
     return static_cast<T*>(p);
 }
 template <typename T>
 static void dfree(T*& p, cudaStream_t st) {
-    if (p) cudaFreeAsync(p, st);
+    if (p && !(g_cache && g_cache->put(p))) cudaFreeAsync(p, st);
     p = nullptr;
 }
 
@@ -609,10 +657,12 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
         CK(cudaMemsetAsync(gkeys, 0xff, sizeof(int) * gtot, st));
         CK(cudaMemsetAsync(gvals, 0, sizeof(ull) * gtot, st));
         CK(cudaMemsetAsync(gcnt, 0, sizeof(int) * nbig, st));
+        vt.lap("agg: big alloc+clear");
         const int bpc = 32;
         if (unit) k_agg_big_insert<true><<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
         else k_agg_big_insert<false><<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
         CKL();
+        vt.lap("agg: big insert");
         k_agg_big_emit<<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
         CKL();
         dfree(goff, st); dfree(gkeys, st); dfree(gvals, st); dfree(glist, st); dfree(gcnt, st);
@@ -632,6 +682,7 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
     nxt.col = dalloc<int32_t>(nxt.nnz, st);
     nxt.w = dalloc<int64_t>(nxt.nnz, st);
     nxt.row = dalloc<int32_t>(nxt.nnz, st);
+    vt.lap("agg: scan+alloc");
     if (nxt.nnz > 0) {
         k_compact<<<grid_for(nxt.nnz, 256, big * 4), 256, 0, st>>>(k, nxt.nnz, eoff, reinterpret_cast<long long*>(nxt.rp),
                                                                     tkey, tval, nxt.col, nxt.w, nxt.row);
@@ -770,7 +821,7 @@ static void ensure_workspace(gala_graph_s* g) {
 
 
 static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
-    PoolScope pool_scope(g->pool);
+    PoolScope pool_scope(g->cache);
     cudaStream_t st = g->stream;
     CK(cudaSetDevice(g->device));
     g->has_result = false;
@@ -955,6 +1006,12 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
         CK(cudaEventElapsedTime(&ms, ev_run0, ev_run1));
         g->run_ms = ms;
         g->launches = g_launches - launches0;
+        if (g->opt_verbose && g->cache) {
+            unsigned long long res = 0, used = 0;
+            cudaMemPoolGetAttribute(g->cache->pool, cudaMemPoolAttrReservedMemCurrent, &res);
+            cudaMemPoolGetAttribute(g->cache->pool, cudaMemPoolAttrUsedMemHigh, &used);
+            fprintf(stderr, "[gala] run %.3f ms, pool reserved %.1f MB, used high %.1f MB\n", ms, res / 1e6, used / 1e6);
+        }
     } catch (...) {
         wk.release();
         delete g->wk;
@@ -1187,7 +1244,7 @@ static void dist_coarsen(gala_graph_s* g, Work& wk, const DevCSR& cur, int64_t n
 }
 
 static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_levels) {
-    PoolScope pool_scope(g->pool);
+    PoolScope pool_scope(g->cache);
     cudaStream_t st = g->stream;
     CK(cudaSetDevice(g->device));
     DistInfo& di = *g->di;
@@ -1406,10 +1463,11 @@ static void init_graph_common(gala_graph_s* g, int64_t n, int device, uintptr_t 
     props.allocType = cudaMemAllocationTypePinned;
     props.location.type = cudaMemLocationTypeDevice;
     props.location.id = device;
-    CK(cudaMemPoolCreate(&g->pool, &props));
+    g->cache = new DevCache();
+    CK(cudaMemPoolCreate(&g->cache->pool, &props));
     uint64_t keep = UINT64_MAX;
-    CK(cudaMemPoolSetAttribute(g->pool, cudaMemPoolAttrReleaseThreshold, &keep));
-    g_pool = g->pool;
+    CK(cudaMemPoolSetAttribute(g->cache->pool, cudaMemPoolAttrReleaseThreshold, &keep));
+    g_cache = g->cache;
 }
 
 // Device-side validation of the copied CSR (GALA_E_INVALID), unit-weight
@@ -1682,6 +1740,7 @@ gala_status gala_modularity(gala_graph g, double* q) {
 void gala_graph_free(gala_graph g) {
     if (!g) return;
     cudaSetDevice(g->device);
+    PoolScope pool_scope(g->cache);
     if (g->di) { delete g->di; g->di = nullptr; }   // communicators are cached (comm_for)
     cudaStream_t st = g->stream;
     if (g->wk) { g->wk->release(); delete g->wk; g->wk = nullptr; }
@@ -1694,16 +1753,22 @@ void gala_graph_free(gala_graph g) {
         dfree(g->d0, st);
         dfree(g->s0, st);
         dfree(g->lab, st);
+        if (g->cache) g->cache->trim(st);
         cudaStreamSynchronize(st);
         if (g->own_stream) cudaStreamDestroy(st);
     }
-    if (g->pool) cudaMemPoolDestroy(g->pool);
-    if (g_pool == g->pool) g_pool = nullptr;
+    if (g->cache) {
+        if (g->cache->pool) cudaMemPoolDestroy(g->cache->pool);
+        delete g->cache;
+    }
+    g_cache = pool_scope.prev == g->cache ? nullptr : pool_scope.prev;
+    pool_scope.prev = g_cache;
     delete g;
 }
 
 gala_status gala_set_option(gala_graph g, const char* key, int64_t value) {
     if (!g || !key) return set_err(GALA_E_INVALID, "null argument");
+    PoolScope pool_scope(g->cache);
     std::string k(key);
     if (k == "prune") g->opt_prune = value != 0;
     else if (k == "trace") g->opt_trace = (int)value;
