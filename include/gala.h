@@ -140,9 +140,11 @@ void gala_graph_free(gala_graph g);
  *   "check"          0/1   debug: verify maintained d'(v) against its definition
  *   "timing"         0/1   per-kernel CUDA-event timing (gala_get_kernel_stats)
  *   "max_iters"      >= 0  per-level iteration cap (0 = none)
- *   "bin_sub4" "bin_sub8" "bin_sub16" "bin_sub32" "bin_warp" "bin_warp512"
+ *   "bin_sub4" "bin_sub8" "bin_sub16" "bin_sub32" "bin_warp" "bin_warp512" "bin_block"
  *                    row-length upper bounds of the dispatch bins (non-decreasing;
- *                    each <= 4, 8, 16, 32, 128, 512 respectively)
+ *                    each <= 4, 8, 16, 32, 128, 512, 2^30 respectively; defaults
+ *                    4 8 16 32 128 512 16384).  Rows longer than "bin_block" take the
+ *                    multi-block hub path (chunks of 1024 entries over all SMs).
  *   "delta_update"   0 = always recompute d', 1 = always delta, 2 = adaptive (default)
  *   "force_i128"     0/1   use the 128-bit gain path even when 64-bit suffices
  *   "force_wide"     0/1   use unpacked 64-bit gains / aggregates (no packed keys)

@@ -16,8 +16,10 @@ typedef unsigned long long ull;
 
 #define FULLMASK 0xffffffffu
 
-// dispatch bins (a2): sub-warp groups of 4/8/16/32 lanes, warp hash (<=128, <=512), block hash
-enum { BIN_S4 = 0, BIN_S8 = 1, BIN_S16 = 2, BIN_S32 = 3, BIN_WARP = 4, BIN_WARP2 = 5, BIN_BLOCK = 6, NBINS = 7 };
+// dispatch bins (a2): sub-warp groups of 4/8/16/32 lanes, warp hash (<=128, <=512), block hash,
+// multi-block hub path (rows split into chunks)
+enum { BIN_S4 = 0, BIN_S8 = 1, BIN_S16 = 2, BIN_S32 = 3, BIN_WARP = 4, BIN_WARP2 = 5, BIN_BLOCK = 6, BIN_HUB = 7,
+       NBINS = 8 };
 
 // Device-resident per-iteration counters (zeroed by k_iter_begin).
 struct IterCounters {
@@ -47,6 +49,20 @@ struct __align__(16) QRec {
     long long sigv; // Sigma_tot[C[v]]
     long long pad;
 };
+
+// Bin queues: bins 2r and 2r+1 share region r of `qstride` records, the even
+// bin filling it upwards from the start and the odd one downwards from the end
+// (their counts sum to at most the number of vertices), so NBINS/2 regions hold
+// every queue.
+struct QView {
+    QRec* base;
+    int dir;
+    __host__ __device__ __forceinline__ QRec& operator[](long long i) const { return base[dir * i]; }
+};
+__host__ __device__ __forceinline__ QView qview(QRec* queues, long long qstride, int b) {
+    QRec* r = queues + (long long)(b >> 1) * qstride;
+    return (b & 1) ? QView{r + qstride - 1, -1} : QView{r, 1};
+}
 
 // Device-resident state carried across iterations of a level.
 struct Carry {

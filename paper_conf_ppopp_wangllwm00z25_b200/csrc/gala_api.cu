@@ -64,11 +64,11 @@ static thread_local long long g_launches = 0;
 
 // ------------------------------------------------------------------ kernel classes
 enum KClass {
-    KC_PRUNE = 0, KC_DEC_SMALL, KC_DEC_WARP, KC_DEC_WARP2, KC_DEC_BLOCK,
+    KC_PRUNE = 0, KC_DEC_SMALL, KC_DEC_WARP, KC_DEC_WARP2, KC_DEC_BLOCK, KC_DEC_HUB,
     KC_APPLY, KC_DP, KC_REDUCE, KC_INIT, KC_PHASE2, KC_COUNT
 };
 static const char* kc_names[KC_COUNT] = {"prune_bin", "decide_small", "decide_warp", "decide_warp512",
-                                         "decide_block", "apply",
+                                         "decide_block", "decide_hub", "apply",
                                          "dp_update", "reduce", "level_init", "phase2"};
 
 struct TraceRec {
@@ -107,7 +107,7 @@ struct gala_graph_s {
     bool rows_distinct0 = false;   // level-0 rows strictly increasing (no duplicate entries)
     int32_t* rev0 = nullptr;       // level-0 reverse-entry index (enables the per-entry community array)
     int opt_ckey = 0;
-    int bins[NBINS - 1] = {4, 8, 16, 32, 128, 512};
+    int bins[NBINS - 1] = {4, 8, 16, 32, 128, 512, 16384};
     int hub_smem_slots = 4096;
     // results
     bool has_result = false;
@@ -295,6 +295,11 @@ struct Work {
     int* glist = nullptr;
     long long gcap = 0;
     int gblocks = 0;
+    // hub tables (k_hub_*), sized per level for the rows longer than the block bin
+    bool hub_on = false;
+    HubWork hw = {};
+    long long hub_ncap = 0, hub_tcap = 0, hub_lcap = 0;
+    ull* hub_size = nullptr;
     IterLog* h_log = nullptr;
     Carry* h_carry = nullptr;
     int reduce_grid = 0;
@@ -306,6 +311,9 @@ struct Work {
         dfree(queues, st); dfree(ckey, st); dfree(Sig, st); dfree(d, st); dfree(s, st); dfree(dp, st); dfree(ctr, st);
         dfree(carry, st); dfree(log, st); dfree(part_dc, st); dfree(part_min, st); dfree(part_s2, st);
         dfree(gkeys, st); dfree(gvals, st); dfree(glist, st);
+        dfree(hw.keys, st); dfree(hw.vals, st); dfree(hw.list, st); dfree(hw.pref, st); dfree(hw.toff, st);
+        dfree(hw.loff, st); dfree(hw.cnt, st); dfree(hub_size, st);
+        hub_ncap = hub_tcap = hub_lcap = 0;
         if (h_log) cudaFreeHost(h_log);
         if (h_carry) cudaFreeHost(h_carry);
         h_log = nullptr;
@@ -332,6 +340,23 @@ static void set_warp_smem() {
 template <int M>
 static size_t block_smem_bytes(int cap) { return (size_t)cap * (sizeof(typename ModeT<M>::VT) + 2 * sizeof(int)); }
 
+// multi-block hub path (bin BIN_HUB), only on levels that have such rows
+template <int M, bool UNIT>
+static void launch_hub(gala_graph_s* g, Work& wk, const DecideArgs& a, typename ModeT<M>::ST qW,
+                       typename ModeT<M>::ST p, Timer& tm) {
+    if (!wk.hub_on) return;
+    cudaStream_t st = g->stream;
+    const QView q = qview(wk.queues, wk.ncap, BIN_HUB);
+    cudaEvent_t e = tm.begin();
+    k_hub_prep<<<1, 1024, 0, st>>>(q, wk.ctr, wk.hw);
+    CKL();
+    k_hub_agg<M, UNIT><<<g->num_sms * 8, HUB_BT, 0, st>>>(q, a, wk.hw);
+    CKL();
+    k_hub_eval<M, UNIT><<<g->num_sms * 2, HUB_EVAL_BT, 0, st>>>(q, a, wk.hw, qW, p);
+    CKL();
+    tm.end(KC_DEC_HUB, e);
+}
+
 template <int M, bool UNIT>
 static void launch_single(gala_graph_s* g, Work& wk, const DecideArgs& a, typename ModeT<M>::ST qW,
                           typename ModeT<M>::ST p, Timer& tm, int64_t maxdeg) {
@@ -343,13 +368,14 @@ static void launch_single(gala_graph_s* g, Work& wk, const DecideArgs& a, typena
     CKL();
     tm.end(KC_DEC_SMALL, e);
     static const int kcs[3] = {KC_DEC_WARP, KC_DEC_WARP2, KC_DEC_BLOCK};
-    for (int b = BIN_WARP; b < NBINS; ++b) {
+    for (int b = BIN_WARP; b <= BIN_BLOCK; ++b) {
         if (maxdeg <= g->bins[b - 1]) break;
         e = tm.begin();
-        k_decide_single<M, UNIT><<<grid, 256, 0, st>>>(wk.queues + b * qs, b, a, qW, p);
+        k_decide_single<M, UNIT><<<grid, 256, 0, st>>>(qview(wk.queues, qs, b), b, a, qW, p);
         CKL();
         tm.end(kcs[b - BIN_WARP], e);
     }
+    launch_hub<M, UNIT>(g, wk, a, qW, p, tm);
 }
 
 template <int M, bool UNIT>
@@ -373,13 +399,13 @@ static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, typename M
     tm.end(KC_DEC_SMALL, e);
     e = tm.begin();
     k_decide_warp<32, 128, M, UNIT><<<grid, 32 * WarpSmem<32, 128, M>::WPB, WarpSmem<32, 128, M>::bytes, st>>>(
-        wk.queues + BIN_WARP * qs, BIN_WARP, a, qW, p);
+        qview(wk.queues, qs, BIN_WARP), BIN_WARP, a, qW, p);
     CKL();
     tm.end(KC_DEC_WARP, e);
     if (maxdeg > g->bins[BIN_WARP]) {
         e = tm.begin();
         k_decide_warp<32, 512, M, UNIT><<<grid, 32 * WarpSmem<32, 512, M>::WPB, WarpSmem<32, 512, M>::bytes, st>>>(
-            wk.queues + BIN_WARP2 * qs, BIN_WARP2, a, qW, p);
+            qview(wk.queues, qs, BIN_WARP2), BIN_WARP2, a, qW, p);
         CKL();
         tm.end(KC_DEC_WARP2, e);
     }
@@ -387,10 +413,67 @@ static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, typename M
         const int smem_cap = g->hub_smem_slots;
         e = tm.begin();
         k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT><<<wk.gblocks, BLOCK_BT, block_smem_bytes<M>(smem_cap), st>>>(
-            wk.queues + BIN_BLOCK * qs, BIN_BLOCK, a, qW, p, smem_cap, wk.gkeys, wk.gvals, wk.glist, wk.gcap);
+            qview(wk.queues, qs, BIN_BLOCK), BIN_BLOCK, a, qW, p, smem_cap, wk.gkeys, wk.gvals, wk.glist, wk.gcap);
         CKL();
         tm.end(KC_DEC_BLOCK, e);
     }
+    launch_hub<M, UNIT>(g, wk, a, qW, p, tm);
+}
+
+// Per level, before its iterations: per-block spill tables of the block bin
+// (rows up to bins[BIN_BLOCK]) and the hub tables of the longer rows.
+static void prepare_level_tables(gala_graph_s* g, Work& wk, const DevCSR& G, int64_t maxdeg) {
+    cudaStream_t st = g->stream;
+    const int64_t bmax = std::min<int64_t>(maxdeg, g->bins[BIN_BLOCK]);
+    long long need = 64;
+    while (need < 2 * bmax) need <<= 1;
+    if (maxdeg > g->bins[BIN_WARP2] && need > wk.gcap) {
+        dfree(wk.gkeys, st);
+        dfree(wk.gvals, st);
+        dfree(wk.glist, st);
+        wk.gcap = need;
+        wk.gkeys = dalloc<int>((size_t)wk.gblocks * wk.gcap, st);
+        wk.gvals = dalloc<ull>((size_t)wk.gblocks * wk.gcap, st);
+        wk.glist = dalloc<int>((size_t)wk.gblocks * wk.gcap, st);
+        CK(cudaMemsetAsync(wk.gkeys, 0xff, sizeof(int) * (size_t)wk.gblocks * wk.gcap, st));
+        CK(cudaMemsetAsync(wk.gvals, 0, sizeof(ull) * (size_t)wk.gblocks * wk.gcap, st));
+    }
+    wk.hub_on = maxdeg > g->bins[BIN_BLOCK];
+    if (!wk.hub_on) return;
+    if (!wk.hub_size) wk.hub_size = dalloc<ull>(3, st);
+    CK(cudaMemsetAsync(wk.hub_size, 0, sizeof(ull) * 3, st));
+    k_hub_size<<<grid_for(G.n, 256, g->num_sms * 8), 256, 0, st>>>(G.n, G.rp, g->bins[BIN_BLOCK], G.n, wk.hub_size);
+    CKL();
+    ull hs[3];
+    CK(cudaMemcpyAsync(hs, wk.hub_size, sizeof(hs), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    const long long nh = (long long)hs[0] + 1, tc = std::max<long long>((long long)hs[1], 1),
+                    lc = std::max<long long>((long long)hs[2], 1);
+    HubWork& h = wk.hw;
+    if (nh > wk.hub_ncap) {
+        dfree(h.pref, st); dfree(h.toff, st); dfree(h.loff, st); dfree(h.cnt, st);
+        h.pref = dalloc<long long>(nh, st);
+        h.toff = dalloc<long long>(nh, st);
+        h.loff = dalloc<long long>(nh, st);
+        h.cnt = dalloc<int>(nh, st);
+        wk.hub_ncap = nh;
+    }
+    if (tc > wk.hub_tcap) {
+        dfree(h.keys, st); dfree(h.vals, st);
+        h.keys = dalloc<int>(tc, st);
+        h.vals = dalloc<ull>(tc, st);
+        wk.hub_tcap = tc;
+    }
+    if (lc > wk.hub_lcap) {
+        dfree(h.list, st);
+        h.list = dalloc<int>(lc, st);
+        wk.hub_lcap = lc;
+    }
+    // tables start empty on every level (evaluation keeps them empty afterwards)
+    CK(cudaMemsetAsync(h.keys, 0xff, sizeof(int) * tc, st));
+    CK(cudaMemsetAsync(h.vals, 0, sizeof(ull) * tc, st));
+    CK(cudaMemsetAsync(h.cnt, 0, sizeof(int) * nh, st));
+    h.nlev = G.n;
 }
 
 // one phase-1 iteration (Alg. 1 lines 3-13) + its device log record
@@ -779,7 +862,7 @@ static void ensure_workspace(gala_graph_s* g) {
             wk.mv_v = dalloc<int32_t>(wk.ncap, st);
             wk.mv_old = dalloc<int32_t>(wk.ncap, st);
             wk.nextC = dalloc<int32_t>(wk.ncap, st);
-            wk.queues = dalloc<QRec>((size_t)wk.ncap * NBINS, st);
+            wk.queues = dalloc<QRec>((size_t)wk.ncap * (NBINS / 2), st);
             if (g->rev0) wk.ckey = dalloc<int32_t>(g->nnz0, st);
             wk.Sig = dalloc<int64_t>(wk.ncap, st);
             wk.d = dalloc<int64_t>(wk.ncap, st);
@@ -870,20 +953,7 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
             ls.maxdeg = maxdeg;
             cudaEvent_t lv0 = wk.ev[2], lv1 = wk.ev[3], lv2 = wk.ev[4];
             CK(cudaEventRecord(lv0, st));
-            // spill tables big enough for this level's largest row
-            long long need = 64;
-            while (need < 2 * maxdeg) need <<= 1;
-            if (maxdeg > g->bins[BIN_WARP2] && need > wk.gcap) {
-                dfree(wk.gkeys, st);
-                dfree(wk.gvals, st);
-                dfree(wk.glist, st);
-                wk.gcap = need;
-                wk.gkeys = dalloc<int>((size_t)wk.gblocks * wk.gcap, st);
-                wk.gvals = dalloc<ull>((size_t)wk.gblocks * wk.gcap, st);
-                wk.glist = dalloc<int>((size_t)wk.gblocks * wk.gcap, st);
-                CK(cudaMemsetAsync(wk.gkeys, 0xff, sizeof(int) * (size_t)wk.gblocks * wk.gcap, st));
-                CK(cudaMemsetAsync(wk.gvals, 0, sizeof(ull) * (size_t)wk.gblocks * wk.gcap, st));
-            }
+            prepare_level_tables(g, wk, cur, maxdeg);
             // a1: level init + starting numerator
             cudaEvent_t e = tm.begin();
             k_level_init<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.d, wk.C, wk.Sig, wk.size, wk.dp, wk.stamp,
@@ -1302,19 +1372,7 @@ static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_level
             ls.nnz = gnnz;
             ls.maxdeg = maxdeg;
             CK(cudaEventRecord(wk.ev[2], st));
-            long long need = 64;
-            while (need < 2 * maxdeg) need <<= 1;
-            if (maxdeg > g->bins[BIN_WARP2] && need > wk.gcap) {
-                dfree(wk.gkeys, st);
-                dfree(wk.gvals, st);
-                dfree(wk.glist, st);
-                wk.gcap = need;
-                wk.gkeys = dalloc<int>((size_t)wk.gblocks * wk.gcap, st);
-                wk.gvals = dalloc<ull>((size_t)wk.gblocks * wk.gcap, st);
-                wk.glist = dalloc<int>((size_t)wk.gblocks * wk.gcap, st);
-                CK(cudaMemsetAsync(wk.gkeys, 0xff, sizeof(int) * (size_t)wk.gblocks * wk.gcap, st));
-                CK(cudaMemsetAsync(wk.gvals, 0, sizeof(ull) * (size_t)wk.gblocks * wk.gcap, st));
-            }
+            prepare_level_tables(g, wk, cur, maxdeg);
             k_level_init<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.d, wk.C, wk.Sig, wk.size, wk.dp, wk.stamp,
                                                                  wk.carry);
             CKL();
@@ -1789,8 +1847,8 @@ gala_status gala_set_option(gala_graph g, const char* key, int64_t value) {
         if (g->wk) { g->wk->release(); delete g->wk; g->wk = nullptr; }
     } else if (k.rfind("bin_", 0) == 0) {
         static const char* names[NBINS - 1] = {"bin_sub4", "bin_sub8", "bin_sub16", "bin_sub32", "bin_warp",
-                                               "bin_warp512"};
-        static const int lanes[NBINS - 1] = {4, 8, 16, 32, 128, 512};
+                                               "bin_warp512", "bin_block"};
+        static const int lanes[NBINS - 1] = {4, 8, 16, 32, 128, 512, 1 << 30};
         int idx = -1;
         for (int i = 0; i < NBINS - 1; ++i) if (k == names[i]) idx = i;
         if (idx < 0) return set_err(GALA_E_INVALID, "unknown option %s", key);

@@ -107,7 +107,7 @@ struct DecideArgs {
 // iteration with all their loads issued before use.
 // ---------------------------------------------------------------------------
 template <int G, int U, int M, bool UNIT>
-__device__ __forceinline__ unsigned decide_sub_bin(const QRec* __restrict__ queue, int bin, const DecideArgs& a,
+__device__ __forceinline__ unsigned decide_sub_bin(QView queue, int bin, const DecideArgs& a,
                                                    typename ModeT<M>::ST qW, typename ModeT<M>::ST p,
                                                    typename ModeT<M>::VT (*s_acc)[32]) {
     typedef typename ModeT<M>::ST ST;
@@ -202,15 +202,15 @@ __device__ __forceinline__ unsigned decide_sub_bin(const QRec* __restrict__ queu
 // bins 0-3 (rows <= 4, 8, 16, 32) in one launch: the block's warps sweep each
 // bin with its own group size, so empty bins cost nothing
 template <int M, bool UNIT>
-__global__ void __launch_bounds__(256) k_decide_small(const QRec* __restrict__ queues, long long qstride,
+__global__ void __launch_bounds__(256) k_decide_small(QRec* queues, long long qstride,
                                                       DecideArgs a, typename ModeT<M>::ST qW,
                                                       typename ModeT<M>::ST p) {
     __shared__ typename ModeT<M>::VT s_acc[8][32];
     if (a.ckey && !*a.ckey_valid) a.ckey = nullptr;
-    unsigned k0 = decide_sub_bin<4, 4, M, UNIT>(queues + BIN_S4 * qstride, BIN_S4, a, qW, p, s_acc);
-    unsigned k1 = decide_sub_bin<8, 4, M, UNIT>(queues + BIN_S8 * qstride, BIN_S8, a, qW, p, s_acc);
-    unsigned k2 = decide_sub_bin<16, 2, M, UNIT>(queues + BIN_S16 * qstride, BIN_S16, a, qW, p, s_acc);
-    unsigned k3 = decide_sub_bin<32, 2, M, UNIT>(queues + BIN_S32 * qstride, BIN_S32, a, qW, p, s_acc);
+    unsigned k0 = decide_sub_bin<4, 4, M, UNIT>(qview(queues, qstride, BIN_S4), BIN_S4, a, qW, p, s_acc);
+    unsigned k1 = decide_sub_bin<8, 4, M, UNIT>(qview(queues, qstride, BIN_S8), BIN_S8, a, qW, p, s_acc);
+    unsigned k2 = decide_sub_bin<16, 2, M, UNIT>(qview(queues, qstride, BIN_S16), BIN_S16, a, qW, p, s_acc);
+    unsigned k3 = decide_sub_bin<32, 2, M, UNIT>(qview(queues, qstride, BIN_S32), BIN_S32, a, qW, p, s_acc);
     const unsigned kk[4] = {k0, k1, k2, k3};
 #pragma unroll
     for (int b = 0; b < 4; ++b) {
@@ -263,7 +263,7 @@ struct WarpSmem {
 
 // GW lanes (16 or 32) per vertex, deg <= MAXDEG = 4 * GW; 32/GW vertices per warp
 template <int GW, int MAXDEG, int M, bool UNIT>
-__global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB) k_decide_warp(const QRec* __restrict__ queue,
+__global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB) k_decide_warp(QView queue,
                                                                                   int bin, DecideArgs a,
                                                                                   typename ModeT<M>::ST qW,
                                                                                   typename ModeT<M>::ST p) {
@@ -396,7 +396,7 @@ __global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB) k_decide_wa
 // ---------------------------------------------------------------------------
 #define HWIN 16
 template <int BT, int E, int M, bool UNIT>
-__global__ void __launch_bounds__(BT) k_decide_block(const QRec* __restrict__ queue, int bin, DecideArgs a,
+__global__ void __launch_bounds__(BT) k_decide_block(QView queue, int bin, DecideArgs a,
                                                      typename ModeT<M>::ST qW, typename ModeT<M>::ST p, int smem_cap,
                                                      int* __restrict__ gkeys_all, ull* __restrict__ gvals_all,
                                                      int* __restrict__ glist_all, long long gcap) {
@@ -543,7 +543,7 @@ __global__ void __launch_bounds__(BT) k_decide_block(const QRec* __restrict__ qu
 //   vertex stream the row, 4 entries per lane in flight.
 // ---------------------------------------------------------------------------
 template <int G, int M, bool UNIT>
-__device__ __forceinline__ unsigned decide_single_bin(const QRec* __restrict__ queue, int bin, const DecideArgs& a,
+__device__ __forceinline__ unsigned decide_single_bin(QView queue, int bin, const DecideArgs& a,
                                                       typename ModeT<M>::ST qW, typename ModeT<M>::ST p) {
     typedef typename ModeT<M>::ST ST;
     const int lane = lane_id(), wib = threadIdx.x >> 5;
@@ -599,13 +599,13 @@ __device__ __forceinline__ unsigned decide_single_bin(const QRec* __restrict__ q
 
 // first iteration: bins 0-3 in one launch (G ~ row length / 4), the other bins one launch each
 template <int M, bool UNIT>
-__global__ void __launch_bounds__(256) k_decide_single_small(const QRec* __restrict__ queues, long long qstride,
+__global__ void __launch_bounds__(256) k_decide_single_small(QRec* queues, long long qstride,
                                                              DecideArgs a, typename ModeT<M>::ST qW,
                                                              typename ModeT<M>::ST p) {
-    const unsigned kk[4] = {decide_single_bin<1, M, UNIT>(queues + BIN_S4 * qstride, BIN_S4, a, qW, p),
-                            decide_single_bin<2, M, UNIT>(queues + BIN_S8 * qstride, BIN_S8, a, qW, p),
-                            decide_single_bin<4, M, UNIT>(queues + BIN_S16 * qstride, BIN_S16, a, qW, p),
-                            decide_single_bin<8, M, UNIT>(queues + BIN_S32 * qstride, BIN_S32, a, qW, p)};
+    const unsigned kk[4] = {decide_single_bin<1, M, UNIT>(qview(queues, qstride, BIN_S4), BIN_S4, a, qW, p),
+                            decide_single_bin<2, M, UNIT>(qview(queues, qstride, BIN_S8), BIN_S8, a, qW, p),
+                            decide_single_bin<4, M, UNIT>(qview(queues, qstride, BIN_S16), BIN_S16, a, qW, p),
+                            decide_single_bin<8, M, UNIT>(qview(queues, qstride, BIN_S32), BIN_S32, a, qW, p)};
 #pragma unroll
     for (int b = 0; b < 4; ++b) {
         ull t = block_sum_ull<256>((ull)kk[b]);
@@ -613,8 +613,240 @@ __global__ void __launch_bounds__(256) k_decide_single_small(const QRec* __restr
     }
 }
 template <int M, bool UNIT>
-__global__ void __launch_bounds__(256) k_decide_single(const QRec* __restrict__ queue, int bin, DecideArgs a,
+__global__ void __launch_bounds__(256) k_decide_single(QView queue, int bin, DecideArgs a,
                                                        typename ModeT<M>::ST qW, typename ModeT<M>::ST p) {
     ull t = block_sum_ull<256>((ull)decide_single_bin<32, M, UNIT>(queue, bin, a, qW, p));
     if (threadIdx.x == 0 && t) atomicAdd(&a.ctr->bin_k[bin], t);
+}
+
+// ---------------------------------------------------------------------------
+// a4 (hubs, rows longer than the block bin): the hierarchical table of §4.2
+// spread over the whole GPU.  A row is cut into HUB_CH-entry
+// chunks; any block takes any chunk (dynamic cursor), sums it in a shared-
+// memory table (one slot per distinct community of the chunk, never full) and
+// flushes the distinct (c, w_c) pairs into the hub's global table (capacity a
+// power of two >= 2 min(deg, n), load <= 1/2) -- the global level of the
+// hierarchy.  Fresh global keys go to the hub's distinct list.  k_hub_eval
+// then evaluates each hub's list with one block and clears the table, so the
+// tables are empty between iterations.  Chunk ranges / table offsets of the
+// queued hubs are laid out by k_hub_prep (one block).
+// ---------------------------------------------------------------------------
+#define HUB_CH 1024
+#define HUB_BT 256
+#define HUB_EVAL_BT 512
+struct HubWork {
+    int* keys;          // global tables (all hubs), -1 = empty
+    ull* vals;
+    int* list;          // distinct-slot lists
+    long long* pref;    // [count+1] chunk prefix of the queued hubs
+    long long* toff;    // [count+1] table offsets
+    long long* loff;    // [count+1] list offsets
+    int* cnt;           // [count] distinct keys inserted (zero between iterations)
+    long long nlev;     // vertices of the level (bound on distinct communities)
+};
+
+__device__ __forceinline__ unsigned hub_hash(int c, unsigned mask) {
+    return (unsigned)(((unsigned long long)(unsigned)c * 0x9E3779B97F4A7C15ull) >> 32) & mask;
+}
+__device__ __forceinline__ long long hub_cap(long long deg, long long nlev) {
+    long long d = deg < nlev ? deg : nlev, c = 64;
+    while (c < 2 * d) c <<= 1;
+    return c;
+}
+
+// exclusive scans of (chunks, table capacity, list length) over the queued hubs
+__global__ void __launch_bounds__(1024) k_hub_prep(QView queue, const IterCounters* __restrict__ ctr, HubWork h) {
+    __shared__ long long s_w[3][32];
+    __shared__ long long s_carry[3];
+    const long long count = (long long)ctr->bin_count[BIN_HUB];
+    const int lane = lane_id(), wib = threadIdx.x >> 5;
+    if (threadIdx.x < 3) s_carry[threadIdx.x] = 0;
+    __syncthreads();
+    for (long long t0 = 0; t0 < count; t0 += 1024) {
+        const long long i = t0 + threadIdx.x;
+        long long x[3] = {0, 0, 0};
+        if (i < count) {
+            const long long deg = queue[i].deg;
+            x[0] = (deg + HUB_CH - 1) / HUB_CH;
+            x[1] = hub_cap(deg, h.nlev);
+            x[2] = deg < h.nlev ? deg : h.nlev;
+        }
+        long long inc[3];
+#pragma unroll
+        for (int k = 0; k < 3; ++k) {
+            inc[k] = x[k];
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                long long y = __shfl_up_sync(FULLMASK, inc[k], o);
+                if (lane >= o) inc[k] += y;
+            }
+            if (lane == 31) s_w[k][wib] = inc[k];
+        }
+        __syncthreads();
+        if (wib == 0) {
+#pragma unroll
+            for (int k = 0; k < 3; ++k) {
+                long long v = s_w[k][lane], iv = v;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    long long y = __shfl_up_sync(FULLMASK, iv, o);
+                    if (lane >= o) iv += y;
+                }
+                s_w[k][lane] = iv - v;   // exclusive warp offsets
+            }
+        }
+        __syncthreads();
+        if (i < count) {
+            h.pref[i] = s_carry[0] + s_w[0][wib] + inc[0] - x[0];
+            h.toff[i] = s_carry[1] + s_w[1][wib] + inc[1] - x[1];
+            h.loff[i] = s_carry[2] + s_w[2][wib] + inc[2] - x[2];
+        }
+        __syncthreads();
+        if (threadIdx.x == 1023)
+            for (int k = 0; k < 3; ++k) s_carry[k] += s_w[k][31] + inc[k];
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) { h.pref[count] = s_carry[0]; h.toff[count] = s_carry[1]; h.loff[count] = s_carry[2]; }
+}
+
+template <int M, bool UNIT>
+__global__ void __launch_bounds__(HUB_BT) k_hub_agg(QView queue, DecideArgs a, HubWork h) {
+    typedef typename ModeT<M>::VT VT;
+    constexpr int SCAP = 2 * HUB_CH;
+    constexpr int E = HUB_CH / HUB_BT;
+    __shared__ int keys[SCAP];
+    __shared__ ull vals[SCAP];
+    __shared__ short list[HUB_CH];
+    __shared__ VT s_scr[HUB_BT / 32][32];
+    __shared__ long long s_item;
+    __shared__ int s_cnt;
+    if (a.ckey && !*a.ckey_valid) a.ckey = nullptr;
+    const int lane = lane_id(), wib = threadIdx.x >> 5;
+    for (int j = threadIdx.x; j < SCAP; j += HUB_BT) { keys[j] = -1; vals[j] = 0; }
+    if (threadIdx.x == 0) s_cnt = 0;
+    const long long count = (long long)a.ctr->bin_count[BIN_HUB];
+    if (count == 0) return;
+    const long long total = h.pref[count];
+    for (;;) {
+        if (threadIdx.x == 0) s_item = (long long)atomicAdd(&a.ctr->cursor[BIN_HUB], 1ull);
+        __syncthreads();
+        const long long item = s_item;
+        if (item >= total) break;
+        long long lo = 0, hi = count - 1;          // last i with pref[i] <= item
+        while (lo < hi) {
+            long long mid = (lo + hi + 1) >> 1;
+            if (h.pref[mid] <= item) lo = mid; else hi = mid - 1;
+        }
+        const long long i = lo;
+        const QRec q = queue[i];
+        const int v = q.v;
+        const long long j0 = (item - h.pref[i]) * HUB_CH;
+        int cc[E];
+        VT ww[E];
+#pragma unroll
+        for (int k = 0; k < E; ++k) {
+            const long long j = j0 + threadIdx.x + k * HUB_BT;
+            int u = -1;
+            if (j < q.deg) u = a.ckey ? a.ckey[q.beg + j] : a.col[q.beg + j];
+            cc[k] = u;
+            ww[k] = (j < q.deg && !UNIT) ? (VT)a.w[q.beg + j] : (VT)1;
+        }
+        if (!a.ckey) {
+#pragma unroll
+            for (int k = 0; k < E; ++k) cc[k] = (cc[k] >= 0 && cc[k] != v) ? a.C[cc[k]] : -1;
+        }
+#pragma unroll
+        for (int k = 0; k < E; ++k) {
+            const unsigned peers = __match_any_sync(FULLMASK, cc[k] >= 0 ? cc[k] : -1 - lane);
+            const VT sum = UNIT ? (VT)__popc(peers) : group_sum(peers, cc[k] >= 0 ? ww[k] : (VT)0, s_scr[wib]);
+            if (cc[k] < 0 || lane != __ffs(peers) - 1) continue;
+            bool fresh;
+            int slot = ht_insert<ull>(cc[k], (ull)sum, keys, vals, SCAP - 1, hash_slot(cc[k], SCAP - 1), SCAP, &fresh);
+            if (fresh) list[atomicAdd(&s_cnt, 1)] = (short)slot;
+        }
+        __syncthreads();
+        const int m = s_cnt;
+        const long long toff = h.toff[i], cap = h.toff[i + 1] - toff, loff = h.loff[i];
+        int* gk = h.keys + toff;
+        ull* gv = h.vals + toff;
+        const unsigned gmask = (unsigned)(cap - 1);
+        for (int t = threadIdx.x; t < m; t += HUB_BT) {
+            const int slot = list[t];
+            const int c = keys[slot];
+            const ull wv = vals[slot];
+            keys[slot] = -1;
+            vals[slot] = 0;
+            bool fresh;
+            int gs = ht_insert<ull>(c, wv, gk, gv, gmask, hub_hash(c, gmask), (int)min(cap, (long long)INT_MAX), &fresh);
+            if (fresh) h.list[loff + atomicAdd(&h.cnt[i], 1)] = gs;
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) s_cnt = 0;
+    }
+}
+
+template <int M, bool UNIT>
+__global__ void __launch_bounds__(HUB_EVAL_BT) k_hub_eval(QView queue, DecideArgs a, HubWork h,
+                                                          typename ModeT<M>::ST qW, typename ModeT<M>::ST p) {
+    typedef typename ModeT<M>::ST ST;
+    typedef Arg<ST, ModeT<M>::PK> A;
+    __shared__ A r_a[HUB_EVAL_BT / 32];
+    __shared__ long long r_own[HUB_EVAL_BT / 32];
+    const int lane = lane_id(), wib = threadIdx.x >> 5;
+    const long long count = (long long)a.ctr->bin_count[BIN_HUB];
+    unsigned my_k = 0;
+    for (long long i = blockIdx.x; i < count; i += gridDim.x) {
+        const QRec q = queue[i];
+        const int m = h.cnt[i];
+        const long long toff = h.toff[i], loff = h.loff[i];
+        const int cv = q.cv;
+        const long long dv = q.dv;
+        A best;
+        best.init(a.idbits, a.idmask);
+        long long own = 0;
+        for (int t = threadIdx.x; t < m; t += HUB_EVAL_BT) {
+            const long long slot = toff + h.list[loff + t];
+            const int c = h.keys[slot];
+            const long long wc = (long long)h.vals[slot];
+            h.keys[slot] = -1;
+            h.vals[slot] = 0;
+            if (c == cv) own = wc;
+            else best.offer(gain<ST>(qW, p, wc, a.Sig[c], dv), c);
+        }
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) best.xor_merge(off);
+        own = warp_sum_ll(own);
+        if (lane == 0) { r_a[wib] = best; r_own[wib] = own; }
+        __syncthreads();
+        if (wib == 0) {
+            if (lane < HUB_EVAL_BT / 32) { best = r_a[lane]; own = r_own[lane]; }
+            else { best.init(a.idbits, a.idmask); own = 0; }
+#pragma unroll
+            for (int off = 16; off > 0; off >>= 1) best.xor_merge(off);
+            own = warp_sum_ll(own);
+            if (lane == 0) {
+                if (a.check && own != a.dp[q.v]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
+                a.nextC[q.v] = decide_final<ST>(cv, q.szv, dv, own, q.sigv, best, a.size, qW, p);
+                h.cnt[i] = 0;
+                my_k += (unsigned)m;
+            }
+        }
+        __syncthreads();
+    }
+    if (threadIdx.x == 0 && my_k) atomicAdd(&a.ctr->bin_k[BIN_HUB], (ull)my_k);
+}
+
+// per level: number of rows longer than t, and the table / list space they can need
+__global__ void k_hub_size(long long n, const int64_t* __restrict__ rp, long long t, long long nlev,
+                           ull* __restrict__ out) {
+    ull c = 0, cap = 0, dist = 0;
+    for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x) {
+        const long long deg = rp[v + 1] - rp[v];
+        if (deg > t) { c++; cap += (ull)hub_cap(deg, nlev); dist += (ull)(deg < nlev ? deg : nlev); }
+    }
+    if (c) {
+        atomicAdd(&out[0], c);
+        atomicAdd(&out[1], cap);
+        atomicAdd(&out[2], dist);
+    }
 }

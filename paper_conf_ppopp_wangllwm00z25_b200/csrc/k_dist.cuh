@@ -15,7 +15,7 @@ __global__ void k_expand_rp(long long n, long long v0, long long v1, const int64
 
 // owned queued vertices whose decision differs -> local move list (v, new), block-aggregated
 __global__ void __launch_bounds__(256) k_collect_moves(const IterCounters* __restrict__ ctr,
-                                                       const QRec* __restrict__ queues, long long qstride,
+                                                       QRec* queues, long long qstride,
                                                        const int32_t* __restrict__ nextC, int2* __restrict__ moves,
                                                        ull* __restrict__ nmoves) {
     __shared__ unsigned s_cnt;
@@ -34,7 +34,7 @@ __global__ void __launch_bounds__(256) k_collect_moves(const IterCounters* __res
 #pragma unroll
             for (int k = 0; k < NBINS - 1; ++k)
                 if (b == k && r >= cnt[k]) { r -= cnt[k]; b = k + 1; }
-            const QRec q = queues[(long long)b * qstride + r];
+            const QRec q = qview(queues, qstride, b)[r];
             v = q.v;
             nc = nextC[v];
             mover = nc != q.cv;

@@ -86,7 +86,7 @@ __global__ void k_iter_begin(IterCounters* ctr) {
 // results (P7).
 // ---------------------------------------------------------------------------
 struct BinThresholds {
-    int t[NBINS - 1];   // upper row-length bound of bins 0..4; bin 5 = rest
+    int t[NBINS - 1];   // upper row-length bound of bins 0..NBINS-2; the last bin takes the rest
 };
 #define PB_BT 256
 #define PB_IPT 4
@@ -182,7 +182,7 @@ __global__ void __launch_bounds__(PB_BT) k_prune_bin(int vlo, int n, const int64
                 q.dv = dv[j];
                 q.sigv = sg[j];
                 q.pad = 0;
-                queues[(long long)bin[j] * qstride + (long long)s_base[bin[j]] + off[j]] = q;
+                qview(queues, qstride, bin[j])[(long long)s_base[bin[j]] + off[j]] = q;
             }
         }
     }
@@ -204,7 +204,7 @@ __global__ void __launch_bounds__(PB_BT) k_prune_bin(int vlo, int n, const int64
 // one global atomic per block and tile.
 // ---------------------------------------------------------------------------
 #define AP_BT 256
-__global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr, const QRec* __restrict__ queues,
+__global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr, QRec* queues,
                                                  long long qstride, const int32_t* __restrict__ nextC,
                                                  int32_t* __restrict__ C, int64_t* __restrict__ Sig,
                                                  int32_t* __restrict__ size, const int64_t* __restrict__ d,
@@ -229,7 +229,7 @@ __global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr,
 #pragma unroll
             for (int k = 0; k < NBINS - 1; ++k)
                 if (b == k && r >= cnt[k]) { r -= cnt[k]; b = k + 1; }
-            const QRec q = queues[(long long)b * qstride + r];
+            const QRec q = qview(queues, qstride, b)[r];
             v = q.v;
             int nc = nextC[v];
             oc = q.cv;

@@ -91,3 +91,9 @@ def test_dist_karate_and_weighted():
 
 def test_dist_more_ranks_than_busy_rows():
     check(gg.make("karate"), 4)
+
+
+def test_dist_hub_path():
+    """Rows split over blocks (hub path) on partitioned ranks, coarse levels included."""
+    check(gg.make("rmat_small"), 3, bin_sub4=4, bin_sub8=8, bin_sub16=16, bin_sub32=32, bin_warp=32,
+          bin_warp512=32, bin_block=32)

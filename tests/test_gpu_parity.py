@@ -33,6 +33,15 @@ def run_gpu(g, gamma=1.0, tol=1e-6, max_levels=0, trace=2, **opts):
     return out
 
 
+def hub(t):
+    """Bin thresholds that send every row longer than t through the multi-block hub path."""
+    names = ["bin_sub4", "bin_sub8", "bin_sub16", "bin_sub32", "bin_warp", "bin_warp512"]
+    caps = [4, 8, 16, 32, 128, 512]
+    d = {k: min(c, t) for k, c in zip(names, caps)}
+    d["bin_block"] = t
+    return d
+
+
 def assert_parity(g, gamma=1.0, tol=1e-6, max_levels=0, prune=True, labels=True, **opts):
     o = oracle.louvain(g, gamma=gamma, tol=tol, max_levels=max_levels, prune=prune, trace=2 if labels else 1,
                        max_iters=opts.get("max_iters", 0))
@@ -81,6 +90,10 @@ def test_synthetic_parity(name, prune):
     dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=0),                  # warp512 hash <= 512
     dict(bin_sub4=4, bin_sub8=4, bin_sub16=4, bin_sub32=32, bin_warp=32),
     dict(hub_smem_slots=64),                                                  # force the global spill table
+    hub(64),                                                                  # rows > 64 through the hub path
+    hub(0),                                                                   # every row through the hub path
+    dict(hub(0), force_i128=1),
+    dict(hub(64), singleton=0, delta_update=1),
     dict(force_i128=1),
     dict(force_wide=1),
     dict(delta_update=0),
@@ -94,7 +107,7 @@ def test_dispatch_independence(opts):
     assert_parity(gg.make("rmat_small"), **opts)
 
 
-@pytest.mark.parametrize("opts", [dict(force_wide=1), dict(force_i128=1)])
+@pytest.mark.parametrize("opts", [dict(force_wide=1), dict(force_i128=1), hub(16), dict(hub(16), force_i128=1)])
 def test_weighted_modes_parity(opts):
     """Weighted random graphs through every gain-arithmetic mode (DM_W64 / DM_W128)."""
     for seed in range(4):
@@ -107,6 +120,11 @@ def test_graph_mode_parity(name):
     """Default launch mode (conditional-while CUDA graph per level, no per-iteration host sync):
     per-iteration N / moved / active counts and final labels equal the oracle's."""
     assert_parity(gg.make(name), labels=False)
+
+
+def test_graph_mode_hub_parity():
+    """Hub path (multi-block rows) inside the conditional graph, coarse levels included."""
+    assert_parity(gg.make("rmat_small"), labels=False, **hub(32))
 
 
 def test_graph_mode_log_relaunch():
