@@ -34,6 +34,7 @@ struct IterCounters {
     ull dp_mismatch;        // check mode: maintained d' != aggregated d'
     ull ticket;             // last-block-done ticket of k_reduce
     ull delta_used;         // 1 if the delta d' update ran this iteration
+    ull cursor2;            // dynamic work cursor of the hub evaluation
 };
 
 // Queue record of an active vertex, written by k_prune_bin (which already

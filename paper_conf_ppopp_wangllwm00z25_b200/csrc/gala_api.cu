@@ -298,7 +298,7 @@ struct Work {
     // hub tables (k_hub_*), sized per level for the rows longer than the block bin
     bool hub_on = false;
     HubWork hw = {};
-    long long hub_ncap = 0, hub_tcap = 0, hub_lcap = 0;
+    long long hub_ncap = 0, hub_tcap = 0, hub_lcap = 0, hub_pcap = 0;
     ull* hub_size = nullptr;
     IterLog* h_log = nullptr;
     Carry* h_carry = nullptr;
@@ -312,8 +312,11 @@ struct Work {
         dfree(carry, st); dfree(log, st); dfree(part_dc, st); dfree(part_min, st); dfree(part_s2, st);
         dfree(gkeys, st); dfree(gvals, st); dfree(glist, st);
         dfree(hw.keys, st); dfree(hw.vals, st); dfree(hw.list, st); dfree(hw.pref, st); dfree(hw.toff, st);
-        dfree(hw.loff, st); dfree(hw.cnt, st); dfree(hub_size, st);
-        hub_ncap = hub_tcap = hub_lcap = 0;
+        dfree(hw.loff, st); dfree(hw.cnt, st); dfree(hub_size, st); dfree(hw.spref, st); dfree(hw.own, st);
+        char* part = static_cast<char*>(hw.part);
+        dfree(part, st);
+        hw.part = nullptr;
+        hub_ncap = hub_tcap = hub_lcap = hub_pcap = 0;
         if (h_log) cudaFreeHost(h_log);
         if (h_carry) cudaFreeHost(h_carry);
         h_log = nullptr;
@@ -352,7 +355,11 @@ static void launch_hub(gala_graph_s* g, Work& wk, const DecideArgs& a, typename 
     CKL();
     k_hub_agg<M, UNIT><<<g->num_sms * 8, HUB_BT, 0, st>>>(q, a, wk.hw);
     CKL();
-    k_hub_eval<M, UNIT><<<g->num_sms * 2, HUB_EVAL_BT, 0, st>>>(q, a, wk.hw, qW, p);
+    k_hub_prep2<<<1, 1024, 0, st>>>(wk.ctr, wk.hw);
+    CKL();
+    k_hub_eval<M, UNIT><<<g->num_sms * 4, HUB_EVAL_BT, 0, st>>>(q, a, wk.hw, qW, p);
+    CKL();
+    k_hub_final<M, UNIT><<<g->num_sms, 256, 0, st>>>(q, a, wk.hw, qW, p);
     CKL();
     tm.end(KC_DEC_HUB, e);
 }
@@ -451,13 +458,24 @@ static void prepare_level_tables(gala_graph_s* g, Work& wk, const DevCSR& G, int
                     lc = std::max<long long>((long long)hs[2], 1);
     HubWork& h = wk.hw;
     if (nh > wk.hub_ncap) {
-        dfree(h.pref, st); dfree(h.toff, st); dfree(h.loff, st); dfree(h.cnt, st);
+        dfree(h.pref, st); dfree(h.toff, st); dfree(h.loff, st); dfree(h.cnt, st); dfree(h.spref, st);
+        dfree(h.own, st);
         h.pref = dalloc<long long>(nh, st);
         h.toff = dalloc<long long>(nh, st);
         h.loff = dalloc<long long>(nh, st);
+        h.spref = dalloc<long long>(nh, st);
         h.cnt = dalloc<int>(nh, st);
+        h.own = dalloc<long long>(nh, st);
         wk.hub_ncap = nh;
     }
+    const long long np = lc / HUB_EV + nh + 1;   // evaluation slices
+    if (np > wk.hub_pcap) {
+        char* part = static_cast<char*>(h.part);
+        dfree(part, st);
+        h.part = dalloc<char>((size_t)np * 32, st);
+        wk.hub_pcap = np;
+    }
+    static_assert(sizeof(Arg<i128, false>) <= 32, "partial argmax record");
     if (tc > wk.hub_tcap) {
         dfree(h.keys, st); dfree(h.vals, st);
         h.keys = dalloc<int>(tc, st);
@@ -473,6 +491,7 @@ static void prepare_level_tables(gala_graph_s* g, Work& wk, const DevCSR& G, int
     CK(cudaMemsetAsync(h.keys, 0xff, sizeof(int) * tc, st));
     CK(cudaMemsetAsync(h.vals, 0, sizeof(ull) * tc, st));
     CK(cudaMemsetAsync(h.cnt, 0, sizeof(int) * nh, st));
+    CK(cudaMemsetAsync(h.own, 0, sizeof(long long) * nh, st));
     h.nlev = G.n;
 }
 

@@ -306,6 +306,7 @@ __global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB) k_decide_wa
         int dmax = deg;
 #pragma unroll
         for (int o = 16; o >= GW; o >>= 1) dmax = max(dmax, __shfl_xor_sync(FULLMASK, dmax, o));
+        long long own = 0;   // the own community only feeds d'(v): summed in registers, never inserted
         for (int r0 = 0; r0 < dmax; r0 += GW * CH) {           // warp-uniform rounds
             int uu[CH];
             VT ww[CH];
@@ -324,6 +325,9 @@ __global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB) k_decide_wa
                 for (int k = 0; k < CH; ++k) cc[k] = (uu[k] >= 0 && uu[k] != v) ? a.C[uu[k]] : -1;
             }
 #pragma unroll
+            for (int k = 0; k < CH; ++k)
+                if (cc[k] == cv) { own += (long long)ww[k]; cc[k] = -1; }
+#pragma unroll
             for (int k = 0; k < CH; ++k) {
                 if (r0 + GW * k >= dmax) break;                // warp-uniform
                 // combine equal communities of this chunk first (one insert per community)
@@ -341,7 +345,6 @@ __global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB) k_decide_wa
         my_k += (gl == 0) ? m : 0;
         Arg<ST, ModeT<M>::PK> best;
         best.init(a.idbits, a.idmask);
-        long long own = 0;
         for (int t0 = gl; t0 < m; t0 += GW * CH) {
             int cs[CH];
             long long ws[CH];
@@ -378,6 +381,7 @@ __global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB) k_decide_wa
         if (valid && gl == 0) {
             if (a.check && own != a.dp[v]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
             a.nextC[v] = decide_final<ST>(cv, q.szv, dv, own, sig_cv, best, a.size, qW, p);
+            my_k += own ? 1u : 0u;
         }
         __syncwarp();
     }
@@ -428,8 +432,9 @@ __global__ void __launch_bounds__(BT) k_decide_block(QView queue, int bin, Decid
         long long i = s_item;
         if (i >= count) break;
         const QRec q = queue[i];
-        const int v = q.v, deg = q.deg;
+        const int v = q.v, deg = q.deg, cv = q.cv;
         const int64_t beg = q.beg;
+        long long own = 0;   // the own community only feeds d'(v): summed in registers, never inserted
         int win = (smem_cap >= 2 * deg) ? smem_cap : HWIN;    // fits at load <= 1/2: never spills
         long long gc = 64;
         while (gc < 2LL * deg && gc < gcap) gc <<= 1;
@@ -452,6 +457,9 @@ __global__ void __launch_bounds__(BT) k_decide_block(QView queue, int bin, Decid
                 for (int k = 0; k < E; ++k) cc[k] = (uu[k] >= 0 && uu[k] != v) ? a.C[uu[k]] : -1;
             }
 #pragma unroll
+            for (int k = 0; k < E; ++k)
+                if (cc[k] == cv) { own += (long long)ww[k]; cc[k] = -1; }
+#pragma unroll
             for (int k = 0; k < E; ++k) {
                 const unsigned peers = __match_any_sync(FULLMASK, cc[k] >= 0 ? cc[k] : -1 - lane);
                 const VT sum = UNIT ? (VT)__popc(peers) : group_sum(peers, cc[k] >= 0 ? ww[k] : (VT)0, s_scr[wib]);
@@ -469,11 +477,9 @@ __global__ void __launch_bounds__(BT) k_decide_block(QView queue, int bin, Decid
         }
         __syncthreads();
         const int m = s_cnt, gm = s_gcnt;
-        const int cv = q.cv;
         const long long dv = q.dv;
         A best;
         best.init(a.idbits, a.idmask);
-        long long own = 0;
         my_k += (threadIdx.x == 0) ? (unsigned)(m + gm) : 0u;
         for (int t0 = threadIdx.x; t0 < m; t0 += BT * E) {
             int cs[E];
@@ -523,6 +529,7 @@ __global__ void __launch_bounds__(BT) k_decide_block(QView queue, int bin, Decid
             if (lane == 0) {
                 if (a.check && own != a.dp[v]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
                 a.nextC[v] = decide_final<ST>(cv, q.szv, dv, own, q.sigv, best, a.size, qW, p);
+                my_k += own ? 1u : 0u;
                 s_cnt = 0;
                 s_gcnt = 0;
             }
@@ -633,6 +640,7 @@ __global__ void __launch_bounds__(256) k_decide_single(QView queue, int bin, Dec
 // ---------------------------------------------------------------------------
 #define HUB_CH 1024
 #define HUB_BT 256
+#define HUB_EV 2048
 #define HUB_EVAL_BT 512
 struct HubWork {
     int* keys;          // global tables (all hubs), -1 = empty
@@ -641,7 +649,10 @@ struct HubWork {
     long long* pref;    // [count+1] chunk prefix of the queued hubs
     long long* toff;    // [count+1] table offsets
     long long* loff;    // [count+1] list offsets
+    long long* spref;   // [count+1] evaluation-slice prefix
     int* cnt;           // [count] distinct keys inserted (zero between iterations)
+    long long* own;     // [count] d'(v) aggregated on the fly (zero between iterations)
+    void* part;         // per evaluation slice: partial argmax (Arg of the level's mode)
     long long nlev;     // vertices of the level (bound on distinct communities)
 };
 
@@ -654,59 +665,78 @@ __device__ __forceinline__ long long hub_cap(long long deg, long long nlev) {
     return c;
 }
 
+// block-wide exclusive scan of NV int64 values per thread (1024 threads), carried over tiles
+template <int NV>
+struct TileScan {
+    long long w[NV][32];
+    long long carry[NV];
+};
+template <int NV>
+__device__ __forceinline__ void tile_scan(TileScan<NV>& sh, const long long (&x)[NV], long long (&ex)[NV]) {
+    const int lane = lane_id(), wib = threadIdx.x >> 5;
+    long long inc[NV];
+#pragma unroll
+    for (int k = 0; k < NV; ++k) {
+        inc[k] = x[k];
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            long long y = __shfl_up_sync(FULLMASK, inc[k], o);
+            if (lane >= o) inc[k] += y;
+        }
+        if (lane == 31) sh.w[k][wib] = inc[k];
+    }
+    __syncthreads();
+    if (wib == 0) {
+#pragma unroll
+        for (int k = 0; k < NV; ++k) {
+            long long v = sh.w[k][lane], iv = v;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                long long y = __shfl_up_sync(FULLMASK, iv, o);
+                if (lane >= o) iv += y;
+            }
+            sh.w[k][lane] = iv - v;
+        }
+    }
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < NV; ++k) ex[k] = sh.carry[k] + sh.w[k][wib] + inc[k] - x[k];
+    __syncthreads();
+    if (threadIdx.x == blockDim.x - 1)
+#pragma unroll
+        for (int k = 0; k < NV; ++k) sh.carry[k] = ex[k] + x[k];
+    __syncthreads();
+}
+
 // exclusive scans of (chunks, table capacity, list length) over the queued hubs
 __global__ void __launch_bounds__(1024) k_hub_prep(QView queue, const IterCounters* __restrict__ ctr, HubWork h) {
-    __shared__ long long s_w[3][32];
-    __shared__ long long s_carry[3];
+    __shared__ TileScan<3> sh;
     const long long count = (long long)ctr->bin_count[BIN_HUB];
-    const int lane = lane_id(), wib = threadIdx.x >> 5;
-    if (threadIdx.x < 3) s_carry[threadIdx.x] = 0;
+    if (threadIdx.x < 3) sh.carry[threadIdx.x] = 0;
     __syncthreads();
     for (long long t0 = 0; t0 < count; t0 += 1024) {
         const long long i = t0 + threadIdx.x;
-        long long x[3] = {0, 0, 0};
+        long long x[3] = {0, 0, 0}, ex[3];
         if (i < count) {
             const long long deg = queue[i].deg;
             x[0] = (deg + HUB_CH - 1) / HUB_CH;
             x[1] = hub_cap(deg, h.nlev);
             x[2] = deg < h.nlev ? deg : h.nlev;
         }
-        long long inc[3];
-#pragma unroll
-        for (int k = 0; k < 3; ++k) {
-            inc[k] = x[k];
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                long long y = __shfl_up_sync(FULLMASK, inc[k], o);
-                if (lane >= o) inc[k] += y;
-            }
-            if (lane == 31) s_w[k][wib] = inc[k];
-        }
-        __syncthreads();
-        if (wib == 0) {
-#pragma unroll
-            for (int k = 0; k < 3; ++k) {
-                long long v = s_w[k][lane], iv = v;
-#pragma unroll
-                for (int o = 1; o < 32; o <<= 1) {
-                    long long y = __shfl_up_sync(FULLMASK, iv, o);
-                    if (lane >= o) iv += y;
-                }
-                s_w[k][lane] = iv - v;   // exclusive warp offsets
-            }
-        }
-        __syncthreads();
-        if (i < count) {
-            h.pref[i] = s_carry[0] + s_w[0][wib] + inc[0] - x[0];
-            h.toff[i] = s_carry[1] + s_w[1][wib] + inc[1] - x[1];
-            h.loff[i] = s_carry[2] + s_w[2][wib] + inc[2] - x[2];
-        }
-        __syncthreads();
-        if (threadIdx.x == 1023)
-            for (int k = 0; k < 3; ++k) s_carry[k] += s_w[k][31] + inc[k];
-        __syncthreads();
+        tile_scan<3>(sh, x, ex);
+        if (i < count) { h.pref[i] = ex[0]; h.toff[i] = ex[1]; h.loff[i] = ex[2]; }
     }
-    if (threadIdx.x == 0) { h.pref[count] = s_carry[0]; h.toff[count] = s_carry[1]; h.loff[count] = s_carry[2]; }
+    if (threadIdx.x == 0) { h.pref[count] = sh.carry[0]; h.toff[count] = sh.carry[1]; h.loff[count] = sh.carry[2]; }
+}
+
+// last i in [0, count) with pref[i] <= item
+__device__ __forceinline__ long long hub_find(const long long* __restrict__ pref, long long count, long long item) {
+    long long lo = 0, hi = count - 1;
+    while (lo < hi) {
+        long long mid = (lo + hi + 1) >> 1;
+        if (pref[mid] <= item) lo = mid; else hi = mid - 1;
+    }
+    return lo;
 }
 
 template <int M, bool UNIT>
@@ -732,14 +762,9 @@ __global__ void __launch_bounds__(HUB_BT) k_hub_agg(QView queue, DecideArgs a, H
         __syncthreads();
         const long long item = s_item;
         if (item >= total) break;
-        long long lo = 0, hi = count - 1;          // last i with pref[i] <= item
-        while (lo < hi) {
-            long long mid = (lo + hi + 1) >> 1;
-            if (h.pref[mid] <= item) lo = mid; else hi = mid - 1;
-        }
-        const long long i = lo;
+        const long long i = hub_find(h.pref, count, item);
         const QRec q = queue[i];
-        const int v = q.v;
+        const int v = q.v, cv = q.cv;
         const long long j0 = (item - h.pref[i]) * HUB_CH;
         int cc[E];
         VT ww[E];
@@ -755,6 +780,11 @@ __global__ void __launch_bounds__(HUB_BT) k_hub_agg(QView queue, DecideArgs a, H
 #pragma unroll
             for (int k = 0; k < E; ++k) cc[k] = (cc[k] >= 0 && cc[k] != v) ? a.C[cc[k]] : -1;
         }
+        // the own community only feeds d'(v): summed in registers, never inserted
+        long long own = 0;
+#pragma unroll
+        for (int k = 0; k < E; ++k)
+            if (cc[k] == cv) { own += (long long)ww[k]; cc[k] = -1; }
 #pragma unroll
         for (int k = 0; k < E; ++k) {
             const unsigned peers = __match_any_sync(FULLMASK, cc[k] >= 0 ? cc[k] : -1 - lane);
@@ -764,6 +794,8 @@ __global__ void __launch_bounds__(HUB_BT) k_hub_agg(QView queue, DecideArgs a, H
             int slot = ht_insert<ull>(cc[k], (ull)sum, keys, vals, SCAP - 1, hash_slot(cc[k], SCAP - 1), SCAP, &fresh);
             if (fresh) list[atomicAdd(&s_cnt, 1)] = (short)slot;
         }
+        own = warp_sum_ll(own);
+        if (lane == 0 && own) atomicAdd(reinterpret_cast<ull*>(&h.own[i]), (ull)own);
         __syncthreads();
         const int m = s_cnt;
         const long long toff = h.toff[i], cap = h.toff[i + 1] - toff, loff = h.loff[i];
@@ -785,55 +817,103 @@ __global__ void __launch_bounds__(HUB_BT) k_hub_agg(QView queue, DecideArgs a, H
     }
 }
 
+// evaluation slices per hub (at least one, so every hub gets a partial)
+__global__ void __launch_bounds__(1024) k_hub_prep2(const IterCounters* __restrict__ ctr, HubWork h) {
+    __shared__ TileScan<1> sh;
+    const long long count = (long long)ctr->bin_count[BIN_HUB];
+    if (threadIdx.x == 0) sh.carry[0] = 0;
+    __syncthreads();
+    for (long long t0 = 0; t0 < count; t0 += 1024) {
+        const long long i = t0 + threadIdx.x;
+        long long x[1] = {0}, ex[1];
+        if (i < count) x[0] = h.cnt[i] > HUB_EV ? (h.cnt[i] + HUB_EV - 1) / HUB_EV : 1;
+        tile_scan<1>(sh, x, ex);
+        if (i < count) h.spref[i] = ex[0];
+    }
+    if (threadIdx.x == 0) h.spref[count] = sh.carry[0];
+}
+
+// slice (hub i, entries [s HUB_EV, (s+1) HUB_EV) of its list): gains, partial argmax, clear slots
 template <int M, bool UNIT>
 __global__ void __launch_bounds__(HUB_EVAL_BT) k_hub_eval(QView queue, DecideArgs a, HubWork h,
                                                           typename ModeT<M>::ST qW, typename ModeT<M>::ST p) {
     typedef typename ModeT<M>::ST ST;
     typedef Arg<ST, ModeT<M>::PK> A;
     __shared__ A r_a[HUB_EVAL_BT / 32];
-    __shared__ long long r_own[HUB_EVAL_BT / 32];
+    __shared__ long long s_item;
     const int lane = lane_id(), wib = threadIdx.x >> 5;
     const long long count = (long long)a.ctr->bin_count[BIN_HUB];
-    unsigned my_k = 0;
-    for (long long i = blockIdx.x; i < count; i += gridDim.x) {
-        const QRec q = queue[i];
-        const int m = h.cnt[i];
+    if (count == 0) return;
+    const long long total = h.spref[count];
+    A* part = reinterpret_cast<A*>(h.part);
+    for (;;) {
+        if (threadIdx.x == 0) s_item = (long long)atomicAdd(&a.ctr->cursor2, 1ull);
+        __syncthreads();
+        const long long item = s_item;
+        if (item >= total) break;
+        const long long i = hub_find(h.spref, count, item);
+        const int cv = queue[i].cv;
+        const long long dv = queue[i].dv;
+        const long long t0 = (item - h.spref[i]) * HUB_EV;
+        const long long t1 = min(t0 + HUB_EV, (long long)h.cnt[i]);
         const long long toff = h.toff[i], loff = h.loff[i];
-        const int cv = q.cv;
-        const long long dv = q.dv;
         A best;
         best.init(a.idbits, a.idmask);
-        long long own = 0;
-        for (int t = threadIdx.x; t < m; t += HUB_EVAL_BT) {
+        for (long long t = t0 + threadIdx.x; t < t1; t += HUB_EVAL_BT) {
             const long long slot = toff + h.list[loff + t];
             const int c = h.keys[slot];
             const long long wc = (long long)h.vals[slot];
             h.keys[slot] = -1;
             h.vals[slot] = 0;
-            if (c == cv) own = wc;
-            else best.offer(gain<ST>(qW, p, wc, a.Sig[c], dv), c);
+            if (c != cv) best.offer(gain<ST>(qW, p, wc, a.Sig[c], dv), c);
         }
 #pragma unroll
         for (int off = 16; off > 0; off >>= 1) best.xor_merge(off);
-        own = warp_sum_ll(own);
-        if (lane == 0) { r_a[wib] = best; r_own[wib] = own; }
+        if (lane == 0) r_a[wib] = best;
         __syncthreads();
         if (wib == 0) {
-            if (lane < HUB_EVAL_BT / 32) { best = r_a[lane]; own = r_own[lane]; }
-            else { best.init(a.idbits, a.idmask); own = 0; }
+            if (lane < HUB_EVAL_BT / 32) best = r_a[lane];
+            else best.init(a.idbits, a.idmask);
 #pragma unroll
             for (int off = 16; off > 0; off >>= 1) best.xor_merge(off);
-            own = warp_sum_ll(own);
-            if (lane == 0) {
-                if (a.check && own != a.dp[q.v]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
-                a.nextC[q.v] = decide_final<ST>(cv, q.szv, dv, own, q.sigv, best, a.size, qW, p);
-                h.cnt[i] = 0;
-                my_k += (unsigned)m;
-            }
+            if (lane == 0) part[item] = best;
         }
         __syncthreads();
     }
-    if (threadIdx.x == 0 && my_k) atomicAdd(&a.ctr->bin_k[BIN_HUB], (ull)my_k);
+}
+
+// one warp per hub: merge its slices' partials, decide, reset the hub's counters
+template <int M, bool UNIT>
+__global__ void __launch_bounds__(256) k_hub_final(QView queue, DecideArgs a, HubWork h, typename ModeT<M>::ST qW,
+                                                   typename ModeT<M>::ST p) {
+    typedef typename ModeT<M>::ST ST;
+    typedef Arg<ST, ModeT<M>::PK> A;
+    const int lane = lane_id();
+    const long long count = (long long)a.ctr->bin_count[BIN_HUB];
+    const A* part = reinterpret_cast<const A*>(h.part);
+    unsigned my_k = 0;
+    const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+    for (long long i = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < count; i += nw) {
+        A best;
+        best.init(a.idbits, a.idmask);
+        for (long long s = h.spref[i] + lane; s < h.spref[i + 1]; s += 32) {
+            A o = part[s];
+            if (o.valid()) best.offer(o.score(), o.comm());
+        }
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) best.xor_merge(off);
+        if (lane == 0) {
+            const QRec q = queue[i];
+            const long long own = h.own[i];
+            if (a.check && own != a.dp[q.v]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
+            a.nextC[q.v] = decide_final<ST>(q.cv, q.szv, q.dv, own, q.sigv, best, a.size, qW, p);
+            my_k += (unsigned)h.cnt[i] + (own ? 1u : 0u);
+            h.cnt[i] = 0;
+            h.own[i] = 0;
+        }
+    }
+    ull k = block_sum_ull<256>((ull)my_k);
+    if (threadIdx.x == 0 && k) atomicAdd(&a.ctr->bin_k[BIN_HUB], k);
 }
 
 // per level: number of rows longer than t, and the table / list space they can need
