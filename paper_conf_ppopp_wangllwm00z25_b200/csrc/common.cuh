@@ -143,23 +143,49 @@ __device__ __forceinline__ long long warp_append(bool flag, ull* counter) {
     return flag ? (long long)(base + __popc(m & lanemask_lt())) : -1;
 }
 
-// Sum of `x` over the lanes of this lane's __match_any_sync group `peers`.
-// 32-bit values use redux.sync with the group mask (every lane of a group
-// passes the same mask, as the warp-primitive contract requires; the
-// match_any + reduce pattern of Alg. 2); 64-bit values go through
-// a per-warp shared-memory scratch (`scratch` = 32 slots of this warp).
-__device__ __forceinline__ unsigned group_sum(unsigned peers, unsigned x, unsigned*) {
-    return __reduce_add_sync(peers, x);
-}
-__device__ __forceinline__ ull group_sum(unsigned peers, ull x, ull* scratch) {
-    const int lane = threadIdx.x & 31;
+// Sum of `x` over the lanes of this lane's __match_any_sync group `peers`
+// (the match_any + reduce pattern of Alg. 2).  Each lane adds its
+// value into the group leader's slot of a per-warp shared scratch (32 slots).
+// redux.sync is not used: with several groups per warp (different masks) it
+// falls into a per-group serial path on sm_100.  32-bit adds are native
+// shared atomics; the 64-bit variant (used only when sums can reach 2^32) is a
+// CAS loop in hardware, hence the 32-bit aggregates wherever they suffice.
+__device__ __forceinline__ unsigned group_sum(unsigned peers, unsigned x, unsigned* scratch) {
+    const int lane = threadIdx.x & 31, leader = __ffs(peers) - 1;
     scratch[lane] = 0;
     __syncwarp();
-    atomicAdd(&scratch[__ffs(peers) - 1], x);
+    if (x) atomicAdd(&scratch[leader], x);
     __syncwarp();
-    ull r = scratch[__ffs(peers) - 1];
+    const unsigned r = scratch[leader];
     __syncwarp();
     return r;
+}
+__device__ __forceinline__ ull group_sum(unsigned peers, ull x, ull* scratch) {
+    const int lane = threadIdx.x & 31, leader = __ffs(peers) - 1;
+    scratch[lane] = 0;
+    __syncwarp();
+    if (x) atomicAdd(&scratch[leader], x);
+    __syncwarp();
+    const ull r = scratch[leader];
+    __syncwarp();
+    return r;
+}
+
+// warp-aggregated append of the lanes with `fresh` set (within group mask gmask)
+// to list[*cnt ...]: one shared atomic per group instead of one per lane.  All
+// 32 lanes must call it converged.
+template <typename LT>
+__device__ __forceinline__ void append_fresh(bool fresh, int slot, unsigned gmask, int* cnt, LT* list) {
+    const int lane = threadIdx.x & 31;
+    const unsigned fm = __ballot_sync(FULLMASK, fresh) & gmask;
+    int base = 0;
+    if (fresh && lane == __ffs(fm) - 1) base = atomicAdd(cnt, __popc(fm));
+    base = __shfl_sync(FULLMASK, base, fm ? __ffs(fm) - 1 : lane);
+    if (fresh) {
+        unsigned lt;
+        asm("mov.u32 %0, %%lanemask_lt;" : "=r"(lt));
+        list[base + __popc(fm & lt)] = (LT)slot;
+    }
 }
 
 __device__ __forceinline__ long long warp_sum_ll(long long x) {

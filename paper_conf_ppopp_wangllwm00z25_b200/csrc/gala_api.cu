@@ -679,7 +679,27 @@ struct VTimer {
 // (reading c10: the diagonal carries D_C(c) once).  See k_phase2.cuh for
 // the per-community aggregation paths.  Coarse d(c) = Sigma_tot(c), s(c) = diagonal.
 #define AGG_BLOCK_BT 512
-static size_t agg_block_smem(int scap) { return (size_t)scap * (sizeof(ull) + sizeof(int)) + (size_t)(scap / 2) * sizeof(int); }
+template <typename V>
+static size_t agg_block_smem(int scap) { return (size_t)scap * (sizeof(V) + sizeof(int)) + (size_t)(scap / 2) * sizeof(int); }
+
+// warp / block aggregation launches with V = table value type (32-bit iff W < 2^32)
+template <typename V>
+static void agg_launch_small(gala_graph_s* g, const AggArgs& a, bool unit, int scap, long long k) {
+    cudaStream_t st = g->stream;
+    const int big = g->num_sms * 8;
+    if (unit) k_agg_warp<true, V><<<big, 256, 0, st>>>(a);
+    else k_agg_warp<false, V><<<big, 256, 0, st>>>(a);
+    CKL();
+    if (scap > AGG_WSLOTS) {
+        const size_t sm = agg_block_smem<V>(scap);
+        CK(cudaFuncSetAttribute(k_agg_block<AGG_BLOCK_BT, true, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+        CK(cudaFuncSetAttribute(k_agg_block<AGG_BLOCK_BT, false, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+        const int gb = (int)std::min<long long>(k, (long long)g->num_sms * 4);
+        if (unit) k_agg_block<AGG_BLOCK_BT, true, V><<<gb, AGG_BLOCK_BT, sm, st>>>(a, scap);
+        else k_agg_block<AGG_BLOCK_BT, false, V><<<gb, AGG_BLOCK_BT, sm, st>>>(a, scap);
+        CKL();
+    }
+}
 
 // Aggregate the rows of `cur` (nrows rows, each with a row-id array) into k
 // target rows: target of row v is newid[v]; entries become (newid[u], w) and
@@ -730,18 +750,9 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
     CKL();
     AggArgs a;
     a.k = k; a.ent = ent; a.eoff = eoff; a.tkey = tkey; a.tval = tval; a.dn = dn; a.snew = snew;
-    if (unit) k_agg_warp<true><<<big, 256, 0, st>>>(a);
-    else k_agg_warp<false><<<big, 256, 0, st>>>(a);
-    CKL();
-    if (scap > AGG_WSLOTS) {
-        const size_t sm = agg_block_smem(scap);
-        CK(cudaFuncSetAttribute(k_agg_block<AGG_BLOCK_BT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
-        CK(cudaFuncSetAttribute(k_agg_block<AGG_BLOCK_BT, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
-        const int gb = (int)std::min<long long>(k, (long long)g->num_sms * 4);
-        if (unit) k_agg_block<AGG_BLOCK_BT, true><<<gb, AGG_BLOCK_BT, sm, st>>>(a, scap);
-        else k_agg_block<AGG_BLOCK_BT, false><<<gb, AGG_BLOCK_BT, sm, st>>>(a, scap);
-        CKL();
-    }
+    const bool v32 = g->W < ((int64_t)1 << 32);   // every aggregated weight is <= W
+    if (v32) agg_launch_small<unsigned>(g, a, unit, scap, k);
+    else agg_launch_small<ull>(g, a, unit, scap, k);
     vt.lap("agg: warp+block");
     int nbig = 0;
     CK(cudaMemcpyAsync(&nbig, nbig_dev, sizeof(int), cudaMemcpyDeviceToHost, st));
@@ -761,8 +772,9 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
         CK(cudaMemsetAsync(gcnt, 0, sizeof(int) * nbig, st));
         vt.lap("agg: big alloc+clear");
         const int bpc = 32;
-        if (unit) k_agg_big_insert<true><<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
-        else k_agg_big_insert<false><<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
+        if (unit) k_agg_big_insert<true, unsigned><<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
+        else if (v32) k_agg_big_insert<false, unsigned><<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
+        else k_agg_big_insert<false, ull><<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
         CKL();
         vt.lap("agg: big insert");
         k_agg_big_emit<<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
@@ -1000,14 +1012,15 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
             const i128 N_start = carry_N(wk.h_carry);
             // gain arithmetic for this level (reading c16):
             //   |score| <= max(p,q) * W * dmax  (dmax = max weighted degree of the level)
-            //   int64 iff that bound < 2^62; packed (score,-c) keys iff < 2^(62 - idbits); 32-bit
-            //   aggregates iff W < 2^31.
+            //   int64 iff that bound < 2^62; packed (score,-c) keys iff < 2^(62 - idbits); the
+            //   int64 modes sum per-vertex aggregates in 32 bits, so they also need dmax < 2^32
+            //   (else the int128 mode, whose aggregates are 64-bit).
             int idbits = 1;
             while (idbits < 31 && ((int64_t)1 << idbits) < nl) ++idbits;
             const long double bound = (long double)mpq * (long double)W * (long double)std::max<int64_t>(dmax, 1);
             int mode = DM_FAST;
-            if (g->opt_force_i128 || bound >= 0x1p62L) mode = DM_W128;
-            else if (W >= ((int64_t)1 << 31) || bound * (long double)((int64_t)1 << idbits) >= 0x1p62L || g->opt_force_wide)
+            if (g->opt_force_i128 || bound >= 0x1p62L || dmax >= ((int64_t)1 << 32)) mode = DM_W128;
+            else if (bound * (long double)((int64_t)1 << idbits) >= 0x1p62L || g->opt_force_wide)
                 mode = DM_W64;
             ls.i128path = mode;
             const long long qW64 = (long long)qW128, p64 = (long long)p;
@@ -1413,8 +1426,8 @@ static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_level
             while (idbits < 31 && ((int64_t)1 << idbits) < nl) ++idbits;
             const long double bound = (long double)mpq * (long double)W * (long double)std::max<int64_t>(dmax, 1);
             int mode = DM_FAST;
-            if (g->opt_force_i128 || bound >= 0x1p62L) mode = DM_W128;
-            else if (W >= ((int64_t)1 << 31) || bound * (long double)((int64_t)1 << idbits) >= 0x1p62L || g->opt_force_wide)
+            if (g->opt_force_i128 || bound >= 0x1p62L || dmax >= ((int64_t)1 << 32)) mode = DM_W128;
+            else if (bound * (long double)((int64_t)1 << idbits) >= 0x1p62L || g->opt_force_wide)
                 mode = DM_W64;
             ls.i128path = mode;
             const long long qW64 = (long long)qW128, p64 = (long long)p;

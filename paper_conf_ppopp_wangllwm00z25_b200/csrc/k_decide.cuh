@@ -27,7 +27,7 @@
 enum { DM_FAST = 0, DM_W64 = 1, DM_W128 = 2 };
 template <int M> struct ModeT;
 template <> struct ModeT<DM_FAST> { typedef long long ST; typedef unsigned VT; static constexpr bool PK = true; };
-template <> struct ModeT<DM_W64> { typedef long long ST; typedef ull VT; static constexpr bool PK = false; };
+template <> struct ModeT<DM_W64> { typedef long long ST; typedef unsigned VT; static constexpr bool PK = false; };
 template <> struct ModeT<DM_W128> { typedef i128 ST; typedef ull VT; static constexpr bool PK = false; };
 
 // running argmax over (score, -community)
@@ -333,11 +333,11 @@ __global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB) k_decide_wa
                 // combine equal communities of this chunk first (one insert per community)
                 const unsigned peers = __match_any_sync(FULLMASK, cc[k] >= 0 ? cc[k] : -1 - lane) & gmask;
                 const VT sum = UNIT ? (VT)__popc(peers) : group_sum(peers, cc[k] >= 0 ? ww[k] : (VT)0, scratch);
-                if (cc[k] >= 0 && lane == __ffs(peers) - 1) {
-                    bool fresh;
-                    int slot = ht_insert<VT>(cc[k], sum, keys, vals, WMASK, hash_slot(cc[k], WMASK), WCAP, &fresh);
-                    if (fresh) list[atomicAdd(cnt, 1)] = (short)slot;
-                }
+                bool fresh = false;
+                int slot = -1;
+                if (cc[k] >= 0 && lane == __ffs(peers) - 1)
+                    slot = ht_insert<VT>(cc[k], sum, keys, vals, WMASK, hash_slot(cc[k], WMASK), WCAP, &fresh);
+                append_fresh<short>(fresh, slot, gmask, cnt, list);
             }
         }
         __syncwarp();
@@ -463,16 +463,16 @@ __global__ void __launch_bounds__(BT) k_decide_block(QView queue, int bin, Decid
             for (int k = 0; k < E; ++k) {
                 const unsigned peers = __match_any_sync(FULLMASK, cc[k] >= 0 ? cc[k] : -1 - lane);
                 const VT sum = UNIT ? (VT)__popc(peers) : group_sum(peers, cc[k] >= 0 ? ww[k] : (VT)0, s_scr[wib]);
-                if (cc[k] < 0 || lane != __ffs(peers) - 1) continue;
-                bool fresh;
-                int slot = ht_insert<VT>(cc[k], sum, keys, vals, smask, hash_slot(cc[k], smask), win, &fresh);
-                if (slot >= 0) {
-                    if (fresh) list[atomicAdd(&s_cnt, 1)] = slot;
-                } else {
-                    slot = ht_insert<ull>(cc[k], (ull)sum, gkeys, gvals, gmask, hash_slot2(cc[k], gmask), (int)gc,
-                                          &fresh);
-                    if (fresh) glist[atomicAdd(&s_gcnt, 1)] = slot;
+                bool fresh = false, gfresh = false;
+                int slot = -1, gslot = -1;
+                if (cc[k] >= 0 && lane == __ffs(peers) - 1) {
+                    slot = ht_insert<VT>(cc[k], sum, keys, vals, smask, hash_slot(cc[k], smask), win, &fresh);
+                    if (slot < 0)
+                        gslot = ht_insert<ull>(cc[k], (ull)sum, gkeys, gvals, gmask, hash_slot2(cc[k], gmask), (int)gc,
+                                               &gfresh);
                 }
+                append_fresh<int>(fresh, slot, FULLMASK, &s_cnt, list);
+                if (__any_sync(FULLMASK, gfresh)) append_fresh<int>(gfresh, gslot, FULLMASK, &s_gcnt, glist);
             }
         }
         __syncthreads();
@@ -745,7 +745,7 @@ __global__ void __launch_bounds__(HUB_BT) k_hub_agg(QView queue, DecideArgs a, H
     constexpr int SCAP = 2 * HUB_CH;
     constexpr int E = HUB_CH / HUB_BT;
     __shared__ int keys[SCAP];
-    __shared__ ull vals[SCAP];
+    __shared__ VT vals[SCAP];
     __shared__ short list[HUB_CH];
     __shared__ VT s_scr[HUB_BT / 32][32];
     __shared__ long long s_item;
@@ -789,10 +789,11 @@ __global__ void __launch_bounds__(HUB_BT) k_hub_agg(QView queue, DecideArgs a, H
         for (int k = 0; k < E; ++k) {
             const unsigned peers = __match_any_sync(FULLMASK, cc[k] >= 0 ? cc[k] : -1 - lane);
             const VT sum = UNIT ? (VT)__popc(peers) : group_sum(peers, cc[k] >= 0 ? ww[k] : (VT)0, s_scr[wib]);
-            if (cc[k] < 0 || lane != __ffs(peers) - 1) continue;
-            bool fresh;
-            int slot = ht_insert<ull>(cc[k], (ull)sum, keys, vals, SCAP - 1, hash_slot(cc[k], SCAP - 1), SCAP, &fresh);
-            if (fresh) list[atomicAdd(&s_cnt, 1)] = (short)slot;
+            bool fresh = false;
+            int slot = -1;
+            if (cc[k] >= 0 && lane == __ffs(peers) - 1)
+                slot = ht_insert<VT>(cc[k], sum, keys, vals, SCAP - 1, hash_slot(cc[k], SCAP - 1), SCAP, &fresh);
+            append_fresh<short>(fresh, slot, FULLMASK, &s_cnt, list);
         }
         own = warp_sum_ll(own);
         if (lane == 0 && own) atomicAdd(reinterpret_cast<ull*>(&h.own[i]), (ull)own);
@@ -805,7 +806,7 @@ __global__ void __launch_bounds__(HUB_BT) k_hub_agg(QView queue, DecideArgs a, H
         for (int t = threadIdx.x; t < m; t += HUB_BT) {
             const int slot = list[t];
             const int c = keys[slot];
-            const ull wv = vals[slot];
+            const ull wv = (ull)vals[slot];
             keys[slot] = -1;
             vals[slot] = 0;
             bool fresh;

@@ -334,10 +334,9 @@ __global__ void __launch_bounds__(256) k_dp_full(IterCounters* __restrict__ ctr,
                                                  const int64_t* __restrict__ w, const int32_t* __restrict__ C,
                                                  int64_t* __restrict__ dp, int mode, long long fnum, long long fden,
                                                  int32_t* __restrict__ ckey, int* __restrict__ carry_valid) {
-    __shared__ ull s_scr[8][32];
     if (use_delta(ctr, nnz, mode, fnum, fden)) return;
     if (ckey && blockIdx.x == 0 && threadIdx.x == 0) carry_valid[0] = 1;   // rewritten below for every entry
-    const int lane = lane_id(), wib = threadIdx.x >> 5;
+    const int lane = lane_id();
     const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
     for (long long base = (((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * 128; base < nnz;
          base += nw * 128) {
@@ -365,10 +364,19 @@ __global__ void __launch_bounds__(256) k_dp_full(IterCounters* __restrict__ ctr,
         for (int t = 0; t < 4; ++t) {
             const bool hit = r[t] >= 0 && u[t] != r[t] && cu[t] == cr[t];
             const unsigned peers = __match_any_sync(FULLMASK, r[t]);
-            const ull x = hit ? (ull)wt[t] : 0ull;
             ull sum;
-            if (UNIT) sum = (ull)__popc(__ballot_sync(FULLMASK, hit) & peers);
-            else sum = group_sum(peers, x, s_scr[wib]);
+            if (UNIT) {
+                sum = (ull)__popc(__ballot_sync(FULLMASK, hit) & peers);
+            } else {   // rows are contiguous lane runs: segmented tree sum, leader = first lane of the run
+                long long x = hit ? wt[t] : 0;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const long long y = __shfl_down_sync(FULLMASK, x, o);
+                    const int ro = __shfl_down_sync(FULLMASK, r[t], o);
+                    if (lane + o < 32 && ro == r[t]) x += y;
+                }
+                sum = (ull)x;
+            }
             if (r[t] >= 0 && lane == __ffs(peers) - 1 && sum) atomicAdd(reinterpret_cast<ull*>(&dp[r[t]]), sum);
         }
     }

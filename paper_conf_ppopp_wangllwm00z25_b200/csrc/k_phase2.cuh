@@ -250,25 +250,27 @@ __device__ __forceinline__ int agg_insert(int key, VT wt, int* keys, VT* vals, u
 // `nt` threads (tid = this thread's index among them, whole warps) stream
 // segment entries [s0, s1) with 4 entries per lane in flight; equal keys of
 // every 32-entry chunk are combined before inserting.
-template <bool UNIT, typename VT>
+// TV: table value type; SV: per-chunk group-sum type (32-bit whenever W < 2^32, so
+// the shared-memory adds are native)
+template <bool UNIT, typename TV, typename SV>
 __device__ __forceinline__ void agg_segment(const AggArgs& a, long long s0, long long s1, int tid, int nt, int* keys,
-                                            VT* vals, unsigned mask, int* list, int* cnt, ull* scratch) {
+                                            TV* vals, unsigned mask, int* list, int* cnt, SV* scratch) {
     const int lane = tid & 31;
     for (long long r0 = s0 + (tid & ~31) * 4; r0 < s1; r0 += (long long)nt * 4) {   // warp-uniform
         int kk[4];
-        ull ww[4];
+        SV ww[4];
 #pragma unroll
         for (int t = 0; t < 4; ++t) {
             long long j = r0 + lane + 32 * t;
             kk[t] = j < s1 ? a.tkey[j] : -1;
-            ww[t] = (j < s1 && !UNIT) ? (ull)a.tval[j] : 1ull;
+            ww[t] = (j < s1 && !UNIT) ? (SV)a.tval[j] : (SV)1;
         }
 #pragma unroll
         for (int t = 0; t < 4; ++t) {
             if (r0 + 32 * t >= s1) break;
             const unsigned peers = __match_any_sync(FULLMASK, kk[t] >= 0 ? kk[t] : -1 - lane);
-            const ull sum = UNIT ? (ull)__popc(peers) : group_sum(peers, kk[t] >= 0 ? ww[t] : 0ull, scratch);
-            if (kk[t] >= 0 && lane == __ffs(peers) - 1) agg_insert<VT>(kk[t], (VT)sum, keys, vals, mask, list, cnt);
+            const SV sum = UNIT ? (SV)__popc(peers) : group_sum(peers, kk[t] >= 0 ? ww[t] : (SV)0, scratch);
+            if (kk[t] >= 0 && lane == __ffs(peers) - 1) agg_insert<TV>(kk[t], (TV)sum, keys, vals, mask, list, cnt);
         }
     }
 }
@@ -291,16 +293,16 @@ __device__ __forceinline__ void agg_emit(const AggArgs& a, long long c, int m, c
 }
 
 #define AGG_WSLOTS 256
-template <bool UNIT>
+template <bool UNIT, typename V>
 __global__ void __launch_bounds__(256) k_agg_warp(AggArgs a) {
     __shared__ int s_key[8][AGG_WSLOTS];
-    __shared__ ull s_val[8][AGG_WSLOTS];
+    __shared__ V s_val[8][AGG_WSLOTS];
     __shared__ int s_list[8][AGG_WSLOTS / 2];
     __shared__ int s_cnt[8];
-    __shared__ ull s_scr[8][32];
+    __shared__ V s_scr[8][32];
     const int lane = lane_id(), wib = threadIdx.x >> 5;
     int* keys = s_key[wib];
-    ull* vals = s_val[wib];
+    V* vals = s_val[wib];
     int* list = s_list[wib];
     for (int j = lane; j < AGG_WSLOTS; j += 32) { keys[j] = -1; vals[j] = 0; }
     if (lane == 0) s_cnt[wib] = 0;
@@ -310,25 +312,25 @@ __global__ void __launch_bounds__(256) k_agg_warp(AggArgs a) {
         long long cap = agg_cap(a.ent[c], a.k);
         if (cap == 0) { if (lane == 0) a.dn[c] = 0; continue; }
         if (cap > AGG_WSLOTS) continue;
-        agg_segment<UNIT, ull>(a, a.eoff[c], a.eoff[c + 1], lane, 32, keys, vals, (unsigned)cap - 1, list, &s_cnt[wib],
-                               s_scr[wib]);
+        agg_segment<UNIT, V, V>(a, a.eoff[c], a.eoff[c + 1], lane, 32, keys, vals, (unsigned)cap - 1, list,
+                                &s_cnt[wib], s_scr[wib]);
         __syncwarp();
         int m = s_cnt[wib];
-        agg_emit<ull>(a, c, m, list, keys, vals, lane, 32);
+        agg_emit<V>(a, c, m, list, keys, vals, lane, 32);
         __syncwarp();
         if (lane == 0) { a.dn[c] = m; s_cnt[wib] = 0; }
         __syncwarp();
     }
 }
 
-template <int BT, bool UNIT>
+template <int BT, bool UNIT, typename V>
 __global__ void __launch_bounds__(BT) k_agg_block(AggArgs a, int scap) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    ull* vals = reinterpret_cast<ull*>(smem_raw);
-    int* keys = reinterpret_cast<int*>(smem_raw + (size_t)scap * sizeof(ull));
+    V* vals = reinterpret_cast<V*>(smem_raw);
+    int* keys = reinterpret_cast<int*>(smem_raw + (size_t)scap * sizeof(V));
     int* list = keys + scap;
     __shared__ int s_cnt;
-    __shared__ ull s_scr[BT / 32][32];
+    __shared__ V s_scr[BT / 32][32];
     const int wib = threadIdx.x >> 5;
     for (int j = threadIdx.x; j < scap; j += BT) { keys[j] = -1; vals[j] = 0; }
     if (threadIdx.x == 0) s_cnt = 0;
@@ -336,11 +338,11 @@ __global__ void __launch_bounds__(BT) k_agg_block(AggArgs a, int scap) {
     for (long long c = blockIdx.x; c < a.k; c += gridDim.x) {
         long long cap = agg_cap(a.ent[c], a.k);
         if (cap <= AGG_WSLOTS || cap > scap) continue;   // block-uniform
-        agg_segment<UNIT, ull>(a, a.eoff[c], a.eoff[c + 1], threadIdx.x, BT, keys, vals, (unsigned)cap - 1, list,
-                               &s_cnt, s_scr[wib]);
+        agg_segment<UNIT, V, V>(a, a.eoff[c], a.eoff[c + 1], threadIdx.x, BT, keys, vals, (unsigned)cap - 1, list,
+                                &s_cnt, s_scr[wib]);
         __syncthreads();
         int m = s_cnt;
-        agg_emit<ull>(a, c, m, list, keys, vals, threadIdx.x, BT);
+        agg_emit<V>(a, c, m, list, keys, vals, threadIdx.x, BT);
         __syncthreads();
         if (threadIdx.x == 0) { a.dn[c] = m; s_cnt = 0; }
         __syncthreads();
@@ -348,12 +350,12 @@ __global__ void __launch_bounds__(BT) k_agg_block(AggArgs a, int scap) {
 }
 
 // big communities: BPC blocks per community stream chunks of its segment into its global table
-template <bool UNIT>
+template <bool UNIT, typename V>
 __global__ void __launch_bounds__(256) k_agg_big_insert(AggArgs a, const int32_t* __restrict__ bigc, int nbig,
                                                         const long long* __restrict__ goff, int* __restrict__ gkeys,
                                                         ull* __restrict__ gvals, int* __restrict__ glist,
                                                         int* __restrict__ gcnt, int bpc) {
-    __shared__ ull s_scr[8][32];
+    __shared__ V s_scr[8][32];
     const int wib = threadIdx.x >> 5;
     for (long long b = blockIdx.x; b < (long long)nbig * bpc; b += gridDim.x) {
         const int bi = (int)(b / bpc), part = (int)(b % bpc);
@@ -362,8 +364,8 @@ __global__ void __launch_bounds__(256) k_agg_big_insert(AggArgs a, const int32_t
         const unsigned mask = (unsigned)(goff[bi + 1] - off) - 1u;
         const long long s0 = a.eoff[c], len = a.eoff[c + 1] - s0;
         const long long lo = s0 + len * part / bpc, hi = s0 + len * (part + 1) / bpc;
-        agg_segment<UNIT, ull>(a, lo, hi, threadIdx.x, 256, gkeys + off, gvals + off, mask, glist + off / 2,
-                               &gcnt[bi], s_scr[wib]);
+        agg_segment<UNIT, ull, V>(a, lo, hi, threadIdx.x, 256, gkeys + off, gvals + off, mask, glist + off / 2,
+                                  &gcnt[bi], s_scr[wib]);
     }
 }
 
