@@ -294,7 +294,8 @@ struct Work {
     ull* gvals = nullptr;
     int* glist = nullptr;
     long long gcap = 0;
-    int gblocks = 0;
+    int gblocks = 0;          // max over modes (spill-table count)
+    int gblocks_m[3] = {0, 0, 0};
     // hub tables (k_hub_*), sized per level for the rows longer than the block bin
     bool hub_on = false;
     HubWork hw = {};
@@ -419,7 +420,7 @@ static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, typename M
     if (maxdeg > g->bins[BIN_WARP2]) {
         const int smem_cap = g->hub_smem_slots;
         e = tm.begin();
-        k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT><<<wk.gblocks, BLOCK_BT, block_smem_bytes<M>(smem_cap), st>>>(
+        k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT><<<wk.gblocks_m[M], BLOCK_BT, block_smem_bytes<M>(smem_cap), st>>>(
             qview(wk.queues, qs, BIN_BLOCK), BIN_BLOCK, a, qW, p, smem_cap, wk.gkeys, wk.gvals, wk.glist, wk.gcap);
         CKL();
         tm.end(KC_DEC_BLOCK, e);
@@ -918,7 +919,20 @@ static void ensure_workspace(gala_graph_s* g) {
             CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, DM_W64, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)block_smem_bytes<DM_W64>(cap)));
             CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, DM_W128, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)block_smem_bytes<DM_W128>(cap)));
             CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, DM_W128, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)block_smem_bytes<DM_W128>(cap)));
-            CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_decide_block<BLOCK_BT, BLOCK_E, DM_W128, false>, BLOCK_BT, block_smem_bytes<DM_W128>(cap)));
+            // resident blocks per SM of each mode's block kernel (the grid of a launch; spill
+            // tables are sized for the largest)
+            auto occ = [&](const void* f, size_t sm) {
+                int b = 0;
+                CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, f, BLOCK_BT, sm));
+                return std::max(b, 1);
+            };
+            wk.gblocks_m[DM_FAST] = g->num_sms * std::min(occ((const void*)k_decide_block<BLOCK_BT, BLOCK_E, DM_FAST, true>, block_smem_bytes<DM_FAST>(cap)),
+                                                          occ((const void*)k_decide_block<BLOCK_BT, BLOCK_E, DM_FAST, false>, block_smem_bytes<DM_FAST>(cap)));
+            wk.gblocks_m[DM_W64] = g->num_sms * std::min(occ((const void*)k_decide_block<BLOCK_BT, BLOCK_E, DM_W64, true>, block_smem_bytes<DM_W64>(cap)),
+                                                         occ((const void*)k_decide_block<BLOCK_BT, BLOCK_E, DM_W64, false>, block_smem_bytes<DM_W64>(cap)));
+            wk.gblocks_m[DM_W128] = g->num_sms * std::min(occ((const void*)k_decide_block<BLOCK_BT, BLOCK_E, DM_W128, true>, block_smem_bytes<DM_W128>(cap)),
+                                                          occ((const void*)k_decide_block<BLOCK_BT, BLOCK_E, DM_W128, false>, block_smem_bytes<DM_W128>(cap)));
+            per_sm = std::max(std::max(wk.gblocks_m[0], wk.gblocks_m[1]), wk.gblocks_m[2]) / g->num_sms;
             set_warp_smem<32, 128, DM_FAST>(); set_warp_smem<32, 128, DM_W64>(); set_warp_smem<32, 128, DM_W128>();
             set_warp_smem<32, 512, DM_FAST>(); set_warp_smem<32, 512, DM_W64>(); set_warp_smem<32, 512, DM_W128>();
             wk.gblocks = g->num_sms * std::max(per_sm, 1);
