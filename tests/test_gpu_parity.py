@@ -201,3 +201,11 @@ def test_invalid_inputs_rejected():
 def test_lfr1m_full_size_parity():
     """BASELINE configs[1] at full size, in bench.py's launch configuration."""
     assert_parity(gg.make("lfr1m"))
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("name", ["rmat_lj", "orkut"])
+def test_full_size_parity_skewed(name):
+    """BASELINE configs[2] / configs[3] at full size: block and hub paths (rows up to 667k
+    entries on coarse R-MAT levels), per-iteration N / moved / active / pruned and final labels."""
+    assert_parity(gg.make(name), labels=False)
