@@ -153,6 +153,8 @@ void gala_graph_free(gala_graph g);
  *                          update (default 0; trades nnz*4 bytes for one gather per entry)
  *   "hub_smem_slots" power of two in [64, 16384], shared-memory slots of the block hash table
  *   "cuda_graph"     0/1   run each level's iterations as a conditional CUDA graph (default 1)
+ *   "concurrent"     0/1   run the degree bins' decide kernels as parallel branches on side
+ *                          streams (default 0: measured slower on B200 -- the bins contend for L2 and smem; off whenever "timing" is on)
  *   "log_cap"        device iteration-log capacity (default 4096)
  *   "sync_mode"      multi-GPU label exchange: 0 adaptive (default), 1 dense, 2 sparse
  *   "verbose"        0/1   host-side phase timings on stderr

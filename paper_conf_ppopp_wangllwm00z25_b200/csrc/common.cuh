@@ -35,6 +35,7 @@ struct IterCounters {
     ull ticket;             // last-block-done ticket of k_reduce
     ull delta_used;         // 1 if the delta d' update ran this iteration
     ull cursor2;            // dynamic work cursor of the hub evaluation
+    ull n_items;            // delta-update work items (one per light mover, one per chunk of a heavy one)
 };
 
 // Queue record of an active vertex, written by k_prune_bin (which already

@@ -129,6 +129,49 @@ struct gala_graph_s {
     int sync_mode = 0;
     std::vector<long long> dbounds0;   // level-0 owned ranges of all ranks
     struct Work* wk = nullptr;   // persistent run workspace (sized for level 0, reused by every run)
+    // side streams of the decide fork: the bins' decide kernels are independent (disjoint
+    // vertices, per-bin cursors and tables), so they run as parallel graph branches
+    int opt_concurrent = 0;
+    cudaStream_t side[4] = {nullptr, nullptr, nullptr, nullptr};
+    cudaEvent_t ev_fork = nullptr, ev_join[4] = {nullptr, nullptr, nullptr, nullptr};
+};
+
+// Fork/join of independent launches onto the side streams.  Inside a stream
+// capture the event record/wait pairs become graph edges (parallel branches of
+// the conditional body); outside they are plain cross-stream dependencies.
+// Per-kernel timing (events on the main stream) keeps everything serial.
+struct Fork {
+    gala_graph_s* g;
+    bool on;
+    int used = 0;
+    explicit Fork(gala_graph_s* gg) : g(gg), on(gg->opt_concurrent && !gg->opt_timing) {
+        if (!on) return;
+        if (!g->ev_fork) {
+            CK(cudaEventCreateWithFlags(&g->ev_fork, cudaEventDisableTiming));
+            for (int i = 0; i < 4; ++i) {
+                CK(cudaStreamCreateWithFlags(&g->side[i], cudaStreamNonBlocking));
+                CK(cudaEventCreateWithFlags(&g->ev_join[i], cudaEventDisableTiming));
+            }
+        }
+        CK(cudaEventRecord(g->ev_fork, g->stream));
+    }
+    // stream for branch i (0..3); the main stream when forking is off
+    cudaStream_t branch(int i) {
+        if (!on) return g->stream;
+        CK(cudaStreamWaitEvent(g->side[i], g->ev_fork, 0));
+        used |= 1 << i;
+        return g->side[i];
+    }
+    void join() {
+        if (!on) return;
+        for (int i = 0; i < 4; ++i)
+            if (used & (1 << i)) {
+                CK(cudaEventRecord(g->ev_join[i], g->side[i]));
+                CK(cudaStreamWaitEvent(g->stream, g->ev_join[i], 0));
+            }
+        used = 0;
+    }
+    ~Fork() { join(); }
 };
 
 // ------------------------------------------------------------------ memory
@@ -280,7 +323,7 @@ static void gamma_to_pq(double gamma, int64_t* p, int64_t* q) {
 struct Work {
     cudaStream_t st;
     int64_t ncap, nnzcap;
-    int32_t *C = nullptr, *size = nullptr, *stamp = nullptr, *mv_v = nullptr, *mv_old = nullptr, *nextC = nullptr;
+    int32_t *C = nullptr, *size = nullptr, *stamp = nullptr, *mv_v = nullptr, *mv_old = nullptr, *mv_chunk = nullptr, *nextC = nullptr;
     QRec* queues = nullptr;
     int32_t* ckey = nullptr;   // level-0 per-entry neighbour community
     int64_t *Sig = nullptr, *d = nullptr, *s = nullptr, *dp = nullptr;
@@ -308,7 +351,7 @@ struct Work {
     cudaEvent_t ev[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};
     void release() {
         for (auto& e : ev) if (e) { cudaEventDestroy(e); e = nullptr; }
-        dfree(C, st); dfree(size, st); dfree(stamp, st); dfree(mv_v, st); dfree(mv_old, st); dfree(nextC, st);
+        dfree(C, st); dfree(size, st); dfree(stamp, st); dfree(mv_v, st); dfree(mv_old, st); dfree(mv_chunk, st); dfree(nextC, st);
         dfree(queues, st); dfree(ckey, st); dfree(Sig, st); dfree(d, st); dfree(s, st); dfree(dp, st); dfree(ctr, st);
         dfree(carry, st); dfree(log, st); dfree(part_dc, st); dfree(part_min, st); dfree(part_s2, st);
         dfree(gkeys, st); dfree(gvals, st); dfree(glist, st);
@@ -347,9 +390,8 @@ static size_t block_smem_bytes(int cap) { return (size_t)cap * (sizeof(typename 
 // multi-block hub path (bin BIN_HUB), only on levels that have such rows
 template <int M, bool UNIT>
 static void launch_hub(gala_graph_s* g, Work& wk, const DecideArgs& a, typename ModeT<M>::ST qW,
-                       typename ModeT<M>::ST p, Timer& tm) {
+                       typename ModeT<M>::ST p, Timer& tm, cudaStream_t st) {
     if (!wk.hub_on) return;
-    cudaStream_t st = g->stream;
     const QView q = qview(wk.queues, wk.ncap, BIN_HUB);
     cudaEvent_t e = tm.begin();
     k_hub_prep<<<1, 1024, 0, st>>>(q, wk.ctr, wk.hw);
@@ -371,6 +413,7 @@ static void launch_single(gala_graph_s* g, Work& wk, const DecideArgs& a, typena
     const long long qs = wk.ncap;
     const int grid = g->num_sms * 8;
     cudaStream_t st = g->stream;
+    Fork fk(g);
     cudaEvent_t e = tm.begin();
     k_decide_single_small<M, UNIT><<<grid, 256, 0, st>>>(wk.queues, qs, a, qW, p);
     CKL();
@@ -379,11 +422,11 @@ static void launch_single(gala_graph_s* g, Work& wk, const DecideArgs& a, typena
     for (int b = BIN_WARP; b <= BIN_BLOCK; ++b) {
         if (maxdeg <= g->bins[b - 1]) break;
         e = tm.begin();
-        k_decide_single<M, UNIT><<<grid, 256, 0, st>>>(qview(wk.queues, qs, b), b, a, qW, p);
+        k_decide_single<M, UNIT><<<grid, 256, 0, fk.branch(b - BIN_WARP)>>>(qview(wk.queues, qs, b), b, a, qW, p);
         CKL();
         tm.end(kcs[b - BIN_WARP], e);
     }
-    launch_hub<M, UNIT>(g, wk, a, qW, p, tm);
+    launch_hub<M, UNIT>(g, wk, a, qW, p, tm, wk.hub_on ? fk.branch(3) : st);
 }
 
 template <int M, bool UNIT>
@@ -400,32 +443,35 @@ static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, typename M
     const long long qs = wk.ncap;
     const int grid = g->num_sms * 8;
     cudaStream_t st = g->stream;
+    Fork fk(g);
     cudaEvent_t e;
+    // the longest-running bins go first so they start on an idle machine
+    if (maxdeg > g->bins[BIN_WARP2]) {
+        const int smem_cap = g->hub_smem_slots;
+        e = tm.begin();
+        k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT><<<wk.gblocks_m[M], BLOCK_BT, block_smem_bytes<M>(smem_cap),
+                                                     fk.branch(0)>>>(
+            qview(wk.queues, qs, BIN_BLOCK), BIN_BLOCK, a, qW, p, smem_cap, wk.gkeys, wk.gvals, wk.glist, wk.gcap);
+        CKL();
+        tm.end(KC_DEC_BLOCK, e);
+    }
+    launch_hub<M, UNIT>(g, wk, a, qW, p, tm, wk.hub_on ? fk.branch(1) : st);
     e = tm.begin();
     k_decide_small<M, UNIT><<<grid, 256, 0, st>>>(wk.queues, qs, a, qW, p);
     CKL();
     tm.end(KC_DEC_SMALL, e);
     e = tm.begin();
-    k_decide_warp<32, 128, M, UNIT><<<grid, 32 * WarpSmem<32, 128, M>::WPB, WarpSmem<32, 128, M>::bytes, st>>>(
+    k_decide_warp<32, 128, M, UNIT><<<grid, 32 * WarpSmem<32, 128, M>::WPB, WarpSmem<32, 128, M>::bytes, fk.branch(2)>>>(
         qview(wk.queues, qs, BIN_WARP), BIN_WARP, a, qW, p);
     CKL();
     tm.end(KC_DEC_WARP, e);
     if (maxdeg > g->bins[BIN_WARP]) {
         e = tm.begin();
-        k_decide_warp<32, 512, M, UNIT><<<grid, 32 * WarpSmem<32, 512, M>::WPB, WarpSmem<32, 512, M>::bytes, st>>>(
-            qview(wk.queues, qs, BIN_WARP2), BIN_WARP2, a, qW, p);
+        k_decide_warp<32, 512, M, UNIT><<<grid, 32 * WarpSmem<32, 512, M>::WPB, WarpSmem<32, 512, M>::bytes,
+                                          fk.branch(3)>>>(qview(wk.queues, qs, BIN_WARP2), BIN_WARP2, a, qW, p);
         CKL();
         tm.end(KC_DEC_WARP2, e);
     }
-    if (maxdeg > g->bins[BIN_WARP2]) {
-        const int smem_cap = g->hub_smem_slots;
-        e = tm.begin();
-        k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT><<<wk.gblocks_m[M], BLOCK_BT, block_smem_bytes<M>(smem_cap), st>>>(
-            qview(wk.queues, qs, BIN_BLOCK), BIN_BLOCK, a, qW, p, smem_cap, wk.gkeys, wk.gvals, wk.glist, wk.gcap);
-        CKL();
-        tm.end(KC_DEC_BLOCK, e);
-    }
-    launch_hub<M, UNIT>(g, wk, a, qW, p, tm);
 }
 
 // Per level, before its iterations: per-block spill tables of the block bin
@@ -516,12 +562,12 @@ static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, typename
     launch_decide<M, UNIT>(g, wk, G, qW, p, tm, maxdeg, idbits, single);
     e = tm.begin();
     k_apply<<<grid_for(n, AP_BT, big), AP_BT, 0, st>>>(wk.ctr, wk.queues, wk.ncap, wk.nextC, wk.C, wk.Sig, wk.size,
-                                                       wk.d, G.rp, wk.stamp, wk.carry, wk.mv_v, wk.mv_old);
+                                                       wk.dp, wk.stamp, wk.carry, wk.mv_v, wk.mv_old, wk.mv_chunk);
     CKL();
     tm.end(KC_APPLY, e);
     e = tm.begin();
     const bool ck = use_ckey(g, wk, G);
-    k_dp_delta<UNIT><<<big, 256, 0, st>>>(wk.ctr, G.rp, G.col, G.w, wk.C, wk.mv_v, wk.mv_old, wk.stamp, wk.dp,
+    k_dp_delta<UNIT><<<big, 256, 0, st>>>(wk.ctr, G.rp, G.col, G.w, wk.C, wk.mv_v, wk.mv_old, wk.mv_chunk, wk.stamp, wk.dp,
                                           wk.carry, G.nnz, g->opt_delta, 1, 2, ck ? wk.ckey : nullptr,
                                           ck ? g->rev0 : nullptr);
     CKL();
@@ -891,8 +937,11 @@ static void ensure_workspace(gala_graph_s* g) {
             wk.C = dalloc<int32_t>(wk.ncap, st);
             wk.size = dalloc<int32_t>(wk.ncap, st);
             wk.stamp = dalloc<int32_t>(wk.ncap, st);
-            wk.mv_v = dalloc<int32_t>(wk.ncap, st);
-            wk.mv_old = dalloc<int32_t>(wk.ncap, st);
+            // delta-update items: one per light mover + one per DCH-entry chunk of a heavy one
+            const size_t icap = (size_t)wk.ncap + (size_t)(g->nnz0 / DCH) + 1;
+            wk.mv_v = dalloc<int32_t>(icap, st);
+            wk.mv_old = dalloc<int32_t>(icap, st);
+            wk.mv_chunk = dalloc<int32_t>(icap, st);
             wk.nextC = dalloc<int32_t>(wk.ncap, st);
             wk.queues = dalloc<QRec>((size_t)wk.ncap * (NBINS / 2), st);
             if (g->rev0) wk.ckey = dalloc<int32_t>(g->nnz0, st);
@@ -1861,6 +1910,11 @@ void gala_graph_free(gala_graph g) {
         cudaStreamSynchronize(st);
         if (g->own_stream) cudaStreamDestroy(st);
     }
+    for (int i = 0; i < 4; ++i) {
+        if (g->side[i]) cudaStreamDestroy(g->side[i]);
+        if (g->ev_join[i]) cudaEventDestroy(g->ev_join[i]);
+    }
+    if (g->ev_fork) cudaEventDestroy(g->ev_fork);
     if (g->cache) {
         if (g->cache->pool) cudaMemPoolDestroy(g->cache->pool);
         delete g->cache;
@@ -1884,6 +1938,7 @@ gala_status gala_set_option(gala_graph g, const char* key, int64_t value) {
     else if (k == "force_wide") g->opt_force_wide = value != 0;
     else if (k == "singleton") g->opt_singleton = value != 0;
     else if (k == "ckey") g->opt_ckey = value != 0;
+    else if (k == "concurrent") g->opt_concurrent = value != 0;
     else if (k == "verbose") g->opt_verbose = (int)value;
     else if (k == "cuda_graph") g->opt_cuda_graph = value != 0;
     else if (k == "log_cap") { if (value < 2 || value > (1 << 20)) return set_err(GALA_E_INVALID, "log_cap in [2, 2^20]"); g->opt_log_cap = (int)value; }

@@ -204,25 +204,31 @@ __global__ void __launch_bounds__(PB_BT) k_prune_bin(int vlo, int n, const int64
 // one global atomic per block and tile.
 // ---------------------------------------------------------------------------
 #define AP_BT 256
+// Delta-update work items: a mover with at most DCH entries is one item, a
+// longer one is split into ceil(deg/DCH) chunk items so a hub's row is spread
+// over many warps instead of serialising one (its d' is then summed by
+// atomics onto a zero written here).  Item capacity: n + nnz/DCH.
+#define DCH 256
 __global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr, QRec* queues,
                                                  long long qstride, const int32_t* __restrict__ nextC,
                                                  int32_t* __restrict__ C, int64_t* __restrict__ Sig,
-                                                 int32_t* __restrict__ size, const int64_t* __restrict__ d,
-                                                 const int64_t* __restrict__ rp, int32_t* __restrict__ stamp,
-                                                 const Carry* __restrict__ carry, int32_t* __restrict__ mv_v,
-                                                 int32_t* __restrict__ mv_old) {
-    __shared__ unsigned s_cnt;
-    __shared__ ull s_base;
+                                                 int32_t* __restrict__ size, int64_t* __restrict__ dp,
+                                                 int32_t* __restrict__ stamp, const Carry* __restrict__ carry,
+                                                 int32_t* __restrict__ it_v, int32_t* __restrict__ it_old,
+                                                 int32_t* __restrict__ it_chunk) {
+    __shared__ unsigned s_cnt, s_items;
+    __shared__ ull s_ibase;
     long long cnt[NBINS];
     long long total = 0;
 #pragma unroll
     for (int b = 0; b < NBINS; ++b) { cnt[b] = (long long)ctr->bin_count[b]; total += cnt[b]; }
     const int iter_id = carry->iter;
+    const int lane = lane_id();
     ull my_deg = 0;
     for (long long t0 = (long long)blockIdx.x * AP_BT; t0 < total; t0 += (long long)gridDim.x * AP_BT) {
         long long i = t0 + threadIdx.x;
         bool mover = false;
-        int v = 0, oc = 0;
+        int v = 0, oc = 0, deg = 0;
         if (i < total) {
             int b = 0;
             long long r = i;
@@ -236,6 +242,7 @@ __global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr,
             if (nc != oc) {
                 mover = true;
                 long long dv = q.dv;
+                deg = q.deg;
                 C[v] = nc;
                 stamp[v] = iter_id;
                 atomicAdd(reinterpret_cast<ull*>(&Sig[oc]), (ull)(-dv));
@@ -243,21 +250,38 @@ __global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr,
                 atomicSub(&size[oc], 1);
                 atomicAdd(&size[nc], 1);
                 my_deg += (ull)q.deg;
+                if (deg > DCH) dp[v] = 0;   // chunk items add onto it
             }
         }
-        if (threadIdx.x == 0) s_cnt = 0;
-        __syncthreads();
-        unsigned m = __ballot_sync(FULLMASK, mover);
-        unsigned off = 0;
-        if (m && lane_id() == __ffs(m) - 1) off = atomicAdd(&s_cnt, (unsigned)__popc(m));
-        off = __shfl_sync(FULLMASK, off, m ? __ffs(m) - 1 : 0) + __popc(m & lanemask_lt());
-        __syncthreads();
-        if (threadIdx.x == 0) s_base = s_cnt ? atomicAdd(&ctr->n_moved, (ull)s_cnt) : 0;
-        __syncthreads();
-        if (mover) {
-            mv_v[s_base + off] = v;
-            mv_old[s_base + off] = oc;
+        // items of this thread (0, 1, or the chunk count of a heavy mover)
+        const unsigned nit = !mover ? 0u : (deg > DCH ? (unsigned)((deg + DCH - 1) / DCH) : 1u);
+        unsigned incl = nit;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            unsigned y = __shfl_up_sync(FULLMASK, incl, o);
+            if (lane >= o) incl += y;
         }
+        if (threadIdx.x == 0) { s_cnt = 0; s_items = 0; }
+        __syncthreads();
+        const unsigned m = __ballot_sync(FULLMASK, mover);
+        if (m && lane == 0) atomicAdd(&s_cnt, (unsigned)__popc(m));
+        unsigned ioff = 0;
+        const unsigned wtot = __shfl_sync(FULLMASK, incl, 31);
+        if (lane == 31 && wtot) ioff = atomicAdd(&s_items, wtot);
+        ioff = __shfl_sync(FULLMASK, ioff, 31) + incl - nit;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            if (s_cnt) atomicAdd(&ctr->n_moved, (ull)s_cnt);
+            s_ibase = s_items ? atomicAdd(&ctr->n_items, (ull)s_items) : 0;
+        }
+        __syncthreads();
+        for (unsigned j = 0; j < nit; ++j) {
+            const ull at = s_ibase + ioff + j;
+            it_v[at] = v;
+            it_old[at] = oc;
+            it_chunk[at] = (int32_t)j;
+        }
+        __syncthreads();   // s_ibase reused by the next tile
     }
     ull md = block_sum_ull<AP_BT>(my_deg);
     if (threadIdx.x == 0 && md) atomicAdd(&ctr->moved_deg, md);
@@ -280,8 +304,9 @@ __device__ __forceinline__ bool use_delta(const IterCounters* ctr, long long nnz
 template <bool UNIT>
 __global__ void __launch_bounds__(256) k_dp_delta(IterCounters* __restrict__ ctr, const int64_t* __restrict__ rp,
                                                   const int32_t* __restrict__ col, const int64_t* __restrict__ w,
-                                                  const int32_t* __restrict__ C, const int32_t* __restrict__ mv_v,
-                                                  const int32_t* __restrict__ mv_old,
+                                                  const int32_t* __restrict__ C, const int32_t* __restrict__ it_v,
+                                                  const int32_t* __restrict__ it_old,
+                                                  const int32_t* __restrict__ it_chunk,
                                                   const int32_t* __restrict__ stamp, int64_t* __restrict__ dp,
                                                   const Carry* __restrict__ carry, long long nnz, int mode,
                                                   long long fnum, long long fden, int32_t* __restrict__ ckey,
@@ -291,29 +316,48 @@ __global__ void __launch_bounds__(256) k_dp_delta(IterCounters* __restrict__ ctr
         ctr->delta_used = 1;
         if (ckey) const_cast<Carry*>(carry)->ckey_valid = 0;   // per-entry communities now stale
     }
+    (void)rev;
     const int iter_id = carry->iter;
     const int lane = lane_id();
-    const long long m = (long long)ctr->n_moved;
+    const long long m = (long long)ctr->n_items;
     long long wid = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
     for (long long i = wid; i < m; i += nw) {
-        int u = mv_v[i], oc = mv_old[i];
-        int nc = C[u];
-        int64_t b = rp[u], e = rp[u + 1];
+        const int u = it_v[i], oc = it_old[i], ch = it_chunk[i];
+        const int nc = C[u];
+        const int64_t rb = rp[u], re = rp[u + 1];
+        const bool heavy = re - rb > DCH;
+        const int64_t b = rb + (int64_t)ch * DCH, e = heavy ? min(b + DCH, re) : re;
         long long acc = 0;
-        for (int64_t j = b + lane; j < e; j += 32) {
-            int x = col[j];
-            if (x == u) continue;
-            long long wt = UNIT ? 1 : w[j];
-            int cx = C[x];
-            if (cx == nc) acc += wt;
-            if (stamp[x] != iter_id) {
-                if (cx == oc) atomicAdd(reinterpret_cast<ull*>(&dp[x]), (ull)(-wt));
-                else if (cx == nc) atomicAdd(reinterpret_cast<ull*>(&dp[x]), (ull)wt);
+        for (int64_t j0 = b; j0 < e; j0 += 128) {   // 4 entries per lane in flight
+            int x[4], cx[4], sx[4];
+            long long wt[4];
+#pragma unroll
+            for (int t = 0; t < 4; ++t) {
+                const int64_t j = j0 + lane + 32 * t;
+                x[t] = j < e ? col[j] : u;
+                wt[t] = (UNIT || j >= e) ? 1 : w[j];
+            }
+#pragma unroll
+            for (int t = 0; t < 4; ++t) {
+                cx[t] = x[t] != u ? C[x[t]] : -1;
+                sx[t] = x[t] != u ? stamp[x[t]] : iter_id;
+            }
+#pragma unroll
+            for (int t = 0; t < 4; ++t) {
+                if (x[t] == u) continue;
+                if (cx[t] == nc) acc += wt[t];
+                if (sx[t] != iter_id) {
+                    if (cx[t] == oc) atomicAdd(reinterpret_cast<ull*>(&dp[x[t]]), (ull)(-wt[t]));
+                    else if (cx[t] == nc) atomicAdd(reinterpret_cast<ull*>(&dp[x[t]]), (ull)wt[t]);
+                }
             }
         }
         acc = warp_sum_ll(acc);
-        if (lane == 0) dp[u] = acc;
+        if (lane == 0) {
+            if (heavy) { if (acc) atomicAdd(reinterpret_cast<ull*>(&dp[u]), (ull)acc); }
+            else dp[u] = acc;
+        }
     }
 }
 

@@ -101,6 +101,8 @@ def test_synthetic_parity(name, prune):
     dict(singleton=0),
     dict(ckey=1),
     dict(delta_update=1, ckey=1),
+    dict(concurrent=1),
+    dict(hub(64), concurrent=1, delta_update=1),
 ])
 def test_dispatch_independence(opts):
     """P7: thresholds / table sizes / integer width / update strategy never change a label."""
