@@ -126,6 +126,25 @@ __device__ __forceinline__ unsigned hash_slot2(int c, unsigned mask) {
     return (((unsigned)c ^ 0x5bd1e995u) * 0x9E3779B1u >> 7) & mask;
 }
 
+// 16-byte volatile load of four consecutive table keys (generic address: shared or global)
+__device__ __forceinline__ int4 ld_volatile_i4(const int* p) {
+    int4 r;
+    asm volatile("ld.volatile.v4.s32 {%0,%1,%2,%3}, [%4];" : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+    return r;
+}
+__device__ __forceinline__ int4 lds_volatile_i4(const int* p) {   // p points into shared memory
+    int4 r;
+    const unsigned a = (unsigned)__cvta_generic_to_shared(p);
+    asm volatile("ld.volatile.shared.v4.s32 {%0,%1,%2,%3}, [%4];" : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "r"(a));
+    return r;
+}
+template <bool SH>
+__device__ __forceinline__ int4 ld_bucket(const int* p) { return SH ? lds_volatile_i4(p) : ld_volatile_i4(p); }
+// bit i set iff lane i of the 4-key bucket equals x
+__device__ __forceinline__ unsigned match4(const int4& k, int x) {
+    return (unsigned)(k.x == x) | ((unsigned)(k.y == x) << 1) | ((unsigned)(k.z == x) << 2) | ((unsigned)(k.w == x) << 3);
+}
+
 __device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
 __device__ __forceinline__ unsigned lanemask_lt() {
     unsigned m;

@@ -731,19 +731,20 @@ static size_t agg_block_smem(int scap) { return (size_t)scap * (sizeof(V) + size
 
 // warp / block aggregation launches with V = table value type (32-bit iff W < 2^32)
 template <typename V>
-static void agg_launch_small(gala_graph_s* g, const AggArgs& a, bool unit, int scap, long long k) {
+static void agg_launch_small(gala_graph_s* g, const AggArgs& a, bool unit, int scap, long long k, const int32_t* wl,
+                             const int* nwl, const int32_t* bl, const int* nbl) {
     cudaStream_t st = g->stream;
     const int big = g->num_sms * 8;
-    if (unit) k_agg_warp<true, V><<<big, 256, 0, st>>>(a);
-    else k_agg_warp<false, V><<<big, 256, 0, st>>>(a);
+    if (unit) k_agg_warp<true, V><<<big, 256, 0, st>>>(a, wl, nwl);
+    else k_agg_warp<false, V><<<big, 256, 0, st>>>(a, wl, nwl);
     CKL();
     if (scap > AGG_WSLOTS) {
         const size_t sm = agg_block_smem<V>(scap);
         CK(cudaFuncSetAttribute(k_agg_block<AGG_BLOCK_BT, true, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
         CK(cudaFuncSetAttribute(k_agg_block<AGG_BLOCK_BT, false, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
         const int gb = (int)std::min<long long>(k, (long long)g->num_sms * 4);
-        if (unit) k_agg_block<AGG_BLOCK_BT, true, V><<<gb, AGG_BLOCK_BT, sm, st>>>(a, scap);
-        else k_agg_block<AGG_BLOCK_BT, false, V><<<gb, AGG_BLOCK_BT, sm, st>>>(a, scap);
+        if (unit) k_agg_block<AGG_BLOCK_BT, true, V><<<gb, AGG_BLOCK_BT, sm, st>>>(a, scap, bl, nbl);
+        else k_agg_block<AGG_BLOCK_BT, false, V><<<gb, AGG_BLOCK_BT, sm, st>>>(a, scap, bl, nbl);
         CKL();
     }
 }
@@ -766,13 +767,15 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
     ull* dev_max = dalloc<ull>(1, st);
     int32_t* bigc = dalloc<int32_t>(k, st);
     long long* bigcap = dalloc<long long>(k + 1, st);
-    int* nbig_dev = dalloc<int>(1, st);
+    int32_t* wlist = dalloc<int32_t>(k, st);
+    int32_t* blist = dalloc<int32_t>(k, st);
+    int* nbig_dev = dalloc<int>(3, st);   // big, warp, block list lengths
     CK(cudaMemsetAsync(cnt, 0, sizeof(long long) * (k + 1), st));
     CK(cudaMemsetAsync(ent, 0, sizeof(long long) * (k + 1), st));
     CK(cudaMemsetAsync(dn, 0, sizeof(long long) * (k + 1), st));
     CK(cudaMemsetAsync(snew, 0, sizeof(int64_t) * k, st));
     CK(cudaMemsetAsync(dev_max, 0, sizeof(ull), st));
-    CK(cudaMemsetAsync(nbig_dev, 0, sizeof(int), st));
+    CK(cudaMemsetAsync(nbig_dev, 0, sizeof(int) * 3, st));
     k_comm_stats<<<grid_for(nrows, 256, big), 256, 0, st>>>((int)nrows, cur.rp, newid, ent);
     CKL();
     scan_excl(ent, eoff, k, st);
@@ -793,13 +796,14 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
     // shared-memory capacity of the block path: up to 8192 slots (14 B each)
     int scap = 512;
     while (scap < 8192 && scap < 2 * k) scap <<= 1;
-    k_agg_bigflag<<<grid_for(k, 256, big), 256, 0, st>>>(k, ent, scap, bigc, bigcap, nbig_dev);
+    k_agg_classify<<<grid_for(k, 256, big), 256, 0, st>>>(k, ent, scap, dn, wlist, nbig_dev + 1, blist, nbig_dev + 2,
+                                                         bigc, bigcap, nbig_dev);
     CKL();
     AggArgs a;
     a.k = k; a.ent = ent; a.eoff = eoff; a.tkey = tkey; a.tval = tval; a.dn = dn; a.snew = snew;
     const bool v32 = g->W < ((int64_t)1 << 32);   // every aggregated weight is <= W
-    if (v32) agg_launch_small<unsigned>(g, a, unit, scap, k);
-    else agg_launch_small<ull>(g, a, unit, scap, k);
+    if (v32) agg_launch_small<unsigned>(g, a, unit, scap, k, wlist, nbig_dev + 1, blist, nbig_dev + 2);
+    else agg_launch_small<ull>(g, a, unit, scap, k, wlist, nbig_dev + 1, blist, nbig_dev + 2);
     vt.lap("agg: warp+block");
     int nbig = 0;
     CK(cudaMemcpyAsync(&nbig, nbig_dev, sizeof(int), cudaMemcpyDeviceToHost, st));
@@ -854,7 +858,7 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
                               (double)nxt.nnz * 24;
     dfree(cnt, st); dfree(ent, st); dfree(eoff, st); dfree(dn, st);
     dfree(tkey, st); dfree(tval, st); dfree(dev_max, st); dfree(bigc, st);
-    dfree(bigcap, st); dfree(nbig_dev, st);
+    dfree(bigcap, st); dfree(nbig_dev, st); dfree(wlist, st); dfree(blist, st);
 }
 
 // ------------------------------------------------------------------ phase 2 (a9)

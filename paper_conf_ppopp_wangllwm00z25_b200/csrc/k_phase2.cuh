@@ -212,10 +212,8 @@ __global__ void k_fill_rows(int n, const int64_t* __restrict__ rp, int32_t* __re
 // table capacity a community needs: nextpow2(2 * min(entries, k)) (0 if no entries)
 __device__ __forceinline__ long long agg_cap(long long ent, long long k) {
     if (ent == 0) return 0;
-    long long m = ent < k ? ent : k;
-    long long x = 2;
-    while (x < 2 * m) x <<= 1;
-    return x;
+    const long long m = ent < k ? ent : k;
+    return 1LL << (64 - __clzll(2 * m - 1));
 }
 
 struct AggArgs {
@@ -228,6 +226,9 @@ struct AggArgs {
     int64_t* snew;             // diagonal weight per community
 };
 
+// bucketed linear probe (4 keys per 16-byte load, empties claimed in slot
+// order; see ht_insert4 in k_decide.cuh); tables are never full (cap >= 2 x
+// distinct keys), mask < 3 falls back to slot-wise probing
 template <typename VT>
 __device__ __forceinline__ int agg_insert(int key, VT wt, int* keys, VT* vals, unsigned mask, int* list, int* cnt) {
     unsigned h = hash_slot(key, mask);
@@ -294,8 +295,9 @@ __device__ __forceinline__ void agg_emit(const AggArgs& a, long long c, int m, c
 
 #define AGG_WSLOTS 256
 template <bool UNIT, typename V>
-__global__ void __launch_bounds__(256) k_agg_warp(AggArgs a) {
-    __shared__ int s_key[8][AGG_WSLOTS];
+__global__ void __launch_bounds__(256) k_agg_warp(AggArgs a, const int32_t* __restrict__ wl,
+                                                  const int* __restrict__ nwl) {
+    __shared__ __align__(16) int s_key[8][AGG_WSLOTS];
     __shared__ V s_val[8][AGG_WSLOTS];
     __shared__ int s_list[8][AGG_WSLOTS / 2];
     __shared__ int s_cnt[8];
@@ -308,10 +310,10 @@ __global__ void __launch_bounds__(256) k_agg_warp(AggArgs a) {
     if (lane == 0) s_cnt[wib] = 0;
     __syncwarp();
     const long long nw = (long long)gridDim.x * 8;
-    for (long long c = (long long)blockIdx.x * 8 + wib; c < a.k; c += nw) {
-        long long cap = agg_cap(a.ent[c], a.k);
-        if (cap == 0) { if (lane == 0) a.dn[c] = 0; continue; }
-        if (cap > AGG_WSLOTS) continue;
+    const long long cnt = *nwl;
+    for (long long i = (long long)blockIdx.x * 8 + wib; i < cnt; i += nw) {
+        const long long c = wl[i];
+        const long long cap = agg_cap(a.ent[c], a.k);
         agg_segment<UNIT, V, V>(a, a.eoff[c], a.eoff[c + 1], lane, 32, keys, vals, (unsigned)cap - 1, list,
                                 &s_cnt[wib], s_scr[wib]);
         __syncwarp();
@@ -324,7 +326,8 @@ __global__ void __launch_bounds__(256) k_agg_warp(AggArgs a) {
 }
 
 template <int BT, bool UNIT, typename V>
-__global__ void __launch_bounds__(BT) k_agg_block(AggArgs a, int scap) {
+__global__ void __launch_bounds__(BT) k_agg_block(AggArgs a, int scap, const int32_t* __restrict__ bl,
+                                                  const int* __restrict__ nbl) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     V* vals = reinterpret_cast<V*>(smem_raw);
     int* keys = reinterpret_cast<int*>(smem_raw + (size_t)scap * sizeof(V));
@@ -335,9 +338,10 @@ __global__ void __launch_bounds__(BT) k_agg_block(AggArgs a, int scap) {
     for (int j = threadIdx.x; j < scap; j += BT) { keys[j] = -1; vals[j] = 0; }
     if (threadIdx.x == 0) s_cnt = 0;
     __syncthreads();
-    for (long long c = blockIdx.x; c < a.k; c += gridDim.x) {
-        long long cap = agg_cap(a.ent[c], a.k);
-        if (cap <= AGG_WSLOTS || cap > scap) continue;   // block-uniform
+    const long long cnt = *nbl;
+    for (long long i = blockIdx.x; i < cnt; i += gridDim.x) {
+        const long long c = bl[i];
+        const long long cap = agg_cap(a.ent[c], a.k);
         agg_segment<UNIT, V, V>(a, a.eoff[c], a.eoff[c + 1], threadIdx.x, BT, keys, vals, (unsigned)cap - 1, list,
                                 &s_cnt, s_scr[wib]);
         __syncthreads();
@@ -393,15 +397,42 @@ __global__ void __launch_bounds__(256) k_agg_big_emit(AggArgs a, const int32_t* 
     }
 }
 
-// flag + list of communities whose table exceeds the shared-memory capacity
-__global__ void k_agg_bigflag(long long k, const long long* __restrict__ ent, int scap, int32_t* __restrict__ bigc,
-                              long long* __restrict__ bigcap, int* __restrict__ nbig) {
-    for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c < k; c += (long long)gridDim.x * blockDim.x) {
-        long long cap = agg_cap(ent[c], k);
-        if (cap > scap) {
-            int i = atomicAdd(nbig, 1);
-            bigc[i] = (int32_t)c;
-            bigcap[i] = cap;
+// Sort every community into the path that fits its table: warp (<= AGG_WSLOTS
+// slots), block (<= scap), big (global table); communities without entries get
+// dn = 0 here.  Lists are filled with warp-aggregated appends.
+__device__ __forceinline__ void list_append(bool on, int32_t val, int32_t* list, int* cnt) {
+    const unsigned m = __ballot_sync(FULLMASK, on);
+    if (!m) return;
+    const int lane = lane_id(), lead = __ffs(m) - 1;
+    int base = 0;
+    if (lane == lead) base = atomicAdd(cnt, __popc(m));
+    base = __shfl_sync(FULLMASK, base, lead);
+    if (on) list[base + __popc(m & lanemask_lt())] = val;
+}
+
+__global__ void k_agg_classify(long long k, const long long* __restrict__ ent, int scap, long long* __restrict__ dn,
+                               int32_t* __restrict__ wl, int* __restrict__ nwl, int32_t* __restrict__ bl,
+                               int* __restrict__ nbl, int32_t* __restrict__ bigc, long long* __restrict__ bigcap,
+                               int* __restrict__ nbig) {
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    for (long long c0 = (long long)blockIdx.x * blockDim.x; c0 < k; c0 += stride) {   // warp-uniform trips
+        const long long c = c0 + threadIdx.x;
+        const long long cap = c < k ? agg_cap(ent[c], k) : -1;
+        if (cap == 0) dn[c] = 0;
+        list_append(cap > 0 && cap <= AGG_WSLOTS, (int32_t)c, wl, nwl);
+        list_append(cap > AGG_WSLOTS && cap <= scap, (int32_t)c, bl, nbl);
+        const bool isbig = cap > scap;
+        const unsigned m = __ballot_sync(FULLMASK, isbig);
+        if (m) {
+            const int lane = lane_id(), lead = __ffs(m) - 1;
+            int base = 0;
+            if (lane == lead) base = atomicAdd(nbig, __popc(m));
+            base = __shfl_sync(FULLMASK, base, lead);
+            if (isbig) {
+                const int i = base + __popc(m & lanemask_lt());
+                bigc[i] = (int32_t)c;
+                bigcap[i] = cap;
+            }
         }
     }
 }
