@@ -4,7 +4,7 @@ NVCC      ?= /usr/local/cuda/bin/nvcc
 HOSTCC    := $(shell test -x /usr/bin/gcc && echo /usr/bin/gcc || echo gcc)
 PKG       := paper_conf_ppopp_wangllwm00z25_b200
 CUDA_ARCH := -gencode arch=compute_100a,code=sm_100a
-NVFLAGS   := -O3 -std=c++17 $(CUDA_ARCH) -lineinfo -Xcompiler -fPIC,-O3,-Wall -Iinclude \
+NVFLAGS   := $(EXTRA) -O3 -std=c++17 $(CUDA_ARCH) -lineinfo -Xcompiler -fPIC,-O3,-Wall -Iinclude \
              --expt-relaxed-constexpr -Xptxas -warn-spills
 CSRC      := $(wildcard $(PKG)/csrc/*.cu) $(wildcard $(PKG)/csrc/*.cuh) $(wildcard $(PKG)/csrc/*.h) include/gala.h
 

@@ -151,7 +151,7 @@ void gala_graph_free(gala_graph g);
  *   "singleton"      0/1   first iteration of a level via the singleton fast path (default 1)
  *   "ckey"           0/1   keep a per-entry copy of C[col] on level 0, maintained by the delta
  *                          update (default 0; trades nnz*4 bytes for one gather per entry)
- *   "hub_smem_slots" power of two in [64, 16384], shared-memory slots of the block hash table
+ *   "hub_smem_slots" power of two in [64, 16384], shared-memory slots of the block hash table (default 8192)
  *   "cuda_graph"     0/1   run each level's iterations as a conditional CUDA graph (default 1)
  *   "concurrent"     0/1   run the degree bins' decide kernels as parallel branches on side
  *                          streams (default 0: measured slower on B200 -- the bins contend for L2 and smem; off whenever "timing" is on)

@@ -108,7 +108,7 @@ struct gala_graph_s {
     int32_t* rev0 = nullptr;       // level-0 reverse-entry index (enables the per-entry community array)
     int opt_ckey = 0;
     int bins[NBINS - 1] = {4, 8, 16, 32, 128, 512, 16384};
-    int hub_smem_slots = 4096;
+    int hub_smem_slots = 8192;
     // results
     bool has_result = false;
     int64_t k = 0, p = 1, q = 1;
@@ -385,7 +385,7 @@ static void set_warp_smem() {
                             (int)WarpSmem<GW, MAXDEG, M>::bytes));
 }
 template <int M>
-static size_t block_smem_bytes(int cap) { return (size_t)cap * (sizeof(typename ModeT<M>::VT) + 2 * sizeof(int)); }
+static size_t block_smem_bytes(int cap) { return (size_t)cap * (sizeof(typename ModeT<M>::VT) + sizeof(int)); }
 
 // multi-block hub path (bin BIN_HUB), only on levels that have such rows
 template <int M, bool UNIT>

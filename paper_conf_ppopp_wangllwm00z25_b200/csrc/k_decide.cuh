@@ -201,16 +201,34 @@ __device__ __forceinline__ unsigned decide_sub_bin(QView queue, int bin, const D
 
 // bins 0-3 (rows <= 4, 8, 16, 32) in one launch: the block's warps sweep each
 // bin with its own group size, so empty bins cost nothing
+#ifndef GALA_SMALL_MINB
+#define GALA_SMALL_MINB 4   // <= 64 registers: 32 warps per SM (measured -30% vs 72-80 regs)
+#endif
+#ifndef GALA_WARP_MINB
+#define GALA_WARP_MINB 4   // <= 64 registers (an explicit min of 1 lets ptxas take 80)
+#endif
+#ifndef GALA_W512_MINB
+#define GALA_W512_MINB 4   // 128 regs, 4 blocks of 128 threads
+#endif
+#ifndef GALA_SINGLE_MINB
+#define GALA_SINGLE_MINB 1
+#endif
+#ifndef GALA_U16
+#define GALA_U16 4
+#endif
+#ifndef GALA_U32
+#define GALA_U32 4
+#endif
 template <int M, bool UNIT>
-__global__ void __launch_bounds__(256) k_decide_small(QRec* queues, long long qstride,
+__global__ void __launch_bounds__(256, GALA_SMALL_MINB) k_decide_small(QRec* queues, long long qstride,
                                                       DecideArgs a, typename ModeT<M>::ST qW,
                                                       typename ModeT<M>::ST p) {
     __shared__ typename ModeT<M>::VT s_acc[8][32];
     if (a.ckey && !*a.ckey_valid) a.ckey = nullptr;
     unsigned k0 = decide_sub_bin<4, 4, M, UNIT>(qview(queues, qstride, BIN_S4), BIN_S4, a, qW, p, s_acc);
     unsigned k1 = decide_sub_bin<8, 4, M, UNIT>(qview(queues, qstride, BIN_S8), BIN_S8, a, qW, p, s_acc);
-    unsigned k2 = decide_sub_bin<16, 2, M, UNIT>(qview(queues, qstride, BIN_S16), BIN_S16, a, qW, p, s_acc);
-    unsigned k3 = decide_sub_bin<32, 2, M, UNIT>(qview(queues, qstride, BIN_S32), BIN_S32, a, qW, p, s_acc);
+    unsigned k2 = decide_sub_bin<16, GALA_U16, M, UNIT>(qview(queues, qstride, BIN_S16), BIN_S16, a, qW, p, s_acc);
+    unsigned k3 = decide_sub_bin<32, GALA_U32, M, UNIT>(qview(queues, qstride, BIN_S32), BIN_S32, a, qW, p, s_acc);
     const unsigned kk[4] = {k0, k1, k2, k3};
 #pragma unroll
     for (int b = 0; b < 4; ++b) {
@@ -299,7 +317,7 @@ struct WarpSmem {
 
 // GW lanes (16 or 32) per vertex, deg <= MAXDEG = 4 * GW; 32/GW vertices per warp
 template <int GW, int MAXDEG, int M, bool UNIT>
-__global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB) k_decide_warp(QView queue,
+__global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB, MAXDEG <= 128 ? GALA_WARP_MINB : GALA_W512_MINB) k_decide_warp(QView queue,
                                                                                   int bin, DecideArgs a,
                                                                                   typename ModeT<M>::ST qW,
                                                                                   typename ModeT<M>::ST p) {
@@ -446,12 +464,13 @@ __global__ void __launch_bounds__(BT) k_decide_block(QView queue, int bin, Decid
     typedef typename ModeT<M>::ST ST;
     typedef typename ModeT<M>::VT VT;
     typedef Arg<ST, ModeT<M>::PK> A;
+    // H0 = keys + values only (no distinct list: the table prefix a vertex used is
+    // scanned instead, <= 4 slots per row entry), so more blocks fit per SM
     extern __shared__ __align__(16) unsigned char smem_raw[];
     VT* vals = reinterpret_cast<VT*>(smem_raw);
     int* keys = reinterpret_cast<int*>(smem_raw + (size_t)smem_cap * sizeof(VT));
-    int* list = keys + smem_cap;
     __shared__ long long s_item;
-    __shared__ int s_cnt, s_gcnt;
+    __shared__ int s_gcnt;
     __shared__ A r_a[BT / 32];
     __shared__ long long r_own[BT / 32];
     __shared__ VT s_scr[BT / 32][32];
@@ -459,9 +478,8 @@ __global__ void __launch_bounds__(BT) k_decide_block(QView queue, int bin, Decid
     int* gkeys = gkeys_all + (long long)blockIdx.x * gcap;
     ull* gvals = gvals_all + (long long)blockIdx.x * gcap;
     int* glist = glist_all + (long long)blockIdx.x * gcap;
-    const unsigned smask = (unsigned)smem_cap - 1;
     for (int j = threadIdx.x; j < smem_cap; j += BT) { keys[j] = -1; vals[j] = 0; }
-    if (threadIdx.x == 0) { s_cnt = 0; s_gcnt = 0; }
+    if (threadIdx.x == 0) s_gcnt = 0;
     const long long count = (long long)a.ctr->bin_count[bin];
     unsigned my_k = 0;
     for (;;) {
@@ -473,11 +491,15 @@ __global__ void __launch_bounds__(BT) k_decide_block(QView queue, int bin, Decid
         const int v = q.v, deg = q.deg, cv = q.cv;
         const int64_t beg = q.beg;
         long long own = 0;   // the own community only feeds d'(v): summed in registers, never inserted
-        int win = (smem_cap >= 2 * deg) ? smem_cap : HWIN;    // fits at load <= 1/2: never spills
-        // spill table: nextpow2(2 deg) slots, at least 64, at most the per-block capacity
-        long long gc = deg > 32 ? (1LL << (64 - __clzll(2LL * deg - 1))) : 64;
+        // H0 prefix used by this vertex: nextpow2(2 deg) slots (load <= 1/2, never spills)
+        // when that fits, else the whole arena probed over a window of HWIN slots
+        const int need = deg > 32 ? (int)(1u << (32 - __clz(2 * deg - 1))) : 64;
+        const int tcap = need <= smem_cap ? need : smem_cap;
+        const int win = need <= smem_cap ? tcap : HWIN;
+        const unsigned smask = (unsigned)tcap - 1;
+        long long gc = deg > 32 ? (1LL << (64 - __clzll(2LL * deg - 1))) : 64;   // H1 slots
         if (gc > gcap) gc = gcap;
-        unsigned gmask = (unsigned)gc - 1;
+        const unsigned gmask = (unsigned)gc - 1;
         for (int r0 = 0; r0 < deg; r0 += BT * E) {          // block-uniform rounds
             int uu[E];
             VT ww[E];
@@ -502,47 +524,43 @@ __global__ void __launch_bounds__(BT) k_decide_block(QView queue, int bin, Decid
             for (int k = 0; k < E; ++k) {
                 const unsigned peers = __match_any_sync(FULLMASK, cc[k] >= 0 ? cc[k] : -1 - lane);
                 const VT sum = UNIT ? (VT)__popc(peers) : group_sum(peers, cc[k] >= 0 ? ww[k] : (VT)0, s_scr[wib]);
-                bool fresh = false, gfresh = false;
-                int slot = -1, gslot = -1;
+                bool gfresh = false;
+                int gslot = -1;
                 if (cc[k] >= 0 && lane == __ffs(peers) - 1) {
-                    slot = ht_insert4<VT, true>(cc[k], sum, keys, vals, smask, hash_slot(cc[k], smask), win, &fresh);
+                    bool fresh;
+                    const int slot = ht_insert4<VT, true>(cc[k], sum, keys, vals, smask, hash_slot(cc[k], smask), win,
+                                                          &fresh);
                     if (slot < 0)
-                        gslot = ht_insert4<ull, false>(cc[k], (ull)sum, gkeys, gvals, gmask, hash_slot2(cc[k], gmask), (int)gc,
-                                               &gfresh);
+                        gslot = ht_insert4<ull, false>(cc[k], (ull)sum, gkeys, gvals, gmask, hash_slot2(cc[k], gmask),
+                                                       (int)gc, &gfresh);
                 }
-                append_fresh<int>(fresh, slot, FULLMASK, &s_cnt, list);
                 if (__any_sync(FULLMASK, gfresh)) append_fresh<int>(gfresh, gslot, FULLMASK, &s_gcnt, glist);
             }
         }
         __syncthreads();
-        const int m = s_cnt, gm = s_gcnt;
+        const int gm = s_gcnt;
         const long long dv = q.dv;
         A best;
         best.init(a.idbits, a.idmask);
-        my_k += (threadIdx.x == 0) ? (unsigned)(m + gm) : 0u;
-        for (int t0 = threadIdx.x; t0 < m; t0 += BT * E) {
-            int cs[E];
-            long long ws[E];
+        my_k += (threadIdx.x == 0) ? (unsigned)gm : 0u;
+        // evaluate and clear the used H0 prefix, four slots (one 16-byte key load) per thread
+        for (int t0 = threadIdx.x * 4; t0 < tcap; t0 += BT * 4) {
+            const int4 k4 = *reinterpret_cast<const int4*>(keys + t0);
+            const int cs[4] = {k4.x, k4.y, k4.z, k4.w};
+            if ((k4.x & k4.y & k4.z & k4.w) == -1) continue;   // all four empty
+            long long ws[4], sg[4];
 #pragma unroll
-            for (int k = 0; k < E; ++k) {
-                int t = t0 + k * BT;
-                cs[k] = -1;
-                if (t < m) {
-                    int slot = list[t];
-                    cs[k] = keys[slot];
-                    ws[k] = (long long)vals[slot];
-                    keys[slot] = -1;
-                    vals[slot] = 0;
-                }
+            for (int k = 0; k < 4; ++k) {
+                ws[k] = cs[k] >= 0 ? (long long)vals[t0 + k] : 0;
+                sg[k] = cs[k] >= 0 ? a.Sig[cs[k]] : 0;
             }
-            long long sg[E];
+            *reinterpret_cast<int4*>(keys + t0) = make_int4(-1, -1, -1, -1);
 #pragma unroll
-            for (int k = 0; k < E; ++k) sg[k] = (cs[k] >= 0 && cs[k] != cv) ? a.Sig[cs[k]] : 0;
-#pragma unroll
-            for (int k = 0; k < E; ++k) {
+            for (int k = 0; k < 4; ++k) {
                 if (cs[k] < 0) continue;
-                if (cs[k] == cv) own = ws[k];
-                else best.offer(gain<ST>(qW, p, ws[k], sg[k], dv), cs[k]);
+                vals[t0 + k] = 0;
+                ++my_k;
+                best.offer(gain<ST>(qW, p, ws[k], sg[k], dv), cs[k]);
             }
         }
         for (int t = threadIdx.x; t < gm; t += BT) {
@@ -551,8 +569,7 @@ __global__ void __launch_bounds__(BT) k_decide_block(QView queue, int bin, Decid
             long long wc = (long long)gvals[slot];
             gkeys[slot] = -1;
             gvals[slot] = 0;
-            if (c == cv) own = wc;
-            else best.offer(gain<ST>(qW, p, wc, a.Sig[c], dv), c);
+            best.offer(gain<ST>(qW, p, wc, a.Sig[c], dv), c);
         }
 #pragma unroll
         for (int off = 16; off > 0; off >>= 1) best.xor_merge(off);
@@ -569,7 +586,6 @@ __global__ void __launch_bounds__(BT) k_decide_block(QView queue, int bin, Decid
                 if (a.check && own != a.dp[v]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
                 a.nextC[v] = decide_final<ST>(cv, q.szv, dv, own, q.sigv, best, a.size, qW, p);
                 my_k += own ? 1u : 0u;
-                s_cnt = 0;
                 s_gcnt = 0;
             }
         }
@@ -645,7 +661,7 @@ __device__ __forceinline__ unsigned decide_single_bin(QView queue, int bin, cons
 
 // first iteration: bins 0-3 in one launch (G ~ row length / 4), the other bins one launch each
 template <int M, bool UNIT>
-__global__ void __launch_bounds__(256) k_decide_single_small(QRec* queues, long long qstride,
+__global__ void __launch_bounds__(256, GALA_SINGLE_MINB) k_decide_single_small(QRec* queues, long long qstride,
                                                              DecideArgs a, typename ModeT<M>::ST qW,
                                                              typename ModeT<M>::ST p) {
     const unsigned kk[4] = {decide_single_bin<1, M, UNIT>(qview(queues, qstride, BIN_S4), BIN_S4, a, qW, p),
@@ -659,7 +675,7 @@ __global__ void __launch_bounds__(256) k_decide_single_small(QRec* queues, long 
     }
 }
 template <int M, bool UNIT>
-__global__ void __launch_bounds__(256) k_decide_single(QView queue, int bin, DecideArgs a,
+__global__ void __launch_bounds__(256, GALA_SINGLE_MINB) k_decide_single(QView queue, int bin, DecideArgs a,
                                                        typename ModeT<M>::ST qW, typename ModeT<M>::ST p) {
     ull t = block_sum_ull<256>((ull)decide_single_bin<32, M, UNIT>(queue, bin, a, qW, p));
     if (threadIdx.x == 0 && t) atomicAdd(&a.ctr->bin_k[bin], t);

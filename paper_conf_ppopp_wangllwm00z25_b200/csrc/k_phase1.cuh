@@ -91,8 +91,11 @@ struct BinThresholds {
 #define PB_BT 256
 #define PB_IPT 4
 
+#ifndef GALA_PRUNE_MINB
+#define GALA_PRUNE_MINB 1
+#endif
 template <typename ST>
-__global__ void __launch_bounds__(PB_BT) k_prune_bin(int vlo, int n, const int64_t* __restrict__ rp,
+__global__ void __launch_bounds__(PB_BT, GALA_PRUNE_MINB) k_prune_bin(int vlo, int n, const int64_t* __restrict__ rp,
                                                      const int64_t* __restrict__ d, const int64_t* __restrict__ dp,
                                                      const int32_t* __restrict__ C, const int64_t* __restrict__ Sig,
                                                      const int32_t* __restrict__ size, int prune, ST qW, ST p,
