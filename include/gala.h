@@ -135,7 +135,16 @@ void gala_graph_free(gala_graph g);
  * (labels are identical for every setting) except "max_iters" (a per-level
  * iteration cap honoured identically by the oracle) and "prune" (pruning
  * changes which vertices are evaluated; the oracle takes the same flag).
- *   "prune"          0/1   MG pruning (Eq. 6/7), default 1
+ *   "prune"          pruning strategy of the active set (§3.2-3.3), default 1:
+ *                    0 none (baseline), 1 MG modularity-gain based (Eq. 6/7, lossless),
+ *                    2 SM strict movement based (lossless), 3 RM relaxed movement
+ *                    based (lossy), 4 MG+RM (lossy, same moves as RM).
+ *                    SM / RM see the moves of the previous iteration of the level
+ *                    (readings c20 / c21).  2-4 are single-GPU only.
+ *   "prune_check"    0/1   instrument the pruning: pruned vertices are evaluated too but
+ *                          never moved; per iteration the trace counts false negatives
+ *                          (pruned, would have moved) and false positives (active, stayed),
+ *                          Eq. 3 / P:145-147.  Results are unchanged.
  *   "trace"          0/1/2 per-iteration records; 2 also copies labels each iteration
  *   "check"          0/1   debug: verify maintained d'(v) against its definition
  *   "timing"         0/1   per-kernel CUDA-event timing (gala_get_kernel_stats)
@@ -171,14 +180,16 @@ gala_status gala_get_stats(gala_graph g, char* json_buf, int64_t cap, int64_t* n
 
 /*
  * Trace access (option "trace" >= 1).  Record i (0 <= i < count) is
- * int64[12]: level, iter, n_level, n_active, n_pruned, n_moved,
+ * int64[16]: level, iter, n_level, n_active, n_pruned, n_moved,
  *            N_hi, N_lo (numerator after the iteration), edges_scanned,
- *            distinct_communities_seen, delta_update_used, reserved.
+ *            distinct_communities_seen, delta_update_used, reserved,
+ *            n_false_negative, n_false_positive (option "prune_check", else 0),
+ *            reserved, reserved.
  * Labels (trace == 2): level-local community of every level vertex after
  * the iteration; out must hold n_level entries.
  */
 gala_status gala_get_trace_count(gala_graph g, int64_t* count);
-gala_status gala_get_trace_record(gala_graph g, int64_t i, int64_t* out12);
+gala_status gala_get_trace_record(gala_graph g, int64_t i, int64_t* out16);
 gala_status gala_get_trace_labels(gala_graph g, int64_t i, int32_t* out, int64_t n_level);
 
 /*

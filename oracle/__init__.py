@@ -83,6 +83,7 @@ class IterRecord:
     n_fn: int
     N: int
     labels: np.ndarray | None
+    n_fp: int = 0
 
 
 @dataclass
@@ -115,9 +116,16 @@ def gamma_pq(gamma: float):
     return p.value, q.value
 
 
+PRUNE_NONE, PRUNE_MG, PRUNE_SM, PRUNE_RM, PRUNE_MG_RM = 0, 1, 2, 3, 4
+
+
 def louvain(g, gamma: float = 1.0, tol: float = 1e-6, max_levels: int = 0, max_iters: int = 0,
-            prune: bool = False, check: bool = False, trace: int = 1) -> OracleResult:
-    """Run the oracle's multi-level BSP Louvain on CSR `g` (graphgen.CSR-like)."""
+            prune: int = 0, check: bool = False, trace: int = 1) -> OracleResult:
+    """Run the oracle's multi-level BSP Louvain on CSR `g` (graphgen.CSR-like).
+
+    prune: 0/False none, 1/True MG (Eq. 6/7), 2 SM, 3 RM, 4 MG+RM (§3.2-3.3; DESIGN.md c20/c21).
+    check: also evaluate pruned vertices -> per-iteration false negatives (n_fn) and, for the
+    active set, false positives (n_fp) in the records."""
     lib = _lib()
     rp, col, w = _csr_arrays(g)
     h = lib.oracle_louvain(g.n, _ptr(rp), _ptr(col), _ptr(w), gamma, tol, max_levels, max_iters,
@@ -129,7 +137,7 @@ def louvain(g, gamma: float = 1.0, tol: float = 1e-6, max_levels: int = 0, max_i
         labels = np.zeros(g.n, dtype=np.int32)
         lib.oracle_labels(h, _ptr(labels))
         recs = []
-        buf = np.zeros(9, dtype=np.int64)
+        buf = np.zeros(10, dtype=np.int64)
         for i in range(int(summ[6])):
             lib.oracle_record(h, i, _ptr(buf))
             lab = None
@@ -137,7 +145,7 @@ def louvain(g, gamma: float = 1.0, tol: float = 1e-6, max_levels: int = 0, max_i
                 lab = np.zeros(int(buf[2]), dtype=np.int32)
                 lib.oracle_record_labels(h, i, _ptr(lab))
             recs.append(IterRecord(int(buf[0]), int(buf[1]), int(buf[2]), int(buf[3]), int(buf[4]),
-                                   int(buf[5]), int(buf[6]), _i128(buf[7], buf[8]), lab))
+                                   int(buf[5]), int(buf[6]), _i128(buf[7], buf[8]), lab, int(buf[9])))
         levs = []
         lb = np.zeros(7, dtype=np.int64)
         for i in range(int(summ[5])):

@@ -44,7 +44,7 @@ typedef __int128 i128;
 /* ---------------------------------------------------------------- results */
 typedef struct {
     int32_t level, iter;
-    int64_t n_level, n_active, n_pruned, n_moved, n_fn;
+    int64_t n_level, n_active, n_pruned, n_moved, n_fn, n_fp;
     i128 N;
     int32_t* labels; /* level-local community of every level vertex after the iteration */
 } orc_rec;
@@ -211,9 +211,22 @@ static void coarsen(const ograph* g, const int32_t* newid, int64_t k, ograph* ou
 /* ------------------------------------------------------------ Louvain */
 /*
  * oracle_louvain: full multi-level run.
- *   prune      : 0 = evaluate every vertex (baseline), 1 = MG pruning (Eq. 6/7)
- *   check      : with prune, also evaluate pruned vertices and count those that
- *                would have moved (false negatives, Theorem 6); they still stay
+ *   prune      : pruning strategy deciding the active set of every iteration
+ *                (§3.2-3.3):
+ *                0 = none (baseline, every vertex evaluated)
+ *                1 = MG, modularity-gain based (Eq. 6/7)
+ *                2 = SM, strict movement based: v inactive iff neither
+ *                    C[v] nor any C[u], u in N(v), gained or lost a member in
+ *                    the previous iteration (reading c20)
+ *                3 = RM, relaxed movement based: v active iff some
+ *                    neighbour u != v changed community in the previous
+ *                    iteration (reading c21)
+ *                4 = MG+RM: inactive iff MG or RM says inactive
+ *                SM and RM have no previous iteration in the first iteration of
+ *                a level: every vertex is active there.
+ *   check      : also evaluate pruned vertices and count those that would have
+ *                moved (false negatives, Eq. 3 / P:147) and the active vertices
+ *                that stay (false positives); pruned vertices still stay
  *   trace      : 0 none, 1 per-iteration records, 2 records + label snapshots
  *   max_iters  : per-level iteration cap (0 = none; honoured identically by the library)
  * Returns an opaque result (free with oracle_free).  status != 0 on error.
@@ -230,7 +243,7 @@ void* oracle_louvain(int64_t n, const int64_t* row_ptr, const int32_t* col, cons
     for (int64_t v = 0; v < n; ++v) lab[v] = (int32_t)v;
     R->lab = lab;
     R->k = n;
-    if (!(tol > 0) || p <= 0) { R->status = 1; return R; }
+    if (!(tol > 0) || p <= 0 || prune < 0 || prune > 4) { R->status = 1; return R; }
     int64_t nnz = row_ptr[n];
     /* level-0 graph (copied; unit weights materialised) */
     ograph G;
@@ -276,6 +289,9 @@ void* oracle_louvain(int64_t n, const int64_t* row_ptr, const int32_t* col, cons
         int32_t* size = (int32_t*)calloc((size_t)nl, sizeof(int32_t));
         int32_t* C = (int32_t*)malloc((size_t)nl * sizeof(int32_t));
         int32_t* nextC = (int32_t*)malloc((size_t)nl * sizeof(int32_t));
+        /* movement history of the previous iteration (SM / RM strategies) */
+        char* moved_prev = (char*)calloc((size_t)nl, 1);     /* v changed community */
+        char* changed_prev = (char*)calloc((size_t)nl, 1);   /* community c gained or lost a member */
         int64_t maxdeg = 0;
         /* level init: every vertex its own community */
         for (int64_t v = 0; v < nl; ++v) {
@@ -301,17 +317,29 @@ void* oracle_louvain(int64_t n, const int64_t* row_ptr, const int32_t* col, cons
             /* min over non-empty communities (reading c3) */
             int64_t minSig = INT64_MAX;
             for (int64_t c = 0; c < nl; ++c) if (Sig[c] > 0 && Sig[c] < minSig) minSig = Sig[c];
-            int64_t n_active = 0, n_pruned = 0, n_fn = 0, bad = 0;
+            int64_t n_active = 0, n_pruned = 0, n_fn = 0, n_fp = 0, bad = 0;
             /* Alg. 1 lines 3-4: every vertex decides from the start-of-iteration state */
-            #pragma omp parallel for schedule(dynamic, 256) reduction(+:n_active, n_pruned, n_fn, bad)
+            #pragma omp parallel for schedule(dynamic, 256) reduction(+:n_active, n_pruned, n_fn, n_fp, bad)
             for (int64_t v = 0; v < nl; ++v) {
                 nextC[v] = C[v];
                 if (d[v] == 0) continue;
                 int pruned = 0;
-                if (prune) {
+                if (prune == 1 || prune == 4) {
                     /* Eq. 6 multiplied by q*W:  q W (2 d' - d) + p (minSig - Sig[C[v]]) d >= 0 */
                     i128 lhs = (i128)q * W * (2 * dp[v] - d[v]) + (i128)p * (minSig - Sig[C[v]]) * d[v];
                     pruned = lhs >= 0;
+                }
+                if (prune == 2 && it > 0) {   /* SM: every community around v unchanged */
+                    int chg = changed_prev[C[v]];
+                    for (int64_t e = G.rp[v]; e < G.rp[v + 1] && !chg; ++e)
+                        if (changed_prev[C[G.col[e]]]) chg = 1;
+                    pruned = !chg;
+                }
+                if ((prune == 3 || prune == 4) && it > 0) {   /* RM: no neighbour moved */
+                    int nb_moved = 0;
+                    for (int64_t e = G.rp[v]; e < G.rp[v + 1] && !nb_moved; ++e)
+                        if (G.col[e] != v && moved_prev[G.col[e]]) nb_moved = 1;
+                    if (!nb_moved) pruned = 1;   /* MG+RM: pruned by either rule */
                 }
                 if (pruned && !check) { n_pruned++; continue; }
                 int64_t d_own = 0;
@@ -319,13 +347,19 @@ void* oracle_louvain(int64_t n, const int64_t* row_ptr, const int32_t* col, cons
                 if (d_own != dp[v]) bad++;                  /* maintained d' must equal its definition */
                 if (pruned) { n_pruned++; if (b != C[v]) n_fn++; continue; }
                 n_active++;
+                if (b == C[v]) n_fp++;
                 nextC[v] = b;
             }
             if (bad) R->status = 3;
             /* Alg. 1 line 5: update the community set (Sigma_tot = D_V, sizes) */
             int64_t n_moved = 0;
+            memset(moved_prev, 0, (size_t)nl);
+            memset(changed_prev, 0, (size_t)nl);
             for (int64_t v = 0; v < nl; ++v) {
                 if (nextC[v] == C[v]) continue;
+                moved_prev[v] = 1;
+                changed_prev[C[v]] = 1;
+                changed_prev[nextC[v]] = 1;
                 Sig[C[v]] -= d[v]; size[C[v]]--;
                 Sig[nextC[v]] += d[v]; size[nextC[v]]++;
                 C[v] = nextC[v];
@@ -350,6 +384,7 @@ void* oracle_louvain(int64_t n, const int64_t* row_ptr, const int32_t* col, cons
                 orc_rec x;
                 x.level = level; x.iter = it; x.n_level = nl;
                 x.n_active = n_active; x.n_pruned = n_pruned; x.n_moved = n_moved; x.n_fn = n_fn;
+                x.n_fp = check ? n_fp : 0;
                 x.N = Nn; x.labels = NULL;
                 if (trace >= 2) {
                     x.labels = (int32_t*)malloc((size_t)nl * sizeof(int32_t));
@@ -380,6 +415,7 @@ void* oracle_louvain(int64_t n, const int64_t* row_ptr, const int32_t* col, cons
         int stop = (k == nl) || (max_levels > 0 && level + 1 >= max_levels) ||
                    (N - N_start < thr);
         free(d); free(s); free(dp); free(Sig); free(size); free(C); free(nextC); free(minmem); free(cnew);
+        free(moved_prev); free(changed_prev);
         if (stop) { free(newid); break; }
         ograph H;
         coarsen(&G, newid, k, &H);
@@ -431,13 +467,14 @@ double oracle_modularity(void* h) {
     if (R->W == 0) return 0.0;
     return (double)((long double)R->N / ((long double)R->q * (long double)R->W * (long double)R->W));
 }
-/* rec: level, iter, n_level, n_active, n_pruned, n_moved, n_fn, N_hi, N_lo */
+/* rec: level, iter, n_level, n_active, n_pruned, n_moved, n_fn, N_hi, N_lo, n_fp */
 void oracle_record(void* h, int64_t i, int64_t* out) {
     orc_rec* x = &((orc_result*)h)->rec[i];
     uint64_t lo;
     out[0] = x->level; out[1] = x->iter; out[2] = x->n_level; out[3] = x->n_active;
     out[4] = x->n_pruned; out[5] = x->n_moved; out[6] = x->n_fn;
     split128(x->N, &out[7], &lo); out[8] = (int64_t)lo;
+    out[9] = x->n_fp;
 }
 int oracle_record_labels(void* h, int64_t i, int32_t* out) {
     orc_rec* x = &((orc_result*)h)->rec[i];

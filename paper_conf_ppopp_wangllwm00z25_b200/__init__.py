@@ -251,12 +251,13 @@ class Graph:
         cnt = ctypes.c_int64()
         _check(L.gala_get_trace_count(self._h, ctypes.byref(cnt)))
         recs = []
-        buf = np.zeros(12, dtype=np.int64)
+        buf = np.zeros(16, dtype=np.int64)
         for i in range(cnt.value):
             _check(L.gala_get_trace_record(self._h, i, _np_ptr(buf)))
             r = dict(level=int(buf[0]), iter=int(buf[1]), n_level=int(buf[2]), n_active=int(buf[3]),
                      n_pruned=int(buf[4]), n_moved=int(buf[5]), N=_i128(buf[6], buf[7]),
-                     edges_scanned=int(buf[8]), distinct=int(buf[9]), delta_used=int(buf[10]))
+                     edges_scanned=int(buf[8]), distinct=int(buf[9]), delta_used=int(buf[10]),
+                     n_fn=int(buf[12]), n_fp=int(buf[13]))
             if labels:
                 lab = np.zeros(r["n_level"], dtype=np.int32)
                 _check(L.gala_get_trace_labels(self._h, i, _np_ptr(lab), r["n_level"]))

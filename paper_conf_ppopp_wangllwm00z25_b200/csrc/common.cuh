@@ -36,6 +36,21 @@ struct IterCounters {
     ull delta_used;         // 1 if the delta d' update ran this iteration
     ull cursor2;            // dynamic work cursor of the hub evaluation
     ull n_items;            // delta-update work items (one per light mover, one per chunk of a heavy one)
+    ull n_fn;               // instrumented pruning: pruned vertices that would have moved (Eq. 3)
+    ull n_fp;               // instrumented pruning: active vertices that stay
+};
+
+// Pruning strategy of the active set (§3.2-3.3; DESIGN.md c20/c21):
+//   0 none, 1 MG (Eq. 6/7), 2 SM (strict movement), 3 RM (relaxed movement), 4 MG+RM.
+// The movement history of the previous iteration lives in per-vertex /
+// per-community arrays holding the iteration id of the last event (-1 = never
+// on this level), so nothing has to be cleared between iterations.
+struct PruneState {
+    int mode;
+    int instr;          // 1: queue pruned vertices too, count n_fn / n_fp, apply only active moves
+    int32_t* rmflag;    // RM: iteration in which some neighbour of v last moved
+    int32_t* smflag;    // SM: iteration in which some neighbour community of v last changed
+    int32_t* chg;       // SM: iteration in which community c last gained or lost a member
 };
 
 // Queue record of an active vertex, written by k_prune_bin (which already

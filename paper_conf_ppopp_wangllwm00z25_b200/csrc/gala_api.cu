@@ -72,7 +72,7 @@ static const char* kc_names[KC_COUNT] = {"prune_bin", "decide_small", "decide_wa
                                          "dp_update", "reduce", "level_init", "phase2"};
 
 struct TraceRec {
-    int64_t v[12];
+    int64_t v[16];
 };
 
 struct DevCSR {
@@ -102,7 +102,7 @@ struct gala_graph_s {
     int64_t* d0 = nullptr;
     int64_t* s0 = nullptr;
     // options
-    int opt_prune = 1, opt_trace = 0, opt_check = 0, opt_timing = 0, opt_max_iters = 0;
+    int opt_prune = 1, opt_prune_check = 0, opt_trace = 0, opt_check = 0, opt_timing = 0, opt_max_iters = 0;
     int opt_delta = 2, opt_force_i128 = 0, opt_force_wide = 0, opt_cuda_graph = 1, opt_log_cap = 4096, opt_singleton = 1, opt_verbose = 0;
     bool rows_distinct0 = false;   // level-0 rows strictly increasing (no duplicate entries)
     int32_t* rev0 = nullptr;       // level-0 reverse-entry index (enables the per-entry community array)
@@ -323,6 +323,7 @@ static void gamma_to_pq(double gamma, int64_t* p, int64_t* q) {
 struct Work {
     cudaStream_t st;
     int64_t ncap, nnzcap;
+    int32_t *rmflag = nullptr, *smflag = nullptr, *chg = nullptr;   // SM / RM movement history (prune 2-4)
     int32_t *C = nullptr, *size = nullptr, *stamp = nullptr, *mv_v = nullptr, *mv_old = nullptr, *mv_chunk = nullptr, *nextC = nullptr;
     QRec* queues = nullptr;
     int32_t* ckey = nullptr;   // level-0 per-entry neighbour community
@@ -351,7 +352,8 @@ struct Work {
     cudaEvent_t ev[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};
     void release() {
         for (auto& e : ev) if (e) { cudaEventDestroy(e); e = nullptr; }
-        dfree(C, st); dfree(size, st); dfree(stamp, st); dfree(mv_v, st); dfree(mv_old, st); dfree(mv_chunk, st); dfree(nextC, st);
+        dfree(C, st); dfree(size, st); dfree(stamp, st); dfree(mv_v, st); dfree(mv_old, st); dfree(mv_chunk, st);
+        dfree(rmflag, st); dfree(smflag, st); dfree(chg, st); dfree(nextC, st);
         dfree(queues, st); dfree(ckey, st); dfree(Sig, st); dfree(d, st); dfree(s, st); dfree(dp, st); dfree(ctr, st);
         dfree(carry, st); dfree(log, st); dfree(part_dc, st); dfree(part_min, st); dfree(part_s2, st);
         dfree(gkeys, st); dfree(gvals, st); dfree(glist, st);
@@ -375,6 +377,22 @@ struct Work {
 // the per-entry neighbour-community array is used on level 0 of single-GPU runs
 static bool use_ckey(const gala_graph_s* g, const Work& wk, const DevCSR& G) {
     return g->opt_ckey && g->rev0 && wk.ckey && !g->di && G.col == g->g0.col;
+}
+
+// pruning strategy state of a run; the SM / RM history arrays are allocated on first use
+static PruneState prune_state(gala_graph_s* g, Work& wk) {
+    PruneState ps;
+    ps.mode = g->opt_prune;
+    ps.instr = g->opt_prune_check;
+    if ((ps.mode == 3 || ps.mode == 4) && !wk.rmflag) wk.rmflag = dalloc<int32_t>(wk.ncap, g->stream);
+    if (ps.mode == 2 && !wk.smflag) {
+        wk.smflag = dalloc<int32_t>(wk.ncap, g->stream);
+        wk.chg = dalloc<int32_t>(wk.ncap, g->stream);
+    }
+    ps.rmflag = (ps.mode == 3 || ps.mode == 4) ? wk.rmflag : nullptr;
+    ps.smflag = ps.mode == 2 ? wk.smflag : nullptr;
+    ps.chg = ps.mode == 2 ? wk.chg : nullptr;
+    return ps;
 }
 
 template <int GW, int MAXDEG, int M>
@@ -555,28 +573,34 @@ static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, typename
     CKL();
     BinThresholds th;
     for (int i = 0; i < NBINS - 1; ++i) th.t[i] = g->bins[i];
+    const PruneState ps = prune_state(g, wk);
     k_prune_bin<typename ModeT<M>::ST><<<grid_for((n + PB_IPT - 1) / PB_IPT, PB_BT, big), PB_BT, 0, st>>>(
-        0, n, G.rp, wk.d, wk.dp, wk.C, wk.Sig, wk.size, g->opt_prune, qW, p, wk.carry, wk.ctr, wk.queues, wk.ncap, th);
+        0, n, G.rp, wk.d, wk.dp, wk.C, wk.Sig, wk.size, ps, qW, p, wk.carry, wk.ctr, wk.queues, wk.ncap, th);
     CKL();
     tm.end(KC_PRUNE, e);
     launch_decide<M, UNIT>(g, wk, G, qW, p, tm, maxdeg, idbits, single);
     e = tm.begin();
     k_apply<<<grid_for(n, AP_BT, big), AP_BT, 0, st>>>(wk.ctr, wk.queues, wk.ncap, wk.nextC, wk.C, wk.Sig, wk.size,
-                                                       wk.dp, wk.stamp, wk.carry, wk.mv_v, wk.mv_old, wk.mv_chunk);
+                                                       wk.dp, wk.stamp, wk.carry, wk.mv_v, wk.mv_old, wk.mv_chunk, ps);
     CKL();
     tm.end(KC_APPLY, e);
     e = tm.begin();
     const bool ck = use_ckey(g, wk, G);
     k_dp_delta<UNIT><<<big, 256, 0, st>>>(wk.ctr, G.rp, G.col, G.w, wk.C, wk.mv_v, wk.mv_old, wk.mv_chunk, wk.stamp, wk.dp,
                                           wk.carry, G.nnz, g->opt_delta, 1, 2, ck ? wk.ckey : nullptr,
-                                          ck ? g->rev0 : nullptr);
+                                          ck ? g->rev0 : nullptr, ps.rmflag);
     CKL();
     k_dp_zero<<<big, 256, 0, st>>>(wk.ctr, 0, n, wk.dp, G.nnz, g->opt_delta, 1, 2);
     CKL();
     k_dp_full<UNIT><<<grid_for((G.nnz + 127) / 128 * 32, 256, big), 256, 0, st>>>(wk.ctr, G.nnz, G.row, G.col, G.w,
                                                                                  wk.C, wk.dp, g->opt_delta, 1, 2,
-                                                                                 ck ? wk.ckey : nullptr, &wk.carry->ckey_valid);
+                                                                                 ck ? wk.ckey : nullptr, &wk.carry->ckey_valid,
+                                                                                 ps.rmflag, wk.stamp, wk.carry);
     CKL();
+    if (ps.mode == 2 && G.nnz) {   // SM: mark rows next to a community that changed
+        k_sm_flags<<<grid_for(G.nnz, 256, big * 4), 256, 0, st>>>(G.nnz, G.row, G.col, wk.C, ps, wk.carry);
+        CKL();
+    }
     tm.end(KC_DP, e);
     e = tm.begin();
     k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>(n, 0, n, wk.dp, wk.s, wk.Sig, wk.part_dc, wk.part_s2, wk.part_min, wk.ctr,
@@ -1055,7 +1079,7 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
             // a1: level init + starting numerator
             cudaEvent_t e = tm.begin();
             k_level_init<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.d, wk.C, wk.Sig, wk.size, wk.dp, wk.stamp,
-                                                                 wk.carry);
+                                                                 wk.carry, prune_state(g, wk));
             CKL();
             if (first_level) {
                 // lab = identity on level 0 (C is the identity right now)
@@ -1117,6 +1141,7 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
                     r.v[4] = (int64_t)c.n_pruned; r.v[5] = (int64_t)c.n_moved;
                     r.v[6] = (int64_t)(N >> 64); r.v[7] = (int64_t)(uint64_t)N;
                     r.v[8] = scanned; r.v[9] = kk; r.v[10] = (int64_t)c.delta_used; r.v[11] = 0;
+                    r.v[12] = (int64_t)c.n_fn; r.v[13] = (int64_t)c.n_fp; r.v[14] = 0; r.v[15] = 0;
                     g->trace.push_back(r);
                 }
             }
@@ -1248,8 +1273,8 @@ static void dist_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, long long
     BinThresholds th;
     for (int i = 0; i < NBINS - 1; ++i) th.t[i] = g->bins[i];
     k_prune_bin<typename ModeT<M>::ST><<<grid_for((lv1 - lv0 + PB_IPT - 1) / PB_IPT, PB_BT, big), PB_BT, 0, st>>>(
-        (int)lv0, (int)lv1, G.rp, wk.d, wk.dp, wk.C, wk.Sig, wk.size, g->opt_prune, qW, p, wk.carry, wk.ctr, wk.queues,
-        wk.ncap, th);
+        (int)lv0, (int)lv1, G.rp, wk.d, wk.dp, wk.C, wk.Sig, wk.size, prune_state(g, wk), qW, p, wk.carry, wk.ctr,
+        wk.queues, wk.ncap, th);
     CKL();
     launch_decide<M, UNIT>(g, wk, G, qW, p, tm, maxdeg, idbits, single);
     vt.lap("dist: prune+decide");
@@ -1296,7 +1321,8 @@ static void dist_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, long long
     CKL();
     if (G.nnz) {
         k_dp_full<UNIT><<<grid_for((G.nnz + 127) / 128 * 32, 256, big), 256, 0, st>>>(wk.ctr, G.nnz, G.row, G.col, G.w,
-                                                                                     wk.C, wk.dp, 0, 1, 2, nullptr, nullptr);
+                                                                                     wk.C, wk.dp, 0, 1, 2, nullptr, nullptr,
+                                                                                     nullptr, nullptr, wk.carry);
         CKL();
     }
     vt.lap("dist: apply+dp");
@@ -1473,7 +1499,7 @@ static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_level
             CK(cudaEventRecord(wk.ev[2], st));
             prepare_level_tables(g, wk, cur, maxdeg);
             k_level_init<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.d, wk.C, wk.Sig, wk.size, wk.dp, wk.stamp,
-                                                                 wk.carry);
+                                                                 wk.carry, prune_state(g, wk));
             CKL();
             if (level == 0) CK(cudaMemcpyAsync(g->lab, wk.C, sizeof(int32_t) * n0, cudaMemcpyDeviceToDevice, st));
             k_iter_begin<<<1, 128, 0, st>>>(wk.ctr);
@@ -1537,6 +1563,7 @@ static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_level
                     r.v[4] = (int64_t)c.n_pruned; r.v[5] = (int64_t)c.n_moved;
                     r.v[6] = (int64_t)(N >> 64); r.v[7] = (int64_t)(uint64_t)N;
                     r.v[8] = scanned; r.v[9] = kk; r.v[10] = 0; r.v[11] = 0;
+                    r.v[12] = 0; r.v[13] = 0; r.v[14] = 0; r.v[15] = 0;
                     g->trace.push_back(r);
                 }
             }
@@ -1816,6 +1843,8 @@ gala_status gala_validate(gala_graph g) {
 }
 
 gala_status gala_run(gala_graph g, double gamma, double tol, int32_t max_levels) {
+    if (g && g->di && (g->opt_prune > 1 || g->opt_prune_check))
+        return set_err(GALA_E_INVALID, "prune strategies 2-4 and prune_check are single-GPU only");
     if (!g) return set_err(GALA_E_INVALID, "null handle");
     if (!(gamma > 0) || !(gamma < 1e12)) return set_err(GALA_E_INVALID, "gamma must be > 0");
     if (!(tol > 0)) return set_err(GALA_E_INVALID, "tol must be > 0");
@@ -1932,7 +1961,10 @@ gala_status gala_set_option(gala_graph g, const char* key, int64_t value) {
     if (!g || !key) return set_err(GALA_E_INVALID, "null argument");
     PoolScope pool_scope(g->cache);
     std::string k(key);
-    if (k == "prune") g->opt_prune = value != 0;
+    if (k == "prune") {
+        if (value < 0 || value > 4) return set_err(GALA_E_INVALID, "prune: 0 none, 1 MG, 2 SM, 3 RM, 4 MG+RM");
+        g->opt_prune = (int)value;
+    } else if (k == "prune_check") g->opt_prune_check = value != 0;
     else if (k == "trace") g->opt_trace = (int)value;
     else if (k == "check") g->opt_check = value != 0;
     else if (k == "timing") g->opt_timing = value != 0;
@@ -1972,10 +2004,10 @@ gala_status gala_get_trace_count(gala_graph g, int64_t* count) {
     *count = (int64_t)g->trace.size();
     return GALA_OK;
 }
-gala_status gala_get_trace_record(gala_graph g, int64_t i, int64_t* out12) {
-    if (!g || !out12) return set_err(GALA_E_INVALID, "null argument");
+gala_status gala_get_trace_record(gala_graph g, int64_t i, int64_t* out16) {
+    if (!g || !out16) return set_err(GALA_E_INVALID, "null argument");
     if (i < 0 || i >= (int64_t)g->trace.size()) return set_err(GALA_E_INVALID, "record index out of range");
-    memcpy(out12, g->trace[i].v, sizeof(int64_t) * 12);
+    memcpy(out16, g->trace[i].v, sizeof(int64_t) * 16);
     return GALA_OK;
 }
 gala_status gala_get_trace_labels(gala_graph g, int64_t i, int32_t* out, int64_t n_level) {

@@ -61,7 +61,7 @@ __global__ void k_degrees(int n, const int64_t* __restrict__ rp, const int32_t* 
 // a1: every vertex its own community
 __global__ void k_level_init(int n, const int64_t* __restrict__ d, int32_t* __restrict__ C,
                              int64_t* __restrict__ Sig, int32_t* __restrict__ size, int64_t* __restrict__ dp,
-                             int32_t* __restrict__ stamp, Carry* __restrict__ carry) {
+                             int32_t* __restrict__ stamp, Carry* __restrict__ carry, PruneState ps) {
     for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n;
          v += (long long)gridDim.x * blockDim.x) {
         C[v] = (int32_t)v;
@@ -69,6 +69,8 @@ __global__ void k_level_init(int n, const int64_t* __restrict__ d, int32_t* __re
         size[v] = 1;
         dp[v] = 0;
         stamp[v] = -1;
+        if (ps.rmflag) ps.rmflag[v] = -1;
+        if (ps.smflag) { ps.smflag[v] = -1; ps.chg[v] = -1; }
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) { carry->iter = 0; carry->converged = 0; carry->log_base = 0; }
 }
@@ -98,12 +100,13 @@ template <typename ST>
 __global__ void __launch_bounds__(PB_BT, GALA_PRUNE_MINB) k_prune_bin(int vlo, int n, const int64_t* __restrict__ rp,
                                                      const int64_t* __restrict__ d, const int64_t* __restrict__ dp,
                                                      const int32_t* __restrict__ C, const int64_t* __restrict__ Sig,
-                                                     const int32_t* __restrict__ size, int prune, ST qW, ST p,
+                                                     const int32_t* __restrict__ size, PruneState ps, ST qW, ST p,
                                                      const Carry* __restrict__ carry, IterCounters* __restrict__ ctr,
                                                      QRec* __restrict__ queues, long long qstride, BinThresholds th) {
     __shared__ unsigned s_cnt[NBINS];
     __shared__ ull s_base[NBINS];
     const long long minSig = carry->minSig;
+    const int prev = carry->iter - 1;   // the previous iteration of this level (-1: none)
     ull my_active = 0, my_pruned = 0;
     ull my_deg[NBINS];
 #pragma unroll
@@ -112,6 +115,7 @@ __global__ void __launch_bounds__(PB_BT, GALA_PRUNE_MINB) k_prune_bin(int vlo, i
     for (long long t0 = vlo + (long long)blockIdx.x * tile; t0 < n; t0 += (long long)gridDim.x * tile) {
         if (threadIdx.x < NBINS) s_cnt[threadIdx.x] = 0;
         int bin[PB_IPT];
+        bool act[PB_IPT];
         long long dv[PB_IPT], dpv[PB_IPT];
         int cv[PB_IPT];
 #pragma unroll
@@ -133,13 +137,20 @@ __global__ void __launch_bounds__(PB_BT, GALA_PRUNE_MINB) k_prune_bin(int vlo, i
             bin[j] = -1;
             deg[j] = 0;
             beg[j] = 0;
+            act[j] = false;
             if (dv[j] > 0) {
                 bool active = true;
-                if (prune) {
+                if (ps.mode == 1 || ps.mode == 4) {
                     ST lhs = qW * (ST)(2 * dpv[j] - dv[j]) + p * (ST)(minSig - sg[j]) * (ST)dv[j];
                     active = lhs < (ST)0;
                 }
-                if (active) {
+                if (ps.mode == 2 && prev >= 0)   // SM: some community around v changed
+                    active = ps.chg[cv[j]] == prev || ps.smflag[v] == prev;
+                if ((ps.mode == 3 || ps.mode == 4) && prev >= 0 && ps.rmflag[v] != prev)
+                    active = false;              // RM: no neighbour moved
+                act[j] = active;
+                if (active) { my_active++; } else { my_pruned++; }
+                if (active || ps.instr) {
                     beg[j] = rp[v];
                     long long dg = rp[v + 1] - beg[j];
                     deg[j] = (int)(dg > INT_MAX ? INT_MAX : dg);
@@ -148,10 +159,7 @@ __global__ void __launch_bounds__(PB_BT, GALA_PRUNE_MINB) k_prune_bin(int vlo, i
                     for (int k = NBINS - 2; k >= 0; --k)
                         if (deg[j] <= th.t[k]) b = k;
                     bin[j] = b;
-                    my_active++;
                     my_deg[b] += (ull)deg[j];
-                } else {
-                    my_pruned++;
                 }
             }
         }
@@ -184,7 +192,7 @@ __global__ void __launch_bounds__(PB_BT, GALA_PRUNE_MINB) k_prune_bin(int vlo, i
                 q.szv = szv[j];
                 q.dv = dv[j];
                 q.sigv = sg[j];
-                q.pad = 0;
+                q.pad = act[j] ? 1 : 0;   // 0: queued only for the FN/FP instrumentation
                 qview(queues, qstride, bin[j])[(long long)s_base[bin[j]] + off[j]] = q;
             }
         }
@@ -218,7 +226,7 @@ __global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr,
                                                  int32_t* __restrict__ size, int64_t* __restrict__ dp,
                                                  int32_t* __restrict__ stamp, const Carry* __restrict__ carry,
                                                  int32_t* __restrict__ it_v, int32_t* __restrict__ it_old,
-                                                 int32_t* __restrict__ it_chunk) {
+                                                 int32_t* __restrict__ it_chunk, PruneState ps) {
     __shared__ unsigned s_cnt, s_items;
     __shared__ ull s_ibase;
     long long cnt[NBINS];
@@ -227,7 +235,7 @@ __global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr,
     for (int b = 0; b < NBINS; ++b) { cnt[b] = (long long)ctr->bin_count[b]; total += cnt[b]; }
     const int iter_id = carry->iter;
     const int lane = lane_id();
-    ull my_deg = 0;
+    ull my_deg = 0, my_fn = 0, my_fp = 0;
     for (long long t0 = (long long)blockIdx.x * AP_BT; t0 < total; t0 += (long long)gridDim.x * AP_BT) {
         long long i = t0 + threadIdx.x;
         bool mover = false;
@@ -242,8 +250,13 @@ __global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr,
             v = q.v;
             int nc = nextC[v];
             oc = q.cv;
+            if (ps.instr) {
+                if (!q.pad) { my_fn += nc != oc; nc = oc; }   // pruned: would it have moved?  it stays
+                else my_fp += nc == oc;
+            }
             if (nc != oc) {
                 mover = true;
+                if (ps.chg) { ps.chg[oc] = iter_id; ps.chg[nc] = iter_id; }
                 long long dv = q.dv;
                 deg = q.deg;
                 C[v] = nc;
@@ -288,6 +301,12 @@ __global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr,
     }
     ull md = block_sum_ull<AP_BT>(my_deg);
     if (threadIdx.x == 0 && md) atomicAdd(&ctr->moved_deg, md);
+    if (ps.instr) {
+        ull f = block_sum_ull<AP_BT>(my_fn);
+        if (threadIdx.x == 0 && f) atomicAdd(&ctr->n_fn, f);
+        f = block_sum_ull<AP_BT>(my_fp);
+        if (threadIdx.x == 0 && f) atomicAdd(&ctr->n_fp, f);
+    }
 }
 
 // ---------------------------------------------------------------------------
@@ -313,7 +332,7 @@ __global__ void __launch_bounds__(256) k_dp_delta(IterCounters* __restrict__ ctr
                                                   const int32_t* __restrict__ stamp, int64_t* __restrict__ dp,
                                                   const Carry* __restrict__ carry, long long nnz, int mode,
                                                   long long fnum, long long fden, int32_t* __restrict__ ckey,
-                                                  const int32_t* __restrict__ rev) {
+                                                  const int32_t* __restrict__ rev, int32_t* __restrict__ rmflag) {
     if (!use_delta(ctr, nnz, mode, fnum, fden)) return;
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         ctr->delta_used = 1;
@@ -349,6 +368,7 @@ __global__ void __launch_bounds__(256) k_dp_delta(IterCounters* __restrict__ ctr
 #pragma unroll
             for (int t = 0; t < 4; ++t) {
                 if (x[t] == u) continue;
+                if (rmflag) rmflag[x[t]] = iter_id;   // RM: a neighbour of x moved
                 if (cx[t] == nc) acc += wt[t];
                 if (sx[t] != iter_id) {
                     if (cx[t] == oc) atomicAdd(reinterpret_cast<ull*>(&dp[x[t]]), (ull)(-wt[t]));
@@ -380,8 +400,11 @@ __global__ void __launch_bounds__(256) k_dp_full(IterCounters* __restrict__ ctr,
                                                  const int32_t* __restrict__ row, const int32_t* __restrict__ col,
                                                  const int64_t* __restrict__ w, const int32_t* __restrict__ C,
                                                  int64_t* __restrict__ dp, int mode, long long fnum, long long fden,
-                                                 int32_t* __restrict__ ckey, int* __restrict__ carry_valid) {
+                                                 int32_t* __restrict__ ckey, int* __restrict__ carry_valid,
+                                                 int32_t* __restrict__ rmflag, const int32_t* __restrict__ stamp,
+                                                 const Carry* __restrict__ carry) {
     if (use_delta(ctr, nnz, mode, fnum, fden)) return;
+    const int iter_id = rmflag ? carry->iter : 0;
     if (ckey && blockIdx.x == 0 && threadIdx.x == 0) carry_valid[0] = 1;   // rewritten below for every entry
     const int lane = lane_id();
     const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
@@ -401,6 +424,11 @@ __global__ void __launch_bounds__(256) k_dp_full(IterCounters* __restrict__ ctr,
         for (int t = 0; t < 4; ++t) {
             cr[t] = r[t] >= 0 ? C[r[t]] : 0;
             cu[t] = u[t] >= 0 ? C[u[t]] : 1;
+        }
+        if (rmflag) {   // RM: mark rows with a neighbour that moved in this iteration
+#pragma unroll
+            for (int t = 0; t < 4; ++t)
+                if (r[t] >= 0 && u[t] != r[t] && stamp[u[t]] == iter_id) rmflag[r[t]] = iter_id;
         }
         if (ckey) {   // refresh the per-entry neighbour communities for the next decide
 #pragma unroll
@@ -435,6 +463,20 @@ __global__ void __launch_bounds__(256) k_dp_full(IterCounters* __restrict__ ctr,
 // to finish combines the per-block partials and takes the convergence
 // decision dN < T (Alg. 1 lines 12-13) on the device.
 // mode 0: level start (N := N'), mode 1: iteration end.
+// SM pruning history: entry (r, u) marks row r when the community of
+// u gained or lost a member in this iteration (communities after the moves).
+// Edge-parallel over all entries; only launched with the SM strategy.
+__global__ void __launch_bounds__(256) k_sm_flags(long long nnz, const int32_t* __restrict__ row,
+                                                  const int32_t* __restrict__ col, const int32_t* __restrict__ C,
+                                                  PruneState ps, const Carry* __restrict__ carry) {
+    const int iter_id = carry->iter;
+    for (long long e = (long long)blockIdx.x * blockDim.x + threadIdx.x; e < nnz;
+         e += (long long)gridDim.x * blockDim.x) {
+        const int u = col[e];
+        if (ps.chg[C[u]] == iter_id) ps.smflag[row[e]] = iter_id;
+    }
+}
+
 // ---------------------------------------------------------------------------
 template <int BT>
 __global__ void __launch_bounds__(BT) k_reduce(int n, int dlo, int dhi, const int64_t* __restrict__ dp,

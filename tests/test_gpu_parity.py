@@ -43,8 +43,9 @@ def hub(t):
 
 
 def assert_parity(g, gamma=1.0, tol=1e-6, max_levels=0, prune=True, labels=True, **opts):
-    o = oracle.louvain(g, gamma=gamma, tol=tol, max_levels=max_levels, prune=prune, trace=2 if labels else 1,
-                       max_iters=opts.get("max_iters", 0))
+    pc = bool(opts.get("prune_check", 0))
+    o = oracle.louvain(g, gamma=gamma, tol=tol, max_levels=max_levels, prune=int(prune), check=pc,
+                       trace=2 if labels else 1, max_iters=opts.get("max_iters", 0))
     assert o.status == 0
     r = run_gpu(g, gamma=gamma, tol=tol, max_levels=max_levels, trace=2 if labels else 1, prune=int(prune),
                 check=1, **opts)
@@ -56,6 +57,8 @@ def assert_parity(g, gamma=1.0, tol=1e-6, max_levels=0, prune=True, labels=True,
         assert x.N == y["N"], f"N differs at level {x.level} iter {x.iter}"
         assert x.n_moved == y["n_moved"]
         assert x.n_active == y["n_active"] and x.n_pruned == y["n_pruned"]
+        if pc:
+            assert (x.n_fn, x.n_fp) == (y["n_fn"], y["n_fp"]), f"FN/FP differ at level {x.level} iter {x.iter}"
     assert np.array_equal(o.labels, r["labels"])
     assert o.N == r["N"]
     assert abs(o.Q - r["Q"]) <= 1e-9
@@ -82,6 +85,24 @@ def test_random_graph_parity(seed):
 @pytest.mark.parametrize("prune", [True, False])
 def test_synthetic_parity(name, prune):
     assert_parity(gg.make(name), prune=prune)
+
+
+@pytest.mark.parametrize("name", ["karate", "lfr_small", "rmat_small"])
+@pytest.mark.parametrize("strategy", [0, 1, 2, 3, 4])
+@pytest.mark.parametrize("check", [0, 1])
+def test_pruning_strategy_parity(name, strategy, check):
+    """§3.2-3.3 strategies (none / MG / SM / RM / MG+RM): labels, N and active / pruned / moved
+    counts bit-exact per iteration; with prune_check also the false negatives / positives."""
+    assert_parity(gg.make(name), prune=strategy, prune_check=check)
+
+
+@pytest.mark.parametrize("strategy", [2, 3, 4])
+def test_pruning_strategy_weighted_and_graph_mode(strategy):
+    for seed in range(3):
+        g = gg.random_graph(300, 2000, seed=3000 + seed, max_w=5, self_loops=4)
+        assert_parity(g, gamma=[1.0, 0.5, 2.0][seed], prune=strategy, prune_check=seed % 2)
+    assert_parity(gg.make("rmat_small"), prune=strategy, labels=False)
+    assert_parity(gg.make("rmat_small"), prune=strategy, labels=False, delta_update=1)
 
 
 @pytest.mark.parametrize("opts", [
