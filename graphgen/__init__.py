@@ -234,6 +234,11 @@ CONFIGS = {
     "lfr_small": dict(desc="LFR n=20,000, <k>=20, kmax=200, mu=0.3, seed 11"),
     "lfr_mid": dict(desc="LFR n=200,000, <k>=40, kmax=1000, mu=0.3, seed 12"),
     "rmat_small": dict(desc="R-MAT scale 15, n=30,000, 300k edges, seed 13"),
+    # Table 4-style NMI graphs (LFR, 100,000 vertices, 0.65M / 1.44M / 1.44M edges;
+    # the paper does not give their mixing, so three mixing levels are used)
+    "lfr100k_1": dict(desc="LFR n=100,000, <k>=13, kmax=100, mu=0.5, seed 21"),
+    "lfr100k_2": dict(desc="LFR n=100,000, <k>=29, kmax=300, mu=0.1, seed 22"),
+    "lfr100k_3": dict(desc="LFR n=100,000, <k>=29, kmax=300, mu=0.45, seed 23"),
 }
 
 
@@ -254,4 +259,10 @@ def make(name: str) -> CSR:
         return lfr(200_000, 40.0, 1000, 0.3, seed=12, name=name)
     if name == "rmat_small":
         return rmat(15, 30_000, 300_000, seed=13, name=name)
+    if name == "lfr100k_1":
+        return lfr(100_000, 13.0, 100, 0.5, cmin=20, cmax=1000, seed=21, name=name)
+    if name == "lfr100k_2":
+        return lfr(100_000, 29.0, 300, 0.1, cmin=20, cmax=1000, seed=22, name=name)
+    if name == "lfr100k_3":
+        return lfr(100_000, 29.0, 300, 0.45, cmin=20, cmax=1000, seed=23, name=name)
     raise KeyError(name)

@@ -569,8 +569,7 @@ static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, typename
     const int n = (int)G.n;
     const int big = g->num_sms * 8;
     cudaEvent_t e = tm.begin();
-    k_iter_begin<<<1, 128, 0, st>>>(wk.ctr);
-    CKL();
+    // the counters were cleared by the previous iteration's reduce (or the level start)
     BinThresholds th;
     for (int i = 0; i < NBINS - 1; ++i) th.t[i] = g->bins[i];
     const PruneState ps = prune_state(g, wk);
@@ -588,9 +587,7 @@ static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, typename
     const bool ck = use_ckey(g, wk, G);
     k_dp_delta<UNIT><<<big, 256, 0, st>>>(wk.ctr, G.rp, G.col, G.w, wk.C, wk.mv_v, wk.mv_old, wk.mv_chunk, wk.stamp, wk.dp,
                                           wk.carry, G.nnz, g->opt_delta, 1, 2, ck ? wk.ckey : nullptr,
-                                          ck ? g->rev0 : nullptr, ps.rmflag);
-    CKL();
-    k_dp_zero<<<big, 256, 0, st>>>(wk.ctr, 0, n, wk.dp, G.nnz, g->opt_delta, 1, 2);
+                                          ck ? g->rev0 : nullptr, ps.rmflag, n);
     CKL();
     k_dp_full<UNIT><<<grid_for((G.nnz + 127) / 128 * 32, 256, big), 256, 0, st>>>(wk.ctr, G.nnz, G.row, G.col, G.w,
                                                                                  wk.C, wk.dp, g->opt_delta, 1, 2,
@@ -605,9 +602,8 @@ static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, typename
     e = tm.begin();
     k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>(n, 0, n, wk.dp, wk.s, wk.Sig, wk.part_dc, wk.part_s2, wk.part_min, wk.ctr,
                                                   wk.carry, (long long)(qW128 >> 64), (ull)qW128, (long long)p,
-                                                  (long long)(T >> 64), (ull)T, 1);
-    CKL();
-    k_record<<<1, 32, 0, st>>>(wk.ctr, wk.carry, wk.log, wk.log_cap, g->opt_max_iters, cond);
+                                                  (long long)(T >> 64), (ull)T, 1, wk.log, wk.log_cap, g->opt_max_iters,
+                                                  cond);
     CKL();
     tm.end(KC_REDUCE, e);
 }

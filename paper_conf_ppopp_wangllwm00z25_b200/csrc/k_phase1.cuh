@@ -28,6 +28,28 @@ __device__ __forceinline__ ull block_sum_ull(ull x) {   // result valid in threa
     return x;
 }
 
+// K per-thread counters summed over the block and added to K global counters
+// with one barrier (instead of one block reduction per counter)
+template <int BT, int K>
+__device__ __forceinline__ void block_add_counters(const ull (&x)[K], ull* const (&dst)[K]) {
+    __shared__ ull sh[BT / 32][K];
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+        ull y = x[k];
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) y += __shfl_xor_sync(FULLMASK, y, o);
+        if (lane == 0) sh[wib][k] = y;
+    }
+    __syncthreads();
+    if (threadIdx.x < K) {
+        ull t = 0;
+#pragma unroll
+        for (int w = 0; w < BT / 32; ++w) t += sh[w][threadIdx.x];
+        if (t) atomicAdd(dst[threadIdx.x], t);
+    }
+}
+
 // ---------------------------------------------------------------------------
 // a1: weighted degree d(v) and self-loop weight s(v) of every vertex (warp per row)
 // ---------------------------------------------------------------------------
@@ -166,7 +188,10 @@ __global__ void __launch_bounds__(PB_BT, GALA_PRUNE_MINB) k_prune_bin(int vlo, i
         int szv[PB_IPT];
 #pragma unroll
         for (int j = 0; j < PB_IPT; ++j) szv[j] = bin[j] >= 0 ? size[cv[j]] : 0;
-        __syncthreads();   // s_cnt reset visible
+        bool anyq = false;
+#pragma unroll
+        for (int j = 0; j < PB_IPT; ++j) anyq |= bin[j] >= 0;
+        if (!__syncthreads_or(anyq)) continue;   // nothing queued in this tile (also: s_cnt reset visible)
         unsigned off[PB_IPT];
 #pragma unroll
         for (int j = 0; j < PB_IPT; ++j) {
@@ -197,15 +222,13 @@ __global__ void __launch_bounds__(PB_BT, GALA_PRUNE_MINB) k_prune_bin(int vlo, i
             }
         }
     }
-    ull a = block_sum_ull<PB_BT>(my_active);
-    if (threadIdx.x == 0 && a) atomicAdd(&ctr->n_active, a);
-    ull pr = block_sum_ull<PB_BT>(my_pruned);
-    if (threadIdx.x == 0 && pr) atomicAdd(&ctr->n_pruned, pr);
+    ull vals[NBINS + 2];
+    ull* dsts[NBINS + 2];
 #pragma unroll
-    for (int b = 0; b < NBINS; ++b) {
-        ull x = block_sum_ull<PB_BT>(my_deg[b]);
-        if (threadIdx.x == 0 && x) atomicAdd(&ctr->bin_deg[b], x);
-    }
+    for (int b = 0; b < NBINS; ++b) { vals[b] = my_deg[b]; dsts[b] = &ctr->bin_deg[b]; }
+    vals[NBINS] = my_active; dsts[NBINS] = &ctr->n_active;
+    vals[NBINS + 1] = my_pruned; dsts[NBINS + 1] = &ctr->n_pruned;
+    block_add_counters<PB_BT, NBINS + 2>(vals, dsts);
 }
 
 // ---------------------------------------------------------------------------
@@ -332,8 +355,14 @@ __global__ void __launch_bounds__(256) k_dp_delta(IterCounters* __restrict__ ctr
                                                   const int32_t* __restrict__ stamp, int64_t* __restrict__ dp,
                                                   const Carry* __restrict__ carry, long long nnz, int mode,
                                                   long long fnum, long long fden, int32_t* __restrict__ ckey,
-                                                  const int32_t* __restrict__ rev, int32_t* __restrict__ rmflag) {
-    if (!use_delta(ctr, nnz, mode, fnum, fden)) return;
+                                                  const int32_t* __restrict__ rev, int32_t* __restrict__ rmflag,
+                                                  int n) {
+    if (!use_delta(ctr, nnz, mode, fnum, fden)) {   // full recompute follows: clear d' (k_dp_zero fused)
+        for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n;
+             v += (long long)gridDim.x * blockDim.x)
+            dp[v] = 0;
+        return;
+    }
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         ctr->delta_used = 1;
         if (ckey) const_cast<Carry*>(carry)->ckey_valid = 0;   // per-entry communities now stale
@@ -477,6 +506,27 @@ __global__ void __launch_bounds__(256) k_sm_flags(long long nnz, const int32_t* 
     }
 }
 
+// end-of-iteration bookkeeping shared by k_record and the fused k_reduce: append
+// the counters to the device log, advance the iteration index and (graph mode)
+// set the loop condition of the enclosing conditional while-node: continue iff
+// not converged, under the iteration cap and with room in the log.
+__device__ __forceinline__ void record_iteration(const IterCounters* ctr, Carry* carry, IterLog* log, int log_cap,
+                                                 int max_iters, unsigned long long cond_handle) {
+    const int it = carry->iter;
+    const int slot = it - carry->log_base;
+    if (slot >= 0 && slot < log_cap) {
+        IterLog& L = log[slot];
+        L.ctr = *ctr;
+        L.N_hi = carry->N_hi;
+        L.N_lo = carry->N_lo;
+        L.converged = carry->converged;
+    }
+    carry->iter = it + 1;
+    const int more = !carry->converged && (max_iters <= 0 || it + 1 < max_iters) && (slot + 1 < log_cap);
+    carry->more = more;
+    if (cond_handle) cudaGraphSetConditional((cudaGraphConditionalHandle)cond_handle, more ? 1u : 0u);
+}
+
 // ---------------------------------------------------------------------------
 template <int BT>
 __global__ void __launch_bounds__(BT) k_reduce(int n, int dlo, int dhi, const int64_t* __restrict__ dp,
@@ -484,7 +534,9 @@ __global__ void __launch_bounds__(BT) k_reduce(int n, int dlo, int dhi, const in
                                                long long* __restrict__ part_dc, i128* __restrict__ part_s2,
                                                long long* __restrict__ part_min, IterCounters* __restrict__ ctr,
                                                Carry* __restrict__ carry, long long qW_hi, ull qW_lo, long long p,
-                                               long long T_hi, ull T_lo, int mode) {
+                                               long long T_hi, ull T_lo, int mode, IterLog* __restrict__ log = nullptr,
+                                               int log_cap = 0, int max_iters = 0,
+                                               unsigned long long cond_handle = 0) {
     __shared__ long long sh_dc[BT / 32];
     __shared__ i128 sh_s2[BT / 32];
     __shared__ long long sh_min[BT / 32];
@@ -586,6 +638,11 @@ __global__ void __launch_bounds__(BT) k_reduce(int n, int dlo, int dhi, const in
         carry->sumDC = tdc;
         carry->converged = conv;
         ctr->ticket = 0;
+        if (log) {   // k_record fused: log the iteration, advance, set the loop condition, clear counters
+            record_iteration(ctr, carry, log, log_cap, max_iters, cond_handle);
+            ull* c = reinterpret_cast<ull*>(ctr);
+            for (int i = 0; i < (int)(sizeof(IterCounters) / sizeof(ull)); ++i) c[i] = 0;
+        }
     }
 }
 
@@ -598,19 +655,7 @@ __global__ void __launch_bounds__(BT) k_reduce(int n, int dlo, int dhi, const in
 __global__ void k_record(const IterCounters* __restrict__ ctr, Carry* __restrict__ carry, IterLog* __restrict__ log,
                          int log_cap, int max_iters, unsigned long long cond_handle) {
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
-    const int it = carry->iter;
-    const int slot = it - carry->log_base;
-    if (slot >= 0 && slot < log_cap) {
-        IterLog& L = log[slot];
-        L.ctr = *ctr;
-        L.N_hi = carry->N_hi;
-        L.N_lo = carry->N_lo;
-        L.converged = carry->converged;
-    }
-    carry->iter = it + 1;
-    const int more = !carry->converged && (max_iters <= 0 || it + 1 < max_iters) && (slot + 1 < log_cap);
-    carry->more = more;
-    if (cond_handle) cudaGraphSetConditional((cudaGraphConditionalHandle)cond_handle, more ? 1u : 0u);
+    record_iteration(ctr, carry, log, log_cap, max_iters, cond_handle);
 }
 
 // level-0 init of the per-entry neighbour communities: C = identity
