@@ -270,7 +270,7 @@ def main():
         tpath = os.path.join(ROOT, "profiles", "traffic.json")
         if os.path.exists(tpath):
             t = json.load(open(tpath))
-            traffic = t.get(name, {}).get("dram_bytes_per_launch")
+            traffic = t.get(args.config, {}).get(name, {}).get("dram_bytes_per_launch")
         roofline = {"bound": "hbm", "kernel": name, "achieved": achieved, "peak": peak, "unit": "GB/s",
                     "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
                     "alg_bytes_per_launch": ks["alg_bytes"] / max(ks["launches"], 1),

@@ -65,11 +65,12 @@ static thread_local long long g_launches = 0;
 // ------------------------------------------------------------------ kernel classes
 enum KClass {
     KC_PRUNE = 0, KC_DEC_SMALL, KC_DEC_WARP, KC_DEC_WARP2, KC_DEC_BLOCK, KC_DEC_HUB,
-    KC_APPLY, KC_DP, KC_REDUCE, KC_INIT, KC_PHASE2, KC_COUNT
+    KC_APPLY, KC_DP, KC_REDUCE, KC_INIT, KC_PHASE2, KC_DEC_SINGLE, KC_COUNT
 };
 static const char* kc_names[KC_COUNT] = {"prune_bin", "decide_small", "decide_warp", "decide_warp512",
                                          "decide_block", "decide_hub", "apply",
-                                         "dp_update", "reduce", "level_init", "phase2"};
+                                         "dp_update", "reduce", "level_init", "phase2",
+                                         "decide_single"};
 
 struct TraceRec {
     int64_t v[16];
@@ -435,14 +436,13 @@ static void launch_single(gala_graph_s* g, Work& wk, const DecideArgs& a, typena
     cudaEvent_t e = tm.begin();
     k_decide_single_small<M, UNIT><<<grid, 256, 0, st>>>(wk.queues, qs, a, qW, p);
     CKL();
-    tm.end(KC_DEC_SMALL, e);
-    static const int kcs[3] = {KC_DEC_WARP, KC_DEC_WARP2, KC_DEC_BLOCK};
+    tm.end(KC_DEC_SINGLE, e);
     for (int b = BIN_WARP; b <= BIN_BLOCK; ++b) {
         if (maxdeg <= g->bins[b - 1]) break;
         e = tm.begin();
         k_decide_single<M, UNIT><<<grid, 256, 0, fk.branch(b - BIN_WARP)>>>(qview(wk.queues, qs, b), b, a, qW, p);
         CKL();
-        tm.end(kcs[b - BIN_WARP], e);
+        tm.end(KC_DEC_SINGLE, e);
     }
     launch_hub<M, UNIT>(g, wk, a, qW, p, tm, wk.hub_on ? fk.branch(3) : st);
 }
@@ -704,14 +704,15 @@ static i128 log_N(const IterLog& l) {
 }
 
 // algorithmic bytes per kernel class of one iteration
-static void account_bytes(gala_graph_s* g, const IterCounters& c, int64_t n, int64_t nnz, bool unit) {
+static void account_bytes(gala_graph_s* g, const IterCounters& c, int64_t n, int64_t nnz, bool unit, bool single) {
     const double om = unit ? 0.0 : 8.0;
     double act = 0;
     for (int b = 0; b < NBINS; ++b) {
         double cnt = (double)c.bin_count[b], deg = (double)c.bin_deg[b], kk = (double)c.bin_k[b];
         // per vertex: queue 4, row_ptr pair 16, C[v] 4, d 8, Sig[C[v]] 8, nextC 4; per entry: col 4 (+w), C[u] 4;
         // per distinct neighbour community: Sig 8
-        const int kc = b <= BIN_S32 ? KC_DEC_SMALL : KC_DEC_WARP + (b - BIN_WARP);
+        int kc = b <= BIN_S32 ? KC_DEC_SMALL : KC_DEC_WARP + (b - BIN_WARP);
+        if (single && kc != KC_DEC_HUB) kc = KC_DEC_SINGLE;   // first iteration: singleton kernels
         g->kc_bytes[kc] += cnt * (4 + 16 + 4 + 8 + 8 + 4) + deg * (4 + om + 4) + 8 * kk;
         act += cnt;
     }
@@ -1124,7 +1125,7 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
             i128 N = N_start;
             for (size_t it = 0; it < logs.size(); ++it) {
                 const IterCounters& c = logs[it].ctr;
-                account_bytes(g, c, nl, cur.nnz, unit);
+                account_bytes(g, c, nl, cur.nnz, unit, it == 0 && g->opt_singleton && (level > 0 || g->rows_distinct0));
                 g->dp_mismatch += (int64_t)c.dp_mismatch;
                 N = log_N(logs[it]);
                 int64_t scanned = 0, kk = 0;
