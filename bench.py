@@ -332,6 +332,7 @@ def main():
         "louvain_seconds": total_s / args.steps,
         "step_ms": [round(x, 3) for x in step_ms],
         "modularity": Q,
+        "nmi_vs_planted": (gala.nmi_device(labels, g.truth) if getattr(g, "truth", None) is not None else None),
         "levels": len(last_stats["levels"]),
         "iterations": sum(lv["iters"] for lv in last_stats["levels"]),
         "gteps_scanned": scanned / total_s / 1e9,

@@ -104,7 +104,8 @@ struct gala_graph_s {
     int64_t* s0 = nullptr;
     // options
     int opt_prune = 1, opt_prune_check = 0, opt_trace = 0, opt_check = 0, opt_timing = 0, opt_max_iters = 0;
-    int opt_delta = 2, opt_force_i128 = 0, opt_force_wide = 0, opt_cuda_graph = 1, opt_log_cap = 4096, opt_singleton = 1, opt_verbose = 0;
+    int opt_delta = 2, opt_force_i128 = 0, opt_force_wide = 0, opt_cuda_graph = 1, opt_log_cap = 4096, opt_singleton = 1, opt_verbose = 0, opt_agg_big_chunk = 1,
+        opt_agg_chunk = AGG_CH, opt_agg_scap = 8192;
     bool rows_distinct0 = false;   // level-0 rows strictly increasing (no duplicate entries)
     int32_t* rev0 = nullptr;       // level-0 reverse-entry index (enables the per-entry community array)
     int opt_ckey = 0;
@@ -816,7 +817,7 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
     vt.lap("agg: stats+gather");
     // shared-memory capacity of the block path: up to 8192 slots (14 B each)
     int scap = 512;
-    while (scap < 8192 && scap < 2 * k) scap <<= 1;
+    while (scap < g->opt_agg_scap && scap < 2 * k) scap <<= 1;
     k_agg_classify<<<grid_for(k, 256, big), 256, 0, st>>>(k, ent, scap, dn, wlist, nbig_dev + 1, blist, nbig_dev + 2,
                                                          bigc, bigcap, nbig_dev);
     CKL();
@@ -843,14 +844,39 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
         CK(cudaMemsetAsync(gvals, 0, sizeof(ull) * gtot, st));
         CK(cudaMemsetAsync(gcnt, 0, sizeof(int) * nbig, st));
         vt.lap("agg: big alloc+clear");
-        const int bpc = 32;
-        if (unit) k_agg_big_insert<true, unsigned><<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
-        else if (v32) k_agg_big_insert<false, unsigned><<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
-        else k_agg_big_insert<false, ull><<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
+        long long* nch = dalloc<long long>(nbig + 1, st);
+        long long* choff = dalloc<long long>(nbig + 1, st);
+        k_agg_big_nchunks<<<grid_for(nbig, 256, big), 256, 0, st>>>(nbig, bigc, ent, nch, g->opt_agg_chunk);
         CKL();
-        vt.lap("agg: big insert");
-        k_agg_big_emit<<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
-        CKL();
+        scan_excl(nch, choff, nbig, st);
+        if (g->opt_agg_big_chunk) {
+            const int gb = g->num_sms * 2;   // 80 KB (32-bit values) / 112 KB smem per block
+            if (unit || v32) {
+                const size_t sm = agg_chunk_smem<unsigned>();
+                auto kf = unit ? k_agg_big_chunk<true, unsigned> : k_agg_big_chunk<false, unsigned>;
+                CK(cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+                kf<<<gb, 256, sm, st>>>(a, bigc, nbig, choff, goff, gkeys, gvals, glist, gcnt, g->opt_agg_chunk);
+            } else {
+                const size_t sm = agg_chunk_smem<ull>();
+                CK(cudaFuncSetAttribute(k_agg_big_chunk<false, ull>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+                k_agg_big_chunk<false, ull><<<gb, 256, sm, st>>>(a, bigc, nbig, choff, goff, gkeys, gvals, glist, gcnt,
+                                                                g->opt_agg_chunk);
+            }
+            CKL();
+            vt.lap("agg: big insert");
+            k_agg_big_emit2<<<big, 256, 0, st>>>(a, bigc, nbig, choff, goff, gkeys, gvals, glist, gcnt, g->opt_agg_chunk);
+            CKL();
+        } else {
+            const int bpc = 32;
+            if (unit) k_agg_big_insert<true, unsigned><<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
+            else if (v32) k_agg_big_insert<false, unsigned><<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
+            else k_agg_big_insert<false, ull><<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
+            CKL();
+            vt.lap("agg: big insert");
+            k_agg_big_emit<<<big, 256, 0, st>>>(a, bigc, nbig, goff, gkeys, gvals, glist, gcnt, bpc);
+            CKL();
+        }
+        dfree(nch, st); dfree(choff, st);
         dfree(goff, st); dfree(gkeys, st); dfree(gvals, st); dfree(glist, st); dfree(gcnt, st);
         if (g->opt_verbose) fprintf(stderr, "[gala] big communities %d, table slots %lld\n", nbig, gtot);
     }
@@ -1970,6 +1996,14 @@ gala_status gala_set_option(gala_graph g, const char* key, int64_t value) {
     else if (k == "force_i128") g->opt_force_i128 = value != 0;
     else if (k == "force_wide") g->opt_force_wide = value != 0;
     else if (k == "singleton") g->opt_singleton = value != 0;
+    else if (k == "agg_big_chunk") g->opt_agg_big_chunk = value != 0;
+    else if (k == "agg_chunk") {   // test hook: entries per big-community chunk (1..AGG_CH)
+        if (value < 1 || value > AGG_CH) return set_err(GALA_E_INVALID, "agg_chunk must be in [1, 4096]");
+        g->opt_agg_chunk = (int)value;
+    } else if (k == "agg_scap") {  // test hook: block-path smem table cap (512..8192 slots)
+        if (value < 512 || value > 8192) return set_err(GALA_E_INVALID, "agg_scap must be in [512, 8192]");
+        g->opt_agg_scap = (int)value;
+    }
     else if (k == "ckey") g->opt_ckey = value != 0;
     else if (k == "concurrent") g->opt_concurrent = value != 0;
     else if (k == "verbose") g->opt_verbose = (int)value;

@@ -447,6 +447,97 @@ __device__ __forceinline__ long long seg_search(const long long* __restrict__ of
     return lo;
 }
 
+// Big communities (table larger than the block path's smem table): their
+// segments are cut into AGG_CH-entry chunks; chunk t of all big communities
+// (prefix choff; AGG_CH by default, option agg_chunk) is taken by any block of the machine, pre-combined in a
+// block-local smem table, and only its distinct (key, sum) pairs are inserted
+// into the community's global table (the global level of the hierarchy, as in
+// the phase-1 hub path).  A giant community therefore spreads over every SM
+// and its hot keys (the diagonal above all) see one global atomic per chunk.
+#define AGG_CH 4096
+#define AGG_CH_SLOTS (2 * AGG_CH)
+template <typename V>
+constexpr size_t agg_chunk_smem() { return (size_t)AGG_CH_SLOTS * (sizeof(V) + sizeof(int)) + (size_t)AGG_CH * sizeof(int); }
+
+__global__ void k_agg_big_nchunks(int nbig, const int32_t* __restrict__ bigc, const long long* __restrict__ ent,
+                                  long long* __restrict__ nch, int ch) {
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < nbig; i += gridDim.x * blockDim.x)
+        nch[i] = (ent[bigc[i]] + ch - 1) / ch;
+}
+
+template <bool UNIT, typename V>
+__global__ void __launch_bounds__(256) k_agg_big_chunk(AggArgs a, const int32_t* __restrict__ bigc, int nbig,
+                                                       const long long* __restrict__ choff,
+                                                       const long long* __restrict__ goff, int* __restrict__ gkeys,
+                                                       ull* __restrict__ gvals, int* __restrict__ glist,
+                                                       int* __restrict__ gcnt, int ch) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    V* vals = reinterpret_cast<V*>(smem_raw);
+    int* keys = reinterpret_cast<int*>(smem_raw + (size_t)AGG_CH_SLOTS * sizeof(V));
+    int* list = keys + AGG_CH_SLOTS;
+    __shared__ int s_cnt;
+    __shared__ V s_scr[8][32];
+    const int wib = threadIdx.x >> 5;
+    for (int j = threadIdx.x; j < AGG_CH_SLOTS; j += 256) { keys[j] = -1; vals[j] = 0; }
+    if (threadIdx.x == 0) s_cnt = 0;
+    __syncthreads();
+    const long long total = choff[nbig];
+    for (long long t = blockIdx.x; t < total; t += gridDim.x) {
+        const int bi = (int)seg_search(choff, 0, nbig - 1, t);
+        const long long c = bigc[bi];
+        const long long s1 = a.eoff[c + 1];
+        const long long lo = a.eoff[c] + (t - choff[bi]) * ch;
+        const long long hi = lo + ch < s1 ? lo + ch : s1;
+        agg_segment<UNIT, V, V>(a, lo, hi, threadIdx.x, 256, keys, vals, AGG_CH_SLOTS - 1, list, &s_cnt, s_scr[wib]);
+        __syncthreads();
+        const int m = s_cnt;
+        const long long off = goff[bi];
+        const unsigned mask = (unsigned)(goff[bi + 1] - off) - 1u;
+        for (int i = threadIdx.x; i < m; i += 256) {
+            const int slot = list[i];
+            const int key = keys[slot];
+            const V val = vals[slot];
+            keys[slot] = -1;
+            vals[slot] = 0;
+            agg_insert<ull>(key, (ull)val, gkeys + off, gvals + off, mask, glist + off / 2, &gcnt[bi]);
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) s_cnt = 0;
+        __syncthreads();
+    }
+}
+
+// distinct entries of the big communities to the start of their segments; list
+// index range of chunk t = [j*AGG_CH, (j+1)*AGG_CH) of its community (m <= entries)
+__global__ void __launch_bounds__(256) k_agg_big_emit2(AggArgs a, const int32_t* __restrict__ bigc, int nbig,
+                                                       const long long* __restrict__ choff,
+                                                       const long long* __restrict__ goff,
+                                                       const int* __restrict__ gkeys, const ull* __restrict__ gvals,
+                                                       const int* __restrict__ glist, const int* __restrict__ gcnt,
+                                                       int ch) {
+    const long long total = choff[nbig];
+    for (long long t = blockIdx.x; t < total; t += gridDim.x) {
+        const int bi = (int)seg_search(choff, 0, nbig - 1, t);
+        const long long c = bigc[bi];
+        const long long off = goff[bi];
+        const int m = gcnt[bi];
+        const long long j = t - choff[bi];
+        const int lo = (int)(j * ch);
+        const int hi = lo + ch < m ? lo + ch : m;
+        const long long o = a.eoff[c];
+        const int* list = glist + off / 2;
+        for (int i = lo + threadIdx.x; i < hi; i += 256) {
+            const int slot = list[i];
+            const int key = gkeys[off + slot];
+            const int64_t val = (int64_t)gvals[off + slot];
+            a.tkey[o + i] = key;
+            a.tval[o + i] = val;
+            if (key == (int)c) a.snew[c] = val;
+        }
+        if (j == 0 && threadIdx.x == 0) a.dn[c] = m;
+    }
+}
+
 // thread per coarse entry t: row c = segment of t in rp_new (bounded search per
 // 256-entry block), copy from the aggregated segment at eoff[c]
 __global__ void __launch_bounds__(256) k_compact(long long k, long long nnz_new, const long long* __restrict__ eoff,

@@ -124,13 +124,17 @@ def test_pruning_strategy_weighted_and_graph_mode(strategy):
     dict(delta_update=1, ckey=1),
     dict(concurrent=1),
     dict(hub(64), concurrent=1, delta_update=1),
+    dict(agg_scap=512, agg_chunk=64),                                        # phase 2: many multi-chunk big communities
+    dict(agg_scap=512, agg_chunk=1),
+    dict(agg_scap=512, agg_big_chunk=0),                                     # phase 2: per-community block split
 ])
 def test_dispatch_independence(opts):
     """P7: thresholds / table sizes / integer width / update strategy never change a label."""
     assert_parity(gg.make("rmat_small"), **opts)
 
 
-@pytest.mark.parametrize("opts", [dict(force_wide=1), dict(force_i128=1), hub(16), dict(hub(16), force_i128=1)])
+@pytest.mark.parametrize("opts", [dict(force_wide=1), dict(force_i128=1), hub(16), dict(hub(16), force_i128=1),
+                                  dict(agg_scap=512, agg_chunk=16)])
 def test_weighted_modes_parity(opts):
     """Weighted random graphs through every gain-arithmetic mode (DM_W64 / DM_W128)."""
     for seed in range(4):
@@ -232,3 +236,19 @@ def test_full_size_parity_skewed(name):
     """BASELINE configs[2] / configs[3] at full size: block and hub paths (rows up to 667k
     entries on coarse R-MAT levels), per-iteration N / moved / active / pruned and final labels."""
     assert_parity(gg.make(name), labels=False)
+
+
+@pytest.mark.gpu
+def test_nmi_vs_planted_partition():
+    """NEXT #4 (Table 4 style): NMI of the GPU result against the LFR planted partition, computed
+    on the device, equals the oracle's fp64 NMI of the same labels; and the planted partition
+    itself has NMI 1."""
+    from oracle.nmi import nmi
+    g = gg.make("lfr_small")
+    with gala.Graph.from_graph(g) as h:
+        h.run()
+        lab = h.communities()
+    got = gala.nmi_device(lab, g.truth)
+    assert got == pytest.approx(nmi(lab, g.truth), abs=1e-9)
+    assert gala.nmi_device(g.truth, g.truth) == pytest.approx(1.0, abs=1e-12)
+    assert 0.0 <= got <= 1.0 + 1e-12
