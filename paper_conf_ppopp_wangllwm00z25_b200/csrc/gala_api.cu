@@ -372,8 +372,14 @@ struct Work {
     }
 };
 
-#define BLOCK_BT 256
-#define BLOCK_E 4
+#ifndef GALA_BLOCK_BT
+#define GALA_BLOCK_BT 256
+#endif
+#ifndef GALA_BLOCK_E
+#define GALA_BLOCK_E 4
+#endif
+#define BLOCK_BT GALA_BLOCK_BT
+#define BLOCK_E GALA_BLOCK_E
 
 // ------------------------------------------------------------------ launch helpers
 // the per-entry neighbour-community array is used on level 0 of single-GPU runs
@@ -751,7 +757,20 @@ struct VTimer {
 template <typename V>
 static size_t agg_block_smem(int scap) { return (size_t)scap * (sizeof(V) + sizeof(int)) + (size_t)(scap / 2) * sizeof(int); }
 
-// warp / block aggregation launches with V = table value type (32-bit iff W < 2^32)
+// warp / block aggregation launches with V = table value type (32-bit iff W < 2^32).
+// The block path runs in three size classes so small tables get small blocks
+// (more communities in flight per SM): <= AGG_BA slots with 128 threads,
+// <= AGG_BB with 256, <= scap with 512.
+template <int BT, bool UNIT, typename V>
+static void agg_block_class(gala_graph_s* g, const AggArgs& a, int cap, const int32_t* bl, const int* nbl) {
+    const size_t sm = agg_block_smem<V>(cap);
+    CK(cudaFuncSetAttribute(k_agg_block<BT, UNIT, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+    int per = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_agg_block<BT, UNIT, V>, BT, sm));
+    k_agg_block<BT, UNIT, V><<<g->num_sms * std::max(per, 1), BT, sm, g->stream>>>(a, cap, bl, nbl);
+    CKL();
+}
+
 template <typename V>
 static void agg_launch_small(gala_graph_s* g, const AggArgs& a, bool unit, int scap, long long k, const int32_t* wl,
                              const int* nwl, const int32_t* bl, const int* nbl) {
@@ -760,14 +779,18 @@ static void agg_launch_small(gala_graph_s* g, const AggArgs& a, bool unit, int s
     if (unit) k_agg_warp<true, V><<<big, 256, 0, st>>>(a, wl, nwl);
     else k_agg_warp<false, V><<<big, 256, 0, st>>>(a, wl, nwl);
     CKL();
+    const int ca = std::min(scap, AGG_BA), cb = std::min(scap, AGG_BB);
     if (scap > AGG_WSLOTS) {
-        const size_t sm = agg_block_smem<V>(scap);
-        CK(cudaFuncSetAttribute(k_agg_block<AGG_BLOCK_BT, true, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
-        CK(cudaFuncSetAttribute(k_agg_block<AGG_BLOCK_BT, false, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
-        const int gb = (int)std::min<long long>(k, (long long)g->num_sms * 4);
-        if (unit) k_agg_block<AGG_BLOCK_BT, true, V><<<gb, AGG_BLOCK_BT, sm, st>>>(a, scap, bl, nbl);
-        else k_agg_block<AGG_BLOCK_BT, false, V><<<gb, AGG_BLOCK_BT, sm, st>>>(a, scap, bl, nbl);
-        CKL();
+        if (unit) agg_block_class<128, true, V>(g, a, ca, bl, nbl);
+        else agg_block_class<128, false, V>(g, a, ca, bl, nbl);
+    }
+    if (scap > AGG_BA) {
+        if (unit) agg_block_class<256, true, V>(g, a, cb, bl + k, nbl + 1);
+        else agg_block_class<256, false, V>(g, a, cb, bl + k, nbl + 1);
+    }
+    if (scap > AGG_BB) {
+        if (unit) agg_block_class<AGG_BLOCK_BT, true, V>(g, a, scap, bl + 2 * k, nbl + 2);
+        else agg_block_class<AGG_BLOCK_BT, false, V>(g, a, scap, bl + 2 * k, nbl + 2);
     }
 }
 
@@ -790,14 +813,14 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
     int32_t* bigc = dalloc<int32_t>(k, st);
     long long* bigcap = dalloc<long long>(k + 1, st);
     int32_t* wlist = dalloc<int32_t>(k, st);
-    int32_t* blist = dalloc<int32_t>(k, st);
-    int* nbig_dev = dalloc<int>(3, st);   // big, warp, block list lengths
+    int32_t* blist = dalloc<int32_t>(3 * k, st);   // block-path classes A, B, C
+    int* nbig_dev = dalloc<int>(5, st);   // big, warp, block A / B / C list lengths
     CK(cudaMemsetAsync(cnt, 0, sizeof(long long) * (k + 1), st));
     CK(cudaMemsetAsync(ent, 0, sizeof(long long) * (k + 1), st));
     CK(cudaMemsetAsync(dn, 0, sizeof(long long) * (k + 1), st));
     CK(cudaMemsetAsync(snew, 0, sizeof(int64_t) * k, st));
     CK(cudaMemsetAsync(dev_max, 0, sizeof(ull), st));
-    CK(cudaMemsetAsync(nbig_dev, 0, sizeof(int) * 3, st));
+    CK(cudaMemsetAsync(nbig_dev, 0, sizeof(int) * 5, st));
     k_comm_stats<<<grid_for(nrows, 256, big), 256, 0, st>>>((int)nrows, cur.rp, newid, ent);
     CKL();
     scan_excl(ent, eoff, k, st);
@@ -819,7 +842,7 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
     int scap = 512;
     while (scap < g->opt_agg_scap && scap < 2 * k) scap <<= 1;
     k_agg_classify<<<grid_for(k, 256, big), 256, 0, st>>>(k, ent, scap, dn, wlist, nbig_dev + 1, blist, nbig_dev + 2,
-                                                         bigc, bigcap, nbig_dev);
+                                                         bigc, bigcap, nbig_dev, k);
     CKL();
     AggArgs a;
     a.k = k; a.ent = ent; a.eoff = eoff; a.tkey = tkey; a.tval = tval; a.dn = dn; a.snew = snew;
@@ -896,9 +919,13 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
     nxt.row = dalloc<int32_t>(nxt.nnz, st);
     vt.lap("agg: scan+alloc");
     if (nxt.nnz > 0) {
-        k_compact<<<grid_for(nxt.nnz, 256, big * 4), 256, 0, st>>>(k, nxt.nnz, eoff, reinterpret_cast<long long*>(nxt.rp),
-                                                                    tkey, tval, nxt.col, nxt.w, nxt.row);
+        int32_t* tmap = dalloc<int32_t>((nxt.nnz + 255) / 256, st);
+        k_tile_map<<<grid_for(k, 256, big), 256, 0, st>>>(k, reinterpret_cast<long long*>(nxt.rp), nxt.nnz, tmap);
         CKL();
+        k_compact<<<grid_for((nxt.nnz + 255) / 256, 1, big * 2), 256, 0, st>>>(
+            k, nxt.nnz, eoff, reinterpret_cast<long long*>(nxt.rp), tmap, tkey, tval, nxt.col, nxt.w, nxt.row);
+        CKL();
+        dfree(tmap, st);
     }
     vt.lap("agg: scan+compact");
     g->kc_bytes[KC_PHASE2] += (double)nrows * (4 + 4 + 8 + 16 + 4 + 4) + (double)cur.nnz * (4 + 4 + (unit ? 0 : 8) + 12) +

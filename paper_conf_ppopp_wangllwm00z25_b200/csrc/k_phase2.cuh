@@ -410,17 +410,23 @@ __device__ __forceinline__ void list_append(bool on, int32_t val, int32_t* list,
     if (on) list[base + __popc(m & lanemask_lt())] = val;
 }
 
+// block-path size classes (table slots): <= AGG_BA (BT 128), <= AGG_BB (BT 256), <= scap (BT 512)
+#define AGG_BA 1024
+#define AGG_BB 4096
 __global__ void k_agg_classify(long long k, const long long* __restrict__ ent, int scap, long long* __restrict__ dn,
                                int32_t* __restrict__ wl, int* __restrict__ nwl, int32_t* __restrict__ bl,
                                int* __restrict__ nbl, int32_t* __restrict__ bigc, long long* __restrict__ bigcap,
-                               int* __restrict__ nbig) {
+                               int* __restrict__ nbig, long long kcap) {
+    // bl holds three lists of capacity kcap each (classes A, B, C), nbl their three counts
     const long long stride = (long long)gridDim.x * blockDim.x;
     for (long long c0 = (long long)blockIdx.x * blockDim.x; c0 < k; c0 += stride) {   // warp-uniform trips
         const long long c = c0 + threadIdx.x;
         const long long cap = c < k ? agg_cap(ent[c], k) : -1;
         if (cap == 0) dn[c] = 0;
         list_append(cap > 0 && cap <= AGG_WSLOTS, (int32_t)c, wl, nwl);
-        list_append(cap > AGG_WSLOTS && cap <= scap, (int32_t)c, bl, nbl);
+        list_append(cap > AGG_WSLOTS && cap <= AGG_BA && cap <= scap, (int32_t)c, bl, nbl);
+        list_append(cap > AGG_BA && cap <= AGG_BB && cap <= scap, (int32_t)c, bl + kcap, nbl + 1);
+        list_append(cap > AGG_BB && cap <= scap, (int32_t)c, bl + 2 * kcap, nbl + 2);
         const bool isbig = cap > scap;
         const unsigned m = __ballot_sync(FULLMASK, isbig);
         if (m) {
@@ -540,25 +546,35 @@ __global__ void __launch_bounds__(256) k_agg_big_emit2(AggArgs a, const int32_t*
 
 // thread per coarse entry t: row c = segment of t in rp_new (bounded search per
 // 256-entry block), copy from the aggregated segment at eoff[c]
+// tile map for k_compact: tmap[t] = the community whose coarse row holds entry 256*t
+__global__ void k_tile_map(long long k, const long long* __restrict__ rp_new, long long nnz_new,
+                           int32_t* __restrict__ tmap) {
+    for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c < k; c += (long long)gridDim.x * blockDim.x) {
+        const long long a = rp_new[c], b = rp_new[c + 1];
+        for (long long t = (a + 255) & ~255LL; t < b; t += 256) tmap[t >> 8] = (int32_t)c;
+    }
+}
+
+// thread per coarse entry t: row c = segment of t in rp_new, searched between the
+// communities of this tile's start and the next tile's start (tile map), copy
+// from the aggregated segment at eoff[c]
 __global__ void __launch_bounds__(256) k_compact(long long k, long long nnz_new, const long long* __restrict__ eoff,
-                                                 const long long* __restrict__ rp_new, const int* __restrict__ tkey,
-                                                 const int64_t* __restrict__ tval, int32_t* __restrict__ col_new,
-                                                 int64_t* __restrict__ w_new, int32_t* __restrict__ row_new) {
-    __shared__ long long s_lo, s_hi;
-    for (long long t0 = (long long)blockIdx.x * 256; t0 < nnz_new; t0 += (long long)gridDim.x * 256) {
-        const long long last = t0 + 255 < nnz_new ? t0 + 255 : nnz_new - 1;
-        if (threadIdx.x == 0) s_lo = seg_search(rp_new, 0, k - 1, t0);
-        if (threadIdx.x == 32) s_hi = seg_search(rp_new, 0, k - 1, last);
-        __syncthreads();
-        const long long t = t0 + threadIdx.x;
+                                                 const long long* __restrict__ rp_new, const int32_t* __restrict__ tmap,
+                                                 const int* __restrict__ tkey, const int64_t* __restrict__ tval,
+                                                 int32_t* __restrict__ col_new, int64_t* __restrict__ w_new,
+                                                 int32_t* __restrict__ row_new) {
+    const long long ntiles = (nnz_new + 255) >> 8;
+    for (long long tb = blockIdx.x; tb < ntiles; tb += gridDim.x) {
+        const long long lo = tmap[tb];
+        const long long hi = tb + 1 < ntiles ? tmap[tb + 1] : k - 1;
+        const long long t = (tb << 8) + threadIdx.x;
         if (t < nnz_new) {
-            const long long c = seg_search(rp_new, s_lo, s_hi, t);
+            const long long c = seg_search(rp_new, lo, hi, t);
             const long long src = eoff[c] + (t - rp_new[c]);
             col_new[t] = tkey[src];
             w_new[t] = tval[src];
             row_new[t] = (int32_t)c;
         }
-        __syncthreads();
     }
 }
 
