@@ -373,10 +373,10 @@ struct Work {
 };
 
 #ifndef GALA_BLOCK_BT
-#define GALA_BLOCK_BT 256
+#define GALA_BLOCK_BT 512
 #endif
 #ifndef GALA_BLOCK_E
-#define GALA_BLOCK_E 4
+#define GALA_BLOCK_E 2
 #endif
 #define BLOCK_BT GALA_BLOCK_BT
 #define BLOCK_E GALA_BLOCK_E
