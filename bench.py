@@ -37,6 +37,7 @@ WORKLOADS = {
     "karate": "Zachary karate club (BASELINE.json configs[0])",
     "rmat_lj": "R-MAT LiveJournal-shaped 4.8M / 69M (BASELINE.json configs[2])",
     "orkut": "Orkut-shaped LFR 3.1M / 117M (BASELINE.json configs[3])",
+    "friendster_q": "Friendster-shaped LFR at 1/4 scale, 16.4M / ~451M (BASELINE.json configs[4] shape on 1 GPU)",
     "lfr_small": "LFR 20k (test size)",
 }
 METRIC = "local-move GTEPS and end-to-end Louvain seconds at 1/2/4/8 B200; modularity Q"

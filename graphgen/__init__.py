@@ -230,6 +230,9 @@ CONFIGS = {
     "orkut": dict(desc="LFR-style n=3,072,441, <k>=76.3, kmax=33,313, tau1=2.0, mu=0.35, seed 3, "
                        "target m=117.2M"),
     "friendster": dict(desc="LFR-style n=65,608,366, <k>=55.06, kmax=5,214, tau1=2.5, mu=0.37, seed 4"),
+    # the Friendster shape at 1/4 of its vertices (same degree law / mixing): the largest FR-shaped
+    # graph one GPU-box host generates comfortably; C + Sigma_tot (197 MB) exceed the 126 MB L2
+    "friendster_q": dict(desc="LFR-style n=16,402,092, <k>=55.06, kmax=5,214, tau1=2.5, mu=0.37, seed 4"),
     # scaled-down shapes for tests (same recipe, smaller n)
     "lfr_small": dict(desc="LFR n=20,000, <k>=20, kmax=200, mu=0.3, seed 11"),
     "lfr_mid": dict(desc="LFR n=200,000, <k>=40, kmax=1000, mu=0.3, seed 12"),
@@ -253,6 +256,8 @@ def make(name: str) -> CSR:
         return lfr(3_072_441, 76.3, 33_313, 0.35, tau1=2.0, cmin=50, cmax=20000, seed=3, name=name)
     if name == "friendster":
         return lfr(65_608_366, 55.06, 5_214, 0.37, seed=4, name=name)
+    if name == "friendster_q":
+        return lfr(16_402_092, 55.06, 5_214, 0.37, seed=4, name=name)
     if name == "lfr_small":
         return lfr(20_000, 20.0, 200, 0.3, cmin=20, cmax=500, seed=11, name=name)
     if name == "lfr_mid":

@@ -35,6 +35,7 @@
 #ifndef GALA_H
 #define GALA_H
 
+#include <stddef.h>
 #include <stdint.h>
 
 #ifdef __cplusplus
@@ -167,8 +168,27 @@ void gala_graph_free(gala_graph g);
  *   "log_cap"        device iteration-log capacity (default 4096)
  *   "sync_mode"      multi-GPU label exchange: 0 adaptive (default), 1 dense, 2 sparse
  *   "verbose"        0/1   host-side phase timings on stderr
+ *   "agg_big_chunk"  0/1   phase 2: big communities in 4096-entry chunks over the whole GPU with a
+ *                          block-smem pre-combine (default 1); 0: 32 blocks per big community
+ *   "agg_chunk"      [1, 4096] entries per big-community chunk (test hook, default 4096)
+ *   "agg_scap"       [512, 8192] largest phase-2 shared-memory table; communities needing more
+ *                          slots take the big (global-table) path (test hook, default 8192)
  */
 gala_status gala_set_option(gala_graph g, const char* key, int64_t value);
+
+/*
+ * gala_set_allocator — device-memory hook (SURVEY.md §8(b) "allocator hook").  Process-wide;
+ * applies to every block any handle allocates AFTER the call (a block is always returned to the
+ * allocator that made it).  alloc(bytes, device, stream, ctx) returns a device pointer valid for
+ * work ordered on `stream` (NULL -> GALA_E_NOMEM from the call that needed it);
+ * free(ptr, bytes, device, stream, ctx) may recycle it for later work on that stream.
+ * Both NULL restores the default (a per-handle stream-ordered cudaMemPool); exactly one NULL is
+ * GALA_E_INVALID.  The Python binding routes it to torch.cuda's caching allocator
+ * (gala.use_torch_allocator()).  Allocation happens per level, so callback cost is immaterial.
+ */
+typedef void* (*gala_alloc_fn)(size_t bytes, int device, uintptr_t stream, void* ctx);
+typedef void (*gala_free_fn)(void* ptr, size_t bytes, int device, uintptr_t stream, void* ctx);
+gala_status gala_set_allocator(gala_alloc_fn alloc_fn, gala_free_fn free_fn, void* ctx);
 
 /*
  * gala_get_stats — JSON object with per-level and per-iteration statistics

@@ -69,6 +69,7 @@ def lib():
         "gala_graph_from_csr_dist": (st, [p, ctypes.c_int, ctypes.c_int, ctypes.c_int, i64, i64, i64, p, p, p,
                                           ctypes.c_size_t, pp]),
         "gala_partition_ranges": (st, [i64, p, ctypes.c_int, p]),
+        "gala_set_allocator": (st, [p, p, p]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -96,6 +97,50 @@ def _np_ptr(a):
 
 def _i128(hi: int, lo: int) -> int:
     return (int(hi) << 64) | (int(lo) & 0xFFFFFFFFFFFFFFFF)
+
+
+ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int, ctypes.c_size_t, ctypes.c_void_p)
+FREE_FN = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int, ctypes.c_size_t, ctypes.c_void_p)
+_ALLOC_HOOK = None   # keeps the ctypes callbacks alive while installed
+
+
+def set_allocator(alloc=None, free=None):
+    """Install a device allocator for every later library allocation (include/gala.h
+    gala_set_allocator): alloc(bytes, device, stream) -> int pointer, free(ptr, bytes, device,
+    stream).  set_allocator() restores the library's own stream-ordered pool."""
+    global _ALLOC_HOOK
+    if alloc is None and free is None:
+        _check(lib().gala_set_allocator(None, None, None))
+        _ALLOC_HOOK = None
+        return
+
+    def _a(nbytes, device, stream, ctx):
+        try:
+            return int(alloc(int(nbytes), int(device), int(stream)))
+        except Exception:   # the library reports GALA_E_NOMEM
+            return None
+
+    def _f(ptr, nbytes, device, stream, ctx):
+        free(int(ptr), int(nbytes), int(device), int(stream))
+
+    hook = (ALLOC_FN(_a), FREE_FN(_f))
+    _check(lib().gala_set_allocator(ctypes.cast(hook[0], ctypes.c_void_p), ctypes.cast(hook[1], ctypes.c_void_p),
+                                    None))
+    _ALLOC_HOOK = hook
+
+
+def use_torch_allocator():
+    """Route the library's device memory through torch.cuda's caching allocator
+    (gala_set_allocator bound to caching_allocator_alloc / _delete)."""
+    import torch
+
+    def alloc(nbytes, device, stream):
+        return torch.cuda.caching_allocator_alloc(nbytes, device, stream)
+
+    def free(ptr, nbytes, device, stream):
+        torch.cuda.caching_allocator_delete(ptr)
+
+    set_allocator(alloc, free)
 
 
 def version() -> str:

@@ -18,6 +18,7 @@
 #include <cstring>
 #include <string>
 #include <map>
+#include <mutex>
 #include <unordered_map>
 #include <vector>
 
@@ -185,10 +186,42 @@ struct Fork {
 // remap physical pages to new virtual ranges (tens of ms per GB on big levels).
 // Every user of a handle's memory is ordered on the handle's stream, which makes
 // reuse without events safe.  The active cache is set per API call (PoolScope).
+// User allocator hook (gala_set_allocator): when set, every device block the
+// library allocates from then on comes from alloc_fn and goes back through free_fn (Python routes
+// it to torch's caching allocator).  Each block remembers which allocator made it.
+struct UserAlloc {
+    gala_alloc_fn alloc = nullptr;
+    gala_free_fn free = nullptr;
+    void* ctx = nullptr;
+};
+static std::mutex g_ualloc_mu;
+static UserAlloc g_ualloc;
+static UserAlloc current_ualloc() {
+    std::lock_guard<std::mutex> lk(g_ualloc_mu);
+    return g_ualloc;
+}
+static int current_device() {
+    int d = 0;
+    cudaGetDevice(&d);
+    return d;
+}
+struct BlockInfo {
+    size_t bytes;
+    UserAlloc ua;   // ua.alloc == nullptr: the stream-ordered pool / cudaMallocAsync
+};
+static void* user_alloc(const UserAlloc& ua, size_t bytes, cudaStream_t st) {
+    void* p = ua.alloc(bytes, current_device(), (uintptr_t)st, ua.ctx);
+    if (!p) {
+        set_err(GALA_E_NOMEM, "user allocator returned NULL for %zu bytes", bytes);
+        throw GalaError{GALA_E_NOMEM};
+    }
+    return p;
+}
+
 struct DevCache {
     cudaMemPool_t pool = nullptr;
     std::multimap<size_t, void*> freeb;        // cached free blocks by size
-    std::unordered_map<void*, size_t> sz;      // every block this cache handed out
+    std::unordered_map<void*, BlockInfo> sz;   // every block this cache handed out
     static size_t round(size_t b) {
         if (b <= 4096) return (b + 255) & ~(size_t)255;
         if (b < ((size_t)2 << 20)) { size_t r = 8192; while (r < b) r <<= 1; return r; }
@@ -196,33 +229,47 @@ struct DevCache {
     }
     void* get(size_t bytes, cudaStream_t st) {
         const size_t r = round(bytes);
+        const UserAlloc ua = current_ualloc();
         auto it = freeb.lower_bound(r);
-        if (it != freeb.end() && it->first <= r + r / 4) {
-            void* p = it->second;
-            freeb.erase(it);
-            return p;
-        }
+        // reuse only blocks of the allocator now in effect
+        for (; it != freeb.end() && it->first <= r + r / 4; ++it)
+            if (sz[it->second].ua.alloc == ua.alloc && sz[it->second].ua.ctx == ua.ctx) {
+                void* p = it->second;
+                freeb.erase(it);
+                return p;
+            }
         void* p = nullptr;
-        cudaError_t e = cudaMallocFromPoolAsync(&p, r, pool, st);
-        if (e == cudaErrorMemoryAllocation) {   // give cached blocks back and retry once
-            cudaGetLastError();
-            trim(st);
-            cudaStreamSynchronize(st);
-            cudaMemPoolTrimTo(pool, 0);
-            e = cudaMallocFromPoolAsync(&p, r, pool, st);
+        if (ua.alloc) {
+            p = user_alloc(ua, r, st);
+        } else {
+            cudaError_t e = cudaMallocFromPoolAsync(&p, r, pool, st);
+            if (e == cudaErrorMemoryAllocation) {   // give cached blocks back and retry once
+                cudaGetLastError();
+                trim(st);
+                cudaStreamSynchronize(st);
+                cudaMemPoolTrimTo(pool, 0);
+                e = cudaMallocFromPoolAsync(&p, r, pool, st);
+            }
+            CK(e);
         }
-        CK(e);
-        sz[p] = r;
+        sz[p] = BlockInfo{r, ua};
         return p;
     }
     bool put(void* p) {
         auto it = sz.find(p);
         if (it == sz.end()) return false;
-        freeb.emplace(it->second, p);
+        freeb.emplace(it->second.bytes, p);
         return true;
     }
+    static void release(void* p, const BlockInfo& b, cudaStream_t st) {
+        if (b.ua.free) b.ua.free(p, b.bytes, current_device(), (uintptr_t)st, b.ua.ctx);
+        else cudaFreeAsync(p, st);
+    }
     void trim(cudaStream_t st) {
-        for (auto& kv : freeb) { cudaFreeAsync(kv.second, st); sz.erase(kv.second); }
+        for (auto& kv : freeb) {
+            release(kv.second, sz[kv.second], st);
+            sz.erase(kv.second);
+        }
         freeb.clear();
     }
 };
@@ -232,17 +279,37 @@ struct PoolScope {
     explicit PoolScope(DevCache* c) : prev(g_cache) { g_cache = c; }
     ~PoolScope() { g_cache = prev; }
 };
+// blocks allocated outside any handle's cache by the user allocator (size + allocator kept for free)
+static std::mutex g_loose_mu;
+static std::unordered_map<void*, BlockInfo> g_loose;
 template <typename T>
 static T* dalloc(size_t count, cudaStream_t st) {
     if (count == 0) count = 1;
     if (g_cache) return static_cast<T*>(g_cache->get(count * sizeof(T), st));
     void* p = nullptr;
+    const UserAlloc ua = current_ualloc();
+    if (ua.alloc) {
+        p = user_alloc(ua, count * sizeof(T), st);
+        std::lock_guard<std::mutex> lk(g_loose_mu);
+        g_loose[p] = BlockInfo{count * sizeof(T), ua};
+        return static_cast<T*>(p);
+    }
     CK(cudaMallocAsync(&p, count * sizeof(T), st));
     return static_cast<T*>(p);
 }
 template <typename T>
 static void dfree(T*& p, cudaStream_t st) {
-    if (p && !(g_cache && g_cache->put(p))) cudaFreeAsync(p, st);
+    if (p && !(g_cache && g_cache->put(p))) {
+        BlockInfo b{0, UserAlloc{}};
+        bool loose = false;
+        {
+            std::lock_guard<std::mutex> lk(g_loose_mu);
+            auto it = g_loose.find((void*)p);
+            if (it != g_loose.end()) { b = it->second; g_loose.erase(it); loose = true; }
+        }
+        if (loose) DevCache::release((void*)p, b, st);
+        else cudaFreeAsync(p, st);
+    }
     p = nullptr;
 }
 
@@ -1787,6 +1854,16 @@ static void finish_graph(gala_graph_s* g) {
     return GALA_OK;
 
 extern "C" {
+
+gala_status gala_set_allocator(gala_alloc_fn alloc_fn, gala_free_fn free_fn, void* ctx) {
+    if ((alloc_fn == nullptr) != (free_fn == nullptr))
+        return set_err(GALA_E_INVALID, "gala_set_allocator: alloc and free must both be set or both NULL");
+    std::lock_guard<std::mutex> lk(g_ualloc_mu);
+    g_ualloc.alloc = alloc_fn;
+    g_ualloc.free = free_fn;
+    g_ualloc.ctx = alloc_fn ? ctx : nullptr;
+    return GALA_OK;
+}
 
 const char* gala_version(void) { return GALA_VERSION; }
 const char* gala_last_error(void) { return g_err.c_str(); }
