@@ -107,6 +107,7 @@ struct gala_graph_s {
     int opt_prune = 1, opt_prune_check = 0, opt_trace = 0, opt_check = 0, opt_timing = 0, opt_max_iters = 0;
     int opt_delta = 2, opt_force_i128 = 0, opt_force_wide = 0, opt_cuda_graph = 1, opt_log_cap = 4096, opt_singleton = 1, opt_verbose = 0, opt_agg_big_chunk = 1,
         opt_agg_chunk = AGG_CH, opt_agg_scap = 8192;
+    long long opt_agg_big_ent = 1LL << 62;
     bool rows_distinct0 = false;   // level-0 rows strictly increasing (no duplicate entries)
     int32_t* rev0 = nullptr;       // level-0 reverse-entry index (enables the per-entry community array)
     int opt_ckey = 0;
@@ -909,7 +910,7 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
     int scap = 512;
     while (scap < g->opt_agg_scap && scap < 2 * k) scap <<= 1;
     k_agg_classify<<<grid_for(k, 256, big), 256, 0, st>>>(k, ent, scap, dn, wlist, nbig_dev + 1, blist, nbig_dev + 2,
-                                                         bigc, bigcap, nbig_dev, k);
+                                                         bigc, bigcap, nbig_dev, k, g->opt_agg_big_ent);
     CKL();
     AggArgs a;
     a.k = k; a.ent = ent; a.eoff = eoff; a.tkey = tkey; a.tval = tval; a.dn = dn; a.snew = snew;
@@ -2104,6 +2105,9 @@ gala_status gala_set_option(gala_graph g, const char* key, int64_t value) {
     else if (k == "agg_chunk") {   // test hook: entries per big-community chunk (1..AGG_CH)
         if (value < 1 || value > AGG_CH) return set_err(GALA_E_INVALID, "agg_chunk must be in [1, 4096]");
         g->opt_agg_chunk = (int)value;
+    } else if (k == "agg_big_ent") {   // phase 2: communities with more entries take the chunked path
+        if (value < 1) return set_err(GALA_E_INVALID, "agg_big_ent must be >= 1");
+        g->opt_agg_big_ent = value;
     } else if (k == "agg_scap") {  // test hook: block-path smem table cap (512..8192 slots)
         if (value < 512 || value > 8192) return set_err(GALA_E_INVALID, "agg_scap must be in [512, 8192]");
         g->opt_agg_scap = (int)value;

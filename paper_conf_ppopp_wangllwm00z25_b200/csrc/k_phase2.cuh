@@ -419,18 +419,21 @@ __device__ __forceinline__ void list_append(bool on, int32_t val, int32_t* list,
 __global__ void k_agg_classify(long long k, const long long* __restrict__ ent, int scap, long long* __restrict__ dn,
                                int32_t* __restrict__ wl, int* __restrict__ nwl, int32_t* __restrict__ bl,
                                int* __restrict__ nbl, int32_t* __restrict__ bigc, long long* __restrict__ bigcap,
-                               int* __restrict__ nbig, long long kcap) {
-    // bl holds three lists of capacity kcap each (classes A, B, C), nbl their three counts
+                               int* __restrict__ nbig, long long kcap, long long big_ent) {
+    // bl holds three lists of capacity kcap each (classes A, B, C), nbl their three counts;
+    // communities with more than big_ent entries take the chunked big path even when their
+    // table fits in shared memory (one block per community would serialise them)
     const long long stride = (long long)gridDim.x * blockDim.x;
     for (long long c0 = (long long)blockIdx.x * blockDim.x; c0 < k; c0 += stride) {   // warp-uniform trips
         const long long c = c0 + threadIdx.x;
-        const long long cap = c < k ? agg_cap(ent[c], k) : -1;
+        const long long e = c < k ? ent[c] : 0;
+        const long long cap = c < k ? agg_cap(e, k) : -1;
         if (cap == 0) dn[c] = 0;
-        list_append(cap > 0 && cap <= AGG_WSLOTS, (int32_t)c, wl, nwl);
-        list_append(cap > AGG_WSLOTS && cap <= AGG_BA && cap <= scap, (int32_t)c, bl, nbl);
-        list_append(cap > AGG_BA && cap <= AGG_BB && cap <= scap, (int32_t)c, bl + kcap, nbl + 1);
-        list_append(cap > AGG_BB && cap <= scap, (int32_t)c, bl + 2 * kcap, nbl + 2);
-        const bool isbig = cap > scap;
+        const bool isbig = cap > scap || e > big_ent;
+        list_append(!isbig && cap > 0 && cap <= AGG_WSLOTS, (int32_t)c, wl, nwl);
+        list_append(!isbig && cap > AGG_WSLOTS && cap <= AGG_BA && cap <= scap, (int32_t)c, bl, nbl);
+        list_append(!isbig && cap > AGG_BA && cap <= AGG_BB && cap <= scap, (int32_t)c, bl + kcap, nbl + 1);
+        list_append(!isbig && cap > AGG_BB && cap <= scap, (int32_t)c, bl + 2 * kcap, nbl + 2);
         const unsigned m = __ballot_sync(FULLMASK, isbig);
         if (m) {
             const int lane = lane_id(), lead = __ffs(m) - 1;

@@ -129,6 +129,7 @@ def test_pruning_strategy_weighted_and_graph_mode(strategy):
     dict(agg_scap=512, agg_chunk=64),                                        # phase 2: many multi-chunk big communities
     dict(agg_scap=512, agg_chunk=1),
     dict(agg_scap=512, agg_big_chunk=0),                                     # phase 2: per-community block split
+    dict(agg_big_ent=64, agg_chunk=32),                                      # phase 2: entry-count big path
 ])
 def test_dispatch_independence(opts):
     """P7: thresholds / table sizes / integer width / update strategy never change a label."""
