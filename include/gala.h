@@ -128,7 +128,11 @@ gala_status gala_modularity(gala_graph g, double* q);
 gala_status gala_modularity_numerator(gala_graph g, int64_t* n_hi, uint64_t* n_lo, int64_t* W,
                                       int64_t* p, int64_t* q);
 
-/* Free the handle and all its device memory.  NULL is a no-op. */
+/* Free the handle and all its device memory.  NULL is a no-op.  The handle's (synchronised,
+ * idle) memory pool of the default allocator is parked per device and adopted by the next
+ * handle created on that device, so create/run/free cycles do not map fresh pages every time;
+ * at most one pool per device is kept (multi-GPU handles and user-allocator blocks are always
+ * released). */
 void gala_graph_free(gala_graph g);
 
 /*

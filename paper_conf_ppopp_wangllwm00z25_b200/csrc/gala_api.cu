@@ -275,6 +275,16 @@ struct DevCache {
     }
 };
 static thread_local DevCache* g_cache = nullptr;
+// One retired cache per device: gala_graph_free parks its (idle, synchronised) pool and free
+// blocks here and the next handle on that device adopts them, so repeated
+// create/run/free cycles (e2e) do not map fresh physical pages each time.
+static std::mutex g_stash_mu;
+static std::map<int, DevCache*> g_stash;
+static bool cache_has_user_blocks(const DevCache* c) {
+    for (auto& kv : c->sz)
+        if (kv.second.ua.alloc) return true;
+    return false;
+}
 struct PoolScope {
     DevCache* prev;
     explicit PoolScope(DevCache* c) : prev(g_cache) { g_cache = c; }
@@ -1765,10 +1775,17 @@ static void init_graph_common(gala_graph_s* g, int64_t n, int device, uintptr_t 
     props.allocType = cudaMemAllocationTypePinned;
     props.location.type = cudaMemLocationTypeDevice;
     props.location.id = device;
-    g->cache = new DevCache();
-    CK(cudaMemPoolCreate(&g->cache->pool, &props));
-    uint64_t keep = UINT64_MAX;
-    CK(cudaMemPoolSetAttribute(g->cache->pool, cudaMemPoolAttrReleaseThreshold, &keep));
+    {
+        std::lock_guard<std::mutex> lk(g_stash_mu);
+        auto it = g_stash.find(device);
+        if (it != g_stash.end()) { g->cache = it->second; g_stash.erase(it); }
+    }
+    if (!g->cache) {
+        g->cache = new DevCache();
+        CK(cudaMemPoolCreate(&g->cache->pool, &props));
+        uint64_t keep = UINT64_MAX;
+        CK(cudaMemPoolSetAttribute(g->cache->pool, cudaMemPoolAttrReleaseThreshold, &keep));
+    }
     g_cache = g->cache;
 }
 
@@ -2054,7 +2071,9 @@ gala_status gala_modularity(gala_graph g, double* q) {
 void gala_graph_free(gala_graph g) {
     if (!g) return;
     cudaSetDevice(g->device);
+    DevCache* const mine = g->cache;
     PoolScope pool_scope(g->cache);
+    const bool dist = g->di != nullptr;
     if (g->di) { delete g->di; g->di = nullptr; }   // communicators are cached (comm_for)
     cudaStream_t st = g->stream;
     if (g->wk) { g->wk->release(); delete g->wk; g->wk = nullptr; }
@@ -2067,6 +2086,16 @@ void gala_graph_free(gala_graph g) {
         dfree(g->d0, st);
         dfree(g->s0, st);
         dfree(g->lab, st);
+        cudaStreamSynchronize(st);
+        // park the idle cache for the next handle on this device (not when it holds blocks of a
+        // user allocator: those go back to their owner now)
+        if (g->cache && !dist && !cache_has_user_blocks(g->cache) && cudaGetLastError() == cudaSuccess) {
+            std::lock_guard<std::mutex> lk(g_stash_mu);
+            if (!g_stash.count(g->device)) {
+                g_stash[g->device] = g->cache;
+                g->cache = nullptr;
+            }
+        }
         if (g->cache) g->cache->trim(st);
         cudaStreamSynchronize(st);
         if (g->own_stream) cudaStreamDestroy(st);
@@ -2080,7 +2109,7 @@ void gala_graph_free(gala_graph g) {
         if (g->cache->pool) cudaMemPoolDestroy(g->cache->pool);
         delete g->cache;
     }
-    g_cache = pool_scope.prev == g->cache ? nullptr : pool_scope.prev;
+    g_cache = pool_scope.prev == mine ? nullptr : pool_scope.prev;
     pool_scope.prev = g_cache;
     delete g;
 }
