@@ -204,6 +204,9 @@ __device__ __forceinline__ unsigned decide_sub_bin(QView queue, int bin, const D
 #ifndef GALA_SMALL_MINB
 #define GALA_SMALL_MINB 4   // <= 64 registers: 32 warps per SM (measured -30% vs 72-80 regs)
 #endif
+#ifndef GALA_WARP_PREFETCH
+#define GALA_WARP_PREFETCH 1   // warp128: next vertex's row loaded during this one's evaluation
+#endif
 #ifndef GALA_WARP_MINB
 #define GALA_WARP_MINB 4   // <= 64 registers (an explicit min of 1 lets ptxas take 80)
 #endif
@@ -347,8 +350,23 @@ __global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB, MAXDEG <= 1
     const long long nwarps = (long long)gridDim.x * SM::WPB;
     unsigned my_k = 0;
     long long base_i = ((long long)blockIdx.x * SM::WPB + wib) * NG;
+    // PF: the row entries of a group's NEXT vertex are loaded while the current one is
+    // evaluated (every row here fits one round: deg <= MAXDEG = GW * CH)
+    constexpr bool PF = GALA_WARP_PREFETCH && MAXDEG <= 128 && MAXDEG == GW * CH;
+    const int* __restrict__ rsrc = a.ckey ? a.ckey : a.col;
+    int pu[CH];
+    VT pw[CH];
     QRec qn;
     if (base_i + gid < count) qn = queue[base_i + gid];
+    if (PF) {
+        const bool ok = base_i + gid < count;
+#pragma unroll
+        for (int k = 0; k < CH; ++k) {
+            const int j = gl + GW * k;
+            pu[k] = ok && j < qn.deg ? rsrc[qn.beg + j] : -1;
+            pw[k] = (ok && j < qn.deg && !UNIT) ? (VT)a.w[qn.beg + j] : (VT)1;
+        }
+    }
     for (; base_i < count; base_i += nwarps * NG) {            // warp-uniform
         const bool valid = base_i + gid < count;
         const QRec q = qn;
@@ -365,11 +383,16 @@ __global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB, MAXDEG <= 1
             int uu[CH];
             VT ww[CH];
             int cc[CH];
+            if (PF) {
 #pragma unroll
-            for (int k = 0; k < CH; ++k) {
-                int j = r0 + gl + GW * k;
-                uu[k] = j < deg ? (a.ckey ? a.ckey[beg + j] : a.col[beg + j]) : -1;
-                ww[k] = (j < deg && !UNIT) ? (VT)a.w[beg + j] : (VT)1;
+                for (int k = 0; k < CH; ++k) { uu[k] = pu[k]; ww[k] = pw[k]; }
+            } else {
+#pragma unroll
+                for (int k = 0; k < CH; ++k) {
+                    int j = r0 + gl + GW * k;
+                    uu[k] = j < deg ? rsrc[beg + j] : -1;
+                    ww[k] = (j < deg && !UNIT) ? (VT)a.w[beg + j] : (VT)1;
+                }
             }
             if (a.ckey) {
 #pragma unroll
@@ -399,6 +422,15 @@ __global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB, MAXDEG <= 1
                                ? ht_insert4<VT, true>(cc[k], sum, keys, vals, WMASK, hash_slot(cc[k], WMASK), WCAP, &fresh)
                                : ht_insert<VT>(cc[k], sum, keys, vals, WMASK, hash_slot(cc[k], WMASK), WCAP, &fresh);
                 append_fresh<short>(fresh, slot, gmask, cnt, list);
+            }
+        }
+        if (PF) {   // next vertex's row: in flight during this vertex's evaluation
+            const bool ok = inext < count;
+#pragma unroll
+            for (int k = 0; k < CH; ++k) {
+                const int j = gl + GW * k;
+                pu[k] = ok && j < qn.deg ? rsrc[qn.beg + j] : -1;
+                pw[k] = (ok && j < qn.deg && !UNIT) ? (VT)a.w[qn.beg + j] : (VT)1;
             }
         }
         __syncwarp();
