@@ -404,16 +404,11 @@ __global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB, MAXDEG <= 1
 #pragma unroll
             for (int k = 0; k < CH; ++k)
                 if (cc[k] == cv) { own += (long long)ww[k]; cc[k] = -1; }
-            // combine equal communities of each chunk first (one insert per community); all
-            // matches are issued before any insert so their latencies overlap
-            unsigned pk[CH];
-#pragma unroll
-            for (int k = 0; k < CH; ++k)
-                pk[k] = r0 + GW * k < dmax ? __match_any_sync(FULLMASK, cc[k] >= 0 ? cc[k] : -1 - lane) & gmask : 0u;
 #pragma unroll
             for (int k = 0; k < CH; ++k) {
                 if (r0 + GW * k >= dmax) break;                // warp-uniform
-                const unsigned peers = pk[k];
+                // combine equal communities of this chunk first (one insert per community)
+                const unsigned peers = __match_any_sync(FULLMASK, cc[k] >= 0 ? cc[k] : -1 - lane) & gmask;
                 const VT sum = UNIT ? (VT)__popc(peers) : group_sum(peers, cc[k] >= 0 ? ww[k] : (VT)0, scratch);
                 bool fresh = false;
                 int slot = -1;
@@ -557,12 +552,9 @@ __global__ void __launch_bounds__(BT) k_decide_block(QView queue, int bin, Decid
 #pragma unroll
             for (int k = 0; k < E; ++k)
                 if (cc[k] == cv) { own += (long long)ww[k]; cc[k] = -1; }
-            unsigned pk[E];   // all matches first: their latencies overlap
-#pragma unroll
-            for (int k = 0; k < E; ++k) pk[k] = __match_any_sync(FULLMASK, cc[k] >= 0 ? cc[k] : -1 - lane);
 #pragma unroll
             for (int k = 0; k < E; ++k) {
-                const unsigned peers = pk[k];
+                const unsigned peers = __match_any_sync(FULLMASK, cc[k] >= 0 ? cc[k] : -1 - lane);
                 const VT sum = UNIT ? (VT)__popc(peers) : group_sum(peers, cc[k] >= 0 ? ww[k] : (VT)0, s_scr[wib]);
                 bool gfresh = false;
                 int gslot = -1;
@@ -880,12 +872,9 @@ __global__ void __launch_bounds__(HUB_BT) k_hub_agg(QView queue, DecideArgs a, H
 #pragma unroll
         for (int k = 0; k < E; ++k)
             if (cc[k] == cv) { own += (long long)ww[k]; cc[k] = -1; }
-        unsigned pk[E];   // all matches first: their latencies overlap
-#pragma unroll
-        for (int k = 0; k < E; ++k) pk[k] = __match_any_sync(FULLMASK, cc[k] >= 0 ? cc[k] : -1 - lane);
 #pragma unroll
         for (int k = 0; k < E; ++k) {
-            const unsigned peers = pk[k];
+            const unsigned peers = __match_any_sync(FULLMASK, cc[k] >= 0 ? cc[k] : -1 - lane);
             const VT sum = UNIT ? (VT)__popc(peers) : group_sum(peers, cc[k] >= 0 ? ww[k] : (VT)0, s_scr[wib]);
             bool fresh = false;
             int slot = -1;

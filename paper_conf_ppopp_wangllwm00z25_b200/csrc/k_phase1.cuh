@@ -116,7 +116,7 @@ struct BinThresholds {
 #define PB_IPT 4
 
 #ifndef GALA_PRUNE_MINB
-#define GALA_PRUNE_MINB 1
+#define GALA_PRUNE_MINB 4   // <= 64 registers: one wave of 1024-vertex tiles (A/B: lfr1m 0.76 -> 0.64 ms)
 #endif
 template <typename ST>
 __global__ void __launch_bounds__(PB_BT, GALA_PRUNE_MINB) k_prune_bin(int vlo, int n, const int64_t* __restrict__ rp,

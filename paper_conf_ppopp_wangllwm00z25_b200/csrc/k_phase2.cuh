@@ -266,13 +266,10 @@ __device__ __forceinline__ void agg_segment(const AggArgs& a, long long s0, long
             kk[t] = j < s1 ? a.tkey[j] : -1;
             ww[t] = (j < s1 && !UNIT) ? (SV)a.tval[j] : (SV)1;
         }
-        unsigned pk[4];   // all matches first: their latencies overlap
-#pragma unroll
-        for (int t = 0; t < 4; ++t) pk[t] = r0 + 32 * t < s1 ? __match_any_sync(FULLMASK, kk[t] >= 0 ? kk[t] : -1 - lane) : 0u;
 #pragma unroll
         for (int t = 0; t < 4; ++t) {
             if (r0 + 32 * t >= s1) break;
-            const unsigned peers = pk[t];
+            const unsigned peers = __match_any_sync(FULLMASK, kk[t] >= 0 ? kk[t] : -1 - lane);
             const SV sum = UNIT ? (SV)__popc(peers) : group_sum(peers, kk[t] >= 0 ? ww[t] : (SV)0, scratch);
             if (kk[t] >= 0 && lane == __ffs(peers) - 1) agg_insert<TV>(kk[t], (TV)sum, keys, vals, mask, list, cnt);
         }
