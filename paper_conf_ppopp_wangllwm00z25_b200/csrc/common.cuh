@@ -38,6 +38,7 @@ struct IterCounters {
     ull n_items;            // delta-update work items (one per light mover, one per chunk of a heavy one)
     ull n_fn;               // instrumented pruning: pruned vertices that would have moved (Eq. 3)
     ull n_fp;               // instrumented pruning: active vertices that stay
+    ull cursor_hi;          // dynamic work cursor of the block bin's long-row class (k_decide_block CLS 2)
 };
 
 // Pruning strategy of the active set (§3.2-3.3; DESIGN.md c20/c21):

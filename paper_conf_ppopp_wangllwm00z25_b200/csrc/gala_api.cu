@@ -108,6 +108,7 @@ struct gala_graph_s {
     int opt_delta = 2, opt_force_i128 = 0, opt_force_wide = 0, opt_cuda_graph = 1, opt_log_cap = 4096, opt_singleton = 1, opt_verbose = 0, opt_agg_big_chunk = 1,
         opt_agg_chunk = AGG_CH, opt_agg_scap = 8192;
     long long opt_agg_big_ent = 1LL << 62;
+    int opt_block_split = 2048;
     bool rows_distinct0 = false;   // level-0 rows strictly increasing (no duplicate entries)
     int32_t* rev0 = nullptr;       // level-0 reverse-entry index (enables the per-entry community array)
     int opt_ckey = 0;
@@ -458,6 +459,9 @@ struct Work {
 #endif
 #define BLOCK_BT GALA_BLOCK_BT
 #define BLOCK_E GALA_BLOCK_E
+// short-row class of the block bin (rows <= opt_block_split): 256 threads, 4 entries each
+#define BLOCK_LO_BT 256
+#define BLOCK_LO_E 4
 
 // ------------------------------------------------------------------ launch helpers
 // the per-entry neighbour-community array is used on level 0 of single-GPU runs
@@ -532,6 +536,27 @@ static void launch_single(gala_graph_s* g, Work& wk, const DecideArgs& a, typena
     launch_hub<M, UNIT>(g, wk, a, qW, p, tm, wk.hub_on ? fk.branch(3) : st);
 }
 
+// grid of the short-row block kernel (rows <= opt_block_split): resident blocks per SM for its
+// arena, computed once per (mode, unit, arena, class)
+template <int M, bool UNIT>
+static int block_lo_grid(gala_graph_s* g, int cap, bool all) {
+    static std::map<std::pair<int, int>, int> memo;
+    static std::mutex mu;
+    const std::pair<int, int> key(cap, all ? 1 : 0);
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = memo.find(key);
+    if (it != memo.end()) return g->num_sms * it->second;
+    const void* f = all ? (const void*)k_decide_block<BLOCK_LO_BT, BLOCK_LO_E, M, UNIT, 0>
+                        : (const void*)k_decide_block<BLOCK_LO_BT, BLOCK_LO_E, M, UNIT, 1>;
+    const size_t sm = block_smem_bytes<M>(cap);
+    CK(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+    int b = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, f, BLOCK_LO_BT, sm));
+    b = std::max(b, 1);
+    memo[key] = b;
+    return g->num_sms * b;
+}
+
 template <int M, bool UNIT>
 static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, typename ModeT<M>::ST qW,
                           typename ModeT<M>::ST p, Timer& tm, int64_t maxdeg, int idbits, bool single) {
@@ -551,12 +576,42 @@ static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, typename M
     // the longest-running bins go first so they start on an idle machine
     if (maxdeg > g->bins[BIN_WARP2]) {
         const int smem_cap = g->hub_smem_slots;
-        e = tm.begin();
-        k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT><<<wk.gblocks_m[M], BLOCK_BT, block_smem_bytes<M>(smem_cap),
-                                                     fk.branch(0)>>>(
-            qview(wk.queues, qs, BIN_BLOCK), BIN_BLOCK, a, qW, p, smem_cap, wk.gkeys, wk.gvals, wk.glist, wk.gcap);
-        CKL();
-        tm.end(KC_DEC_BLOCK, e);
+        const int split = g->opt_block_split;
+        int cap1 = 64;
+        while (cap1 < 2 * split) cap1 <<= 1;
+        if (split > 0 && cap1 < smem_cap) {
+            // rows <= split: small blocks with an arena that never spills; longer rows: the full arena
+            const int grid1 = block_lo_grid<M, UNIT>(g, cap1, maxdeg <= split);
+            e = tm.begin();
+            if (maxdeg <= split)
+                k_decide_block<BLOCK_LO_BT, BLOCK_LO_E, M, UNIT, 0><<<grid1, BLOCK_LO_BT, block_smem_bytes<M>(cap1),
+                                                                     fk.branch(0)>>>(
+                    qview(wk.queues, qs, BIN_BLOCK), BIN_BLOCK, a, qW, p, cap1, wk.gkeys, wk.gvals, wk.glist, wk.gcap,
+                    split);
+            else
+                k_decide_block<BLOCK_LO_BT, BLOCK_LO_E, M, UNIT, 1><<<grid1, BLOCK_LO_BT, block_smem_bytes<M>(cap1),
+                                                                     fk.branch(0)>>>(
+                    qview(wk.queues, qs, BIN_BLOCK), BIN_BLOCK, a, qW, p, cap1, wk.gkeys, wk.gvals, wk.glist, wk.gcap,
+                    split);
+            CKL();
+            tm.end(KC_DEC_BLOCK, e);
+            if (maxdeg > split) {
+                e = tm.begin();
+                k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT, 2><<<wk.gblocks_m[M], BLOCK_BT, block_smem_bytes<M>(smem_cap),
+                                                               fk.branch(0)>>>(
+                    qview(wk.queues, qs, BIN_BLOCK), BIN_BLOCK, a, qW, p, smem_cap, wk.gkeys, wk.gvals, wk.glist,
+                    wk.gcap, split);
+                CKL();
+                tm.end(KC_DEC_BLOCK, e);
+            }
+        } else {
+            e = tm.begin();
+            k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT><<<wk.gblocks_m[M], BLOCK_BT, block_smem_bytes<M>(smem_cap),
+                                                         fk.branch(0)>>>(
+                qview(wk.queues, qs, BIN_BLOCK), BIN_BLOCK, a, qW, p, smem_cap, wk.gkeys, wk.gvals, wk.glist, wk.gcap);
+            CKL();
+            tm.end(KC_DEC_BLOCK, e);
+        }
     }
     launch_hub<M, UNIT>(g, wk, a, qW, p, tm, wk.hub_on ? fk.branch(1) : st);
     e = tm.begin();
@@ -2134,6 +2189,9 @@ gala_status gala_set_option(gala_graph g, const char* key, int64_t value) {
     else if (k == "agg_chunk") {   // test hook: entries per big-community chunk (1..AGG_CH)
         if (value < 1 || value > AGG_CH) return set_err(GALA_E_INVALID, "agg_chunk must be in [1, 4096]");
         g->opt_agg_chunk = (int)value;
+    } else if (k == "block_split") {   // block bin: rows <= split in small blocks (0: one class)
+        if (value < 0 || value > (1 << 20)) return set_err(GALA_E_INVALID, "block_split must be in [0, 2^20]");
+        g->opt_block_split = (int)value;
     } else if (k == "agg_big_ent") {   // phase 2: communities with more entries take the chunked path
         if (value < 1) return set_err(GALA_E_INVALID, "agg_big_ent must be >= 1");
         g->opt_agg_big_ent = value;

@@ -487,11 +487,36 @@ __global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB, MAXDEG <= 1
 // vertices.  Vertices are fetched dynamically; each thread batches E entries.
 // ---------------------------------------------------------------------------
 #define HWIN 16
-template <int BT, int E, int M, bool UNIT>
+// CLS 0: every queued vertex; CLS 1: rows <= split only; CLS 2: rows > split only (two launches
+// with arenas sized for their class: short rows get small blocks, more vertices in flight per SM).
+// A class kernel fetches the queue in batches of FETCH_B indices (thread 0) and skips the rows of
+// the other class.
+#define FETCH_B 8
+template <int CLS>
+__device__ __forceinline__ long long block_next_item(QView queue, long long count, ull* cursor, int split,
+                                                     int* s_batch, int* s_nb, int* s_bi) {
+    if (CLS == 0) return (long long)atomicAdd(cursor, 1ull);
+    for (;;) {
+        if (*s_bi < *s_nb) return s_batch[(*s_bi)++];
+        const long long b0 = (long long)atomicAdd(cursor, (ull)FETCH_B);
+        if (b0 >= count) return count;
+        int dg[FETCH_B];
+#pragma unroll
+        for (int t = 0; t < FETCH_B; ++t) dg[t] = b0 + t < count ? queue[b0 + t].deg : -1;
+        int nb = 0;
+#pragma unroll
+        for (int t = 0; t < FETCH_B; ++t)
+            if (dg[t] >= 0 && ((dg[t] <= split) == (CLS == 1))) s_batch[nb++] = (int)(b0 + t);
+        *s_nb = nb;
+        *s_bi = 0;
+    }
+}
+
+template <int BT, int E, int M, bool UNIT, int CLS = 0>
 __global__ void __launch_bounds__(BT) k_decide_block(QView queue, int bin, DecideArgs a,
                                                      typename ModeT<M>::ST qW, typename ModeT<M>::ST p, int smem_cap,
                                                      int* __restrict__ gkeys_all, ull* __restrict__ gvals_all,
-                                                     int* __restrict__ glist_all, long long gcap) {
+                                                     int* __restrict__ glist_all, long long gcap, int split = 0) {
     if (a.ckey && !*a.ckey_valid) a.ckey = nullptr;
     typedef typename ModeT<M>::ST ST;
     typedef typename ModeT<M>::VT VT;
@@ -514,8 +539,11 @@ __global__ void __launch_bounds__(BT) k_decide_block(QView queue, int bin, Decid
     if (threadIdx.x == 0) s_gcnt = 0;
     const long long count = (long long)a.ctr->bin_count[bin];
     unsigned my_k = 0;
+    __shared__ int s_batch[FETCH_B], s_nb, s_bi;
+    if (threadIdx.x == 0) { s_nb = 0; s_bi = 0; }
+    ull* const cursor = CLS == 2 ? &a.ctr->cursor_hi : &a.ctr->cursor[bin];
     for (;;) {
-        if (threadIdx.x == 0) s_item = (long long)atomicAdd(&a.ctr->cursor[bin], 1ull);
+        if (threadIdx.x == 0) s_item = block_next_item<CLS>(queue, count, cursor, split, s_batch, &s_nb, &s_bi);
         __syncthreads();
         long long i = s_item;
         if (i >= count) break;
