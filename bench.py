@@ -259,6 +259,16 @@ def main():
     labels = h.communities()
     Q = h.modularity()
     last_stats = h.stats()
+    # per-iteration pruned fraction (north star reporting), from one more (untimed) traced run:
+    # |inactive| / |{v : d(v) > 0}| = n_pruned / (n_active + n_pruned)
+    h.set_option("trace", 1)
+    h.set_option("timing", 0)
+    h.run()
+    pruned = {}
+    for r in h.trace():
+        tot = r["n_active"] + r["n_pruned"]
+        pruned.setdefault(f"L{r['level']}", []).append(round(r["n_pruned"] / tot, 4) if tot else 0.0)
+    h.set_option("trace", 0)
     h.free()
     total_s = sum(step_ms) / 1e3
     value = edges / total_s / 1e9
@@ -342,6 +352,7 @@ def main():
         "step_ms": [round(x, 3) for x in step_ms],
         "modularity": Q,
         "nmi_vs_planted": (gala.nmi_device(labels, g.truth) if getattr(g, "truth", None) is not None else None),
+        "pruned_fraction_per_iteration": pruned,
         "levels": len(last_stats["levels"]),
         "iterations": sum(lv["iters"] for lv in last_stats["levels"]),
         "gteps_scanned": scanned / total_s / 1e9,
