@@ -596,6 +596,12 @@ static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, typename M
             CKL();
             tm.end(KC_DEC_BLOCK, e);
             if (maxdeg > split) {
+                static std::once_flag attr2;   // the class-2 instantiation's dynamic smem limit
+                std::call_once(attr2, [&] {
+                    CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT, 2>,
+                                            cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                            (int)block_smem_bytes<M>(16384)));
+                });
                 e = tm.begin();
                 k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT, 2><<<wk.gblocks_m[M], BLOCK_BT, block_smem_bytes<M>(smem_cap),
                                                                fk.branch(0)>>>(
