@@ -31,6 +31,8 @@ struct Comm {
     virtual void allreduce_sum_i64(int64_t* buf, size_t count, cudaStream_t st) = 0;
     // host scalar from every rank (synchronises)
     virtual std::vector<int64_t> allgather_host(int64_t x, cudaStream_t st) = 0;
+    // this rank failed mid-run: release peers blocked in a collective (they raise CommError)
+    virtual void abort() {}
 };
 
 // ------------------------------------------------------------------ NCCL (dlopen)
@@ -125,18 +127,28 @@ struct LoopShared {
     std::vector<const void*> ptr;
     std::vector<cudaEvent_t> ev;
     std::vector<int64_t> scal;
-    void barrier() {
-        std::unique_lock<std::mutex> lk(mu);
-        long long gen = generation;
-        if (++arrived == world) {
-            arrived = 0;
-            ++generation;
-            cv.notify_all();
-        } else {
-            cv.wait(lk, [&] { return generation != gen; });
-        }
+    bool aborted = false;
+    void barrier();
+    void abort() {
+        std::lock_guard<std::mutex> lk(mu);
+        aborted = true;
+        cv.notify_all();
     }
 };
+struct CommError;
+inline void LoopShared::barrier() {
+    std::unique_lock<std::mutex> lk(mu);
+    long long gen = generation;
+    if (aborted) throw CommError{"loopback: a peer rank failed"};
+    if (++arrived == world) {
+        arrived = 0;
+        ++generation;
+        cv.notify_all();
+    } else {
+        cv.wait(lk, [&] { return generation != gen || aborted; });
+        if (generation == gen) throw CommError{"loopback: a peer rank failed"};
+    }
+}
 static std::mutex g_loop_mu;
 static std::map<std::string, std::shared_ptr<LoopShared>> g_loops;
 
@@ -150,6 +162,7 @@ __global__ void k_sum_rows_i64(int64_t* out, const int64_t* in, size_t count, in
 
 struct LoopComm : Comm {
     std::shared_ptr<LoopShared> sh;
+    void abort() override { sh->abort(); }
     LoopComm(const void* uid, int r, int w) {
         rank = r;
         world = w;

@@ -1806,10 +1806,12 @@ static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_level
         g->run_ms = ms;
         g->launches = g_launches - launches0;
     } catch (CommError& e) {
+        cm.abort();
         dfree(lmoves, st); dfree(gmoves, st); dfree(newC, st); dfree(dcnt, st); dfree(vec, st);
         set_err(GALA_E_NCCL, "%s", e.msg.c_str());
         throw GalaError{GALA_E_NCCL};
     } catch (...) {
+        cm.abort();   // peers blocked in a collective raise instead of waiting forever
         dfree(lmoves, st); dfree(gmoves, st); dfree(newC, st); dfree(dcnt, st); dfree(vec, st);
         throw;
     }
