@@ -172,6 +172,9 @@ void gala_graph_free(gala_graph g);
  *   "log_cap"        device iteration-log capacity (default 4096)
  *   "sync_mode"      multi-GPU label exchange: 0 adaptive (default), 1 dense, 2 sparse
  *   "verbose"        0/1   host-side phase timings on stderr
+ *   "block_split"    block bin split point (default 1024; 0: one class): on levels with rows longer
+ *                          than it, rows <= split run in 256-thread blocks with a small arena, the
+ *                          rest in the 512-thread full-arena kernel
  *   "agg_big_chunk"  0/1   phase 2: big communities in 4096-entry chunks over the whole GPU with a
  *                          block-smem pre-combine (default 1); 0: 32 blocks per big community
  *   "agg_chunk"      [1, 4096] entries per big-community chunk (test hook, default 4096)

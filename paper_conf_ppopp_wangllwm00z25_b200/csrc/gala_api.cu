@@ -108,7 +108,7 @@ struct gala_graph_s {
     int opt_delta = 2, opt_force_i128 = 0, opt_force_wide = 0, opt_cuda_graph = 1, opt_log_cap = 4096, opt_singleton = 1, opt_verbose = 0, opt_agg_big_chunk = 1,
         opt_agg_chunk = AGG_CH, opt_agg_scap = 8192;
     long long opt_agg_big_ent = 1LL << 62;
-    int opt_block_split = 2048;
+    int opt_block_split = 1024;
     bool rows_distinct0 = false;   // level-0 rows strictly increasing (no duplicate entries)
     int32_t* rev0 = nullptr;       // level-0 reverse-entry index (enables the per-entry community array)
     int opt_ckey = 0;
@@ -579,23 +579,19 @@ static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, typename M
         const int split = g->opt_block_split;
         int cap1 = 64;
         while (cap1 < 2 * split) cap1 <<= 1;
-        if (split > 0 && cap1 < smem_cap) {
-            // rows <= split: small blocks with an arena that never spills; longer rows: the full arena
-            const int grid1 = block_lo_grid<M, UNIT>(g, cap1, maxdeg <= split);
+        if (split > 0 && cap1 < smem_cap && maxdeg > split) {
+            // rows <= split: small blocks with an arena that never spills; longer rows: the full
+            // arena (a level whose rows all fit the split keeps the single full-arena kernel:
+            // measured faster there, lfr1m)
+            const int grid1 = block_lo_grid<M, UNIT>(g, cap1, false);
             e = tm.begin();
-            if (maxdeg <= split)
-                k_decide_block<BLOCK_LO_BT, BLOCK_LO_E, M, UNIT, 0><<<grid1, BLOCK_LO_BT, block_smem_bytes<M>(cap1),
-                                                                     fk.branch(0)>>>(
-                    qview(wk.queues, qs, BIN_BLOCK), BIN_BLOCK, a, qW, p, cap1, wk.gkeys, wk.gvals, wk.glist, wk.gcap,
-                    split);
-            else
-                k_decide_block<BLOCK_LO_BT, BLOCK_LO_E, M, UNIT, 1><<<grid1, BLOCK_LO_BT, block_smem_bytes<M>(cap1),
-                                                                     fk.branch(0)>>>(
-                    qview(wk.queues, qs, BIN_BLOCK), BIN_BLOCK, a, qW, p, cap1, wk.gkeys, wk.gvals, wk.glist, wk.gcap,
-                    split);
+            k_decide_block<BLOCK_LO_BT, BLOCK_LO_E, M, UNIT, 1><<<grid1, BLOCK_LO_BT, block_smem_bytes<M>(cap1),
+                                                                 fk.branch(0)>>>(
+                qview(wk.queues, qs, BIN_BLOCK), BIN_BLOCK, a, qW, p, cap1, wk.gkeys, wk.gvals, wk.glist, wk.gcap,
+                split);
             CKL();
             tm.end(KC_DEC_BLOCK, e);
-            if (maxdeg > split) {
+            {
                 static std::once_flag attr2;   // the class-2 instantiation's dynamic smem limit
                 std::call_once(attr2, [&] {
                     CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT, 2>,

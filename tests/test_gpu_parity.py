@@ -132,7 +132,7 @@ def test_pruning_strategy_weighted_and_graph_mode(strategy):
     dict(agg_big_ent=64, agg_chunk=32),                                      # phase 2: entry-count big path
     dict(block_split=0),                                                     # block bin as one class
     dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=0, bin_warp512=0, block_split=64),
-    dict(bin_warp=16, bin_warp512=32, block_split=100, force_i128=1),
+    dict(bin_sub32=16, bin_warp=16, bin_warp512=32, block_split=100, force_i128=1),
 ])
 def test_dispatch_independence(opts):
     """P7: thresholds / table sizes / integer width / update strategy never change a label."""
