@@ -177,6 +177,8 @@ void gala_graph_free(gala_graph g);
  *                          rest in the 512-thread full-arena kernel
  *   "agg_big_chunk"  0/1   phase 2: big communities in 4096-entry chunks over the whole GPU with a
  *                          block-smem pre-combine (default 1); 0: 32 blocks per big community
+ *   "agg_bound"      0/1   phase 2: big-community global tables sized from the chunks' distinct counts
+ *                          (two passes, default 1) instead of from min(entries, k)
  *   "agg_chunk"      [1, 4096] entries per big-community chunk (test hook, default 4096)
  *   "agg_scap"       [512, 8192] largest phase-2 shared-memory table; communities needing more
  *                          slots take the big (global-table) path (test hook, default 8192)

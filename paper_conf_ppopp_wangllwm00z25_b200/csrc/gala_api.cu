@@ -109,6 +109,7 @@ struct gala_graph_s {
         opt_agg_chunk = AGG_CH, opt_agg_scap = 8192;
     long long opt_agg_big_ent = 1LL << 62;
     int opt_block_split = 1024;
+    int opt_agg_bound = 1;
     bool rows_distinct0 = false;   // level-0 rows strictly increasing (no duplicate entries)
     int32_t* rev0 = nullptr;       // level-0 reverse-entry index (enables the per-entry community array)
     int opt_ckey = 0;
@@ -988,7 +989,52 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
     int nbig = 0;
     CK(cudaMemcpyAsync(&nbig, nbig_dev, sizeof(int), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
-    if (nbig > 0) {
+    if (nbig > 0 && g->opt_agg_big_chunk && g->opt_agg_bound) {
+        // two-pass: chunk combine in place -> tables sized from the chunks' distinct counts
+        const int ch = g->opt_agg_chunk;
+        long long* nch = dalloc<long long>(nbig + 1, st);
+        long long* choff = dalloc<long long>(nbig + 1, st);
+        k_agg_big_nchunks<<<grid_for(nbig, 256, big), 256, 0, st>>>(nbig, bigc, ent, nch, ch);
+        CKL();
+        scan_excl(nch, choff, nbig, st);
+        int* ndc = dalloc<int>(cur.nnz / ch + nbig + 1, st);   // >= total chunks
+        const int gb = g->num_sms * 2;
+        if (unit || v32) {
+            const size_t sm = agg_chunk_smem<unsigned>();
+            auto kf = unit ? k_agg_big_combine<true, unsigned> : k_agg_big_combine<false, unsigned>;
+            CK(cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+            kf<<<gb, 256, sm, st>>>(a, bigc, nbig, choff, ndc, ch);
+        } else {
+            const size_t sm = agg_chunk_smem<ull>();
+            CK(cudaFuncSetAttribute(k_agg_big_combine<false, ull>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+            k_agg_big_combine<false, ull><<<gb, 256, sm, st>>>(a, bigc, nbig, choff, ndc, ch);
+        }
+        CKL();
+        k_agg_big_bound<<<grid_for((long long)nbig * 32, 256, big), 256, 0, st>>>(nbig, k, choff, ndc, bigcap);
+        CKL();
+        vt.lap("agg: big combine");
+        long long* goff = dalloc<long long>(nbig + 1, st);
+        scan_excl(bigcap, goff, nbig, st);
+        long long gtot = 0;
+        CK(cudaMemcpyAsync(&gtot, goff + nbig, sizeof(long long), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        int* gkeys = dalloc<int>(gtot, st);
+        ull* gvals = dalloc<ull>(gtot, st);
+        int* glist = dalloc<int>(gtot / 2 + 1, st);
+        int* gcnt = dalloc<int>(nbig, st);
+        CK(cudaMemsetAsync(gkeys, 0xff, sizeof(int) * gtot, st));
+        CK(cudaMemsetAsync(gvals, 0, sizeof(ull) * gtot, st));
+        CK(cudaMemsetAsync(gcnt, 0, sizeof(int) * nbig, st));
+        vt.lap("agg: big alloc+clear");
+        k_agg_big_insert2<<<big, 256, 0, st>>>(a, bigc, nbig, choff, ndc, ch, goff, gkeys, gvals, glist, gcnt);
+        CKL();
+        vt.lap("agg: big insert");
+        k_agg_big_emit2<<<big, 256, 0, st>>>(a, bigc, nbig, choff, goff, gkeys, gvals, glist, gcnt, ch);
+        CKL();
+        dfree(nch, st); dfree(choff, st); dfree(ndc, st);
+        dfree(goff, st); dfree(gkeys, st); dfree(gvals, st); dfree(glist, st); dfree(gcnt, st);
+        if (g->opt_verbose) fprintf(stderr, "[gala] big communities %d, table slots %lld (bounded)\n", nbig, gtot);
+    } else if (nbig > 0) {
         long long* goff = dalloc<long long>(nbig + 1, st);
         scan_excl(bigcap, goff, nbig, st);
         long long gtot = 0;
@@ -2193,6 +2239,8 @@ gala_status gala_set_option(gala_graph g, const char* key, int64_t value) {
     else if (k == "agg_chunk") {   // test hook: entries per big-community chunk (1..AGG_CH)
         if (value < 1 || value > AGG_CH) return set_err(GALA_E_INVALID, "agg_chunk must be in [1, 4096]");
         g->opt_agg_chunk = (int)value;
+    } else if (k == "agg_bound") {   // phase 2: size big-community tables from chunk distinct counts
+        g->opt_agg_bound = value != 0;
     } else if (k == "block_split") {   // block bin: rows <= split in small blocks (0: one class)
         if (value < 0 || value > (1 << 20)) return set_err(GALA_E_INVALID, "block_split must be in [0, 2^20]");
         g->opt_block_split = (int)value;

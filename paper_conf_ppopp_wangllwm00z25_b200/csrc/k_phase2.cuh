@@ -516,6 +516,85 @@ __global__ void __launch_bounds__(256) k_agg_big_chunk(AggArgs a, const int32_t*
     }
 }
 
+// Two-pass variant (option agg_bound, default): pass 1 combines every chunk in block smem and
+// writes its distinct (key, sum) pairs back to the start of the chunk's own range of the
+// segment (ndc[t] of them); the global table of a community is then sized from
+// B = sum of its chunks' distinct counts (<= entries, usually far below), nextpow2(2 min(B, k))
+// slots, and pass 2 inserts the chunk-distinct pairs.
+template <bool UNIT, typename V>
+__global__ void __launch_bounds__(256) k_agg_big_combine(AggArgs a, const int32_t* __restrict__ bigc, int nbig,
+                                                         const long long* __restrict__ choff, int* __restrict__ ndc,
+                                                         int ch) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    V* vals = reinterpret_cast<V*>(smem_raw);
+    int* keys = reinterpret_cast<int*>(smem_raw + (size_t)AGG_CH_SLOTS * sizeof(V));
+    int* list = keys + AGG_CH_SLOTS;
+    __shared__ int s_cnt;
+    __shared__ V s_scr[8][32];
+    const int wib = threadIdx.x >> 5;
+    for (int j = threadIdx.x; j < AGG_CH_SLOTS; j += 256) { keys[j] = -1; vals[j] = 0; }
+    if (threadIdx.x == 0) s_cnt = 0;
+    __syncthreads();
+    const long long total = choff[nbig];
+    for (long long t = blockIdx.x; t < total; t += gridDim.x) {
+        const int bi = (int)seg_search(choff, 0, nbig - 1, t);
+        const long long c = bigc[bi];
+        const long long s1 = a.eoff[c + 1];
+        const long long lo = a.eoff[c] + (t - choff[bi]) * ch;
+        const long long hi = lo + ch < s1 ? lo + ch : s1;
+        agg_segment<UNIT, V, V>(a, lo, hi, threadIdx.x, 256, keys, vals, AGG_CH_SLOTS - 1, list, &s_cnt, s_scr[wib]);
+        __syncthreads();   // every entry of the chunk is read before its range is overwritten
+        const int m = s_cnt;
+        for (int i = threadIdx.x; i < m; i += 256) {
+            const int slot = list[i];
+            a.tkey[lo + i] = keys[slot];
+            a.tval[lo + i] = (int64_t)vals[slot];
+            keys[slot] = -1;
+            vals[slot] = 0;
+        }
+        if (threadIdx.x == 0) ndc[t] = m;
+        __syncthreads();
+        if (threadIdx.x == 0) s_cnt = 0;
+        __syncthreads();
+    }
+}
+
+// table slots of big community i: nextpow2(2 min(B_i, k)), B_i = sum of its chunks' distinct counts
+__global__ void k_agg_big_bound(int nbig, long long k, const long long* __restrict__ choff,
+                                const int* __restrict__ ndc, long long* __restrict__ bigcap) {
+    const int lane = lane_id();
+    const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+    for (long long i = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < nbig; i += nw) {
+        long long b = 0;
+        for (long long t = choff[i] + lane; t < choff[i + 1]; t += 32) b += ndc[t];
+        b = warp_sum_ll(b);
+        if (lane == 0) {
+            const long long m = b < k ? b : k;
+            bigcap[i] = m > 0 ? 1LL << (64 - __clzll(2 * m - 1)) : 1;
+        }
+    }
+}
+
+__global__ void __launch_bounds__(256) k_agg_big_insert2(AggArgs a, const int32_t* __restrict__ bigc, int nbig,
+                                                         const long long* __restrict__ choff,
+                                                         const int* __restrict__ ndc, int ch,
+                                                         const long long* __restrict__ goff, int* __restrict__ gkeys,
+                                                         ull* __restrict__ gvals, int* __restrict__ glist,
+                                                         int* __restrict__ gcnt) {
+    const long long total = choff[nbig];
+    for (long long t = blockIdx.x; t < total; t += gridDim.x) {
+        const int bi = (int)seg_search(choff, 0, nbig - 1, t);
+        const long long c = bigc[bi];
+        const long long lo = a.eoff[c] + (t - choff[bi]) * ch;
+        const int m = ndc[t];
+        const long long off = goff[bi];
+        const unsigned mask = (unsigned)(goff[bi + 1] - off) - 1u;
+        for (int i = threadIdx.x; i < m; i += 256)
+            agg_insert<ull>(a.tkey[lo + i], (ull)a.tval[lo + i], gkeys + off, gvals + off, mask, glist + off / 2,
+                            &gcnt[bi]);
+    }
+}
+
 // distinct entries of the big communities to the start of their segments; list
 // index range of chunk t = [j*AGG_CH, (j+1)*AGG_CH) of its community (m <= entries)
 __global__ void __launch_bounds__(256) k_agg_big_emit2(AggArgs a, const int32_t* __restrict__ bigc, int nbig,

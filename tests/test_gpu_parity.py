@@ -128,6 +128,7 @@ def test_pruning_strategy_weighted_and_graph_mode(strategy):
     dict(hub(64), concurrent=1, delta_update=1),
     dict(agg_scap=512, agg_chunk=64),                                        # phase 2: many multi-chunk big communities
     dict(agg_scap=512, agg_chunk=1),
+    dict(agg_scap=512, agg_chunk=64, agg_bound=0),                           # phase 2: one-pass big path
     dict(agg_scap=512, agg_big_chunk=0),                                     # phase 2: per-community block split
     dict(agg_big_ent=64, agg_chunk=32),                                      # phase 2: entry-count big path
     dict(block_split=0),                                                     # block bin as one class
