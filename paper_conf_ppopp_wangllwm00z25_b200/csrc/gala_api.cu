@@ -558,6 +558,17 @@ static int block_lo_grid(gala_graph_s* g, int cap, bool all) {
     return g->num_sms * b;
 }
 
+// every block-kernel attribute / grid the launches need, set up front: nothing of this may run
+// while a level's iteration body is being captured into a CUDA graph
+template <int M, bool UNIT>
+static void block_setup(gala_graph_s* g) {
+    int cap1 = 64;
+    while (cap1 < 2 * std::max(g->opt_block_split, 1)) cap1 <<= 1;
+    (void)block_lo_grid<M, UNIT>(g, cap1, false);
+    CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)block_smem_bytes<M>(16384)));
+}
+
 template <int M, bool UNIT>
 static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, typename ModeT<M>::ST qW,
                           typename ModeT<M>::ST p, Timer& tm, int64_t maxdeg, int idbits, bool single) {
@@ -593,12 +604,6 @@ static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, typename M
             CKL();
             tm.end(KC_DEC_BLOCK, e);
             {
-                static std::once_flag attr2;   // the class-2 instantiation's dynamic smem limit
-                std::call_once(attr2, [&] {
-                    CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT, 2>,
-                                            cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                            (int)block_smem_bytes<M>(16384)));
-                });
                 e = tm.begin();
                 k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT, 2><<<wk.gblocks_m[M], BLOCK_BT, block_smem_bytes<M>(smem_cap),
                                                                fk.branch(0)>>>(
@@ -762,6 +767,7 @@ static void phase1_level(gala_graph_s* g, Work& wk, const DevCSR& G, typename Mo
                          std::vector<IterLog>& out, int level, bool single_ok) {
     cudaStream_t st = g->stream;
     const bool stepwise = !g->opt_cuda_graph || g->opt_trace >= 2 || g->opt_timing;
+    block_setup<M, UNIT>(g);   // host-side attributes / grids before any capture (block_split may have changed)
     out.clear();
     // first iteration of a level: singleton fast path when rows hold distinct columns
     bool first_single = single_ok && g->opt_singleton;
@@ -1243,6 +1249,9 @@ static void ensure_workspace(gala_graph_s* g) {
             per_sm = std::max(std::max(wk.gblocks_m[0], wk.gblocks_m[1]), wk.gblocks_m[2]) / g->num_sms;
             set_warp_smem<32, 128, DM_FAST>(); set_warp_smem<32, 128, DM_W64>(); set_warp_smem<32, 128, DM_W128>();
             set_warp_smem<32, 512, DM_FAST>(); set_warp_smem<32, 512, DM_W64>(); set_warp_smem<32, 512, DM_W128>();
+            block_setup<DM_FAST, true>(g); block_setup<DM_FAST, false>(g);
+            block_setup<DM_W64, true>(g); block_setup<DM_W64, false>(g);
+            block_setup<DM_W128, true>(g); block_setup<DM_W128, false>(g);
             wk.gblocks = g->num_sms * std::max(per_sm, 1);
             wk.gcap = 0;   // spill tables sized on demand (coarse levels can have larger rows than level 0)
             wk.smem_cap = cap;
