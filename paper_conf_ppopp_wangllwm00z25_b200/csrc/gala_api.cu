@@ -895,7 +895,13 @@ struct VTimer {
 // Coarsen level graph `cur` with community ids newid[v] in [0, k) into `nxt`
 // (reading c10: the diagonal carries D_C(c) once).  See k_phase2.cuh for
 // the per-community aggregation paths.  Coarse d(c) = Sigma_tot(c), s(c) = diagonal.
-#define AGG_BLOCK_BT 512
+#ifndef GALA_AGG_BT_C
+#define GALA_AGG_BT_C 512    // threads of the largest block-path class (tables <= scap slots)
+#endif
+#ifndef GALA_AGG_BT_B
+#define GALA_AGG_BT_B 256    // threads of the middle class (tables <= AGG_BB slots)
+#endif
+#define AGG_BLOCK_BT GALA_AGG_BT_C
 template <typename V>
 static size_t agg_block_smem(int scap) { return (size_t)scap * (sizeof(V) + sizeof(int)) + (size_t)(scap / 2) * sizeof(int); }
 
@@ -927,8 +933,8 @@ static void agg_launch_small(gala_graph_s* g, const AggArgs& a, bool unit, int s
         else agg_block_class<128, false, V>(g, a, ca, bl, nbl);
     }
     if (scap > AGG_BA) {
-        if (unit) agg_block_class<256, true, V>(g, a, cb, bl + k, nbl + 1);
-        else agg_block_class<256, false, V>(g, a, cb, bl + k, nbl + 1);
+        if (unit) agg_block_class<GALA_AGG_BT_B, true, V>(g, a, cb, bl + k, nbl + 1);
+        else agg_block_class<GALA_AGG_BT_B, false, V>(g, a, cb, bl + k, nbl + 1);
     }
     if (scap > AGG_BB) {
         if (unit) agg_block_class<AGG_BLOCK_BT, true, V>(g, a, scap, bl + 2 * k, nbl + 2);
