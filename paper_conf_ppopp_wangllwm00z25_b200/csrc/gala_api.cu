@@ -111,6 +111,7 @@ struct gala_graph_s {
     int opt_block_split = 1024;
     int opt_agg_bound = 1;
     bool rows_distinct0 = false;   // level-0 rows strictly increasing (no duplicate entries)
+    bool self0 = true;             // level 0 has a self-loop (s0 not all zero)
     int32_t* rev0 = nullptr;       // level-0 reverse-entry index (enables the per-entry community array)
     int opt_ckey = 0;
     int bins[NBINS - 1] = {4, 8, 16, 32, 128, 512, 16384};
@@ -410,6 +411,8 @@ struct Work {
     QRec* queues = nullptr;
     int32_t* ckey = nullptr;   // level-0 per-entry neighbour community
     int64_t *Sig = nullptr, *d = nullptr, *s = nullptr, *dp = nullptr;
+    bool s_zero = false;   // this level has no self-loops: k_reduce skips s (level 0 of a loop-free graph)
+    const int64_t* s_live() const { return s_zero ? nullptr : s; }
     IterCounters* ctr = nullptr;
     Carry* carry = nullptr;
     IterLog* log = nullptr;
@@ -538,19 +541,23 @@ static void launch_single(gala_graph_s* g, Work& wk, const DecideArgs& a, typena
 }
 
 // grid of the short-row block kernel (rows <= opt_block_split): resident blocks per SM for its
-// arena, computed once per (mode, unit, arena, class)
+// arena, computed once per (mode, unit, arena, class).  The dynamic shared-memory limit is a
+// per-function, process-wide attribute, so `setup` (outside any graph capture) re-sets it to
+// this arena on every call: a memo hit alone would keep the limit of whichever arena was set
+// last (a smaller block_split on another handle) and the launch would fail.
 template <int M, bool UNIT>
-static int block_lo_grid(gala_graph_s* g, int cap, bool all) {
+static int block_lo_grid(gala_graph_s* g, int cap, bool all, bool setup = false) {
     static std::map<std::pair<int, int>, int> memo;
     static std::mutex mu;
     const std::pair<int, int> key(cap, all ? 1 : 0);
-    std::lock_guard<std::mutex> lk(mu);
-    auto it = memo.find(key);
-    if (it != memo.end()) return g->num_sms * it->second;
     const void* f = all ? (const void*)k_decide_block<BLOCK_LO_BT, BLOCK_LO_E, M, UNIT, 0>
                         : (const void*)k_decide_block<BLOCK_LO_BT, BLOCK_LO_E, M, UNIT, 1>;
     const size_t sm = block_smem_bytes<M>(cap);
-    CK(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+    std::lock_guard<std::mutex> lk(mu);
+    if (setup) CK(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+    auto it = memo.find(key);
+    if (it != memo.end()) return g->num_sms * it->second;
+    if (!setup) CK(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
     int b = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, f, BLOCK_LO_BT, sm));
     b = std::max(b, 1);
@@ -564,9 +571,12 @@ template <int M, bool UNIT>
 static void block_setup(gala_graph_s* g) {
     int cap1 = 64;
     while (cap1 < 2 * std::max(g->opt_block_split, 1)) cap1 <<= 1;
-    (void)block_lo_grid<M, UNIT>(g, cap1, false);
+    (void)block_lo_grid<M, UNIT>(g, cap1, false, true);
     CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                             (int)block_smem_bytes<M>(16384)));
+    // single-class block kernel: this handle's arena (another handle may have set a smaller one)
+    CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)block_smem_bytes<M>(g->hub_smem_slots)));
 }
 
 template <int M, bool UNIT>
@@ -748,7 +758,7 @@ static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, typename
     }
     tm.end(KC_DP, e);
     e = tm.begin();
-    k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>(n, 0, n, wk.dp, wk.s, wk.Sig, wk.part_dc, wk.part_s2, wk.part_min, wk.ctr,
+    k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>(n, 0, n, wk.dp, wk.s_live(), wk.Sig, wk.part_dc, wk.part_s2, wk.part_min, wk.ctr,
                                                   wk.carry, (long long)(qW128 >> 64), (ull)qW128, (long long)p,
                                                   (long long)(T >> 64), (ull)T, 1, wk.log, wk.log_cap, g->opt_max_iters,
                                                   cond);
@@ -1149,6 +1159,7 @@ static void coarsen(gala_graph_s* g, Work& wk, const DevCSR& cur, int64_t nl, lo
     CK(cudaMemcpyAsync(&hm, dev_max, sizeof(ull), cudaMemcpyDeviceToHost, st));
     CK(cudaMemcpyAsync(wk.d, dnew, sizeof(int64_t) * k, cudaMemcpyDeviceToDevice, st));
     CK(cudaMemcpyAsync(wk.s, snew, sizeof(int64_t) * k, cudaMemcpyDeviceToDevice, st));
+    wk.s_zero = false;
     CK(cudaStreamSynchronize(st));
     dmax = (int64_t)hm;
     dfree(snew, st);
@@ -1308,6 +1319,7 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
         bool cur_owned = false;
         CK(cudaMemcpyAsync(wk.d, g->d0, sizeof(int64_t) * n0, cudaMemcpyDeviceToDevice, st));
         CK(cudaMemcpyAsync(wk.s, g->s0, sizeof(int64_t) * n0, cudaMemcpyDeviceToDevice, st));
+        wk.s_zero = !g->self0;
         int64_t maxdeg = g->maxdeg0, dmax = g->maxw0;
         bool first_level = true;
         Timer tm(g);
@@ -1339,7 +1351,7 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
             }
             k_iter_begin<<<1, 128, 0, st>>>(wk.ctr);
             CKL();
-            k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>((int)nl, 0, (int)nl, wk.dp, wk.s, wk.Sig, wk.part_dc, wk.part_s2,
+            k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>((int)nl, 0, (int)nl, wk.dp, wk.s_live(), wk.Sig, wk.part_dc, wk.part_s2,
                                                           wk.part_min, wk.ctr, wk.carry, (long long)(qW128 >> 64),
                                                           (ull)qW128, (long long)p, 0, 0, 0);
             CKL();
@@ -1572,7 +1584,7 @@ static void dist_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, long long
         CKL();
     }
     vt.lap("dist: apply+dp");
-    k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>((int)n, (int)lv0, (int)lv1, wk.dp, wk.s, wk.Sig, wk.part_dc,
+    k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>((int)n, (int)lv0, (int)lv1, wk.dp, wk.s_live(), wk.Sig, wk.part_dc,
                                                   wk.part_s2, wk.part_min, wk.ctr, wk.carry, 0, 0, 0, 0, 0, 3);
     CKL();
     k_pack_counters<<<1, 32, 0, st>>>(wk.carry, wk.ctr, vec);
@@ -1644,6 +1656,7 @@ static void dist_coarsen(gala_graph_s* g, Work& wk, const DevCSR& cur, int64_t n
     CKL();
     CK(cudaMemcpyAsync(wk.d, dnew, sizeof(int64_t) * k, cudaMemcpyDeviceToDevice, st));
     CK(cudaMemcpyAsync(wk.s, snew, sizeof(int64_t) * k, cudaMemcpyDeviceToDevice, st));
+    wk.s_zero = false;
     // edge-balanced split of the coarse graph; keep this rank's rows
     long long* dbounds = dalloc<long long>(cm.world + 1, st);
     k_partition_bounds<<<1, 64, 0, st>>>(k, full.rp, cm.world, dbounds);
@@ -1728,6 +1741,7 @@ static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_level
         bool cur_owned = false;
         CK(cudaMemcpyAsync(wk.d, g->d0, sizeof(int64_t) * n0, cudaMemcpyDeviceToDevice, st));
         CK(cudaMemcpyAsync(wk.s, g->s0, sizeof(int64_t) * n0, cudaMemcpyDeviceToDevice, st));
+        wk.s_zero = !g->self0;
         int64_t maxdeg = g->maxdeg0, dmax = g->maxw0;
         std::vector<long long> bounds = g->dbounds0;
         Timer tm(g);
@@ -1750,7 +1764,7 @@ static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_level
             if (level == 0) CK(cudaMemcpyAsync(g->lab, wk.C, sizeof(int32_t) * n0, cudaMemcpyDeviceToDevice, st));
             k_iter_begin<<<1, 128, 0, st>>>(wk.ctr);
             CKL();
-            k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>((int)nl, (int)lv0, (int)lv1, wk.dp, wk.s, wk.Sig, wk.part_dc,
+            k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>((int)nl, (int)lv0, (int)lv1, wk.dp, wk.s_live(), wk.Sig, wk.part_dc,
                                                           wk.part_s2, wk.part_min, wk.ctr, wk.carry, 0, 0, 0, 0, 0, 2);
             CKL();
             k_pack_counters<<<1, 32, 0, st>>>(wk.carry, wk.ctr, vec);
@@ -1934,8 +1948,8 @@ static void finish_graph(gala_graph_s* g) {
     g->g0.row = dalloc<int32_t>(g->g0.nnz, st);
     k_fill_rows<<<grid_for(n * 32, 256, big), 256, 0, st>>>((int)n, g->g0.rp, g->g0.row);
     CKL();
-    ull* mx = dalloc<ull>(3, st);
-    CK(cudaMemsetAsync(mx, 0, 3 * sizeof(ull), st));
+    ull* mx = dalloc<ull>(4, st);
+    CK(cudaMemsetAsync(mx, 0, 4 * sizeof(ull), st));
     int grid = grid_for(n * 32, 256, big);
     if (g->g0.w == nullptr)
         k_degrees<true><<<grid, 256, 0, st>>>((int)n, g->g0.rp, g->g0.col, g->g0.w, g->d0, g->s0, mx);
@@ -1952,14 +1966,15 @@ static void finish_graph(gala_graph_s* g) {
     CK(cudaMemsetAsync(ticket, 0, sizeof(ull), st));
     k_sum_i128<<<grid_for(n, 256, big), 256, 0, st>>>(n, g->d0, part, ticket, wsum);
     CKL();
-    ull hm[3];
+    ull hm[4];
     i128 hW = 0;
-    CK(cudaMemcpyAsync(hm, mx, 3 * sizeof(ull), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(hm, mx, 4 * sizeof(ull), cudaMemcpyDeviceToHost, st));
     CK(cudaMemcpyAsync(&hW, wsum, sizeof(i128), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
     g->maxdeg0 = (int64_t)hm[0];
     g->maxw0 = (int64_t)hm[1];
     g->rows_distinct0 = (hm[2] == 0);
+    g->self0 = (hm[3] != 0);
     dfree(mx, st);
     dfree(part, st);
     dfree(ticket, st);

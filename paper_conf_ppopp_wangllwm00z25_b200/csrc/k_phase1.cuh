@@ -74,6 +74,7 @@ __global__ void k_degrees(int n, const int64_t* __restrict__ rp, const int32_t* 
         if (lane == 0) {
             d[v] = dv;
             s[v] = sv;
+            if (sv) maxdeg[3] = 1;   // some self-loop: the level's s(v) are not all zero
             if ((ull)(e - b) > mymax) mymax = (ull)(e - b);
         }
     }
@@ -256,6 +257,7 @@ __global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr,
     long long total = 0;
 #pragma unroll
     for (int b = 0; b < NBINS; ++b) { cnt[b] = (long long)ctr->bin_count[b]; total += cnt[b]; }
+    if ((long long)blockIdx.x * AP_BT >= total) return;   // no queued vertex for this block
     const int iter_id = carry->iter;
     const int lane = lane_id();
     ull my_deg = 0, my_fn = 0, my_fp = 0;
@@ -559,10 +561,16 @@ __global__ void __launch_bounds__(BT) k_reduce(int n, int dlo, int dhi, const in
         if (sg > 0 && sg < mn) mn = sg;
     }
     v = dlo + (long long)blockIdx.x * BT + threadIdx.x;
-    for (; v + 3 * stride < dhi; v += 4 * stride)
-        dc += dp[v] + dp[v + stride] + dp[v + 2 * stride] + dp[v + 3 * stride] + s[v] + s[v + stride] +
-              s[v + 2 * stride] + s[v + 3 * stride];
-    for (; v < dhi; v += stride) dc += dp[v] + s[v];
+    if (s) {
+        for (; v + 3 * stride < dhi; v += 4 * stride)
+            dc += dp[v] + dp[v + stride] + dp[v + 2 * stride] + dp[v + 3 * stride] + s[v] + s[v + stride] +
+                  s[v + 2 * stride] + s[v + 3 * stride];
+        for (; v < dhi; v += stride) dc += dp[v] + s[v];
+    } else {   // level without self-loops (s == 0): only d'
+        for (; v + 3 * stride < dhi; v += 4 * stride)
+            dc += dp[v] + dp[v + stride] + dp[v + 2 * stride] + dp[v + 3 * stride];
+        for (; v < dhi; v += stride) dc += dp[v];
+    }
     const int lane = lane_id(), wib = threadIdx.x >> 5;
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {

@@ -309,3 +309,12 @@ def test_torch_allocator_hook():
             assert np.array_equal(h.communities(), o.labels)
     finally:
         gala.set_allocator()
+
+
+def test_block_split_across_handles_graph_mode():
+    """A handle with a small block_split (small short-row arena) followed by one with the default
+    split, both in graph mode: the second handle's block kernels must get their own dynamic
+    shared-memory limit (the limit is a process-wide, per-function attribute)."""
+    assert_parity(gg.make("lfr_small"), labels=False, block_split=64)
+    assert_parity(gg.make("lfr_small"), labels=False, block_split=100, force_i128=1)
+    assert_parity(gg.make("lfr_small"), labels=False)
