@@ -20,7 +20,8 @@ import re
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libgala.so")
+# GALA_LIB_PATH: another in-tree build of the same library (tools/ab.py build-variant A/B only)
+LIB_PATH = os.environ.get("GALA_LIB_PATH") or os.path.join(_HERE, "libgala.so")
 HEADER_PATH = os.path.join(os.path.dirname(_HERE), "include", "gala.h")
 
 STATUS = {0: "GALA_OK", 1: "GALA_E_INVALID", 2: "GALA_E_OVERFLOW", 3: "GALA_E_NOMEM", 4: "GALA_E_CUDA",

@@ -112,7 +112,7 @@ struct gala_graph_s {
     int opt_agg_bound = 1;
     bool rows_distinct0 = false;   // level-0 rows strictly increasing (no duplicate entries)
     bool self0 = true;             // level 0 has a self-loop (s0 not all zero)
-    int32_t* rev0 = nullptr;       // level-0 reverse-entry index (enables the per-entry community array)
+    bool ckey_ok = false;          // level 0 may use the per-entry neighbour-community array (ckey)
     int opt_ckey = 0;
     int bins[NBINS - 1] = {4, 8, 16, 32, 128, 512, 16384};
     int hub_smem_slots = 8192;
@@ -470,7 +470,7 @@ struct Work {
 // ------------------------------------------------------------------ launch helpers
 // the per-entry neighbour-community array is used on level 0 of single-GPU runs
 static bool use_ckey(const gala_graph_s* g, const Work& wk, const DevCSR& G) {
-    return g->opt_ckey && g->rev0 && wk.ckey && !g->di && G.col == g->g0.col;
+    return g->opt_ckey && g->ckey_ok && wk.ckey && !g->di && G.col == g->g0.col;
 }
 
 // pruning strategy state of a run; the SM / RM history arrays are allocated on first use
@@ -745,7 +745,7 @@ static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, typename
     const bool ck = use_ckey(g, wk, G);
     k_dp_delta<UNIT><<<big, 256, 0, st>>>(wk.ctr, G.rp, G.col, G.w, wk.C, wk.mv_v, wk.mv_old, wk.mv_chunk, wk.stamp, wk.dp,
                                           wk.carry, G.nnz, g->opt_delta, 1, 2, ck ? wk.ckey : nullptr,
-                                          ck ? g->rev0 : nullptr, ps.rmflag, n);
+                                          nullptr, ps.rmflag, n);
     CKL();
     k_dp_full<UNIT><<<grid_for((G.nnz + 127) / 128 * 32, 256, big), 256, 0, st>>>(wk.ctr, G.nnz, G.row, G.col, G.w,
                                                                                  wk.C, wk.dp, g->opt_delta, 1, 2,
@@ -1226,7 +1226,7 @@ static void ensure_workspace(gala_graph_s* g) {
             wk.mv_chunk = dalloc<int32_t>(icap, st);
             wk.nextC = dalloc<int32_t>(wk.ncap, st);
             wk.queues = dalloc<QRec>((size_t)wk.ncap * (NBINS / 2), st);
-            if (g->rev0) wk.ckey = dalloc<int32_t>(g->nnz0, st);
+            if (g->ckey_ok) wk.ckey = dalloc<int32_t>(g->nnz0, st);
             wk.Sig = dalloc<int64_t>(wk.ncap, st);
             wk.d = dalloc<int64_t>(wk.ncap, st);
             wk.s = dalloc<int64_t>(wk.ncap, st);
@@ -1894,9 +1894,8 @@ static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_level
 static void init_graph_common(gala_graph_s* g, int64_t n, int device, uintptr_t stream) {
     g->device = device;
     CK(cudaSetDevice(device));
-    cudaDeviceProp prop;
-    CK(cudaGetDeviceProperties(&prop, device));
-    g->num_sms = prop.multiProcessorCount;
+    // one attribute query (cudaGetDeviceProperties fills the whole struct: milliseconds per handle)
+    CK(cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, device));
     if (stream) {
         g->stream = reinterpret_cast<cudaStream_t>(stream);
         g->own_stream = false;
@@ -1982,20 +1981,9 @@ static void finish_graph(gala_graph_s* g) {
     if (n == 0) hW = 0;
     if (hW >= ((i128)1 << 62)) { set_err(GALA_E_OVERFLOW, "total weight W >= 2^62"); throw GalaError{GALA_E_OVERFLOW}; }
     g->W = (int64_t)hW;
-    // reverse-entry index for the per-entry neighbour-community array (single GPU, sorted rows)
-    if (!g->di && g->rows_distinct0 && g->g0.nnz > 0 && g->g0.nnz < ((int64_t)1 << 31)) {
-        g->rev0 = dalloc<int32_t>(g->g0.nnz, st);
-        ull* bad = dalloc<ull>(1, st);
-        CK(cudaMemsetAsync(bad, 0, sizeof(ull), st));
-        k_reverse_entries<<<grid_for(g->g0.nnz, 256, big), 256, 0, st>>>(g->g0.nnz, g->g0.rp, g->g0.row, g->g0.col,
-                                                                         g->rev0, bad);
-        CKL();
-        ull hb = 0;
-        CK(cudaMemcpyAsync(&hb, bad, sizeof(ull), cudaMemcpyDeviceToHost, st));
-        CK(cudaStreamSynchronize(st));
-        dfree(bad, st);
-        if (hb) dfree(g->rev0, st);   // not symmetric: keep gathering C[col] in the decide kernels
-    }
+    // per-entry neighbour communities (ckey[e] = C[col[e]], rewritten by every full d' pass and
+    // invalidated by a delta pass) need no reverse-entry index: single GPU, sorted rows, int32 entry ids
+    g->ckey_ok = !g->di && g->rows_distinct0 && g->g0.nnz > 0 && g->g0.nnz < ((int64_t)1 << 31);
 }
 
 #define API_BEGIN try {
@@ -2217,7 +2205,6 @@ void gala_graph_free(gala_graph g) {
         dfree(g->g0.col, st);
         dfree(g->g0.w, st);
         dfree(g->g0.row, st);
-        dfree(g->rev0, st);
         dfree(g->d0, st);
         dfree(g->s0, st);
         dfree(g->lab, st);

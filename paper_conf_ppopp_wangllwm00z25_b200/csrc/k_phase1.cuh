@@ -674,18 +674,3 @@ __global__ void k_ckey_init(long long nnz, const int32_t* __restrict__ row, cons
         ckey[e] = col[e] == row[e] ? -1 : col[e];
 }
 
-// reverse entry of every CSR entry (rows sorted, distinct): rev[e] = position of
-// (col[e], row[e]) in row col[e]; *bad != 0 if some reverse entry is missing
-__global__ void k_reverse_entries(long long nnz, const int64_t* __restrict__ rp, const int32_t* __restrict__ row,
-                                  const int32_t* __restrict__ col, int32_t* __restrict__ rev, ull* __restrict__ bad) {
-    for (long long e = (long long)blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += (long long)gridDim.x * blockDim.x) {
-        const int v = row[e], u = col[e];
-        long long lo = rp[u], hi = rp[u + 1];
-        while (lo < hi) {
-            long long mid = (lo + hi) >> 1;
-            if (col[mid] < v) lo = mid + 1; else hi = mid;
-        }
-        if (lo < rp[u + 1] && col[lo] == v) rev[e] = (int32_t)lo;
-        else { rev[e] = 0; atomicAdd(bad, 1ull); }
-    }
-}
