@@ -19,6 +19,9 @@ for i in range(6):
     k = ctypes.c_int64()
     gala._check(L.gala_get_communities(hh, lab.data_ptr(), g.n, ctypes.byref(k)))
     torch.cuda.synchronize(); t3 = time.perf_counter()
+    view = gala.Graph(hh, g.n)
+    dev_ms = view.stats().get("run_ms", float("nan"))   # device time of the run
+    view._h = None                                      # a view: freed below through the C ABI
     L.gala_graph_free(hh)
     torch.cuda.synchronize(); t4 = time.perf_counter()
-    print(f"create {1e3*(t1-t0):7.2f} ms  run {1e3*(t2-t1):7.2f}  labels {1e3*(t3-t2):6.2f}  free {1e3*(t4-t3):6.2f}", flush=True)
+    print(f"create {1e3*(t1-t0):7.2f} ms  run {1e3*(t2-t1):7.2f}  (device {dev_ms:7.2f})  labels {1e3*(t3-t2):6.2f}  free {1e3*(t4-t3):6.2f}", flush=True)
