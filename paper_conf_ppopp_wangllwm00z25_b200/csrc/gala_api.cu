@@ -283,6 +283,27 @@ static thread_local DevCache* g_cache = nullptr;
 // create/run/free cycles (e2e) do not map fresh physical pages each time.
 static std::mutex g_stash_mu;
 static std::map<int, DevCache*> g_stash;
+
+// Process-wide stash of the small pinned host buffers of a run workspace (device log and carry
+// mirrors): cudaMallocHost / cudaFreeHost cost milliseconds and synchronise the device, once per
+// handle otherwise (the e2e create -> run -> free cycle).
+static std::mutex g_pin_mu;
+static std::multimap<size_t, void*> g_pin;
+static void* pin_get(size_t n) {
+    {
+        std::lock_guard<std::mutex> lk(g_pin_mu);
+        auto it = g_pin.find(n);
+        if (it != g_pin.end()) { void* p = it->second; g_pin.erase(it); return p; }
+    }
+    void* p = nullptr;
+    if (cudaMallocHost(&p, n) != cudaSuccess) return nullptr;
+    return p;
+}
+static void pin_put(void* p, size_t n) {
+    if (!p) return;
+    std::lock_guard<std::mutex> lk(g_pin_mu);
+    g_pin.emplace(n, p);
+}
 static bool cache_has_user_blocks(const DevCache* c) {
     for (auto& kv : c->sz)
         if (kv.second.ua.alloc) return true;
@@ -448,8 +469,8 @@ struct Work {
         dfree(part, st);
         hw.part = nullptr;
         hub_ncap = hub_tcap = hub_lcap = hub_pcap = 0;
-        if (h_log) cudaFreeHost(h_log);
-        if (h_carry) cudaFreeHost(h_carry);
+        pin_put(h_log, sizeof(IterLog) * (size_t)log_cap);
+        pin_put(h_carry, sizeof(Carry));
         h_log = nullptr;
         h_carry = nullptr;
     }
@@ -1238,8 +1259,9 @@ static void ensure_workspace(gala_graph_s* g) {
             wk.part_dc = dalloc<long long>(wk.reduce_grid, st);
             wk.part_min = dalloc<long long>(wk.reduce_grid, st);
             wk.part_s2 = dalloc<i128>(wk.reduce_grid, st);
-            CK(cudaMallocHost(&wk.h_log, sizeof(IterLog) * wk.log_cap));
-            CK(cudaMallocHost(&wk.h_carry, sizeof(Carry)));
+            wk.h_log = static_cast<IterLog*>(pin_get(sizeof(IterLog) * (size_t)wk.log_cap));
+            wk.h_carry = static_cast<Carry*>(pin_get(sizeof(Carry)));
+            if (!wk.h_log || !wk.h_carry) { set_err(GALA_E_NOMEM, "pinned host buffers"); throw GalaError{GALA_E_NOMEM}; }
             for (int i = 0; i < 5; ++i) CK(cudaEventCreate(&wk.ev[i]));
             // dynamic shared memory opt-ins, once per workspace
             int per_sm = 0;
@@ -2198,8 +2220,18 @@ void gala_graph_free(gala_graph g) {
     PoolScope pool_scope(g->cache);
     const bool dist = g->di != nullptr;
     if (g->di) { delete g->di; g->di = nullptr; }   // communicators are cached (comm_for)
+    // GALA_DEBUG_FREE=1: host time of each teardown step on stderr (e2e create/run/free cycles)
+    static const bool dbg = getenv("GALA_DEBUG_FREE") != nullptr;
+    auto t_prev = std::chrono::steady_clock::now();
+    auto lap = [&](const char* what) {
+        if (!dbg) return;
+        const auto t = std::chrono::steady_clock::now();
+        fprintf(stderr, "[gala free] %-10s %8.3f ms\n", what, std::chrono::duration<double, std::milli>(t - t_prev).count());
+        t_prev = t;
+    };
     cudaStream_t st = g->stream;
     if (g->wk) { g->wk->release(); delete g->wk; g->wk = nullptr; }
+    lap("workspace");
     if (st) {
         dfree(g->g0.rp, st);
         dfree(g->g0.col, st);
@@ -2209,6 +2241,7 @@ void gala_graph_free(gala_graph g) {
         dfree(g->s0, st);
         dfree(g->lab, st);
         cudaStreamSynchronize(st);
+        lap("graph+sync");
         // park the idle cache for the next handle on this device (not when it holds blocks of a
         // user allocator: those go back to their owner now)
         if (g->cache && !dist && !cache_has_user_blocks(g->cache) && cudaGetLastError() == cudaSuccess) {
@@ -2218,19 +2251,23 @@ void gala_graph_free(gala_graph g) {
                 g->cache = nullptr;
             }
         }
+        lap(g->cache ? "not parked" : "parked");
         if (g->cache) g->cache->trim(st);
         cudaStreamSynchronize(st);
         if (g->own_stream) cudaStreamDestroy(st);
+        lap("trim");
     }
     for (int i = 0; i < 4; ++i) {
         if (g->side[i]) cudaStreamDestroy(g->side[i]);
         if (g->ev_join[i]) cudaEventDestroy(g->ev_join[i]);
     }
     if (g->ev_fork) cudaEventDestroy(g->ev_fork);
+    lap("streams");
     if (g->cache) {
         if (g->cache->pool) cudaMemPoolDestroy(g->cache->pool);
         delete g->cache;
     }
+    lap("pool");
     g_cache = pool_scope.prev == mine ? nullptr : pool_scope.prev;
     pool_scope.prev = g_cache;
     delete g;

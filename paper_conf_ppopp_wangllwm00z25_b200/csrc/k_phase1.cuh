@@ -530,6 +530,9 @@ __device__ __forceinline__ void record_iteration(const IterCounters* ctr, Carry*
 }
 
 // ---------------------------------------------------------------------------
+#ifndef GALA_REDUCE_U
+#define GALA_REDUCE_U 4   // (<= 64 registers: 4 blocks per SM) Sigma_tot / d' values per thread per batch in k_reduce (0: the strided loops)
+#endif
 template <int BT>
 __global__ void __launch_bounds__(BT) k_reduce(int n, int dlo, int dhi, const int64_t* __restrict__ dp,
                                                const int64_t* __restrict__ s, const int64_t* __restrict__ Sig,
@@ -546,6 +549,26 @@ __global__ void __launch_bounds__(BT) k_reduce(int n, int dlo, int dhi, const in
     long long dc = 0, mn = LLONG_MAX;
     i128 s2 = 0;
     const long long stride = (long long)gridDim.x * BT;
+#if GALA_REDUCE_U > 0
+    // every load of a batch (U Sigma_tot and U d' (+ s) values per thread) issued before any use:
+    // one memory latency per batch instead of one per tail element (latency-bound kernel)
+    for (long long v0 = (long long)blockIdx.x * BT + threadIdx.x; v0 < n; v0 += GALA_REDUCE_U * stride) {
+        long long g[GALA_REDUCE_U], q[GALA_REDUCE_U], r[GALA_REDUCE_U];
+#pragma unroll
+        for (int k = 0; k < GALA_REDUCE_U; ++k) {
+            const long long v = v0 + k * stride, x = dlo + v;
+            g[k] = v < n ? Sig[v] : 0;
+            q[k] = x < dhi ? dp[x] : 0;
+            r[k] = (s && x < dhi) ? s[x] : 0;
+        }
+#pragma unroll
+        for (int k = 0; k < GALA_REDUCE_U; ++k) {
+            s2 += (i128)g[k] * g[k];
+            if (g[k] > 0 && g[k] < mn) mn = g[k];
+            dc += q[k] + r[k];
+        }
+    }
+#else
     long long v = (long long)blockIdx.x * BT + threadIdx.x;
     for (; v + 3 * stride < n; v += 4 * stride) {
         long long g0 = Sig[v], g1 = Sig[v + stride], g2 = Sig[v + 2 * stride], g3 = Sig[v + 3 * stride];
@@ -571,6 +594,7 @@ __global__ void __launch_bounds__(BT) k_reduce(int n, int dlo, int dhi, const in
             dc += dp[v] + dp[v + stride] + dp[v + 2 * stride] + dp[v + 3 * stride];
         for (; v < dhi; v += stride) dc += dp[v];
     }
+#endif
     const int lane = lane_id(), wib = threadIdx.x >> 5;
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
