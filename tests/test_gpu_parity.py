@@ -318,3 +318,15 @@ def test_block_split_across_handles_graph_mode():
     assert_parity(gg.make("lfr_small"), labels=False, block_split=64)
     assert_parity(gg.make("lfr_small"), labels=False, block_split=100, force_i128=1)
     assert_parity(gg.make("lfr_small"), labels=False)
+
+
+def test_handle_cycles_reuse_pinned_and_pool():
+    """create -> run -> free cycles (the e2e pattern) with alternating device-log capacities: the
+    next handle adopts the parked device pool and the stashed pinned mirrors (a mirror of another
+    size must not be handed out), and every cycle stays bit-exact."""
+    g = gg.make("lfr_small")
+    o = oracle.louvain(g, prune=1, trace=1)
+    for cap in (4096, 3, 4096, 2, 3):
+        r = run_gpu(g, trace=1, log_cap=cap)
+        assert np.array_equal(r["labels"], o.labels)
+        assert r["N"] == o.N and len(r["trace"]) == len(o.records)
