@@ -116,6 +116,9 @@ struct BinThresholds {
 #define PB_BT 256
 #define PB_IPT 4
 
+#ifndef GALA_PRUNE_EAGER
+#define GALA_PRUNE_EAGER 0   // 1: row bounds + community size loaded up front (A/B: slower, 0.63 -> 0.67 ms on lfr1m; profiles/r01j_ab_prune.txt)
+#endif
 #ifndef GALA_PRUNE_MINB
 #define GALA_PRUNE_MINB 4   // <= 64 registers: one wave of 1024-vertex tiles (A/B: lfr1m 0.76 -> 0.64 ms)
 #endif
@@ -150,8 +153,26 @@ __global__ void __launch_bounds__(PB_BT, GALA_PRUNE_MINB) k_prune_bin(int vlo, i
             cv[j] = ok ? C[v] : 0;
         }
         long long sg[PB_IPT];
+#if GALA_PRUNE_EAGER
+        // row bounds and the community size loaded with the vertex state / Sigma_tot gather (one
+        // dependent round fewer for queued vertices; the extra bytes are coalesced or L2 hits)
+        long long rb[PB_IPT], re[PB_IPT];
+        int szv[PB_IPT];
+#pragma unroll
+        for (int j = 0; j < PB_IPT; ++j) {
+            long long v = t0 + (long long)j * PB_BT + threadIdx.x;
+            rb[j] = v < n ? rp[v] : 0;
+            re[j] = v < n ? rp[v + 1] : 0;
+        }
+#pragma unroll
+        for (int j = 0; j < PB_IPT; ++j) {
+            sg[j] = dv[j] > 0 ? Sig[cv[j]] : 0;
+            szv[j] = dv[j] > 0 ? size[cv[j]] : 0;
+        }
+#else
 #pragma unroll
         for (int j = 0; j < PB_IPT; ++j) sg[j] = dv[j] > 0 ? Sig[cv[j]] : 0;
+#endif
         int deg[PB_IPT];
         long long beg[PB_IPT];
 #pragma unroll
@@ -174,8 +195,13 @@ __global__ void __launch_bounds__(PB_BT, GALA_PRUNE_MINB) k_prune_bin(int vlo, i
                 act[j] = active;
                 if (active) { my_active++; } else { my_pruned++; }
                 if (active || ps.instr) {
+#if GALA_PRUNE_EAGER
+                    beg[j] = rb[j];
+                    long long dg = re[j] - rb[j];
+#else
                     beg[j] = rp[v];
                     long long dg = rp[v + 1] - beg[j];
+#endif
                     deg[j] = (int)(dg > INT_MAX ? INT_MAX : dg);
                     int b = NBINS - 1;
 #pragma unroll
@@ -186,9 +212,11 @@ __global__ void __launch_bounds__(PB_BT, GALA_PRUNE_MINB) k_prune_bin(int vlo, i
                 }
             }
         }
+#if !GALA_PRUNE_EAGER
         int szv[PB_IPT];
 #pragma unroll
         for (int j = 0; j < PB_IPT; ++j) szv[j] = bin[j] >= 0 ? size[cv[j]] : 0;
+#endif
         bool anyq = false;
 #pragma unroll
         for (int j = 0; j < PB_IPT; ++j) anyq |= bin[j] >= 0;
