@@ -558,6 +558,9 @@ __device__ __forceinline__ void record_iteration(const IterCounters* ctr, Carry*
 }
 
 // ---------------------------------------------------------------------------
+#ifndef GALA_REDUCE_PTAIL
+#define GALA_REDUCE_PTAIL 1   // last block copies / clears the iteration counters with all its threads
+#endif
 #ifndef GALA_REDUCE_U
 #define GALA_REDUCE_U 4   // (<= 64 registers: 4 blocks per SM) Sigma_tot / d' values per thread per batch in k_reduce (0: the strided loops)
 #endif
@@ -574,6 +577,7 @@ __global__ void __launch_bounds__(BT) k_reduce(int n, int dlo, int dhi, const in
     __shared__ i128 sh_s2[BT / 32];
     __shared__ long long sh_min[BT / 32];
     __shared__ bool amLast;
+    __shared__ int s_tail, s_slot;
     long long dc = 0, mn = LLONG_MAX;
     i128 s2 = 0;
     const long long stride = (long long)gridDim.x * BT;
@@ -678,10 +682,10 @@ __global__ void __launch_bounds__(BT) k_reduce(int n, int dlo, int dhi, const in
         carry->S2_lo = lo128(ts2);
         carry->minSig = tmn;
         carry->sumDC = tdc;
+        s_tail = 0;
         if (mode & 2) {   // multi-GPU: sumDC is rank-local; k_finish completes after the all-reduce
             ctr->ticket = 0;
-            return;
-        }
+        } else {
         i128 qW = mk128(qW_hi, qW_lo);
         i128 Nn = qW * (i128)tdc - (i128)p * ts2;
         i128 N = mk128(carry->N_hi, carry->N_lo);
@@ -699,11 +703,41 @@ __global__ void __launch_bounds__(BT) k_reduce(int n, int dlo, int dhi, const in
         carry->converged = conv;
         ctr->ticket = 0;
         if (log) {   // k_record fused: log the iteration, advance, set the loop condition, clear counters
+#if GALA_REDUCE_PTAIL
+            // the counter copy into the log and the clear are done by the whole block below
+            const int it = carry->iter;
+            const int slot = it - carry->log_base;
+            s_slot = (slot >= 0 && slot < log_cap) ? slot : -1;
+            if (s_slot >= 0) {
+                IterLog& L = log[slot];
+                L.N_hi = carry->N_hi;
+                L.N_lo = carry->N_lo;
+                L.converged = carry->converged;
+            }
+            carry->iter = it + 1;
+            const int more = !carry->converged && (max_iters <= 0 || it + 1 < max_iters) && (slot + 1 < log_cap);
+            carry->more = more;
+            if (cond_handle) cudaGraphSetConditional((cudaGraphConditionalHandle)cond_handle, more ? 1u : 0u);
+            s_tail = 1;
+#else
             record_iteration(ctr, carry, log, log_cap, max_iters, cond_handle);
             ull* c = reinterpret_cast<ull*>(ctr);
             for (int i = 0; i < (int)(sizeof(IterCounters) / sizeof(ull)); ++i) c[i] = 0;
+#endif
+        }
+        }   // mode & 2
+    }
+#if GALA_REDUCE_PTAIL
+    __syncthreads();
+    if (s_tail) {   // log[slot].ctr = *ctr; *ctr = 0 -- one counter per thread (same values as record_iteration)
+        ull* c = reinterpret_cast<ull*>(ctr);
+        for (int i = threadIdx.x; i < (int)(sizeof(IterCounters) / sizeof(ull)); i += BT) {
+            const ull x = c[i];
+            if (s_slot >= 0) reinterpret_cast<ull*>(&log[s_slot].ctr)[i] = x;
+            c[i] = 0;
         }
     }
+#endif
 }
 
 // ---------------------------------------------------------------------------
