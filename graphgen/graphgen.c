@@ -273,6 +273,96 @@ static int64_t pl_draw(const double* t, int64_t lo, int64_t hi, double u) {
     return lo + l;
 }
 
+/* ------------------------------------------------------------------------ */
+/* degree-preserving rewiring of a configuration-model edge list             */
+/* ------------------------------------------------------------------------ */
+/* open-addressing set of undirected edge keys (min << 32 | max) with tombstones */
+#define ES_EMPTY (~0ULL)
+#define ES_TOMB (~1ULL)
+typedef struct { uint64_t* t; uint64_t mask; } edgeset;
+static inline uint64_t ekey(int64_t u, int64_t v) {
+    return u < v ? ((uint64_t)u << 32) | (uint64_t)v : ((uint64_t)v << 32) | (uint64_t)u;
+}
+static inline uint64_t es_slot(uint64_t k) { return mix64(k); }
+static int es_has(const edgeset* s, uint64_t k) {
+    for (uint64_t i = es_slot(k) & s->mask;; i = (i + 1) & s->mask) {
+        if (s->t[i] == k) return 1;
+        if (s->t[i] == ES_EMPTY) return 0;
+    }
+}
+static int es_insert(edgeset* s, uint64_t k) {   /* 0 if already present */
+    uint64_t tomb = ES_EMPTY;
+    for (uint64_t i = es_slot(k) & s->mask;; i = (i + 1) & s->mask) {
+        if (s->t[i] == k) return 0;
+        if (s->t[i] == ES_TOMB && tomb == ES_EMPTY) tomb = i;
+        if (s->t[i] == ES_EMPTY) { s->t[tomb != ES_EMPTY ? tomb : i] = k; return 1; }
+    }
+}
+static void es_erase(edgeset* s, uint64_t k) {
+    for (uint64_t i = es_slot(k) & s->mask;; i = (i + 1) & s->mask) {
+        if (s->t[i] == k) { s->t[i] = ES_TOMB; return; }
+        if (s->t[i] == ES_EMPTY) return;
+    }
+}
+
+/*
+ * Edges [0, n_int) are internal, grouped by community (community j owns
+ * [ioff[j], ioff[j+1])); edges [n_int, ne) are external.  An edge is bad if it
+ * is a self pair, repeats an earlier edge, or (external) joins one community.
+ * Each bad edge (u, v), in index order, is swapped with a random good edge
+ * (c, d) of its class -> (u, d), (c, v) when both are new, distinct, non-self
+ * and (external) cross communities; every vertex keeps its internal and
+ * external degree.  Up to 256 draws per bad edge (stream 20), then it is
+ * dropped.  Sequential, so the output is a pure function of the seed.
+ * Returns the compacted edge count.
+ */
+static int64_t lfr_rewire(int64_t ne, int64_t n_int, int64_t* src, int64_t* dst, const int64_t* comm,
+                          const int64_t* ioff, uint64_t seed) {
+    uint64_t cap = 1024;
+    while (cap < (uint64_t)(2 * ne + 2)) cap <<= 1;
+    edgeset s = { (uint64_t*)malloc(cap * sizeof(uint64_t)), cap - 1 };
+    memset(s.t, 0xff, cap * sizeof(uint64_t));
+    unsigned char* bad = (unsigned char*)calloc((size_t)ne + 1, 1);
+    for (int64_t e = 0; e < ne; ++e) {
+        const int64_t u = src[e], v = dst[e];
+        if (u == v || (e >= n_int && comm[u] == comm[v]) || !es_insert(&s, ekey(u, v))) bad[e] = 1;
+    }
+    const int64_t n_ext = ne - n_int;
+    for (int64_t e = 0; e < ne; ++e) {
+        if (!bad[e]) continue;
+        const int64_t u = src[e], v = dst[e];
+        const int internal = e < n_int;
+        int64_t lo, len;
+        if (internal) { const int64_t c = comm[u]; lo = ioff[c]; len = ioff[c + 1] - lo; }
+        else { lo = n_int; len = n_ext; }
+        if (len < 2) continue;
+        for (uint64_t t = 0; t < 256; ++t) {
+            const uint64_t r = rng_u64(seed, 20, ((uint64_t)e << 8) | t);
+            const int64_t j = lo + (int64_t)((r >> 1) % (uint64_t)len);
+            if (j == e || bad[j]) continue;
+            int64_t c = src[j], d = dst[j];
+            if (r & 1) { const int64_t x = c; c = d; d = x; }
+            if (u == d || c == v) continue;
+            if (!internal && (comm[u] == comm[d] || comm[c] == comm[v])) continue;
+            const uint64_t k1 = ekey(u, d), k2 = ekey(c, v);
+            if (k1 == k2 || es_has(&s, k1) || es_has(&s, k2)) continue;
+            es_erase(&s, ekey(c, d));
+            es_insert(&s, k1);
+            es_insert(&s, k2);
+            src[e] = u; dst[e] = d;
+            src[j] = c; dst[j] = v;
+            bad[e] = 0;
+            break;
+        }
+    }
+    int64_t w = 0;
+    for (int64_t e = 0; e < ne; ++e)
+        if (!bad[e]) { src[w] = src[e]; dst[w] = dst[e]; ++w; }
+    free(bad);
+    free(s.t);
+    return w;
+}
+
 /*
  * gg_lfr: LFR-style benchmark graph.
  *   1. degrees k_i ~ discrete power law (tau1) on [kmin, kmax]; kmin is the
@@ -290,9 +380,9 @@ static int64_t pl_draw(const double* t, int64_t lo, int64_t hi, double u) {
  * removes them), membership[n] (ground truth, permuted ids).
  * Two-call protocol: if out_src == NULL returns the edge count upper bound.
  */
-int64_t gg_lfr(int64_t n, double avg_k, int64_t kmax, double tau1, double tau2,
-               int64_t cmin, int64_t cmax, double mu, uint64_t seed,
-               int64_t* out_src, int64_t* out_dst, int64_t* membership, int64_t* out_kmin) {
+int64_t gg_lfr_ex(int64_t n, double avg_k, int64_t kmax, double tau1, double tau2,
+                  int64_t cmin, int64_t cmax, double mu, uint64_t seed, int fit_frac, double alpha,
+                  int rewire, int64_t* out_src, int64_t* out_dst, int64_t* membership, int64_t* out_kmin) {
     /* 1. degrees */
     int64_t best_kmin = 1; double best_err = 1e300;
     for (int64_t km = 1; km < kmax; ++km) {
@@ -300,8 +390,32 @@ int64_t gg_lfr(int64_t n, double avg_k, int64_t kmax, double tau1, double tau2,
         if (e < best_err) { best_err = e; best_kmin = km; }
     }
     int64_t kmin = best_kmin;
+    double* tk;
+    if (fit_frac) {
+        /* exact mean: the law on [K0, kmax] with the weight of k = K0 scaled by f in (0, 1],
+           K0 the largest integer whose full law has mean <= avg_k; f by bisection */
+        int64_t k0 = 1;
+        while (k0 + 1 < kmax && pl_mean(k0 + 1, kmax, tau1) <= avg_k) ++k0;
+        double lo = 1e-9, hi = 1.0, f = 1.0;
+        double s_rest = 0, sk_rest = 0;
+        for (int64_t k = k0 + 1; k <= kmax; ++k) { double p = pow((double)k, -tau1); s_rest += p; sk_rest += p * (double)k; }
+        const double p0 = pow((double)k0, -tau1);
+        for (int it = 0; it < 200; ++it) {
+            f = 0.5 * (lo + hi);
+            const double m = (sk_rest + f * p0 * (double)k0) / (s_rest + f * p0);
+            if (m > avg_k) lo = f; else hi = f;   /* larger f -> more mass at k0 -> smaller mean */
+        }
+        kmin = k0;
+        tk = pl_table(kmin, kmax, tau1);
+        const int64_t m = kmax - kmin + 1;
+        double s = s_rest + f * p0, acc = f * p0;
+        tk[0] = acc / s;
+        for (int64_t i = 1; i < m; ++i) { acc += pow((double)(kmin + i), -tau1); tk[i] = acc / s; }
+        tk[m - 1] = 1.0;
+    } else {
+        tk = pl_table(kmin, kmax, tau1);
+    }
     if (out_kmin) *out_kmin = kmin;
-    double* tk = pl_table(kmin, kmax, tau1);
     int64_t* k = (int64_t*)malloc((size_t)n * sizeof(int64_t));
     #pragma omp parallel for
     for (int64_t i = 0; i < n; ++i) k[i] = pl_draw(tk, kmin, kmax, rng_unit(seed, 1, (uint64_t)i));
@@ -332,7 +446,8 @@ int64_t gg_lfr(int64_t n, double avg_k, int64_t kmax, double tau1, double tau2,
     int64_t* kin = (int64_t*)malloc((size_t)n * sizeof(int64_t));
     for (int64_t i = 0; i < n; ++i) {
         int64_t ki = (int64_t)llround((1.0 - mu) * (double)k[i]);
-        if (ki > maxc - 1) ki = maxc - 1;
+        const int64_t cap = (int64_t)floor(alpha * (double)(maxc - 1));
+        if (ki > cap) ki = cap;   /* the excess becomes external stubs (k_out = k - k_in) */
         kin[i] = ki;
     }
 
@@ -348,20 +463,23 @@ int64_t gg_lfr(int64_t n, double avg_k, int64_t kmax, double tau1, double tau2,
         int64_t chosen = -1;
         for (int tr = 0; tr < 64 && chosen < 0; ++tr) {
             int64_t c = (int64_t)(rng_u64(seed, 3, (uint64_t)t * 64 + (uint64_t)tr) % (uint64_t)nc);
-            if (fill[c] < csize[c] && csize[c] > kin[v]) chosen = c;
+            if (fill[c] < csize[c] && alpha * (double)(csize[c] - 1) >= (double)kin[v]) chosen = c;
         }
         if (chosen < 0) {   /* deterministic scan fallback */
             int64_t st = (int64_t)(rng_u64(seed, 3, (uint64_t)t * 64 + 63) % (uint64_t)nc);
             for (int64_t j = 0; j < nc && chosen < 0; ++j) {
                 int64_t c = (st + j) % nc;
-                if (fill[c] < csize[c] && csize[c] > kin[v]) chosen = c;
+                if (fill[c] < csize[c] && alpha * (double)(csize[c] - 1) >= (double)kin[v]) chosen = c;
             }
             if (chosen < 0) {   /* no community large enough: any with room; cap k_in */
                 for (int64_t j = 0; j < nc && chosen < 0; ++j) {
                     int64_t c = (st + j) % nc;
                     if (fill[c] < csize[c]) chosen = c;
                 }
-                if (kin[v] > csize[chosen] - 1) kin[v] = csize[chosen] - 1;
+                {
+                    const int64_t cap = (int64_t)floor(alpha * (double)(csize[chosen] - 1));
+                    if (kin[v] > cap) kin[v] = cap;   /* excess -> external stubs */
+                }
             }
         }
         comm[v] = chosen;
@@ -447,10 +565,13 @@ int64_t gg_lfr(int64_t n, double avg_k, int64_t kmax, double tau1, double tau2,
     }
     for (int64_t e = 0; e < np; ++e) {
         int64_t u = (int64_t)sv[2 * e], v = (int64_t)sv[2 * e + 1];
-        if (comm[u] == comm[v]) continue;   /* dropped after two re-pairings */
+        if (comm[u] == comm[v] && !rewire) continue;   /* dropped after two re-pairings */
         out_src[ne] = u; out_dst[ne] = v; ++ne;
     }
     free(sk); free(sv);
+    /* 5c. (rewire) degree-preserving double-edge swaps replace self pairs, duplicates and
+       external pairs inside one community instead of dropping them */
+    if (rewire) ne = lfr_rewire(ne, n_int, out_src, out_dst, comm, istub_off, seed);
 
     /* 6. permute ids */
     int64_t* perm = (int64_t*)malloc((size_t)n * sizeof(int64_t));
@@ -463,4 +584,11 @@ int64_t gg_lfr(int64_t n, double avg_k, int64_t kmax, double tau1, double tau2,
     }
     free(perm); free(k); free(kin); free(csize); free(fill); free(comm); free(coff); free(mem); free(istub_off);
     return ne;
+}
+
+/* the original entry point: integer k_min, internal degree capped at community size - 1 */
+int64_t gg_lfr(int64_t n, double avg_k, int64_t kmax, double tau1, double tau2,
+               int64_t cmin, int64_t cmax, double mu, uint64_t seed,
+               int64_t* out_src, int64_t* out_dst, int64_t* membership, int64_t* out_kmin) {
+    return gg_lfr_ex(n, avg_k, kmax, tau1, tau2, cmin, cmax, mu, seed, 0, 1.0, 0, out_src, out_dst, membership, out_kmin);
 }
