@@ -43,6 +43,8 @@ def _lib():
         lib.oracle_record.argtypes = [p, i64, p]
         lib.oracle_record_labels.restype = ctypes.c_int
         lib.oracle_record_labels.argtypes = [p, i64, p]
+        lib.oracle_record_pruned.restype = ctypes.c_int
+        lib.oracle_record_pruned.argtypes = [p, i64, p]
         lib.oracle_level.restype = None
         lib.oracle_level.argtypes = [p, i64, p]
         lib.oracle_free.restype = None
@@ -84,6 +86,7 @@ class IterRecord:
     N: int
     labels: np.ndarray | None
     n_fp: int = 0
+    pruned: np.ndarray | None = None   # trace >= 3: per-vertex inactive flags (bool)
 
 
 @dataclass
@@ -125,7 +128,8 @@ def louvain(g, gamma: float = 1.0, tol: float = 1e-6, max_levels: int = 0, max_i
 
     prune: 0/False none, 1/True MG (Eq. 6/7), 2 SM, 3 RM, 4 MG+RM (§3.2-3.3; DESIGN.md c20/c21).
     check: also evaluate pruned vertices -> per-iteration false negatives (n_fn) and, for the
-    active set, false positives (n_fp) in the records."""
+    active set, false positives (n_fp) in the records.
+    trace: 1 records, 2 + label snapshots, 3 + per-vertex inactive flags (IterRecord.pruned)."""
     lib = _lib()
     rp, col, w = _csr_arrays(g)
     h = lib.oracle_louvain(g.n, _ptr(rp), _ptr(col), _ptr(w), gamma, tol, max_levels, max_iters,
@@ -141,11 +145,16 @@ def louvain(g, gamma: float = 1.0, tol: float = 1e-6, max_levels: int = 0, max_i
         for i in range(int(summ[6])):
             lib.oracle_record(h, i, _ptr(buf))
             lab = None
+            pf = None
             if trace >= 2:
                 lab = np.zeros(int(buf[2]), dtype=np.int32)
                 lib.oracle_record_labels(h, i, _ptr(lab))
+            if trace >= 3:
+                pf = np.zeros(int(buf[2]), dtype=np.uint8)
+                lib.oracle_record_pruned(h, i, _ptr(pf))
+                pf = pf.astype(bool)
             recs.append(IterRecord(int(buf[0]), int(buf[1]), int(buf[2]), int(buf[3]), int(buf[4]),
-                                   int(buf[5]), int(buf[6]), _i128(buf[7], buf[8]), lab, int(buf[9])))
+                                   int(buf[5]), int(buf[6]), _i128(buf[7], buf[8]), lab, int(buf[9]), pf))
         levs = []
         lb = np.zeros(7, dtype=np.int64)
         for i in range(int(summ[5])):

@@ -47,6 +47,7 @@ typedef struct {
     int64_t n_level, n_active, n_pruned, n_moved, n_fn, n_fp;
     i128 N;
     int32_t* labels; /* level-local community of every level vertex after the iteration */
+    unsigned char* pruned; /* trace >= 3: 1 iff the pruning rule made the vertex inactive */
 } orc_rec;
 
 typedef struct {
@@ -227,7 +228,8 @@ static void coarsen(const ograph* g, const int32_t* newid, int64_t k, ograph* ou
  *   check      : also evaluate pruned vertices and count those that would have
  *                moved (false negatives, Eq. 3 / P:147) and the active vertices
  *                that stay (false positives); pruned vertices still stay
- *   trace      : 0 none, 1 per-iteration records, 2 records + label snapshots
+ *   trace      : 0 none, 1 per-iteration records, 2 records + label snapshots,
+ *                3 also the per-vertex inactive flags of every iteration
  *   max_iters  : per-level iteration cap (0 = none; honoured identically by the library)
  * Returns an opaque result (free with oracle_free).  status != 0 on error.
  */
@@ -318,6 +320,7 @@ void* oracle_louvain(int64_t n, const int64_t* row_ptr, const int32_t* col, cons
             int64_t minSig = INT64_MAX;
             for (int64_t c = 0; c < nl; ++c) if (Sig[c] > 0 && Sig[c] < minSig) minSig = Sig[c];
             int64_t n_active = 0, n_pruned = 0, n_fn = 0, n_fp = 0, bad = 0;
+            unsigned char* pflag = trace >= 3 ? (unsigned char*)calloc((size_t)nl + 1, 1) : NULL;
             /* Alg. 1 lines 3-4: every vertex decides from the start-of-iteration state */
             #pragma omp parallel for schedule(dynamic, 256) reduction(+:n_active, n_pruned, n_fn, n_fp, bad)
             for (int64_t v = 0; v < nl; ++v) {
@@ -341,6 +344,7 @@ void* oracle_louvain(int64_t n, const int64_t* row_ptr, const int32_t* col, cons
                         if (G.col[e] != v && moved_prev[G.col[e]]) nb_moved = 1;
                     if (!nb_moved) pruned = 1;   /* MG+RM: pruned by either rule */
                 }
+                if (pruned && pflag) pflag[v] = 1;
                 if (pruned && !check) { n_pruned++; continue; }
                 int64_t d_own = 0;
                 int32_t b = decide(&G, v, C, Sig, size, d, dp, W, p, q, bufs[omp_get_thread_num()], &d_own);
@@ -385,13 +389,14 @@ void* oracle_louvain(int64_t n, const int64_t* row_ptr, const int32_t* col, cons
                 x.level = level; x.iter = it; x.n_level = nl;
                 x.n_active = n_active; x.n_pruned = n_pruned; x.n_moved = n_moved; x.n_fn = n_fn;
                 x.n_fp = check ? n_fp : 0;
-                x.N = Nn; x.labels = NULL;
+                x.N = Nn; x.labels = NULL; x.pruned = pflag; pflag = NULL;
                 if (trace >= 2) {
                     x.labels = (int32_t*)malloc((size_t)nl * sizeof(int32_t));
                     memcpy(x.labels, C, (size_t)nl * sizeof(int32_t));
                 }
                 push_rec(R, x);
             }
+            free(pflag);
             /* Alg. 1 lines 12-13: Delta Q < theta (moves of this iteration are kept, c6) */
             int converged = (n_moved == 0) || (Nn - N < thr);
             N = Nn;
@@ -482,6 +487,12 @@ int oracle_record_labels(void* h, int64_t i, int32_t* out) {
     memcpy(out, x->labels, (size_t)x->n_level * sizeof(int32_t));
     return 0;
 }
+int oracle_record_pruned(void* h, int64_t i, unsigned char* out) {
+    orc_rec* x = &((orc_result*)h)->rec[i];
+    if (!x->pruned) return 1;
+    memcpy(out, x->pruned, (size_t)x->n_level);
+    return 0;
+}
 /* level: n, nnz, iters, Nstart_hi, Nstart_lo, Nend_hi, Nend_lo */
 void oracle_level(void* h, int64_t i, int64_t* out) {
     orc_level* L = &((orc_result*)h)->lev[i];
@@ -493,7 +504,7 @@ void oracle_level(void* h, int64_t i, int64_t* out) {
 void oracle_free(void* h) {
     orc_result* R = (orc_result*)h;
     if (!R) return;
-    for (int64_t i = 0; i < R->nrec; ++i) free(R->rec[i].labels);
+    for (int64_t i = 0; i < R->nrec; ++i) { free(R->rec[i].labels); free(R->rec[i].pruned); }
     free(R->rec); free(R->lev); free(R->lab); free(R);
 }
 
