@@ -303,7 +303,8 @@ class Graph:
             r = dict(level=int(buf[0]), iter=int(buf[1]), n_level=int(buf[2]), n_active=int(buf[3]),
                      n_pruned=int(buf[4]), n_moved=int(buf[5]), N=_i128(buf[6], buf[7]),
                      edges_scanned=int(buf[8]), distinct=int(buf[9]), delta_used=int(buf[10]),
-                     n_fn=int(buf[12]), n_fp=int(buf[13]))
+                     sync=int(buf[11]), n_fn=int(buf[12]), n_fp=int(buf[13]), us=int(buf[14]) / 1e3,
+                     alg_bytes=int(buf[15]))
             if labels:
                 lab = np.zeros(r["n_level"], dtype=np.int32)
                 _check(L.gala_get_trace_labels(self._h, i, _np_ptr(lab), r["n_level"]))

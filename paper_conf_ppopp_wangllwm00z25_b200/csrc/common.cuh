@@ -98,6 +98,7 @@ struct Carry {
     int log_base;           // log slot of iteration `log_base` is 0
     int ckey_valid;         // the per-entry community array matches C (set by full d' passes)
     int pad2;
+    ull t_ns;               // %globaltimer at the end of the last reduction (level start / iteration end)
 };
 
 // One record per phase-1 iteration, written on the device by k_record.
@@ -107,7 +108,14 @@ struct IterLog {
     ull N_lo;
     int converged;
     int pad;
+    ull t_ns;   // %globaltimer when the iteration's reduction finished (per-iteration device timing)
 };
+
+__device__ __forceinline__ ull globaltimer_ns() {
+    ull t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
 
 __device__ __forceinline__ i128 mk128(long long hi, ull lo) {
     return (i128)(((unsigned __int128)(ull)hi << 64) | (unsigned __int128)lo);

@@ -90,6 +90,8 @@ struct LevelStat {
     int i128path;
     double ms_phase1, ms_phase2;
     int64_t edges_scanned, nominal_edges;
+    double alg_bytes;   // algorithmic bytes of the level's phase-1 iterations
+    double ms_iters;    // device time of the level's iterations (globaltimer, first reduce -> last reduce)
 };
 
 struct gala_graph_s {
@@ -1381,6 +1383,7 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
             CK(cudaMemcpyAsync(wk.h_carry, wk.carry, sizeof(Carry), cudaMemcpyDeviceToHost, st));
             CK(cudaStreamSynchronize(st));
             const i128 N_start = carry_N(wk.h_carry);
+            const ull t_level = wk.h_carry->t_ns;
             // gain arithmetic for this level (reading c16):
             //   |score| <= max(p,q) * W * dmax  (dmax = max weighted degree of the level)
             //   int64 iff that bound < 2^62; packed (score,-c) keys iff < 2^(62 - idbits); the
@@ -1406,9 +1409,16 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
                 else phase1_level<DM_FAST, false>(g, wk, cur, qW64, p64, qW128, T, tm, maxdeg, idbits, logs, level, level > 0 || g->rows_distinct0);
             }
             i128 N = N_start;
+            ull t_prev = t_level;
             for (size_t it = 0; it < logs.size(); ++it) {
                 const IterCounters& c = logs[it].ctr;
+                double b0 = 0, b1 = 0;
+                for (int i = 0; i < KC_COUNT; ++i) b0 += g->kc_bytes[i];
                 account_bytes(g, c, nl, cur.nnz, unit, it == 0 && g->opt_singleton && (level > 0 || g->rows_distinct0));
+                for (int i = 0; i < KC_COUNT; ++i) b1 += g->kc_bytes[i];
+                ls.alg_bytes += b1 - b0;
+                const int64_t it_ns = logs[it].t_ns >= t_prev ? (int64_t)(logs[it].t_ns - t_prev) : 0;
+                t_prev = logs[it].t_ns;
                 g->dp_mismatch += (int64_t)c.dp_mismatch;
                 N = log_N(logs[it]);
                 int64_t scanned = 0, kk = 0;
@@ -1421,11 +1431,12 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
                     r.v[4] = (int64_t)c.n_pruned; r.v[5] = (int64_t)c.n_moved;
                     r.v[6] = (int64_t)(N >> 64); r.v[7] = (int64_t)(uint64_t)N;
                     r.v[8] = scanned; r.v[9] = kk; r.v[10] = (int64_t)c.delta_used; r.v[11] = 0;
-                    r.v[12] = (int64_t)c.n_fn; r.v[13] = (int64_t)c.n_fp; r.v[14] = 0; r.v[15] = 0;
+                    r.v[12] = (int64_t)c.n_fn; r.v[13] = (int64_t)c.n_fp; r.v[14] = it_ns; r.v[15] = (int64_t)(b1 - b0);
                     g->trace.push_back(r);
                 }
             }
             ls.iters = (int64_t)logs.size();
+            ls.ms_iters = logs.empty() ? 0.0 : (double)(logs.back().t_ns - t_level) * 1e-6;
             CK(cudaEventRecord(lv1, st));
             // a8: relabel in min-member order + compose
             e = tm.begin();
@@ -2383,9 +2394,10 @@ gala_status gala_get_stats(gala_graph g, char* buf, int64_t cap, int64_t* needed
         const LevelStat& l = g->levels[i];
         snprintf(tmp, sizeof tmp,
                  "%s{\"n\":%lld,\"nnz\":%lld,\"iters\":%lld,\"maxdeg\":%lld,\"mode\":%d,\"ms_phase1\":%.6f,"
-                 "\"ms_phase2\":%.6f,\"edges_scanned\":%lld,\"nominal_edges\":%lld}",
+                 "\"ms_phase2\":%.6f,\"edges_scanned\":%lld,\"nominal_edges\":%lld,\"alg_bytes\":%.0f,\"ms_iters\":%.6f}",
                  i ? "," : "", (long long)l.n, (long long)l.nnz, (long long)l.iters, (long long)l.maxdeg, l.i128path,
-                 l.ms_phase1, l.ms_phase2, (long long)l.edges_scanned, (long long)l.nominal_edges);
+                 l.ms_phase1, l.ms_phase2, (long long)l.edges_scanned, (long long)l.nominal_edges, l.alg_bytes,
+                 l.ms_iters);
         s += tmp;
     }
     s += "],\"kernels\":{";

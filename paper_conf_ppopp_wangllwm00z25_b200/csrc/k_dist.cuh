@@ -135,6 +135,7 @@ __global__ void k_finish(const int64_t* __restrict__ vec, IterCounters* __restri
     carry->N_lo = lo128(Nn);
     carry->sumDC = tdc;
     carry->converged = conv;
+    carry->t_ns = globaltimer_ns();
     ctr->n_active = (ull)vec[1];
     ctr->n_pruned = (ull)vec[2];
     for (int b = 0; b < NBINS; ++b) { ctr->bin_deg[b] = 0; ctr->bin_k[b] = 0; }

@@ -550,6 +550,7 @@ __device__ __forceinline__ void record_iteration(const IterCounters* ctr, Carry*
         L.N_hi = carry->N_hi;
         L.N_lo = carry->N_lo;
         L.converged = carry->converged;
+        L.t_ns = carry->t_ns;
     }
     carry->iter = it + 1;
     const int more = !carry->converged && (max_iters <= 0 || it + 1 < max_iters) && (slot + 1 < log_cap);
@@ -682,6 +683,7 @@ __global__ void __launch_bounds__(BT) k_reduce(int n, int dlo, int dhi, const in
         carry->S2_lo = lo128(ts2);
         carry->minSig = tmn;
         carry->sumDC = tdc;
+        carry->t_ns = globaltimer_ns();
         s_tail = 0;
         if (mode & 2) {   // multi-GPU: sumDC is rank-local; k_finish completes after the all-reduce
             ctr->ticket = 0;
@@ -713,6 +715,7 @@ __global__ void __launch_bounds__(BT) k_reduce(int n, int dlo, int dhi, const in
                 L.N_hi = carry->N_hi;
                 L.N_lo = carry->N_lo;
                 L.converged = carry->converged;
+                L.t_ns = carry->t_ns;
             }
             carry->iter = it + 1;
             const int more = !carry->converged && (max_iters <= 0 || it + 1 < max_iters) && (slot + 1 < log_cap);
