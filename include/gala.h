@@ -170,7 +170,12 @@ void gala_graph_free(gala_graph g);
  *   "concurrent"     0/1   run the degree bins' decide kernels as parallel branches on side
  *                          streams (default 0: measured slower on B200 -- the bins contend for L2 and smem; off whenever "timing" is on)
  *   "log_cap"        device iteration-log capacity (default 4096)
- *   "sync_mode"      multi-GPU label exchange: 0 adaptive (default), 1 dense, 2 sparse
+ *   "sync_mode"      multi-GPU label exchange: 0 adaptive (default), 1 dense, 2 sparse (host
+ *                          backend; the fabric sends sparse whenever the list fits, 2 = 0 there)
+ *   "dist_backend"   multi-GPU iteration: 0 fabric (default; device-resident over peer memory,
+ *                          no host round trip per iteration, CUDA-graph captured, delta d' via the
+ *                          mirror block, send-to-owner phase 2), 1 host-driven collectives (one
+ *                          host round trip per iteration, d' recomputed, phase 2 all-gathered)
  *   "verbose"        0/1   host-side phase timings on stderr
  *   "block_split"    block bin split point (default 1024; 0: one class): on levels with rows longer
  *                          than it, rows <= split run in 256-thread blocks with a small arena, the
@@ -180,6 +185,9 @@ void gala_graph_free(gala_graph g);
  *   "agg_bound"      0/1   phase 2: big-community global tables sized from the chunks' distinct counts
  *                          (two passes, default 1) instead of from min(entries, k)
  *   "agg_chunk"      [1, 4096] entries per big-community chunk (test hook, default 4096)
+ *   "agg_big_ent"    >= 1  phase 2: communities with more entries than this take the chunked big
+ *                          path even when their table fits in shared memory (default 32768: one
+ *                          block per huge community serialised the Orkut level-0 coarsening)
  *   "agg_scap"       [512, 8192] largest phase-2 shared-memory table; communities needing more
  *                          slots take the big (global-table) path (test hook, default 8192)
  */
@@ -210,10 +218,13 @@ gala_status gala_get_stats(gala_graph g, char* json_buf, int64_t cap, int64_t* n
 /*
  * Trace access (option "trace" >= 1).  Record i (0 <= i < count) is
  * int64[16]: level, iter, n_level, n_active, n_pruned, n_moved,
- *            N_hi, N_lo (numerator after the iteration), edges_scanned,
- *            distinct_communities_seen, delta_update_used, reserved,
- *            n_false_negative, n_false_positive (option "prune_check", else 0),
- *            reserved, reserved.
+ *            N_hi, N_lo (numerator after the iteration), edges_scanned
+ *            (sum of deg(v) over the active vertices), distinct_communities_seen,
+ *            delta_update_used, sync (multi-GPU fabric: 1 + senders that exchanged their
+ *            whole label slice; 0 otherwise), n_false_negative (option "prune_check"),
+ *            n_false_positive ("prune_check"; multi-GPU fabric: bytes this rank received),
+ *            iteration device time in ns (%globaltimer, reduction to reduction),
+ *            algorithmic bytes of the iteration (single GPU).
  * Labels (trace == 2): level-local community of every level vertex after
  * the iteration; out must hold n_level entries.
  */
@@ -232,10 +243,15 @@ gala_status gala_get_kernel_stats(gala_graph g, int32_t k, const char** name, in
 /* ---------------------------------------------------------------- multi-GPU
  * 1D vertex partition, one process per GPU (§4.3).  Rank r owns
  * the contiguous vertex range [v_begin, v_end) and its CSR rows (global
- * column ids).  Community state is replicated; after every iteration labels
- * are synchronised densely (broadcast of every rank's slice) or sparsely
- * (allgather of (vertex, community) deltas) by moved volume, and Sigma_tot
- * deltas are all-reduced, all over NCCL.  Results are identical to 1 GPU.
+ * column ids).  Community state (C, Sigma_tot, size, d) is replicated.  After
+ * every iteration each rank's moves reach every replica, densely (its whole
+ * label slice) or sparsely ((vertex, community) pairs), chosen per sender by
+ * bytes; every replica then applies the same moves, so Sigma_tot
+ * needs no all-reduce (the zero-communication equivalent of SURVEY.md §8(e)).
+ * Default backend ("dist_backend" 0): the exchange, two device-side barriers and
+ * the counter sums run in kernels over peer memory (CUDA IPC mappings set up
+ * once over NCCL), so an iteration has no host round trip.  Backend 1 issues
+ * NCCL collectives from the host.  Results are identical to 1 GPU.
  */
 
 /* 128-byte ncclUniqueId for rank 0 to broadcast (GALA_E_NCCL if NCCL cannot be loaded). */

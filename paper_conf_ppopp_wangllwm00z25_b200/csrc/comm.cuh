@@ -33,6 +33,18 @@ struct Comm {
     virtual std::vector<int64_t> allgather_host(int64_t x, cudaStream_t st) = 0;
     // this rank failed mid-run: release peers blocked in a collective (they raise CommError)
     virtual void abort() {}
+    // peer memory (fabric.cuh): every rank passes one cudaMalloc'd device region and gets every
+    // rank's region mapped into its address space (index = rank; its own pointer at `rank`).
+    // Collective.  The mappings stay valid until release_region.
+    virtual std::vector<void*> share_region(void* mine, cudaStream_t st) = 0;
+    virtual void release_region(const std::vector<void*>& peers) { (void)peers; }
+    // host-side rendezvous of ranks that share one process (loopback); a no-op across processes
+    virtual void host_barrier() {}
+    // personalised exchange (bytes): send + sdispls[p] .. + scounts[p] goes to rank p, which
+    // receives it at recv + its rdispls[this rank]; device buffers on `st`
+    virtual void alltoallv(const void* send, const std::vector<size_t>& scounts, const std::vector<size_t>& sdispls,
+                           void* recv, const std::vector<size_t>& rcounts, const std::vector<size_t>& rdispls,
+                           cudaStream_t st) = 0;
 };
 
 // ------------------------------------------------------------------ NCCL (dlopen)
@@ -46,6 +58,8 @@ struct NcclApi {
     ncclResult_t (*Broadcast)(const void*, void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
     ncclResult_t (*GroupStart)() = nullptr;
     ncclResult_t (*GroupEnd)() = nullptr;
+    ncclResult_t (*Send)(const void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*Recv)(void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
     const char* (*GetErrorString)(ncclResult_t) = nullptr;
     bool load() {
         if (h) return true;
@@ -58,9 +72,10 @@ struct NcclApi {
 #define NCCL_SYM(f) f = reinterpret_cast<decltype(f)>(dlsym(h, "nccl" #f))
         NCCL_SYM(GetUniqueId); NCCL_SYM(CommInitRank); NCCL_SYM(CommDestroy); NCCL_SYM(AllReduce);
         NCCL_SYM(AllGather); NCCL_SYM(Broadcast); NCCL_SYM(GroupStart); NCCL_SYM(GroupEnd); NCCL_SYM(GetErrorString);
+        NCCL_SYM(Send); NCCL_SYM(Recv);
 #undef NCCL_SYM
         return GetUniqueId && CommInitRank && CommDestroy && AllReduce && AllGather && Broadcast && GroupStart &&
-               GroupEnd && GetErrorString;
+               GroupEnd && GetErrorString && Send && Recv;
     }
 };
 static NcclApi& nccl_api() {
@@ -101,19 +116,69 @@ struct NcclComm : Comm {
     void allreduce_sum_i64(int64_t* buf, size_t count, cudaStream_t st) override {
         ck(api.AllReduce(buf, buf, count, ncclInt64, ncclSum, comm, st));
     }
+    void alltoallv(const void* send, const std::vector<size_t>& scounts, const std::vector<size_t>& sdispls, void* recv,
+                   const std::vector<size_t>& rcounts, const std::vector<size_t>& rdispls, cudaStream_t st) override {
+        ck(api.GroupStart());
+        for (int p = 0; p < world; ++p) {
+            if (scounts[p]) ck(api.Send(static_cast<const char*>(send) + sdispls[p], scounts[p], ncclChar, p, comm, st));
+            if (rcounts[p]) ck(api.Recv(static_cast<char*>(recv) + rdispls[p], rcounts[p], ncclChar, p, comm, st));
+        }
+        ck(api.GroupEnd());
+    }
     int64_t* scratch = nullptr;   // world + 1 int64, allocated once
     int64_t* hscratch = nullptr;  // pinned mirror
-    std::vector<int64_t> allgather_host(int64_t x, cudaStream_t st) override {
-        if (!scratch) {
-            cudaMalloc(&scratch, sizeof(int64_t) * (world + 1));
-            cudaMallocHost(&hscratch, sizeof(int64_t) * (world + 1));
+    void ensure_scratch() {
+        if (scratch) return;
+        if (cudaMalloc(&scratch, sizeof(int64_t) * (world + 1)) != cudaSuccess) {
+            scratch = nullptr;
+            throw CommError{"allgather_host: cudaMalloc failed"};
         }
+        if (cudaMallocHost(&hscratch, sizeof(int64_t) * (world + 1)) != cudaSuccess) {
+            cudaFree(scratch);
+            scratch = nullptr;
+            hscratch = nullptr;
+            throw CommError{"allgather_host: cudaMallocHost failed"};
+        }
+    }
+    std::vector<int64_t> allgather_host(int64_t x, cudaStream_t st) override {
+        ensure_scratch();
         hscratch[world] = x;
         cudaMemcpyAsync(scratch + world, hscratch + world, sizeof(int64_t), cudaMemcpyHostToDevice, st);
         ck(api.AllGather(scratch + world, scratch, 1, ncclInt64, comm, st));
         cudaMemcpyAsync(hscratch, scratch, sizeof(int64_t) * world, cudaMemcpyDeviceToHost, st);
         cudaStreamSynchronize(st);
         return std::vector<int64_t>(hscratch, hscratch + world);
+    }
+    // CUDA IPC handles of every rank's region over one NCCL allgather; peers mapped with lazy
+    // peer access (NVLink / NVSwitch P2P)
+    std::vector<void*> share_region(void* mine, cudaStream_t st) override {
+        std::vector<void*> out(world, nullptr);
+        out[rank] = mine;
+        if (world == 1) return out;
+        cudaIpcMemHandle_t h;
+        if (cudaIpcGetMemHandle(&h, mine) != cudaSuccess) throw CommError{"cudaIpcGetMemHandle failed"};
+        const size_t hb = sizeof(cudaIpcMemHandle_t);
+        char* dbuf = nullptr;
+        if (cudaMalloc(&dbuf, hb * (world + 1)) != cudaSuccess) throw CommError{"share_region: cudaMalloc failed"};
+        std::vector<char> hbuf(hb * world);
+        cudaMemcpyAsync(dbuf + hb * world, &h, hb, cudaMemcpyHostToDevice, st);
+        ncclResult_t r = api.AllGather(dbuf + hb * world, dbuf, hb, ncclChar, comm, st);
+        cudaMemcpyAsync(hbuf.data(), dbuf, hb * world, cudaMemcpyDeviceToHost, st);
+        cudaStreamSynchronize(st);
+        cudaFree(dbuf);
+        ck(r);
+        for (int p = 0; p < world; ++p) {
+            if (p == rank) continue;
+            cudaIpcMemHandle_t hp;
+            memcpy(&hp, hbuf.data() + hb * p, hb);
+            if (cudaIpcOpenMemHandle(&out[p], hp, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess)
+                throw CommError{"cudaIpcOpenMemHandle failed (no P2P path between the GPUs?)"};
+        }
+        return out;
+    }
+    void release_region(const std::vector<void*>& peers) override {
+        for (int p = 0; p < (int)peers.size(); ++p)
+            if (p != rank && peers[p]) cudaIpcCloseMemHandle(peers[p]);
     }
 };
 
@@ -125,6 +190,7 @@ struct LoopShared {
     int arrived = 0;
     long long generation = 0;
     std::vector<const void*> ptr;
+    std::vector<std::vector<size_t>> displs;   // alltoallv: every rank's send displacements
     std::vector<cudaEvent_t> ev;
     std::vector<int64_t> scal;
     bool aborted = false;
@@ -173,6 +239,7 @@ struct LoopComm : Comm {
             s = std::make_shared<LoopShared>();
             s->world = w;
             s->ptr.assign(w, nullptr);
+            s->displs.assign(w, {});
             s->ev.assign(w, nullptr);
             s->scal.assign(w, 0);
         }
@@ -204,6 +271,17 @@ struct LoopComm : Comm {
                 cudaMemcpyAsync(static_cast<char*>(recv) + displs[r], sh->ptr[r], counts[r], cudaMemcpyDeviceToDevice, st);
         finish(st);
     }
+    void alltoallv(const void* send, const std::vector<size_t>& scounts, const std::vector<size_t>& sdispls, void* recv,
+                   const std::vector<size_t>& rcounts, const std::vector<size_t>& rdispls, cudaStream_t st) override {
+        (void)scounts;
+        sh->displs[rank] = sdispls;
+        publish(send, st);
+        for (int p = 0; p < world; ++p)
+            if (rcounts[p])
+                cudaMemcpyAsync(static_cast<char*>(recv) + rdispls[p], static_cast<const char*>(sh->ptr[p]) + sh->displs[p][rank],
+                                rcounts[p], cudaMemcpyDeviceToDevice, st);
+        finish(st);
+    }
     int64_t* tmp = nullptr;
     size_t tmp_cap = 0;
     void allreduce_sum_i64(int64_t* buf, size_t count, cudaStream_t st) override {
@@ -224,6 +302,17 @@ struct LoopComm : Comm {
         sh->scal[rank] = x;
         sh->barrier();
         std::vector<int64_t> out = sh->scal;
+        sh->barrier();
+        return out;
+    }
+    void host_barrier() override { sh->barrier(); }
+    // same process, same device: the peers' regions are plain device pointers
+    std::vector<void*> share_region(void* mine, cudaStream_t st) override {
+        cudaStreamSynchronize(st);
+        sh->ptr[rank] = mine;
+        sh->barrier();
+        std::vector<void*> out(world);
+        for (int r = 0; r < world; ++r) out[r] = const_cast<void*>(sh->ptr[r]);
         sh->barrier();
         return out;
     }

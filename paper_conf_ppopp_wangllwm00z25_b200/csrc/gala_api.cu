@@ -29,6 +29,7 @@
 #include "k_phase2.cuh"
 #include "comm.cuh"
 #include "k_dist.cuh"
+#include "fabric.cuh"
 
 #define GALA_VERSION "gala-b200 0.1 (sm_100a)"
 
@@ -66,12 +67,12 @@ static thread_local long long g_launches = 0;
 // ------------------------------------------------------------------ kernel classes
 enum KClass {
     KC_PRUNE = 0, KC_DEC_SMALL, KC_DEC_WARP, KC_DEC_WARP2, KC_DEC_BLOCK, KC_DEC_HUB,
-    KC_APPLY, KC_DP, KC_REDUCE, KC_INIT, KC_PHASE2, KC_DEC_SINGLE, KC_COUNT
+    KC_APPLY, KC_DP, KC_REDUCE, KC_INIT, KC_PHASE2, KC_DEC_SINGLE, KC_XCHG, KC_COUNT
 };
 static const char* kc_names[KC_COUNT] = {"prune_bin", "decide_small", "decide_warp", "decide_warp512",
                                          "decide_block", "decide_hub", "apply",
                                          "dp_update", "reduce", "level_init", "phase2",
-                                         "decide_single"};
+                                         "decide_single", "exchange"};
 
 struct TraceRec {
     int64_t v[16];
@@ -109,7 +110,7 @@ struct gala_graph_s {
     int opt_prune = 1, opt_prune_check = 0, opt_trace = 0, opt_check = 0, opt_timing = 0, opt_max_iters = 0;
     int opt_delta = 2, opt_force_i128 = 0, opt_force_wide = 0, opt_cuda_graph = 1, opt_log_cap = 4096, opt_singleton = 1, opt_verbose = 0, opt_agg_big_chunk = 1,
         opt_agg_chunk = AGG_CH, opt_agg_scap = 8192;
-    long long opt_agg_big_ent = 1LL << 62;
+    long long opt_agg_big_ent = 32768;   // communities with more entries take the chunked big path (any table size)
     int opt_block_split = 1024;
     int opt_agg_bound = 1;
     bool rows_distinct0 = false;   // level-0 rows strictly increasing (no duplicate entries)
@@ -138,6 +139,7 @@ struct gala_graph_s {
     int sync_mode = 0;
     std::vector<long long> dbounds0;   // level-0 owned ranges of all ranks
     struct Work* wk = nullptr;   // persistent run workspace (sized for level 0, reused by every run)
+    int64_t cur_n = 0;           // vertex count of the level being iterated (trace label snapshots)
     // side streams of the decide fork: the bins' decide kernels are independent (disjoint
     // vertices, per-bin cursors and tables), so they run as parallel graph branches
     int opt_concurrent = 0;
@@ -429,6 +431,7 @@ static void gamma_to_pq(double gamma, int64_t* p, int64_t* q) {
 struct Work {
     cudaStream_t st;
     int64_t ncap, nnzcap;
+    int64_t qcap = 0;   // queue stride (records per bin pair): n on one GPU, the largest owned range so far with several
     int32_t *rmflag = nullptr, *smflag = nullptr, *chg = nullptr;   // SM / RM movement history (prune 2-4)
     int32_t *C = nullptr, *size = nullptr, *stamp = nullptr, *mv_v = nullptr, *mv_old = nullptr, *mv_chunk = nullptr, *nextC = nullptr;
     QRec* queues = nullptr;
@@ -527,7 +530,7 @@ template <int M, bool UNIT>
 static void launch_hub(gala_graph_s* g, Work& wk, const DecideArgs& a, typename ModeT<M>::ST qW,
                        typename ModeT<M>::ST p, Timer& tm, cudaStream_t st) {
     if (!wk.hub_on) return;
-    const QView q = qview(wk.queues, wk.ncap, BIN_HUB);
+    const QView q = qview(wk.queues, wk.qcap, BIN_HUB);
     cudaEvent_t e = tm.begin();
     k_hub_prep<<<1, 1024, 0, st>>>(q, wk.ctr, wk.hw);
     CKL();
@@ -545,7 +548,7 @@ static void launch_hub(gala_graph_s* g, Work& wk, const DecideArgs& a, typename 
 template <int M, bool UNIT>
 static void launch_single(gala_graph_s* g, Work& wk, const DecideArgs& a, typename ModeT<M>::ST qW,
                           typename ModeT<M>::ST p, Timer& tm, int64_t maxdeg) {
-    const long long qs = wk.ncap;
+    const long long qs = wk.qcap;
     const int grid = g->num_sms * 8;
     cudaStream_t st = g->stream;
     Fork fk(g);
@@ -613,7 +616,7 @@ static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, typename M
     a.idbits = idbits;
     a.idmask = (1LL << idbits) - 1;
     if (single) return launch_single<M, UNIT>(g, wk, a, qW, p, tm, maxdeg);
-    const long long qs = wk.ncap;
+    const long long qs = wk.qcap;
     const int grid = g->num_sms * 8;
     cudaStream_t st = g->stream;
     Fork fk(g);
@@ -755,12 +758,12 @@ static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, typename
     for (int i = 0; i < NBINS - 1; ++i) th.t[i] = g->bins[i];
     const PruneState ps = prune_state(g, wk);
     k_prune_bin<typename ModeT<M>::ST><<<grid_for((n + PB_IPT - 1) / PB_IPT, PB_BT, big), PB_BT, 0, st>>>(
-        0, n, G.rp, wk.d, wk.dp, wk.C, wk.Sig, wk.size, ps, qW, p, wk.carry, wk.ctr, wk.queues, wk.ncap, th);
+        0, n, G.rp, wk.d, wk.dp, wk.C, wk.Sig, wk.size, ps, qW, p, wk.carry, wk.ctr, wk.queues, wk.qcap, th);
     CKL();
     tm.end(KC_PRUNE, e);
     launch_decide<M, UNIT>(g, wk, G, qW, p, tm, maxdeg, idbits, single);
     e = tm.begin();
-    k_apply<<<grid_for(n, AP_BT, big), AP_BT, 0, st>>>(wk.ctr, wk.queues, wk.ncap, wk.nextC, wk.C, wk.Sig, wk.size,
+    k_apply<<<grid_for(n, AP_BT, big), AP_BT, 0, st>>>(wk.ctr, wk.queues, wk.qcap, wk.nextC, wk.C, wk.Sig, wk.size,
                                                        wk.dp, wk.stamp, wk.carry, wk.mv_v, wk.mv_old, wk.mv_chunk, ps);
     CKL();
     tm.end(KC_APPLY, e);
@@ -790,29 +793,33 @@ static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, typename
 }
 
 // Phase 1 of one level to convergence.  Graph mode: the iteration body is
-// captured once into the body of a conditional WHILE node whose condition
-// k_record sets on the device (no host round trip per iteration).  Stepwise
-// mode (trace labels, per-kernel timing, or cuda_graph=0): one host loop trip
-// per iteration.  Both issue the identical kernels.
-template <int M, bool UNIT>
-static void phase1_level(gala_graph_s* g, Work& wk, const DevCSR& G, typename ModeT<M>::ST qW,
-                         typename ModeT<M>::ST p, i128 qW128, i128 T, Timer& tm, int64_t maxdeg, int idbits,
-                         std::vector<IterLog>& out, int level, bool single_ok) {
+// captured once into the body of a conditional WHILE node whose condition the
+// iteration's last kernel sets on the device (no host round trip per iteration).
+// Stepwise mode (trace labels, per-kernel timing, or cuda_graph=0): one host loop
+// trip per iteration.  Both issue the identical kernels.  `issue(cond, single)`
+// enqueues one iteration (single: the level's first, singleton fast path); the
+// single-GPU and the multi-GPU (fabric) drivers share this loop.
+struct NoHook {
+    void operator()() const {}
+};
+template <typename Issue, typename PreLaunch = NoHook>
+static void level_loop(gala_graph_s* g, Work& wk, std::vector<IterLog>& out, bool single_ok, Timer& tm, Issue issue,
+                       PreLaunch pre_launch = PreLaunch()) {
     cudaStream_t st = g->stream;
     const bool stepwise = !g->opt_cuda_graph || g->opt_trace >= 2 || g->opt_timing;
-    block_setup<M, UNIT>(g);   // host-side attributes / grids before any capture (block_split may have changed)
     out.clear();
     // first iteration of a level: singleton fast path when rows hold distinct columns
     bool first_single = single_ok && g->opt_singleton;
     int log_base_host = 0;   // mirror of carry->log_base
     if (stepwise || first_single) {
         for (;;) {
-            issue_iteration<M, UNIT>(g, wk, G, qW, p, qW128, T, tm, maxdeg, idbits, 0ull, first_single);            CK(cudaMemcpyAsync(wk.h_carry, wk.carry, sizeof(Carry), cudaMemcpyDeviceToHost, st));
+            issue(0ull, first_single);
+            CK(cudaMemcpyAsync(wk.h_carry, wk.carry, sizeof(Carry), cudaMemcpyDeviceToHost, st));
             const int slot = (int)out.size() - log_base_host;
             CK(cudaMemcpyAsync(wk.h_log, wk.log + slot, sizeof(IterLog), cudaMemcpyDeviceToHost, st));
             if (g->opt_trace >= 2) {
-                g->trace_labels.emplace_back(G.n);
-                CK(cudaMemcpyAsync(g->trace_labels.back().data(), wk.C, sizeof(int32_t) * G.n, cudaMemcpyDeviceToHost, st));
+                g->trace_labels.emplace_back(g->cur_n);
+                CK(cudaMemcpyAsync(g->trace_labels.back().data(), wk.C, sizeof(int32_t) * g->cur_n, cudaMemcpyDeviceToHost, st));
             }
             CK(cudaStreamSynchronize(st));
             tm.resolve();
@@ -845,7 +852,7 @@ static void phase1_level(gala_graph_s* g, Work& wk, const DevCSR& G, typename Mo
         cudaGraph_t body = cp.conditional.phGraph_out[0];
         CK(cudaStreamBeginCaptureToGraph(st, body, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed));
         try {
-            issue_iteration<M, UNIT>(g, wk, G, qW, p, qW128, T, tm, maxdeg, idbits, (unsigned long long)handle, false);
+            issue((unsigned long long)handle, false);
         } catch (...) {
             cudaGraph_t dummy;
             cudaStreamEndCapture(st, &dummy);
@@ -853,6 +860,7 @@ static void phase1_level(gala_graph_s* g, Work& wk, const DevCSR& G, typename Mo
         }
         CK(cudaStreamEndCapture(st, &body));
         CK(cudaGraphInstantiate(&exec, graph, 0));
+        pre_launch();
         for (;;) {
             CK(cudaGraphLaunch(exec, st));
             CK(cudaMemcpyAsync(wk.h_carry, wk.carry, sizeof(Carry), cudaMemcpyDeviceToHost, st));
@@ -875,7 +883,18 @@ static void phase1_level(gala_graph_s* g, Work& wk, const DevCSR& G, typename Mo
     }
     cudaGraphExecDestroy(exec);
     cudaGraphDestroy(graph);
+}
+
+template <int M, bool UNIT>
+static void phase1_level(gala_graph_s* g, Work& wk, const DevCSR& G, typename ModeT<M>::ST qW,
+                         typename ModeT<M>::ST p, i128 qW128, i128 T, Timer& tm, int64_t maxdeg, int idbits,
+                         std::vector<IterLog>& out, int level, bool single_ok) {
+    block_setup<M, UNIT>(g);   // host-side attributes / grids before any capture (block_split may have changed)
+    g->cur_n = G.n;
     (void)level;
+    level_loop(g, wk, out, single_ok, tm, [&](unsigned long long cond, bool single) {
+        issue_iteration<M, UNIT>(g, wk, G, qW, p, qW128, T, tm, maxdeg, idbits, cond, single);
+    });
 }
 
 static i128 carry_N(const Carry* c) {
@@ -1248,7 +1267,14 @@ static void ensure_workspace(gala_graph_s* g) {
             wk.mv_old = dalloc<int32_t>(icap, st);
             wk.mv_chunk = dalloc<int32_t>(icap, st);
             wk.nextC = dalloc<int32_t>(wk.ncap, st);
-            wk.queues = dalloc<QRec>((size_t)wk.ncap * (NBINS / 2), st);
+            // multi-GPU: only owned vertices are queued (largest owned range; grown per level if needed)
+            wk.qcap = wk.ncap;
+            if (g->di && g->dbounds0.size() > 1) {
+                long long mx = 1;
+                for (size_t r = 0; r + 1 < g->dbounds0.size(); ++r) mx = std::max(mx, g->dbounds0[r + 1] - g->dbounds0[r]);
+                wk.qcap = mx;
+            }
+            wk.queues = dalloc<QRec>((size_t)wk.qcap * (NBINS / 2), st);
             if (g->ckey_ok) wk.ckey = dalloc<int32_t>(g->nnz0, st);
             wk.Sig = dalloc<int64_t>(wk.ncap, st);
             wk.d = dalloc<int64_t>(wk.ncap, st);
@@ -1522,9 +1548,53 @@ struct DistInfo {
     Comm* comm = nullptr;
     long long v0 = 0, v1 = 0;        // level-0 owned range
     int sync_mode = 0;               // 0 adaptive, 1 dense, 2 sparse
+    int backend = 0;                 // 0 fabric (device-resident, peer memory), 1 host-driven NCCL collectives
     long long n_dense = 0, n_sparse = 0;
     double bytes_exchanged = 0;
+    // fabric (fabric.cuh): this rank's symmetric region and every rank's mapping of it
+    void* region = nullptr;
+    std::vector<void*> peers;
+    FabDev fab = {};
 };
+
+// Symmetric region of a rank (cudaMalloc: CUDA IPC needs it), byte offsets:
+//   0     arrival counter (ull)          256   epoch (ull, local)      264  error flag (int, local)
+//   512   headers [2][FAB_MAXP] ull      1024  scalars [2][FAB_MAXP][FAB_NSCAL] int64
+//   4096  inbox [2][istride] int32 (istride = n + 2 world + 2, even)
+static void fabric_setup(gala_graph_s* g, DistInfo& di, int64_t n) {
+    Comm& cm = *di.comm;
+    if (cm.world > FAB_MAXP) { set_err(GALA_E_INVALID, "world > %d", FAB_MAXP); throw GalaError{GALA_E_INVALID}; }
+    const long long istride = ((n + 2LL * cm.world + 2) + 1) & ~1LL;
+    const size_t bytes = 4096 + sizeof(int32_t) * 2 * (size_t)istride;
+    CK(cudaMalloc(&di.region, bytes));
+    CK(cudaMemsetAsync(di.region, 0, 4096, g->stream));
+    CK(cudaStreamSynchronize(g->stream));
+    try {
+        di.peers = cm.share_region(di.region, g->stream);   // collective; nobody arrives before all zeroed
+    } catch (CommError& e) {
+        set_err(GALA_E_NCCL, "%s", e.msg.c_str());
+        throw GalaError{GALA_E_NCCL};
+    }
+    FabDev& f = di.fab;
+    f.P = cm.world;
+    f.rank = cm.rank;
+    for (int r = 0; r < cm.world; ++r) {
+        char* b = static_cast<char*>(di.peers[r]);
+        f.arrive[r] = reinterpret_cast<ull*>(b);
+        f.hdr[r] = reinterpret_cast<ull*>(b + 512);
+        f.scal[r] = reinterpret_cast<long long*>(b + 1024);
+        f.inbox[r] = reinterpret_cast<int32_t*>(b + 4096);
+    }
+    f.epoch = reinterpret_cast<ull*>(static_cast<char*>(di.region) + 256);
+    f.err = reinterpret_cast<int*>(static_cast<char*>(di.region) + 264);
+    f.istride = istride;
+}
+static void fabric_release(DistInfo& di) {
+    if (!di.region) return;
+    if (di.comm) di.comm->release_region(di.peers);
+    cudaFree(di.region);
+    di.region = nullptr;
+}
 
 // Communicators are created once per (uid, rank) and cached for the process
 // lifetime: handles built with the same uid share one NCCL communicator, so
@@ -1565,12 +1635,12 @@ static void dist_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, long long
     for (int i = 0; i < NBINS - 1; ++i) th.t[i] = g->bins[i];
     k_prune_bin<typename ModeT<M>::ST><<<grid_for((lv1 - lv0 + PB_IPT - 1) / PB_IPT, PB_BT, big), PB_BT, 0, st>>>(
         (int)lv0, (int)lv1, G.rp, wk.d, wk.dp, wk.C, wk.Sig, wk.size, prune_state(g, wk), qW, p, wk.carry, wk.ctr,
-        wk.queues, wk.ncap, th);
+        wk.queues, wk.qcap, th);
     CKL();
     launch_decide<M, UNIT>(g, wk, G, qW, p, tm, maxdeg, idbits, single);
     vt.lap("dist: prune+decide");
     CK(cudaMemsetAsync(dcnt, 0, 2 * sizeof(ull), st));
-    k_collect_moves<<<grid_for(lv1 - lv0, 256, big), 256, 0, st>>>(wk.ctr, wk.queues, wk.ncap, wk.nextC, lmoves, dcnt);
+    k_collect_moves<<<grid_for(lv1 - lv0, 256, big), 256, 0, st>>>(wk.ctr, wk.queues, wk.qcap, wk.nextC, lmoves, dcnt);
     CKL();
     ull mloc = 0;
     CK(cudaMemcpyAsync(&mloc, dcnt, sizeof(ull), cudaMemcpyDeviceToHost, st));
@@ -1730,6 +1800,258 @@ static void dist_coarsen(gala_graph_s* g, Work& wk, const DevCSR& cur, int64_t n
     dfree(dnew, st); dfree(dev_max, st); dfree(dbounds, st); dfree(rmax, st); dfree(snew, st);
 }
 
+// Phase 2 across ranks, send-to-owner (SURVEY.md §8(e) "Phase 2"): every rank aggregates its
+// owned rows into partial coarse rows (the single-GPU aggregation); the next level's coarse
+// vertex ranges are cut edge-balanced on the all-reduced partial row lengths (an upper bound of
+// the merged lengths, identical on every rank); each partial row goes to its owner only
+// (alltoallv), which merges what it received into its own coarse rows.  No rank ever holds the
+// whole coarse graph.  Coarse d = Sigma_tot (replicated), s = the merged diagonal (owned rows).
+static void dist_coarsen_s2o(gala_graph_s* g, Work& wk, const DevCSR& cur, int64_t nl, long long k,
+                             const int32_t* newid, const int32_t* minmem, bool unit, DevCSR& local,
+                             std::vector<long long>& bounds, int64_t& maxdeg, int64_t& dmax) {
+    Comm& cm = *g->di->comm;
+    cudaStream_t st = g->stream;
+    const int big = g->num_sms * 8;
+    const int P = cm.world;
+    DevCSR part;
+    int64_t md = 0;
+    int64_t* snew = dalloc<int64_t>(k, st);
+    aggregate_rows(g, cur, nl, k, newid, newid, unit, part, md, snew);
+    // next level's ranges from the summed partial lengths
+    long long* plen = dalloc<long long>(k + 1, st);
+    k_row_lengths<<<grid_for(k, 256, big), 256, 0, st>>>(k, part.rp, plen);
+    CKL();
+    cm.allreduce_sum_i64(reinterpret_cast<int64_t*>(plen), (size_t)k, st);
+    long long* prp = dalloc<long long>(k + 1, st);
+    scan_excl(plen, prp, k, st);
+    long long* dbounds = dalloc<long long>(P + 1, st);
+    k_partition_bounds<<<1, 64, 0, st>>>(k, reinterpret_cast<const int64_t*>(prp), P, dbounds);
+    CKL();
+    bounds.assign(P + 1, 0);
+    CK(cudaMemcpyAsync(bounds.data(), dbounds, sizeof(long long) * (P + 1), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    dfree(plen, st); dfree(prp, st); dfree(dbounds, st);
+    // entries of part destined to every rank (rows [b_p, b_{p+1}) are contiguous), counts matrix
+    std::vector<long long> eb(P + 1, 0);
+    for (int p = 0; p <= P; ++p)
+        CK(cudaMemcpyAsync(&eb[p], part.rp + bounds[p], sizeof(long long), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    int64_t* mat = dalloc<int64_t>((size_t)P * P, st);
+    std::vector<int64_t> hm((size_t)P * P, 0);
+    for (int p = 0; p < P; ++p) hm[(size_t)cm.rank * P + p] = eb[p + 1] - eb[p];
+    CK(cudaMemcpyAsync(mat, hm.data(), sizeof(int64_t) * P * P, cudaMemcpyHostToDevice, st));
+    cm.allreduce_sum_i64(mat, (size_t)P * P, st);
+    CK(cudaMemcpyAsync(hm.data(), mat, sizeof(int64_t) * P * P, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    dfree(mat, st);
+    std::vector<size_t> sc(P), sd(P), rc(P), rd(P);
+    long long R = 0;
+    for (int p = 0; p < P; ++p) {
+        sc[p] = (size_t)(eb[p + 1] - eb[p]);
+        sd[p] = (size_t)eb[p];
+        rc[p] = (size_t)hm[(size_t)p * P + cm.rank];
+        rd[p] = (size_t)R;
+        R += (long long)rc[p];
+    }
+    auto scale = [](std::vector<size_t> v, size_t b) { for (auto& x : v) x *= b; return v; };
+    int32_t* arow = dalloc<int32_t>(std::max<long long>(R, 1), st);
+    int32_t* acol = dalloc<int32_t>(std::max<long long>(R, 1), st);
+    int64_t* aw = dalloc<int64_t>(std::max<long long>(R, 1), st);
+    cm.alltoallv(part.row, scale(sc, 4), scale(sd, 4), arow, scale(rc, 4), scale(rd, 4), st);
+    cm.alltoallv(part.col, scale(sc, 4), scale(sd, 4), acol, scale(rc, 4), scale(rd, 4), st);
+    cm.alltoallv(part.w, scale(sc, 8), scale(sd, 8), aw, scale(rc, 8), scale(rd, 8), st);
+    g->di->bytes_exchanged += 16.0 * (double)(R - (long long)rc[cm.rank]);
+    dfree(part.rp, st); dfree(part.col, st); dfree(part.w, st); dfree(part.row, st);
+    // received triplets (own coarse rows only) -> multigraph in global-row form -> merged rows
+    DevCSR mg;
+    mg.n = k;
+    mg.nnz = R;
+    long long* cnt = dalloc<long long>(k + 1, st);
+    CK(cudaMemsetAsync(cnt, 0, sizeof(long long) * (k + 1), st));
+    k_count_rows<<<grid_for(R, 256, big), 256, 0, st>>>(R, arow, cnt);
+    CKL();
+    mg.rp = dalloc<int64_t>(k + 1, st);
+    scan_excl(cnt, reinterpret_cast<long long*>(mg.rp), k, st);
+    CK(cudaMemsetAsync(cnt, 0, sizeof(long long) * (k + 1), st));
+    mg.row = dalloc<int32_t>(std::max<long long>(R, 1), st);
+    mg.col = dalloc<int32_t>(std::max<long long>(R, 1), st);
+    mg.w = dalloc<int64_t>(std::max<long long>(R, 1), st);
+    k_scatter_rows<<<grid_for(R, 256, big), 256, 0, st>>>(R, arow, acol, aw, reinterpret_cast<long long*>(mg.rp), cnt,
+                                                          mg.row, mg.col, mg.w);
+    CKL();
+    dfree(arow, st); dfree(acol, st); dfree(aw, st); dfree(cnt, st);
+    int32_t* id = dalloc<int32_t>(k, st);
+    k_iota<<<grid_for(k, 256, big), 256, 0, st>>>(k, id);
+    CKL();
+    int64_t* snew2 = dalloc<int64_t>(k, st);
+    aggregate_rows(g, mg, k, k, id, id, false, local, maxdeg, snew2);
+    dfree(mg.rp, st); dfree(mg.col, st); dfree(mg.w, st); dfree(mg.row, st); dfree(id, st); dfree(snew, st);
+    // replicated coarse d = Sigma_tot, s = merged diagonal (owned rows; others 0, never read)
+    int64_t* dnew = dalloc<int64_t>(k, st);
+    ull* dev_max = dalloc<ull>(1, st);
+    CK(cudaMemsetAsync(dev_max, 0, sizeof(ull), st));
+    k_coarsen_deg<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.C, minmem, newid, wk.Sig, dnew);
+    CKL();
+    k_max_i64<<<grid_for(k, 256, big), 256, 0, st>>>(k, dnew, dev_max);
+    CKL();
+    CK(cudaMemcpyAsync(wk.d, dnew, sizeof(int64_t) * k, cudaMemcpyDeviceToDevice, st));
+    CK(cudaMemcpyAsync(wk.s, snew2, sizeof(int64_t) * k, cudaMemcpyDeviceToDevice, st));
+    wk.s_zero = false;
+    ull hm2 = 0;
+    CK(cudaMemcpyAsync(&hm2, dev_max, sizeof(ull), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    dmax = (int64_t)hm2;
+    dfree(dnew, st); dfree(dev_max, st); dfree(snew2, st);
+}
+
+// ------------------------------------------------------------------ multi-GPU, fabric backend
+// Per-level device state of the fabric iteration (fabric.cuh): the local move list, the mirror
+// block of the owned rows (§8(e)) and the d' work items.
+struct DistLevel {
+    long long lv0 = 0, lv1 = 0;
+    int2* lmoves = nullptr;
+    ull* lcount = nullptr;
+    int64_t* mrp = nullptr;
+    int32_t* mcol = nullptr;
+    int64_t* mw = nullptr;
+    int32_t *it_v = nullptr, *it_old = nullptr, *it_chunk = nullptr;
+    FabDev f = {};
+    void release(cudaStream_t st) {
+        dfree(lmoves, st); dfree(lcount, st); dfree(mrp, st); dfree(mcol, st); dfree(mw, st);
+        dfree(it_v, st); dfree(it_old, st); dfree(it_chunk, st);
+    }
+};
+
+static void dist_level_setup(gala_graph_s* g, const DevCSR& G, const std::vector<long long>& bounds, DistLevel& L) {
+    cudaStream_t st = g->stream;
+    DistInfo& di = *g->di;
+    const int P = di.comm->world, r = di.comm->rank;
+    const int big = g->num_sms * 8;
+    const long long n = G.n;
+    L.lv0 = bounds[r];
+    L.lv1 = bounds[r + 1];
+    L.f = di.fab;
+    for (int s = 0; s <= P; ++s) L.f.bnd[s] = bounds[s];
+    for (int s = 0; s < P; ++s) L.f.off[s] = (bounds[s] + 2LL * s) & ~1LL;
+    L.f.force_dense = di.sync_mode == 1;
+    L.lmoves = dalloc<int2>(std::max<long long>(L.lv1 - L.lv0, 1), st);
+    L.lcount = dalloc<ull>(1, st);
+    CK(cudaMemsetAsync(L.lcount, 0, sizeof(ull), st));
+    // mirror block: owned entries (v, u, w) counting-sorted by u
+    long long* cnt = dalloc<long long>(n + 1, st);
+    CK(cudaMemsetAsync(cnt, 0, sizeof(long long) * (n + 1), st));
+    k_mirror_count<<<grid_for(G.nnz, 256, big), 256, 0, st>>>(G.nnz, G.col, cnt);
+    CKL();
+    L.mrp = dalloc<int64_t>(n + 1, st);
+    scan_excl(cnt, reinterpret_cast<long long*>(L.mrp), n, st);
+    CK(cudaMemsetAsync(cnt, 0, sizeof(long long) * (n + 1), st));
+    L.mcol = dalloc<int32_t>(std::max<long long>(G.nnz, 1), st);
+    if (G.w) L.mw = dalloc<int64_t>(std::max<long long>(G.nnz, 1), st);
+    k_mirror_scatter<<<grid_for(G.nnz, 256, big), 256, 0, st>>>(G.nnz, G.row, G.col, G.w,
+                                                                 reinterpret_cast<long long*>(L.mrp), cnt, L.mcol, L.mw);
+    CKL();
+    dfree(cnt, st);
+    // d' items: one per global mover with a row here + one per DCH-entry chunk of own / mirror rows
+    const size_t icap = (size_t)n + (size_t)(2 * G.nnz / DCH) + (size_t)P + 1;
+    L.it_v = dalloc<int32_t>(icap, st);
+    L.it_old = dalloc<int32_t>(icap, st);
+    L.it_chunk = dalloc<int32_t>(icap, st);
+}
+
+// one device-resident iteration of the fabric backend (see fabric.cuh for the sequence)
+template <int M, bool UNIT>
+static void dist_iteration_fab(gala_graph_s* g, Work& wk, const DevCSR& G, const DistLevel& L,
+                               typename ModeT<M>::ST qW, typename ModeT<M>::ST p, i128 qW128, i128 T, Timer& tm,
+                               int64_t maxdeg, int idbits, unsigned long long cond, bool single) {
+    cudaStream_t st = g->stream;
+    const long long n = G.n, lv0 = L.lv0, lv1 = L.lv1;
+    const int big = g->num_sms * 8;
+    BinThresholds th;
+    for (int i = 0; i < NBINS - 1; ++i) th.t[i] = g->bins[i];
+    cudaEvent_t e = tm.begin();
+    k_prune_bin<typename ModeT<M>::ST><<<grid_for((lv1 - lv0 + PB_IPT - 1) / PB_IPT, PB_BT, big), PB_BT, 0, st>>>(
+        (int)lv0, (int)lv1, G.rp, wk.d, wk.dp, wk.C, wk.Sig, wk.size, prune_state(g, wk), qW, p, wk.carry, wk.ctr,
+        wk.queues, wk.qcap, th);
+    CKL();
+    tm.end(KC_PRUNE, e);
+    launch_decide<M, UNIT>(g, wk, G, qW, p, tm, maxdeg, idbits, single);
+    e = tm.begin();
+    k_collect_moves<<<grid_for(lv1 - lv0, 256, big), 256, 0, st>>>(wk.ctr, wk.queues, wk.qcap, wk.nextC, L.lmoves,
+                                                                    L.lcount);
+    CKL();
+    k_fab_push<<<g->num_sms * 2, 256, 0, st>>>(L.f, L.lmoves, L.lcount, wk.C, wk.carry);
+    CKL();
+    k_fab_push_fix<<<g->num_sms, 256, 0, st>>>(L.f, L.lmoves, L.lcount, wk.carry);
+    CKL();
+    k_fab_barrier<<<1, 32, 0, st>>>(L.f);
+    CKL();
+    tm.end(KC_XCHG, e);
+    e = tm.begin();
+    k_fab_apply<<<grid_for(n, 256, big), 256, 0, st>>>(L.f, wk.carry, wk.ctr, wk.C, wk.Sig, wk.size, wk.d, wk.stamp,
+                                                       wk.dp, G.rp, L.mrp, lv0, lv1, L.it_v, L.it_old, L.it_chunk);
+    CKL();
+    tm.end(KC_APPLY, e);
+    e = tm.begin();
+    k_fab_dp_delta<UNIT><<<big, 256, 0, st>>>(wk.ctr, G.rp, G.col, G.w, L.mrp, L.mcol, L.mw, wk.C, L.it_v, L.it_old,
+                                              L.it_chunk, wk.stamp, wk.dp, wk.carry, G.nnz, g->opt_delta, lv0, lv1);
+    CKL();
+    k_dp_zero<<<big, 256, 0, st>>>(wk.ctr, (int)lv0, (int)lv1, wk.dp, G.nnz, g->opt_delta, 1, 2);
+    CKL();
+    if (G.nnz) {
+        k_dp_full<UNIT><<<grid_for((G.nnz + 127) / 128 * 32, 256, big), 256, 0, st>>>(
+            wk.ctr, G.nnz, G.row, G.col, G.w, wk.C, wk.dp, g->opt_delta, 1, 2, nullptr, nullptr, nullptr, nullptr,
+            wk.carry);
+        CKL();
+    }
+    tm.end(KC_DP, e);
+    e = tm.begin();
+    k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>((int)n, (int)lv0, (int)lv1, wk.dp, wk.s_live(), wk.Sig, wk.part_dc,
+                                                  wk.part_s2, wk.part_min, wk.ctr, wk.carry, 0, 0, 0, 0, 0, 3);
+    CKL();
+    k_fab_scal<<<1, 32, 0, st>>>(L.f, wk.carry, wk.ctr, L.lcount, 0);
+    CKL();
+    k_fab_barrier<<<1, 32, 0, st>>>(L.f);
+    CKL();
+    k_fab_finish<<<1, 32, 0, st>>>(L.f, wk.ctr, wk.carry, L.lcount, (long long)(qW128 >> 64), (ull)qW128, (long long)p,
+                                   (long long)(T >> 64), (ull)T, 1, wk.log, wk.log_cap, g->opt_max_iters, cond);
+    CKL();
+    tm.end(KC_REDUCE, e);
+}
+
+// level start on the fabric: singletons, N of the singleton partition from rank-ordered sums
+static void dist_level_start_fab(gala_graph_s* g, Work& wk, const DevCSR& G, const DistLevel& L, i128 qW128,
+                                 int64_t p) {
+    cudaStream_t st = g->stream;
+    const long long n = G.n;
+    k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>((int)n, (int)L.lv0, (int)L.lv1, wk.dp, wk.s_live(), wk.Sig,
+                                                  wk.part_dc, wk.part_s2, wk.part_min, wk.ctr, wk.carry, 0, 0, 0, 0, 0,
+                                                  2);
+    CKL();
+    k_fab_scal<<<1, 32, 0, st>>>(L.f, wk.carry, wk.ctr, L.lcount, 1);
+    CKL();
+    k_fab_barrier<<<1, 32, 0, st>>>(L.f);
+    CKL();
+    k_fab_finish<<<1, 32, 0, st>>>(L.f, wk.ctr, wk.carry, L.lcount, (long long)(qW128 >> 64), (ull)qW128, (long long)p,
+                                   0, 0, 0, nullptr, 0, 0, 0ull);
+    CKL();
+}
+
+template <int M, bool UNIT>
+static void dist_phase1_fab(gala_graph_s* g, Work& wk, const DevCSR& G, const DistLevel& L, typename ModeT<M>::ST qW,
+                            typename ModeT<M>::ST p, i128 qW128, i128 T, Timer& tm, int64_t maxdeg, int idbits,
+                            std::vector<IterLog>& out, bool single_ok) {
+    block_setup<M, UNIT>(g);
+    g->cur_n = G.n;
+    // ranks sharing a process (loopback) meet before launching the level's graph, so no rank's
+    // barrier kernel spins while another rank's thread is still instantiating
+    level_loop(
+        g, wk, out, single_ok, tm,
+        [&](unsigned long long cond, bool single) {
+            dist_iteration_fab<M, UNIT>(g, wk, G, L, qW, p, qW128, T, tm, maxdeg, idbits, cond, single);
+        },
+        [&]() { g->di->comm->host_barrier(); });
+}
+
 static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_levels) {
     PoolScope pool_scope(g->cache);
     cudaStream_t st = g->stream;
@@ -1790,6 +2112,11 @@ static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_level
             ls.nnz = gnnz;
             ls.maxdeg = maxdeg;
             CK(cudaEventRecord(wk.ev[2], st));
+            if (lv1 - lv0 > wk.qcap) {   // this level's owned range is longer than any before
+                dfree(wk.queues, st);
+                wk.qcap = lv1 - lv0;
+                wk.queues = dalloc<QRec>((size_t)wk.qcap * (NBINS / 2), st);
+            }
             prepare_level_tables(g, wk, cur, maxdeg);
             k_level_init<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.d, wk.C, wk.Sig, wk.size, wk.dp, wk.stamp,
                                                                  wk.carry, prune_state(g, wk));
@@ -1797,17 +2124,25 @@ static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_level
             if (level == 0) CK(cudaMemcpyAsync(g->lab, wk.C, sizeof(int32_t) * n0, cudaMemcpyDeviceToDevice, st));
             k_iter_begin<<<1, 128, 0, st>>>(wk.ctr);
             CKL();
-            k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>((int)nl, (int)lv0, (int)lv1, wk.dp, wk.s_live(), wk.Sig, wk.part_dc,
-                                                          wk.part_s2, wk.part_min, wk.ctr, wk.carry, 0, 0, 0, 0, 0, 2);
-            CKL();
-            k_pack_counters<<<1, 32, 0, st>>>(wk.carry, wk.ctr, vec);
-            CKL();
-            cm.allreduce_sum_i64(vec, 5, st);
-            k_finish<<<1, 32, 0, st>>>(vec, wk.ctr, wk.carry, (long long)(qW128 >> 64), (ull)qW128, (long long)p, 0, 0, 0);
-            CKL();
+            const bool fab = di.backend == 0;
+            DistLevel L;
+            if (fab) {
+                dist_level_setup(g, cur, bounds, L);
+                dist_level_start_fab(g, wk, cur, L, qW128, p);
+            } else {
+                k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>((int)nl, (int)lv0, (int)lv1, wk.dp, wk.s_live(), wk.Sig, wk.part_dc,
+                                                              wk.part_s2, wk.part_min, wk.ctr, wk.carry, 0, 0, 0, 0, 0, 2);
+                CKL();
+                k_pack_counters<<<1, 32, 0, st>>>(wk.carry, wk.ctr, vec);
+                CKL();
+                cm.allreduce_sum_i64(vec, 5, st);
+                k_finish<<<1, 32, 0, st>>>(vec, wk.ctr, wk.carry, (long long)(qW128 >> 64), (ull)qW128, (long long)p, 0, 0, 0);
+                CKL();
+            }
             CK(cudaMemcpyAsync(wk.h_carry, wk.carry, sizeof(Carry), cudaMemcpyDeviceToHost, st));
             CK(cudaStreamSynchronize(st));
             const i128 N_start = carry_N(wk.h_carry);
+            const ull t_level = wk.h_carry->t_ns;
             int idbits = 1;
             while (idbits < 31 && ((int64_t)1 << idbits) < nl) ++idbits;
             const long double bound = (long double)mpq * (long double)W * (long double)std::max<int64_t>(dmax, 1);
@@ -1818,8 +2153,21 @@ static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_level
             ls.i128path = mode;
             const long long qW64 = (long long)qW128, p64 = (long long)p;
             logs.clear();
-            for (int it = 0;; ++it) {
-                const bool single = it == 0 && g->opt_singleton && (level > 0 || g->rows_distinct0);
+            const bool single_ok = level > 0 || g->rows_distinct0;
+            if (fab) {
+#define DIST_FAB(MM, UU, QW, PP) dist_phase1_fab<MM, UU>(g, wk, cur, L, QW, PP, qW128, T, tm, maxdeg, idbits, logs, single_ok)
+                if (mode == DM_W128) { if (unit) DIST_FAB(DM_W128, true, (i128)qW128, (i128)p); else DIST_FAB(DM_W128, false, (i128)qW128, (i128)p); }
+                else if (mode == DM_W64) { if (unit) DIST_FAB(DM_W64, true, qW64, p64); else DIST_FAB(DM_W64, false, qW64, p64); }
+                else { if (unit) DIST_FAB(DM_FAST, true, qW64, p64); else DIST_FAB(DM_FAST, false, qW64, p64); }
+#undef DIST_FAB
+                L.release(st);
+                int err = 0;
+                CK(cudaMemcpyAsync(&err, di.fab.err, sizeof(int), cudaMemcpyDeviceToHost, st));
+                CK(cudaStreamSynchronize(st));
+                if (err) throw CommError{"fabric: a peer rank stopped answering (barrier timeout)"};
+            }
+            for (int it = 0; !fab; ++it) {
+                const bool single = it == 0 && g->opt_singleton && single_ok;
 #define DIST_IT(MM, UU, QW, PP) dist_iteration<MM, UU>(g, wk, cur, lv0, lv1, bounds, QW, PP, qW128, T, tm, maxdeg, \
                                                        idbits, single, lmoves, gmoves, newC, dcnt, vec)
                 if (mode == DM_W128) { if (unit) DIST_IT(DM_W128, true, (i128)qW128, (i128)p); else DIST_IT(DM_W128, false, (i128)qW128, (i128)p); }
@@ -1843,6 +2191,7 @@ static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_level
                 if (c.converged || (g->opt_max_iters > 0 && c.iter >= g->opt_max_iters)) break;
             }
             i128 N = N_start;
+            ull t_prev = t_level;
             for (size_t it = 0; it < logs.size(); ++it) {
                 const IterCounters& c = logs[it].ctr;
                 N = log_N(logs[it]);
@@ -1850,17 +2199,25 @@ static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_level
                 for (int b = 0; b < NBINS; ++b) { scanned += (int64_t)c.bin_deg[b]; kk += (int64_t)c.bin_k[b]; }
                 ls.edges_scanned += scanned;
                 ls.nominal_edges += gnnz;
+                const int64_t it_ns = fab && logs[it].t_ns >= t_prev ? (int64_t)(logs[it].t_ns - t_prev) : 0;
+                if (fab) {
+                    t_prev = logs[it].t_ns;
+                    if (c.n_dense) di.n_dense++; else di.n_sparse++;
+                    di.bytes_exchanged += (double)c.xbytes;
+                }
                 if (g->opt_trace >= 1) {
                     TraceRec r;
                     r.v[0] = level; r.v[1] = (int64_t)it; r.v[2] = nl; r.v[3] = (int64_t)c.n_active;
                     r.v[4] = (int64_t)c.n_pruned; r.v[5] = (int64_t)c.n_moved;
                     r.v[6] = (int64_t)(N >> 64); r.v[7] = (int64_t)(uint64_t)N;
-                    r.v[8] = scanned; r.v[9] = kk; r.v[10] = 0; r.v[11] = 0;
-                    r.v[12] = 0; r.v[13] = 0; r.v[14] = 0; r.v[15] = 0;
+                    r.v[8] = scanned; r.v[9] = kk; r.v[10] = (int64_t)c.delta_used;
+                    r.v[11] = fab ? 1 + (int64_t)c.n_dense : 0;   // fabric: 1 + senders that went dense
+                    r.v[12] = 0; r.v[13] = (int64_t)c.xbytes; r.v[14] = it_ns; r.v[15] = 0;
                     g->trace.push_back(r);
                 }
             }
             ls.iters = (int64_t)logs.size();
+            if (fab && !logs.empty()) ls.ms_iters = (double)(logs.back().t_ns - t_level) * 1e-6;
             CK(cudaEventRecord(wk.ev[3], st));
             // a8: relabel (replicated state: identical on every rank)
             int32_t* minmem = dalloc<int32_t>(nl, st);
@@ -1882,7 +2239,10 @@ static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_level
             CK(cudaStreamSynchronize(st));
             const bool stop = (kcomm == nl) || (max_levels > 0 && level + 1 >= max_levels) || (N - N_start < T);
             DevCSR nxt;
-            if (!stop) dist_coarsen(g, wk, cur, nl, kcomm, newid, minmem, unit, nxt, bounds, maxdeg, dmax);
+            if (!stop) {
+                if (di.backend == 0) dist_coarsen_s2o(g, wk, cur, nl, kcomm, newid, minmem, unit, nxt, bounds, maxdeg, dmax);
+                else dist_coarsen(g, wk, cur, nl, kcomm, newid, minmem, unit, nxt, bounds, maxdeg, dmax);
+            }
             dfree(minmem, st);
             dfree(pos, st);
             dfree(newid, st);
@@ -2230,7 +2590,12 @@ void gala_graph_free(gala_graph g) {
     DevCache* const mine = g->cache;
     PoolScope pool_scope(g->cache);
     const bool dist = g->di != nullptr;
-    if (g->di) { delete g->di; g->di = nullptr; }   // communicators are cached (comm_for)
+    if (g->di) {   // communicators are cached (comm_for); the fabric region is this handle's
+        if (g->stream) cudaStreamSynchronize(g->stream);
+        fabric_release(*g->di);
+        delete g->di;
+        g->di = nullptr;
+    }
     // GALA_DEBUG_FREE=1: host time of each teardown step on stderr (e2e create/run/free cycles)
     static const bool dbg = getenv("GALA_DEBUG_FREE") != nullptr;
     auto t_prev = std::chrono::steady_clock::now();
@@ -2338,6 +2703,9 @@ gala_status gala_set_option(gala_graph g, const char* key, int64_t value) {
         if (value < 0 || value > 2) return set_err(GALA_E_INVALID, "sync_mode: 0 adaptive, 1 dense, 2 sparse");
         g->sync_mode = (int)value;
         if (g->di) g->di->sync_mode = (int)value;
+    } else if (k == "dist_backend") {
+        if (value < 0 || value > 1) return set_err(GALA_E_INVALID, "dist_backend: 0 fabric (peer memory), 1 host-driven NCCL");
+        if (g->di) g->di->backend = (int)value;
     } else return set_err(GALA_E_INVALID, "unknown option %s", key);
     return GALA_OK;
 }
@@ -2466,6 +2834,14 @@ gala_status gala_graph_from_csr_dist(const void* uid128, int rank, int world, in
     const int64_t n_own = v_end - v_begin;
     if (local_row_ptr[0] != 0 || local_row_ptr[n_own] < 0) return set_err(GALA_E_INVALID, "local row_ptr[0] != 0");
     const bool loop = memcmp(uid128, "GALALOOP", 8) == 0;
+    if (loop && world > 1) {
+        // loopback ranks share one CUDA context: a kernel loaded lazily on first use waits for the
+        // context to go idle, which a peer's fabric barrier kernel (spinning for this rank) never
+        // does -- the ranks would deadlock until the barrier timeout
+        const char* ml = getenv("CUDA_MODULE_LOADING");
+        if (!ml || strcmp(ml, "EAGER") != 0)
+            return set_err(GALA_E_INVALID, "loopback with world > 1 needs CUDA_MODULE_LOADING=EAGER (set before CUDA starts)");
+    }
     if (!loop && !nccl_api().load()) return set_err(GALA_E_NCCL, "libnccl.so.2 could not be loaded");
     gala_graph_s* g = new gala_graph_s();
     PoolScope pool_scope(nullptr);
@@ -2492,6 +2868,7 @@ gala_status gala_graph_from_csr_dist(const void* uid128, int rank, int world, in
         }
         g->dbounds0[world] = b1[world - 1];
         if (g->dbounds0[world] != n_global) { set_err(GALA_E_INVALID, "owned ranges do not cover n"); throw GalaError{GALA_E_INVALID}; }
+        fabric_setup(g, *g->di, n_global);   // peer-memory region of the device-resident iteration (collective)
         const int64_t nnz = local_row_ptr[n_own];
         g->nnz0 = nnz;
         g->g0.n = n_global;

@@ -938,15 +938,27 @@ __global__ void __launch_bounds__(HUB_BT) k_hub_agg(QView queue, DecideArgs a, H
         int* gk = h.keys + toff;
         ull* gv = h.vals + toff;
         const unsigned gmask = (unsigned)(cap - 1);
-        for (int t = threadIdx.x; t < m; t += HUB_BT) {
-            const int slot = list[t];
-            const int c = keys[slot];
-            const ull wv = (ull)vals[slot];
-            keys[slot] = -1;
-            vals[slot] = 0;
-            bool fresh;
-            int gs = ht_insert<ull>(c, wv, gk, gv, gmask, hub_hash(c, gmask), (int)min(cap, (long long)INT_MAX), &fresh);
-            if (fresh) h.list[loff + atomicAdd(&h.cnt[i], 1)] = gs;
+        for (int t0 = threadIdx.x & ~31; t0 < m; t0 += HUB_BT) {   // warp-uniform trips
+            const int t = t0 + lane;
+            bool fresh = false;
+            int gs = -1;
+            if (t < m) {
+                const int slot = list[t];
+                const int c = keys[slot];
+                const ull wv = (ull)vals[slot];
+                keys[slot] = -1;
+                vals[slot] = 0;
+                gs = ht_insert<ull>(c, wv, gk, gv, gmask, hub_hash(c, gmask), (int)min(cap, (long long)INT_MAX), &fresh);
+            }
+            // one list-counter atomic per warp instead of one per fresh key
+            const unsigned fm = __ballot_sync(FULLMASK, fresh);
+            if (fm) {
+                const int lead = __ffs(fm) - 1;
+                int base = 0;
+                if (lane == lead) base = atomicAdd(&h.cnt[i], __popc(fm));
+                base = __shfl_sync(FULLMASK, base, lead);
+                if (fresh) h.list[loff + base + __popc(fm & lanemask_lt())] = gs;
+            }
         }
         __syncthreads();
         if (threadIdx.x == 0) s_cnt = 0;
@@ -995,13 +1007,30 @@ __global__ void __launch_bounds__(HUB_EVAL_BT) k_hub_eval(QView queue, DecideArg
         const long long toff = h.toff[i], loff = h.loff[i];
         A best;
         best.init(a.idbits, a.idmask);
-        for (long long t = t0 + threadIdx.x; t < t1; t += HUB_EVAL_BT) {
-            const long long slot = toff + h.list[loff + t];
-            const int c = h.keys[slot];
-            const long long wc = (long long)h.vals[slot];
-            h.keys[slot] = -1;
-            h.vals[slot] = 0;
-            if (c != cv) best.offer(gain<ST>(qW, p, wc, a.Sig[c], dv), c);
+        // the slice's list entries, then their slots, then Sigma_tot of their communities, each
+        // batch issued before any use: three dependent load rounds per thread, not three per entry
+        constexpr int U = HUB_EV / HUB_EVAL_BT;
+        long long slot[U];
+        int c[U];
+        long long wc[U], sg[U];
+#pragma unroll
+        for (int k = 0; k < U; ++k) {
+            const long long t = t0 + threadIdx.x + (long long)k * HUB_EVAL_BT;
+            slot[k] = t < t1 ? toff + h.list[loff + t] : -1;
+        }
+#pragma unroll
+        for (int k = 0; k < U; ++k) {
+            c[k] = slot[k] >= 0 ? h.keys[slot[k]] : -1;
+            wc[k] = slot[k] >= 0 ? (long long)h.vals[slot[k]] : 0;
+        }
+#pragma unroll
+        for (int k = 0; k < U; ++k) sg[k] = (c[k] >= 0 && c[k] != cv) ? a.Sig[c[k]] : 0;
+#pragma unroll
+        for (int k = 0; k < U; ++k) {
+            if (slot[k] < 0) continue;
+            h.keys[slot[k]] = -1;
+            h.vals[slot[k]] = 0;
+            if (c[k] != cv) best.offer(gain<ST>(qW, p, wc[k], sg[k], dv), c[k]);
         }
 #pragma unroll
         for (int off = 16; off > 0; off >>= 1) best.xor_merge(off);

@@ -191,3 +191,9 @@ __global__ void k_restrict_rp(long long n, long long lo, long long hi, const int
         out[v] = x - a;
     }
 }
+
+// partial coarse row lengths (send-to-owner phase 2): len[c] = rp[c + 1] - rp[c]
+__global__ void k_row_lengths(long long k, const int64_t* __restrict__ rp, long long* __restrict__ len) {
+    for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c < k; c += (long long)gridDim.x * blockDim.x)
+        len[c] = rp[c + 1] - rp[c];
+}
