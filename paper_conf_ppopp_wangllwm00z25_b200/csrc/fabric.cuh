@@ -53,6 +53,8 @@ struct FabDev {
     long long bnd[FAB_MAXP + 1]; // owned vertex ranges of this level
     long long off[FAB_MAXP];     // slot start (ints, even) of every sender in an inbox parity
     int force_dense;             // option sync_mode = 1: every sender exchanges its whole slice
+    ull timeout_ns;              // barrier wait before giving up (env GALA_FABRIC_TIMEOUT_MS, default 20 s)
+    ull* diag;                   // this rank: [epoch, counter seen] of the barrier that timed out
 };
 
 __device__ __forceinline__ ull ld_acquire_sys(const ull* p) {
@@ -62,8 +64,8 @@ __device__ __forceinline__ ull ld_acquire_sys(const ull* p) {
 }
 
 // All ranks arrive (one system-scope atomic on every peer's counter), then wait until this
-// rank's counter shows P arrivals for this barrier.  A barrier that waits > 20 s (a peer
-// died) sets the error flag and lets the run finish instead of hanging the GPU.
+// rank's counter shows P arrivals for this barrier.  A barrier that waits longer than the
+// timeout (a peer died) sets the error flag and lets the run finish instead of hanging the GPU.
 __global__ void k_fab_barrier(FabDev f) {
     const int lane = threadIdx.x;
     __threadfence_system();
@@ -71,8 +73,13 @@ __global__ void k_fab_barrier(FabDev f) {
     if (lane == 0) {
         const ull target = (*f.epoch + 1) * (ull)f.P;
         const ull t0 = globaltimer_ns();
-        while (ld_acquire_sys(f.arrive[f.rank]) < target) {
-            if (globaltimer_ns() - t0 > 20000000000ull) { *f.err = 1; break; }
+        ull seen;
+        while ((seen = ld_acquire_sys(f.arrive[f.rank])) < target) {
+            if (globaltimer_ns() - t0 > f.timeout_ns) {
+                if (!*f.err) { f.diag[0] = *f.epoch; f.diag[1] = seen; }
+                *f.err = 1;
+                break;
+            }
             __nanosleep(64);
         }
         *f.epoch += 1;

@@ -563,7 +563,18 @@ static void launch_single(gala_graph_s* g, Work& wk, const DecideArgs& a, typena
         CKL();
         tm.end(KC_DEC_SINGLE, e);
     }
-    launch_hub<M, UNIT>(g, wk, a, qW, p, tm, wk.hub_on ? fk.branch(3) : st);
+    if (wk.hub_on) {   // singleton hubs: chunked argmax, no tables
+        const QView q = qview(wk.queues, wk.qcap, BIN_HUB);
+        cudaStream_t hs = fk.branch(3);
+        e = tm.begin();
+        k_hub_prep<<<1, 1024, 0, hs>>>(q, wk.ctr, wk.hw);
+        CKL();
+        k_hub_single_chunk<M, UNIT><<<g->num_sms * 8, HUB_BT, 0, hs>>>(q, a, wk.hw, qW, p);
+        CKL();
+        k_hub_single_final<M, UNIT><<<g->num_sms, 256, 0, hs>>>(q, a, wk.hw);
+        CKL();
+        tm.end(KC_DEC_HUB, e);
+    }
 }
 
 // grid of the short-row block kernel (rows <= opt_block_split): resident blocks per SM for its
@@ -717,7 +728,7 @@ static void prepare_level_tables(gala_graph_s* g, Work& wk, const DevCSR& G, int
         h.own = dalloc<long long>(nh, st);
         wk.hub_ncap = nh;
     }
-    const long long np = lc / HUB_EV + nh + 1;   // evaluation slices
+    const long long np = lc / HUB_CH + nh + 1;   // evaluation slices (HUB_EV) or singleton chunks (HUB_CH)
     if (np > wk.hub_pcap) {
         char* part = static_cast<char*>(h.part);
         dfree(part, st);
@@ -813,6 +824,7 @@ static void level_loop(gala_graph_s* g, Work& wk, std::vector<IterLog>& out, boo
     int log_base_host = 0;   // mirror of carry->log_base
     if (stepwise || first_single) {
         for (;;) {
+            pre_launch();
             issue(0ull, first_single);
             CK(cudaMemcpyAsync(wk.h_carry, wk.carry, sizeof(Carry), cudaMemcpyDeviceToHost, st));
             const int slot = (int)out.size() - log_base_host;
@@ -860,8 +872,8 @@ static void level_loop(gala_graph_s* g, Work& wk, std::vector<IterLog>& out, boo
         }
         CK(cudaStreamEndCapture(st, &body));
         CK(cudaGraphInstantiate(&exec, graph, 0));
-        pre_launch();
         for (;;) {
+            pre_launch();
             CK(cudaGraphLaunch(exec, st));
             CK(cudaMemcpyAsync(wk.h_carry, wk.carry, sizeof(Carry), cudaMemcpyDeviceToHost, st));
             CK(cudaStreamSynchronize(st));
@@ -1555,6 +1567,7 @@ struct DistInfo {
     void* region = nullptr;
     std::vector<void*> peers;
     FabDev fab = {};
+    bool failed = false;   // a run ended in an error: peers may still touch the region
 };
 
 // Symmetric region of a rank (cudaMalloc: CUDA IPC needs it), byte offsets:
@@ -1587,10 +1600,14 @@ static void fabric_setup(gala_graph_s* g, DistInfo& di, int64_t n) {
     }
     f.epoch = reinterpret_cast<ull*>(static_cast<char*>(di.region) + 256);
     f.err = reinterpret_cast<int*>(static_cast<char*>(di.region) + 264);
+    f.diag = reinterpret_cast<ull*>(static_cast<char*>(di.region) + 272);
+    const char* to = getenv("GALA_FABRIC_TIMEOUT_MS");
+    f.timeout_ns = (to && atoll(to) > 0 ? (ull)atoll(to) : 20000ull) * 1000000ull;
     f.istride = istride;
 }
 static void fabric_release(DistInfo& di) {
     if (!di.region) return;
+    if (di.failed) cudaDeviceSynchronize();   // stragglers (loopback: same device) finish first
     if (di.comm) di.comm->release_region(di.peers);
     cudaFree(di.region);
     di.region = nullptr;
@@ -2042,8 +2059,9 @@ static void dist_phase1_fab(gala_graph_s* g, Work& wk, const DevCSR& G, const Di
                             std::vector<IterLog>& out, bool single_ok) {
     block_setup<M, UNIT>(g);
     g->cur_n = G.n;
-    // ranks sharing a process (loopback) meet before launching the level's graph, so no rank's
-    // barrier kernel spins while another rank's thread is still instantiating
+    // ranks sharing a process (loopback) meet on the host before every launch of fabric work, so
+    // no rank's barrier kernel spins while another rank's thread is still in host calls that may
+    // wait for the whole (shared) device: graph instantiation, pool growth, pageable copies
     level_loop(
         g, wk, out, single_ok, tm,
         [&](unsigned long long cond, bool single) {
@@ -2128,6 +2146,7 @@ static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_level
             DistLevel L;
             if (fab) {
                 dist_level_setup(g, cur, bounds, L);
+                cm.host_barrier();   // loopback: every rank's host-side level setup done (see dist_phase1_fab)
                 dist_level_start_fab(g, wk, cur, L, qW128, p);
             } else {
                 k_reduce<256><<<wk.reduce_grid, 256, 0, st>>>((int)nl, (int)lv0, (int)lv1, wk.dp, wk.s_live(), wk.Sig, wk.part_dc,
@@ -2162,9 +2181,16 @@ static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_level
 #undef DIST_FAB
                 L.release(st);
                 int err = 0;
+                ull diag[2] = {0, 0};
                 CK(cudaMemcpyAsync(&err, di.fab.err, sizeof(int), cudaMemcpyDeviceToHost, st));
+                CK(cudaMemcpyAsync(diag, di.fab.diag, sizeof(diag), cudaMemcpyDeviceToHost, st));
                 CK(cudaStreamSynchronize(st));
-                if (err) throw CommError{"fabric: a peer rank stopped answering (barrier timeout)"};
+                if (err) {
+                    char msg[256];
+                    snprintf(msg, sizeof msg, "fabric: a peer rank stopped answering (rank %d, level %d, barrier %llu, "
+                             "arrivals %llu of %llu)", cm.rank, level, diag[0], diag[1], (diag[0] + 1) * (ull)cm.world);
+                    throw CommError{msg};
+                }
             }
             for (int it = 0; !fab; ++it) {
                 const bool single = it == 0 && g->opt_singleton && single_ok;
@@ -2271,11 +2297,13 @@ static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_level
         g->launches = g_launches - launches0;
     } catch (CommError& e) {
         cm.abort();
+        di.failed = true;
         dfree(lmoves, st); dfree(gmoves, st); dfree(newC, st); dfree(dcnt, st); dfree(vec, st);
         set_err(GALA_E_NCCL, "%s", e.msg.c_str());
         throw GalaError{GALA_E_NCCL};
     } catch (...) {
         cm.abort();   // peers blocked in a collective raise instead of waiting forever
+        di.failed = true;
         dfree(lmoves, st); dfree(gmoves, st); dfree(newC, st); dfree(dcnt, st); dfree(vec, st);
         throw;
     }

@@ -1081,6 +1081,92 @@ __global__ void __launch_bounds__(256) k_hub_final(QView queue, DecideArgs a, Hu
     if (threadIdx.x == 0 && k) atomicAdd(&a.ctr->bin_k[BIN_HUB], k);
 }
 
+// First iteration of a level (all singletons, rows with distinct columns): a hub needs no
+// aggregation at all -- score(u) = qW w(v,u) - p d(u) d(v) per entry (decide_single_bin's closed
+// form).  Any block takes any HUB_CH-entry chunk of any hub (prefix h.pref from k_hub_prep) and
+// writes the chunk's partial argmax; k_hub_single_final merges them per hub.
+template <int M, bool UNIT>
+__global__ void __launch_bounds__(HUB_BT) k_hub_single_chunk(QView queue, DecideArgs a, HubWork h,
+                                                             typename ModeT<M>::ST qW, typename ModeT<M>::ST p) {
+    typedef typename ModeT<M>::ST ST;
+    typedef Arg<ST, ModeT<M>::PK> A;
+    constexpr int E = HUB_CH / HUB_BT;
+    __shared__ A r_a[HUB_BT / 32];
+    __shared__ long long s_item;
+    const int lane = lane_id(), wib = threadIdx.x >> 5;
+    const long long count = (long long)a.ctr->bin_count[BIN_HUB];
+    if (count == 0) return;
+    const long long total = h.pref[count];
+    A* part = reinterpret_cast<A*>(h.part);
+    for (;;) {
+        if (threadIdx.x == 0) s_item = (long long)atomicAdd(&a.ctr->cursor[BIN_HUB], 1ull);
+        __syncthreads();
+        const long long item = s_item;
+        if (item >= total) break;
+        const long long i = hub_find(h.pref, count, item);
+        const QRec q = queue[i];
+        const long long j0 = (item - h.pref[i]) * HUB_CH;
+        int uu[E];
+        long long ww[E], du[E];
+#pragma unroll
+        for (int k = 0; k < E; ++k) {
+            const long long j = j0 + threadIdx.x + k * HUB_BT;
+            uu[k] = j < q.deg ? a.col[q.beg + j] : -1;
+            ww[k] = (j < q.deg && !UNIT) ? a.w[q.beg + j] : 1;
+        }
+#pragma unroll
+        for (int k = 0; k < E; ++k) du[k] = (uu[k] >= 0 && uu[k] != q.v) ? a.Sig[uu[k]] : 0;
+        A best;
+        best.init(a.idbits, a.idmask);
+#pragma unroll
+        for (int k = 0; k < E; ++k)
+            if (uu[k] >= 0 && uu[k] != q.v) best.offer(gain<ST>(qW, p, ww[k], du[k], q.dv), uu[k]);
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) best.xor_merge(off);
+        if (lane == 0) r_a[wib] = best;
+        __syncthreads();
+        if (wib == 0) {
+            if (lane < HUB_BT / 32) best = r_a[lane];
+            else best.init(a.idbits, a.idmask);
+#pragma unroll
+            for (int off = 16; off > 0; off >>= 1) best.xor_merge(off);
+            if (lane == 0) part[item] = best;
+        }
+        __syncthreads();
+    }
+}
+
+template <int M, bool UNIT>
+__global__ void __launch_bounds__(256) k_hub_single_final(QView queue, DecideArgs a, HubWork h) {
+    typedef typename ModeT<M>::ST ST;
+    typedef Arg<ST, ModeT<M>::PK> A;
+    const int lane = lane_id();
+    const long long count = (long long)a.ctr->bin_count[BIN_HUB];
+    const A* part = reinterpret_cast<const A*>(h.part);
+    ull my_k = 0;
+    const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+    for (long long i = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < count; i += nw) {
+        A best;
+        best.init(a.idbits, a.idmask);
+        for (long long s = h.pref[i] + lane; s < h.pref[i + 1]; s += 32) {
+            A o = part[s];
+            if (o.valid()) best.offer(o.score(), o.comm());
+        }
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) best.xor_merge(off);
+        if (lane == 0) {
+            const QRec q = queue[i];
+            int tgt = q.v;
+            if (best.valid() && best.score() > (ST)0 && best.comm() < q.v) tgt = best.comm();
+            if (a.check && a.dp[q.v] != 0) atomicAdd(&a.ctr->dp_mismatch, 1ull);
+            a.nextC[q.v] = tgt;
+            my_k += (ull)q.deg;
+        }
+    }
+    ull k = block_sum_ull<256>(my_k);
+    if (threadIdx.x == 0 && k) atomicAdd(&a.ctr->bin_k[BIN_HUB], k);
+}
+
 // per level: number of rows longer than t, and the table / list space they can need
 __global__ void k_hub_size(long long n, const int64_t* __restrict__ rp, long long t, long long nlev,
                            ull* __restrict__ out) {

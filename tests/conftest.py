@@ -3,14 +3,6 @@ import sys
 
 import pytest
 
-# the loopback multi-GPU tests run several "ranks" as streams of one device whose fabric
-# barriers spin until every rank arrives: give every stream its own hardware queue (must be
-# set before the CUDA context exists)
-os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
-# ... and load every kernel up front: a kernel loaded lazily on first use waits for the shared
-# context to go idle, which a peer's spinning barrier prevents (libgala refuses loopback world > 1
-# without this)
-os.environ.setdefault("CUDA_MODULE_LOADING", "EAGER")
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 if ROOT not in sys.path:

@@ -1,22 +1,21 @@
-"""Multi-GPU path (§8(e), a10) exercised on one GPU: `world` ranks run as threads
-of one process through the loopback communicator (test hook); the partitioned
-algorithm (owned-range prune/decide, dense/sparse label exchange, replicated
-Sigma_tot updates, all-reduced counters, distributed coarsening and
-re-partitioning) must reproduce the oracle bit for bit at every iteration.
+"""Multi-GPU path (§8(e), a10) exercised on one GPU: `world` ranks run as threads of one
+process through the loopback communicator (test hook); the partitioned algorithm (owned-range
+prune/decide, dense/sparse label exchange, replicated Sigma_tot updates, summed counters,
+distributed coarsening and re-partitioning) must reproduce the oracle bit for bit at every
+iteration.  Each case runs in its own process (tests/dist_loopback_case.py).
 
 Both backends: 0 = the fabric (device-resident iteration over peer memory, fabric.cuh:
-per-sender dense/sparse slots, on-device barriers, mirror-block delta d', CUDA-graph
-captured), 1 = host-driven collectives (one host round trip per iteration)."""
-import threading
+per-sender dense/sparse slots, on-device barriers, mirror-block delta d', send-to-owner phase
+2, CUDA-graph captured), 1 = host-driven collectives (one host round trip per iteration)."""
+import json
+import os
+import subprocess
+import sys
 
-import numpy as np
 import pytest
 
-import graphgen as gg
-import oracle
-import paper_conf_ppopp_wangllwm00z25_b200 as gala
-
 pytestmark = pytest.mark.gpu
+HERE = os.path.dirname(os.path.abspath(__file__))
 
 
 @pytest.fixture(scope="module", autouse=True)
@@ -26,67 +25,27 @@ def _need_gpu():
         pytest.skip("no CUDA device")
 
 
-def run_dist(g, world, gamma=1.0, sync_mode=0, trace=2, backend=0, **opts):
-    bounds = gala.partition_ranges(g.row_ptr, world)
-    uid = gala.loopback_unique_id()
-    out = [None] * world
-    err = []
-
-    def worker(r):
-        try:
-            lrp, lcol, lw = gala.local_rows(g.row_ptr, g.col, g.w, bounds[r], bounds[r + 1])
-            h = gala.Graph.from_csr_dist(uid, r, world, 0, g.n, int(bounds[r]), int(bounds[r + 1]), lrp, lcol, lw)
-            h.set_option("trace", trace)
-            h.set_option("sync_mode", sync_mode)
-            h.set_option("dist_backend", backend)
-            for k, v in opts.items():
-                h.set_option(k, v)
-            h.run(gamma=gamma)
-            out[r] = dict(labels=h.communities(), N=h.numerator()[0], trace=h.trace(labels=trace >= 2),
-                          stats=h.stats())
-            h.free()
-        except Exception as e:  # noqa: BLE001
-            err.append(e)
-
-    ts = [threading.Thread(target=worker, args=(r,)) for r in range(world)]
-    for t in ts:
-        t.start()
-    for t in ts:
-        t.join(timeout=600)
-    if err:
-        raise err[0]
-    return out
-
-
-def check(g, world, gamma=1.0, sync_mode=0, backend=0, trace=2, **opts):
-    o = oracle.louvain(g, gamma=gamma, prune=True, trace=2)
-    res = run_dist(g, world, gamma=gamma, sync_mode=sync_mode, backend=backend, trace=trace, **opts)
-    for r in res:
-        assert np.array_equal(r["labels"], o.labels)
-        assert r["N"] == o.N
-        assert len(r["trace"]) == len(o.records)
-        for x, y in zip(o.records, r["trace"]):
-            assert (x.level, x.iter) == (y["level"], y["iter"])
-            if trace >= 2:
-                assert np.array_equal(x.labels, y["labels"]), f"level {x.level} iter {x.iter}"
-            assert x.N == y["N"] and x.n_moved == y["n_moved"]
-            assert x.n_active == y["n_active"] and x.n_pruned == y["n_pruned"]
-    return res
+def check(graph, world, gamma=1.0, sync_mode=0, backend=0, trace=2, **opts):
+    cfg = dict(graph=graph, world=world, gamma=gamma, sync_mode=sync_mode, backend=backend, trace=trace, opts=opts)
+    env = dict(os.environ, CUDA_MODULE_LOADING="EAGER", GALA_FABRIC_TIMEOUT_MS="10000")
+    r = subprocess.run([sys.executable, os.path.join(HERE, "dist_loopback_case.py"), json.dumps(cfg)],
+                       capture_output=True, text=True, timeout=600, env=env)
+    assert r.returncode == 0, (r.stdout[-2000:], r.stderr[-3000:])
+    return json.loads(r.stdout.strip().splitlines()[-1])
 
 
 @pytest.mark.parametrize("backend", [0, 1])
 @pytest.mark.parametrize("world", [2, 3, 4])
 def test_dist_lfr_small(world, backend):
-    res = check(gg.make("lfr_small"), world, backend=backend)
-    d = res[0]["stats"]["dist"]
+    res = check("lfr_small", world, backend=backend)
+    d = res["dist"][0]
     assert d["world"] == world and d["dense_iters"] + d["sparse_iters"] > 0
 
 
 @pytest.mark.parametrize("backend", [0, 1])
 @pytest.mark.parametrize("sync_mode", [1, 2])
 def test_dist_forced_sync_modes(sync_mode, backend):
-    res = check(gg.make("rmat_small"), 2, sync_mode=sync_mode, backend=backend)
-    d = res[0]["stats"]["dist"]
+    d = check("rmat_small", 2, sync_mode=sync_mode, backend=backend)["dist"][0]
     if sync_mode == 1:   # forced dense: every exchange dense
         assert d["dense_iters"] > 0 and d["sparse_iters"] == 0
     elif backend == 1:   # forced sparse (host backend): every exchange sparse
@@ -97,20 +56,19 @@ def test_dist_forced_sync_modes(sync_mode, backend):
 
 @pytest.mark.parametrize("backend", [0, 1])
 def test_dist_karate_and_weighted(backend):
-    check(gg.karate(), 2, backend=backend)
-    g = gg.random_graph(400, 3000, seed=77, max_w=5, self_loops=4)
-    check(g, 3, gamma=1.5, backend=backend)
+    check("karate", 2, backend=backend)
+    check(["random", 400, 3000, 77, 5, 4], 3, gamma=1.5, backend=backend)
 
 
 @pytest.mark.parametrize("backend", [0, 1])
 def test_dist_more_ranks_than_busy_rows(backend):
-    check(gg.make("karate"), 4, backend=backend)
+    check("karate", 4, backend=backend)
 
 
 @pytest.mark.parametrize("backend", [0, 1])
 def test_dist_hub_path(backend):
     """Rows split over blocks (hub path) on partitioned ranks, coarse levels included."""
-    check(gg.make("rmat_small"), 3, backend=backend, bin_sub4=4, bin_sub8=8, bin_sub16=16, bin_sub32=32,
+    check("rmat_small", 3, backend=backend, bin_sub4=4, bin_sub8=8, bin_sub16=16, bin_sub32=32,
           bin_warp=32, bin_warp512=32, bin_block=32)
 
 
@@ -118,12 +76,11 @@ def test_dist_hub_path(backend):
 def test_dist_fabric_delta_modes(delta):
     """§3.5 across ranks: forced delta (mirror-block pushes every iteration), forced recompute
     and the adaptive choice give identical d' (the per-iteration N and labels match)."""
-    check(gg.make("lfr_small"), 3, backend=0, delta_update=delta)
+    check("lfr_small", 3, backend=0, delta_update=delta)
 
 
 def test_dist_fabric_graph_mode():
     """trace=1: the fabric iterations run inside the level's conditional CUDA graph (no host
     round trip per iteration); per-iteration N / counts still match the oracle."""
-    res = check(gg.make("lfr_small"), 4, backend=0, trace=1)
-    tr = res[0]["trace"]
-    assert any(r["us"] > 0 for r in tr)
+    res = check("lfr_small", 4, backend=0, trace=1)
+    assert any(u > 0 for u in res["us"])
