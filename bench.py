@@ -275,6 +275,7 @@ def main():
     import torch
     import graphgen as gg
     import paper_conf_ppopp_wangllwm00z25_b200 as gala
+    import quality
 
     if world > 1 or args.force_dist:
         import torch.distributed as dist
@@ -445,7 +446,7 @@ def main():
         "gteps_scanned_all_levels": scanned / total_s / 1e9,
         "step_ms": [round(x, 3) for x in step_ms],
         "modularity": Q,
-        "nmi_vs_planted": (gala.nmi_device(labels, g.truth) if getattr(g, "truth", None) is not None else None),
+        "nmi_vs_planted": (quality.nmi_device(labels, g.truth) if getattr(g, "truth", None) is not None else None),
         "pruned_fraction_per_iteration": pruned,
         "levels": len(last_stats["levels"]),
         "iterations": sum(lv["iters"] for lv in last_stats["levels"]),
@@ -456,6 +457,12 @@ def main():
         "phase1_roofline": {"bound": "hbm", "scope": "level 0, all phase-1 kernels", "achieved": p1_achieved,
                             "peak": peak, "unit": "GB/s", "frac": p1_achieved / peak if p1_achieved else None,
                             "alg_bytes": l0_bytes / args.steps},
+        "phase2_roofline": ({"bound": "hbm", "achieved": kstats["phase2"]["alg_bytes"] / (kstats["phase2"]["ms"] / 1e3) / 1e9,
+                             "peak": peak, "unit": "GB/s",
+                             "frac": kstats["phase2"]["alg_bytes"] / (kstats["phase2"]["ms"] / 1e3) / 1e9 / peak,
+                             "alg_bytes_per_run": kstats["phase2"]["alg_bytes"] / len(inst_ms)}
+                            if kstats.get("phase2", {}).get("ms") else None),
+        "phase2_share": sum(lv["ms_phase2"] for lv in last_stats["levels"]) / (total_s * 1e3 / args.steps),
         "decide_roofline": {"achieved": dec_by / (dec_ms / 1e3) / 1e9 if dec_ms else None, "peak": peak,
                             "frac": (dec_by / (dec_ms / 1e3) / 1e9) / peak if dec_ms else None,
                             "ms_per_step": dec_ms / max(len(inst_ms), 1)},

@@ -160,8 +160,14 @@ void gala_graph_free(gala_graph g);
  *                    4 8 16 32 128 512 16384).  Rows longer than "bin_block" take the
  *                    multi-block hub path (chunks of 1024 entries over all SMs).
  *   "delta_update"   0 = always recompute d', 1 = always delta, 2 = adaptive (default)
+ *   "delta_den"      [1, 64] adaptive rule: delta iff the moved vertices' row entries are
+ *                          <= nnz / delta_den (default 2)
  *   "force_i128"     0/1   use the 128-bit gain path even when 64-bit suffices
- *   "force_wide"     0/1   use unpacked 64-bit gains / aggregates (no packed keys)
+ *   "force_wide"     0/1/2 1: unpacked 64-bit gains everywhere (no packed keys); 2: the level runs
+ *                          as if it needed them but the short-row bins may still pack (bin_packed)
+ *   "bin_packed"     0/1   on a level whose hubs need unpacked (score, c) keys, the bins of rows
+ *                          <= bin_warp512 still use packed keys when max(p,q) W row 2^idbits < 2^62
+ *                          (default 1; unit-weight levels only)
  *   "singleton"      0/1   first iteration of a level via the singleton fast path (default 1)
  *   "ckey"           0/1   keep a per-entry copy of C[col] on level 0, maintained by the delta
  *                          update (default 0; trades nnz*4 bytes for one gather per entry)

@@ -254,8 +254,8 @@ __global__ void __launch_bounds__(256) k_fab_dp_delta(IterCounters* __restrict__
                                                       const int32_t* __restrict__ it_chunk,
                                                       const int32_t* __restrict__ stamp, int64_t* __restrict__ dp,
                                                       const Carry* __restrict__ carry, long long nnz_own, int mode,
-                                                      long long lv0, long long lv1) {
-    if (!use_delta(ctr, nnz_own, mode, 1, 2)) return;
+                                                      long long lv0, long long lv1, int den) {
+    if (!use_delta(ctr, nnz_own, mode, 1, den)) return;
     if (blockIdx.x == 0 && threadIdx.x == 0) ctr->delta_used = 1;
     const int iter_id = carry->iter;
     const int lane = lane_id();

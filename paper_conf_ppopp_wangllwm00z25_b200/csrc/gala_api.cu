@@ -108,11 +108,14 @@ struct gala_graph_s {
     int64_t* s0 = nullptr;
     // options
     int opt_prune = 1, opt_prune_check = 0, opt_trace = 0, opt_check = 0, opt_timing = 0, opt_max_iters = 0;
+    int opt_delta_den = 2;   // adaptive d' update: delta iff moved row entries <= nnz / opt_delta_den
     int opt_delta = 2, opt_force_i128 = 0, opt_force_wide = 0, opt_cuda_graph = 1, opt_log_cap = 4096, opt_singleton = 1, opt_verbose = 0, opt_agg_big_chunk = 1,
         opt_agg_chunk = AGG_CH, opt_agg_scap = 8192;
     long long opt_agg_big_ent = 32768;   // communities with more entries take the chunked big path (any table size)
     int opt_block_split = 1024;
     int opt_agg_bound = 1;
+    int opt_agg_dense = 1;
+    int opt_bin_packed = 1;  // DM_W64 levels: packed argmax keys for the short-row bins where they fit   // phase 2: dense k x k accumulation when k <= AGG_DENSE_K and nnz >= 4 k^2
     bool rows_distinct0 = false;   // level-0 rows strictly increasing (no duplicate entries)
     bool self0 = true;             // level 0 has a self-loop (s0 not all zero)
     bool ckey_ok = false;          // level 0 may use the per-entry neighbour-community array (ckey)
@@ -545,6 +548,15 @@ static void launch_hub(gala_graph_s* g, Work& wk, const DecideArgs& a, typename 
     tm.end(KC_DEC_HUB, e);
 }
 
+// DM_FAST's packed (score, -c) argmax keys need max(p,q) W d(v) 2^idbits < 2^62 for the vertices
+// a kernel evaluates -- not for the level's largest degree.  On a unit-weight level d(v) is the row
+// length, so the bins of rows up to `rowmax` can use packed keys (one 64-bit max per reduction
+// step) even when the level's hubs need DM_W64's (score, c) pairs.  Same integers either way.
+static bool packed_ok(const gala_graph_s* g, int idbits, int64_t rowmax) {
+    return (long double)std::max(g->p, g->q) * (long double)g->W * (long double)std::max<int64_t>(rowmax, 1) *
+               (long double)((int64_t)1 << idbits) < 0x1p62L;
+}
+
 template <int M, bool UNIT>
 static void launch_single(gala_graph_s* g, Work& wk, const DecideArgs& a, typename ModeT<M>::ST qW,
                           typename ModeT<M>::ST p, Timer& tm, int64_t maxdeg) {
@@ -552,14 +564,21 @@ static void launch_single(gala_graph_s* g, Work& wk, const DecideArgs& a, typena
     const int grid = g->num_sms * 8;
     cudaStream_t st = g->stream;
     Fork fk(g);
+    // rows <= bins[BIN_WARP2] with packed argmax keys where they fit (packed_ok)
+    bool fast = false;
+    if constexpr (M == DM_W64 && UNIT)
+        fast = g->opt_bin_packed && g->opt_force_wide != 1 && packed_ok(g, a.idbits, std::min<int64_t>(maxdeg, g->bins[BIN_WARP2]));
     cudaEvent_t e = tm.begin();
-    k_decide_single_small<M, UNIT><<<grid, 256, 0, st>>>(wk.queues, qs, a, qW, p);
+    if (fast) k_decide_single_small<DM_FAST, UNIT><<<grid, 256, 0, st>>>(wk.queues, qs, a, qW, p);
+    else k_decide_single_small<M, UNIT><<<grid, 256, 0, st>>>(wk.queues, qs, a, qW, p);
     CKL();
     tm.end(KC_DEC_SINGLE, e);
     for (int b = BIN_WARP; b <= BIN_BLOCK; ++b) {
         if (maxdeg <= g->bins[b - 1]) break;
         e = tm.begin();
-        k_decide_single<M, UNIT><<<grid, 256, 0, fk.branch(b - BIN_WARP)>>>(qview(wk.queues, qs, b), b, a, qW, p);
+        if (fast && b <= BIN_WARP2)
+            k_decide_single<DM_FAST, UNIT><<<grid, 256, 0, fk.branch(b - BIN_WARP)>>>(qview(wk.queues, qs, b), b, a, qW, p);
+        else k_decide_single<M, UNIT><<<grid, 256, 0, fk.branch(b - BIN_WARP)>>>(qview(wk.queues, qs, b), b, a, qW, p);
         CKL();
         tm.end(KC_DEC_SINGLE, e);
     }
@@ -577,13 +596,35 @@ static void launch_single(gala_graph_s* g, Work& wk, const DecideArgs& a, typena
     }
 }
 
-// grid of the short-row block kernel (rows <= opt_block_split): resident blocks per SM for its
-// arena, computed once per (mode, unit, arena, class).  The dynamic shared-memory limit is a
-// per-function, process-wide attribute, so `setup` (outside any graph capture) re-sets it to
-// this arena on every call: a memo hit alone would keep the limit of whichever arena was set
-// last (a smaller block_split on another handle) and the launch would fail.
+// Dynamic shared-memory limits of the block kernels.  The limit is a per-function, process-wide
+// attribute, so it is set ONCE (under a lock, before any capture) to the largest arena any handle's
+// options allow: 16384 slots (hub_smem_slots <= 16384; the short-row class uses < hub_smem_slots).
+// It is only an upper bound -- occupancy and the launch follow the dynamic shared memory each launch
+// requests -- so handles with different options (loopback ranks are threads) never race on it.
 template <int M, bool UNIT>
-static int block_lo_grid(gala_graph_s* g, int cap, bool all, bool setup = false) {
+static void block_attr_mode() {
+    const int mx = (int)block_smem_bytes<M>(16384);
+    CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
+    CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
+    CK(cudaFuncSetAttribute(k_decide_block<BLOCK_LO_BT, BLOCK_LO_E, M, UNIT, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
+    CK(cudaFuncSetAttribute(k_decide_block<BLOCK_LO_BT, BLOCK_LO_E, M, UNIT, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
+}
+static void block_attrs_once() {
+    static std::mutex mu;
+    static std::map<int, bool> done;   // per device
+    std::lock_guard<std::mutex> lk(mu);
+    const int dev = current_device();
+    if (done[dev]) return;
+    block_attr_mode<DM_FAST, true>(); block_attr_mode<DM_FAST, false>();
+    block_attr_mode<DM_W64, true>(); block_attr_mode<DM_W64, false>();
+    block_attr_mode<DM_W128, true>(); block_attr_mode<DM_W128, false>();
+    done[dev] = true;
+}
+
+// grid of the short-row block kernel (rows <= opt_block_split): resident blocks per SM for its
+// arena, computed once per (mode, unit, arena, class)
+template <int M, bool UNIT>
+static int block_lo_grid(gala_graph_s* g, int cap, bool all) {
     static std::map<std::pair<int, int>, int> memo;
     static std::mutex mu;
     const std::pair<int, int> key(cap, all ? 1 : 0);
@@ -591,10 +632,8 @@ static int block_lo_grid(gala_graph_s* g, int cap, bool all, bool setup = false)
                         : (const void*)k_decide_block<BLOCK_LO_BT, BLOCK_LO_E, M, UNIT, 1>;
     const size_t sm = block_smem_bytes<M>(cap);
     std::lock_guard<std::mutex> lk(mu);
-    if (setup) CK(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
     auto it = memo.find(key);
     if (it != memo.end()) return g->num_sms * it->second;
-    if (!setup) CK(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
     int b = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, f, BLOCK_LO_BT, sm));
     b = std::max(b, 1);
@@ -606,14 +645,35 @@ static int block_lo_grid(gala_graph_s* g, int cap, bool all, bool setup = false)
 // while a level's iteration body is being captured into a CUDA graph
 template <int M, bool UNIT>
 static void block_setup(gala_graph_s* g) {
+    block_attrs_once();
     int cap1 = 64;
     while (cap1 < 2 * std::max(g->opt_block_split, 1)) cap1 <<= 1;
-    (void)block_lo_grid<M, UNIT>(g, cap1, false, true);
-    CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                            (int)block_smem_bytes<M>(16384)));
-    // single-class block kernel: this handle's arena (another handle may have set a smaller one)
-    CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                            (int)block_smem_bytes<M>(g->hub_smem_slots)));
+    if (cap1 < g->hub_smem_slots) (void)block_lo_grid<M, UNIT>(g, cap1, false);   // the only case it launches
+}
+
+// the sub-warp and warp bins (rows <= bins[BIN_WARP2])
+template <int M, bool UNIT>
+static void launch_short_bins(gala_graph_s* g, Work& wk, const DecideArgs& a, typename ModeT<M>::ST qW,
+                              typename ModeT<M>::ST p, Timer& tm, int64_t maxdeg, Fork& fk) {
+    const long long qs = wk.qcap;
+    const int grid = g->num_sms * 8;
+    cudaStream_t st = g->stream;
+    cudaEvent_t e = tm.begin();
+    k_decide_small<M, UNIT><<<grid, 256, 0, st>>>(wk.queues, qs, a, qW, p);
+    CKL();
+    tm.end(KC_DEC_SMALL, e);
+    e = tm.begin();
+    k_decide_warp<32, 128, M, UNIT><<<grid, 32 * WarpSmem<32, 128, M>::WPB, WarpSmem<32, 128, M>::bytes, fk.branch(2)>>>(
+        qview(wk.queues, qs, BIN_WARP), BIN_WARP, a, qW, p);
+    CKL();
+    tm.end(KC_DEC_WARP, e);
+    if (maxdeg > g->bins[BIN_WARP]) {
+        e = tm.begin();
+        k_decide_warp<32, 512, M, UNIT><<<grid, 32 * WarpSmem<32, 512, M>::WPB, WarpSmem<32, 512, M>::bytes,
+                                          fk.branch(3)>>>(qview(wk.queues, qs, BIN_WARP2), BIN_WARP2, a, qW, p);
+        CKL();
+        tm.end(KC_DEC_WARP2, e);
+    }
 }
 
 template <int M, bool UNIT>
@@ -669,22 +729,11 @@ static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, typename M
         }
     }
     launch_hub<M, UNIT>(g, wk, a, qW, p, tm, wk.hub_on ? fk.branch(1) : st);
-    e = tm.begin();
-    k_decide_small<M, UNIT><<<grid, 256, 0, st>>>(wk.queues, qs, a, qW, p);
-    CKL();
-    tm.end(KC_DEC_SMALL, e);
-    e = tm.begin();
-    k_decide_warp<32, 128, M, UNIT><<<grid, 32 * WarpSmem<32, 128, M>::WPB, WarpSmem<32, 128, M>::bytes, fk.branch(2)>>>(
-        qview(wk.queues, qs, BIN_WARP), BIN_WARP, a, qW, p);
-    CKL();
-    tm.end(KC_DEC_WARP, e);
-    if (maxdeg > g->bins[BIN_WARP]) {
-        e = tm.begin();
-        k_decide_warp<32, 512, M, UNIT><<<grid, 32 * WarpSmem<32, 512, M>::WPB, WarpSmem<32, 512, M>::bytes,
-                                          fk.branch(3)>>>(qview(wk.queues, qs, BIN_WARP2), BIN_WARP2, a, qW, p);
-        CKL();
-        tm.end(KC_DEC_WARP2, e);
+    if constexpr (M == DM_W64 && UNIT) {   // short rows may use packed argmax keys (packed_ok)
+        if (g->opt_bin_packed && g->opt_force_wide != 1 && packed_ok(g, idbits, std::min<int64_t>(maxdeg, g->bins[BIN_WARP2])))
+            return launch_short_bins<DM_FAST, UNIT>(g, wk, a, qW, p, tm, maxdeg, fk);
     }
+    launch_short_bins<M, UNIT>(g, wk, a, qW, p, tm, maxdeg, fk);
 }
 
 // Per level, before its iterations: per-block spill tables of the block bin
@@ -781,11 +830,11 @@ static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, typename
     e = tm.begin();
     const bool ck = use_ckey(g, wk, G);
     k_dp_delta<UNIT><<<big, 256, 0, st>>>(wk.ctr, G.rp, G.col, G.w, wk.C, wk.mv_v, wk.mv_old, wk.mv_chunk, wk.stamp, wk.dp,
-                                          wk.carry, G.nnz, g->opt_delta, 1, 2, ck ? wk.ckey : nullptr,
+                                          wk.carry, G.nnz, g->opt_delta, 1, g->opt_delta_den, ck ? wk.ckey : nullptr,
                                           nullptr, ps.rmflag, n);
     CKL();
     k_dp_full<UNIT><<<grid_for((G.nnz + 127) / 128 * 32, 256, big), 256, 0, st>>>(wk.ctr, G.nnz, G.row, G.col, G.w,
-                                                                                 wk.C, wk.dp, g->opt_delta, 1, 2,
+                                                                                 wk.C, wk.dp, g->opt_delta, 1, g->opt_delta_den,
                                                                                  ck ? wk.ckey : nullptr, &wk.carry->ckey_valid,
                                                                                  ps.rmflag, wk.stamp, wk.carry);
     CKL();
@@ -1010,11 +1059,58 @@ static void agg_launch_small(gala_graph_s* g, const AggArgs& a, bool unit, int s
 // target rows: target of row v is newid[v]; entries become (newid[u], w) and
 // equal (target, key) pairs are summed.  Output CSR in pool memory with int64
 // weights and row ids; snew[c] (caller-allocated, k) receives the diagonal.
+// few communities: dense k x k accumulation (k_agg_dense_*); V = 32-bit iff W < 2^32
+template <typename V>
+static void aggregate_rows_dense(gala_graph_s* g, const DevCSR& cur, long long k, const int32_t* newid,
+                                 const int32_t* keymap, bool unit, DevCSR& nxt, int64_t& maxdeg, int64_t* snew) {
+    cudaStream_t st = g->stream;
+    const int big = g->num_sms * 8;
+    V* M = dalloc<V>((size_t)k * k, st);
+    CK(cudaMemsetAsync(M, 0, sizeof(V) * (size_t)k * k, st));
+    if (cur.nnz) {
+        const int grid = grid_for((cur.nnz + 127) / 128 * 32, 256, big);
+        if (unit) k_agg_dense_accum<true, V><<<grid, 256, 0, st>>>(cur.nnz, cur.row, cur.col, cur.w, newid, keymap, k, M);
+        else k_agg_dense_accum<false, V><<<grid, 256, 0, st>>>(cur.nnz, cur.row, cur.col, cur.w, newid, keymap, k, M);
+        CKL();
+    }
+    long long* dn = dalloc<long long>(k + 1, st);
+    k_agg_dense_count<V><<<grid_for(k * 32, 256, big), 256, 0, st>>>(k, M, dn, snew);
+    CKL();
+    nxt.n = k;
+    nxt.rp = dalloc<int64_t>(k + 1, st);
+    scan_excl(dn, reinterpret_cast<long long*>(nxt.rp), k, st);
+    ull* dev_max = dalloc<ull>(1, st);
+    CK(cudaMemsetAsync(dev_max, 0, sizeof(ull), st));
+    k_rowmax<<<grid_for(k, 256, big), 256, 0, st>>>(k, reinterpret_cast<long long*>(nxt.rp), dev_max);
+    CKL();
+    ull hm = 0;
+    CK(cudaMemcpyAsync(&nxt.nnz, nxt.rp + k, sizeof(long long), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(&hm, dev_max, sizeof(ull), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    maxdeg = (int64_t)hm;
+    nxt.col = dalloc<int32_t>(nxt.nnz, st);
+    nxt.w = dalloc<int64_t>(nxt.nnz, st);
+    nxt.row = dalloc<int32_t>(nxt.nnz, st);
+    k_agg_dense_emit<V><<<grid_for(k * 32, 256, big), 256, 0, st>>>(k, M, reinterpret_cast<long long*>(nxt.rp), nxt.col,
+                                                                    nxt.w, nxt.row);
+    CKL();
+    g->kc_bytes[KC_PHASE2] += (double)cur.nnz * (4 + 4 + (unit ? 0 : 8) + 4) + (double)k * k * sizeof(V) * 2 +
+                              (double)nxt.nnz * 16;
+    dfree(M, st); dfree(dn, st); dfree(dev_max, st);
+}
+
 static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, long long k, const int32_t* newid,
                            const int32_t* keymap, bool unit, DevCSR& nxt, int64_t& maxdeg, int64_t* snew) {
     cudaStream_t st = g->stream;
     const int big = g->num_sms * 8;
     VTimer vt(g);
+    // few communities, many entries: dense accumulation (the coarse graph has at most k^2 entries)
+    if (g->opt_agg_dense && k <= AGG_DENSE_K && (g->opt_agg_dense == 2 || cur.nnz >= 4 * k * k) && cur.row) {
+        if (g->W < ((int64_t)1 << 32)) aggregate_rows_dense<unsigned>(g, cur, k, newid, keymap, unit, nxt, maxdeg, snew);
+        else aggregate_rows_dense<ull>(g, cur, k, newid, keymap, unit, nxt, maxdeg, snew);
+        vt.lap("agg: dense");
+        return;
+    }
     long long* cnt = dalloc<long long>(k + 1, st);
     long long* ent = dalloc<long long>(k + 1, st);
     long long* eoff = dalloc<long long>(k + 1, st);
@@ -1033,13 +1129,19 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
     CK(cudaMemsetAsync(snew, 0, sizeof(int64_t) * k, st));
     CK(cudaMemsetAsync(dev_max, 0, sizeof(ull), st));
     CK(cudaMemsetAsync(nbig_dev, 0, sizeof(int) * 5, st));
-    k_comm_stats<<<grid_for(nrows, 256, big), 256, 0, st>>>((int)nrows, cur.rp, newid, ent);
+    const bool hist = k <= AGG_HIST_K;   // few communities: block-local histograms first
+    const unsigned htiles = (unsigned)std::max<long long>((nrows + AGG_HIST_T - 1) / AGG_HIST_T, 1);
+    if (hist) k_comm_stats_hist<<<htiles, 256, k * sizeof(unsigned), st>>>((int)nrows, k, cur.rp, newid, ent);
+    else k_comm_stats<<<grid_for(nrows, 256, big), 256, 0, st>>>((int)nrows, cur.rp, newid, ent);
     CKL();
     scan_excl(ent, eoff, k, st);
     // segment position of every row (cnt reused as the per-community cursor), then an
     // edge-parallel copy of the keys keymap[u] into the segments
     long long* vpos = dalloc<long long>(nrows, st);
-    k_vpos<<<grid_for(nrows, 256, big), 256, 0, st>>>((int)nrows, cur.rp, newid, eoff, cnt, vpos);
+    if (hist)
+        k_vpos_hist<<<htiles, 256, ((k * sizeof(unsigned) + 15) & ~(size_t)15) + k * sizeof(long long), st>>>(
+            (int)nrows, k, cur.rp, newid, eoff, cnt, vpos);
+    else k_vpos<<<grid_for(nrows, 256, big), 256, 0, st>>>((int)nrows, cur.rp, newid, eoff, cnt, vpos);
     CKL();
     if (unit)
         k_gather_flat<true><<<grid_for((cur.nnz + 127) / 128 * 32, 256, big), 256, 0, st>>>(
@@ -1303,15 +1405,10 @@ static void ensure_workspace(gala_graph_s* g) {
             wk.h_carry = static_cast<Carry*>(pin_get(sizeof(Carry)));
             if (!wk.h_log || !wk.h_carry) { set_err(GALA_E_NOMEM, "pinned host buffers"); throw GalaError{GALA_E_NOMEM}; }
             for (int i = 0; i < 5; ++i) CK(cudaEventCreate(&wk.ev[i]));
-            // dynamic shared memory opt-ins, once per workspace
+            // dynamic shared memory opt-ins (process-wide upper bounds, set once)
             int per_sm = 0;
             const int cap = g->hub_smem_slots;
-            CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, DM_FAST, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)block_smem_bytes<DM_FAST>(cap)));
-            CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, DM_FAST, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)block_smem_bytes<DM_FAST>(cap)));
-            CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, DM_W64, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)block_smem_bytes<DM_W64>(cap)));
-            CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, DM_W64, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)block_smem_bytes<DM_W64>(cap)));
-            CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, DM_W128, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)block_smem_bytes<DM_W128>(cap)));
-            CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, DM_W128, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)block_smem_bytes<DM_W128>(cap)));
+            block_attrs_once();
             // resident blocks per SM of each mode's block kernel (the grid of a launch; spill
             // tables are sized for the largest)
             auto occ = [&](const void* f, size_t sm) {
@@ -1328,9 +1425,6 @@ static void ensure_workspace(gala_graph_s* g) {
             per_sm = std::max(std::max(wk.gblocks_m[0], wk.gblocks_m[1]), wk.gblocks_m[2]) / g->num_sms;
             set_warp_smem<32, 128, DM_FAST>(); set_warp_smem<32, 128, DM_W64>(); set_warp_smem<32, 128, DM_W128>();
             set_warp_smem<32, 512, DM_FAST>(); set_warp_smem<32, 512, DM_W64>(); set_warp_smem<32, 512, DM_W128>();
-            block_setup<DM_FAST, true>(g); block_setup<DM_FAST, false>(g);
-            block_setup<DM_W64, true>(g); block_setup<DM_W64, false>(g);
-            block_setup<DM_W128, true>(g); block_setup<DM_W128, false>(g);
             wk.gblocks = g->num_sms * std::max(per_sm, 1);
             wk.gcap = 0;   // spill tables sized on demand (coarse levels can have larger rows than level 0)
             wk.smem_cap = cap;
@@ -2010,13 +2104,13 @@ static void dist_iteration_fab(gala_graph_s* g, Work& wk, const DevCSR& G, const
     tm.end(KC_APPLY, e);
     e = tm.begin();
     k_fab_dp_delta<UNIT><<<big, 256, 0, st>>>(wk.ctr, G.rp, G.col, G.w, L.mrp, L.mcol, L.mw, wk.C, L.it_v, L.it_old,
-                                              L.it_chunk, wk.stamp, wk.dp, wk.carry, G.nnz, g->opt_delta, lv0, lv1);
+                                              L.it_chunk, wk.stamp, wk.dp, wk.carry, G.nnz, g->opt_delta, lv0, lv1, g->opt_delta_den);
     CKL();
-    k_dp_zero<<<big, 256, 0, st>>>(wk.ctr, (int)lv0, (int)lv1, wk.dp, G.nnz, g->opt_delta, 1, 2);
+    k_dp_zero<<<big, 256, 0, st>>>(wk.ctr, (int)lv0, (int)lv1, wk.dp, G.nnz, g->opt_delta, 1, g->opt_delta_den);
     CKL();
     if (G.nnz) {
         k_dp_full<UNIT><<<grid_for((G.nnz + 127) / 128 * 32, 256, big), 256, 0, st>>>(
-            wk.ctr, G.nnz, G.row, G.col, G.w, wk.C, wk.dp, g->opt_delta, 1, 2, nullptr, nullptr, nullptr, nullptr,
+            wk.ctr, G.nnz, G.row, G.col, G.w, wk.C, wk.dp, g->opt_delta, 1, g->opt_delta_den, nullptr, nullptr, nullptr, nullptr,
             wk.carry);
         CKL();
     }
@@ -2689,9 +2783,13 @@ gala_status gala_set_option(gala_graph g, const char* key, int64_t value) {
     else if (k == "check") g->opt_check = value != 0;
     else if (k == "timing") g->opt_timing = value != 0;
     else if (k == "max_iters") { if (value < 0) return set_err(GALA_E_INVALID, "max_iters < 0"); g->opt_max_iters = (int)value; }
+    else if (k == "delta_den") { if (value < 1 || value > 64) return set_err(GALA_E_INVALID, "delta_den in 1..64"); g->opt_delta_den = (int)value; }
     else if (k == "delta_update") { if (value < 0 || value > 2) return set_err(GALA_E_INVALID, "delta_update in 0..2"); g->opt_delta = (int)value; }
     else if (k == "force_i128") g->opt_force_i128 = value != 0;
-    else if (k == "force_wide") g->opt_force_wide = value != 0;
+    else if (k == "force_wide") {   // 1: DM_W64 everywhere; 2: DM_W64 levels, packed short-row bins
+        if (value < 0 || value > 2) return set_err(GALA_E_INVALID, "force_wide in 0..2");
+        g->opt_force_wide = (int)value;
+    }
     else if (k == "singleton") g->opt_singleton = value != 0;
     else if (k == "agg_big_chunk") g->opt_agg_big_chunk = value != 0;
     else if (k == "agg_chunk") {   // test hook: entries per big-community chunk (1..AGG_CH)
@@ -2699,6 +2797,11 @@ gala_status gala_set_option(gala_graph g, const char* key, int64_t value) {
         g->opt_agg_chunk = (int)value;
     } else if (k == "agg_bound") {   // phase 2: size big-community tables from chunk distinct counts
         g->opt_agg_bound = value != 0;
+    } else if (k == "bin_packed") {   // DM_W64 unit levels: packed argmax keys for rows <= bin_warp512
+        g->opt_bin_packed = value != 0;
+    } else if (k == "agg_dense") {   // phase 2: dense k x k accumulation (0 never, 1 auto, 2 whenever k fits)
+        if (value < 0 || value > 2) return set_err(GALA_E_INVALID, "agg_dense in 0..2");
+        g->opt_agg_dense = (int)value;
     } else if (k == "block_split") {   // block bin: rows <= split in small blocks (0: one class)
         if (value < 0 || value > (1 << 20)) return set_err(GALA_E_INVALID, "block_split must be in [0, 2^20]");
         g->opt_block_split = (int)value;

@@ -163,6 +163,58 @@ __global__ void k_vpos(int n, const int64_t* __restrict__ rp, const int32_t* __r
     }
 }
 
+// Few communities (k <= AGG_HIST_K): the per-community sums above hit the same few counters
+// from every thread (thousands of same-address atomics each).  These variants first count in a
+// block-local shared histogram over a contiguous tile of AGG_HIST_T vertices, then add each
+// nonzero bin once per block; k_vpos_hist also hands every vertex its offset inside the block's
+// share of its community segment.
+#define AGG_HIST_K 4096
+#define AGG_HIST_T 2048
+__global__ void __launch_bounds__(256) k_comm_stats_hist(int n, long long k, const int64_t* __restrict__ rp,
+                                                         const int32_t* __restrict__ newid, long long* __restrict__ ent) {
+    extern __shared__ unsigned hist[];
+    for (long long c = threadIdx.x; c < k; c += 256) hist[c] = 0;
+    __syncthreads();
+    const long long v0 = (long long)blockIdx.x * AGG_HIST_T;
+    for (long long v = v0 + threadIdx.x; v < min((long long)n, v0 + AGG_HIST_T); v += 256) {
+        const long long dg = rp[v + 1] - rp[v];
+        if (dg) atomicAdd(&hist[newid[v]], (unsigned)dg);
+    }
+    __syncthreads();
+    for (long long c = threadIdx.x; c < k; c += 256)
+        if (hist[c]) atomicAdd(reinterpret_cast<ull*>(&ent[c]), (ull)hist[c]);
+}
+__global__ void __launch_bounds__(256) k_vpos_hist(int n, long long k, const int64_t* __restrict__ rp,
+                                                   const int32_t* __restrict__ newid, const long long* __restrict__ eoff,
+                                                   long long* __restrict__ ecur, long long* __restrict__ vpos) {
+    extern __shared__ unsigned char hraw[];
+    unsigned* hist = reinterpret_cast<unsigned*>(hraw);
+    long long* base = reinterpret_cast<long long*>(hraw + ((k * sizeof(unsigned) + 15) & ~(long long)15));
+    constexpr int PER = AGG_HIST_T / 256;
+    for (long long c = threadIdx.x; c < k; c += 256) hist[c] = 0;
+    __syncthreads();
+    const long long v0 = (long long)blockIdx.x * AGG_HIST_T;
+    unsigned loc[PER];
+    int cc[PER];
+    long long dgs[PER];
+#pragma unroll
+    for (int t = 0; t < PER; ++t) {
+        const long long v = v0 + threadIdx.x + 256 * t;
+        dgs[t] = v < n ? rp[v + 1] - rp[v] : 0;
+        cc[t] = v < n ? newid[v] : 0;
+        loc[t] = dgs[t] ? atomicAdd(&hist[cc[t]], (unsigned)dgs[t]) : 0;
+    }
+    __syncthreads();
+    for (long long c = threadIdx.x; c < k; c += 256)
+        base[c] = hist[c] ? (long long)atomicAdd(reinterpret_cast<ull*>(&ecur[c]), (ull)hist[c]) : 0;
+    __syncthreads();
+#pragma unroll
+    for (int t = 0; t < PER; ++t) {
+        const long long v = v0 + threadIdx.x + 256 * t;
+        if (v < n) vpos[v] = dgs[t] ? eoff[cc[t]] + base[cc[t]] + loc[t] : 0;
+    }
+}
+
 // edge-parallel: entry e of row r goes to vpos[r] + (e - rp[r]) with key newid[col[e]];
 // 4 entries per lane in flight, coalesced row/col streams
 template <bool UNIT>
@@ -197,6 +249,88 @@ __global__ void __launch_bounds__(256) k_gather_flat(long long nnz, const int32_
                 tkey[dst[t]] = kk[t];
                 if (!UNIT) tval[dst[t]] = w[e];
             }
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// a9, few communities (k <= AGG_DENSE_K): the coarse graph has at most k^2 entries, so it is
+// accumulated straight into a dense k x k matrix M (L2-resident: 1202^2 x 4 B = 5.8 MB for the
+// Orkut-shaped level 0) -- no community-major segments, no hash tables.  Edge-parallel over the
+// CSR (4 entries per lane in flight); the entries of a 32-entry chunk with the same (c1, c2) are
+// combined with __match_any_sync first, so the diagonal (most entries of a good partition) sees
+// one atomic per chunk.  M[c][c] is D_C(c) (every entry inside c, reading c10).  Rows are then
+// counted, scanned and emitted in ascending column order.
+// ---------------------------------------------------------------------------
+#define AGG_DENSE_K 4096
+template <bool UNIT, typename V>
+__global__ void __launch_bounds__(256) k_agg_dense_accum(long long nnz, const int32_t* __restrict__ row,
+                                                         const int32_t* __restrict__ col, const int64_t* __restrict__ w,
+                                                         const int32_t* __restrict__ newid,
+                                                         const int32_t* __restrict__ keymap, long long k,
+                                                         V* __restrict__ M) {
+    __shared__ V s_scr[8][32];   // per-warp group sums (weighted levels)
+    const int lane = lane_id();
+    const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+    for (long long base = (((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * 128; base < nnz;
+         base += nw * 128) {
+        int r[4], u[4];
+        V wt[4];
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+            const long long e = base + lane + 32 * t;
+            r[t] = e < nnz ? row[e] : -1;
+            u[t] = e < nnz ? col[e] : 0;
+            wt[t] = (e < nnz && !UNIT) ? (V)w[e] : (V)1;
+        }
+        long long key[4];
+#pragma unroll
+        for (int t = 0; t < 4; ++t) key[t] = r[t] >= 0 ? (long long)newid[r[t]] * k + keymap[u[t]] : -1 - lane;
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+            const unsigned peers = __match_any_sync(FULLMASK, key[t]);
+            const V sum = UNIT ? (V)__popc(peers) : group_sum(peers, r[t] >= 0 ? wt[t] : (V)0, s_scr[threadIdx.x >> 5]);
+            if (r[t] >= 0 && lane == __ffs(peers) - 1) atomicAdd(&M[key[t]], sum);
+        }
+    }
+}
+
+// warp per coarse row: distinct entries -> dn[c], diagonal -> snew[c]
+template <typename V>
+__global__ void k_agg_dense_count(long long k, const V* __restrict__ M, long long* __restrict__ dn,
+                                  int64_t* __restrict__ snew) {
+    const int lane = lane_id();
+    const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+    for (long long c = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < k; c += nw) {
+        const V* rowp = M + c * k;
+        long long cnt = 0;
+        for (long long j = lane; j < k; j += 32) cnt += rowp[j] != 0;
+        cnt = warp_sum_ll(cnt);
+        if (lane == 0) { dn[c] = cnt; snew[c] = (int64_t)rowp[c]; }
+    }
+}
+
+// warp per coarse row: nonzeros in ascending column order -> CSR (col, w, row); M cleared
+template <typename V>
+__global__ void k_agg_dense_emit(long long k, V* __restrict__ M, const long long* __restrict__ rp,
+                                 int32_t* __restrict__ ocol, int64_t* __restrict__ ow, int32_t* __restrict__ orow) {
+    const int lane = lane_id();
+    const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+    for (long long c = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < k; c += nw) {
+        V* rowp = M + c * k;
+        long long o = rp[c];
+        for (long long j0 = 0; j0 < k; j0 += 32) {
+            const long long j = j0 + lane;
+            const V x = j < k ? rowp[j] : (V)0;
+            const unsigned nz = __ballot_sync(FULLMASK, x != 0);
+            if (x != 0) {
+                const long long at = o + __popc(nz & lanemask_lt());
+                ocol[at] = (int32_t)j;
+                ow[at] = (int64_t)x;
+                orow[at] = (int32_t)c;
+                rowp[j] = 0;
+            }
+            o += __popc(nz);
         }
     }
 }

@@ -12,6 +12,7 @@ import pytest
 import graphgen as gg
 import oracle
 import paper_conf_ppopp_wangllwm00z25_b200 as gala
+import quality
 
 pytestmark = pytest.mark.gpu
 
@@ -131,6 +132,10 @@ def test_pruning_strategy_weighted_and_graph_mode(strategy):
     dict(agg_scap=512, agg_chunk=64, agg_bound=0),                           # phase 2: one-pass big path
     dict(agg_scap=512, agg_big_chunk=0),                                     # phase 2: per-community block split
     dict(agg_big_ent=64, agg_chunk=32),                                      # phase 2: entry-count big path
+    dict(agg_dense=0),                                                       # phase 2: never the dense k x k path
+    dict(force_wide=2),                                                      # W64 level, packed short-row bins
+    dict(force_wide=2, bin_packed=0),
+    dict(delta_den=8),                                                       # d' delta rule threshold
     dict(block_split=0),                                                     # block bin as one class
     dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=0, bin_warp512=0, block_split=64),
     dict(bin_sub32=16, bin_warp=16, bin_warp512=32, block_split=100, force_i128=1),
@@ -140,8 +145,8 @@ def test_dispatch_independence(opts):
     assert_parity(gg.make("rmat_small"), **opts)
 
 
-@pytest.mark.parametrize("opts", [dict(force_wide=1), dict(force_i128=1), hub(16), dict(hub(16), force_i128=1),
-                                  dict(agg_scap=512, agg_chunk=16)])
+@pytest.mark.parametrize("opts", [dict(force_wide=1), dict(force_wide=2), dict(force_i128=1), hub(16),
+                                  dict(hub(16), force_i128=1), dict(agg_scap=512, agg_chunk=16), dict(agg_dense=0)])
 def test_weighted_modes_parity(opts):
     """Weighted random graphs through every gain-arithmetic mode (DM_W64 / DM_W128)."""
     for seed in range(4):
@@ -246,6 +251,26 @@ def test_full_size_parity_skewed(name):
 
 
 @pytest.mark.slow
+def test_friendster_shape_bounded_parity():
+    """BASELINE configs[4] shape on one GPU at 1/4 of its vertices (16.4M vertices, 786M entries,
+    C + Sigma_tot = 197 MB beyond the 126 MB L2), bounded so the driver's GPU run can afford the
+    oracle: level 0, first three iterations (max_iters, honoured identically by both sides).
+    Labels at every iteration (stepwise launch), then the bench's launch configuration (conditional
+    CUDA graph): N / moved / active / pruned per iteration and the final labels."""
+    g = gg.make("friendster_q")
+    o = oracle.louvain(g, prune=1, trace=2, max_levels=1, max_iters=3)
+    assert o.status == 0 and len(o.records) == 3
+    for trace in (2, 1):
+        r = run_gpu(g, max_levels=1, trace=trace, prune=1, max_iters=3)
+        assert len(r["trace"]) == 3
+        for x, y in zip(o.records, r["trace"]):
+            if trace == 2:
+                assert np.array_equal(x.labels, y["labels"]), f"labels differ at iter {x.iter}"
+            assert (x.N, x.n_moved, x.n_active, x.n_pruned) == (y["N"], y["n_moved"], y["n_active"], y["n_pruned"])
+        assert np.array_equal(o.labels, r["labels"]) and o.N == r["N"]
+
+
+@pytest.mark.slow
 @pytest.mark.skipif(not os.environ.get("GALA_XL"), reason="~5 min (generator + oracle on 786M entries); GALA_XL=1")
 def test_friendster_shape_full_parity():
     """BASELINE configs[4] shape on one GPU at 1/4 of its vertices (16.4M vertices, 786M entries,
@@ -263,9 +288,9 @@ def test_nmi_vs_planted_partition():
     with gala.Graph.from_graph(g) as h:
         h.run()
         lab = h.communities()
-    got = gala.nmi_device(lab, g.truth)
+    got = quality.nmi_device(lab, g.truth)
     assert got == pytest.approx(nmi(lab, g.truth), abs=1e-9)
-    assert gala.nmi_device(g.truth, g.truth) == pytest.approx(1.0, abs=1e-12)
+    assert quality.nmi_device(g.truth, g.truth) == pytest.approx(1.0, abs=1e-12)
     assert 0.0 <= got <= 1.0 + 1e-12
 
 
@@ -330,3 +355,19 @@ def test_handle_cycles_reuse_pinned_and_pool():
         r = run_gpu(g, trace=1, log_cap=cap)
         assert np.array_equal(r["labels"], o.labels)
         assert r["N"] == o.N and len(r["trace"]) == len(o.records)
+
+
+@pytest.mark.parametrize("name", ["lfr_small", "lfr_mid", "rmat_small"])
+@pytest.mark.parametrize("dense", [0, 1, 2])
+def test_dense_coarsening_parity(name, dense):
+    """Phase 2 with few communities: the dense k x k accumulation (auto: k <= 4096 and
+    nnz >= 4 k^2; 2: whenever k <= 4096) and the segmented hash path give the same coarse
+    graphs (per-level labels and N equal the oracle's)."""
+    o, r = assert_parity(gg.make(name), agg_dense=dense)
+    assert len(r["stats"]["levels"]) >= 2
+
+
+def test_dense_coarsening_weighted():
+    for seed in range(3):
+        g = gg.random_graph(300, 2000, seed=2100 + seed, max_w=7, self_loops=5)
+        assert_parity(g, gamma=[1.0, 0.5, 2.0][seed], agg_dense=2)
