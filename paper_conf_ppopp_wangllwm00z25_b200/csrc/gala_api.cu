@@ -115,6 +115,7 @@ struct gala_graph_s {
     int opt_block_split = 1024;
     int opt_agg_bound = 1;
     int opt_agg_dense = 1;
+    int opt_agg_spill = 1;   // phase 2: class D (one block, shared H0 spilling to global H1) for short segments
     int opt_bin_packed = 1;  // DM_W64 levels: packed argmax keys for the short-row bins where they fit   // phase 2: dense k x k accumulation when k <= AGG_DENSE_K and nnz >= 4 k^2
     bool rows_distinct0 = false;   // level-0 rows strictly increasing (no duplicate entries)
     bool self0 = true;             // level 0 has a self-loop (s0 not all zero)
@@ -597,29 +598,33 @@ static void launch_single(gala_graph_s* g, Work& wk, const DecideArgs& a, typena
 }
 
 // Dynamic shared-memory limits of the block kernels.  The limit is a per-function, process-wide
-// attribute, so it is set ONCE (under a lock, before any capture) to the largest arena any handle's
-// options allow: 16384 slots (hub_smem_slots <= 16384; the short-row class uses < hub_smem_slots).
-// It is only an upper bound -- occupancy and the launch follow the dynamic shared memory each launch
-// requests -- so handles with different options (loopback ranks are threads) never race on it.
+// attribute: it is only ever RAISED (under a lock, before any capture) to the largest arena a handle
+// needs, so handles with different options (loopback ranks are threads) never see a limit below
+// their own arena.  It is not simply set to the largest arena any option allows: a larger limit
+// measurably slows the default configuration (orkut decide_block 8.6 -> 11.3 ms with a 16384-slot
+// limit; the shared-memory carveout follows the limit, leaving less L1 for the gathers).
 template <int M, bool UNIT>
-static void block_attr_mode() {
-    const int mx = (int)block_smem_bytes<M>(16384);
+static void block_attr_mode(int slots) {
+    const int mx = (int)block_smem_bytes<M>(slots);
     CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
     CK(cudaFuncSetAttribute(k_decide_block<BLOCK_BT, BLOCK_E, M, UNIT, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
     CK(cudaFuncSetAttribute(k_decide_block<BLOCK_LO_BT, BLOCK_LO_E, M, UNIT, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
     CK(cudaFuncSetAttribute(k_decide_block<BLOCK_LO_BT, BLOCK_LO_E, M, UNIT, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
 }
-static void block_attrs_once() {
+static void block_attrs_ensure(int slots) {
     static std::mutex mu;
-    static std::map<int, bool> done;   // per device
+    static std::map<int, int> cur;   // per device: slots the limits allow
     std::lock_guard<std::mutex> lk(mu);
     const int dev = current_device();
-    if (done[dev]) return;
-    block_attr_mode<DM_FAST, true>(); block_attr_mode<DM_FAST, false>();
-    block_attr_mode<DM_W64, true>(); block_attr_mode<DM_W64, false>();
-    block_attr_mode<DM_W128, true>(); block_attr_mode<DM_W128, false>();
-    done[dev] = true;
+    if (cur[dev] >= slots) return;
+    block_attr_mode<DM_FAST, true>(slots); block_attr_mode<DM_FAST, false>(slots);
+    block_attr_mode<DM_W64, true>(slots); block_attr_mode<DM_W64, false>(slots);
+    block_attr_mode<DM_W128, true>(slots); block_attr_mode<DM_W128, false>(slots);
+    cur[dev] = slots;
 }
+// the largest block arena this handle launches (the short-row class runs only when its arena is
+// smaller than hub_smem_slots)
+static int block_arena_slots(const gala_graph_s* g) { return g->hub_smem_slots; }
 
 // grid of the short-row block kernel (rows <= opt_block_split): resident blocks per SM for its
 // arena, computed once per (mode, unit, arena, class)
@@ -645,21 +650,23 @@ static int block_lo_grid(gala_graph_s* g, int cap, bool all) {
 // while a level's iteration body is being captured into a CUDA graph
 template <int M, bool UNIT>
 static void block_setup(gala_graph_s* g) {
-    block_attrs_once();
+    block_attrs_ensure(block_arena_slots(g));
     int cap1 = 64;
     while (cap1 < 2 * std::max(g->opt_block_split, 1)) cap1 <<= 1;
     if (cap1 < g->hub_smem_slots) (void)block_lo_grid<M, UNIT>(g, cap1, false);   // the only case it launches
 }
 
-// the sub-warp and warp bins (rows <= bins[BIN_WARP2])
-template <int M, bool UNIT>
+// the sub-warp and warp bins (rows <= bins[BIN_WARP2]); MS: mode of the sub-warp kernel (packed keys
+// pay there: A/B on orkut decide_small 2.37 -> 2.16 ms), M: the warp kernels' (the packed variant of
+// the 128-row warp kernel spills; measured 4.98 -> 5.34 ms)
+template <int M, bool UNIT, int MS = M>
 static void launch_short_bins(gala_graph_s* g, Work& wk, const DecideArgs& a, typename ModeT<M>::ST qW,
                               typename ModeT<M>::ST p, Timer& tm, int64_t maxdeg, Fork& fk) {
     const long long qs = wk.qcap;
     const int grid = g->num_sms * 8;
     cudaStream_t st = g->stream;
     cudaEvent_t e = tm.begin();
-    k_decide_small<M, UNIT><<<grid, 256, 0, st>>>(wk.queues, qs, a, qW, p);
+    k_decide_small<MS, UNIT><<<grid, 256, 0, st>>>(wk.queues, qs, a, qW, p);
     CKL();
     tm.end(KC_DEC_SMALL, e);
     e = tm.begin();
@@ -688,7 +695,6 @@ static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, typename M
     a.idmask = (1LL << idbits) - 1;
     if (single) return launch_single<M, UNIT>(g, wk, a, qW, p, tm, maxdeg);
     const long long qs = wk.qcap;
-    const int grid = g->num_sms * 8;
     cudaStream_t st = g->stream;
     Fork fk(g);
     cudaEvent_t e;
@@ -730,8 +736,8 @@ static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, typename M
     }
     launch_hub<M, UNIT>(g, wk, a, qW, p, tm, wk.hub_on ? fk.branch(1) : st);
     if constexpr (M == DM_W64 && UNIT) {   // short rows may use packed argmax keys (packed_ok)
-        if (g->opt_bin_packed && g->opt_force_wide != 1 && packed_ok(g, idbits, std::min<int64_t>(maxdeg, g->bins[BIN_WARP2])))
-            return launch_short_bins<DM_FAST, UNIT>(g, wk, a, qW, p, tm, maxdeg, fk);
+        if (g->opt_bin_packed && g->opt_force_wide != 1 && packed_ok(g, idbits, std::min<int64_t>(maxdeg, g->bins[BIN_S32])))
+            return launch_short_bins<M, UNIT, DM_FAST>(g, wk, a, qW, p, tm, maxdeg, fk);
     }
     launch_short_bins<M, UNIT>(g, wk, a, qW, p, tm, maxdeg, fk);
 }
@@ -1121,14 +1127,14 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
     int32_t* bigc = dalloc<int32_t>(k, st);
     long long* bigcap = dalloc<long long>(k + 1, st);
     int32_t* wlist = dalloc<int32_t>(k, st);
-    int32_t* blist = dalloc<int32_t>(3 * k, st);   // block-path classes A, B, C
-    int* nbig_dev = dalloc<int>(5, st);   // big, warp, block A / B / C list lengths
+    int32_t* blist = dalloc<int32_t>(4 * k, st);   // block-path classes A, B, C, D (spilling)
+    int* nbig_dev = dalloc<int>(6, st);   // big, warp, block A / B / C / D list lengths
     CK(cudaMemsetAsync(cnt, 0, sizeof(long long) * (k + 1), st));
     CK(cudaMemsetAsync(ent, 0, sizeof(long long) * (k + 1), st));
     CK(cudaMemsetAsync(dn, 0, sizeof(long long) * (k + 1), st));
     CK(cudaMemsetAsync(snew, 0, sizeof(int64_t) * k, st));
     CK(cudaMemsetAsync(dev_max, 0, sizeof(ull), st));
-    CK(cudaMemsetAsync(nbig_dev, 0, sizeof(int) * 5, st));
+    CK(cudaMemsetAsync(nbig_dev, 0, sizeof(int) * 6, st));
     const bool hist = k <= AGG_HIST_K;   // few communities: block-local histograms first
     const unsigned htiles = (unsigned)std::max<long long>((nrows + AGG_HIST_T - 1) / AGG_HIST_T, 1);
     if (hist) k_comm_stats_hist<<<htiles, 256, k * sizeof(unsigned), st>>>((int)nrows, k, cur.rp, newid, ent);
@@ -1155,8 +1161,9 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
     // shared-memory capacity of the block path: up to 8192 slots (14 B each)
     int scap = 512;
     while (scap < g->opt_agg_scap && scap < 2 * k) scap <<= 1;
+    const long long spill_ent = g->opt_agg_spill ? g->opt_agg_big_ent : 0;
     k_agg_classify<<<grid_for(k, 256, big), 256, 0, st>>>(k, ent, scap, dn, wlist, nbig_dev + 1, blist, nbig_dev + 2,
-                                                         bigc, bigcap, nbig_dev, k, g->opt_agg_big_ent);
+                                                         bigc, bigcap, nbig_dev, k, g->opt_agg_big_ent, spill_ent);
     CKL();
     AggArgs a;
     a.k = k; a.ent = ent; a.eoff = eoff; a.tkey = tkey; a.tval = tval; a.dn = dn; a.snew = snew;
@@ -1164,9 +1171,34 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
     if (v32) agg_launch_small<unsigned>(g, a, unit, scap, k, wlist, nbig_dev + 1, blist, nbig_dev + 2);
     else agg_launch_small<ull>(g, a, unit, scap, k, wlist, nbig_dev + 1, blist, nbig_dev + 2);
     vt.lap("agg: warp+block");
-    int nbig = 0;
-    CK(cudaMemcpyAsync(&nbig, nbig_dev, sizeof(int), cudaMemcpyDeviceToHost, st));
+    int hcnt[6] = {0, 0, 0, 0, 0, 0};
+    CK(cudaMemcpyAsync(hcnt, nbig_dev, sizeof(hcnt), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
+    const int nbig = hcnt[0];
+    if (hcnt[5] > 0) {   // class D: shared H0 spilling to per-block global H1 tables
+        long long gcap = 64;
+        while (gcap < 2 * std::min<long long>(spill_ent, k)) gcap <<= 1;
+        const size_t sm = (size_t)scap * (v32 ? sizeof(unsigned) : sizeof(ull)) + (size_t)scap * 2 * sizeof(int);
+        auto kf = unit ? (v32 ? (void*)k_agg_block_h<true, unsigned> : (void*)k_agg_block_h<true, ull>)
+                       : (v32 ? (void*)k_agg_block_h<false, unsigned> : (void*)k_agg_block_h<false, ull>);
+        CK(cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+        int per = 0;
+        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, kf, 512, sm));
+        const int gd = (int)std::min<long long>((long long)g->num_sms * std::max(per, 1), hcnt[5]);
+        int* hk = dalloc<int>((size_t)gd * gcap, st);
+        ull* hv = dalloc<ull>((size_t)gd * gcap, st);
+        int* hl = dalloc<int>((size_t)gd * gcap, st);
+        CK(cudaMemsetAsync(hk, 0xff, sizeof(int) * (size_t)gd * gcap, st));
+        CK(cudaMemsetAsync(hv, 0, sizeof(ull) * (size_t)gd * gcap, st));
+        const int32_t* bld = blist + 3 * k;
+        if (unit && v32) k_agg_block_h<true, unsigned><<<gd, 512, sm, st>>>(a, scap, bld, nbig_dev + 5, hk, hv, hl, gcap);
+        else if (unit) k_agg_block_h<true, ull><<<gd, 512, sm, st>>>(a, scap, bld, nbig_dev + 5, hk, hv, hl, gcap);
+        else if (v32) k_agg_block_h<false, unsigned><<<gd, 512, sm, st>>>(a, scap, bld, nbig_dev + 5, hk, hv, hl, gcap);
+        else k_agg_block_h<false, ull><<<gd, 512, sm, st>>>(a, scap, bld, nbig_dev + 5, hk, hv, hl, gcap);
+        CKL();
+        dfree(hk, st); dfree(hv, st); dfree(hl, st);
+        vt.lap("agg: spilling block");
+    }
     if (nbig > 0 && g->opt_agg_big_chunk && g->opt_agg_bound) {
         // two-pass: chunk combine in place -> tables sized from the chunks' distinct counts
         const int ch = g->opt_agg_chunk;
@@ -1408,7 +1440,7 @@ static void ensure_workspace(gala_graph_s* g) {
             // dynamic shared memory opt-ins (process-wide upper bounds, set once)
             int per_sm = 0;
             const int cap = g->hub_smem_slots;
-            block_attrs_once();
+            block_attrs_ensure(block_arena_slots(g));
             // resident blocks per SM of each mode's block kernel (the grid of a launch; spill
             // tables are sized for the largest)
             auto occ = [&](const void* f, size_t sm) {
@@ -2799,6 +2831,8 @@ gala_status gala_set_option(gala_graph g, const char* key, int64_t value) {
         g->opt_agg_bound = value != 0;
     } else if (k == "bin_packed") {   // DM_W64 unit levels: packed argmax keys for rows <= bin_warp512
         g->opt_bin_packed = value != 0;
+    } else if (k == "agg_spill") {   // phase 2: spilling block class for segments <= agg_big_ent entries
+        g->opt_agg_spill = value != 0;
     } else if (k == "agg_dense") {   // phase 2: dense k x k accumulation (0 never, 1 auto, 2 whenever k fits)
         if (value < 0 || value > 2) return set_err(GALA_E_INVALID, "agg_dense in 0..2");
         g->opt_agg_dense = (int)value;

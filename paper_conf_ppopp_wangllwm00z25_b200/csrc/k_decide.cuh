@@ -527,8 +527,20 @@ __device__ __forceinline__ long long block_next_item(QView queue, long long coun
     }
 }
 
+#ifndef GALA_BLOCK_MINB
+#define GALA_BLOCK_MINB 0      // >0: min resident 512-thread blocks per SM of the long-row class (register cap);
+                               // 0: no bound (an explicit 1 lets ptxas take 75-100 registers and halves occupancy)
+#endif
+#ifndef GALA_BLOCK_PIPE
+#define GALA_BLOCK_PIPE 1      // the next round's row entries are loaded while the current round is inserted
+#endif
+#if GALA_BLOCK_MINB > 0
+#define BLOCK_LB(BT) __launch_bounds__(BT, BT >= 512 ? GALA_BLOCK_MINB : 1)
+#else
+#define BLOCK_LB(BT) __launch_bounds__(BT)
+#endif
 template <int BT, int E, int M, bool UNIT, int CLS = 0>
-__global__ void __launch_bounds__(BT) k_decide_block(QView queue, int bin, DecideArgs a,
+__global__ void BLOCK_LB(BT) k_decide_block(QView queue, int bin, DecideArgs a,
                                                      typename ModeT<M>::ST qW, typename ModeT<M>::ST p, int smem_cap,
                                                      int* __restrict__ gkeys_all, ull* __restrict__ gvals_all,
                                                      int* __restrict__ glist_all, long long gcap, int split = 0) {
@@ -580,15 +592,34 @@ __global__ void __launch_bounds__(BT) k_decide_block(QView queue, int bin, Decid
         long long gc = deg > 32 ? (1LL << (64 - __clzll(2LL * deg - 1))) : 64;   // H1 slots
         if (gc > gcap) gc = gcap;
         const unsigned gmask = (unsigned)gc - 1;
-        for (int r0 = 0; r0 < deg; r0 += BT * E) {          // block-uniform rounds
-            int uu[E];
-            VT ww[E];
-            int cc[E];
+        int uu[E];
+        VT ww[E];
 #pragma unroll
-            for (int k = 0; k < E; ++k) {
-                int j = r0 + threadIdx.x + k * BT;
-                uu[k] = j < deg ? (a.ckey ? a.ckey[beg + j] : a.col[beg + j]) : -1;
-                ww[k] = (j < deg && !UNIT) ? (VT)a.w[beg + j] : (VT)1;
+        for (int k = 0; k < E; ++k) {
+            int j = threadIdx.x + k * BT;
+            uu[k] = j < deg ? (a.ckey ? a.ckey[beg + j] : a.col[beg + j]) : -1;
+            ww[k] = (j < deg && !UNIT) ? (VT)a.w[beg + j] : (VT)1;
+        }
+        for (int r0 = 0; r0 < deg; r0 += BT * E) {          // block-uniform rounds
+            int cc[E];
+            if (r0 > 0 && !GALA_BLOCK_PIPE) {
+#pragma unroll
+                for (int k = 0; k < E; ++k) {
+                    int j = r0 + threadIdx.x + k * BT;
+                    uu[k] = j < deg ? (a.ckey ? a.ckey[beg + j] : a.col[beg + j]) : -1;
+                    ww[k] = (j < deg && !UNIT) ? (VT)a.w[beg + j] : (VT)1;
+                }
+            }
+            // next round's entries in flight during this round's gathers and inserts
+            int nu[E];
+            VT nw[E];
+            if (GALA_BLOCK_PIPE) {
+#pragma unroll
+                for (int k = 0; k < E; ++k) {
+                    int j = r0 + BT * E + threadIdx.x + k * BT;
+                    nu[k] = j < deg ? (a.ckey ? a.ckey[beg + j] : a.col[beg + j]) : -1;
+                    nw[k] = (j < deg && !UNIT) ? (VT)a.w[beg + j] : (VT)1;
+                }
             }
             if (a.ckey) {
 #pragma unroll
@@ -615,6 +646,10 @@ __global__ void __launch_bounds__(BT) k_decide_block(QView queue, int bin, Decid
                                                        (int)gc, &gfresh);
                 }
                 if (__any_sync(FULLMASK, gfresh)) append_fresh<int>(gfresh, gslot, FULLMASK, &s_gcnt, glist);
+            }
+            if (GALA_BLOCK_PIPE) {
+#pragma unroll
+                for (int k = 0; k < E; ++k) { uu[k] = nu[k]; ww[k] = nw[k]; }
             }
         }
         __syncthreads();

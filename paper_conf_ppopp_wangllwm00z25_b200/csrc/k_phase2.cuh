@@ -382,6 +382,35 @@ __device__ __forceinline__ int agg_insert(int key, VT wt, int* keys, VT* vals, u
     }
 }
 
+// Global-table form for a whole warp (all 32 lanes call it, converged; `on` marks lanes with a key):
+// insert / accumulate without touching the list, then append the warp's fresh slots with ONE
+// returning atomic on the community's list counter (every block working on a community hits that
+// counter; one atomic per fresh key serialised them -- the friendster_q level-0 coarsening).
+__device__ __forceinline__ void agg_insert_warp(bool on, int key, ull wt, int* keys, ull* vals, unsigned mask,
+                                                int* list, int* cnt) {
+    bool fresh = false;
+    unsigned h = 0;
+    if (on) {
+        h = hash_slot(key, mask);
+        for (;;) {
+            const int k0 = *(volatile int*)&keys[h];
+            if (k0 == key) { atomicAdd(&vals[h], wt); break; }
+            if (k0 == -1) {
+                const int old = atomicCAS(&keys[h], -1, key);
+                if (old == -1 || old == key) { fresh = old == -1; atomicAdd(&vals[h], wt); break; }
+            }
+            h = (h + 1) & mask;
+        }
+    }
+    const unsigned fm = __ballot_sync(FULLMASK, fresh);
+    if (!fm) return;
+    const int lane = threadIdx.x & 31, lead = __ffs(fm) - 1;
+    int base = 0;
+    if (lane == lead) base = atomicAdd(cnt, __popc(fm));
+    base = __shfl_sync(FULLMASK, base, lead);
+    if (fresh) list[base + __popc(fm & ((1u << lane) - 1u))] = (int)h;
+}
+
 // `nt` threads (tid = this thread's index among them, whole warps) stream
 // segment entries [s0, s1) with 4 entries per lane in flight; equal keys of
 // every 32-entry chunk are combined before inserting.
@@ -487,6 +516,118 @@ __global__ void __launch_bounds__(BT) k_agg_block(AggArgs a, int scap, const int
     }
 }
 
+// Class D: communities whose table bound (2 min(entries, k)) exceeds the shared arena but whose
+// segment is short enough for one block (entries <= agg_big_ent): the hierarchical table of §4.2
+// -- the block's shared H0 (scap slots, probed over a window of AGG_HWIN slots once
+// the bound exceeds it) spills to the block's own global H1 (linear probing, sized for the
+// longest class-D segment), both with distinct lists.  The bound is pessimistic (the Friendster-
+// shaped level 0 averages ~5k distinct keys in ~15k entries), so almost every key stays in H0
+// and the chunked global path (every key a global atomic) is left to the truly big communities.
+#define AGG_HWIN 32
+template <bool UNIT, typename V>
+__global__ void __launch_bounds__(512) k_agg_block_h(AggArgs a, int scap, const int32_t* __restrict__ bl,
+                                                     const int* __restrict__ nbl, int* __restrict__ gkeys_all,
+                                                     ull* __restrict__ gvals_all, int* __restrict__ glist_all,
+                                                     long long gcap) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    V* vals = reinterpret_cast<V*>(smem_raw);
+    int* keys = reinterpret_cast<int*>(smem_raw + (size_t)scap * sizeof(V));
+    int* list = keys + scap;
+    __shared__ int s_cnt, s_gcnt;
+    __shared__ V s_scr[16][32];
+    const int lane = lane_id(), wib = threadIdx.x >> 5;
+    int* gkeys = gkeys_all + (long long)blockIdx.x * gcap;
+    ull* gvals = gvals_all + (long long)blockIdx.x * gcap;
+    int* glist = glist_all + (long long)blockIdx.x * gcap;
+    const unsigned smask = (unsigned)scap - 1, gmask = (unsigned)gcap - 1;
+    for (int j = threadIdx.x; j < scap; j += 512) { keys[j] = -1; vals[j] = 0; }
+    if (threadIdx.x == 0) { s_cnt = 0; s_gcnt = 0; }
+    __syncthreads();
+    const long long cnt = *nbl;
+    for (long long i = blockIdx.x; i < cnt; i += gridDim.x) {
+        const long long c = bl[i];
+        const long long s0 = a.eoff[c], s1 = a.eoff[c + 1];
+        for (long long r0 = s0 + (threadIdx.x & ~31) * 4; r0 < s1; r0 += 512LL * 4) {   // warp-uniform
+            int kk[4];
+            V ww[4];
+#pragma unroll
+            for (int t = 0; t < 4; ++t) {
+                const long long j = r0 + lane + 32 * t;
+                kk[t] = j < s1 ? a.tkey[j] : -1;
+                ww[t] = (j < s1 && !UNIT) ? (V)a.tval[j] : (V)1;
+            }
+#pragma unroll
+            for (int t = 0; t < 4; ++t) {
+                if (r0 + 32 * t >= s1) break;
+                const unsigned peers = __match_any_sync(FULLMASK, kk[t] >= 0 ? kk[t] : -1 - lane);
+                const V sum = UNIT ? (V)__popc(peers) : group_sum(peers, kk[t] >= 0 ? ww[t] : (V)0, s_scr[wib]);
+                bool gfresh = false;
+                unsigned gh = 0;
+                if (kk[t] >= 0 && lane == __ffs(peers) - 1) {
+                    // H0: window of AGG_HWIN slots
+                    unsigned h = hash_slot(kk[t], smask);
+                    bool done = false;
+                    for (int p = 0; p < AGG_HWIN && !done; ++p, h = (h + 1) & smask) {
+                        const int k0 = keys[h];
+                        if (k0 == kk[t]) { atomicAdd(&vals[h], sum); done = true; }
+                        else if (k0 == -1) {
+                            const int old = atomicCAS(&keys[h], -1, kk[t]);
+                            if (old == -1) { atomicAdd(&vals[h], sum); list[atomicAdd(&s_cnt, 1)] = (int)h; done = true; }
+                            else if (old == kk[t]) { atomicAdd(&vals[h], sum); done = true; }
+                        }
+                    }
+                    if (!done) {   // H1
+                        gh = hash_slot(kk[t], gmask);
+                        for (;;) {
+                            const int k0 = *(volatile int*)&gkeys[gh];
+                            if (k0 == kk[t]) { atomicAdd(&gvals[gh], (ull)sum); break; }
+                            if (k0 == -1) {
+                                const int old = atomicCAS(&gkeys[gh], -1, kk[t]);
+                                if (old == -1 || old == kk[t]) { gfresh = old == -1; atomicAdd(&gvals[gh], (ull)sum); break; }
+                            }
+                            gh = (gh + 1) & gmask;
+                        }
+                    }
+                }
+                const unsigned fm = __ballot_sync(FULLMASK, gfresh);
+                if (fm) {
+                    const int lead = __ffs(fm) - 1;
+                    int base = 0;
+                    if (lane == lead) base = atomicAdd(&s_gcnt, __popc(fm));
+                    base = __shfl_sync(FULLMASK, base, lead);
+                    if (gfresh) glist[base + __popc(fm & lanemask_lt())] = (int)gh;
+                }
+            }
+        }
+        __syncthreads();
+        const int m0 = s_cnt, m1 = s_gcnt;
+        // distinct entries to the start of the segment (m0 + m1 <= entries), tables cleared
+        for (int t = threadIdx.x; t < m0 + m1; t += 512) {
+            int key;
+            int64_t val;
+            if (t < m0) {
+                const int slot = list[t];
+                key = keys[slot];
+                val = (int64_t)vals[slot];
+                keys[slot] = -1;
+                vals[slot] = 0;
+            } else {
+                const int slot = glist[t - m0];
+                key = gkeys[slot];
+                val = (int64_t)gvals[slot];
+                gkeys[slot] = -1;
+                gvals[slot] = 0;
+            }
+            a.tkey[s0 + t] = key;
+            a.tval[s0 + t] = val;
+            if (key == (int)c) a.snew[c] = val;
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) { a.dn[c] = m0 + m1; s_cnt = 0; s_gcnt = 0; }
+        __syncthreads();
+    }
+}
+
 // big communities: BPC blocks per community stream chunks of its segment into its global table
 template <bool UNIT, typename V>
 __global__ void __launch_bounds__(256) k_agg_big_insert(AggArgs a, const int32_t* __restrict__ bigc, int nbig,
@@ -550,7 +691,7 @@ __device__ __forceinline__ void list_append(bool on, int32_t val, int32_t* list,
 __global__ void k_agg_classify(long long k, const long long* __restrict__ ent, int scap, long long* __restrict__ dn,
                                int32_t* __restrict__ wl, int* __restrict__ nwl, int32_t* __restrict__ bl,
                                int* __restrict__ nbl, int32_t* __restrict__ bigc, long long* __restrict__ bigcap,
-                               int* __restrict__ nbig, long long kcap, long long big_ent) {
+                               int* __restrict__ nbig, long long kcap, long long big_ent, long long spill_ent) {
     // bl holds three lists of capacity kcap each (classes A, B, C), nbl their three counts;
     // communities with more than big_ent entries take the chunked big path even when their
     // table fits in shared memory (one block per community would serialise them)
@@ -560,7 +701,10 @@ __global__ void k_agg_classify(long long k, const long long* __restrict__ ent, i
         const long long e = c < k ? ent[c] : 0;
         const long long cap = c < k ? agg_cap(e, k) : -1;
         if (cap == 0) dn[c] = 0;
-        const bool isbig = cap > scap || e > big_ent;
+        // class D (spilling block path, bl + 3 kcap): table beyond the arena, segment short enough
+        const bool spill = cap > scap && e <= spill_ent;
+        list_append(spill, (int32_t)c, bl + 3 * kcap, nbl + 3);
+        const bool isbig = !spill && (cap > scap || e > big_ent);
         list_append(!isbig && cap > 0 && cap <= AGG_WSLOTS, (int32_t)c, wl, nwl);
         list_append(!isbig && cap > AGG_WSLOTS && cap <= AGG_BA && cap <= scap, (int32_t)c, bl, nbl);
         list_append(!isbig && cap > AGG_BA && cap <= AGG_BB && cap <= scap, (int32_t)c, bl + kcap, nbl + 1);
@@ -636,13 +780,19 @@ __global__ void __launch_bounds__(256) k_agg_big_chunk(AggArgs a, const int32_t*
         const int m = s_cnt;
         const long long off = goff[bi];
         const unsigned mask = (unsigned)(goff[bi + 1] - off) - 1u;
-        for (int i = threadIdx.x; i < m; i += 256) {
-            const int slot = list[i];
-            const int key = keys[slot];
-            const V val = vals[slot];
-            keys[slot] = -1;
-            vals[slot] = 0;
-            agg_insert<ull>(key, (ull)val, gkeys + off, gvals + off, mask, glist + off / 2, &gcnt[bi]);
+        for (int i0 = threadIdx.x & ~31; i0 < m; i0 += 256) {   // warp-uniform trips
+            const int i = i0 + (threadIdx.x & 31);
+            const bool on = i < m;
+            int key = 0;
+            V val = 0;
+            if (on) {
+                const int slot = list[i];
+                key = keys[slot];
+                val = vals[slot];
+                keys[slot] = -1;
+                vals[slot] = 0;
+            }
+            agg_insert_warp(on, key, (ull)val, gkeys + off, gvals + off, mask, glist + off / 2, &gcnt[bi]);
         }
         __syncthreads();
         if (threadIdx.x == 0) s_cnt = 0;
@@ -723,9 +873,12 @@ __global__ void __launch_bounds__(256) k_agg_big_insert2(AggArgs a, const int32_
         const int m = ndc[t];
         const long long off = goff[bi];
         const unsigned mask = (unsigned)(goff[bi + 1] - off) - 1u;
-        for (int i = threadIdx.x; i < m; i += 256)
-            agg_insert<ull>(a.tkey[lo + i], (ull)a.tval[lo + i], gkeys + off, gvals + off, mask, glist + off / 2,
-                            &gcnt[bi]);
+        for (int i0 = threadIdx.x & ~31; i0 < m; i0 += 256) {   // warp-uniform trips
+            const int i = i0 + (threadIdx.x & 31);
+            const bool on = i < m;
+            agg_insert_warp(on, on ? a.tkey[lo + i] : 0, on ? (ull)a.tval[lo + i] : 0, gkeys + off, gvals + off, mask,
+                            glist + off / 2, &gcnt[bi]);
+        }
     }
 }
 

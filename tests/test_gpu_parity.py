@@ -127,10 +127,12 @@ def test_pruning_strategy_weighted_and_graph_mode(strategy):
     dict(delta_update=1, ckey=1),
     dict(concurrent=1),
     dict(hub(64), concurrent=1, delta_update=1),
-    dict(agg_scap=512, agg_chunk=64),                                        # phase 2: many multi-chunk big communities
-    dict(agg_scap=512, agg_chunk=1),
-    dict(agg_scap=512, agg_chunk=64, agg_bound=0),                           # phase 2: one-pass big path
-    dict(agg_scap=512, agg_big_chunk=0),                                     # phase 2: per-community block split
+    dict(agg_scap=512, agg_chunk=64, agg_spill=0),                           # phase 2: many multi-chunk big communities
+    dict(agg_scap=512, agg_chunk=1, agg_spill=0),
+    dict(agg_scap=512, agg_chunk=64, agg_bound=0, agg_spill=0),              # phase 2: one-pass big path
+    dict(agg_scap=512, agg_big_chunk=0, agg_spill=0),                        # phase 2: per-community block split
+    dict(agg_scap=512),                                                      # phase 2: spilling block class (H0 512 slots)
+    dict(agg_scap=512, agg_big_ent=200),                                     # phase 2: spilling block + big paths
     dict(agg_big_ent=64, agg_chunk=32),                                      # phase 2: entry-count big path
     dict(agg_dense=0),                                                       # phase 2: never the dense k x k path
     dict(force_wide=2),                                                      # W64 level, packed short-row bins
@@ -146,7 +148,8 @@ def test_dispatch_independence(opts):
 
 
 @pytest.mark.parametrize("opts", [dict(force_wide=1), dict(force_wide=2), dict(force_i128=1), hub(16),
-                                  dict(hub(16), force_i128=1), dict(agg_scap=512, agg_chunk=16), dict(agg_dense=0)])
+                                  dict(hub(16), force_i128=1), dict(agg_scap=512, agg_chunk=16, agg_spill=0),
+                                  dict(agg_scap=512), dict(agg_dense=0)])
 def test_weighted_modes_parity(opts):
     """Weighted random graphs through every gain-arithmetic mode (DM_W64 / DM_W128)."""
     for seed in range(4):
