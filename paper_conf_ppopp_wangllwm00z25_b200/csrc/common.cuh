@@ -39,6 +39,7 @@ struct IterCounters {
     ull n_fn;               // instrumented pruning: pruned vertices that would have moved (Eq. 3)
     ull n_fp;               // instrumented pruning: active vertices that stay
     ull cursor_hi;          // dynamic work cursor of the block bin's long-row class (k_decide_block CLS 2)
+    ull n_items_hi;         // delta-update items of movers with rows > DLIGHT, stored from the END of the item arrays
     ull n_dense;            // multi-GPU (fabric): senders whose label exchange went dense this iteration
     ull xbytes;             // multi-GPU (fabric): bytes this rank received in its inbox this iteration
 };

@@ -435,6 +435,7 @@ static void gamma_to_pq(double gamma, int64_t* p, int64_t* q) {
 struct Work {
     cudaStream_t st;
     int64_t ncap, nnzcap;
+    long long icap = 0;   // capacity of the delta-update item arrays (light items from the front, others from the back)
     int64_t qcap = 0;   // queue stride (records per bin pair): n on one GPU, the largest owned range so far with several
     int32_t *rmflag = nullptr, *smflag = nullptr, *chg = nullptr;   // SM / RM movement history (prune 2-4)
     int32_t *C = nullptr, *size = nullptr, *stamp = nullptr, *mv_v = nullptr, *mv_old = nullptr, *mv_chunk = nullptr, *nextC = nullptr;
@@ -830,14 +831,14 @@ static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, typename
     launch_decide<M, UNIT>(g, wk, G, qW, p, tm, maxdeg, idbits, single);
     e = tm.begin();
     k_apply<<<grid_for(n, AP_BT, big), AP_BT, 0, st>>>(wk.ctr, wk.queues, wk.qcap, wk.nextC, wk.C, wk.Sig, wk.size,
-                                                       wk.dp, wk.stamp, wk.carry, wk.mv_v, wk.mv_old, wk.mv_chunk, ps);
+                                                       wk.dp, wk.stamp, wk.carry, wk.mv_v, wk.mv_old, wk.mv_chunk, ps, wk.icap);
     CKL();
     tm.end(KC_APPLY, e);
     e = tm.begin();
     const bool ck = use_ckey(g, wk, G);
     k_dp_delta<UNIT><<<big, 256, 0, st>>>(wk.ctr, G.rp, G.col, G.w, wk.C, wk.mv_v, wk.mv_old, wk.mv_chunk, wk.stamp, wk.dp,
                                           wk.carry, G.nnz, g->opt_delta, 1, g->opt_delta_den, ck ? wk.ckey : nullptr,
-                                          nullptr, ps.rmflag, n);
+                                          nullptr, ps.rmflag, n, wk.icap);
     CKL();
     k_dp_full<UNIT><<<grid_for((G.nnz + 127) / 128 * 32, 256, big), 256, 0, st>>>(wk.ctr, G.nnz, G.row, G.col, G.w,
                                                                                  wk.C, wk.dp, g->opt_delta, 1, g->opt_delta_den,
@@ -1409,6 +1410,7 @@ static void ensure_workspace(gala_graph_s* g) {
             wk.stamp = dalloc<int32_t>(wk.ncap, st);
             // delta-update items: one per light mover + one per DCH-entry chunk of a heavy one
             const size_t icap = (size_t)wk.ncap + (size_t)(g->nnz0 / DCH) + 1;
+            wk.icap = (long long)icap;
             wk.mv_v = dalloc<int32_t>(icap, st);
             wk.mv_old = dalloc<int32_t>(icap, st);
             wk.mv_chunk = dalloc<int32_t>(icap, st);

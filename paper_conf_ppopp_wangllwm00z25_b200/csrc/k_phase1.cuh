@@ -272,15 +272,16 @@ __global__ void __launch_bounds__(PB_BT, GALA_PRUNE_MINB) k_prune_bin(int vlo, i
 // over many warps instead of serialising one (its d' is then summed by
 // atomics onto a zero written here).  Item capacity: n + nnz/DCH.
 #define DCH 256
+#define DLIGHT 64   // movers with rows up to this many entries: half-warp delta items
 __global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr, QRec* queues,
                                                  long long qstride, const int32_t* __restrict__ nextC,
                                                  int32_t* __restrict__ C, int64_t* __restrict__ Sig,
                                                  int32_t* __restrict__ size, int64_t* __restrict__ dp,
                                                  int32_t* __restrict__ stamp, const Carry* __restrict__ carry,
                                                  int32_t* __restrict__ it_v, int32_t* __restrict__ it_old,
-                                                 int32_t* __restrict__ it_chunk, PruneState ps) {
-    __shared__ unsigned s_cnt, s_items;
-    __shared__ ull s_ibase;
+                                                 int32_t* __restrict__ it_chunk, PruneState ps, long long icap) {
+    __shared__ unsigned s_cnt, s_items, s_hitems;
+    __shared__ ull s_ibase, s_hbase;
     long long cnt[NBINS];
     long long total = 0;
 #pragma unroll
@@ -322,30 +323,44 @@ __global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr,
                 if (deg > DCH) dp[v] = 0;   // chunk items add onto it
             }
         }
-        // items of this thread (0, 1, or the chunk count of a heavy mover)
-        const unsigned nit = !mover ? 0u : (deg > DCH ? (unsigned)((deg + DCH - 1) / DCH) : 1u);
+        // items of this thread: a light mover (row <= DLIGHT) is one item at the FRONT of the
+        // item arrays (half-warp per item in k_dp_delta), any other mover is one item or the chunk
+        // count of a heavy mover at the BACK (warp per item)
+        const bool light = mover && deg <= DLIGHT;
+        const unsigned nit = (!mover || light) ? 0u : (deg > DCH ? (unsigned)((deg + DCH - 1) / DCH) : 1u);
         unsigned incl = nit;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
             unsigned y = __shfl_up_sync(FULLMASK, incl, o);
             if (lane >= o) incl += y;
         }
-        if (threadIdx.x == 0) { s_cnt = 0; s_items = 0; }
+        if (threadIdx.x == 0) { s_cnt = 0; s_items = 0; s_hitems = 0; }
         __syncthreads();
         const unsigned m = __ballot_sync(FULLMASK, mover);
         if (m && lane == 0) atomicAdd(&s_cnt, (unsigned)__popc(m));
+        const unsigned lm = __ballot_sync(FULLMASK, light);
+        unsigned loff = 0;
+        if (lm && lane == 0) loff = atomicAdd(&s_items, (unsigned)__popc(lm));
+        loff = __shfl_sync(FULLMASK, loff, 0) + __popc(lm & lanemask_lt());
         unsigned ioff = 0;
         const unsigned wtot = __shfl_sync(FULLMASK, incl, 31);
-        if (lane == 31 && wtot) ioff = atomicAdd(&s_items, wtot);
+        if (lane == 31 && wtot) ioff = atomicAdd(&s_hitems, wtot);
         ioff = __shfl_sync(FULLMASK, ioff, 31) + incl - nit;
         __syncthreads();
         if (threadIdx.x == 0) {
             if (s_cnt) atomicAdd(&ctr->n_moved, (ull)s_cnt);
             s_ibase = s_items ? atomicAdd(&ctr->n_items, (ull)s_items) : 0;
+            s_hbase = s_hitems ? atomicAdd(&ctr->n_items_hi, (ull)s_hitems) : 0;
         }
         __syncthreads();
+        if (light) {
+            const ull at = s_ibase + loff;
+            it_v[at] = v;
+            it_old[at] = oc;
+            it_chunk[at] = 0;
+        }
         for (unsigned j = 0; j < nit; ++j) {
-            const ull at = s_ibase + ioff + j;
+            const long long at = icap - 1 - (long long)(s_hbase + ioff + j);
             it_v[at] = v;
             it_old[at] = oc;
             it_chunk[at] = (int32_t)j;
@@ -386,7 +401,7 @@ __global__ void __launch_bounds__(256) k_dp_delta(IterCounters* __restrict__ ctr
                                                   const Carry* __restrict__ carry, long long nnz, int mode,
                                                   long long fnum, long long fden, int32_t* __restrict__ ckey,
                                                   const int32_t* __restrict__ rev, int32_t* __restrict__ rmflag,
-                                                  int n) {
+                                                  int n, long long icap) {
     if (!use_delta(ctr, nnz, mode, fnum, fden)) {   // full recompute follows: clear d' (k_dp_zero fused)
         for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n;
              v += (long long)gridDim.x * blockDim.x)
@@ -400,11 +415,51 @@ __global__ void __launch_bounds__(256) k_dp_delta(IterCounters* __restrict__ ctr
     (void)rev;
     const int iter_id = carry->iter;
     const int lane = lane_id();
-    const long long m = (long long)ctr->n_items;
     long long wid = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+    // light movers (rows <= DLIGHT = 64): a half-warp per item, 4 entries per lane, two items per warp
+    {
+        const long long ml = (long long)ctr->n_items;
+        const int hl = lane & 15, half = lane >> 4;
+        for (long long i0 = wid * 2; i0 < ml; i0 += nw * 2) {   // warp-uniform
+            const long long i = i0 + half;
+            const bool ok = i < ml;
+            const int u = ok ? it_v[i] : 0, oc = ok ? it_old[i] : -1;
+            const int nc = ok ? C[u] : -1;
+            const int64_t b = ok ? rp[u] : 0, e = ok ? rp[u + 1] : 0;
+            int x[4], cx[4], sx[4];
+            long long wt[4];
+#pragma unroll
+            for (int t = 0; t < 4; ++t) {
+                const int64_t j = b + hl + 16 * t;
+                x[t] = j < e ? col[j] : u;
+                wt[t] = (UNIT || j >= e) ? 1 : w[j];
+            }
+#pragma unroll
+            for (int t = 0; t < 4; ++t) {
+                cx[t] = x[t] != u ? C[x[t]] : -1;
+                sx[t] = x[t] != u ? stamp[x[t]] : iter_id;
+            }
+            long long acc = 0;
+#pragma unroll
+            for (int t = 0; t < 4; ++t) {
+                if (x[t] == u) continue;
+                if (rmflag) rmflag[x[t]] = iter_id;
+                if (cx[t] == nc) acc += wt[t];
+                if (sx[t] != iter_id) {
+                    if (cx[t] == oc) atomicAdd(reinterpret_cast<ull*>(&dp[x[t]]), (ull)(-wt[t]));
+                    else if (cx[t] == nc) atomicAdd(reinterpret_cast<ull*>(&dp[x[t]]), (ull)wt[t]);
+                }
+            }
+#pragma unroll
+            for (int o = 8; o > 0; o >>= 1) acc += __shfl_xor_sync(FULLMASK, acc, o);
+            if (ok && hl == 0) dp[u] = acc;
+        }
+    }
+    const long long m = (long long)ctr->n_items_hi;
     for (long long i = wid; i < m; i += nw) {
-        const int u = it_v[i], oc = it_old[i], ch = it_chunk[i];
+        const long long ii = icap - 1 - i;
+        const int u = it_v[ii], oc = it_old[ii], ch = it_chunk[ii];
         const int nc = C[u];
         const int64_t rb = rp[u], re = rp[u + 1];
         const bool heavy = re - rb > DCH;
