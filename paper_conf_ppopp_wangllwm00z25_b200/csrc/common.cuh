@@ -40,6 +40,8 @@ struct IterCounters {
     ull n_fp;               // instrumented pruning: active vertices that stay
     ull cursor_hi;          // dynamic work cursor of the block bin's long-row class (k_decide_block CLS 2)
     ull n_items_hi;         // delta-update items of movers with rows > DLIGHT, stored from the END of the item arrays
+    ull h0_acc, h1_acc;     // block-bin hash inserts landing in the shared H0 / the global H1 (§4.2 access rate)
+    ull h0_keys, h1_keys;   // distinct communities held in H0 / H1 (§4.2 maintenance rate)
     ull n_dense;            // multi-GPU (fabric): senders whose label exchange went dense this iteration
     ull xbytes;             // multi-GPU (fabric): bytes this rank received in its inbox this iteration
 };

@@ -115,6 +115,9 @@ struct gala_graph_s {
     int opt_block_split = 1024;
     int opt_agg_bound = 1;
     int opt_agg_dense = 1;
+    int opt_l2_window = 0;   // persisting L2 access-policy window on C (A/B option)
+    int opt_table_mode = 0;  // block bin's hash table: 0 hierarchical (§4.2), 1 global-only, 2 unified (ablation)
+    double tbl[4] = {0, 0, 0, 0};   // last run: H0 / H1 accesses, H0 / H1 distinct keys of the block bin
     int opt_agg_spill = 1;   // phase 2: class D (one block, shared H0 spilling to global H1) for short segments
     int opt_bin_packed = 1;  // DM_W64 levels: packed argmax keys for the short-row bins where they fit   // phase 2: dense k x k accumulation when k <= AGG_DENSE_K and nnz >= 4 k^2
     bool rows_distinct0 = false;   // level-0 rows strictly increasing (no duplicate entries)
@@ -690,6 +693,7 @@ static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, typename M
     DecideArgs a;
     a.rp = G.rp; a.col = G.col; a.w = G.w; a.C = wk.C; a.Sig = wk.Sig; a.size = wk.size; a.d = wk.d;
     a.dp = wk.dp; a.nextC = wk.nextC; a.ctr = wk.ctr; a.check = g->opt_check;
+    a.table_mode = g->opt_table_mode;
     a.ckey = use_ckey(g, wk, G) ? wk.ckey : nullptr;
     a.ckey_valid = &wk.carry->ckey_valid;
     a.idbits = idbits;
@@ -1481,6 +1485,7 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
     g->trace_labels.clear();
     g->levels.clear();
     for (int i = 0; i < KC_COUNT; ++i) { g->kc_ms[i] = 0; g->kc_bytes[i] = 0; g->kc_launches[i] = 0; }
+    for (double& x : g->tbl) x = 0;
     g->dp_mismatch = 0;
     const long long launches0 = g_launches;
     int64_t p, q;
@@ -1500,6 +1505,33 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
     if (!g->lab) g->lab = dalloc<int32_t>(n0, st);
     ensure_workspace(g);
     Work& wk = *g->wk;
+    // option l2_window: keep the label array C (the per-entry random gathers) persisting in L2
+    // through a stream access-policy window (matters once C + Sigma_tot outgrow the 126 MB L2)
+    struct L2Window {
+        cudaStream_t st = nullptr;
+        ~L2Window() {
+            if (!st) return;
+            cudaStreamAttrValue v = {};
+            v.accessPolicyWindow.num_bytes = 0;
+            cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &v);
+            cudaCtxResetPersistingL2Cache();
+        }
+    } l2w;
+    if (g->opt_l2_window) {
+        int maxwin = 0, maxpers = 0;
+        CK(cudaDeviceGetAttribute(&maxwin, cudaDevAttrMaxAccessPolicyWindowSize, g->device));
+        CK(cudaDeviceGetAttribute(&maxpers, cudaDevAttrMaxPersistingL2CacheSize, g->device));
+        const size_t bytes = std::min<size_t>((size_t)n0 * sizeof(int32_t), (size_t)std::max(maxwin, 0));
+        CK(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, std::min<size_t>(bytes, (size_t)std::max(maxpers, 0))));
+        cudaStreamAttrValue v = {};
+        v.accessPolicyWindow.base_ptr = wk.C;
+        v.accessPolicyWindow.num_bytes = bytes;
+        v.accessPolicyWindow.hitRatio = 1.0f;
+        v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        CK(cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &v));
+        l2w.st = st;
+    }
     cudaEvent_t ev_run0 = wk.ev[0], ev_run1 = wk.ev[1];
     CK(cudaEventRecord(ev_run0, st));
     try {
@@ -1581,6 +1613,8 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
                 double b0 = 0, b1 = 0;
                 for (int i = 0; i < KC_COUNT; ++i) b0 += g->kc_bytes[i];
                 account_bytes(g, c, nl, cur.nnz, unit, it == 0 && g->opt_singleton && (level > 0 || g->rows_distinct0));
+                g->tbl[0] += (double)c.h0_acc; g->tbl[1] += (double)c.h1_acc;
+                g->tbl[2] += (double)c.h0_keys; g->tbl[3] += (double)c.h1_keys;
                 for (int i = 0; i < KC_COUNT; ++i) b1 += g->kc_bytes[i];
                 ls.alg_bytes += b1 - b0;
                 const int64_t it_ns = logs[it].t_ns >= t_prev ? (int64_t)(logs[it].t_ns - t_prev) : 0;
@@ -2835,6 +2869,11 @@ gala_status gala_set_option(gala_graph g, const char* key, int64_t value) {
         g->opt_bin_packed = value != 0;
     } else if (k == "agg_spill") {   // phase 2: spilling block class for segments <= agg_big_ent entries
         g->opt_agg_spill = value != 0;
+    } else if (k == "l2_window") {   // persisting-L2 access-policy window on the label array
+        g->opt_l2_window = value != 0;
+    } else if (k == "table_mode") {   // block-bin hash table (§4.2 ablation): 0 hierarchical, 1 global-only, 2 unified
+        if (value < 0 || value > 2) return set_err(GALA_E_INVALID, "table_mode: 0 hierarchical, 1 global-only, 2 unified");
+        g->opt_table_mode = (int)value;
     } else if (k == "agg_dense") {   // phase 2: dense k x k accumulation (0 never, 1 auto, 2 whenever k fits)
         if (value < 0 || value > 2) return set_err(GALA_E_INVALID, "agg_dense in 0..2");
         g->opt_agg_dense = (int)value;
@@ -2916,6 +2955,9 @@ gala_status gala_get_stats(gala_graph g, char* buf, int64_t cap, int64_t* needed
              "\"kernel_launches\":%lld,\"check_mismatch\":%d,",
              (long long)g->n0, (long long)g->nnz0, (long long)g->W, (long long)g->p, (long long)g->q, g->run_ms,
              (long long)g->dp_mismatch, g->launches, g->check_mismatch);
+    s += tmp;
+    snprintf(tmp, sizeof tmp, "\"table\":{\"h0_access\":%.0f,\"h1_access\":%.0f,\"h0_keys\":%.0f,\"h1_keys\":%.0f},",
+             g->tbl[0], g->tbl[1], g->tbl[2], g->tbl[3]);
     s += tmp;
     if (g->di) {
         snprintf(tmp, sizeof tmp, "\"dist\":{\"rank\":%d,\"world\":%d,\"v0\":%lld,\"v1\":%lld,\"dense_iters\":%lld,"

@@ -95,6 +95,7 @@ struct DecideArgs {
     const int* ckey_valid;
     IterCounters* ctr;
     int check;
+    int table_mode;     // block bin's table (§4.2): 0 hierarchical, 1 global-only, 2 unified
     int idbits;         // packed-key layout (DM_FAST)
     long long idmask;
 };
@@ -571,6 +572,7 @@ __global__ void BLOCK_LB(BT) k_decide_block(QView queue, int bin, DecideArgs a,
     for (int j = threadIdx.x; j < smem_cap; j += BT) { keys[j] = -1; vals[j] = 0; }
     if (threadIdx.x == 0) s_gcnt = 0;
     unsigned my_k = 0;
+    ull my_h0 = 0, my_h1 = 0, my_k0 = 0, my_k1 = 0;   // table access / maintenance counters (§4.2)
     __shared__ int s_batch[FETCH_B], s_nb, s_bi;
     if (threadIdx.x == 0) { s_nb = 0; s_bi = 0; }
     ull* const cursor = CLS == 2 ? &a.ctr->cursor_hi : &a.ctr->cursor[bin];
@@ -639,11 +641,24 @@ __global__ void BLOCK_LB(BT) k_decide_block(QView queue, int bin, DecideArgs a,
                 int gslot = -1;
                 if (cc[k] >= 0 && lane == __ffs(peers) - 1) {
                     bool fresh;
-                    const int slot = ht_insert4<VT, true>(cc[k], sum, keys, vals, smask, hash_slot(cc[k], smask), win,
-                                                          &fresh);
-                    if (slot < 0)
-                        gslot = ht_insert4<ull, false>(cc[k], (ull)sum, gkeys, gvals, gmask, hash_slot2(cc[k], gmask),
-                                                       (int)gc, &gfresh);
+                    int slot = -1;
+                    unsigned g0 = hash_slot2(cc[k], gmask);
+                    // (the short-row class's arena never spills and its grid can exceed the H1 tables)
+                    const int tmode = CLS == 1 ? 0 : a.table_mode;
+                    if (tmode == 0) {                 // hierarchical: H0 first (own hash), H1 on collision
+                        slot = ht_insert4<VT, true>(cc[k], sum, keys, vals, smask, hash_slot(cc[k], smask), win, &fresh);
+                    } else if (tmode == 2) {          // unified: one hash over the s + g buckets
+                        const unsigned uh = (unsigned)(((unsigned long long)(unsigned)cc[k] * 2654435761ull) %
+                                                       (unsigned long long)(tcap + gc));
+                        if (uh < (unsigned)tcap) slot = ht_insert4<VT, true>(cc[k], sum, keys, vals, smask, uh, win, &fresh);
+                        else g0 = uh - (unsigned)tcap;
+                    }                                 // global-only: H1 always
+                    if (slot < 0) {
+                        gslot = ht_insert4<ull, false>(cc[k], (ull)sum, gkeys, gvals, gmask, g0, (int)gc, &gfresh);
+                        ++my_h1;
+                    } else {
+                        ++my_h0;
+                    }
                 }
                 if (__any_sync(FULLMASK, gfresh)) append_fresh<int>(gfresh, gslot, FULLMASK, &s_gcnt, glist);
             }
@@ -658,6 +673,7 @@ __global__ void BLOCK_LB(BT) k_decide_block(QView queue, int bin, DecideArgs a,
         A best;
         best.init(a.idbits, a.idmask);
         my_k += (threadIdx.x == 0) ? (unsigned)gm : 0u;
+        my_k1 += (threadIdx.x == 0) ? (ull)gm : 0ull;
         // evaluate and clear the used H0 prefix, four slots (one 16-byte key load) per thread
         for (int t0 = threadIdx.x * 4; t0 < tcap; t0 += BT * 4) {
             const int4 k4 = *reinterpret_cast<const int4*>(keys + t0);
@@ -675,6 +691,7 @@ __global__ void BLOCK_LB(BT) k_decide_block(QView queue, int bin, DecideArgs a,
                 if (cs[k] < 0) continue;
                 vals[t0 + k] = 0;
                 ++my_k;
+                ++my_k0;
                 best.offer(gain<ST>(qW, p, ws[k], sg[k], dv), cs[k]);
             }
         }
@@ -706,8 +723,9 @@ __global__ void BLOCK_LB(BT) k_decide_block(QView queue, int bin, DecideArgs a,
         }
         __syncthreads();   // table / list / s_item reuse
     }
-    ull k = block_sum_ull<BT>((ull)my_k);
-    if (threadIdx.x == 0 && k) atomicAdd(&a.ctr->bin_k[bin], k);
+    ull vals5[5] = {(ull)my_k, my_h0, my_h1, my_k0, my_k1};
+    ull* const dsts5[5] = {&a.ctr->bin_k[bin], &a.ctr->h0_acc, &a.ctr->h1_acc, &a.ctr->h0_keys, &a.ctr->h1_keys};
+    block_add_counters<BT, 5>(vals5, dsts5);
 }
 
 // ---------------------------------------------------------------------------

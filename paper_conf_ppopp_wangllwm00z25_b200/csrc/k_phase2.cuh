@@ -476,8 +476,27 @@ __global__ void __launch_bounds__(256) k_agg_warp(AggArgs a, const int32_t* __re
     const long long cnt = *nwl;
     for (long long i = (long long)blockIdx.x * 8 + wib; i < cnt; i += nw) {
         const long long c = wl[i];
+        const long long s0 = a.eoff[c], s1 = a.eoff[c + 1];
+        if (s1 - s0 <= 32) {   // one lane per entry: __match_any_sync alone finds the distinct keys
+            const int j = lane;
+            const bool on = j < s1 - s0;
+            const int key = on ? a.tkey[s0 + j] : -1 - lane;
+            const V wt = (on && !UNIT) ? (V)a.tval[s0 + j] : (V)(on ? 1 : 0);
+            const unsigned peers = __match_any_sync(FULLMASK, key);
+            const V sum = UNIT ? (V)__popc(peers) : group_sum(peers, wt, s_scr[wib]);
+            const bool lead = on && lane == __ffs(peers) - 1;
+            const unsigned lm = __ballot_sync(FULLMASK, lead);
+            if (lead) {   // distinct entries to the start of the segment (lead lanes ascend, never overtake)
+                const int t = __popc(lm & lanemask_lt());
+                a.tkey[s0 + t] = key;
+                a.tval[s0 + t] = (int64_t)sum;
+                if (key == (int)c) a.snew[c] = (int64_t)sum;
+            }
+            if (lane == 0) a.dn[c] = __popc(lm);
+            continue;
+        }
         const long long cap = agg_cap(a.ent[c], a.k);
-        agg_segment<UNIT, V, V>(a, a.eoff[c], a.eoff[c + 1], lane, 32, keys, vals, (unsigned)cap - 1, list,
+        agg_segment<UNIT, V, V>(a, s0, s1, lane, 32, keys, vals, (unsigned)cap - 1, list,
                                 &s_cnt[wib], s_scr[wib]);
         __syncwarp();
         int m = s_cnt[wib];

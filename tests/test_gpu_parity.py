@@ -110,6 +110,9 @@ def test_pruning_strategy_weighted_and_graph_mode(strategy):
 
 @pytest.mark.parametrize("opts", [
     dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=0, bin_warp512=0),   # block hash
+    dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=0, bin_warp512=0, table_mode=1),  # global-only
+    dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=0, bin_warp512=0, table_mode=2),  # unified
+    dict(table_mode=2, hub_smem_slots=64),
     dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=128),                # warp hash <= 128
     dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=0),                  # warp512 hash <= 512
     dict(bin_sub4=4, bin_sub8=4, bin_sub16=4, bin_sub32=32, bin_warp=32),
@@ -374,3 +377,21 @@ def test_dense_coarsening_weighted():
     for seed in range(3):
         g = gg.random_graph(300, 2000, seed=2100 + seed, max_w=7, self_loops=5)
         assert_parity(g, gamma=[1.0, 0.5, 2.0][seed], agg_dense=2)
+
+
+def test_table_mode_access_counters():
+    """§4.2 ablation counters: every block-bin insert lands in H0 or H1; global-only
+    never touches H0; the hierarchical table keeps more accesses in shared memory than the unified
+    one (Fig. 4's direction) on a graph whose block-bin tables overflow a small H0."""
+    g = gg.make("rmat_small")
+    base = dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=0, bin_warp512=0, hub_smem_slots=256,
+                block_split=0)
+    t = {}
+    for mode in (0, 1, 2):
+        r = run_gpu(g, trace=1, table_mode=mode, **base)
+        t[mode] = r["stats"]["table"]
+    assert t[1]["h0_access"] == 0 and t[1]["h1_access"] > 0 and t[1]["h0_keys"] == 0
+    for mode in (0, 2):
+        assert t[mode]["h0_access"] + t[mode]["h1_access"] == t[1]["h1_access"]
+    rate = {m: t[m]["h0_access"] / (t[m]["h0_access"] + t[m]["h1_access"]) for m in (0, 2)}
+    assert rate[0] > rate[2]

@@ -10,7 +10,8 @@ NEXT #2-#4), one JSON object per line.
   ablations  : Fig. 6 (no pruning + global-memory tables vs MG vs MG + memory
                management), Fig. 8 (B / P1 / P2 breakdown of DecideAndMove vs weight
                update), Fig. 9 (P:410-422: shuffle vs shared vs global tables for small rows;
-               hierarchical vs global-only for rows > 2000).
+               hierarchical vs unified vs global-only tables for long rows, with the shared-
+               memory access / maintenance rates of Fig. 4).
 usage: python tools/pruning_eval.py strategies|ablations CONFIG [CONFIG ...]
 """
 import json
@@ -104,9 +105,9 @@ def strategies(name):
 
 def ablations(name):
     g = gg.make(name)
-    # "global-memory tables": every row through the block kernel with a 64-slot shared H0, so
-    # nearly every community lives in the block's global H1 (the paper's baseline table)
-    glob = dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=0, bin_warp512=0, hub_smem_slots=64)
+    # "global-memory tables": every row through the block kernel with the global-only table
+    # (table_mode 1: every community in the block's global H1 -- the paper's baseline)
+    glob = dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=0, bin_warp512=0, table_mode=1)
     rows = [
         ("fig6", "baseline: no pruning, global-memory tables", dict(glob, prune=0, delta_update=0)),
         ("fig6", "MG pruning, global-memory tables", dict(glob, prune=1)),
@@ -117,18 +118,26 @@ def ablations(name):
         ("fig9a", "rows <= 32: sub-warp shuffle (default)", dict()),
         ("fig9a", "rows <= 32: warp shared-memory hash", dict((k, 0) for k in SMALL)),
         ("fig9a", "all rows: block kernel, 64-slot H0 (global-memory hash)", glob),
-        ("fig9b", "rows > 512: hierarchical smem + global (default)", dict()),
-        ("fig9b", "rows > 512: 64-slot H0, i.e. global-only tables", dict(hub_smem_slots=64)),
+        ("fig9b", "rows > 512: hierarchical smem H0 + global H1 (default, P:308)", dict()),
+        ("fig9b", "rows > 512: unified smem + global, one hash (P:306)", dict(table_mode=2)),
+        ("fig9b", "rows > 512: global-only (P:302)", dict(table_mode=1)),
+        ("fig9b", "rows > 512: hierarchical, 1024-slot H0 (more spilling)", dict(hub_smem_slots=1024)),
+        ("fig9b", "rows > 512: unified, 1024-slot H0", dict(hub_smem_slots=1024, table_mode=2)),
         ("fig9b", "rows > 512: multi-block hub path (global tables)", dict(bin_block=512)),
     ]
     for fig, label, opts in rows:
         h, ms = timed(g, opts, reps=3)
         Q = h.modularity()
+        tb = h.stats()["table"]
         h.free()
+        acc = tb["h0_access"] + tb["h1_access"]
+        keys = tb["h0_keys"] + tb["h1_keys"]
         ks, st = kernel_ms(g, opts)
         dec = sum(v for k, v in ks.items() if k.startswith("decide"))
         print(json.dumps(dict(kind="ablation", figure=fig, config=name, variant=label, options=opts,
                               run_ms=round(ms, 3), Q=round(Q, 6), decide_ms=round(dec, 3),
+                              smem_access_rate=round(tb["h0_access"] / acc, 4) if acc else None,
+                              smem_maintenance_rate=round(tb["h0_keys"] / keys, 4) if keys else None,
                               dp_update_ms=ks.get("dp_update", 0.0), kernels_ms=ks)), flush=True)
 
 
