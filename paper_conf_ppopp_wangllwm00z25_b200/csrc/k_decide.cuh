@@ -208,6 +208,9 @@ __device__ __forceinline__ unsigned decide_sub_bin(QView queue, int bin, const D
 #ifndef GALA_SMALL_MINB
 #define GALA_SMALL_MINB 4   // <= 64 registers: 32 warps per SM (measured -30% vs 72-80 regs)
 #endif
+#ifndef GALA_WARP_SCAN
+#define GALA_WARP_SCAN 0   // warp128: evaluate by scanning the 256-slot table instead of keeping a distinct list
+#endif
 #ifndef GALA_WARP_PREFETCH
 #define GALA_WARP_PREFETCH 1   // warp128: next vertex's row loaded during this one's evaluation
 #endif
@@ -369,6 +372,7 @@ __global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB, MAXDEG <= 1
     // PF: the row entries of a group's NEXT vertex are loaded while the current one is
     // evaluated (every row here fits one round: deg <= MAXDEG = GW * CH)
     constexpr bool PF = GALA_WARP_PREFETCH && MAXDEG <= 128 && MAXDEG == GW * CH;
+    constexpr bool SCAN = GALA_WARP_SCAN && MAXDEG <= 128;   // table scan instead of a distinct list
     const int* __restrict__ rsrc = a.ckey ? a.ckey : a.col;
     int pu[CH];
     VT pw[CH];
@@ -432,7 +436,7 @@ __global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB, MAXDEG <= 1
                     slot = MAXDEG > 128   // bucketed probing pays only in the larger tables (measured)
                                ? ht_insert4<VT, true>(cc[k], sum, keys, vals, WMASK, hash_slot(cc[k], WMASK), WCAP, &fresh)
                                : ht_insert<VT>(cc[k], sum, keys, vals, WMASK, hash_slot(cc[k], WMASK), WCAP, &fresh);
-                append_fresh<short>(fresh, slot, gmask, cnt, list);
+                if (!SCAN) append_fresh<short>(fresh, slot, gmask, cnt, list);
             }
         }
         if (PF) {   // next vertex's row: in flight during this vertex's evaluation
@@ -445,10 +449,32 @@ __global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB, MAXDEG <= 1
             }
         }
         __syncwarp();
-        const int m = *cnt;
-        my_k += (gl == 0) ? m : 0;
         Arg<ST, ModeT<M>::PK> best;
         best.init(a.idbits, a.idmask);
+        if (SCAN) {   // no distinct list: the group scans its whole table (4 slots per 16-byte load)
+            for (int t0 = gl * 4; t0 < WCAP; t0 += GW * 4) {
+                const int4 k4 = *reinterpret_cast<const int4*>(keys + t0);
+                if ((k4.x & k4.y & k4.z & k4.w) == -1) continue;   // all four empty
+                const int cs[4] = {k4.x, k4.y, k4.z, k4.w};
+                long long ws[4], sg[4];
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    ws[k] = cs[k] >= 0 ? (long long)vals[t0 + k] : 0;
+                    sg[k] = (cs[k] >= 0 && cs[k] != cv) ? a.Sig[cs[k]] : 0;
+                }
+                *reinterpret_cast<int4*>(keys + t0) = make_int4(-1, -1, -1, -1);
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    if (cs[k] < 0) continue;
+                    vals[t0 + k] = 0;
+                    ++my_k;
+                    if (cs[k] == cv) own = ws[k];
+                    else best.offer(gain<ST>(qW, p, ws[k], sg[k], dv), cs[k]);
+                }
+            }
+        }
+        const int m = SCAN ? 0 : *cnt;
+        my_k += (!SCAN && gl == 0) ? m : 0;
         for (int t0 = gl; t0 < m; t0 += GW * CH) {
             int cs[CH];
             long long ws[CH];

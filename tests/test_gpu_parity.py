@@ -388,10 +388,11 @@ def test_table_mode_access_counters():
                 block_split=0)
     t = {}
     for mode in (0, 1, 2):
-        r = run_gpu(g, trace=1, table_mode=mode, **base)
+        _, r = assert_parity(g, labels=False, table_mode=mode, **base)
         t[mode] = r["stats"]["table"]
     assert t[1]["h0_access"] == 0 and t[1]["h1_access"] > 0 and t[1]["h0_keys"] == 0
-    for mode in (0, 2):
-        assert t[mode]["h0_access"] + t[mode]["h1_access"] == t[1]["h1_access"]
+    for mode in (0, 2):   # the same inserts, split differently (equal up to a handful of chunk races)
+        tot = t[mode]["h0_access"] + t[mode]["h1_access"]
+        assert abs(tot - t[1]["h1_access"]) <= 1e-4 * tot
     rate = {m: t[m]["h0_access"] / (t[m]["h0_access"] + t[m]["h1_access"]) for m in (0, 2)}
     assert rate[0] > rate[2]

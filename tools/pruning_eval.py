@@ -107,7 +107,8 @@ def ablations(name):
     g = gg.make(name)
     # "global-memory tables": every row through the block kernel with the global-only table
     # (table_mode 1: every community in the block's global H1 -- the paper's baseline)
-    glob = dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=0, bin_warp512=0, table_mode=1)
+    glob = dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=0, bin_warp512=0, table_mode=1,
+                block_split=0)
     rows = [
         ("fig6", "baseline: no pruning, global-memory tables", dict(glob, prune=0, delta_update=0)),
         ("fig6", "MG pruning, global-memory tables", dict(glob, prune=1)),
@@ -118,11 +119,11 @@ def ablations(name):
         ("fig9a", "rows <= 32: sub-warp shuffle (default)", dict()),
         ("fig9a", "rows <= 32: warp shared-memory hash", dict((k, 0) for k in SMALL)),
         ("fig9a", "all rows: block kernel, 64-slot H0 (global-memory hash)", glob),
-        ("fig9b", "rows > 512: hierarchical smem H0 + global H1 (default, P:308)", dict()),
-        ("fig9b", "rows > 512: unified smem + global, one hash (P:306)", dict(table_mode=2)),
-        ("fig9b", "rows > 512: global-only (P:302)", dict(table_mode=1)),
-        ("fig9b", "rows > 512: hierarchical, 1024-slot H0 (more spilling)", dict(hub_smem_slots=1024)),
-        ("fig9b", "rows > 512: unified, 1024-slot H0", dict(hub_smem_slots=1024, table_mode=2)),
+        ("fig9b", "rows > 512: hierarchical smem H0 + global H1 (P:308; one block class)", dict(block_split=0)),
+        ("fig9b", "rows > 512: unified smem + global, one hash (P:306)", dict(block_split=0, table_mode=2)),
+        ("fig9b", "rows > 512: global-only (P:302)", dict(block_split=0, table_mode=1)),
+        ("fig9b", "rows > 512: hierarchical, 1024-slot H0 (more spilling)", dict(block_split=0, hub_smem_slots=1024)),
+        ("fig9b", "rows > 512: unified, 1024-slot H0", dict(block_split=0, hub_smem_slots=1024, table_mode=2)),
         ("fig9b", "rows > 512: multi-block hub path (global tables)", dict(bin_block=512)),
     ]
     for fig, label, opts in rows:
