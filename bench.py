@@ -275,7 +275,6 @@ def main():
     import torch
     import graphgen as gg
     import paper_conf_ppopp_wangllwm00z25_b200 as gala
-    import quality
 
     if world > 1 or args.force_dist:
         import torch.distributed as dist
@@ -446,7 +445,9 @@ def main():
         "gteps_scanned_all_levels": scanned / total_s / 1e9,
         "step_ms": [round(x, 3) for x in step_ms],
         "modularity": Q,
-        "nmi_vs_planted": (quality.nmi_device(labels, g.truth) if getattr(g, "truth", None) is not None else None),
+        "nmi_vs_planted": (gala.nmi(torch.as_tensor(labels, dtype=torch.int32).cuda(),
+                                    torch.as_tensor(g.truth, dtype=torch.int32).cuda())
+                           if getattr(g, "truth", None) is not None else None),
         "pruned_fraction_per_iteration": pruned,
         "levels": len(last_stats["levels"]),
         "iterations": sum(lv["iters"] for lv in last_stats["levels"]),

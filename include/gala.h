@@ -289,6 +289,23 @@ gala_status gala_graph_from_csr_dist(const void* uid128, int rank, int world, in
                                      const int64_t* weights, uintptr_t stream, gala_graph* out);
 
 /*
+ * gala_nmi_device — normalised mutual information of two partitions (quality report of
+ * Table 4; definition of ref. [52], Strehl & Ghosh 2002):
+ *   NMI = I(X;Y) / sqrt(H(X) H(Y)),  I = sum_ab (n_ab/n) ln(n n_ab / (n_a n_b)),
+ *   H(X) = -sum_a (n_a/n) ln(n_a/n);  1 if both partitions have one cluster, 0 if only one has.
+ *   d_x, d_y : DEVICE int32[n] on `device`, labels in [0, n) (e.g. gala_get_communities_device
+ *              output and an LFR planted partition); read only, caller keeps ownership
+ *   n        : 0 <= n < 2^31 (n = 0 gives 1)
+ *   stream   : cudaStream_t as an integer (0 = legacy default stream); synchronised on return
+ *   out      : receives the NMI (fp64; contingency counts are exact integers, the three log
+ *              sums are reduced in a fixed order, so the value is reproducible)
+ * GALA_E_INVALID for a null pointer, n out of range or a label outside [0, n); GALA_E_CUDA on
+ * a device error.  Not a step of the Louvain path: it reports the quality of a result.
+ */
+gala_status gala_nmi_device(const int32_t* d_x, const int32_t* d_y, int64_t n, int device, uintptr_t stream,
+                            double* out);
+
+/*
  * gala_partition_ranges — host-only helper: edge-balanced contiguous split of
  * n vertices over `world` ranks (each range's entry count ~ nnz/world).
  * bounds: int64[world+1].

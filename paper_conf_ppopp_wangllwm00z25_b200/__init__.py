@@ -71,6 +71,7 @@ def lib():
                                           ctypes.c_size_t, pp]),
         "gala_partition_ranges": (st, [i64, p, ctypes.c_int, p]),
         "gala_set_allocator": (st, [p, p, p]),
+        "gala_nmi_device": (st, [p, p, i64, ctypes.c_int, ctypes.c_size_t, ctypes.POINTER(dbl)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -167,6 +168,22 @@ def loopback_unique_id() -> bytes:
     buf = ctypes.create_string_buffer(128)
     _check(lib().gala_loopback_unique_id(buf))
     return buf.raw
+
+
+def nmi(x, y, stream: int = 0) -> float:
+    """NMI of two partitions (include/gala.h gala_nmi_device, ref. [52]):
+    x, y are int32 CUDA tensors of equal length with labels in [0, n).  Computed by the
+    library's kernels on the tensors' device (argument marshalling only here)."""
+    import torch
+    if not (torch.is_tensor(x) and torch.is_tensor(y) and x.is_cuda and y.is_cuda):
+        raise TypeError("nmi: x and y must be CUDA tensors")
+    if x.dtype != torch.int32 or y.dtype != torch.int32 or x.numel() != y.numel() or x.device != y.device:
+        raise ValueError("nmi: x and y must be int32 tensors of equal length on one device")
+    xc, yc = x.contiguous(), y.contiguous()
+    out = ctypes.c_double()
+    _check(lib().gala_nmi_device(xc.data_ptr(), yc.data_ptr(), xc.numel(), x.device.index, stream,
+                                 ctypes.byref(out)))
+    return out.value
 
 
 def local_rows(row_ptr, col, w, v0: int, v1: int):

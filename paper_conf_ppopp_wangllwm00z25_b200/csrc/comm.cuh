@@ -40,6 +40,11 @@ struct Comm {
     virtual void release_region(const std::vector<void*>& peers) { (void)peers; }
     // host-side rendezvous of ranks that share one process (loopback); a no-op across processes
     virtual void host_barrier() {}
+    // may a kernel of this rank spin until the other ranks' kernels arrive (fabric device
+    // barrier)?  Only when every rank has its own GPU: kernels of several ranks on ONE device
+    // are not guaranteed to be co-resident (B200_PROFILING.md: Xid 109 when they are not), so
+    // the loopback ranks meet on the host instead (stream sync + host barrier).
+    virtual bool device_barrier_ok() const { return true; }
     // personalised exchange (bytes): send + sdispls[p] .. + scounts[p] goes to rank p, which
     // receives it at recv + its rdispls[this rank]; device buffers on `st`
     virtual void alltoallv(const void* send, const std::vector<size_t>& scounts, const std::vector<size_t>& sdispls,
@@ -306,6 +311,7 @@ struct LoopComm : Comm {
         return out;
     }
     void host_barrier() override { sh->barrier(); }
+    bool device_barrier_ok() const override { return world == 1; }
     // same process, same device: the peers' regions are plain device pointers
     std::vector<void*> share_region(void* mine, cudaStream_t st) override {
         cudaStreamSynchronize(st);

@@ -30,6 +30,7 @@
 #include "comm.cuh"
 #include "k_dist.cuh"
 #include "fabric.cuh"
+#include "k_nmi.cuh"
 
 #define GALA_VERSION "gala-b200 0.1 (sm_100a)"
 
@@ -143,6 +144,7 @@ struct gala_graph_s {
     int check_mismatch = 0;   // check mode: final N on G0 differs from the last level's N
     // multi-GPU (one process per GPU)
     struct DistInfo* di = nullptr;
+    bool fab_host_bar = false;   // = di->host_bar (fabric barriers on the host: loopback ranks on one device)
     int sync_mode = 0;
     std::vector<long long> dbounds0;   // level-0 owned ranges of all ranks
     struct Work* wk = nullptr;   // persistent run workspace (sized for level 0, reused by every run)
@@ -877,7 +879,7 @@ template <typename Issue, typename PreLaunch = NoHook>
 static void level_loop(gala_graph_s* g, Work& wk, std::vector<IterLog>& out, bool single_ok, Timer& tm, Issue issue,
                        PreLaunch pre_launch = PreLaunch()) {
     cudaStream_t st = g->stream;
-    const bool stepwise = !g->opt_cuda_graph || g->opt_trace >= 2 || g->opt_timing;
+    const bool stepwise = !g->opt_cuda_graph || g->opt_trace >= 2 || g->opt_timing || g->fab_host_bar;
     out.clear();
     // first iteration of a level: singleton fast path when rows hold distinct columns
     bool first_single = single_ok && g->opt_singleton;
@@ -1730,6 +1732,7 @@ struct DistInfo {
     std::vector<void*> peers;
     FabDev fab = {};
     bool failed = false;   // a run ended in an error: peers may still touch the region
+    bool host_bar = false; // fabric barriers on the host (ranks sharing one device: loopback world > 1)
 };
 
 // Symmetric region of a rank (cudaMalloc: CUDA IPC needs it), byte offsets:
@@ -2137,6 +2140,20 @@ static void dist_level_setup(gala_graph_s* g, const DevCSR& G, const std::vector
     L.it_chunk = dalloc<int32_t>(icap, st);
 }
 
+// Fabric barrier: the device-side k_fab_barrier when every rank has its own GPU; ranks that
+// share one device (loopback test backend) never spin in a kernel on each other -- each syncs
+// its stream (its peer stores are complete and visible on the shared device) and they meet on
+// the host.  The level loop then runs stepwise (no CUDA graph) for those ranks.
+static void fab_barrier(gala_graph_s* g, const DistLevel& L, cudaStream_t st) {
+    if (g->di->host_bar) {
+        CK(cudaStreamSynchronize(st));
+        g->di->comm->host_barrier();
+        return;
+    }
+    k_fab_barrier<<<1, 32, 0, st>>>(L.f);
+    CKL();
+}
+
 // one device-resident iteration of the fabric backend (see fabric.cuh for the sequence)
 template <int M, bool UNIT>
 static void dist_iteration_fab(gala_graph_s* g, Work& wk, const DevCSR& G, const DistLevel& L,
@@ -2162,8 +2179,7 @@ static void dist_iteration_fab(gala_graph_s* g, Work& wk, const DevCSR& G, const
     CKL();
     k_fab_push_fix<<<g->num_sms, 256, 0, st>>>(L.f, L.lmoves, L.lcount, wk.carry);
     CKL();
-    k_fab_barrier<<<1, 32, 0, st>>>(L.f);
-    CKL();
+    fab_barrier(g, L, st);
     tm.end(KC_XCHG, e);
     e = tm.begin();
     k_fab_apply<<<grid_for(n, 256, big), 256, 0, st>>>(L.f, wk.carry, wk.ctr, wk.C, wk.Sig, wk.size, wk.d, wk.stamp,
@@ -2189,8 +2205,7 @@ static void dist_iteration_fab(gala_graph_s* g, Work& wk, const DevCSR& G, const
     CKL();
     k_fab_scal<<<1, 32, 0, st>>>(L.f, wk.carry, wk.ctr, L.lcount, 0);
     CKL();
-    k_fab_barrier<<<1, 32, 0, st>>>(L.f);
-    CKL();
+    fab_barrier(g, L, st);
     k_fab_finish<<<1, 32, 0, st>>>(L.f, wk.ctr, wk.carry, L.lcount, (long long)(qW128 >> 64), (ull)qW128, (long long)p,
                                    (long long)(T >> 64), (ull)T, 1, wk.log, wk.log_cap, g->opt_max_iters, cond);
     CKL();
@@ -2208,8 +2223,7 @@ static void dist_level_start_fab(gala_graph_s* g, Work& wk, const DevCSR& G, con
     CKL();
     k_fab_scal<<<1, 32, 0, st>>>(L.f, wk.carry, wk.ctr, L.lcount, 1);
     CKL();
-    k_fab_barrier<<<1, 32, 0, st>>>(L.f);
-    CKL();
+    fab_barrier(g, L, st);
     k_fab_finish<<<1, 32, 0, st>>>(L.f, wk.ctr, wk.carry, L.lcount, (long long)(qW128 >> 64), (ull)qW128, (long long)p,
                                    0, 0, 0, nullptr, 0, 0, 0ull);
     CKL();
@@ -3010,6 +3024,51 @@ gala_status gala_partition_ranges(int64_t n, const int64_t* row_ptr, int world, 
     return GALA_OK;
 }
 
+gala_status gala_nmi_device(const int32_t* d_x, const int32_t* d_y, int64_t n, int device, uintptr_t stream,
+                            double* out) {
+    if (!out || n < 0 || (n > 0 && (!d_x || !d_y))) return set_err(GALA_E_INVALID, "null argument or n < 0");
+    if (n >= ((int64_t)1 << 31)) return set_err(GALA_E_INVALID, "n >= 2^31");
+    if (n == 0) { *out = 1.0; return GALA_OK; }
+    API_BEGIN
+    CK(cudaSetDevice(device));
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    long long cap = 64;
+    while (cap < 2 * n) cap <<= 1;
+    unsigned* hist = nullptr;
+    ull* keys = nullptr;
+    unsigned* cnt = nullptr;
+    double* part = nullptr;
+    int* bad = nullptr;
+    CK(cudaMallocAsync(&hist, sizeof(unsigned) * 2 * (size_t)n, st));
+    CK(cudaMallocAsync(&keys, sizeof(ull) * (size_t)cap, st));
+    CK(cudaMallocAsync(&cnt, sizeof(unsigned) * (size_t)cap, st));
+    CK(cudaMallocAsync(&part, sizeof(double) * (3 * NMI_GRID + 1), st));
+    CK(cudaMallocAsync(&bad, sizeof(int), st));
+    CK(cudaMemsetAsync(hist, 0, sizeof(unsigned) * 2 * (size_t)n, st));
+    CK(cudaMemsetAsync(keys, 0xff, sizeof(ull) * (size_t)cap, st));
+    CK(cudaMemsetAsync(cnt, 0, sizeof(unsigned) * (size_t)cap, st));
+    CK(cudaMemsetAsync(bad, 0, sizeof(int), st));
+    k_nmi_count<<<NMI_GRID, NMI_BT, 0, st>>>(n, d_x, d_y, hist, hist + n, keys, cnt, (ull)(cap - 1), bad);
+    CKL();
+    k_nmi_terms<<<NMI_GRID, NMI_BT, 0, st>>>(n, hist, hist + n, keys, cnt, cap, part);
+    CKL();
+    k_nmi_final<<<1, 32, 0, st>>>(part, NMI_GRID, part + 3 * NMI_GRID);
+    CKL();
+    int hbad = 0;
+    double res = 0;
+    CK(cudaMemcpyAsync(&hbad, bad, sizeof(int), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(&res, part + 3 * NMI_GRID, sizeof(double), cudaMemcpyDeviceToHost, st));
+    CK(cudaFreeAsync(hist, st));
+    CK(cudaFreeAsync(keys, st));
+    CK(cudaFreeAsync(cnt, st));
+    CK(cudaFreeAsync(part, st));
+    CK(cudaFreeAsync(bad, st));
+    CK(cudaStreamSynchronize(st));
+    if (hbad) return set_err(GALA_E_INVALID, "gala_nmi_device: a label outside [0, n)");
+    *out = res;
+    API_END
+}
+
 gala_status gala_nccl_unique_id(void* out128) {
     if (!out128) return set_err(GALA_E_INVALID, "null argument");
     if (!nccl_api().load()) return set_err(GALA_E_NCCL, "libnccl.so.2 could not be loaded");
@@ -3045,8 +3104,8 @@ gala_status gala_graph_from_csr_dist(const void* uid128, int rank, int world, in
     const bool loop = memcmp(uid128, "GALALOOP", 8) == 0;
     if (loop && world > 1) {
         // loopback ranks share one CUDA context: a kernel loaded lazily on first use waits for the
-        // context to go idle, which a peer's fabric barrier kernel (spinning for this rank) never
-        // does -- the ranks would deadlock until the barrier timeout
+        // context to go idle, which another rank's long-running work on the shared device can
+        // delay indefinitely (the fabric meets on the host for these ranks, see fab_barrier)
         const char* ml = getenv("CUDA_MODULE_LOADING");
         if (!ml || strcmp(ml, "EAGER") != 0)
             return set_err(GALA_E_INVALID, "loopback with world > 1 needs CUDA_MODULE_LOADING=EAGER (set before CUDA starts)");
@@ -3061,6 +3120,8 @@ gala_status gala_graph_from_csr_dist(const void* uid128, int rank, int world, in
         g->di = new DistInfo();
         try {
             g->di->comm = comm_for(uid128, rank, world, loop);
+            g->di->host_bar = !g->di->comm->device_barrier_ok();
+            g->fab_host_bar = g->di->host_bar;
         } catch (CommError& e) {
             set_err(GALA_E_NCCL, "%s", e.msg.c_str());
             throw GalaError{GALA_E_NCCL};

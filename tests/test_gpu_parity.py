@@ -12,7 +12,6 @@ import pytest
 import graphgen as gg
 import oracle
 import paper_conf_ppopp_wangllwm00z25_b200 as gala
-import quality
 
 pytestmark = pytest.mark.gpu
 
@@ -284,20 +283,47 @@ def test_friendster_shape_full_parity():
     assert_parity(gg.make("friendster_q"), labels=False)
 
 
+def _dev(a):
+    import torch
+    return torch.as_tensor(np.ascontiguousarray(a, dtype=np.int32)).cuda()
+
+
 @pytest.mark.gpu
 def test_nmi_vs_planted_partition():
     """NEXT #4 (Table 4 style): NMI of the GPU result against the LFR planted partition, computed
-    on the device, equals the oracle's fp64 NMI of the same labels; and the planted partition
-    itself has NMI 1."""
+    by the library's kernels (gala_nmi_device), equals the oracle's fp64 NMI of the same labels;
+    the planted partition itself has NMI 1."""
     from oracle.nmi import nmi
     g = gg.make("lfr_small")
     with gala.Graph.from_graph(g) as h:
         h.run()
         lab = h.communities()
-    got = quality.nmi_device(lab, g.truth)
+    got = gala.nmi(_dev(lab), _dev(g.truth))
     assert got == pytest.approx(nmi(lab, g.truth), abs=1e-9)
-    assert quality.nmi_device(g.truth, g.truth) == pytest.approx(1.0, abs=1e-12)
+    assert gala.nmi(_dev(g.truth), _dev(g.truth)) == pytest.approx(1.0, abs=1e-12)
     assert 0.0 <= got <= 1.0 + 1e-12
+
+
+@pytest.mark.gpu
+def test_nmi_kernel_cases():
+    """gala_nmi_device against the oracle on random partitions (sizes spanning several blocks and
+    a ragged tail), the hand example of tests/test_oracle_nmi.py, product partitions (0), the
+    single-cluster conventions, n = 0, and a label outside [0, n) (rejected)."""
+    import math
+    from oracle.nmi import nmi
+    rng = np.random.default_rng(5)
+    for n, kx, ky in [(1, 1, 1), (7, 3, 2), (1000, 10, 37), (200003, 5000, 300), (1 << 20, 60000, 60000)]:
+        x = rng.integers(0, kx, n)
+        y = np.where(rng.random(n) < 0.6, x % ky, rng.integers(0, ky, n))
+        assert gala.nmi(_dev(x), _dev(y)) == pytest.approx(nmi(x, y), abs=1e-9), (n, kx, ky)
+    want = (2.0 / 3.0) * math.log(2) / math.sqrt(math.log(2) * math.log(3))
+    assert gala.nmi(_dev([0, 0, 0, 1, 1, 1]), _dev([0, 0, 1, 1, 2, 2])) == pytest.approx(want, rel=1e-13)
+    assert gala.nmi(_dev(np.repeat(np.arange(4), 6)), _dev(np.tile(np.arange(6), 4))) == pytest.approx(0.0, abs=1e-12)
+    assert gala.nmi(_dev([3] * 10), _dev([1] * 10)) == 1.0
+    assert gala.nmi(_dev([3] * 10), _dev(np.arange(10))) == 0.0
+    assert gala.nmi(_dev([]), _dev([])) == 1.0
+    with pytest.raises(gala.GalaError):
+        gala.nmi(_dev([0, 5]), _dev([0, 1]))
 
 
 @pytest.mark.gpu
