@@ -380,9 +380,21 @@ static int64_t lfr_rewire(int64_t ne, int64_t n_int, int64_t* src, int64_t* dst,
  * removes them), membership[n] (ground truth, permuted ids).
  * Two-call protocol: if out_src == NULL returns the edge count upper bound.
  */
-int64_t gg_lfr_ex(int64_t n, double avg_k, int64_t kmax, double tau1, double tau2,
-                  int64_t cmin, int64_t cmax, double mu, uint64_t seed, int fit_frac, double alpha,
-                  int rewire, int64_t* out_src, int64_t* out_dst, int64_t* membership, int64_t* out_kmin) {
+/* LFR plan (steps 1-4 of gg_lfr_ex): degrees k, and unless degrees_only, community sizes, internal
+   degrees kin, the placement comm and the per-community member lists (coff, mem).  Shared by
+   gg_lfr_ex and the memory-lean gg_lfr_csr. */
+typedef struct {
+    int64_t kmin, stubs_total, nc, maxc;
+    int64_t *k, *kin, *csize, *fill, *comm, *coff, *mem;
+} lfr_plan_t;
+
+static void lfr_plan_free(lfr_plan_t* P) {
+    free(P->k); free(P->kin); free(P->csize); free(P->fill); free(P->comm); free(P->coff); free(P->mem);
+}
+
+static void lfr_plan(int64_t n, double avg_k, int64_t kmax, double tau1, double tau2, int64_t cmin, int64_t cmax,
+                     double mu, uint64_t seed, int fit_frac, double alpha, int degrees_only, lfr_plan_t* P) {
+    memset(P, 0, sizeof(*P));
     /* 1. degrees */
     int64_t best_kmin = 1; double best_err = 1e300;
     for (int64_t km = 1; km < kmax; ++km) {
@@ -415,14 +427,16 @@ int64_t gg_lfr_ex(int64_t n, double avg_k, int64_t kmax, double tau1, double tau
     } else {
         tk = pl_table(kmin, kmax, tau1);
     }
-    if (out_kmin) *out_kmin = kmin;
+    P->kmin = kmin;
     int64_t* k = (int64_t*)malloc((size_t)n * sizeof(int64_t));
     #pragma omp parallel for
     for (int64_t i = 0; i < n; ++i) k[i] = pl_draw(tk, kmin, kmax, rng_unit(seed, 1, (uint64_t)i));
     free(tk);
     int64_t stubs_total = 0;
     for (int64_t i = 0; i < n; ++i) stubs_total += k[i];
-    if (!out_src) { free(k); return stubs_total / 2 + n; }
+    P->k = k;
+    P->stubs_total = stubs_total;
+    if (degrees_only) return;
 
     /* 2. community sizes */
     double* tc = pl_table(cmin, cmax, tau2);
@@ -498,6 +512,19 @@ int64_t gg_lfr_ex(int64_t n, double avg_k, int64_t kmax, double tau1, double tau
         for (int64_t i = 0; i < n; ++i) mem[cur[comm[i]]++] = i;
         free(cur);
     }
+    P->kin = kin; P->csize = csize; P->fill = fill; P->comm = comm; P->coff = coff; P->mem = mem;
+    P->nc = nc; P->maxc = maxc;
+}
+
+int64_t gg_lfr_ex(int64_t n, double avg_k, int64_t kmax, double tau1, double tau2,
+                  int64_t cmin, int64_t cmax, double mu, uint64_t seed, int fit_frac, double alpha,
+                  int rewire, int64_t* out_src, int64_t* out_dst, int64_t* membership, int64_t* out_kmin) {
+    lfr_plan_t P;
+    lfr_plan(n, avg_k, kmax, tau1, tau2, cmin, cmax, mu, seed, fit_frac, alpha, out_src == NULL, &P);
+    if (out_kmin) *out_kmin = P.kmin;
+    if (!out_src) { lfr_plan_free(&P); return P.stubs_total / 2 + n; }
+    int64_t *k = P.k, *kin = P.kin, *comm = P.comm, *coff = P.coff, *mem = P.mem;
+    const int64_t nc = P.nc;
 
     /* 5a. internal wiring: per community stub shuffle */
     int64_t* istub_off = (int64_t*)calloc((size_t)nc + 1, sizeof(int64_t));
@@ -582,7 +609,7 @@ int64_t gg_lfr_ex(int64_t n, double avg_k, int64_t kmax, double tau1, double tau
         #pragma omp parallel for
         for (int64_t i = 0; i < n; ++i) membership[perm[i]] = comm[i];
     }
-    free(perm); free(k); free(kin); free(csize); free(fill); free(comm); free(coff); free(mem); free(istub_off);
+    free(perm); lfr_plan_free(&P); free(istub_off);
     return ne;
 }
 
@@ -591,4 +618,159 @@ int64_t gg_lfr(int64_t n, double avg_k, int64_t kmax, double tau1, double tau2,
                int64_t cmin, int64_t cmax, double mu, uint64_t seed,
                int64_t* out_src, int64_t* out_dst, int64_t* membership, int64_t* out_kmin) {
     return gg_lfr_ex(n, avg_k, kmax, tau1, tau2, cmin, cmax, mu, seed, 0, 1.0, 0, out_src, out_dst, membership, out_kmin);
+}
+
+/* ---------------------------------------------------------------------------------------------
+ * Memory-lean LFR-style generator straight to CSR, for graphs whose edge list does not fit the
+ * host twice over (the Friendster shape: 65.6M vertices, ~1.8B edges).
+ * Same plan as gg_lfr_ex (degrees, community sizes, placement, per-community internal wiring),
+ * but the external stubs are paired through a counter-based random bijection of the stub
+ * sequence instead of a sort by random key: stub j of the shuffled sequence is pi(j), pi a
+ * 4-round Feistel permutation of [0, 2^2h) restricted to [0, S) by cycle walking, and pair e is
+ * (pi(2e), pi(2e+1)).  Every pair is a pure function of (seed, e), so the O(S) stub arrays and
+ * their sort buffers are never built.  External pairs inside one community, self pairs and
+ * duplicate edges are dropped (no re-pairing, no rewiring; realised counts reported).
+ * Peak host memory ~ 8 B per edge (packed edge list) + 4 B per CSR entry + O(n).
+ * Returns nnz; *out_col receives a malloc'd int32[nnz] (free with gg_free), row_ptr is int64[n+1].
+ * -------------------------------------------------------------------------------------------*/
+static inline uint64_t feistel_perm(uint64_t x, uint64_t S, int half, uint64_t seed) {
+    const uint64_t mask = (1ull << half) - 1;
+    do {
+        uint64_t L = x >> half, R = x & mask;
+        for (int r = 0; r < 4; ++r) {
+            const uint64_t F = mix64(R ^ (seed * 0x9E3779B97F4A7C15ull) ^ ((uint64_t)(r + 1) << 56)) & mask;
+            const uint64_t t = L ^ F;
+            L = R;
+            R = t;
+        }
+        x = (L << half) | R;
+    } while (x >= S);   /* cycle walking: a bijection of [0, S) */
+    return x;
+}
+
+static int64_t stub_owner(const int64_t* off, int64_t n, uint64_t s) {   /* largest v with off[v] <= s */
+    int64_t lo = 0, hi = n - 1;
+    while (lo < hi) {
+        const int64_t mid = (lo + hi + 1) / 2;
+        if ((uint64_t)off[mid] <= s) lo = mid; else hi = mid - 1;
+    }
+    return lo;
+}
+
+static int cmp_i32(const void* a, const void* b) {
+    const int32_t x = *(const int32_t*)a, y = *(const int32_t*)b;
+    return (x > y) - (x < y);
+}
+
+void gg_free(void* p) { free(p); }
+
+int64_t gg_lfr_csr(int64_t n, double avg_k, int64_t kmax, double tau1, double tau2, int64_t cmin, int64_t cmax,
+                   double mu, uint64_t seed, int64_t* row_ptr, int32_t** out_col, int64_t* membership,
+                   int64_t* out_kmin, int64_t* out_stats /* [internal edges, external pairs, dropped] */) {
+    lfr_plan_t P;
+    lfr_plan(n, avg_k, kmax, tau1, tau2, cmin, cmax, mu, seed, 0, 1.0, 0, &P);
+    if (out_kmin) *out_kmin = P.kmin;
+    int64_t *k = P.k, *kin = P.kin, *comm = P.comm, *coff = P.coff, *mem = P.mem;
+    const int64_t nc = P.nc;
+    /* internal edges per community */
+    int64_t* ioff = (int64_t*)calloc((size_t)nc + 1, sizeof(int64_t));
+    for (int64_t j = 0; j < nc; ++j) {
+        int64_t s = 0;
+        for (int64_t t = coff[j]; t < coff[j + 1]; ++t) s += kin[mem[t]];
+        ioff[j + 1] = ioff[j] + s / 2;
+    }
+    const int64_t n_int = ioff[nc];
+    int64_t* xoff = (int64_t*)malloc((size_t)(n + 1) * sizeof(int64_t));   /* external stub prefix */
+    xoff[0] = 0;
+    for (int64_t i = 0; i < n; ++i) xoff[i + 1] = xoff[i] + (k[i] - kin[i]);
+    const uint64_t S = (uint64_t)xoff[n];
+    const int64_t np = (int64_t)(S / 2);
+    int half = 1;
+    while (half < 32 && (1ull << (2 * half)) < S) ++half;
+    int64_t* perm = (int64_t*)malloc((size_t)n * sizeof(int64_t));
+    gg_random_permutation(n, seed, 8, perm);
+    uint64_t* E = (uint64_t*)malloc((size_t)(n_int + np + 1) * sizeof(uint64_t));   /* (u << 32 | v), ids permuted */
+    const uint64_t DROP = ~0ull;
+    /* 5a. internal wiring (per-community Fisher-Yates of its stubs, as gg_lfr_ex) */
+    #pragma omp parallel
+    {
+        int64_t bufcap = 0; int64_t* buf = NULL;
+        #pragma omp for schedule(dynamic, 16)
+        for (int64_t j = 0; j < nc; ++j) {
+            int64_t s = 0;
+            for (int64_t t = coff[j]; t < coff[j + 1]; ++t) s += kin[mem[t]];
+            if (s > bufcap) { bufcap = s; buf = (int64_t*)realloc(buf, (size_t)bufcap * sizeof(int64_t)); }
+            int64_t p = 0;
+            for (int64_t t = coff[j]; t < coff[j + 1]; ++t)
+                for (int64_t q = 0; q < kin[mem[t]]; ++q) buf[p++] = mem[t];
+            for (int64_t i = s - 1; i > 0; --i) {
+                int64_t r = (int64_t)(rng_u64(seed, 4, ((uint64_t)j << 32) ^ (uint64_t)i) % (uint64_t)(i + 1));
+                int64_t tmp = buf[i]; buf[i] = buf[r]; buf[r] = tmp;
+            }
+            for (int64_t e = 0; e < s / 2; ++e) {
+                const int64_t u = buf[2 * e], v = buf[2 * e + 1];
+                E[ioff[j] + e] = u == v ? DROP : ((uint64_t)perm[u] << 32) | (uint64_t)perm[v];
+            }
+        }
+        free(buf);
+    }
+    /* 5b. external pairs through the Feistel bijection */
+    int64_t dropped_x = 0;
+    #pragma omp parallel for reduction(+ : dropped_x) schedule(static, 1 << 16)
+    for (int64_t e = 0; e < np; ++e) {
+        const uint64_t a = feistel_perm(2 * (uint64_t)e, S, half, seed ^ 0x5A5Aull);
+        const uint64_t b = feistel_perm(2 * (uint64_t)e + 1, S, half, seed ^ 0x5A5Aull);
+        const int64_t u = stub_owner(xoff, n, a), v = stub_owner(xoff, n, b);
+        if (u == v || comm[u] == comm[v]) { E[n_int + e] = DROP; ++dropped_x; continue; }
+        E[n_int + e] = ((uint64_t)perm[u] << 32) | (uint64_t)perm[v];
+    }
+    const int64_t m = n_int + np;
+    if (membership) {
+        #pragma omp parallel for
+        for (int64_t i = 0; i < n; ++i) membership[perm[i]] = comm[i];
+    }
+    free(xoff); free(perm); free(ioff); lfr_plan_free(&P);
+    /* 6. CSR: count, scatter both directions, sort + dedup every row, compact */
+    for (int64_t v = 0; v <= n; ++v) row_ptr[v] = 0;
+    #pragma omp parallel for
+    for (int64_t e = 0; e < m; ++e) {
+        if (E[e] == DROP) continue;
+        __atomic_fetch_add(&row_ptr[(E[e] >> 32) + 1], 1, __ATOMIC_RELAXED);
+        __atomic_fetch_add(&row_ptr[(E[e] & 0xFFFFFFFFull) + 1], 1, __ATOMIC_RELAXED);
+    }
+    for (int64_t v = 0; v < n; ++v) row_ptr[v + 1] += row_ptr[v];
+    const int64_t tot = row_ptr[n];
+    int32_t* col = (int32_t*)malloc((size_t)(tot + 1) * sizeof(int32_t));
+    int64_t* cur = (int64_t*)malloc((size_t)n * sizeof(int64_t));
+    memcpy(cur, row_ptr, (size_t)n * sizeof(int64_t));
+    #pragma omp parallel for
+    for (int64_t e = 0; e < m; ++e) {
+        if (E[e] == DROP) continue;
+        const int64_t u = (int64_t)(E[e] >> 32), v = (int64_t)(E[e] & 0xFFFFFFFFull);
+        col[__atomic_fetch_add(&cur[u], 1, __ATOMIC_RELAXED)] = (int32_t)v;
+        col[__atomic_fetch_add(&cur[v], 1, __ATOMIC_RELAXED)] = (int32_t)u;
+    }
+    free(E);
+    /* per row: sort, unique (cur[v] = its distinct count) */
+    #pragma omp parallel for schedule(dynamic, 4096)
+    for (int64_t v = 0; v < n; ++v) {
+        int32_t* r = col + row_ptr[v];
+        const int64_t len = row_ptr[v + 1] - row_ptr[v];
+        qsort(r, (size_t)len, sizeof(int32_t), cmp_i32);
+        int64_t w = 0;
+        for (int64_t i = 0; i < len; ++i) if (i == 0 || r[i] != r[i - 1]) r[w++] = r[i];
+        cur[v] = w;
+    }
+    int64_t nnz = 0;   /* compact left to right (new start <= old start: memmove is safe in order) */
+    for (int64_t v = 0; v < n; ++v) {
+        const int64_t b = row_ptr[v];
+        if (nnz != b) memmove(col + nnz, col + b, (size_t)cur[v] * sizeof(int32_t));
+        row_ptr[v] = nnz;
+        nnz += cur[v];
+    }
+    row_ptr[n] = nnz;
+    free(cur);
+    *out_col = (int32_t*)realloc(col, (size_t)(nnz + 1) * sizeof(int32_t));
+    if (out_stats) { out_stats[0] = n_int; out_stats[1] = np; out_stats[2] = m - nnz / 2; }
+    return nnz;
 }

@@ -446,6 +446,7 @@ struct Work {
     int32_t *C = nullptr, *size = nullptr, *stamp = nullptr, *mv_v = nullptr, *mv_old = nullptr, *mv_chunk = nullptr, *nextC = nullptr;
     QRec* queues = nullptr;
     int32_t* ckey = nullptr;   // level-0 per-entry neighbour community
+    int2* cst = nullptr;       // (C[v], stamp[v]) pairs: one 8-byte gather per entry in k_dp_delta
     int64_t *Sig = nullptr, *d = nullptr, *s = nullptr, *dp = nullptr;
     bool s_zero = false;   // this level has no self-loops: k_reduce skips s (level 0 of a loop-free graph)
     const int64_t* s_live() const { return s_zero ? nullptr : s; }
@@ -475,7 +476,7 @@ struct Work {
         for (auto& e : ev) if (e) { cudaEventDestroy(e); e = nullptr; }
         dfree(C, st); dfree(size, st); dfree(stamp, st); dfree(mv_v, st); dfree(mv_old, st); dfree(mv_chunk, st);
         dfree(rmflag, st); dfree(smflag, st); dfree(chg, st); dfree(nextC, st);
-        dfree(queues, st); dfree(ckey, st); dfree(Sig, st); dfree(d, st); dfree(s, st); dfree(dp, st); dfree(ctr, st);
+        dfree(queues, st); dfree(ckey, st); dfree(cst, st); dfree(Sig, st); dfree(d, st); dfree(s, st); dfree(dp, st); dfree(ctr, st);
         dfree(carry, st); dfree(log, st); dfree(part_dc, st); dfree(part_min, st); dfree(part_s2, st);
         dfree(gkeys, st); dfree(gvals, st); dfree(glist, st);
         dfree(hw.keys, st); dfree(hw.vals, st); dfree(hw.list, st); dfree(hw.pref, st); dfree(hw.toff, st);
@@ -837,12 +838,12 @@ static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, typename
     launch_decide<M, UNIT>(g, wk, G, qW, p, tm, maxdeg, idbits, single);
     e = tm.begin();
     k_apply<<<grid_for(n, AP_BT, big), AP_BT, 0, st>>>(wk.ctr, wk.queues, wk.qcap, wk.nextC, wk.C, wk.Sig, wk.size,
-                                                       wk.dp, wk.stamp, wk.carry, wk.mv_v, wk.mv_old, wk.mv_chunk, ps, wk.icap);
+                                                       wk.dp, wk.stamp, wk.cst, wk.carry, wk.mv_v, wk.mv_old, wk.mv_chunk, ps, wk.icap);
     CKL();
     tm.end(KC_APPLY, e);
     e = tm.begin();
     const bool ck = use_ckey(g, wk, G);
-    k_dp_delta<UNIT><<<big, 256, 0, st>>>(wk.ctr, G.rp, G.col, G.w, wk.C, wk.mv_v, wk.mv_old, wk.mv_chunk, wk.stamp, wk.dp,
+    k_dp_delta<UNIT><<<big, 256, 0, st>>>(wk.ctr, G.rp, G.col, G.w, wk.C, wk.cst, wk.mv_v, wk.mv_old, wk.mv_chunk, wk.stamp, wk.dp,
                                           wk.carry, G.nnz, g->opt_delta, 1, g->opt_delta_den, ck ? wk.ckey : nullptr,
                                           nullptr, ps.rmflag, n, wk.icap);
     CKL();
@@ -1414,6 +1415,7 @@ static void ensure_workspace(gala_graph_s* g) {
             wk.C = dalloc<int32_t>(wk.ncap, st);
             wk.size = dalloc<int32_t>(wk.ncap, st);
             wk.stamp = dalloc<int32_t>(wk.ncap, st);
+            wk.cst = dalloc<int2>(wk.ncap, st);
             // delta-update items: one per light mover + one per DCH-entry chunk of a heavy one
             const size_t icap = (size_t)wk.ncap + (size_t)(g->nnz0 / DCH) + 1;
             wk.icap = (long long)icap;
@@ -1560,7 +1562,7 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
             prepare_level_tables(g, wk, cur, maxdeg);
             // a1: level init + starting numerator
             cudaEvent_t e = tm.begin();
-            k_level_init<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.d, wk.C, wk.Sig, wk.size, wk.dp, wk.stamp,
+            k_level_init<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.d, wk.C, wk.Sig, wk.size, wk.dp, wk.stamp, wk.cst,
                                                                  wk.carry, prune_state(g, wk));
             CKL();
             if (first_level) {
@@ -2312,7 +2314,7 @@ static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_level
                 wk.queues = dalloc<QRec>((size_t)wk.qcap * (NBINS / 2), st);
             }
             prepare_level_tables(g, wk, cur, maxdeg);
-            k_level_init<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.d, wk.C, wk.Sig, wk.size, wk.dp, wk.stamp,
+            k_level_init<<<grid_for(nl, 256, big), 256, 0, st>>>((int)nl, wk.d, wk.C, wk.Sig, wk.size, wk.dp, wk.stamp, wk.cst,
                                                                  wk.carry, prune_state(g, wk));
             CKL();
             if (level == 0) CK(cudaMemcpyAsync(g->lab, wk.C, sizeof(int32_t) * n0, cudaMemcpyDeviceToDevice, st));

@@ -211,6 +211,9 @@ __device__ __forceinline__ unsigned decide_sub_bin(QView queue, int bin, const D
 #ifndef GALA_WARP_SCAN
 #define GALA_WARP_SCAN 0   // warp128: evaluate by scanning the 256-slot table instead of keeping a distinct list
 #endif
+#ifndef GALA_WARP_KV
+#define GALA_WARP_KV 1   // warp kernels: packed 64-bit (key, sum) table slots, batched list evaluation
+#endif
 #ifndef GALA_WARP_PREFETCH
 #define GALA_WARP_PREFETCH 1   // warp128: next vertex's row loaded during this one's evaluation
 #endif
@@ -317,6 +320,30 @@ __device__ __forceinline__ int ht_insert4(int c, VT wt, int* keys, VT* vals, uns
     return -1;
 }
 
+// Packed form for 32-bit aggregates: one 64-bit word per slot, key in the high half, the
+// weight sum in the low half (KV_EMPTY = key -1, sum 0).  A fresh key is created with ONE
+// 64-bit CAS that also stores its first sum; an existing key takes a native 32-bit add on the
+// low half (the sum never reaches 2^32: it is at most W < 2^31 on these levels).  Same
+// slot-wise linear probe, hence the same table contents as ht_insert.
+#define KV_EMPTY 0xFFFFFFFF00000000ull
+__device__ __forceinline__ int kv_insert(int c, unsigned wt, ull* tbl, unsigned mask, unsigned h, int win, bool* fresh) {
+    *fresh = false;
+    const ull mine = ((ull)(unsigned)c << 32) | wt;
+    for (int t = 0; t < win; ++t) {
+        ull k = *(volatile ull*)&tbl[h];
+        if (k == KV_EMPTY) {
+            k = atomicCAS(&tbl[h], KV_EMPTY, mine);
+            if (k == KV_EMPTY) { *fresh = true; return (int)h; }
+        }
+        if ((int)(k >> 32) == c) {
+            atomicAdd(reinterpret_cast<unsigned*>(&tbl[h]), wt);   // low half (little endian)
+            return (int)h;
+        }
+        h = (h + 1) & mask;
+    }
+    return -1;
+}
+
 // ---------------------------------------------------------------------------
 // a4 (mid degree): one warp per vertex (deg <= MAXDEG), per-warp shared-memory
 // table of 2*MAXDEG slots (load <= 1/2, never spills) and a distinct-key list.
@@ -363,7 +390,11 @@ __global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB, MAXDEG <= 1
     int* keys = reinterpret_cast<int*>(base + (size_t)WCAP * sizeof(VT));
     short* list = reinterpret_cast<short*>(base + (size_t)WCAP * (sizeof(VT) + sizeof(int)));
     int* cnt = reinterpret_cast<int*>(base + (size_t)WCAP * (sizeof(VT) + sizeof(int)) + (size_t)MAXDEG * sizeof(short));
-    for (int j = gl; j < WCAP; j += GW) { keys[j] = -1; vals[j] = 0; }
+    // KV: packed 64-bit (key, 32-bit sum) slots over the same bytes as keys + vals
+    constexpr bool KV = GALA_WARP_KV && sizeof(VT) == 4 && !(GALA_WARP_SCAN && MAXDEG <= 128);
+    ull* tbl = reinterpret_cast<ull*>(base);
+    if (KV) { for (int j = gl; j < WCAP; j += GW) tbl[j] = KV_EMPTY; }
+    else { for (int j = gl; j < WCAP; j += GW) { keys[j] = -1; vals[j] = 0; } }
     if (gl == 0) *cnt = 0;
     __syncwarp();
     const long long nwarps = (long long)gridDim.x * SM::WPB;
@@ -432,10 +463,12 @@ __global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB, MAXDEG <= 1
                 const VT sum = UNIT ? (VT)__popc(peers) : group_sum(peers, cc[k] >= 0 ? ww[k] : (VT)0, scratch);
                 bool fresh = false;
                 int slot = -1;
-                if (cc[k] >= 0 && lane == __ffs(peers) - 1)
-                    slot = MAXDEG > 128   // bucketed probing pays only in the larger tables (measured)
+                if (cc[k] >= 0 && lane == __ffs(peers) - 1) {
+                    if (KV) slot = kv_insert(cc[k], (unsigned)sum, tbl, WMASK, hash_slot(cc[k], WMASK), WCAP, &fresh);
+                    else slot = MAXDEG > 128   // bucketed probing pays only in the larger tables (measured)
                                ? ht_insert4<VT, true>(cc[k], sum, keys, vals, WMASK, hash_slot(cc[k], WMASK), WCAP, &fresh)
                                : ht_insert<VT>(cc[k], sum, keys, vals, WMASK, hash_slot(cc[k], WMASK), WCAP, &fresh);
+                }
                 if (!SCAN) append_fresh<short>(fresh, slot, gmask, cnt, list);
             }
         }
@@ -475,7 +508,32 @@ __global__ void __launch_bounds__(32 * WarpSmem<GW, MAXDEG, M>::WPB, MAXDEG <= 1
         }
         const int m = SCAN ? 0 : *cnt;
         my_k += (!SCAN && gl == 0) ? m : 0;
-        for (int t0 = gl; t0 < m; t0 += GW * CH) {
+        // KV: the group's distinct list in batches of 4 slots per lane, the batch count bounded
+        // by the group's own list length (no predicated-off batches)
+        for (int b0 = 0; KV && b0 < m; b0 += GW * 4) {
+            int cs[4];
+            unsigned ws[4];
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                cs[k] = -1;
+                ws[k] = 0;
+                const int t = b0 + gl + GW * k;
+                if (b0 + GW * k < m && t < m) {
+                    const int slot = list[t];
+                    const ull kv = tbl[slot];
+                    tbl[slot] = KV_EMPTY;
+                    cs[k] = (int)(kv >> 32);
+                    ws[k] = (unsigned)kv;
+                }
+            }
+            long long sg[4];
+#pragma unroll
+            for (int k = 0; k < 4; ++k) sg[k] = cs[k] >= 0 ? a.Sig[cs[k]] : 0;
+#pragma unroll
+            for (int k = 0; k < 4; ++k)
+                if (cs[k] >= 0) best.offer(gain<ST>(qW, p, (long long)ws[k], sg[k], dv), cs[k]);
+        }
+        for (int t0 = gl; !KV && t0 < m; t0 += GW * CH) {
             int cs[CH];
             long long ws[CH];
 #pragma unroll
@@ -701,6 +759,7 @@ __global__ void BLOCK_LB(BT) k_decide_block(QView queue, int bin, DecideArgs a,
         my_k += (threadIdx.x == 0) ? (unsigned)gm : 0u;
         my_k1 += (threadIdx.x == 0) ? (ull)gm : 0ull;
         // evaluate and clear the used H0 prefix, four slots (one 16-byte key load) per thread
+        // (two groups per pass measured slower: the extra registers halve the resident blocks)
         for (int t0 = threadIdx.x * 4; t0 < tcap; t0 += BT * 4) {
             const int4 k4 = *reinterpret_cast<const int4*>(keys + t0);
             const int cs[4] = {k4.x, k4.y, k4.z, k4.w};

@@ -84,7 +84,8 @@ __global__ void k_degrees(int n, const int64_t* __restrict__ rp, const int32_t* 
 // a1: every vertex its own community
 __global__ void k_level_init(int n, const int64_t* __restrict__ d, int32_t* __restrict__ C,
                              int64_t* __restrict__ Sig, int32_t* __restrict__ size, int64_t* __restrict__ dp,
-                             int32_t* __restrict__ stamp, Carry* __restrict__ carry, PruneState ps) {
+                             int32_t* __restrict__ stamp, int2* __restrict__ cst, Carry* __restrict__ carry,
+                             PruneState ps) {
     for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n;
          v += (long long)gridDim.x * blockDim.x) {
         C[v] = (int32_t)v;
@@ -92,6 +93,7 @@ __global__ void k_level_init(int n, const int64_t* __restrict__ d, int32_t* __re
         size[v] = 1;
         dp[v] = 0;
         stamp[v] = -1;
+        cst[v] = make_int2((int)v, -1);
         if (ps.rmflag) ps.rmflag[v] = -1;
         if (ps.smflag) { ps.smflag[v] = -1; ps.chg[v] = -1; }
     }
@@ -277,8 +279,8 @@ __global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr,
                                                  long long qstride, const int32_t* __restrict__ nextC,
                                                  int32_t* __restrict__ C, int64_t* __restrict__ Sig,
                                                  int32_t* __restrict__ size, int64_t* __restrict__ dp,
-                                                 int32_t* __restrict__ stamp, const Carry* __restrict__ carry,
-                                                 int32_t* __restrict__ it_v, int32_t* __restrict__ it_old,
+                                                 int32_t* __restrict__ stamp, int2* __restrict__ cst,
+                                                 const Carry* __restrict__ carry, int32_t* __restrict__ it_v, int32_t* __restrict__ it_old,
                                                  int32_t* __restrict__ it_chunk, PruneState ps, long long icap) {
     __shared__ unsigned s_cnt, s_items, s_hitems;
     __shared__ ull s_ibase, s_hbase;
@@ -315,6 +317,7 @@ __global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr,
                 deg = q.deg;
                 C[v] = nc;
                 stamp[v] = iter_id;
+                cst[v] = make_int2(nc, iter_id);
                 atomicAdd(reinterpret_cast<ull*>(&Sig[oc]), (ull)(-dv));
                 atomicAdd(reinterpret_cast<ull*>(&Sig[nc]), (ull)dv);
                 atomicSub(&size[oc], 1);
@@ -394,8 +397,8 @@ __device__ __forceinline__ bool use_delta(const IterCounters* ctr, long long nnz
 template <bool UNIT>
 __global__ void __launch_bounds__(256) k_dp_delta(IterCounters* __restrict__ ctr, const int64_t* __restrict__ rp,
                                                   const int32_t* __restrict__ col, const int64_t* __restrict__ w,
-                                                  const int32_t* __restrict__ C, const int32_t* __restrict__ it_v,
-                                                  const int32_t* __restrict__ it_old,
+                                                  const int32_t* __restrict__ C, const int2* __restrict__ cst,
+                                                  const int32_t* __restrict__ it_v, const int32_t* __restrict__ it_old,
                                                   const int32_t* __restrict__ it_chunk,
                                                   const int32_t* __restrict__ stamp, int64_t* __restrict__ dp,
                                                   const Carry* __restrict__ carry, long long nnz, int mode,
@@ -437,8 +440,9 @@ __global__ void __launch_bounds__(256) k_dp_delta(IterCounters* __restrict__ ctr
             }
 #pragma unroll
             for (int t = 0; t < 4; ++t) {
-                cx[t] = x[t] != u ? C[x[t]] : -1;
-                sx[t] = x[t] != u ? stamp[x[t]] : iter_id;
+                const int2 cs = x[t] != u ? cst[x[t]] : make_int2(-1, iter_id);   // one 8-byte gather
+                cx[t] = cs.x;
+                sx[t] = cs.y;
             }
             long long acc = 0;
 #pragma unroll
@@ -476,8 +480,9 @@ __global__ void __launch_bounds__(256) k_dp_delta(IterCounters* __restrict__ ctr
             }
 #pragma unroll
             for (int t = 0; t < 4; ++t) {
-                cx[t] = x[t] != u ? C[x[t]] : -1;
-                sx[t] = x[t] != u ? stamp[x[t]] : iter_id;
+                const int2 cs = x[t] != u ? cst[x[t]] : make_int2(-1, iter_id);
+                cx[t] = cs.x;
+                sx[t] = cs.y;
             }
 #pragma unroll
             for (int t = 0; t < 4; ++t) {

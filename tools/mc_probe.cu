@@ -34,21 +34,41 @@ int main() {
     if (!mc) { printf("NO MULTICAST\n"); return 0; }
     CUmulticastObjectProp p = {};
     p.numDevices = 1;
-    p.handleTypes = CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR;
     p.size = 2 << 20;
     size_t gran = 0;
-    CKD(cuMulticastGetGranularity(&gran, &p, CU_MULTICAST_GRANULARITY_RECOMMENDED));
-    size_t size = ((2 << 20) + gran - 1) / gran * gran;
-    p.size = size;
-    printf("granularity %zu size %zu\n", gran, size);
     CUmemGenericAllocationHandle mch, mh;
-    CKD(cuMulticastCreate(&mch, &p));
+    // which handle types does cuMulticastCreate accept here?
+    const unsigned long long types[3] = {0ull, (unsigned long long)CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR,
+                                         (unsigned long long)CU_MEM_HANDLE_TYPE_FABRIC};
+    int ok_type = -1;
+    for (int t = 0; t < 3; ++t) {
+        for (int nd = 1; nd <= 2; ++nd) {
+            p.handleTypes = types[t];
+            p.numDevices = nd;
+            CUresult rg = cuMulticastGetGranularity(&gran, &p, CU_MULTICAST_GRANULARITY_RECOMMENDED);
+            p.size = gran ? ((2 << 20) + gran - 1) / gran * gran : (2 << 20);
+            CUresult rc = cuMulticastCreate(&mch, &p);
+            const char* es = nullptr;
+            cuGetErrorString(rc, &es);
+            printf("handleTypes %llu numDevices %d: granularity rc %d (%zu), create rc %d %s\n", types[t], nd, (int)rg,
+                   gran, (int)rc, es);
+            if (rc == CUDA_SUCCESS) {
+                if (nd == 1 && ok_type < 0) ok_type = t;
+                else cuMemRelease(mch);
+                if (nd == 1) goto made;
+            }
+        }
+    }
+    printf("NO MULTICAST OBJECT\n");
+    return 0;
+made:
+    size_t size = p.size;
     CKD(cuMulticastAddDevice(mch, d));
     CUmemAllocationProp ap = {};
     ap.type = CU_MEM_ALLOCATION_TYPE_PINNED;
     ap.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
     ap.location.id = 0;
-    ap.requestedHandleTypes = CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR;
+    ap.requestedHandleTypes = (CUmemAllocationHandleType)types[ok_type];
     size_t mg = 0;
     CKD(cuMemGetAllocationGranularity(&mg, &ap, CU_MEM_ALLOC_GRANULARITY_RECOMMENDED));
     CKD(cuMemCreate(&mh, size, &ap, 0));

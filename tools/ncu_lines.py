@@ -7,7 +7,7 @@ import subprocess
 import sys
 
 
-def main(rep, kernel_regex=None, top=25):
+def main(rep, kernel_regex=None, top=25, fn_sub=None):
     args = ['ncu', '-i', rep, '--page', 'source', '--csv', '--print-source=cuda,sass']
     if kernel_regex:
         args += ['-k', 'regex:' + kernel_regex]
@@ -17,8 +17,14 @@ def main(rep, kernel_regex=None, top=25):
     hdr = None
     total = 0
     itotal = [0]
+    keep = True
     for row in csv.reader(io.StringIO(out)):
         if not row:
+            continue
+        if row[0] == 'Function Name':
+            keep = fn_sub is None or fn_sub in row[1]
+            continue
+        if not keep:
             continue
         if row[0] == 'File Path':
             fname = row[1].split('/')[-1]
@@ -57,4 +63,5 @@ def main(rep, kernel_regex=None, top=25):
 
 
 if __name__ == '__main__':
-    main(sys.argv[1], sys.argv[2] if len(sys.argv) > 2 else None, int(sys.argv[3]) if len(sys.argv) > 3 else 25)
+    main(sys.argv[1], sys.argv[2] if len(sys.argv) > 2 else None, int(sys.argv[3]) if len(sys.argv) > 3 else 25,
+         sys.argv[4] if len(sys.argv) > 4 else None)
