@@ -43,6 +43,8 @@ WORKLOADS = {
     "rmat_lj": "R-MAT LiveJournal-shaped 4.8M / 69M (BASELINE.json configs[2])",
     "orkut": "Orkut-shaped LFR 3.1M / 117.2M edges, max degree 33.1k (BASELINE.json configs[3]; largest single-GPU config)",
     "friendster_q": "Friendster-shaped LFR at 1/4 scale, 16.4M / ~451M (BASELINE.json configs[4] shape on 1 GPU)",
+    "friendster": "Friendster-shaped LFR 65.6M / 1.806B edges (BASELINE.json configs[4]) on ONE B200 (memory-lean "
+                  "host generator, ~4 min on 16 cores; the 8-GPU partitioned run needs a multi-GPU box)",
     "lfr_small": "LFR 20k (test size)",
 }
 METRIC = "local-move GTEPS and end-to-end Louvain seconds at 1/2/4/8 B200; modularity Q"

@@ -40,8 +40,8 @@ def _lib():
         lib.gg_lfr_ex.argtypes = [i64, dbl, i64, dbl, dbl, i64, i64, dbl, u64, ctypes.c_int, dbl, ctypes.c_int,
                                   p, p, p, p]
         lib.gg_lfr_csr.restype = i64
-        lib.gg_lfr_csr.argtypes = [i64, dbl, i64, dbl, dbl, i64, i64, dbl, u64, p, ctypes.POINTER(ctypes.c_void_p),
-                                   p, p, p]
+        lib.gg_lfr_csr.argtypes = [i64, dbl, i64, dbl, dbl, i64, i64, dbl, u64, ctypes.c_int, p,
+                                   ctypes.POINTER(ctypes.c_void_p), p, p, p]
         lib.gg_free.restype = None
         lib.gg_free.argtypes = [p]
         lib.gg_random_permutation.restype = None
@@ -199,7 +199,7 @@ def lfr(n: int, avg_k: float, kmax: int, mu: float, tau1=2.5, tau2=1.5, cmin=50,
 
 
 def lfr_csr(n: int, avg_k: float, kmax: int, mu: float, tau1=2.5, tau2=1.5, cmin=50, cmax=2000, seed=1,
-            name="lfr") -> CSR:
+            name="lfr", fit_frac: bool = False) -> CSR:
     """Memory-lean LFR-style graph built straight into CSR (graphgen.c gg_lfr_csr): the plan of
     lfr() (degrees, community sizes, placement, internal wiring), external stubs paired through a
     counter-based random bijection instead of a sort, self pairs / duplicates / same-community
@@ -212,13 +212,13 @@ def lfr_csr(n: int, avg_k: float, kmax: int, mu: float, tau1=2.5, tau2=1.5, cmin
     colp = ctypes.c_void_p()
     kmin = ctypes.c_int64(0)
     stats = np.zeros(3, dtype=np.int64)
-    nnz = lib.gg_lfr_csr(n, avg_k, kmax, tau1, tau2, cmin, cmax, mu, seed, _ptr(row_ptr), ctypes.byref(colp),
+    nnz = lib.gg_lfr_csr(n, avg_k, kmax, tau1, tau2, cmin, cmax, mu, seed, int(fit_frac), _ptr(row_ptr), ctypes.byref(colp),
                          _ptr(truth), ctypes.byref(kmin), _ptr(stats))
     col = np.ctypeslib.as_array(ctypes.cast(colp, ctypes.POINTER(ctypes.c_int32)), shape=(max(nnz, 1),))[:nnz]
     weakref.finalize(col.base, lib.gg_free, colp.value)
     g = CSR(n=n, row_ptr=row_ptr, col=col, w=None, name=name, truth=truth)
     g.meta.update(dict(generator="lfr_csr", avg_k=avg_k, kmax=kmax, kmin=int(kmin.value), mu=mu, tau1=tau1,
-                       tau2=tau2, cmin=cmin, cmax=cmax, seed=seed, internal_edges=int(stats[0]),
+                       tau2=tau2, cmin=cmin, cmax=cmax, seed=seed, fit_frac=fit_frac, internal_edges=int(stats[0]),
                        external_pairs=int(stats[1]), dropped=int(stats[2])))
     return g
 
@@ -270,7 +270,8 @@ CONFIGS = {
     "rmat_lj": dict(desc="R-MAT scale 23 (0.48,0.20,0.20,0.12), n=4,847,571, 69.0M undirected edges, seed 2"),
     "orkut": dict(desc="LFR-style n=3,072,441, <k>=76.3 (m=117.2M), kmax=33,313, tau1=2.3, c in [50,50000], "
                        "mu=0.35, internal degree <= (size-1)/2, rewired to a simple graph, seed 3"),
-    "friendster": dict(desc="LFR-style n=65,608,366, <k>=55.06, kmax=5,214, tau1=2.5, mu=0.37, seed 4; memory-lean "
+    "friendster": dict(desc="LFR-style n=65,608,366, realised <k>=55.06 (1.806B edges), kmax=5,214, tau1=2.5, mu=0.37, "
+                            "seed 4; memory-lean "
                             "generator straight to CSR (gg_lfr_csr: external stubs paired by a counter-based "
                             "bijection; ~30 GB host, minutes on 16 cores)"),
     # the Friendster shape at 1/4 of its vertices (same degree law / mixing): the largest FR-shaped
@@ -303,7 +304,11 @@ def make(name: str) -> CSR:
         return lfr(3_072_441, 76.68, 33_313, 0.35, tau1=2.3, cmin=50, cmax=50000, seed=3, name=name,
                    fit_frac=True, alpha=0.5, rewire=True)
     if name == "friendster":
-        return lfr_csr(65_608_366, 55.06, 5_214, 0.37, seed=4, name=name)
+        # avg_k 63.85 with the exact-mean law: the configuration-model wiring drops ~13.8 % of the
+        # pairs (duplicates inside small dense communities, same-community external pairs), so the
+        # law's mean is raised until the REALISED mean degree is FR's 55.06 (1.806B edges;
+        # calibrated at n = 2M: 63 -> 54.35, 64 -> 55.18; the drop fraction does not depend on n)
+        return lfr_csr(65_608_366, 63.85, 5_214, 0.37, seed=4, name=name, fit_frac=True)
     if name == "friendster_q":
         return lfr(16_402_092, 55.06, 5_214, 0.37, seed=4, name=name)
     if name == "lfr_small":

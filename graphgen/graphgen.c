@@ -665,10 +665,10 @@ static int cmp_i32(const void* a, const void* b) {
 void gg_free(void* p) { free(p); }
 
 int64_t gg_lfr_csr(int64_t n, double avg_k, int64_t kmax, double tau1, double tau2, int64_t cmin, int64_t cmax,
-                   double mu, uint64_t seed, int64_t* row_ptr, int32_t** out_col, int64_t* membership,
+                   double mu, uint64_t seed, int fit_frac, int64_t* row_ptr, int32_t** out_col, int64_t* membership,
                    int64_t* out_kmin, int64_t* out_stats /* [internal edges, external pairs, dropped] */) {
     lfr_plan_t P;
-    lfr_plan(n, avg_k, kmax, tau1, tau2, cmin, cmax, mu, seed, 0, 1.0, 0, &P);
+    lfr_plan(n, avg_k, kmax, tau1, tau2, cmin, cmax, mu, seed, fit_frac, 1.0, 0, &P);
     if (out_kmin) *out_kmin = P.kmin;
     int64_t *k = P.k, *kin = P.kin, *comm = P.comm, *coff = P.coff, *mem = P.mem;
     const int64_t nc = P.nc;

@@ -49,7 +49,7 @@ lv0 = st["levels"][0]
 out.update(run_ms=ts, levels=len(st["levels"]), iterations=sum(l["iters"] for l in st["levels"]),
            Q=h.modularity(), level0_ms_phase1=lv0["ms_phase1"], level0_active_edges=lv0["edges_scanned"],
            per_level=[{k: l[k] for k in ("n", "nnz", "iters", "ms_phase1", "ms_phase2")} for l in st["levels"]],
-           pool_mb=torch.cuda.max_memory_reserved() / 2**20)
+           device_used_gb=round((torch.cuda.mem_get_info()[1] - torch.cuda.mem_get_info()[0]) / 2**30, 1))
 out["level0_gteps"] = lv0["edges_scanned"] / (lv0["ms_phase1"] * 1e-3) / 1e9
 labels = h.communities()
 N_gpu = h.numerator()[0]
