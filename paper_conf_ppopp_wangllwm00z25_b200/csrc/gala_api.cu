@@ -127,6 +127,7 @@ struct gala_graph_s {
     int opt_ckey = 0;
     int bins[NBINS - 1] = {4, 8, 16, 32, 128, 512, 16384};
     int hub_smem_slots = 8192;
+    int opt_hub_cluster = 1;
     // results
     bool has_result = false;
     int64_t k = 0, p = 1, q = 1;
@@ -145,6 +146,7 @@ struct gala_graph_s {
     // multi-GPU (one process per GPU)
     struct DistInfo* di = nullptr;
     bool fab_host_bar = false;   // = di->host_bar (fabric barriers on the host: loopback ranks on one device)
+    int64_t k_final = -1;        // communities of the last completed run (labels 0..k-1)
     int sync_mode = 0;
     std::vector<long long> dbounds0;   // level-0 owned ranges of all ranks
     struct Work* wk = nullptr;   // persistent run workspace (sized for level 0, reused by every run)
@@ -464,6 +466,7 @@ struct Work {
     int gblocks_m[3] = {0, 0, 0};
     // hub tables (k_hub_*), sized per level for the rows longer than the block bin
     bool hub_on = false;
+    bool hub_cluster = false;   // this level's hubs take the cluster kernel (k_decide_cluster)
     HubWork hw = {};
     long long hub_ncap = 0, hub_tcap = 0, hub_lcap = 0, hub_pcap = 0;
     ull* hub_size = nullptr;
@@ -543,6 +546,15 @@ static void launch_hub(gala_graph_s* g, Work& wk, const DecideArgs& a, typename 
     if (!wk.hub_on) return;
     const QView q = qview(wk.queues, wk.qcap, BIN_HUB);
     cudaEvent_t e = tm.begin();
+    if constexpr (M != DM_W128) {
+        if (wk.hub_cluster) {   // tables in the distributed shared memory of a thread-block cluster
+            const int grid = std::max(g->num_sms / CL_CS, 1) * CL_CS;
+            k_decide_cluster<M, UNIT><<<grid, CL_BT, CL_SLOTS * sizeof(ull), st>>>(q, a, qW, p);
+            CKL();
+            tm.end(KC_DEC_HUB, e);
+            return;
+        }
+    }
     k_hub_prep<<<1, 1024, 0, st>>>(q, wk.ctr, wk.hw);
     CKL();
     k_hub_agg<M, UNIT><<<g->num_sms * 8, HUB_BT, 0, st>>>(q, a, wk.hw);
@@ -627,6 +639,14 @@ static void block_attrs_ensure(int slots) {
     block_attr_mode<DM_FAST, true>(slots); block_attr_mode<DM_FAST, false>(slots);
     block_attr_mode<DM_W64, true>(slots); block_attr_mode<DM_W64, false>(slots);
     block_attr_mode<DM_W128, true>(slots); block_attr_mode<DM_W128, false>(slots);
+    if (!cur.count(-1 - dev)) {   // cluster hub kernel: its fixed 128 KB per CTA
+        const int cs = CL_SLOTS * (int)sizeof(ull);
+        CK(cudaFuncSetAttribute(k_decide_cluster<DM_FAST, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, cs));
+        CK(cudaFuncSetAttribute(k_decide_cluster<DM_FAST, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, cs));
+        CK(cudaFuncSetAttribute(k_decide_cluster<DM_W64, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, cs));
+        CK(cudaFuncSetAttribute(k_decide_cluster<DM_W64, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, cs));
+        cur[-1 - dev] = 1;
+    }
     cur[dev] = slots;
 }
 // the largest block arena this handle launches (the short-row class runs only when its arena is
@@ -697,6 +717,7 @@ static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, typename M
     a.rp = G.rp; a.col = G.col; a.w = G.w; a.C = wk.C; a.Sig = wk.Sig; a.size = wk.size; a.d = wk.d;
     a.dp = wk.dp; a.nextC = wk.nextC; a.ctr = wk.ctr; a.check = g->opt_check;
     a.table_mode = g->opt_table_mode;
+    a.nlev = G.n;
     a.ckey = use_ckey(g, wk, G) ? wk.ckey : nullptr;
     a.ckey_valid = &wk.carry->ckey_valid;
     a.idbits = idbits;
@@ -769,6 +790,12 @@ static void prepare_level_tables(gala_graph_s* g, Work& wk, const DevCSR& G, int
         CK(cudaMemsetAsync(wk.gvals, 0, sizeof(ull) * (size_t)wk.gblocks * wk.gcap, st));
     }
     wk.hub_on = maxdeg > g->bins[BIN_BLOCK];
+    {   // every hub's table fits the cluster's distributed shared memory (load <= 1/2)
+        long long need = 64LL * CL_CS;
+        while (need < 2 * std::min<long long>(maxdeg, G.n)) need <<= 1;
+        // (32-bit packed sums: launched only in the modes with 32-bit aggregates, d(v) < 2^32)
+        wk.hub_cluster = wk.hub_on && g->opt_hub_cluster && need <= (long long)CL_CS * CL_SLOTS;
+    }
     if (!wk.hub_on) return;
     if (!wk.hub_size) wk.hub_size = dalloc<ull>(3, st);
     CK(cudaMemsetAsync(wk.hub_size, 0, sizeof(ull) * 3, st));
@@ -1130,7 +1157,11 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
     long long* eoff = dalloc<long long>(k + 1, st);
     long long* dn = dalloc<long long>(k + 1, st);
     int* tkey = dalloc<int>(cur.nnz, st);
-    int64_t* tval = dalloc<int64_t>(cur.nnz, st);
+    // segment weights: 32-bit when W < 2^32 (every aggregated weight is <= W): halves the largest
+    // phase-2 temporary (14.5 GB of 29 GB on the level-0 Friendster shape)
+    TVal tval;
+    tval.w32 = g->W < ((int64_t)1 << 32);
+    tval.p = dalloc<char>((size_t)cur.nnz * (tval.w32 ? 4 : 8), st);
     ull* dev_max = dalloc<ull>(1, st);
     int32_t* bigc = dalloc<int32_t>(k, st);
     long long* bigcap = dalloc<long long>(k + 1, st);
@@ -1330,7 +1361,8 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
     g->kc_bytes[KC_PHASE2] += (double)nrows * (4 + 4 + 8 + 16 + 4 + 4) + (double)cur.nnz * (4 + 4 + (unit ? 0 : 8) + 12) +
                               (double)nxt.nnz * 24;
     dfree(cnt, st); dfree(ent, st); dfree(eoff, st); dfree(dn, st);
-    dfree(tkey, st); dfree(tval, st); dfree(dev_max, st); dfree(bigc, st);
+    { char* tp = static_cast<char*>(tval.p); dfree(tp, st); }
+    dfree(tkey, st); dfree(dev_max, st); dfree(bigc, st);
     dfree(bigcap, st); dfree(nbig_dev, st); dfree(wlist, st); dfree(blist, st);
 }
 
@@ -1661,6 +1693,7 @@ static void do_run(gala_graph_s* g, double gamma, double tol, int max_levels) {
             long long kcomm = 0;
             CK(cudaMemcpyAsync(&kcomm, pos + nl, sizeof(long long), cudaMemcpyDeviceToHost, st));
             CK(cudaStreamSynchronize(st));
+            g->k_final = kcomm;   // canonical final labels are 0..k-1 (reading c19)
             const bool stop = (kcomm == nl) || (max_levels > 0 && level + 1 >= max_levels) || (N - N_start < T);
             DevCSR nxt;
             if (!stop) coarsen(g, wk, cur, nl, kcomm, newid, minmem, unit, nxt, maxdeg, dmax);
@@ -2441,6 +2474,7 @@ static void do_run_dist(gala_graph_s* g, double gamma, double tol, int max_level
             long long kcomm = 0;
             CK(cudaMemcpyAsync(&kcomm, pos + nl, sizeof(long long), cudaMemcpyDeviceToHost, st));
             CK(cudaStreamSynchronize(st));
+            g->k_final = kcomm;   // canonical final labels are 0..k-1 (reading c19)
             const bool stop = (kcomm == nl) || (max_levels > 0 && level + 1 >= max_levels) || (N - N_start < T);
             DevCSR nxt;
             if (!stop) {
@@ -2728,6 +2762,7 @@ gala_status gala_run(gala_graph g, double gamma, double tol, int32_t max_levels)
         CK(cudaStreamSynchronize(g->stream));
         gamma_to_pq(gamma, &g->p, &g->q);
         g->N = 0;
+        g->k_final = g->n0;
         g->levels.clear();
         g->trace.clear();
         g->trace_labels.clear();
@@ -2751,7 +2786,9 @@ static gala_status fetch_labels(gala_graph g, int32_t* out, int64_t n, int64_t* 
     if (n) CK(cudaMemcpyAsync(dst, g->lab, sizeof(int32_t) * n, device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost,
                               g->stream));
     CK(cudaStreamSynchronize(g->stream));
-    if (k) {
+    if (k && g->k_final >= 0) {   // known from the run's last relabel: no host pass over the labels
+        *k = g->k_final;
+    } else if (k) {
         if (device) {
             h.resize(n);
             if (n) CK(cudaMemcpy(h.data(), g->lab, sizeof(int32_t) * n, cudaMemcpyDeviceToHost));
@@ -2904,6 +2941,7 @@ gala_status gala_set_option(gala_graph g, const char* key, int64_t value) {
         g->opt_agg_scap = (int)value;
     }
     else if (k == "ckey") g->opt_ckey = value != 0;
+    else if (k == "hub_cluster") g->opt_hub_cluster = value != 0;   // hubs on a thread-block cluster (DSMEM tables)
     else if (k == "concurrent") g->opt_concurrent = value != 0;
     else if (k == "verbose") g->opt_verbose = (int)value;
     else if (k == "cuda_graph") g->opt_cuda_graph = value != 0;

@@ -98,6 +98,7 @@ struct DecideArgs {
     int table_mode;     // block bin's table (§4.2): 0 hierarchical, 1 global-only, 2 unified
     int idbits;         // packed-key layout (DM_FAST)
     long long idmask;
+    long long nlev;     // vertices of the level (bound on distinct communities per row)
 };
 
 // ---------------------------------------------------------------------------
@@ -1318,4 +1319,140 @@ __global__ void k_hub_size(long long n, const int64_t* __restrict__ rp, long lon
         atomicAdd(&out[1], cap);
         atomicAdd(&out[2], dist);
     }
+}
+
+// ---------------------------------------------------------------------------
+// a4, hubs (rows longer than the block bin) on a THREAD-BLOCK CLUSTER: the hierarchical
+// table's upper level (§4.2: "if H0 cannot hold a community, H1") lives in the
+// distributed shared memory of CS CTAs instead of global memory.  One cluster per hub vertex
+// (dynamic fetch by CTA 0, broadcast over DSMEM):
+//   * every CTA streams a contiguous 1/CS of the row (E entries per thread in flight), combines
+//     the equal communities of each 32-entry chunk with __match_any_sync (Alg. 2) and inserts the
+//     chunk's distinct (c, sum) into the table of the OWNER CTA of c (hub_hash bits), a packed
+//     64-bit slot per key (kv_insert through the cluster-mapped address: DSMEM atomics);
+//   * the own community only feeds d'(v) (summed in registers, one DSMEM add per CTA);
+//   * cluster barrier; each CTA evaluates and clears the occupied slots of its own table
+//     (Sigma_tot gathered once per distinct community), block argmax, partial written into
+//     CTA 0 over DSMEM; cluster barrier; CTA 0 decides (reading c1/c4/c5).
+// Table: nextpow2(2 min(deg, n_level)) slots split evenly over the CS CTAs (load <= 1/2, never
+// spills); used on levels whose longest row fits CS * CL_SLOTS slots and whose aggregates are
+// 32-bit (not DM_W128), else the global multi-block hub path above runs.
+// ---------------------------------------------------------------------------
+#include <cooperative_groups.h>
+#define CL_CS 8          // CTAs per cluster (portable maximum)
+#define CL_SLOTS 16384   // packed slots per CTA (128 KB of shared memory)
+#define CL_BT 512
+#define CL_E 4
+template <int M, bool UNIT>
+__global__ void __cluster_dims__(CL_CS, 1, 1) __launch_bounds__(CL_BT, 1)
+    k_decide_cluster(QView queue, DecideArgs a, typename ModeT<M>::ST qW, typename ModeT<M>::ST p) {
+    namespace cg = cooperative_groups;
+    typedef typename ModeT<M>::ST ST;
+    typedef Arg<ST, ModeT<M>::PK> A;
+    static_assert(sizeof(typename ModeT<M>::VT) == 4, "packed slots need 32-bit aggregates");
+    cg::cluster_group cl = cg::this_cluster();
+    const unsigned crank = cl.block_rank();
+    extern __shared__ __align__(16) ull ctbl[];
+    __shared__ long long s_item;
+    __shared__ long long s_own;
+    __shared__ A s_part[CL_CS];
+    __shared__ A r_a[CL_BT / 32];
+    __shared__ long long r_own[CL_BT / 32];
+    __shared__ unsigned s_scr[CL_BT / 32][32];
+    if (a.ckey && !*a.ckey_valid) a.ckey = nullptr;
+    const int lane = lane_id(), wib = threadIdx.x >> 5;
+    for (int j = threadIdx.x; j < CL_SLOTS; j += CL_BT) ctbl[j] = KV_EMPTY;
+    if (threadIdx.x == 0) s_own = 0;
+    const long long count = (long long)a.ctr->bin_count[BIN_HUB];
+    ull* const cursor = &a.ctr->cursor[BIN_HUB];
+    long long* const own0 = cl.map_shared_rank(&s_own, 0);
+    A* const part0 = cl.map_shared_rank(s_part, 0);
+    const long long* const item0 = cl.map_shared_rank(&s_item, 0);
+    unsigned my_k = 0;
+    for (;;) {
+        if (crank == 0 && threadIdx.x == 0) s_item = (long long)atomicAdd(cursor, 1ull);
+        cl.sync();   // s_item published; the previous hub's tables are clear everywhere
+        const long long i = *item0;
+        if (i >= count) break;
+        const QRec q = queue[i];
+        const int v = q.v, deg = q.deg, cv = q.cv;
+        const long long span = deg < a.nlev ? deg : a.nlev;
+        long long need = 64LL * CL_CS;
+        while (need < 2 * span) need <<= 1;
+        const unsigned tmask = (unsigned)(need / CL_CS) - 1;   // this hub's slots per CTA
+        const long long per = (deg + CL_CS - 1) / CL_CS;
+        const long long r0 = (long long)crank * per, r1 = min((long long)deg, r0 + per);
+        long long own = 0;
+        for (long long j0 = r0; j0 < r1; j0 += (long long)CL_BT * CL_E) {   // block-uniform rounds
+            int cc[CL_E];
+            unsigned ww[CL_E];
+#pragma unroll
+            for (int k = 0; k < CL_E; ++k) {
+                const long long j = j0 + threadIdx.x + (long long)k * CL_BT;
+                const bool in = j < r1;
+                int u = in ? (a.ckey ? a.ckey[q.beg + j] : a.col[q.beg + j]) : -1;
+                ww[k] = (in && !UNIT) ? (unsigned)a.w[q.beg + j] : 1u;
+                if (!a.ckey) u = (u >= 0 && u != v) ? a.C[u] : -1;
+                cc[k] = in ? u : -1;
+            }
+#pragma unroll
+            for (int k = 0; k < CL_E; ++k) {
+                if (cc[k] == cv) { own += (long long)ww[k]; cc[k] = -1; }
+                const unsigned peers = __match_any_sync(FULLMASK, cc[k] >= 0 ? cc[k] : -1 - lane);
+                const unsigned sum = UNIT ? (unsigned)__popc(peers) : group_sum(peers, cc[k] >= 0 ? ww[k] : 0u, s_scr[wib]);
+                if (cc[k] >= 0 && lane == __ffs(peers) - 1) {
+                    const unsigned hh = hub_hash(cc[k], 0xFFFFFFFFu);
+                    ull* const t = cl.map_shared_rank(ctbl, hh % CL_CS);
+                    bool fresh;
+                    kv_insert(cc[k], sum, t, tmask, (hh / CL_CS) & tmask, (int)tmask + 1, &fresh);
+                }
+            }
+        }
+        own = warp_sum_ll(own);
+        if (lane == 0 && own) atomicAdd(reinterpret_cast<ull*>(own0), (ull)own);
+        cl.sync();   // every insert (and every own contribution) has landed
+        const long long dv = q.dv;
+        A best;
+        best.init(a.idbits, a.idmask);
+        for (unsigned t0 = threadIdx.x * 2; t0 <= tmask; t0 += CL_BT * 2) {   // two slots (16 bytes) per load
+            const ulonglong2 kv = *reinterpret_cast<const ulonglong2*>(ctbl + t0);
+            const ull e[2] = {kv.x, kv.y};
+            if (e[0] == KV_EMPTY && e[1] == KV_EMPTY) continue;
+            long long sg[2];
+#pragma unroll
+            for (int k = 0; k < 2; ++k) sg[k] = e[k] != KV_EMPTY ? a.Sig[(int)(e[k] >> 32)] : 0;
+            *reinterpret_cast<ulonglong2*>(ctbl + t0) = make_ulonglong2(KV_EMPTY, KV_EMPTY);
+#pragma unroll
+            for (int k = 0; k < 2; ++k) {
+                if (e[k] == KV_EMPTY) continue;
+                ++my_k;
+                best.offer(gain<ST>(qW, p, (long long)(unsigned)e[k], sg[k], dv), (int)(e[k] >> 32));
+            }
+        }
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) best.xor_merge(off);
+        if (lane == 0) r_a[wib] = best;
+        __syncthreads();
+        if (wib == 0) {
+            best = lane < CL_BT / 32 ? r_a[lane] : best;
+            if (lane >= CL_BT / 32) best.init(a.idbits, a.idmask);
+#pragma unroll
+            for (int off = 16; off > 0; off >>= 1) best.xor_merge(off);
+            if (lane == 0) part0[crank] = best;
+        }
+        cl.sync();   // every CTA's partial is in CTA 0
+        if (crank == 0 && threadIdx.x == 0) {
+            A b = s_part[0];
+            for (int r = 1; r < CL_CS; ++r)
+                if (s_part[r].valid()) b.offer(s_part[r].score(), s_part[r].comm());
+            const long long ownv = s_own;
+            if (a.check && ownv != a.dp[v]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
+            a.nextC[v] = decide_final<ST>(cv, q.szv, dv, ownv, q.sigv, b, a.size, qW, p);
+            my_k += ownv ? 1u : 0u;
+            s_own = 0;
+        }
+    }
+    (void)r_own;
+    ull k = block_sum_ull<CL_BT>((ull)my_k);
+    if (threadIdx.x == 0 && k) atomicAdd(&a.ctr->bin_k[BIN_HUB], k);
 }

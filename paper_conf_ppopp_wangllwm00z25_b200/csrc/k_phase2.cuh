@@ -215,6 +215,20 @@ __global__ void __launch_bounds__(256) k_vpos_hist(int n, long long k, const int
     }
 }
 
+// per-entry weights of the community-major segments: 32-bit when every aggregated weight fits
+// (W < 2^32, the common case: the level-0 graph of every config), else 64-bit
+struct TVal {
+    void* p;
+    int w32;
+    __device__ __forceinline__ long long get(long long j) const {
+        return w32 ? (long long)static_cast<const unsigned*>(p)[j] : static_cast<const long long*>(p)[j];
+    }
+    __device__ __forceinline__ void set(long long j, long long v) const {
+        if (w32) static_cast<unsigned*>(p)[j] = (unsigned)v;
+        else static_cast<long long*>(p)[j] = v;
+    }
+};
+
 // edge-parallel: entry e of row r goes to vpos[r] + (e - rp[r]) with key newid[col[e]];
 // 4 entries per lane in flight, coalesced row/col streams
 template <bool UNIT>
@@ -222,7 +236,7 @@ __global__ void __launch_bounds__(256) k_gather_flat(long long nnz, const int32_
                                                      const int64_t* __restrict__ rp, const int32_t* __restrict__ col,
                                                      const int64_t* __restrict__ w, const int32_t* __restrict__ newid,
                                                      const long long* __restrict__ vpos, int* __restrict__ tkey,
-                                                     int64_t* __restrict__ tval) {
+                                                     TVal tval) {
     const int lane = lane_id();
     const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
     for (long long base = (((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * 128; base < nnz;
@@ -247,7 +261,7 @@ __global__ void __launch_bounds__(256) k_gather_flat(long long nnz, const int32_
             long long e = base + lane + 32 * t;
             if (e < nnz) {
                 tkey[dst[t]] = kk[t];
-                if (!UNIT) tval[dst[t]] = w[e];
+                if (!UNIT) tval.set(dst[t], w[e]);
             }
         }
     }
@@ -355,7 +369,7 @@ struct AggArgs {
     const long long* ent;
     const long long* eoff;     // segment offsets (exclusive scan of ent)
     int* tkey;                 // segments: coarse keys in, distinct keys out
-    int64_t* tval;             // weights in (weighted levels), aggregated weights out
+    TVal tval;                 // weights in (weighted levels), aggregated weights out
     long long* dn;             // distinct entries per community
     int64_t* snew;             // diagonal weight per community
 };
@@ -427,7 +441,7 @@ __device__ __forceinline__ void agg_segment(const AggArgs& a, long long s0, long
         for (int t = 0; t < 4; ++t) {
             long long j = r0 + lane + 32 * t;
             kk[t] = j < s1 ? a.tkey[j] : -1;
-            ww[t] = (j < s1 && !UNIT) ? (SV)a.tval[j] : (SV)1;
+            ww[t] = (j < s1 && !UNIT) ? (SV)a.tval.get(j) : (SV)1;
         }
 #pragma unroll
         for (int t = 0; t < 4; ++t) {
@@ -451,7 +465,7 @@ __device__ __forceinline__ void agg_emit(const AggArgs& a, long long c, int m, c
         keys[slot] = -1;
         vals[slot] = 0;
         a.tkey[o + t] = key;
-        a.tval[o + t] = val;
+        a.tval.set(o + t, val);
         if (key == (int)c) a.snew[c] = val;
     }
 }
@@ -481,7 +495,7 @@ __global__ void __launch_bounds__(256) k_agg_warp(AggArgs a, const int32_t* __re
             const int j = lane;
             const bool on = j < s1 - s0;
             const int key = on ? a.tkey[s0 + j] : -1 - lane;
-            const V wt = (on && !UNIT) ? (V)a.tval[s0 + j] : (V)(on ? 1 : 0);
+            const V wt = (on && !UNIT) ? (V)a.tval.get(s0 + j) : (V)(on ? 1 : 0);
             const unsigned peers = __match_any_sync(FULLMASK, key);
             const V sum = UNIT ? (V)__popc(peers) : group_sum(peers, wt, s_scr[wib]);
             const bool lead = on && lane == __ffs(peers) - 1;
@@ -489,7 +503,7 @@ __global__ void __launch_bounds__(256) k_agg_warp(AggArgs a, const int32_t* __re
             if (lead) {   // distinct entries to the start of the segment (lead lanes ascend, never overtake)
                 const int t = __popc(lm & lanemask_lt());
                 a.tkey[s0 + t] = key;
-                a.tval[s0 + t] = (int64_t)sum;
+                a.tval.set(s0 + t, (int64_t)sum);
                 if (key == (int)c) a.snew[c] = (int64_t)sum;
             }
             if (lane == 0) a.dn[c] = __popc(lm);
@@ -573,7 +587,7 @@ __global__ void __launch_bounds__(512) k_agg_block_h(AggArgs a, int scap, const 
             for (int t = 0; t < 4; ++t) {
                 const long long j = r0 + lane + 32 * t;
                 kk[t] = j < s1 ? a.tkey[j] : -1;
-                ww[t] = (j < s1 && !UNIT) ? (V)a.tval[j] : (V)1;
+                ww[t] = (j < s1 && !UNIT) ? (V)a.tval.get(j) : (V)1;
             }
 #pragma unroll
             for (int t = 0; t < 4; ++t) {
@@ -638,7 +652,7 @@ __global__ void __launch_bounds__(512) k_agg_block_h(AggArgs a, int scap, const 
                 gvals[slot] = 0;
             }
             a.tkey[s0 + t] = key;
-            a.tval[s0 + t] = val;
+            a.tval.set(s0 + t, val);
             if (key == (int)c) a.snew[c] = val;
         }
         __syncthreads();
@@ -684,7 +698,7 @@ __global__ void __launch_bounds__(256) k_agg_big_emit(AggArgs a, const int32_t* 
             const int key = gkeys[off + slot];
             const int64_t val = (int64_t)gvals[off + slot];
             a.tkey[o + t] = key;
-            a.tval[o + t] = val;
+            a.tval.set(o + t, val);
             if (key == (int)c) a.snew[c] = val;
         }
         if (part == 0 && threadIdx.x == 0) a.dn[c] = m;
@@ -851,7 +865,7 @@ __global__ void __launch_bounds__(256) k_agg_big_combine(AggArgs a, const int32_
         for (int i = threadIdx.x; i < m; i += 256) {
             const int slot = list[i];
             a.tkey[lo + i] = keys[slot];
-            a.tval[lo + i] = (int64_t)vals[slot];
+            a.tval.set(lo + i, (int64_t)vals[slot]);
             keys[slot] = -1;
             vals[slot] = 0;
         }
@@ -895,7 +909,7 @@ __global__ void __launch_bounds__(256) k_agg_big_insert2(AggArgs a, const int32_
         for (int i0 = threadIdx.x & ~31; i0 < m; i0 += 256) {   // warp-uniform trips
             const int i = i0 + (threadIdx.x & 31);
             const bool on = i < m;
-            agg_insert_warp(on, on ? a.tkey[lo + i] : 0, on ? (ull)a.tval[lo + i] : 0, gkeys + off, gvals + off, mask,
+            agg_insert_warp(on, on ? a.tkey[lo + i] : 0, on ? (ull)a.tval.get(lo + i) : 0, gkeys + off, gvals + off, mask,
                             glist + off / 2, &gcnt[bi]);
         }
     }
@@ -925,7 +939,7 @@ __global__ void __launch_bounds__(256) k_agg_big_emit2(AggArgs a, const int32_t*
             const int key = gkeys[off + slot];
             const int64_t val = (int64_t)gvals[off + slot];
             a.tkey[o + i] = key;
-            a.tval[o + i] = val;
+            a.tval.set(o + i, val);
             if (key == (int)c) a.snew[c] = val;
         }
         if (j == 0 && threadIdx.x == 0) a.dn[c] = m;
@@ -948,7 +962,7 @@ __global__ void k_tile_map(long long k, const long long* __restrict__ rp_new, lo
 // from the aggregated segment at eoff[c]
 __global__ void __launch_bounds__(256) k_compact(long long k, long long nnz_new, const long long* __restrict__ eoff,
                                                  const long long* __restrict__ rp_new, const int32_t* __restrict__ tmap,
-                                                 const int* __restrict__ tkey, const int64_t* __restrict__ tval,
+                                                 const int* __restrict__ tkey, TVal tval,
                                                  int32_t* __restrict__ col_new, int64_t* __restrict__ w_new,
                                                  int32_t* __restrict__ row_new) {
     const long long ntiles = (nnz_new + 255) >> 8;
@@ -960,7 +974,7 @@ __global__ void __launch_bounds__(256) k_compact(long long k, long long nnz_new,
             const long long c = seg_search(rp_new, lo, hi, t);
             const long long src = eoff[c] + (t - rp_new[c]);
             col_new[t] = tkey[src];
-            w_new[t] = tval[src];
+            w_new[t] = tval.get(src);
             row_new[t] = (int32_t)c;
         }
     }

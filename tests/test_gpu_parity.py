@@ -31,6 +31,7 @@ def run_gpu(g, gamma=1.0, tol=1e-6, max_levels=0, trace=2, **opts):
     h.run(gamma=gamma, tol=tol, max_levels=max_levels)
     out = dict(labels=h.communities(), Q=h.modularity(), N=h.numerator()[0], trace=h.trace(labels=trace >= 2),
                stats=h.stats())
+    out["k"] = h.k   # the C ABI's community count (from the run's last relabel)
     h.free()
     return out
 
@@ -62,6 +63,7 @@ def assert_parity(g, gamma=1.0, tol=1e-6, max_levels=0, prune=True, labels=True,
         if pc:
             assert (x.n_fn, x.n_fp) == (y["n_fn"], y["n_fp"]), f"FN/FP differ at level {x.level} iter {x.iter}"
     assert np.array_equal(o.labels, r["labels"])
+    assert r["k"] == o.k == (int(o.labels.max()) + 1 if len(o.labels) else 0)
     assert o.N == r["N"]
     assert abs(o.Q - r["Q"]) <= 1e-9
     assert r["stats"]["dp_mismatch"] == 0
@@ -116,8 +118,10 @@ def test_pruning_strategy_weighted_and_graph_mode(strategy):
     dict(bin_sub4=0, bin_sub8=0, bin_sub16=0, bin_sub32=0, bin_warp=0),                  # warp512 hash <= 512
     dict(bin_sub4=4, bin_sub8=4, bin_sub16=4, bin_sub32=32, bin_warp=32),
     dict(hub_smem_slots=64),                                                  # force the global spill table
-    hub(64),                                                                  # rows > 64 through the hub path
+    hub(64),                                                                  # rows > 64: hub path (cluster DSMEM tables)
     hub(0),                                                                   # every row through the hub path
+    dict(hub(64), hub_cluster=0),                                             # hub path with global tables
+    dict(hub(0), hub_cluster=0, delta_update=1),
     dict(hub(0), force_i128=1),
     dict(hub(64), singleton=0, delta_update=1),
     dict(force_i128=1),

@@ -25,6 +25,8 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="friendster")
 ap.add_argument("--runs", type=int, default=3)
 ap.add_argument("--oracle-iters", type=int, default=2)
+ap.add_argument("--opts", default="{}", help="JSON library options (set_option) for every run")
+ap.add_argument("--verbose-last", action="store_true", help="option verbose=1 on the last timed run")
 args = ap.parse_args()
 out = {"config": args.config}
 t = time.time()
@@ -36,8 +38,12 @@ t = time.time()
 h = gala.Graph.from_graph(g, stream=stream.cuda_stream)
 torch.cuda.synchronize()
 out["create_s"] = round(time.time() - t, 2)
+for k, v in json.loads(args.opts).items():
+    h.set_option(k, v)
 ts = []
 for i in range(args.runs):
+    if args.verbose_last and i == args.runs - 1:
+        h.set_option("verbose", 1)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(stream)
     h.run()
