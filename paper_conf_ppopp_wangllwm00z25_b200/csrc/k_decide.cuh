@@ -617,6 +617,9 @@ __device__ __forceinline__ long long block_next_item(QView queue, long long coun
 #define GALA_BLOCK_MINB 0      // >0: min resident 512-thread blocks per SM of the long-row class (register cap);
                                // 0: no bound (an explicit 1 lets ptxas take 75-100 registers and halves occupancy)
 #endif
+#ifndef GALA_BLOCK_NEXT
+#define GALA_BLOCK_NEXT 1      // the next vertex is fetched while the current one is processed
+#endif
 #ifndef GALA_BLOCK_PIPE
 #define GALA_BLOCK_PIPE 1      // the next round's row entries are loaded while the current round is inserted
 #endif
@@ -661,12 +664,28 @@ __global__ void BLOCK_LB(BT) k_decide_block(QView queue, int bin, DecideArgs a,
     __shared__ int s_batch[FETCH_B], s_nb, s_bi;
     if (threadIdx.x == 0) { s_nb = 0; s_bi = 0; }
     ull* const cursor = CLS == 2 ? &a.ctr->cursor_hi : &a.ctr->cursor[bin];
+    // NEXT: the next item is fetched by thread 0 while the block works on the current one (its
+    // cursor atomic and queue loads are off the per-vertex critical path)
+    // (with its queue record: the block reads the current record from shared memory)
+    __shared__ long long s_next;
+    __shared__ QRec s_q, s_qn;
+    if (GALA_BLOCK_NEXT && threadIdx.x == 0) {
+        s_next = block_next_item<CLS>(queue, count, cursor, split, s_batch, &s_nb, &s_bi);
+        if (s_next < count) s_qn = queue[s_next];
+    }
     for (;;) {
-        if (threadIdx.x == 0) s_item = block_next_item<CLS>(queue, count, cursor, split, s_batch, &s_nb, &s_bi);
+        if (threadIdx.x == 0) {
+            if (GALA_BLOCK_NEXT) { s_item = s_next; s_q = s_qn; }
+            else s_item = block_next_item<CLS>(queue, count, cursor, split, s_batch, &s_nb, &s_bi);
+        }
         __syncthreads();
         long long i = s_item;
         if (i >= count) break;
-        const QRec q = queue[i];
+        const QRec q = GALA_BLOCK_NEXT ? s_q : queue[i];
+        if (GALA_BLOCK_NEXT && threadIdx.x == 0) {
+            s_next = block_next_item<CLS>(queue, count, cursor, split, s_batch, &s_nb, &s_bi);
+            if (s_next < count) s_qn = queue[s_next];
+        }
         const int v = q.v, deg = q.deg, cv = q.cv;
         const int64_t beg = q.beg;
         long long own = 0;   // the own community only feeds d'(v): summed in registers, never inserted
@@ -1373,7 +1392,10 @@ __global__ void __cluster_dims__(CL_CS, 1, 1) __launch_bounds__(CL_BT, 1)
         if (crank == 0 && threadIdx.x == 0) s_item = (long long)atomicAdd(cursor, 1ull);
         cl.sync();   // s_item published; the previous hub's tables are clear everywhere
         const long long i = *item0;
-        if (i >= count) break;
+        if (i >= count) {   // no CTA may exit while another still reads its shared memory (s_item)
+            cl.sync();
+            break;
+        }
         const QRec q = queue[i];
         const int v = q.v, deg = q.deg, cv = q.cv;
         const long long span = deg < a.nlev ? deg : a.nlev;

@@ -372,6 +372,21 @@ def test_torch_allocator_hook():
         gala.set_allocator()
 
 
+def test_cluster_hub_handle_cycles():
+    """Hub rows on the thread-block cluster across repeated create / run / free cycles in graph
+    mode (adopted pools, stale workspace contents): every cycle bit-exact (final labels, N)."""
+    g = gg.make("rmat_small")
+    o = oracle.louvain(g, prune=True)
+    for cyc in range(6):
+        h = gala.Graph.from_graph(g)
+        for k, v in hub(48 + 16 * (cyc % 3)).items():
+            h.set_option(k, v)
+        h.run()
+        assert np.array_equal(h.communities(), o.labels) and h.numerator()[0] == o.N, cyc
+        assert h.k == o.k
+        h.free()
+
+
 def test_block_split_across_handles_graph_mode():
     """A handle with a small block_split (small short-row arena) followed by one with the default
     split, both in graph mode: the second handle's block kernels must get their own dynamic
