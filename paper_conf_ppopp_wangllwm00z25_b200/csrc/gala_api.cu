@@ -31,6 +31,9 @@
 #include "k_dist.cuh"
 #include "fabric.cuh"
 #include "k_nmi.cuh"
+#ifndef GALA_APPLY_AGG
+#define GALA_APPLY_AGG 1   // k_apply: warp-combined Sigma_tot / size atomics (d(v) < 2^32)
+#endif
 
 #define GALA_VERSION "gala-b200 0.1 (sm_100a)"
 
@@ -865,7 +868,8 @@ static void issue_iteration(gala_graph_s* g, Work& wk, const DevCSR& G, typename
     launch_decide<M, UNIT>(g, wk, G, qW, p, tm, maxdeg, idbits, single);
     e = tm.begin();
     k_apply<<<grid_for(n, AP_BT, big), AP_BT, 0, st>>>(wk.ctr, wk.queues, wk.qcap, wk.nextC, wk.C, wk.Sig, wk.size,
-                                                       wk.dp, wk.stamp, wk.cst, wk.carry, wk.mv_v, wk.mv_old, wk.mv_chunk, ps, wk.icap);
+                                                       wk.dp, wk.stamp, wk.cst, wk.carry, wk.mv_v, wk.mv_old, wk.mv_chunk, ps, wk.icap,
+                                                       GALA_APPLY_AGG && g->W < ((int64_t)1 << 32) ? 1 : 0);
     CKL();
     tm.end(KC_APPLY, e);
     e = tm.begin();

@@ -281,8 +281,10 @@ __global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr,
                                                  int32_t* __restrict__ size, int64_t* __restrict__ dp,
                                                  int32_t* __restrict__ stamp, int2* __restrict__ cst,
                                                  const Carry* __restrict__ carry, int32_t* __restrict__ it_v, int32_t* __restrict__ it_old,
-                                                 int32_t* __restrict__ it_chunk, PruneState ps, long long icap) {
+                                                 int32_t* __restrict__ it_chunk, PruneState ps, long long icap,
+                                                 int agg32) {
     __shared__ unsigned s_cnt, s_items, s_hitems;
+    __shared__ unsigned s_scr[AP_BT / 32][32];
     __shared__ ull s_ibase, s_hbase;
     long long cnt[NBINS];
     long long total = 0;
@@ -295,7 +297,8 @@ __global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr,
     for (long long t0 = (long long)blockIdx.x * AP_BT; t0 < total; t0 += (long long)gridDim.x * AP_BT) {
         long long i = t0 + threadIdx.x;
         bool mover = false;
-        int v = 0, oc = 0, deg = 0;
+        int v = 0, oc = 0, deg = 0, mnc = 0;
+        unsigned mdv = 0;
         if (i < total) {
             int b = 0;
             long long r = i;
@@ -318,12 +321,31 @@ __global__ void __launch_bounds__(AP_BT) k_apply(IterCounters* __restrict__ ctr,
                 C[v] = nc;
                 stamp[v] = iter_id;
                 cst[v] = make_int2(nc, iter_id);
-                atomicAdd(reinterpret_cast<ull*>(&Sig[oc]), (ull)(-dv));
-                atomicAdd(reinterpret_cast<ull*>(&Sig[nc]), (ull)dv);
-                atomicSub(&size[oc], 1);
-                atomicAdd(&size[nc], 1);
+                if (!agg32) {
+                    atomicAdd(reinterpret_cast<ull*>(&Sig[oc]), (ull)(-dv));
+                    atomicAdd(reinterpret_cast<ull*>(&Sig[nc]), (ull)dv);
+                    atomicSub(&size[oc], 1);
+                    atomicAdd(&size[nc], 1);
+                }
                 my_deg += (ull)q.deg;
                 if (deg > DCH) dp[v] = 0;   // chunk items add onto it
+                mdv = (unsigned)dv;
+                mnc = nc;
+            }
+        }
+        if (agg32) {   // d(v) < 2^32: the warp's movers into / out of the same community are combined
+                       // (match_any + a shared group sum) into one Sigma_tot and one size atomic
+            const unsigned pn = __match_any_sync(FULLMASK, mover ? mnc : -1 - lane);
+            const unsigned sn = group_sum(pn, mover ? mdv : 0u, s_scr[threadIdx.x >> 5]);
+            if (mover && lane == __ffs(pn) - 1) {
+                atomicAdd(reinterpret_cast<ull*>(&Sig[mnc]), (ull)sn);
+                atomicAdd(&size[mnc], __popc(pn));
+            }
+            const unsigned po = __match_any_sync(FULLMASK, mover ? oc : -1 - lane);
+            const unsigned so = group_sum(po, mover ? mdv : 0u, s_scr[threadIdx.x >> 5]);
+            if (mover && lane == __ffs(po) - 1) {
+                atomicAdd(reinterpret_cast<ull*>(&Sig[oc]), (ull)(-(long long)so));
+                atomicSub(&size[oc], __popc(po));
             }
         }
         // items of this thread: a light mover (row <= DLIGHT) is one item at the FRONT of the

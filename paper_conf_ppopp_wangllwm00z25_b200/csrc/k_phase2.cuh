@@ -374,23 +374,19 @@ struct AggArgs {
     int64_t* snew;             // diagonal weight per community
 };
 
-// bucketed linear probe (4 keys per 16-byte load, empties claimed in slot
-// order; see ht_insert4 in k_decide.cuh); tables are never full (cap >= 2 x
-// distinct keys), mask < 3 falls back to slot-wise probing
+// open-addressing insert / accumulate (slot-wise linear probe; tables are never full: cap >= 2 x
+// distinct keys).  Returns the slot, *fresh when this lane created the key; the caller appends
+// the warp's fresh slots to the distinct list with ONE counter atomic (append_fresh) -- a per-key
+// append serialised the 32 lanes of a chunk on one shared counter whenever most keys were new.
 template <typename VT>
-__device__ __forceinline__ int agg_insert(int key, VT wt, int* keys, VT* vals, unsigned mask, int* list, int* cnt) {
+__device__ __forceinline__ int agg_insert_nl(int key, VT wt, int* keys, VT* vals, unsigned mask, bool* fresh) {
     unsigned h = hash_slot(key, mask);
     for (;;) {
         int k0 = *(volatile int*)&keys[h];
-        if (k0 == key) { atomicAdd(&vals[h], wt); return 0; }
+        if (k0 == key) { atomicAdd(&vals[h], wt); *fresh = false; return (int)h; }
         if (k0 == -1) {
             int old = atomicCAS(&keys[h], -1, key);
-            if (old == -1) {
-                atomicAdd(&vals[h], wt);
-                list[atomicAdd(cnt, 1)] = (int)h;
-                return 1;
-            }
-            if (old == key) { atomicAdd(&vals[h], wt); return 0; }
+            if (old == -1 || old == key) { atomicAdd(&vals[h], wt); *fresh = old == -1; return (int)h; }
         }
         h = (h + 1) & mask;
     }
@@ -448,7 +444,10 @@ __device__ __forceinline__ void agg_segment(const AggArgs& a, long long s0, long
             if (r0 + 32 * t >= s1) break;
             const unsigned peers = __match_any_sync(FULLMASK, kk[t] >= 0 ? kk[t] : -1 - lane);
             const SV sum = UNIT ? (SV)__popc(peers) : group_sum(peers, kk[t] >= 0 ? ww[t] : (SV)0, scratch);
-            if (kk[t] >= 0 && lane == __ffs(peers) - 1) agg_insert<TV>(kk[t], (TV)sum, keys, vals, mask, list, cnt);
+            bool fresh = false;
+            int slot = -1;
+            if (kk[t] >= 0 && lane == __ffs(peers) - 1) slot = agg_insert_nl<TV>(kk[t], (TV)sum, keys, vals, mask, &fresh);
+            append_fresh<int>(fresh, slot, FULLMASK, cnt, list);   // one list-counter atomic per warp
         }
     }
 }
@@ -594,8 +593,8 @@ __global__ void __launch_bounds__(512) k_agg_block_h(AggArgs a, int scap, const 
                 if (r0 + 32 * t >= s1) break;
                 const unsigned peers = __match_any_sync(FULLMASK, kk[t] >= 0 ? kk[t] : -1 - lane);
                 const V sum = UNIT ? (V)__popc(peers) : group_sum(peers, kk[t] >= 0 ? ww[t] : (V)0, s_scr[wib]);
-                bool gfresh = false;
-                unsigned gh = 0;
+                bool gfresh = false, sfresh = false;
+                unsigned gh = 0, sh = 0;
                 if (kk[t] >= 0 && lane == __ffs(peers) - 1) {
                     // H0: window of AGG_HWIN slots
                     unsigned h = hash_slot(kk[t], smask);
@@ -605,7 +604,7 @@ __global__ void __launch_bounds__(512) k_agg_block_h(AggArgs a, int scap, const 
                         if (k0 == kk[t]) { atomicAdd(&vals[h], sum); done = true; }
                         else if (k0 == -1) {
                             const int old = atomicCAS(&keys[h], -1, kk[t]);
-                            if (old == -1) { atomicAdd(&vals[h], sum); list[atomicAdd(&s_cnt, 1)] = (int)h; done = true; }
+                            if (old == -1) { atomicAdd(&vals[h], sum); sfresh = true; sh = h; done = true; }
                             else if (old == kk[t]) { atomicAdd(&vals[h], sum); done = true; }
                         }
                     }
@@ -622,6 +621,7 @@ __global__ void __launch_bounds__(512) k_agg_block_h(AggArgs a, int scap, const 
                         }
                     }
                 }
+                append_fresh<int>(sfresh, (int)sh, FULLMASK, &s_cnt, list);   // one counter atomic per warp
                 const unsigned fm = __ballot_sync(FULLMASK, gfresh);
                 if (fm) {
                     const int lead = __ffs(fm) - 1;

@@ -9,11 +9,14 @@ set -x
 TAG=$1; shift
 mkdir -p gpurun_out /tmp/ncu
 make -s >/dev/null
-ncu --metrics gpu__time_duration.sum --clock-control none --profile-from-start off --csv \
-    --log-file gpurun_out/${TAG}_launches_lfr1m.csv python tools/profile_run.py --config lfr1m > /dev/null 2>&1
+for LC in lfr1m orkut; do
+  ncu --metrics gpu__time_duration.sum --clock-control none --profile-from-start off --csv \
+      --log-file gpurun_out/${TAG}_launches_$LC.csv python tools/profile_run.py --config $LC > /dev/null 2>&1
+  python tools/launches.py gpurun_out/${TAG}_launches_$LC.csv 40 > gpurun_out/${TAG}_launches_$LC.txt
+done
 declare -A RX=( [prune_bin]='k_prune_bin' [decide_single]='k_decide_single' [decide_small]='k_decide_small'
   [decide_warp]='k_decide_warp<[^,]*32, [^,]*128' [decide_warp512]='k_decide_warp<[^,]*32, [^,]*512' [decide_block]='k_decide_block'
-  [decide_hub]='k_hub_' [apply]='k_apply' [dp_update]='k_dp_|k_sm_flags' [reduce]='k_reduce'
+  [decide_hub]='k_hub_|k_decide_cluster' [apply]='k_apply' [dp_update]='k_dp_|k_sm_flags' [reduce]='k_reduce'
   [phase2]='k_agg_|k_gather_flat|k_compact' )
 for spec in "$@"; do
   C=${spec%%:*}; CL=${spec#*:}

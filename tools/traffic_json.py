@@ -22,6 +22,7 @@ CLASSES = [
     ("decide_warp512", r"^k_decide_warp<32, 512", True),
     ("decide_block", r"^k_decide_block", True),
     ("decide_hub", r"^k_hub_prep[(<]", True),
+    ("decide_hub", r"^k_decide_cluster", True),             # hubs on a thread-block cluster
     ("decide_hub", r"^k_hub_(agg|prep2|eval|final|single)", False),
     ("apply", r"^k_apply", True),
     ("dp_update", r"^k_dp_delta", True),
