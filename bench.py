@@ -385,7 +385,7 @@ def main():
     rp = torch.from_numpy(g.row_ptr).pin_memory()
     col = torch.from_numpy(g.col).pin_memory()
     lab_host = torch.empty(g.n, dtype=torch.int32).pin_memory()
-    e2e_ms, e2e_edges, iters_total = [], 0, 0
+    e2e_ms, e2e_edges, iters_total, e2e_parts = [], 0, 0, []
     import ctypes
     L = gala.lib()
     for i in range(args.warmup + args.steps):
@@ -393,11 +393,14 @@ def main():
             flush.add_(1)
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ec, er = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
         hh = ctypes.c_void_p()
         gala._check(L.gala_graph_from_csr(g.n, rp.data_ptr(), col.data_ptr(), None, dev, stream.cuda_stream,
                                           ctypes.byref(hh)))
+        ec.record(stream)
         gala._check(L.gala_run(hh, 1.0, 1e-6, 0))
+        er.record(stream)
         k = ctypes.c_int64()
         gala._check(L.gala_get_communities(hh, lab_host.data_ptr(), g.n, ctypes.byref(k)))
         e1.record(stream)
@@ -407,6 +410,7 @@ def main():
         gh.free()
         if i >= args.warmup:
             e2e_ms.append(e0.elapsed_time(e1))
+            e2e_parts.append((e0.elapsed_time(ec), ec.elapsed_time(er), er.elapsed_time(e1)))
             e2e_edges += level0_edges_ms(st)[0]
             iters_total = sum(lv["iters"] for lv in st["levels"])
     e2e_value = e2e_edges / (sum(e2e_ms) / 1e3) / 1e9
@@ -476,11 +480,48 @@ def main():
         "oracle_1thread": o1,
         "oracle_parity": parity,
         "e2e": {"value": e2e_value, "unit": "GTEPS", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-                "louvain_seconds": sum(e2e_ms) / 1e3 / len(e2e_ms)},
+                "louvain_seconds": sum(e2e_ms) / 1e3 / len(e2e_ms), "step_ms": [round(x, 3) for x in e2e_ms],
+                "median_create_run_labels_ms": [round(statistics.median(p[j] for p in e2e_parts), 3) for j in range(3)]},
         "gpu_launches": launches,
         "clocks": clk.summary(),
     }
     print(json.dumps(line), flush=True)
+
+
+def shared_graph(config: str, rank: int, world: int):
+    """The workload graph on every rank of an N-process run, generated ONCE: rank 0 builds it and
+    writes its arrays to a scratch directory, the other ranks map them read-only after a barrier
+    (8 ranks generating the full Friendster shape side by side would need 8 x 30 GB of host
+    memory and 8x the generator time).  Returns (CSR, cleanup) -- call cleanup() once every rank
+    has copied its rows."""
+    import shutil
+    import tempfile
+    import torch.distributed as dist
+    import graphgen as gg
+    base = os.environ.get("GALA_SHARED_GRAPH_DIR", tempfile.gettempdir())
+    tag = [f"gala_graph_{config}_{os.getpid()}_{int(time.time() * 1e3)}" if rank == 0 else None]
+    dist.broadcast_object_list(tag, src=0)
+    d = os.path.join(base, tag[0])
+    if rank == 0:
+        g = gg.make(config)
+        os.makedirs(d, exist_ok=True)
+        np.save(os.path.join(d, "row_ptr.npy"), g.row_ptr)
+        np.save(os.path.join(d, "col.npy"), np.asarray(g.col))
+        if g.w is not None:
+            np.save(os.path.join(d, "w.npy"), g.w)
+        if g.truth is not None:
+            np.save(os.path.join(d, "truth.npy"), g.truth)
+    dist.barrier()
+    if rank != 0:
+        ld = lambda f: np.load(os.path.join(d, f), mmap_mode="r") if os.path.exists(os.path.join(d, f)) else None
+        rp = ld("row_ptr.npy")
+        g = gg.CSR(n=len(rp) - 1, row_ptr=rp, col=ld("col.npy"), w=ld("w.npy"), name=config, truth=ld("truth.npy"))
+
+    def cleanup():
+        dist.barrier()
+        if rank == 0:
+            shutil.rmtree(d, ignore_errors=True)
+    return g, cleanup
 
 
 def run_dist(args, rank, world, local_rank):
@@ -493,10 +534,11 @@ def run_dist(args, rank, world, local_rank):
     import paper_conf_ppopp_wangllwm00z25_b200 as gala
 
     dev = local_rank
-    g = gg.make(args.config)                      # identical on every rank (seeded)
+    g, cleanup = shared_graph(args.config, rank, world)   # generated once (rank 0), mapped by the others
     bounds = gala.partition_ranges(g.row_ptr, world)
     v0, v1 = int(bounds[rank]), int(bounds[rank + 1])
     lrp, lcol, lw = gala.local_rows(g.row_ptr, g.col, g.w, v0, v1)
+    cleanup()
     uid = [gala.nccl_unique_id() if rank == 0 else None]
     dist.broadcast_object_list(uid, src=0)
     stream = torch.cuda.Stream(device=dev)

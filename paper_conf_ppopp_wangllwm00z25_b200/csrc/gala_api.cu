@@ -1272,17 +1272,30 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
         CK(cudaMemcpyAsync(&gtot, goff + nbig, sizeof(long long), cudaMemcpyDeviceToHost, st));
         CK(cudaStreamSynchronize(st));
         int* gkeys = dalloc<int>(gtot, st);
-        ull* gvals = dalloc<ull>(gtot, st);
+        // table values 32-bit whenever W < 2^32 (every aggregated weight is <= W)
+        const size_t gvb = v32 ? sizeof(unsigned) : sizeof(ull);
+        char* gvals = dalloc<char>((size_t)gtot * gvb, st);
         int* glist = dalloc<int>(gtot / 2 + 1, st);
         int* gcnt = dalloc<int>(nbig, st);
         CK(cudaMemsetAsync(gkeys, 0xff, sizeof(int) * gtot, st));
-        CK(cudaMemsetAsync(gvals, 0, sizeof(ull) * gtot, st));
+        CK(cudaMemsetAsync(gvals, 0, gvb * gtot, st));
         CK(cudaMemsetAsync(gcnt, 0, sizeof(int) * nbig, st));
         vt.lap("agg: big alloc+clear");
-        k_agg_big_insert2<<<big, 256, 0, st>>>(a, bigc, nbig, choff, ndc, ch, goff, gkeys, gvals, glist, gcnt);
-        CKL();
-        vt.lap("agg: big insert");
-        k_agg_big_emit2<<<big, 256, 0, st>>>(a, bigc, nbig, choff, goff, gkeys, gvals, glist, gcnt, ch);
+        if (v32) {
+            k_agg_big_insert2<unsigned><<<big, 256, 0, st>>>(a, bigc, nbig, choff, ndc, ch, goff, gkeys,
+                                                             reinterpret_cast<unsigned*>(gvals), glist, gcnt);
+            CKL();
+            vt.lap("agg: big insert");
+            k_agg_big_emit2<unsigned><<<big, 256, 0, st>>>(a, bigc, nbig, choff, goff, gkeys,
+                                                           reinterpret_cast<unsigned*>(gvals), glist, gcnt, ch);
+        } else {
+            k_agg_big_insert2<ull><<<big, 256, 0, st>>>(a, bigc, nbig, choff, ndc, ch, goff, gkeys,
+                                                        reinterpret_cast<ull*>(gvals), glist, gcnt);
+            CKL();
+            vt.lap("agg: big insert");
+            k_agg_big_emit2<ull><<<big, 256, 0, st>>>(a, bigc, nbig, choff, goff, gkeys, reinterpret_cast<ull*>(gvals),
+                                                      glist, gcnt, ch);
+        }
         CKL();
         dfree(nch, st); dfree(choff, st); dfree(ndc, st);
         dfree(goff, st); dfree(gkeys, st); dfree(gvals, st); dfree(glist, st); dfree(gcnt, st);
@@ -1321,7 +1334,7 @@ static void aggregate_rows(gala_graph_s* g, const DevCSR& cur, int64_t nrows, lo
             }
             CKL();
             vt.lap("agg: big insert");
-            k_agg_big_emit2<<<big, 256, 0, st>>>(a, bigc, nbig, choff, goff, gkeys, gvals, glist, gcnt, g->opt_agg_chunk);
+            k_agg_big_emit2<ull><<<big, 256, 0, st>>>(a, bigc, nbig, choff, goff, gkeys, gvals, glist, gcnt, g->opt_agg_chunk);
             CKL();
         } else {
             const int bpc = 32;
@@ -2594,7 +2607,7 @@ static void finish_graph(gala_graph_s* g) {
     CKL();
     k_max_i64<<<grid_for(n, 256, big), 256, 0, st>>>(n, g->d0, mx + 1);
     CKL();
-    k_rows_not_increasing<<<grid_for(n, 256, big), 256, 0, st>>>((int)n, g->g0.rp, g->g0.col, mx + 2);
+    k_rows_not_increasing<<<grid_for(g->g0.nnz, 256, big), 256, 0, st>>>(g->g0.nnz, g->g0.row, g->g0.col, mx + 2);
     CKL();
     i128* part = dalloc<i128>(big, st);
     ull* ticket = dalloc<ull>(1, st);

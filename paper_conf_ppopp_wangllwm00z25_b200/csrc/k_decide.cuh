@@ -1376,7 +1376,6 @@ __global__ void __cluster_dims__(CL_CS, 1, 1) __launch_bounds__(CL_BT, 1)
     __shared__ long long s_own;
     __shared__ A s_part[CL_CS];
     __shared__ A r_a[CL_BT / 32];
-    __shared__ long long r_own[CL_BT / 32];
     __shared__ unsigned s_scr[CL_BT / 32][32];
     if (a.ckey && !*a.ckey_valid) a.ckey = nullptr;
     const int lane = lane_id(), wib = threadIdx.x >> 5;
@@ -1474,7 +1473,6 @@ __global__ void __cluster_dims__(CL_CS, 1, 1) __launch_bounds__(CL_BT, 1)
             s_own = 0;
         }
     }
-    (void)r_own;
     ull k = block_sum_ull<CL_BT>((ull)my_k);
     if (threadIdx.x == 0 && k) atomicAdd(&a.ctr->bin_k[BIN_HUB], k);
 }

@@ -396,7 +396,8 @@ __device__ __forceinline__ int agg_insert_nl(int key, VT wt, int* keys, VT* vals
 // insert / accumulate without touching the list, then append the warp's fresh slots with ONE
 // returning atomic on the community's list counter (every block working on a community hits that
 // counter; one atomic per fresh key serialised them -- the friendster_q level-0 coarsening).
-__device__ __forceinline__ void agg_insert_warp(bool on, int key, ull wt, int* keys, ull* vals, unsigned mask,
+template <typename GV>
+__device__ __forceinline__ void agg_insert_warp(bool on, int key, GV wt, int* keys, GV* vals, unsigned mask,
                                                 int* list, int* cnt) {
     bool fresh = false;
     unsigned h = 0;
@@ -825,7 +826,7 @@ __global__ void __launch_bounds__(256) k_agg_big_chunk(AggArgs a, const int32_t*
                 keys[slot] = -1;
                 vals[slot] = 0;
             }
-            agg_insert_warp(on, key, (ull)val, gkeys + off, gvals + off, mask, glist + off / 2, &gcnt[bi]);
+            agg_insert_warp<ull>(on, key, (ull)val, gkeys + off, gvals + off, mask, glist + off / 2, &gcnt[bi]);
         }
         __syncthreads();
         if (threadIdx.x == 0) s_cnt = 0;
@@ -892,11 +893,13 @@ __global__ void k_agg_big_bound(int nbig, long long k, const long long* __restri
     }
 }
 
+// GV: global table value type, 32-bit whenever W < 2^32 (halves the tables' value bytes)
+template <typename GV>
 __global__ void __launch_bounds__(256) k_agg_big_insert2(AggArgs a, const int32_t* __restrict__ bigc, int nbig,
                                                          const long long* __restrict__ choff,
                                                          const int* __restrict__ ndc, int ch,
                                                          const long long* __restrict__ goff, int* __restrict__ gkeys,
-                                                         ull* __restrict__ gvals, int* __restrict__ glist,
+                                                         GV* __restrict__ gvals, int* __restrict__ glist,
                                                          int* __restrict__ gcnt) {
     const long long total = choff[nbig];
     for (long long t = blockIdx.x; t < total; t += gridDim.x) {
@@ -909,7 +912,7 @@ __global__ void __launch_bounds__(256) k_agg_big_insert2(AggArgs a, const int32_
         for (int i0 = threadIdx.x & ~31; i0 < m; i0 += 256) {   // warp-uniform trips
             const int i = i0 + (threadIdx.x & 31);
             const bool on = i < m;
-            agg_insert_warp(on, on ? a.tkey[lo + i] : 0, on ? (ull)a.tval.get(lo + i) : 0, gkeys + off, gvals + off, mask,
+            agg_insert_warp<GV>(on, on ? a.tkey[lo + i] : 0, on ? (GV)a.tval.get(lo + i) : (GV)0, gkeys + off, gvals + off, mask,
                             glist + off / 2, &gcnt[bi]);
         }
     }
@@ -917,10 +920,11 @@ __global__ void __launch_bounds__(256) k_agg_big_insert2(AggArgs a, const int32_
 
 // distinct entries of the big communities to the start of their segments; list
 // index range of chunk t = [j*AGG_CH, (j+1)*AGG_CH) of its community (m <= entries)
+template <typename GV>
 __global__ void __launch_bounds__(256) k_agg_big_emit2(AggArgs a, const int32_t* __restrict__ bigc, int nbig,
                                                        const long long* __restrict__ choff,
                                                        const long long* __restrict__ goff,
-                                                       const int* __restrict__ gkeys, const ull* __restrict__ gvals,
+                                                       const int* __restrict__ gkeys, const GV* __restrict__ gvals,
                                                        const int* __restrict__ glist, const int* __restrict__ gcnt,
                                                        int ch) {
     const long long total = choff[nbig];
@@ -1037,13 +1041,16 @@ __global__ void __launch_bounds__(256) k_sum_i128(long long n, const int64_t* __
 }
 
 // *bad != 0 iff some row is not strictly increasing (so may hold duplicate columns)
-__global__ void k_rows_not_increasing(int n, const int64_t* __restrict__ rp, const int32_t* __restrict__ col,
+// entries that do not strictly increase within their row (duplicates / unsorted rows), edge-parallel
+// over the row-id array (a thread per row walked the longest rows -- 33k entries -- serially)
+__global__ void k_rows_not_increasing(long long nnz, const int32_t* __restrict__ row, const int32_t* __restrict__ col,
                                       ull* __restrict__ bad) {
     const long long stride = (long long)gridDim.x * blockDim.x;
-    for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) {
-        for (int64_t j = rp[v] + 1; j < rp[v + 1]; ++j)
-            if (col[j] <= col[j - 1]) { atomicAdd(bad, 1ull); break; }
-    }
+    unsigned f = 0;
+    for (long long e = (long long)blockIdx.x * blockDim.x + threadIdx.x + 1; e < nnz; e += stride)
+        if (row[e] == row[e - 1] && col[e] <= col[e - 1]) f = 1;
+    f = __reduce_or_sync(FULLMASK, f);
+    if (lane_id() == 0 && f) atomicAdd(bad, 1ull);
 }
 
 // max of a non-negative int64 array

@@ -65,3 +65,37 @@ def test_gloo_world2_partition_uid_and_timing():
         assert ulen == 128 and head == b"GALALOOP"
         assert t == 11.0                       # max over ranks
         assert max(loads) - min(loads) <= 2 * 200 + 1   # edge-balanced within one max row
+
+
+def _worker_shared(rank, world, port, q, tmp):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), GALA_SHARED_GRAPH_DIR=tmp)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from bench import shared_graph
+    g, cleanup = shared_graph("lfr_small", rank, world)
+    ref = gg.make("lfr_small")
+    same = (np.array_equal(np.asarray(g.row_ptr), ref.row_ptr) and np.array_equal(np.asarray(g.col), ref.col)
+            and np.array_equal(np.asarray(g.truth), ref.truth) and g.n == ref.n and g.nnz == ref.nnz)
+    bounds = gala.partition_ranges(g.row_ptr, world)
+    lrp, lcol, _ = gala.local_rows(g.row_ptr, g.col, g.w, int(bounds[rank]), int(bounds[rank + 1]))
+    cleanup()
+    left = os.listdir(tmp)
+    q.put((rank, same, int(lrp[-1]) == len(lcol), left))
+    dist.destroy_process_group()
+
+
+def test_gloo_world2_shared_graph(tmp_path):
+    """bench.py's N-rank graph loading: rank 0 generates, the other ranks map its arrays; every
+    rank sees the generator's graph exactly and the scratch directory is gone afterwards."""
+    world, port = 2, _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_worker_shared, args=(r, world, port, q, str(tmp_path))) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = sorted(q.get(timeout=300) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for rank, same, rows_ok, left in res:
+        assert same and rows_ok
+    assert os.listdir(str(tmp_path)) == []

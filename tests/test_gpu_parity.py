@@ -91,6 +91,12 @@ def test_synthetic_parity(name, prune):
     assert_parity(gg.make(name), prune=prune)
 
 
+def test_lean_generator_graph_parity():
+    """The Friendster recipe's graph type (gg_lfr_csr: Feistel-paired external stubs, exact-mean
+    degree law) at 200k vertices: every iteration and level bit-exact against the oracle."""
+    assert_parity(gg.lfr_csr(200_000, 63.85, 5_214, 0.37, seed=4, fit_frac=True, name="fr_small"))
+
+
 @pytest.mark.parametrize("name", ["karate", "lfr_small", "rmat_small"])
 @pytest.mark.parametrize("strategy", [0, 1, 2, 3, 4])
 @pytest.mark.parametrize("check", [0, 1])
