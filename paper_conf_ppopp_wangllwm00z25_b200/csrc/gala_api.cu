@@ -265,12 +265,27 @@ struct DevCache {
             p = user_alloc(ua, r, st);
         } else {
             cudaError_t e = cudaMallocFromPoolAsync(&p, r, pool, st);
-            if (e == cudaErrorMemoryAllocation) {   // give cached blocks back and retry once
+            if (e == cudaErrorMemoryAllocation) {
+                // first the largest cached blocks back to the pool (stream-ordered: the pool reuses
+                // their physical pages for this request, nothing is unmapped), then -- only if that
+                // is not enough -- every cached block and the pool's unused reserve
                 cudaGetLastError();
-                trim(st);
-                cudaStreamSynchronize(st);
-                cudaMemPoolTrimTo(pool, 0);
+                size_t freed = 0;
+                while (!freeb.empty() && freed < 2 * r) {
+                    auto last = std::prev(freeb.end());
+                    release(last->second, sz[last->second], st);
+                    freed += last->first;
+                    sz.erase(last->second);
+                    freeb.erase(last);
+                }
                 e = cudaMallocFromPoolAsync(&p, r, pool, st);
+                if (e == cudaErrorMemoryAllocation) {
+                    cudaGetLastError();
+                    trim(st);
+                    cudaStreamSynchronize(st);
+                    cudaMemPoolTrimTo(pool, 0);
+                    e = cudaMallocFromPoolAsync(&p, r, pool, st);
+                }
             }
             CK(e);
         }
@@ -689,7 +704,7 @@ static void block_setup(gala_graph_s* g) {
 // the sub-warp and warp bins (rows <= bins[BIN_WARP2]); MS: mode of the sub-warp kernel (packed keys
 // pay there: A/B on orkut decide_small 2.37 -> 2.16 ms), M: the warp kernels' (the packed variant of
 // the 128-row warp kernel spills; measured 4.98 -> 5.34 ms)
-template <int M, bool UNIT, int MS = M>
+template <int M, bool UNIT, int MS = M, int MW = M>
 static void launch_short_bins(gala_graph_s* g, Work& wk, const DecideArgs& a, typename ModeT<M>::ST qW,
                               typename ModeT<M>::ST p, Timer& tm, int64_t maxdeg, Fork& fk) {
     const long long qs = wk.qcap;
@@ -700,14 +715,14 @@ static void launch_short_bins(gala_graph_s* g, Work& wk, const DecideArgs& a, ty
     CKL();
     tm.end(KC_DEC_SMALL, e);
     e = tm.begin();
-    k_decide_warp<32, 128, M, UNIT><<<grid, 32 * WarpSmem<32, 128, M>::WPB, WarpSmem<32, 128, M>::bytes, fk.branch(2)>>>(
+    k_decide_warp<32, 128, MW, UNIT><<<grid, 32 * WarpSmem<32, 128, MW>::WPB, WarpSmem<32, 128, MW>::bytes, fk.branch(2)>>>(
         qview(wk.queues, qs, BIN_WARP), BIN_WARP, a, qW, p);
     CKL();
     tm.end(KC_DEC_WARP, e);
     if (maxdeg > g->bins[BIN_WARP]) {
         e = tm.begin();
-        k_decide_warp<32, 512, M, UNIT><<<grid, 32 * WarpSmem<32, 512, M>::WPB, WarpSmem<32, 512, M>::bytes,
-                                          fk.branch(3)>>>(qview(wk.queues, qs, BIN_WARP2), BIN_WARP2, a, qW, p);
+        k_decide_warp<32, 512, MW, UNIT><<<grid, 32 * WarpSmem<32, 512, MW>::WPB, WarpSmem<32, 512, MW>::bytes,
+                                           fk.branch(3)>>>(qview(wk.queues, qs, BIN_WARP2), BIN_WARP2, a, qW, p);
         CKL();
         tm.end(KC_DEC_WARP2, e);
     }
@@ -767,7 +782,9 @@ static void launch_decide(gala_graph_s* g, Work& wk, const DevCSR& G, typename M
         }
     }
     launch_hub<M, UNIT>(g, wk, a, qW, p, tm, wk.hub_on ? fk.branch(1) : st);
-    if constexpr (M == DM_W64 && UNIT) {   // short rows may use packed argmax keys (packed_ok)
+    if constexpr (M == DM_W64 && UNIT) {   // short / mid rows may use packed argmax keys (packed_ok)
+        if (g->opt_bin_packed && g->opt_force_wide != 1 && packed_ok(g, idbits, std::min<int64_t>(maxdeg, g->bins[BIN_WARP2])))
+            return launch_short_bins<M, UNIT, DM_FAST, DM_FAST>(g, wk, a, qW, p, tm, maxdeg, fk);
         if (g->opt_bin_packed && g->opt_force_wide != 1 && packed_ok(g, idbits, std::min<int64_t>(maxdeg, g->bins[BIN_S32])))
             return launch_short_bins<M, UNIT, DM_FAST>(g, wk, a, qW, p, tm, maxdeg, fk);
     }
