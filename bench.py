@@ -611,6 +611,8 @@ def run_dist(args, rank, world, local_rank):
         "iterations": sum(lv["iters"] for lv in st["levels"]),
         "sync": {"dense_iters": d.get("dense_iters"), "sparse_iters": d.get("sparse_iters"),
                  "bytes_exchanged_per_run": d.get("bytes_exchanged")},
+        "per_level": [{"n": lv["n"], "nnz": lv["nnz"], "iters": lv["iters"], "ms_phase1": round(lv["ms_phase1"], 4),
+                       "ms_phase2": round(lv["ms_phase2"], 4)} for lv in st["levels"]],
         "roofline": None, "cpu_baseline": None,
         "e2e": {"value": e2e_value, "unit": "GTEPS", "h2d_bytes_per_step": int(lrp.nbytes + lcol.nbytes),
                 "d2h_bytes_per_step": int(g.n * 4)},

@@ -1802,6 +1802,10 @@ struct DistInfo {
     FabDev fab = {};
     bool failed = false;   // a run ended in an error: peers may still touch the region
     bool host_bar = false; // fabric barriers on the host (ranks sharing one device: loopback world > 1)
+    // mirror block of the level-0 owned rows: depends only on the graph, built by the first run
+    int64_t* m0rp = nullptr;
+    int32_t* m0col = nullptr;
+    int64_t* m0w = nullptr;
 };
 
 // Symmetric region of a rank (cudaMalloc: CUDA IPC needs it), byte offsets:
@@ -2167,8 +2171,10 @@ struct DistLevel {
     int64_t* mw = nullptr;
     int32_t *it_v = nullptr, *it_old = nullptr, *it_chunk = nullptr;
     FabDev f = {};
+    bool mirror_cached = false;   // level 0: the mirror belongs to DistInfo (kept across runs)
     void release(cudaStream_t st) {
-        dfree(lmoves, st); dfree(lcount, st); dfree(mrp, st); dfree(mcol, st); dfree(mw, st);
+        dfree(lmoves, st); dfree(lcount, st);
+        if (!mirror_cached) { dfree(mrp, st); dfree(mcol, st); dfree(mw, st); }
         dfree(it_v, st); dfree(it_old, st); dfree(it_chunk, st);
     }
 };
@@ -2188,7 +2194,12 @@ static void dist_level_setup(gala_graph_s* g, const DevCSR& G, const std::vector
     L.lmoves = dalloc<int2>(std::max<long long>(L.lv1 - L.lv0, 1), st);
     L.lcount = dalloc<ull>(1, st);
     CK(cudaMemsetAsync(L.lcount, 0, sizeof(ull), st));
-    // mirror block: owned entries (v, u, w) counting-sorted by u
+    // mirror block: owned entries (v, u, w) counting-sorted by u (level 0: built once per handle)
+    const bool lvl0 = G.col == g->g0.col;
+    if (lvl0 && di.m0rp) {
+        L.mrp = di.m0rp; L.mcol = di.m0col; L.mw = di.m0w;
+        L.mirror_cached = true;
+    } else {
     long long* cnt = dalloc<long long>(n + 1, st);
     CK(cudaMemsetAsync(cnt, 0, sizeof(long long) * (n + 1), st));
     k_mirror_count<<<grid_for(G.nnz, 256, big), 256, 0, st>>>(G.nnz, G.col, cnt);
@@ -2202,6 +2213,8 @@ static void dist_level_setup(gala_graph_s* g, const DevCSR& G, const std::vector
                                                                  reinterpret_cast<long long*>(L.mrp), cnt, L.mcol, L.mw);
     CKL();
     dfree(cnt, st);
+    if (lvl0) { di.m0rp = L.mrp; di.m0col = L.mcol; di.m0w = L.mw; L.mirror_cached = true; }
+    }
     // d' items: one per global mover with a row here + one per DCH-entry chunk of own / mirror rows
     const size_t icap = (size_t)n + (size_t)(2 * G.nnz / DCH) + (size_t)P + 1;
     L.it_v = dalloc<int32_t>(icap, st);
@@ -2870,6 +2883,7 @@ void gala_graph_free(gala_graph g) {
     if (g->di) {   // communicators are cached (comm_for); the fabric region is this handle's
         if (g->stream) cudaStreamSynchronize(g->stream);
         fabric_release(*g->di);
+        if (g->stream) { dfree(g->di->m0rp, g->stream); dfree(g->di->m0col, g->stream); dfree(g->di->m0w, g->stream); }
         delete g->di;
         g->di = nullptr;
     }
