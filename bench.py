@@ -481,7 +481,8 @@ def main():
         "oracle_parity": parity,
         "e2e": {"value": e2e_value, "unit": "GTEPS", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                 "louvain_seconds": sum(e2e_ms) / 1e3 / len(e2e_ms), "step_ms": [round(x, 3) for x in e2e_ms],
-                "median_create_run_labels_ms": [round(statistics.median(p[j] for p in e2e_parts), 3) for j in range(3)]},
+                "median_create_run_labels_ms": [round(statistics.median(p[j] for p in e2e_parts), 3) for j in range(3)],
+                "create_run_labels_ms_per_step": [[round(x, 2) for x in p] for p in e2e_parts]},
         "gpu_launches": launches,
         "clocks": clk.summary(),
     }
