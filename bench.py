@@ -382,6 +382,9 @@ def main():
     p1_achieved = l0_bytes / (l0_ms / 1e3) / 1e9 if l0_ms else None
 
     # ------------------------------------------------------------ e2e through the C ABI with host buffers
+    # (the resident handle of the device-timed leg is released first: one graph on the device at a
+    # time, as a user of the C ABI runs it; its parked pool serves the e2e handles)
+    h.free()
     rp = torch.from_numpy(g.row_ptr).pin_memory()
     col = torch.from_numpy(g.col).pin_memory()
     lab_host = torch.empty(g.n, dtype=torch.int32).pin_memory()

@@ -8,12 +8,16 @@ rp = torch.from_numpy(g.row_ptr).pin_memory()
 col = torch.from_numpy(g.col).pin_memory()
 lab = torch.empty(g.n, dtype=torch.int32).pin_memory()
 L = gala.lib()
-for i in range(6):
+NC = int(sys.argv[2]) if len(sys.argv) > 2 else 6
+VERB = len(sys.argv) > 3
+for i in range(NC):
     torch.cuda.synchronize()
     t0 = time.perf_counter()
     hh = ctypes.c_void_p()
     gala._check(L.gala_graph_from_csr(g.n, rp.data_ptr(), col.data_ptr(), None, 0, stream.cuda_stream, ctypes.byref(hh)))
     torch.cuda.synchronize(); t1 = time.perf_counter()
+    if VERB:
+        gala._check(L.gala_set_option(hh, b"verbose", 1))
     gala._check(L.gala_run(hh, 1.0, 1e-6, 0))
     torch.cuda.synchronize(); t2 = time.perf_counter()
     k = ctypes.c_int64()
