@@ -1372,25 +1372,27 @@ __global__ void __cluster_dims__(CL_CS, 1, 1) __launch_bounds__(CL_BT, 1)
     cg::cluster_group cl = cg::this_cluster();
     const unsigned crank = cl.block_rank();
     extern __shared__ __align__(16) ull ctbl[];
-    __shared__ long long s_item;
-    __shared__ long long s_own;
+    // hub index and own-community sum double-buffered by hub parity: two cluster barriers per hub
+    // (the next hub's index is fetched before the barrier that publishes the partials)
+    __shared__ long long s_item[2];
+    __shared__ long long s_own[2];
     __shared__ A s_part[CL_CS];
     __shared__ A r_a[CL_BT / 32];
     __shared__ unsigned s_scr[CL_BT / 32][32];
     if (a.ckey && !*a.ckey_valid) a.ckey = nullptr;
     const int lane = lane_id(), wib = threadIdx.x >> 5;
     for (int j = threadIdx.x; j < CL_SLOTS; j += CL_BT) ctbl[j] = KV_EMPTY;
-    if (threadIdx.x == 0) s_own = 0;
+    if (threadIdx.x == 0) { s_own[0] = 0; s_own[1] = 0; }
     const long long count = (long long)a.ctr->bin_count[BIN_HUB];
     ull* const cursor = &a.ctr->cursor[BIN_HUB];
-    long long* const own0 = cl.map_shared_rank(&s_own, 0);
+    long long* const own0 = cl.map_shared_rank(s_own, 0);
     A* const part0 = cl.map_shared_rank(s_part, 0);
-    const long long* const item0 = cl.map_shared_rank(&s_item, 0);
+    const long long* const item0 = cl.map_shared_rank(s_item, 0);
     unsigned my_k = 0;
-    for (;;) {
-        if (crank == 0 && threadIdx.x == 0) s_item = (long long)atomicAdd(cursor, 1ull);
-        cl.sync();   // s_item published; the previous hub's tables are clear everywhere
-        const long long i = *item0;
+    if (crank == 0 && threadIdx.x == 0) s_item[0] = (long long)atomicAdd(cursor, 1ull);
+    cl.sync();   // tables initialised everywhere, the first hub index published
+    for (int par = 0;; par ^= 1) {
+        const long long i = item0[par];
         if (i >= count) {   // no CTA may exit while another still reads its shared memory (s_item)
             cl.sync();
             break;
@@ -1430,7 +1432,7 @@ __global__ void __cluster_dims__(CL_CS, 1, 1) __launch_bounds__(CL_BT, 1)
             }
         }
         own = warp_sum_ll(own);
-        if (lane == 0 && own) atomicAdd(reinterpret_cast<ull*>(own0), (ull)own);
+        if (lane == 0 && own) atomicAdd(reinterpret_cast<ull*>(own0 + par), (ull)own);
         cl.sync();   // every insert (and every own contribution) has landed
         const long long dv = q.dv;
         A best;
@@ -1461,16 +1463,17 @@ __global__ void __cluster_dims__(CL_CS, 1, 1) __launch_bounds__(CL_BT, 1)
             for (int off = 16; off > 0; off >>= 1) best.xor_merge(off);
             if (lane == 0) part0[crank] = best;
         }
-        cl.sync();   // every CTA's partial is in CTA 0
+        if (crank == 0 && threadIdx.x == 0) s_item[par ^ 1] = (long long)atomicAdd(cursor, 1ull);   // next hub
+        cl.sync();   // every CTA's partial is in CTA 0, the next hub index is published, tables clear
         if (crank == 0 && threadIdx.x == 0) {
             A b = s_part[0];
             for (int r = 1; r < CL_CS; ++r)
                 if (s_part[r].valid()) b.offer(s_part[r].score(), s_part[r].comm());
-            const long long ownv = s_own;
+            const long long ownv = s_own[par];
             if (a.check && ownv != a.dp[v]) atomicAdd(&a.ctr->dp_mismatch, 1ull);
             a.nextC[v] = decide_final<ST>(cv, q.szv, dv, ownv, q.sigv, b, a.size, qW, p);
             my_k += ownv ? 1u : 0u;
-            s_own = 0;
+            s_own[par] = 0;   // reused two hubs later, after two more barriers
         }
     }
     ull k = block_sum_ull<CL_BT>((ull)my_k);
